@@ -1,0 +1,158 @@
+"""CPU oracle for the FluidFaaS pipeline-construction search -- TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  The product path
+(``paper_conf_hpdc_hui0s25_b200``) never imports it and shares no code with it.
+
+``ffs_oracle.c`` holds the definitions (plan, bind, eviction score, victim), each
+citing the paper passage it follows; this module only marshals numpy arrays to it.
+The problem object is duck-typed (any object with the attributes of
+``workload.Problem``), so this package imports nothing from the product tree.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "ffs_oracle.c")
+_LIB = os.path.join(_HERE, "libffs_oracle.so")
+_lock = threading.Lock()
+_lib = None
+
+KEY_NONE = np.iinfo(np.int64).max
+PLAN_OK, PLAN_INFEASIBLE, PLAN_BAD_REQ = 0, 1, 2
+ST_EXCL_HOT, ST_TIME_SHARING, ST_WARM, ST_COLD = 0, 1, 2, 3
+
+
+def build(force: bool = False) -> str:
+    """Compile ffs_oracle.c with gcc (plain -O2, no fast-math)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-pthread", "-o", tmp, _SRC])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+class _PlanArgs(C.Structure):
+    _fields_ = [
+        ("P", C.c_int), ("gpcs", C.c_void_p), ("cap_mib", C.c_void_p),
+        ("F", C.c_int), ("comp_off", C.c_void_p), ("lat_us", C.c_void_p), ("mem_mib", C.c_void_p),
+        ("xfer_us", C.c_void_p), ("load_us", C.c_void_p),
+        ("n_nodes", C.c_int), ("n_slices", C.c_int),
+        ("sl_node", C.c_void_p), ("sl_gpu", C.c_void_p), ("sl_slice", C.c_void_p), ("sl_prof", C.c_void_p),
+        ("sl_busy", C.c_void_p),
+        ("R", C.c_int), ("req_func", C.c_void_p), ("req_node", C.c_void_p), ("req_slo_us", C.c_void_p),
+        ("k_max", C.c_int),
+        ("key", C.c_void_p), ("status", C.c_void_p), ("k", C.c_void_p), ("slice", C.c_void_p),
+        ("cut_mask", C.c_void_p), ("e2e_us", C.c_void_p), ("bottleneck_us", C.c_void_p),
+        ("gpcs_out", C.c_void_p), ("cvq", C.c_void_p), ("prof", C.c_void_p), ("checks", C.c_void_p),
+    ]
+
+
+def lib():
+    global _lib
+    with _lock:
+        if _lib is None:
+            _lib = C.CDLL(build())
+            _lib.oracle_plan.argtypes = [C.POINTER(_PlanArgs), C.c_int]
+            _lib.oracle_plan.restype = C.c_int
+            _lib.oracle_evict.restype = None
+            _lib.oracle_victim.restype = None
+    return _lib
+
+
+def _p(a):
+    return a.ctypes.data_as(C.c_void_p)
+
+
+def _c(a, dt):
+    return np.ascontiguousarray(a, dtype=dt)
+
+
+class _Held:
+    """Keeps the contiguous copies alive while the C call runs."""
+
+    def __init__(self, prob, k_max, with_checks):
+        self.gpcs = _c(prob.gpcs, np.uint32)
+        self.cap = _c(prob.cap_mib, np.uint32)
+        self.comp_off = _c(prob.comp_off, np.uint32)
+        self.lat = _c(prob.lat_us, np.uint32)
+        self.mem = _c(prob.mem_mib, np.uint32)
+        self.xfer = _c(prob.xfer_us, np.uint32)
+        self.load = _c(prob.load_us, np.uint32)
+        sl = prob.slices
+        self.sl_node = _c(sl["node"], np.uint16)
+        self.sl_gpu = _c(sl["gpu"], np.uint8)
+        self.sl_slice = _c(sl["slice"], np.uint8)
+        self.sl_prof = _c(sl["profile"], np.uint8)
+        self.sl_busy = _c(sl["busy"], np.uint8)
+        self.func = _c(prob.req["func"], np.uint32)
+        self.node = _c(prob.req["node"], np.uint32)
+        self.slo = _c(prob.slo_us, np.uint32)
+        R = self.func.shape[0]
+        self.out = {
+            "key": np.zeros(R, np.int64), "status": np.zeros(R, np.int32), "k": np.zeros(R, np.int32),
+            "slice": np.zeros((R, 8), np.int32), "cut_mask": np.zeros(R, np.uint32),
+            "e2e_us": np.zeros(R, np.uint32), "bottleneck_us": np.zeros(R, np.uint32),
+            "gpcs": np.zeros(R, np.uint32), "cvq": np.zeros(R, np.uint32), "prof": np.zeros((R, 8), np.uint8),
+        }
+        if with_checks:
+            self.out["checks"] = np.zeros((R, 3), np.uint64)
+        o = self.out
+        self.args = _PlanArgs(
+            int(self.gpcs.shape[0]), _p(self.gpcs), _p(self.cap),
+            int(self.comp_off.shape[0] - 1), _p(self.comp_off), _p(self.lat), _p(self.mem), _p(self.xfer),
+            _p(self.load), int(prob.n_nodes), int(self.sl_node.shape[0]),
+            _p(self.sl_node), _p(self.sl_gpu), _p(self.sl_slice), _p(self.sl_prof), _p(self.sl_busy),
+            int(R), _p(self.func), _p(self.node), _p(self.slo), int(k_max),
+            _p(o["key"]), _p(o["status"]), _p(o["k"]), _p(o["slice"]), _p(o["cut_mask"]), _p(o["e2e_us"]),
+            _p(o["bottleneck_us"]), _p(o["gpcs"]), _p(o["cvq"]), _p(o["prof"]),
+            _p(o["checks"]) if with_checks else None)
+
+
+def plan(prob, k_max: int | None = None, threads: int | None = None, checks: bool = True) -> dict:
+    """Brute-force plan of every request of ``prob`` (see ffs_oracle.c: oracle_plan).
+
+    Returns a dict of numpy arrays: key, status, k, cut_mask, e2e_us, bottleneck_us,
+    gpcs, cvq, prof[R,8] (0xFF = unused), slice[R,8] (-1 = unused) and, when
+    ``checks``, checks[R,3] = (candidates scored, feasible count, sum of feasible keys
+    mod 2^64)."""
+    k_max = int(prob.k_max if k_max is None else k_max)
+    threads = os.cpu_count() if threads is None else threads
+    h = _Held(prob, k_max, checks)
+    rc = lib().oracle_plan(C.byref(h.args), int(threads))
+    if rc != 0:
+        raise ValueError("oracle_plan rejected its arguments")
+    return h.out
+
+
+def evict(inst: np.ndarray, now_us: int, util_thr_pct: int = 30, window_us: int = 10_000_000,
+          cold_after_us: int = 600_000_000):
+    """Eviction state + LRU score of one snapshot (ffs_oracle.c: oracle_evict)."""
+    n = int(inst.shape[0])
+    sl = _c(inst["slice"], np.int32)
+    fl = _c(inst["flags"], np.uint8)
+    bu = _c(inst["busy_us"], np.uint32)
+    lu = _c(inst["last_used_us"], np.uint64)
+    score = np.zeros(n, np.int64)
+    state = np.zeros(n, np.uint8)
+    lib().oracle_evict(C.c_int(n), _p(sl), _p(fl), _p(bu), _p(lu), C.c_uint64(int(now_us)),
+                       C.c_uint32(util_thr_pct), C.c_uint32(window_us), C.c_uint64(int(cold_after_us)),
+                       _p(score), _p(state))
+    return score, state
+
+
+def victim(prob, status: np.ndarray, inst: np.ndarray, score: np.ndarray, k_max: int | None = None) -> np.ndarray:
+    """Time-share victim per INFEASIBLE request (ffs_oracle.c: oracle_victim)."""
+    h = _Held(prob, int(prob.k_max if k_max is None else k_max), False)
+    st = _c(status, np.int32)
+    sl = _c(inst["slice"], np.int32)
+    sc = _c(score, np.int64)
+    out = np.zeros(h.func.shape[0], np.int32)
+    lib().oracle_victim(C.byref(h.args), _p(st), C.c_int(int(inst.shape[0])), _p(sl), _p(sc), _p(out))
+    return out

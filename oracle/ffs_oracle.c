@@ -1,0 +1,393 @@
+/*
+ * ffs_oracle.c -- CPU ORACLE for the FluidFaaS batched pipeline-construction search.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  The product path
+ * (paper_conf_hpdc_hui0s25_b200/csrc, libffs.so) never links, includes or calls it,
+ * and this file includes nothing from the product tree.
+ *
+ * It is the plain, slow definition of what the hot path computes, written from the
+ * paper (P:<line> = line of /root/reference/PAPER.md) and the readings fixed in
+ * DESIGN.md §3 (R1..R21, which restate SURVEY.md §8(c)):
+ *
+ *   plan  (oracle_plan)   : for every request, brute force over every contiguous split
+ *                           of the component chain into k <= k_max stages (P:339,
+ *                           §5.2.2, "2^4 possible consecutive partitions") and every
+ *                           assignment of a MIG profile to each stage,
+ *                           feasibility = SLO + memory + free slices (P:217, P:343,
+ *                           P:392-394), balance = CV of stage times (Eq. 1),
+ *                           selection = argmin of the packed key (R1).  Stage sums are
+ *                           DIRECT sums over components ("Run all components in
+ *                           stage"), no prefix tables; masks are enumerated by nested
+ *                           choice of cut positions, not by the GPU's Gosper/unranking.
+ *   bind                  : lowest (gpu, slice) free slice of the stage's profile in the
+ *                           request's node, stages in order (R11, "available MIGs
+ *                           within the invoker").
+ *   evict (oracle_evict)  : multi-level keep-alive state + LRU key (§5.3).
+ *   victim(oracle_victim) : LRU time-sharing victim for a request with no free-slice
+ *                           plan.
+ *
+ * Arithmetic is exact integer arithmetic; the CV^2 quotient is taken with 128-bit
+ * integers so no bound has to be argued for the oracle itself.
+ *
+ * Parity status: every function here is pinned by tests/test_oracle_*.py against hand
+ * enumerations, the paper's worked scenarios (Fig. 1, Fig. 4, Table 5), closed forms,
+ * an independent Python brute force and the north_star invariants (a)-(d).
+ */
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+#include <pthread.h>
+
+#define ORACLE_MAX_STAGES 8
+#define ORACLE_MAX_P 8
+#define ORACLE_MAX_N 32
+#define KEY_NONE INT64_MAX
+
+/* per-plan status codes (R: "an infeasible request is not an error") */
+#define PLAN_OK 0
+#define PLAN_INFEASIBLE 1
+#define PLAN_BAD_REQ 2
+
+typedef struct {
+    /* profiles, Table 2 */
+    int P;
+    const uint32_t *gpcs, *cap_mib;
+    /* profile table, one chain per function */
+    int F;
+    const uint32_t *comp_off, *lat_us /* [C][P] */, *mem_mib, *xfer_us, *load_us;
+    /* cluster: slices sorted by (node, gpu, slice) */
+    int n_nodes, n_slices;
+    const uint16_t *sl_node;
+    const uint8_t *sl_gpu, *sl_slice, *sl_prof, *sl_busy;
+    /* requests */
+    int R;
+    const uint32_t *req_func, *req_node, *req_slo_us;
+    int k_max;
+    /* outputs, one row per request */
+    int64_t *key;
+    int32_t *status, *k, *slice /* [R][8] */;
+    uint32_t *cut_mask, *e2e_us, *bottleneck_us, *gpcs_out, *cvq;
+    uint8_t *prof /* [R][8] */;
+    uint64_t *checks /* [R][3] = scored, feasible, sum of feasible keys mod 2^64; nullable */;
+} oracle_plan_args;
+
+/* ---- state of one request's search ---------------------------------------------- */
+typedef struct {
+    const oracle_plan_args *a;
+    int f, v, n, k;
+    uint32_t B;
+    uint32_t free_cnt[ORACLE_MAX_P];
+    uint64_t idx; /* canonical candidate index (R1, R11) */
+    int64_t best;
+    int best_k;
+    uint32_t best_mask;
+    int best_prof[ORACLE_MAX_STAGES];
+    uint64_t nfeas, ksum;
+} req_state;
+
+static uint32_t lat_of(const oracle_plan_args *a, int f, int c, int p) {
+    return a->lat_us[(size_t)(a->comp_off[f] + c) * a->P + p];
+}
+
+/* Score every profile sequence for one cut mask (stages = maximal runs of components,
+ * a cut after component j iff bit j is set; "consecutive partitions"). */
+static void score_mask(req_state *s, uint32_t mask) {
+    const oracle_plan_args *a = s->a;
+    const int k = s->k, n = s->n, P = a->P;
+    /* stage boundaries: stage i covers components [first[i], last[i]] */
+    int first[ORACLE_MAX_STAGES], last[ORACLE_MAX_STAGES];
+    int st = 0;
+    first[0] = 0;
+    for (int c = 0; c < n; c++) {
+        int cut_after = (c < n - 1) && ((mask >> c) & 1u);
+        if (c == n - 1 || cut_after) {
+            last[st] = c;
+            st++;
+            if (st < k) first[st] = c + 1;
+        }
+    }
+    /* transfer cost of the cuts (R7): one xfer per cut position, counted in e2e only */
+    uint64_t xfer = 0;
+    for (int j = 0; j < n - 1; j++)
+        if ((mask >> j) & 1u) xfer += a->xfer_us[a->comp_off[s->f] + j];
+
+    uint64_t nseq = 1;
+    for (int i = 0; i < k; i++) nseq *= (uint64_t)P;
+
+    for (uint64_t seq = 0; seq < nseq; seq++) {
+        /* digits, p_1 most significant (R11) */
+        int p[ORACLE_MAX_STAGES];
+        uint64_t rest = seq;
+        for (int i = k - 1; i >= 0; i--) {
+            p[i] = (int)(rest % (uint64_t)P);
+            rest /= (uint64_t)P;
+        }
+        uint64_t t[ORACLE_MAX_STAGES], m[ORACLE_MAX_STAGES];
+        uint64_t sum_t = 0;
+        for (int i = 0; i < k; i++) {
+            t[i] = 0;
+            m[i] = 0;
+            for (int c = first[i]; c <= last[i]; c++) {
+                t[i] += lat_of(a, s->f, c, p[i]);            /* R5: sequential stage */
+                m[i] += a->mem_mib[a->comp_off[s->f] + c];    /* R6: all models loaded */
+            }
+            sum_t += t[i];
+        }
+        uint64_t e2e = sum_t + xfer;
+        /* feasibility (A4): memory per slice, free slices per profile, SLO (R8 inclusive) */
+        int feasible = 1;
+        for (int i = 0; i < k; i++)
+            if (m[i] > a->cap_mib[p[i]]) feasible = 0;
+        for (int q = 0; q < P; q++) {
+            uint32_t used = 0;
+            for (int i = 0; i < k; i++)
+                if (p[i] == q) used++;
+            if (used > s->free_cnt[q]) feasible = 0;
+        }
+        if (e2e > s->B) feasible = 0;
+
+        if (feasible) {
+            /* Eq. 1 squared, population std (R3): CV^2 = (k*sum t^2 - (sum t)^2)/(sum t)^2 */
+            unsigned __int128 sum_sq = 0;
+            for (int i = 0; i < k; i++) sum_sq += (unsigned __int128)t[i] * t[i];
+            unsigned __int128 D = (unsigned __int128)sum_t * sum_t;
+            unsigned __int128 N = (unsigned __int128)k * sum_sq - D;
+            uint64_t cvq = (uint64_t)(((unsigned __int128)1024 * N) / D); /* R4: Q10 floor */
+            uint64_t g = 0;
+            for (int i = 0; i < k; i++) g += a->gpcs[p[i]];
+            int64_t key = (int64_t)((cvq << 50) | ((uint64_t)(k - 1) << 47) | (g << 41) | s->idx);
+            if (key < s->best) {
+                s->best = key;
+                s->best_k = k;
+                s->best_mask = mask;
+                for (int i = 0; i < k; i++) s->best_prof[i] = p[i];
+            }
+            s->nfeas++;
+            s->ksum += (uint64_t)key;
+        }
+        s->idx++;
+    }
+}
+
+/* All masks over cut positions 0..limit-1 with `remaining` more bits, in ascending
+ * numeric order: the highest cut is chosen first, ascending, then the next lower one. */
+static void enum_masks(req_state *s, int remaining, int limit, uint32_t mask) {
+    if (remaining == 0) {
+        score_mask(s, mask);
+        return;
+    }
+    for (int j = remaining - 1; j < limit; j++) enum_masks(s, remaining - 1, j, mask | (1u << j));
+}
+
+static uint64_t binom(int n, int r) {
+    if (r < 0 || r > n) return 0;
+    uint64_t c = 1;
+    for (int i = 1; i <= r; i++) c = c * (uint64_t)(n - r + i) / (uint64_t)i;
+    return c;
+}
+
+static void plan_one(const oracle_plan_args *a, int r) {
+    int64_t *key = &a->key[r];
+    a->status[r] = PLAN_BAD_REQ;
+    *key = KEY_NONE;
+    a->k[r] = 0;
+    a->cut_mask[r] = 0;
+    a->e2e_us[r] = 0;
+    a->bottleneck_us[r] = 0;
+    a->gpcs_out[r] = 0;
+    a->cvq[r] = 0;
+    for (int i = 0; i < ORACLE_MAX_STAGES; i++) {
+        a->prof[(size_t)r * 8 + i] = 0xFF;
+        a->slice[(size_t)r * 8 + i] = -1;
+    }
+    if (a->checks) {
+        a->checks[(size_t)r * 3 + 0] = 0;
+        a->checks[(size_t)r * 3 + 1] = 0;
+        a->checks[(size_t)r * 3 + 2] = 0;
+    }
+    if (a->req_func[r] >= (uint32_t)a->F || a->req_node[r] >= (uint32_t)a->n_nodes) return;
+
+    req_state s;
+    memset(&s, 0, sizeof s);
+    s.a = a;
+    s.f = (int)a->req_func[r];
+    s.v = (int)a->req_node[r];
+    s.n = (int)(a->comp_off[s.f + 1] - a->comp_off[s.f]);
+    s.B = a->req_slo_us[r];
+    s.best = KEY_NONE;
+    /* free slices of each profile in the request's node (R10) */
+    for (int i = 0; i < a->n_slices; i++)
+        if (a->sl_node[i] == s.v && !a->sl_busy[i]) s.free_cnt[a->sl_prof[i]]++;
+
+    int kmax = a->k_max < s.n ? a->k_max : s.n;
+    for (int k = 1; k <= kmax; k++) {
+        s.k = k;
+        enum_masks(&s, k - 1, s.n - 1, 0u);
+    }
+    /* coverage: idx must equal S(n, K) = sum_k C(n-1, k-1) P^k */
+    uint64_t S = 0;
+    for (int k = 1; k <= kmax; k++) {
+        uint64_t pk = 1;
+        for (int i = 0; i < k; i++) pk *= (uint64_t)a->P;
+        S += binom(s.n - 1, k - 1) * pk;
+    }
+    if (s.idx != S) abort();
+    if (a->checks) {
+        a->checks[(size_t)r * 3 + 0] = s.idx;
+        a->checks[(size_t)r * 3 + 1] = s.nfeas;
+        a->checks[(size_t)r * 3 + 2] = s.ksum;
+    }
+    if (s.best == KEY_NONE) {
+        a->status[r] = PLAN_INFEASIBLE;
+        return;
+    }
+    /* the plan (A6): recompute the winner's figures from the table */
+    a->status[r] = PLAN_OK;
+    *key = s.best;
+    a->k[r] = s.best_k;
+    a->cut_mask[r] = s.best_mask;
+    a->cvq[r] = (uint32_t)((uint64_t)s.best >> 50);
+    uint64_t e2e = 0, bott = 0, g = 0;
+    int stage = 0;
+    uint64_t t = 0;
+    for (int c = 0; c < s.n; c++) {
+        t += lat_of(a, s.f, c, s.best_prof[stage]);
+        int cut_after = (c < s.n - 1) && ((s.best_mask >> c) & 1u);
+        if (cut_after) e2e += a->xfer_us[a->comp_off[s.f] + c];
+        if (c == s.n - 1 || cut_after) {
+            e2e += t;
+            if (t > bott) bott = t;
+            t = 0;
+            stage++;
+        }
+    }
+    for (int i = 0; i < s.best_k; i++) g += a->gpcs[s.best_prof[i]];
+    a->e2e_us[r] = (uint32_t)e2e;
+    a->bottleneck_us[r] = (uint32_t)bott; /* throughput = 1e6 / bottleneck_us (R17) */
+    a->gpcs_out[r] = (uint32_t)g;
+    /* bind: stage i takes the lowest-index free slice of its profile in node v that no
+     * earlier stage took (slices are sorted by (node, gpu, slice)) */
+    for (int i = 0; i < s.best_k; i++) {
+        a->prof[(size_t)r * 8 + i] = (uint8_t)s.best_prof[i];
+        for (int x = 0; x < a->n_slices; x++) {
+            if (a->sl_node[x] != s.v || a->sl_busy[x] || a->sl_prof[x] != s.best_prof[i]) continue;
+            int taken = 0;
+            for (int j = 0; j < i; j++)
+                if (a->slice[(size_t)r * 8 + j] == x) taken = 1;
+            if (taken) continue;
+            a->slice[(size_t)r * 8 + i] = x;
+            break;
+        }
+    }
+}
+
+typedef struct {
+    const oracle_plan_args *a;
+    int tid, nthreads;
+} worker_arg;
+
+static void *worker(void *p) {
+    worker_arg *w = (worker_arg *)p;
+    for (int r = w->tid; r < w->a->R; r += w->nthreads) plan_one(w->a, r); /* interleaved */
+    return NULL;
+}
+
+/* Returns 0 on success, -1 on bad arguments. */
+int oracle_plan(const oracle_plan_args *a, int n_threads) {
+    if (!a || a->P < 1 || a->P > ORACLE_MAX_P || a->k_max < 1 || a->k_max > ORACLE_MAX_STAGES) return -1;
+    for (int f = 0; f < a->F; f++) {
+        int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+        if (n < 1 || n > ORACLE_MAX_N) return -1;
+    }
+    if (n_threads < 1) n_threads = 1;
+    if (n_threads == 1) {
+        for (int r = 0; r < a->R; r++) plan_one(a, r);
+        return 0;
+    }
+    pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)n_threads);
+    worker_arg *wa = (worker_arg *)malloc(sizeof(worker_arg) * (size_t)n_threads);
+    for (int i = 0; i < n_threads; i++) {
+        wa[i].a = a;
+        wa[i].tid = i;
+        wa[i].nthreads = n_threads;
+        pthread_create(&th[i], NULL, worker, &wa[i]);
+    }
+    for (int i = 0; i < n_threads; i++) pthread_join(th[i], NULL);
+    free(th);
+    free(wa);
+    return 0;
+}
+
+/* ---- hotness-aware eviction ------------------------------------------ */
+#define ST_EXCL_HOT 0
+#define ST_TIME_SHARING 1
+#define ST_WARM 2
+#define ST_COLD 3
+#define FL_PIPELINE 1u
+#define FL_BUSY 2u
+
+/* One snapshot (tick).  Rules, in order (R18-R20):
+ *   idle >= cold_after                 -> COLD  ("no requests ... for 10 minutes")
+ *   not resident (slice < 0)           -> WARM  (evicted to CPU memory)
+ *   pipeline, or busy*100 >= thr*window -> EXCL_HOT (P:358 pipelines; P:370 threshold)
+ *   otherwise                          -> TIME_SHARING (utilization below 30%)
+ * score = (last_used << 20) | instance index for a resident, idle (not BUSY)
+ * time-sharing instance (LRU); every other instance scores INT64_MAX. */
+void oracle_evict(int n_inst, const int32_t *inst_slice, const uint8_t *inst_flags, const uint32_t *inst_busy_us,
+                  const uint64_t *inst_last_used_us, uint64_t now_us, uint32_t util_thr_pct, uint32_t window_us,
+                  uint64_t cold_after_us, int64_t *score, uint8_t *state) {
+    for (int i = 0; i < n_inst; i++) {
+        uint64_t last = inst_last_used_us[i];
+        uint64_t idle = now_us >= last ? now_us - last : 0;
+        uint8_t st;
+        if (idle >= cold_after_us)
+            st = ST_COLD;
+        else if (inst_slice[i] < 0)
+            st = ST_WARM;
+        else if ((inst_flags[i] & FL_PIPELINE) ||
+                 (uint64_t)inst_busy_us[i] * 100u >= (uint64_t)util_thr_pct * window_us)
+            st = ST_EXCL_HOT;
+        else
+            st = ST_TIME_SHARING;
+        state[i] = st;
+        if (st == ST_TIME_SHARING && !(inst_flags[i] & FL_BUSY))
+            score[i] = (int64_t)((last << 20) | (uint64_t)i);
+        else
+            score[i] = KEY_NONE;
+    }
+}
+
+/* Time-share victim for each request whose status is INFEASIBLE: among the
+ * instances with a finite score whose slice is in the request's node, whose slice
+ * profile holds the whole function (time-sharing instances are non-pipeline) and
+ * whose monolithic latency plus the reload time meets the budget ("deadlines
+ * subtracted by estimated execution and instance load times"), the one with
+ * the smallest score (least recently used).  -1 when there is none or when the
+ * request is not INFEASIBLE. */
+void oracle_victim(const oracle_plan_args *a, const int32_t *status, int n_inst, const int32_t *inst_slice,
+                   const int64_t *score, int32_t *victim) {
+    for (int r = 0; r < a->R; r++) {
+        victim[r] = -1;
+        if (status[r] != PLAN_INFEASIBLE) continue;
+        int f = (int)a->req_func[r], v = (int)a->req_node[r];
+        int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+        uint64_t mem = 0;
+        for (int c = 0; c < n; c++) mem += a->mem_mib[a->comp_off[f] + c];
+        int64_t best = KEY_NONE;
+        for (int i = 0; i < n_inst; i++) {
+            if (score[i] == KEY_NONE) continue;
+            int s = inst_slice[i];
+            if (s < 0 || s >= a->n_slices || a->sl_node[s] != v) continue;
+            int p = a->sl_prof[s];
+            if (mem > a->cap_mib[p]) continue;
+            uint64_t lat = 0;
+            for (int c = 0; c < n; c++) lat += lat_of(a, f, c, p);
+            if (lat + a->load_us[f] > a->req_slo_us[r]) continue;
+            if (score[i] < best) {
+                best = score[i];
+                victim[r] = i;
+            }
+        }
+    }
+}
