@@ -1,0 +1,247 @@
+/*
+ * ffs.h -- C ABI of libffs.so, the B200 (sm_100a) batched pipeline-construction search of
+ * FluidFaaS (Hui, Xu, Shen, HPDC '25).  Citations "P:<line>" are lines of the paper text
+ * (PAPER.md); "R<n>" are the readings fixed in DESIGN.md §3.
+ *
+ * What the library computes:
+ *   For every pending invocation (request) the invoker picks "the appropriate assignment
+ *   of MIG slices to the components in the DAG" by evaluating "all possible
+ *   partitions" of the component chain (§5.2.2) against "the available MIGs
+ *   within the invoker", ranking by the coefficient of variation of stage times
+ *   (Eq. 1), under the SLO and each slice's memory.
+ *   Candidate = (k stages <= k_max, cut mask, ordered profile sequence); the plan is the
+ *   feasible argmin of the packed key
+ *        key = cvq << 50 | (k-1) << 47 | gpcs << 41 | idx          (R1, R4)
+ *   cvq = floor(1024 * CV^2) with population std (R3), gpcs = sum of the stage profiles'
+ *   GPCs (ESG's "most resource-efficient option"), idx = canonical candidate index
+ *   (k ascending, cut masks in ascending numeric order, profile digits p_1 most
+ *   significant).  A feasible key is < 2^63 - 1, so INT64_MAX (FFS_KEY_NONE) = infeasible.
+ *   The hotness-aware eviction score is the second entry point.
+ *
+ * Conventions
+ *   - Every call returns ffs_status; no exception or abort crosses the ABI.  On a non-OK
+ *     status ffs_last_error() describes it.
+ *   - Integers are little-endian, fixed width; times in microseconds, memory in MiB (R14).
+ *   - Pointers prefixed d_ are DEVICE pointers on the context's device, caller-owned, read
+ *     or written only by stream work enqueued by the call (the call returns before that
+ *     work finishes unless stated).  h_ pointers are host memory (pinned recommended).
+ *     Tables passed to ffs_stage_tables are host memory copied during the call.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *   - The library allocates only context-owned scratch; it never frees caller memory.
+ *   - There is no CPU fallback: a context can only be created on a CUDA device with
+ *     compute capability 10.0 (sm_100a).
+ */
+#ifndef FFS_H
+#define FFS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    FFS_OK = 0,
+    FFS_ERR_ARG = -1,   /* null/ill-formed argument: lat = 0, non-monotone comp_off, unsorted slices ... */
+    FFS_ERR_RANGE = -2, /* a bound of the exact integer encoding is exceeded (see each call)  */
+    FFS_ERR_CUDA = -3,  /* a CUDA runtime call failed (message has the CUDA error string)       */
+    FFS_ERR_STATE = -4  /* tables not staged, or staged for a different shape                   */
+} ffs_status;
+
+#define FFS_MAX_PROFILES 8
+#define FFS_MAX_STAGES 8
+#define FFS_MAX_CHAIN 32
+#define FFS_KEY_NONE INT64_MAX
+
+/* per-plan status (an infeasible request is not an error) */
+#define FFS_PLAN_OK 0u
+#define FFS_PLAN_INFEASIBLE 1u
+#define FFS_PLAN_BAD_REQ 2u /* func >= n_funcs or node >= n_nodes */
+
+/* keep-alive states (Fig. 8) */
+#define FFS_ST_EXCL_HOT 0u
+#define FFS_ST_TIME_SHARING 1u
+#define FFS_ST_WARM 2u
+#define FFS_ST_COLD 3u
+/* ffs_instance.flags */
+#define FFS_INST_PIPELINE 1u /* pipeline instances are exclusive hot */
+#define FFS_INST_BUSY 2u     /* currently serving a request: never evicted   */
+
+typedef struct ffs_ctx ffs_ctx; /* opaque; one per device; owns staged tables and scratch */
+
+/* MIG profile table (Table 2).  gpcs[p] in 1..7, mem_mib[p] = slice memory. */
+typedef struct {
+    uint32_t n_profiles; /* P; this build is compiled for P = 5 (FFS_ERR_RANGE otherwise) */
+    uint32_t gpcs[FFS_MAX_PROFILES];
+    uint32_t mem_mib[FFS_MAX_PROFILES];
+} ffs_profiles;
+
+/* Per-component profile of every function ("the size of the required memory and
+ * the running speeds of the component on each size of MIG").  Function f's chain is
+ * components comp_off[f] .. comp_off[f+1]-1 (1 <= n_f <= 32).  Host pointers. */
+typedef struct {
+    uint32_t n_funcs;
+    const uint32_t *comp_off; /* [F+1], comp_off[0] = 0, strictly increasing          */
+    const uint32_t *lat_us;   /* [C][P] latency of component c alone on profile p, >= 1 */
+    const uint32_t *mem_mib;  /* [C] memory of component c                            */
+    const uint32_t *xfer_us;  /* [C] cost of a stage cut after component c (R7); the
+                                 last component's entry is ignored                     */
+    const uint32_t *load_us;  /* [F] warm -> MIG reload time (victim rule)     */
+} ffs_profile_table;
+
+/* One MIG slice of the cluster (12 bytes). */
+typedef struct {
+    uint16_t node;    /* invoker / node id (R10)           */
+    uint8_t gpu;      /* GPU within the node                */
+    uint8_t slice;    /* slice within the GPU               */
+    uint8_t profile;  /* index into ffs_profiles            */
+    uint8_t busy;     /* 1 = occupied (not free)            */
+    uint16_t pad;
+    int32_t instance; /* occupying instance or -1 (informational) */
+} ffs_slice;
+
+/* Cluster free-slice state.  Slices sorted by (node, gpu, slice) ascending; the free
+ * count of (node, profile) is derived from them.  Host pointer. */
+typedef struct {
+    uint32_t n_nodes;
+    uint32_t n_slices;
+    const ffs_slice *slices;
+} ffs_cluster;
+
+/* A pending invocation: function and home node.  Its latency budget B_r (remaining SLO,
+ * R9) is passed in a parallel uint32 array. */
+typedef struct {
+    uint32_t func, node;
+} ffs_request;
+
+/* The plan of one request (80 bytes) -- the "configuration layer" content: stages
+ * (cut_mask) and the MIG slice of every stage (Listing 1). */
+typedef struct {
+    int64_t key;            /* FFS_KEY_NONE when not OK                                  */
+    uint32_t status;        /* FFS_PLAN_*                                                 */
+    uint32_t k;             /* number of stages                                           */
+    uint32_t cut_mask;      /* bit j = stage boundary after component j                   */
+    uint32_t e2e_us;        /* sum of stage latencies + transfers of the cuts             */
+    uint32_t bottleneck_us; /* max stage latency; throughput = 1e6 / bottleneck_us rps    */
+    uint32_t gpcs;          /* sum of GPCs of the stages' profiles                        */
+    uint32_t cvq;           /* floor(1024 * CV^2) of the stage latencies (Eq. 1)          */
+    uint8_t prof[FFS_MAX_STAGES];  /* profile of stage i (0xFF unused)                    */
+    int32_t slice[FFS_MAX_STAGES]; /* bound slice index into ffs_cluster.slices (-1 unused) */
+    int32_t victim;         /* time-share victim instance (INFEASIBLE only) or -1          */
+} ffs_plan;
+
+/* A function instance as seen by the invoker's keep-alive manager (24 bytes). */
+typedef struct {
+    uint32_t func;
+    int32_t slice; /* resident on this slice, -1 = not resident (warm/cold) */
+    uint8_t flags; /* FFS_INST_* */
+    uint8_t pad[3];
+    uint32_t busy_us;      /* busy time within the utilisation window          */
+    uint64_t last_used_us; /* time of the last request (< 2^43)                */
+} ffs_instance;
+
+typedef struct {
+    uint32_t util_thr_pct;  /* 30                                    */
+    uint32_t window_us;     /* utilisation window (R18; default 10 s)        */
+    uint64_t cold_after_us; /* 600e6 = 10 minutes             */
+} ffs_evict_params;
+
+/* ---- context --------------------------------------------------------------------- */
+/* Create a context on `cuda_device`.  FFS_ERR_CUDA if the device is not sm_100. */
+ffs_status ffs_create(int cuda_device, ffs_ctx **out);
+void ffs_destroy(ffs_ctx *ctx);
+/* Message for the last non-OK status returned on this context (never NULL). */
+const char *ffs_last_error(const ffs_ctx *ctx);
+
+/* ---- A0: stage tables --------------------------------------------------------------
+ * Validate, prefix-sum and upload the profile table and the cluster free-slice state
+ * (P:217).  Synchronous; host memory is only read during the call.
+ * FFS_ERR_ARG   : null pointers, lat = 0, comp_off not strictly increasing, slices not
+ *                 sorted by (node, gpu, slice), node >= n_nodes, profile >= P, gpcs not
+ *                 in 1..7.
+ * FFS_ERR_RANGE : P != 5, n_f > 32, sum_c max_p lat >= 2^24, sum xfer >= 2^24,
+ *                 sum mem >= 2^31, n_nodes >= 2^16. */
+ffs_status ffs_stage_tables(ffs_ctx *ctx, const ffs_profiles *profiles, const ffs_profile_table *table,
+                            const ffs_cluster *cluster);
+
+/* ---- A1-A5: keys ---------------------------------------------------------------------
+ * Partial argmin keys of shard `rank` of `world` (0 <= rank < world): for every k the
+ * flattened (request, cut mask) task list is split into `world` equal contiguous ranges
+ * and this call scores every candidate of range `rank`.  d_keys[r] receives the minimum
+ * feasible key of request r within the shard, FFS_KEY_NONE where none (overwritten, not
+ * combined with its previous content).  Combine shards with an element-wise MIN
+ * (torch.distributed.all_reduce(keys, MIN) over NCCL) before ffs_plan_decode.
+ * d_checksums (nullable; verify mode, slower): uint64[3*n_req] = per request {candidates
+ * scored, feasible candidates, sum of feasible keys mod 2^64} of this shard; combine
+ * with SUM.  Asynchronous on `stream`.
+ * FFS_ERR_RANGE: k_max not in 1..8, S(n, k_max) >= 2^41 for a staged function,
+ * k_max * max gpcs >= 64.  FFS_ERR_STATE: tables not staged. */
+ffs_status ffs_plan_keys(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                         uint32_t k_max, uint32_t rank, uint32_t world, int64_t *d_keys, uint64_t *d_checksums,
+                         void *stream);
+
+/* ---- A6 (+A8): decode and bind ---------------------------------------------------------
+ * Decode the combined keys into plans and bind every stage, in stage order, to the
+ * lowest-index free slice of its profile in the request's node not taken by an earlier
+ * stage (R11).  When d_inst and d_evict_scores are non-null, an INFEASIBLE request gets
+ * the time-share victim of A8: the instance with the smallest eviction score
+ * (from ffs_evict_scores on the same snapshot) resident in the request's node on a slice
+ * that holds the whole function and meets lat + load <= budget; -1 if none.
+ * Asynchronous on `stream`.  k_max must equal the one given to ffs_plan_keys. */
+ffs_status ffs_plan_decode(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, const int64_t *d_keys,
+                           uint32_t n_req, uint32_t k_max, const ffs_instance *d_inst,
+                           const int64_t *d_evict_scores, uint32_t n_inst, ffs_plan *d_out, void *stream);
+
+/* ---- one-GPU convenience: keys + decode (no victims) ---------------------------------
+ * Uses context scratch for the keys.  Asynchronous on `stream`. */
+ffs_status ffs_plan_batch(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                          uint32_t k_max, ffs_plan *d_out, void *stream);
+
+/* Same with HOST buffers: copies the requests and budgets host->device, plans, copies
+ * the plans device->host and synchronises `stream` before returning (the end-to-end
+ * call of a user holding host data). */
+ffs_status ffs_plan_batch_host(ffs_ctx *ctx, const ffs_request *h_req, const uint32_t *h_slo_us, uint32_t n_req,
+                               uint32_t k_max, ffs_plan *h_out, void *stream);
+
+/* ---- A7: hotness-aware eviction scores -------------------------------------------------
+ * One snapshot of n_inst instances at time now_us.  State, in order:
+ *   idle = now - last_used (0 if negative) >= cold_after   -> COLD
+ *   slice < 0 (not resident)                               -> WARM
+ *   PIPELINE flag, or busy_us*100 >= util_thr_pct*window_us -> EXCL_HOT
+ *   otherwise                                              -> TIME_SHARING
+ * d_score[i] = (last_used_us << 20) | i for a TIME_SHARING instance without the BUSY
+ * flag (the LRU key), FFS_KEY_NONE otherwise.  d_state[i] = FFS_ST_*.
+ * FFS_ERR_RANGE: n_inst > 2^20.  (last_used_us >= 2^43 scores FFS_KEY_NONE.)  Async. */
+ffs_status ffs_evict_scores(ffs_ctx *ctx, const ffs_instance *d_inst, uint32_t n_inst, uint64_t now_us,
+                            const ffs_evict_params *params, int64_t *d_score, uint8_t *d_state, void *stream);
+
+/* Batched over n_ticks snapshots: tick t owns instances d_tick_off[t] .. d_tick_off[t+1]-1
+ * (device array, n_ticks+1 entries, non-decreasing) at time d_now_us[t]; the index in the
+ * score is the index within the tick.  An instance at index >= 2^20 within its tick
+ * scores FFS_KEY_NONE.  Async. */
+ffs_status ffs_evict_scores_ticks(ffs_ctx *ctx, const ffs_instance *d_inst, const uint32_t *d_tick_off,
+                                  const uint64_t *d_now_us, uint32_t n_ticks, const ffs_evict_params *params,
+                                  int64_t *d_score, uint8_t *d_state, void *stream);
+
+/* A8 batched over ticks: for every request r (tick d_req_tick[r]) the victim among the
+ * instances of that tick, by the rule of ffs_plan_decode, regardless of the request's
+ * plan (the caller passes the loads that need one).  d_victim[r] = index within the tick
+ * or -1.  Async. */
+ffs_status ffs_evict_victims(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us,
+                             const uint32_t *d_req_tick, uint32_t n_req, const ffs_instance *d_inst,
+                             const uint32_t *d_tick_off, const int64_t *d_score, uint32_t n_ticks,
+                             int32_t *d_victim, void *stream);
+
+/* ---- measurement / debug helpers ------------------------------------------------------
+ * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
+ * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */
+ffs_status ffs_bench_int_peak(ffs_ctx *ctx, double *ops_per_s, double *seconds);
+/* Number of candidates, since the context was created, that the fast float filter
+ * rejected although their exact key would have beaten the running minimum (verify mode
+ * only; must be 0).  Synchronous. */
+ffs_status ffs_debug_filter_misses(ffs_ctx *ctx, uint64_t *out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FFS_H */

@@ -1,0 +1,478 @@
+// ffs_host.cu -- host side of libffs.so: context, validation and staging of the tables
+// (A0), scratch management and the C-ABI entry points declared in include/ffs.h.
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "ffs_internal.h"
+
+using namespace ffsk;
+
+namespace {
+
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  cudaError_t ensure(size_t n) {
+    if (n <= bytes) return cudaSuccess;
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+    cudaError_t e = cudaMalloc(&p, n);
+    if (e == cudaSuccess) bytes = n;
+    return e;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+  }
+  template <class T>
+  T* as() const { return reinterpret_cast<T*>(p); }
+};
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace
+
+struct ffs_ctx {
+  int device = 0;
+  int sms = 0;
+  std::string err;
+  // staged tables
+  bool staged = false;
+  ImageLayout lay{};
+  uint32_t P = 0, F = 0, n_nodes = 0, n_slices = 0, max_n = 0, max_gpcs = 0;
+  std::vector<uint32_t> fn_len;
+  DevBuf image, node_free, free_list, slice_node, slice_prof;
+  // scratch
+  DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses;
+  // cached occupancy per (ks, verify, smem)
+  size_t occ_smem = 0;
+  int occ[2][kMaxK + 1] = {};
+};
+
+static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  if (c) c->err = buf;
+  return s;
+}
+
+static ffs_status cuda_fail(ffs_ctx* c, cudaError_t e, const char* what) {
+  return fail(c, FFS_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(expr, what)                              \
+  do {                                              \
+    cudaError_t _e = (expr);                        \
+    if (_e != cudaSuccess) return cuda_fail(c, _e, what); \
+  } while (0)
+
+static uint64_t binom64(int n, int r) {
+  if (r < 0 || n < 0 || r > n) return 0;
+  uint64_t v = 1;
+  for (int i = 1; i <= r; ++i) v = v * (uint64_t)(n - r + i) / (uint64_t)i;
+  return v;
+}
+
+extern "C" {
+
+ffs_status ffs_create(int cuda_device, ffs_ctx** out) {
+  if (!out) return FFS_ERR_ARG;
+  *out = nullptr;
+  int n = 0;
+  cudaError_t e = cudaGetDeviceCount(&n);
+  if (e != cudaSuccess || cuda_device < 0 || cuda_device >= n) return FFS_ERR_CUDA;
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, cuda_device) != cudaSuccess) return FFS_ERR_CUDA;
+  if (prop.major != 10 || prop.minor != 0) return FFS_ERR_CUDA;  // built for sm_100a only
+  ffs_ctx* c = new ffs_ctx;
+  c->device = cuda_device;
+  c->sms = prop.multiProcessorCount;
+  {
+    DeviceGuard g(c->device);
+    if (c->misses.ensure(8) != cudaSuccess || cudaMemset(c->misses.p, 0, 8) != cudaSuccess) {
+      delete c;
+      return FFS_ERR_CUDA;
+    }
+  }
+  *out = c;
+  return FFS_OK;
+}
+
+void ffs_destroy(ffs_ctx* c) {
+  if (!c) return;
+  {
+    DeviceGuard g(c->device);
+    for (DevBuf* b : {&c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
+                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses})
+      b->release();
+  }
+  delete c;
+}
+
+const char* ffs_last_error(const ffs_ctx* c) { return c ? c->err.c_str() : "null context"; }
+
+ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profile_table* tb, const ffs_cluster* cl) {
+  if (!c) return FFS_ERR_ARG;
+  c->staged = false;
+  if (!pr || !tb || !cl) return fail(c, FFS_ERR_ARG, "null table pointer");
+  if (pr->n_profiles != (uint32_t)kP)
+    return fail(c, FFS_ERR_RANGE, "this build is compiled for P=%d profiles (got %u)", kP, pr->n_profiles);
+  const uint32_t P = pr->n_profiles, F = tb->n_funcs;
+  if (F == 0 || !tb->comp_off || !tb->lat_us || !tb->mem_mib || !tb->xfer_us || !tb->load_us)
+    return fail(c, FFS_ERR_ARG, "empty or null profile table");
+  uint32_t max_g = 0;
+  for (uint32_t p = 0; p < P; ++p) {
+    if (pr->gpcs[p] < 1 || pr->gpcs[p] > 7) return fail(c, FFS_ERR_ARG, "gpcs[%u]=%u not in 1..7", p, pr->gpcs[p]);
+    max_g = std::max(max_g, pr->gpcs[p]);
+  }
+  if (tb->comp_off[0] != 0) return fail(c, FFS_ERR_ARG, "comp_off[0] != 0");
+  uint32_t max_n = 0;
+  std::vector<uint32_t> len(F);
+  for (uint32_t f = 0; f < F; ++f) {
+    if (tb->comp_off[f + 1] <= tb->comp_off[f]) return fail(c, FFS_ERR_ARG, "comp_off not strictly increasing at %u", f);
+    len[f] = tb->comp_off[f + 1] - tb->comp_off[f];
+    if (len[f] > (uint32_t)kMaxN) return fail(c, FFS_ERR_RANGE, "function %u has %u > 32 components", f, len[f]);
+    max_n = std::max(max_n, len[f]);
+  }
+  const uint32_t C = tb->comp_off[F];
+  // exact-encoding bounds (DESIGN.md §3 R4): sum_c max_p lat < 2^24, sum xfer < 2^24, sum mem < 2^31
+  for (uint32_t f = 0; f < F; ++f) {
+    uint64_t smax = 0, sx = 0, sm = 0;
+    for (uint32_t i = tb->comp_off[f]; i < tb->comp_off[f + 1]; ++i) {
+      uint32_t mx = 0;
+      for (uint32_t p = 0; p < P; ++p) {
+        const uint32_t l = tb->lat_us[(uint64_t)i * P + p];
+        if (l == 0) return fail(c, FFS_ERR_ARG, "lat[%u][%u] = 0", i, p);
+        mx = std::max(mx, l);
+      }
+      smax += mx;
+      if (i + 1 < tb->comp_off[f + 1]) sx += tb->xfer_us[i];
+      sm += tb->mem_mib[i];
+    }
+    if (smax >= (1u << 24)) return fail(c, FFS_ERR_RANGE, "function %u: sum of latencies >= 2^24 us", f);
+    if (sx >= (1u << 24)) return fail(c, FFS_ERR_RANGE, "function %u: sum of transfer costs >= 2^24 us", f);
+    if (sm >= (1ull << 31)) return fail(c, FFS_ERR_RANGE, "function %u: memory >= 2^31 MiB", f);
+  }
+  if (cl->n_nodes == 0 || cl->n_nodes >= (1u << 16)) return fail(c, FFS_ERR_RANGE, "n_nodes must be in 1..65535");
+  if (cl->n_slices && !cl->slices) return fail(c, FFS_ERR_ARG, "null slices");
+  for (uint32_t s = 0; s < cl->n_slices; ++s) {
+    const ffs_slice& x = cl->slices[s];
+    if (x.node >= cl->n_nodes) return fail(c, FFS_ERR_ARG, "slice %u: node %u >= n_nodes", s, x.node);
+    if (x.profile >= P) return fail(c, FFS_ERR_ARG, "slice %u: profile %u >= P", s, x.profile);
+    if (s) {
+      const ffs_slice& y = cl->slices[s - 1];
+      const uint64_t ky = ((uint64_t)y.node << 16) | ((uint64_t)y.gpu << 8) | y.slice;
+      const uint64_t kx = ((uint64_t)x.node << 16) | ((uint64_t)x.gpu << 8) | x.slice;
+      if (kx <= ky) return fail(c, FFS_ERR_ARG, "slices not sorted by (node, gpu, slice) at %u", s);
+    }
+  }
+
+  // ---- build the table image (ImageLayout) ----
+  ImageLayout L{};
+  uint32_t w = 0;
+  auto take = [&](uint32_t n, uint32_t align) {
+    w = (w + align - 1) / align * align;
+    uint32_t o = w;
+    w += n;
+    return o;
+  };
+  L.F = F;
+  L.o_gpcs = take(8, 4);
+  L.o_cap = take(8, 4);
+  L.o_binom = take(33 * 8, 4);
+  L.o_offk = take(33 * 10 * 2, 4);
+  L.o_fdesc = take(4 * F, 4);
+  const uint32_t rows = C + F;  // n_f + 1 boundaries per function
+  L.o_pl = take(rows * kRowW, 4);
+  L.o_pm = take(rows, 4);
+  L.o_xf = take(rows, 4);
+  L.words = (w + 3) / 4 * 4;
+  std::vector<uint32_t> img(L.words, 0);
+  for (uint32_t p = 0; p < 8; ++p) {
+    img[L.o_gpcs + p] = p < P ? pr->gpcs[p] : 0;
+    img[L.o_cap + p] = p < P ? pr->mem_mib[p] : 0;
+  }
+  for (int n = 0; n <= 32; ++n)
+    for (int i = 0; i < 8; ++i) img[L.o_binom + n * 8 + i] = (uint32_t)binom64(n, i);
+  for (int n = 1; n <= 32; ++n) {
+    uint64_t acc = 0, pk = 1;
+    for (int k = 1; k <= 9; ++k) {
+      img[L.o_offk + 2 * (n * 10 + k)] = (uint32_t)acc;
+      img[L.o_offk + 2 * (n * 10 + k) + 1] = (uint32_t)(acc >> 32);
+      pk *= P;
+      if (k <= 8) acc += binom64(n - 1, k - 1) * pk;
+    }
+  }
+  uint32_t row = 0;
+  for (uint32_t f = 0; f < F; ++f) {
+    const uint32_t c0 = tb->comp_off[f], n = len[f];
+    uint64_t mtot = 0;
+    for (uint32_t i = 0; i < n; ++i) mtot += tb->mem_mib[c0 + i];
+    img[L.o_fdesc + 4 * f + 0] = row;
+    img[L.o_fdesc + 4 * f + 1] = n;
+    img[L.o_fdesc + 4 * f + 2] = tb->load_us[f];
+    img[L.o_fdesc + 4 * f + 3] = (uint32_t)mtot;
+    for (uint32_t p = 0; p < 8; ++p) img[L.o_pl + row * kRowW + p] = 0;
+    img[L.o_pm + row] = 0;
+    for (uint32_t i = 0; i < n; ++i) {
+      for (uint32_t p = 0; p < 8; ++p)
+        img[L.o_pl + (row + i + 1) * kRowW + p] =
+            img[L.o_pl + (row + i) * kRowW + p] + (p < P ? tb->lat_us[(uint64_t)(c0 + i) * P + p] : 0);
+      img[L.o_pm + row + i + 1] = img[L.o_pm + row + i] + tb->mem_mib[c0 + i];
+      img[L.o_xf + row + i] = (i + 1 < n) ? tb->xfer_us[c0 + i] : 0;
+    }
+    row += n + 1;
+  }
+  if ((size_t)L.words * 4 > 200 * 1024)
+    return fail(c, FFS_ERR_RANGE, "table image %u bytes exceeds the 200 KB shared-memory stage", L.words * 4);
+
+  // ---- per node: free counts (clamped to 8) and the first 8 free slices per profile ----
+  const uint32_t NN = cl->n_nodes;
+  std::vector<uint64_t> node_free(NN, 0);
+  std::vector<int32_t> free_list((size_t)NN * 64, -1);
+  std::vector<uint16_t> snode(std::max(1u, cl->n_slices));
+  std::vector<uint8_t> sprof(std::max(1u, cl->n_slices));
+  std::vector<uint8_t> cnt((size_t)NN * 8, 0);
+  for (uint32_t s = 0; s < cl->n_slices; ++s) {
+    const ffs_slice& x = cl->slices[s];
+    snode[s] = x.node;
+    sprof[s] = x.profile;
+    if (x.busy) continue;
+    uint8_t& k = cnt[(size_t)x.node * 8 + x.profile];
+    if (k < 8) free_list[((size_t)x.node * 8 + x.profile) * 8 + k] = (int32_t)s;
+    if (k < 255) ++k;
+  }
+  for (uint32_t v = 0; v < NN; ++v)
+    for (uint32_t p = 0; p < 8; ++p)
+      node_free[v] |= (uint64_t)std::min<uint32_t>(cnt[(size_t)v * 8 + p], 8) << (8 * p);
+
+  DeviceGuard g(c->device);
+  CK(c->image.ensure((size_t)L.words * 4), "cudaMalloc(image)");
+  CK(cudaMemcpy(c->image.p, img.data(), (size_t)L.words * 4, cudaMemcpyHostToDevice), "upload image");
+  CK(c->node_free.ensure(NN * 8), "cudaMalloc(node_free)");
+  CK(cudaMemcpy(c->node_free.p, node_free.data(), NN * 8, cudaMemcpyHostToDevice), "upload node_free");
+  CK(c->free_list.ensure(free_list.size() * 4), "cudaMalloc(free_list)");
+  CK(cudaMemcpy(c->free_list.p, free_list.data(), free_list.size() * 4, cudaMemcpyHostToDevice), "upload free_list");
+  CK(c->slice_node.ensure(snode.size() * 2), "cudaMalloc(slice_node)");
+  CK(cudaMemcpy(c->slice_node.p, snode.data(), snode.size() * 2, cudaMemcpyHostToDevice), "upload slice_node");
+  CK(c->slice_prof.ensure(sprof.size()), "cudaMalloc(slice_prof)");
+  CK(cudaMemcpy(c->slice_prof.p, sprof.data(), sprof.size(), cudaMemcpyHostToDevice), "upload slice_prof");
+  c->lay = L;
+  c->P = P;
+  c->F = F;
+  c->n_nodes = NN;
+  c->n_slices = cl->n_slices;
+  c->max_n = max_n;
+  c->max_gpcs = max_g;
+  c->fn_len = len;
+  c->staged = true;
+  c->occ_smem = 0;
+  return FFS_OK;
+}
+
+static ffs_status check_kmax(ffs_ctx* c, uint32_t k_max) {
+  if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  if (k_max < 1 || k_max > (uint32_t)kMaxK) return fail(c, FFS_ERR_RANGE, "k_max %u not in 1..8", k_max);
+  if (k_max * c->max_gpcs >= 64) return fail(c, FFS_ERR_RANGE, "k_max * max gpcs >= 64 (6-bit key field)");
+  // S(n, K) < 2^41 for every staged function (idx field)
+  uint64_t pk = 1, S = 0;
+  for (uint32_t k = 1; k <= std::min(k_max, c->max_n); ++k) {
+    pk *= c->P;
+    S += binom64((int)c->max_n - 1, (int)k - 1) * pk;
+  }
+  if (S >= (1ull << kIdxBits)) return fail(c, FFS_ERR_RANGE, "S(n=%u, K=%u) >= 2^41", c->max_n, k_max);
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req, uint32_t k_max,
+                         uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  ffs_status s = check_kmax(c, k_max);
+  if (s != FFS_OK) return s;
+  if (world == 0 || rank >= world) return fail(c, FFS_ERR_ARG, "rank %u / world %u", rank, world);
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_keys) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const uint64_t len = (uint64_t)n_req + 1;
+  CK(c->prefix.ensure(len * k_max * 8), "cudaMalloc(prefix)");
+  const uint64_t nb = (len + 2047) / 2048;
+  CK(c->block_sums.ensure(nb * k_max * 8 + 8), "cudaMalloc(block_sums)");
+  CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, c->prefix.as<uint64_t>(),
+                        c->block_sums.as<uint64_t>(), d_keys, reinterpret_cast<unsigned long long*>(d_checks), st),
+     "count/scan kernels");
+  const size_t smem = (size_t)c->lay.words * 4;
+  if (c->occ_smem != smem) {
+    for (int v = 0; v < 2; ++v)
+      for (int k = 1; k <= kMaxK; ++k) {
+        int b = 0;
+        CK(search_kernel_config(k, v != 0, smem, &b), "search kernel occupancy");
+        c->occ[v][k] = std::max(1, b);
+      }
+    c->occ_smem = smem;
+  }
+  SearchArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.req = d_req;
+  a.slo = d_slo;
+  a.node_free = c->node_free.as<uint64_t>();
+  a.prefix = c->prefix.as<uint64_t>();
+  a.n_req = n_req;
+  a.rank = rank;
+  a.world = world;
+  a.keys = d_keys;
+  a.checks = reinterpret_cast<unsigned long long*>(d_checks);
+  a.misses = c->misses.as<unsigned long long>();
+  const bool verify = d_checks != nullptr;
+  for (uint32_t k = 1; k <= std::min(k_max, c->max_n); ++k) {
+    const int grid = c->sms * c->occ[verify ? 1 : 0][k];
+    CK(launch_search((int)k, verify, a, grid, smem, st), "search kernel");
+  }
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_decode(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, const int64_t* d_keys,
+                           uint32_t n_req, uint32_t k_max, const ffs_instance* d_inst, const int64_t* d_scores,
+                           uint32_t n_inst, ffs_plan* d_out, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  ffs_status s = check_kmax(c, k_max);
+  if (s != FFS_OK) return s;
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_keys || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
+  if ((d_inst == nullptr) != (d_scores == nullptr)) return fail(c, FFS_ERR_ARG, "d_inst and d_evict_scores must both be set");
+  DeviceGuard g(c->device);
+  DecodeArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.req = d_req;
+  a.slo = d_slo;
+  a.keys = d_keys;
+  a.n_req = n_req;
+  a.k_max = k_max;
+  a.n_nodes = c->n_nodes;
+  a.n_slices = c->n_slices;
+  a.free_list = c->free_list.as<int32_t>();
+  a.slice_node = c->slice_node.as<uint16_t>();
+  a.slice_prof = c->slice_prof.as<uint8_t>();
+  a.inst = d_inst;
+  a.score = d_scores;
+  a.n_inst = d_inst ? n_inst : 0;
+  a.out = d_out;
+  CK(launch_decode(a, (cudaStream_t)stream), "decode kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_batch(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req, uint32_t k_max,
+                          ffs_plan* d_out, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  {
+    DeviceGuard g(c->device);
+    CK(c->keys.ensure((size_t)std::max(1u, n_req) * 8), "cudaMalloc(keys)");
+  }
+  ffs_status s = ffs_plan_keys(c, d_req, d_slo, n_req, k_max, 0, 1, c->keys.as<int64_t>(), nullptr, stream);
+  if (s != FFS_OK) return s;
+  return ffs_plan_decode(c, d_req, d_slo, c->keys.as<int64_t>(), n_req, k_max, nullptr, nullptr, 0, d_out, stream);
+}
+
+ffs_status ffs_plan_batch_host(ffs_ctx* c, const ffs_request* h_req, const uint32_t* h_slo, uint32_t n_req,
+                               uint32_t k_max, ffs_plan* h_out, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (n_req == 0) return FFS_OK;
+  if (!h_req || !h_slo || !h_out) return fail(c, FFS_ERR_ARG, "null host pointer");
+  cudaStream_t st = (cudaStream_t)stream;
+  {
+    DeviceGuard g(c->device);
+    CK(c->req_dev.ensure((size_t)n_req * sizeof(ffs_request)), "cudaMalloc(req)");
+    CK(c->slo_dev.ensure((size_t)n_req * 4), "cudaMalloc(slo)");
+    CK(c->plans_dev.ensure((size_t)n_req * sizeof(ffs_plan)), "cudaMalloc(plans)");
+    CK(cudaMemcpyAsync(c->req_dev.p, h_req, (size_t)n_req * sizeof(ffs_request), cudaMemcpyHostToDevice, st), "H2D req");
+    CK(cudaMemcpyAsync(c->slo_dev.p, h_slo, (size_t)n_req * 4, cudaMemcpyHostToDevice, st), "H2D slo");
+  }
+  ffs_status s = ffs_plan_batch(c, c->req_dev.as<ffs_request>(), c->slo_dev.as<uint32_t>(), n_req, k_max,
+                                c->plans_dev.as<ffs_plan>(), stream);
+  if (s != FFS_OK) return s;
+  DeviceGuard g(c->device);
+  CK(cudaMemcpyAsync(h_out, c->plans_dev.p, (size_t)n_req * sizeof(ffs_plan), cudaMemcpyDeviceToHost, st), "D2H plans");
+  CK(cudaStreamSynchronize(st), "stream sync");
+  return FFS_OK;
+}
+
+ffs_status ffs_evict_scores(ffs_ctx* c, const ffs_instance* d_inst, uint32_t n_inst, uint64_t now_us,
+                            const ffs_evict_params* prm, int64_t* d_score, uint8_t* d_state, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!prm) return fail(c, FFS_ERR_ARG, "null params");
+  if (n_inst > (1u << 20)) return fail(c, FFS_ERR_RANGE, "n_inst %u > 2^20", n_inst);
+  if (n_inst == 0) return FFS_OK;
+  if (!d_inst || !d_score || !d_state) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  CK(launch_evict(d_inst, n_inst, nullptr, nullptr, 0, now_us, *prm, d_score, d_state, (cudaStream_t)stream),
+     "evict kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_evict_scores_ticks(ffs_ctx* c, const ffs_instance* d_inst, const uint32_t* d_tick_off,
+                                  const uint64_t* d_now_us, uint32_t n_ticks, const ffs_evict_params* prm,
+                                  int64_t* d_score, uint8_t* d_state, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!prm) return fail(c, FFS_ERR_ARG, "null params");
+  if (n_ticks == 0) return FFS_OK;
+  if (!d_inst || !d_tick_off || !d_now_us || !d_score || !d_state) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  CK(launch_evict(d_inst, 0, d_tick_off, d_now_us, n_ticks, 0, *prm, d_score, d_state, (cudaStream_t)stream),
+     "evict kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_evict_victims(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, const uint32_t* d_req_tick,
+                             uint32_t n_req, const ffs_instance* d_inst, const uint32_t* d_tick_off,
+                             const int64_t* d_score, uint32_t n_ticks, int32_t* d_victim, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_req_tick || !d_inst || !d_tick_off || !d_score || !d_victim)
+    return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  CK(launch_victims(c->image.as<uint32_t>(), c->lay, d_req, d_slo, d_req_tick, n_req, d_inst, d_tick_off, d_score,
+                    n_ticks, c->slice_node.as<uint16_t>(), c->slice_prof.as<uint8_t>(), c->n_slices, d_victim,
+                    (cudaStream_t)stream),
+     "victims kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_bench_int_peak(ffs_ctx* c, double* ops, double* seconds) {
+  if (!c || !ops || !seconds) return FFS_ERR_ARG;
+  DeviceGuard g(c->device);
+  CK(run_int_peak(c->sms, ops, seconds), "int peak kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_debug_filter_misses(ffs_ctx* c, uint64_t* out) {
+  if (!c || !out) return FFS_ERR_ARG;
+  DeviceGuard g(c->device);
+  CK(cudaDeviceSynchronize(), "sync");
+  CK(cudaMemcpy(out, c->misses.p, 8, cudaMemcpyDeviceToHost), "read misses");
+  return FFS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,84 @@
+// ffs_internal.h -- shared between the host side (ffs_host.cu) and the kernels
+// (ffs_kernels.cu) of libffs.so.  Not part of the ABI.  Nothing here is shared with the
+// CPU oracle (oracle/), which is independent test infrastructure.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "ffs.h"
+
+namespace ffsk {
+
+constexpr int kP = 5;          // profiles this build is compiled for (Table 2)
+constexpr int kRowW = 8;       // words per prefix-latency row (P padded to 8 -> 2 x LDS.128)
+constexpr int kMaxN = 32;      // max components per chain (cut masks fit in uint32)
+constexpr int kMaxK = 8;       // max stages
+constexpr int kIdxBits = 41;   // canonical index field of the key
+constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
+constexpr int kBlock = 256;    // threads per CTA of the search kernel
+
+// Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
+// image into shared memory once per CTA (A0 of DESIGN.md §4); every other kernel reads
+// it from global memory.
+struct ImageLayout {
+  uint32_t words;     // total size in words, multiple of 4 (16-byte copies)
+  uint32_t F;         // functions
+  uint32_t o_gpcs;    // [8] u32
+  uint32_t o_cap;     // [8] u32 slice memory (MiB)
+  uint32_t o_binom;   // [33][8] u32 C(c, i), c <= 32, i <= 7
+  uint32_t o_offk;    // [33][10] u64 (word pairs) offk[n][k] = sum_{k'<k} C(n-1,k'-1) P^k'
+  uint32_t o_fdesc;   // [F][4] u32 {row0, n, load_us, mem_total}
+  uint32_t o_pl;      // [rows][8] u32 PL[row0+i][p] = sum_{c<i} lat[c][p]  (16-byte aligned)
+  uint32_t o_pm;      // [rows] u32 PM[row0+i] = sum_{c<i} mem[c]
+  uint32_t o_xf;      // [rows] u32 xfer cost of a cut after component i (row0+i)
+};
+
+struct SearchArgs {
+  const uint32_t* image;        // device copy of the table image
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  const uint64_t* node_free;    // [n_nodes] 8 x u8 free counts clamped to 8
+  const uint64_t* prefix;       // [K][n_req+1] exclusive task prefix of segment k
+  uint32_t n_req;
+  uint32_t rank, world;
+  int64_t* keys;
+  unsigned long long* checks;   // [n_req][3] or null
+  unsigned long long* misses;   // debug counter (verify mode)
+};
+
+struct DecodeArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  const int64_t* keys;
+  uint32_t n_req, k_max, n_nodes, n_slices;
+  const int32_t* free_list;     // [n_nodes][8][8] slice index of the j-th free slice
+  const uint16_t* slice_node;   // [n_slices]
+  const uint8_t* slice_prof;    // [n_slices]
+  const ffs_instance* inst;     // nullable
+  const int64_t* score;
+  uint32_t n_inst;
+  ffs_plan* out;
+};
+
+// launchers (ffs_kernels.cu)
+cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
+                               uint32_t n_nodes, uint32_t n_req, uint32_t k_max, uint64_t* prefix,
+                               uint64_t* block_sums, int64_t* keys, unsigned long long* checks,
+                               cudaStream_t st);
+cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, size_t smem, cudaStream_t st);
+cudaError_t search_kernel_config(int ks, bool verify, size_t smem, int* blocks_per_sm);
+cudaError_t launch_decode(const DecodeArgs& a, cudaStream_t st);
+cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32_t* tick_off,
+                         const uint64_t* now_us, uint32_t n_ticks, uint64_t now_single,
+                         ffs_evict_params prm, int64_t* score, uint8_t* state, cudaStream_t st);
+cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const ffs_request* req,
+                           const uint32_t* slo, const uint32_t* req_tick, uint32_t n_req,
+                           const ffs_instance* inst, const uint32_t* tick_off, const int64_t* score,
+                           uint32_t n_ticks, const uint16_t* slice_node, const uint8_t* slice_prof,
+                           uint32_t n_slices, int32_t* victim, cudaStream_t st);
+cudaError_t run_int_peak(int sms, double* ops, double* seconds);
+
+}  // namespace ffsk

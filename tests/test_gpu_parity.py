@@ -1,0 +1,251 @@
+"""GPU <-> oracle parity through the C ABI (libffs.so).  Needs a B200: marked gpu.
+
+Bar: bit-exact keys, plans and per-request checksums (candidates scored,
+feasible count, sum of feasible keys mod 2^64) against the CPU oracle on the same seeded
+inputs; zero filter misses; sharding invariance.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from helpers import problem
+from test_oracle_pins import random_tiny
+from paper_conf_hpdc_hui0s25_b200 import workload as W
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+
+
+@pytest.fixture(scope="module")
+def F():
+    from paper_conf_hpdc_hui0s25_b200 import ffs
+    assert torch.cuda.is_available(), "gpu tests need a CUDA device"
+    return ffs
+
+
+@pytest.fixture(scope="module")
+def planner(F):
+    return F.Planner(0)
+
+
+def run_gpu(F, planner, prob, k_max=None, verify=True, world=1):
+    """keys (+ checksums) over `world` shards combined with a host MIN/SUM (fake
+    collective), then decode.  Returns (plans numpy, keys, checks)."""
+    k_max = prob.k_max if k_max is None else k_max
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    R = prob.R
+    keys = torch.full((R,), F.KEY_NONE, dtype=torch.int64, device="cuda")
+    checks = torch.zeros((R, 3), dtype=torch.int64, device="cuda") if verify else None
+    for rank in range(world):
+        k = torch.empty(R, dtype=torch.int64, device="cuda")
+        c = torch.empty((R, 3), dtype=torch.int64, device="cuda") if verify else None
+        planner.plan_keys(req, slo, k_max, rank, world, keys=k, checks=c)
+        keys = torch.minimum(keys, k)
+        if verify:
+            checks += c  # int64 wrap-around == uint64 sum mod 2^64
+    plans = planner.plan_decode(req, slo, keys, k_max)
+    torch.cuda.synchronize()
+    ch = checks.cpu().numpy().view(np.uint64) if verify else None
+    return F.plans_to_numpy(plans), keys.cpu().numpy(), ch
+
+
+def assert_plans_equal(p, o, idx=None):
+    idx = np.arange(len(o["key"])) if idx is None else idx
+    g = p[idx]
+    np.testing.assert_array_equal(g["key"], o["key"])
+    np.testing.assert_array_equal(g["status"], o["status"])
+    ok = o["status"] == oracle.PLAN_OK
+    for a, b in (("k", "k"), ("cut_mask", "cut_mask"), ("e2e_us", "e2e_us"), ("bottleneck_us", "bottleneck_us"),
+                 ("gpcs", "gpcs"), ("cvq", "cvq")):
+        np.testing.assert_array_equal(g[a][ok], o[b][ok], err_msg=a)
+    np.testing.assert_array_equal(g["prof"], o["prof"])
+    np.testing.assert_array_equal(g["slice"], o["slice"])
+
+
+def test_exports_and_context(F, planner):
+    assert planner.device == 0
+
+
+def test_golden_hand_cases_gpu(F, planner):
+    import json, os
+    with open(os.path.join(os.path.dirname(__file__), "golden", "hand_cases.json")) as fh:
+        cases = json.load(fh)
+    for case in cases:
+        nodes = [[[s if isinstance(s, int) else tuple(s) for s in gpu] for gpu in node] for node in case["nodes"]]
+        prob = problem(case["funcs"], nodes, [tuple(r) for r in case["requests"]], k_max=case["k_max"])
+        p, keys, ch = run_gpu(F, planner, prob)
+        o = oracle.plan(prob)
+        assert_plans_equal(p, o)
+        np.testing.assert_array_equal(ch, o["checks"])
+
+
+@pytest.mark.parametrize("seed", range(1000, 1040))
+def test_tiny_random_bit_exact(F, planner, seed):
+    prob = random_tiny(seed)
+    p, keys, ch = run_gpu(F, planner, prob)
+    o = oracle.plan(prob)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    # production (non-verify) path gives the same keys
+    p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
+    np.testing.assert_array_equal(keys2, o["key"])
+
+
+@pytest.mark.parametrize("K", [1, 2, 3, 4, 5, 6, 7, 8])
+def test_every_stage_count(F, planner, K):
+    # chains of 1..10 components so that every KS template runs, with ragged tails
+    rng = W.SplitMix64(777 + K)
+    lengths = [1, 2, 3, 5, 8, 10]
+    prob = W._problem("ks", rng, lengths, W.NODE_BLOCK, 96, k_max=K)
+    p, keys, ch = run_gpu(F, planner, prob, k_max=K)
+    o = oracle.plan(prob, k_max=K)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    assert planner.filter_misses() == 0
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C1b", "C2"])
+def test_small_configs_full(F, planner, cfg):
+    prob = {"C1": W.config1, "C1b": W.config1b, "C2": W.config2}[cfg]()
+    p, keys, ch = run_gpu(F, planner, prob)
+    o = oracle.plan(prob)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
+    np.testing.assert_array_equal(keys2, o["key"])
+    assert planner.filter_misses() == 0
+
+
+def test_c3_sample_and_checksums(F, planner):
+    prob = W.config3()
+    p, keys, ch = run_gpu(F, planner, prob)
+    idx = np.concatenate([np.arange(0, prob.R, 97), np.arange(prob.R - 50, prob.R)])
+    o = oracle.plan(prob.subset(idx))
+    assert_plans_equal(p, o, idx)
+    np.testing.assert_array_equal(ch[idx], o["checks"])
+    # every request scored exactly S(n, K) candidates
+    n = prob.chain_len()[prob.req["func"]]
+    from math import comb
+    S = {m: sum(comb(m - 1, k - 1) * 5 ** k for k in range(1, min(m, 4) + 1)) for m in set(n.tolist())}
+    np.testing.assert_array_equal(ch[:, 0], np.array([S[m] for m in n], dtype=np.uint64))
+    _, keys2, _ = run_gpu(F, planner, prob, verify=False)
+    np.testing.assert_array_equal(keys2, keys)
+    assert planner.filter_misses() == 0
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_sharding_invariance(F, planner, world):
+    prob = W.config2(R=2048)
+    p1, k1, c1 = run_gpu(F, planner, prob)
+    pw, kw, cw = run_gpu(F, planner, prob, world=world)
+    np.testing.assert_array_equal(k1, kw)
+    np.testing.assert_array_equal(c1, cw)
+    np.testing.assert_array_equal(p1.view(np.uint8), pw.view(np.uint8))
+
+
+def test_c5_bench_configuration_sampled(F, planner):
+    """C5 at full size in the launch configuration bench.py times (world 1, production
+    path), checked on a stratified sample against the oracle."""
+    prob = W.config5()
+    p, keys, _ = run_gpu(F, planner, prob, verify=False)
+    rng = W.SplitMix64(55)
+    idx = np.unique(np.concatenate([np.arange(0, prob.R, 4099), prob.R - 1 - np.arange(8),
+                                    rng.integers(0, prob.R - 1, 64)]))
+    o = oracle.plan(prob.subset(idx), checks=False)
+    assert_plans_equal(p, o, idx)
+    # properties at any size: statuses consistent with keys, slices valid
+    ok = p["status"] == 0
+    assert (p["key"][~ok] == np.iinfo(np.int64).max).all()
+    assert (p["e2e_us"][ok] <= prob.slo_us[ok]).all()
+
+
+def test_bad_requests_and_empty(F, planner):
+    prob = random_tiny(1001)
+    req = prob.req.copy()
+    req["func"][0] = 99
+    req["node"][1] = 7
+    bad = prob.with_requests(req, prob.slo_us)
+    p, keys, ch = run_gpu(F, planner, bad)
+    assert p["status"][0] == 2 and p["status"][1] == 2
+    assert (ch[:2] == 0).all()
+    o = oracle.plan(bad)
+    assert_plans_equal(p, o)
+    empty = prob.subset(np.arange(0))
+    planner.stage(empty)
+    req_t, slo_t = F.to_device(empty)
+    out = planner.plan_batch(req_t, slo_t, 4)
+    assert out.shape[0] == 0
+
+
+def test_validation_errors(F, planner):
+    prob = random_tiny(1002)
+    bad = prob.with_requests(prob.req, prob.slo_us)
+    bad.lat_us = prob.lat_us.copy()
+    bad.lat_us[0, 0] = 0
+    with pytest.raises(F.FFSError) as e:
+        planner.stage(bad)
+    assert e.value.status == F.FFS_ERR_ARG
+    bad2 = prob.with_requests(prob.req, prob.slo_us)
+    bad2.slices = prob.slices[::-1].copy()
+    with pytest.raises(F.FFSError) as e:
+        planner.stage(bad2)
+    assert e.value.status == F.FFS_ERR_ARG
+    bad3 = prob.with_requests(prob.req, prob.slo_us)
+    bad3.lat_us = prob.lat_us.copy()
+    bad3.lat_us[:, :] = 1 << 23
+    with pytest.raises(F.FFSError) as e:
+        planner.stage(bad3)
+    assert e.value.status == F.FFS_ERR_RANGE
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    with pytest.raises(F.FFSError) as e:
+        planner.plan_keys(req, slo, 9)
+    assert e.value.status == F.FFS_ERR_RANGE
+
+
+def test_host_entry_point_matches(F, planner):
+    prob = W.config2(R=1024)
+    p, _, _ = run_gpu(F, planner, prob, verify=False)
+    h = planner.plan_batch_host(np.ascontiguousarray(prob.req), np.ascontiguousarray(prob.slo_us), prob.k_max)
+    np.testing.assert_array_equal(h.view(np.uint8), p.view(np.uint8))
+
+
+def test_eviction_scores_and_victims(F, planner):
+    wl = W.config4(T=64)
+    prob = wl.problem
+    planner.stage(prob)
+    inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
+    toff = torch.from_numpy(wl.tick_off.view(np.int32)).cuda()
+    now = torch.from_numpy(wl.now_us.view(np.int64)).cuda()
+    score, state = planner.evict_scores_ticks(inst, toff, now, window_us=wl.window_us)
+    req, slo = F.to_device(prob)
+    rt = torch.from_numpy(wl.req_tick.view(np.int32)).cuda()
+    vic = planner.evict_victims(req, slo, rt, inst, toff, score)
+    torch.cuda.synchronize()
+    score, state, vic = score.cpu().numpy(), state.cpu().numpy(), vic.cpu().numpy()
+    for t in range(len(wl.now_us)):
+        a, b = int(wl.tick_off[t]), int(wl.tick_off[t + 1])
+        s_o, st_o = oracle.evict(wl.inst[a:b], int(wl.now_us[t]), 30, wl.window_us)
+        np.testing.assert_array_equal(score[a:b], s_o)
+        np.testing.assert_array_equal(state[a:b], st_o)
+        rs = np.where(wl.req_tick == t)[0]
+        sub = prob.subset(rs)
+        v_o = oracle.victim(sub, np.full(len(rs), oracle.PLAN_INFEASIBLE, np.int32), wl.inst[a:b], s_o)
+        np.testing.assert_array_equal(vic[rs], v_o)
+    assert (vic >= 0).sum() > 0
+
+
+def test_decode_victims_single_snapshot(F, planner):
+    wl = W.config4(T=1)
+    prob = wl.problem
+    p, keys, _ = run_gpu(F, planner, prob, verify=False)
+    inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
+    score, _ = planner.evict_scores(inst, int(wl.now_us[0]), window_us=wl.window_us)
+    req, slo = F.to_device(prob)
+    plans = F.plans_to_numpy(planner.plan_decode(req, slo, torch.from_numpy(keys).cuda(), prob.k_max, inst, score))
+    o = oracle.plan(prob, checks=False)
+    s_o, _ = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
+    v_o = oracle.victim(prob, o["status"], wl.inst, s_o)
+    np.testing.assert_array_equal(plans["victim"], v_o)
