@@ -1,0 +1,318 @@
+"""Benchmark of the batched pipeline-construction search (BASELINE.json metric:
+candidates scored/s and plans/s at 1/2/4/8 B200, % of the integer roofline).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ffs|reference] [--config 5]
+
+One step = the whole hot path over one batch: ffs_plan_keys on this rank's shard (K0
+scan + K1 search segments) -> all_reduce(keys, MIN) over NCCL (N > 1) -> ffs_plan_decode
+of this rank's slice of the requests.  Inputs are resident in HBM when the timed region
+starts; L2 is flushed (256 MiB write) between timed steps, outside the events.  Each
+step is timed with CUDA events on the launching stream; ranks report the max.
+`--impl reference` times the CPU oracle (oracle/, the plain brute force) on a bounded
+sample of the same workload on this box's host cores (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+from math import comb
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_hpdc_hui0s25_b200 import workload as W  # noqa: E402
+
+ALG_OPS = 5  # hoisted per-candidate ops of A3-A5: add, fma, 2 compares, argmin flag
+P = 5
+
+
+def candidates_per_request(prob, k_max):
+    n = prob.chain_len()
+    S = np.array([sum(comb(int(m) - 1, k - 1) * P ** k for k in range(1, min(int(m), k_max) + 1)) for m in n],
+                 dtype=np.int64)
+    return S[prob.req["func"]]
+
+
+def segment_candidates(prob, k_max, rank, world):
+    """Candidates of segment ks processed by shard `rank` (same split as the kernel)."""
+    n = prob.chain_len()[prob.req["func"]]
+    out = []
+    for ks in range(1, k_max + 1):
+        tab = np.array([comb(m - 1, ks - 1) if m >= ks else 0 for m in range(33)], dtype=np.int64)
+        T = int(tab[n].sum())
+        sb, se = T * rank // world, T * (rank + 1) // world
+        out.append((se - sb) * P ** ks)
+    return out
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            return json.load(fh)
+    except OSError:
+        return {}
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={index}", f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                       "-lms", "100"], stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait()
+        self.f.flush()
+        rows = [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.count(",") >= 8]
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[1]) for r in rows]
+        mx = max(float(r[2]) for r in rows)
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].strip() == "Active"})
+        loaded = [s for s in sm if s > 0.5 * mx] or sm
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": reasons, "samples": len(rows)}
+
+
+def cpu_baseline(prob, k_max, budget_s=12.0):
+    """The oracle as it stands, on a bounded sample (every s-th request), all host cores."""
+    import oracle
+    cores = os.cpu_count() or 1
+    S = candidates_per_request(prob, k_max)
+    # calibrate on a small strided sample, then size the sample for ~budget_s
+    idx = np.arange(0, prob.R, max(1, prob.R // 64))
+    t = time.perf_counter()
+    oracle.plan(prob.subset(idx), k_max=k_max, threads=cores, checks=False)
+    rate = S[idx].sum() / (time.perf_counter() - t)
+    want = rate * budget_s
+    stride = max(1, int(S.sum() / max(want, 1.0)))
+    idx = np.arange(0, prob.R, stride)
+    t = time.perf_counter()
+    oracle.plan(prob.subset(idx), k_max=k_max, threads=cores, checks=False)
+    dt = time.perf_counter() - t
+    return {"value": float(S[idx].sum() / dt), "unit": "candidates/s", "cores": cores, "kind": "oracle",
+            "sample": f"every {stride}th request of {prob.name} ({len(idx)} requests, {int(S[idx].sum())} "
+                      f"candidates) in {dt:.1f} s", "plans_per_s": len(idx) / dt}
+
+
+def run_reference(args, prob):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    cores = os.cpu_count() or 1
+    S = candidates_per_request(prob, prob.k_max)
+    # per step: a bounded sample sized so the whole run stays within a few minutes
+    n_steps = args.steps + args.warmup
+    idx0 = np.arange(0, prob.R, max(1, prob.R // 64))
+    t = time.perf_counter()
+    oracle.plan(prob.subset(idx0), threads=cores, checks=False)
+    rate = S[idx0].sum() / (time.perf_counter() - t)
+    per_step = min(20.0, 150.0 / max(n_steps, 1))
+    stride = max(1, int(S.sum() / (rate * per_step)))
+    times, cands, plans = [], 0, 0
+    for s in range(n_steps):
+        idx = np.arange(s % stride, prob.R, stride)
+        t = time.perf_counter()
+        oracle.plan(prob.subset(idx), threads=cores, checks=False)
+        dt = time.perf_counter() - t
+        if s >= args.warmup:
+            times.append(dt)
+            cands += int(S[idx].sum())
+            plans += len(idx)
+    tot = sum(times)
+    v = cands / tot
+    line = {"metric": "candidates_scored_per_s", "value": v, "unit": "candidates/s", "impl": "reference",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/u64",
+            "data": "synthetic", "plans_per_s": plans / tot,
+            "config": {"workload": prob.meta["workload"], "R": prob.R, "k_max": prob.k_max},
+            "cpu_baseline": {"value": v, "unit": "candidates/s", "cores": cores, "kind": "oracle",
+                             "sample": f"every {stride}th request (offset by step) of {prob.name}"},
+            "e2e": {"value": v, "unit": "candidates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ffs", choices=["ffs", "reference"])
+    ap.add_argument("--config", type=int, default=5, choices=[2, 3, 5])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    assert args.warmup >= 3 or args.impl == "reference", "timing rules: >= 3 warm-up steps"
+
+    prob = W.CONFIGS[args.config]()
+    desc = {2: "C2: 6 functions n in {3,3,5,6,8,12}, 1 Hybrid node (26 slices), R=4096, K=4",
+            3: "C3: 20 functions n in U[3,24], 8 nodes = 64 GPUs, R=65536, K=4",
+            5: "C5: 64 functions n in U[3,32], 128 nodes = 1024 GPUs, R=1048576, K=4"}
+    prob.meta["workload"] = desc[args.config]
+    if args.impl == "reference":
+        run_reference(args, prob)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_hpdc_hui0s25_b200 import ffs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    K = prob.k_max
+    R = prob.R
+    pl = ffs.Planner(local)
+    pl.stage(prob)
+    req, slo = ffs.to_device(prob)
+    keys = torch.empty(R, dtype=torch.int64, device="cuda")
+    lo, hi = R * rank // world, R * (rank + 1) // world
+    plans = torch.empty((hi - lo, 80), dtype=torch.uint8, device="cuda")
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def step():
+        pl.plan_keys(req, slo, K, rank, world, keys=keys)
+        if world > 1:
+            dist.all_reduce(keys, op=dist.ReduceOp.MIN)
+        pl.plan_decode(req[lo:hi], slo[lo:hi], keys[lo:hi], K, out=plans)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    clocks = Clocks(local)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    seg_ms = np.zeros(8)
+    barrier()
+    for i in range(args.steps):
+        flush.fill_(i & 0xFF)  # L2 flush, outside the timed events
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+        seg_ms += np.array(pl.segment_times())  # waits for this step's search segments
+    barrier()
+    clk = clocks.stop()
+    ms = sum(a.elapsed_time(b) for a, b in ev)
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    total_cands = int(candidates_per_request(prob, K).sum())
+    value = total_cands * args.steps / (ms * 1e-3)
+    plans_per_s = R * args.steps / (ms * 1e-3)
+
+    # dominant kernel: the KS = K search segment on this rank
+    seg_c = segment_candidates(prob, K, rank, world)
+    top = int(np.argmax(seg_ms)) + 1
+    top_ms = seg_ms[top - 1] / args.steps
+    peaks = measured_peaks()
+    sm_count = torch.cuda.get_device_properties(local).multi_processor_count
+    max_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+    peak_ops = sm_count * 4 * 32 * max_mhz * 1e6  # issue-limited lane-ops/s
+    achieved = seg_c[top - 1] * ALG_OPS / (top_ms * 1e-3)
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tpath):
+        traffic = json.load(open(tpath)).get(f"k_plan_search<{top}>")
+
+    # e2e through the public host-buffer API (N = 1: ffs_plan_batch_host)
+    e2e = None
+    if not args.no_e2e:
+        h_req = torch.from_numpy(np.ascontiguousarray(prob.req).view(np.uint8)).pin_memory()
+        h_slo = torch.from_numpy(np.ascontiguousarray(prob.slo_us).view(np.uint8)).pin_memory()
+        h_out = torch.empty((hi - lo) * 80, dtype=torch.uint8).pin_memory()
+        req_np = h_req.numpy().view(W.REQ_DTYPE)
+        slo_np = h_slo.numpy().view(np.uint32)
+        out_np = h_out.numpy().view(ffs.PLAN_DTYPE)
+        d_req = torch.empty_like(req)
+        d_slo = torch.empty_like(slo)
+
+        def e2e_step():
+            if world == 1:
+                pl.plan_batch_host(req_np, slo_np, K, out=out_np)
+            else:
+                d_req.copy_(h_req.view(-1, 8).cuda(non_blocking=True).view_as(d_req))
+                d_slo.copy_(h_slo.view(torch.int32).cuda(non_blocking=True))
+                pl.plan_keys(d_req, d_slo, K, rank, world, keys=keys)
+                dist.all_reduce(keys, op=dist.ReduceOp.MIN)
+                pl.plan_decode(d_req[lo:hi], d_slo[lo:hi], keys[lo:hi], K, out=plans)
+                h_out.copy_(plans.view(-1), non_blocking=True)
+                torch.cuda.synchronize()
+
+        for _ in range(2):
+            e2e_step()
+        barrier()
+        t0 = time.perf_counter()
+        n_e2e = max(3, args.steps // 2)
+        for _ in range(n_e2e):
+            e2e_step()
+        barrier()
+        dt = time.perf_counter() - t0
+        if world > 1:
+            t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+        e2e = {"value": total_cands * n_e2e / dt, "unit": "candidates/s", "plans_per_s": R * n_e2e / dt,
+               "h2d_bytes_per_step": int(R * 12), "d2h_bytes_per_step": int((hi - lo) * 80),
+               "timer": "host wall clock around the blocking call, max over ranks"}
+
+    if rank == 0:
+        cpu = None
+        if world == 1 and not args.no_cpu_baseline:
+            cpu = cpu_baseline(prob, K)
+        launches_per_step = 1 + 3 + min(K, int(prob.chain_len().max())) + 1
+        line = {
+            "metric": "candidates_scored_per_s", "value": value, "unit": "candidates/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/u64",
+            "data": "synthetic", "plans_per_s": plans_per_s,
+            "config": {"workload": prob.meta["workload"], "R": R, "k_max": K, "candidates_per_step": total_cands,
+                       "l2": "flushed between steps (256 MiB write, outside the events)",
+                       "parallelism": f"candidate-range shards x{world} + all_reduce(MIN) over NCCL" if world > 1
+                       else "single GPU"},
+            "roofline": {"bound": "alu", "kernel": f"k_plan_search<{top}>", "achieved": achieved, "peak": peak_ops,
+                         "unit": "int lane-ops/s", "frac": achieved / peak_ops, "traffic": traffic,
+                         "alg_ops_per_candidate": ALG_OPS, "kernel_ms": top_ms,
+                         "kernel_share_of_step": top_ms / (ms / args.steps),
+                         "peak_source": f"{sm_count} SMs x 4 SMSP x 32 lanes x {max_mhz:.0f} MHz "
+                                        f"(MEASURED_PEAKS.json sm_max_mhz)"},
+            "clocks": clk,
+            "gpu_launches": launches_per_step * args.steps,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -236,6 +236,10 @@ ffs_status ffs_evict_victims(ffs_ctx *ctx, const ffs_request *d_req, const uint3
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
  * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */
 ffs_status ffs_bench_int_peak(ffs_ctx *ctx, double *ops_per_s, double *seconds);
+/* Device time (ms, CUDA events recorded on the launch stream) of each search-kernel
+ * segment of the last ffs_plan_keys call on this context: ms[ks-1] for ks = 1..8 stages,
+ * 0 where no segment ran.  Waits for those events.  */
+ffs_status ffs_segment_times(ffs_ctx *ctx, float *ms /* [8] */);
 /* Number of candidates, since the context was created, that the fast float filter
  * rejected although their exact key would have beaten the running minimum (verify mode
  * only; must be 0).  Synchronous. */

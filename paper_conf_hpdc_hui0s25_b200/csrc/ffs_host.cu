@@ -64,6 +64,9 @@ struct ffs_ctx {
   // cached occupancy per (ks, verify, smem)
   size_t occ_smem = 0;
   int occ[2][kMaxK + 1] = {};
+  // per-segment timing of the last plan_keys call
+  cudaEvent_t ev[kMaxK + 1] = {};
+  int seg_first = 0, seg_last = -1;
 };
 
 static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
@@ -113,6 +116,7 @@ ffs_status ffs_create(int cuda_device, ffs_ctx** out) {
       delete c;
       return FFS_ERR_CUDA;
     }
+    for (auto& e : c->ev) cudaEventCreate(&e);
   }
   *out = c;
   return FFS_OK;
@@ -122,6 +126,8 @@ void ffs_destroy(ffs_ctx* c) {
   if (!c) return;
   {
     DeviceGuard g(c->device);
+    for (auto& e : c->ev)
+      if (e) cudaEventDestroy(e);
     for (DevBuf* b : {&c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses})
       b->release();
@@ -345,9 +351,14 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
   a.checks = reinterpret_cast<unsigned long long*>(d_checks);
   a.misses = c->misses.as<unsigned long long>();
   const bool verify = d_checks != nullptr;
-  for (uint32_t k = 1; k <= std::min(k_max, c->max_n); ++k) {
+  const uint32_t kk = std::min(k_max, c->max_n);
+  c->seg_first = 1;
+  c->seg_last = (int)kk;
+  CK(cudaEventRecord(c->ev[0], st), "event");
+  for (uint32_t k = 1; k <= kk; ++k) {
     const int grid = c->sms * c->occ[verify ? 1 : 0][k];
     CK(launch_search((int)k, verify, a, grid, smem, st), "search kernel");
+    CK(cudaEventRecord(c->ev[k], st), "event");
   }
   return FFS_OK;
 }
@@ -464,6 +475,17 @@ ffs_status ffs_bench_int_peak(ffs_ctx* c, double* ops, double* seconds) {
   if (!c || !ops || !seconds) return FFS_ERR_ARG;
   DeviceGuard g(c->device);
   CK(run_int_peak(c->sms, ops, seconds), "int peak kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_segment_times(ffs_ctx* c, float* ms) {
+  if (!c || !ms) return FFS_ERR_ARG;
+  for (int k = 0; k < kMaxK; ++k) ms[k] = 0.f;
+  DeviceGuard g(c->device);
+  for (int k = c->seg_first; k <= c->seg_last; ++k) {
+    CK(cudaEventSynchronize(c->ev[k]), "event sync");
+    CK(cudaEventElapsedTime(&ms[k - 1], c->ev[k - 1], c->ev[k]), "event time");
+  }
   return FFS_OK;
 }
 

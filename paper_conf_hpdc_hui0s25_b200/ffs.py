@@ -61,6 +61,7 @@ _sig = {
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
+    "ffs_segment_times": ([_vp, C.POINTER(C.c_float)], _i32),
     "ffs_debug_filter_misses": ([_vp, C.POINTER(C.c_uint64)], _i32),
 }
 for _name, (_args, _res) in _sig.items():
@@ -219,6 +220,12 @@ class Planner:
         ops, sec = C.c_double(), C.c_double()
         self._check(_lib.ffs_bench_int_peak(self._h, C.byref(ops), C.byref(sec)))
         return ops.value, sec.value
+
+    def segment_times(self) -> list[float]:
+        """Device ms of each search segment (ks = 1..8) of the last plan_keys call."""
+        ms = (C.c_float * 8)()
+        self._check(_lib.ffs_segment_times(self._h, ms))
+        return [float(x) for x in ms]
 
     def filter_misses(self) -> int:
         v = C.c_uint64()
