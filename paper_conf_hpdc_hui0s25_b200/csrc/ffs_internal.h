@@ -15,7 +15,13 @@ constexpr int kMaxN = 32;      // max components per chain (cut masks fit in uin
 constexpr int kMaxK = 8;       // max stages
 constexpr int kIdxBits = 41;   // canonical index field of the key
 constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
-constexpr int kBlock = 256;    // threads per CTA of the search kernel
+#ifndef FFS_BLOCK
+#define FFS_BLOCK 256
+#endif
+#ifndef FFS_MINB4
+#define FFS_MINB4 1
+#endif
+constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
 // image into shared memory once per CTA (A0 of DESIGN.md §4); every other kernel reads

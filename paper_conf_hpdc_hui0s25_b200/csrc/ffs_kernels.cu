@@ -159,6 +159,7 @@ struct SearchState {
   uint32_t memst[KS];
   uint32_t X;         // transfer cost of the cuts
   float blim_raw, blim;
+  int32_t blim_i_raw, blim_i;  // e2e bound of the unrolled path: sum t <= blim_i
   // register tables of the last two stages: q = stage KS-2, p = stage KS-1
   float tq[kP], sqq[kP], aq[kP], tp[kP], sqp[kP], ap[kP];
   int pd[KS];         // digits of the outer levels
@@ -178,10 +179,11 @@ __device__ __forceinline__ void set_threshold(SearchState<KS>& c) {
     c.none_can_win = cthr < 0;
     // can-win: cvq <= cthr  <=>  1024*KS*sum t^2 < (1025 + cthr) * (sum t)^2
     // filter: (sum t)^2 > alpha * sum t^2 with alpha rounded down by a 2^-16 margin
-    const double a = 1024.0 * KS / (1025.0 + cthr) * (1.0 - 1.0 / 65536.0);
-    c.alpha = __double2float_rd(a);
+    // 1024*KS*(1 - 2^-16) = KS*65535/64 is exact in fp32; the quotient is rounded down
+    c.alpha = __fdiv_rd((float)(KS * 65535) * (1.f / 64.f), (float)(1025 + cthr));
   }
   c.blim = c.none_can_win ? -1.f : c.blim_raw;
+  c.blim_i = c.none_can_win ? -1 : c.blim_i_raw;
 #pragma unroll
   for (int p = 0; p < kP; ++p) {
     c.aq[p] = c.alpha * c.sqq[p];
@@ -319,6 +321,165 @@ __device__ __forceinline__ void load_stage(const SearchState<KS>& c, int s, floa
   }
 }
 
+// ---- fully unrolled path for KS = 2..4 ----------------------------
+// Every level is a compile-time loop, so the multiplicity m of a profile within the
+// sequence is a constant and the free-slice check is folded into per-request variant
+// tables vi[s][m][x] = t (stage s on profile x fits memory and the node has > m free
+// slices of x) else kInfI.  Per candidate (p = last stage, prefix sums S, L, B of the
+// group): d2 = B - vi (sign = SLO or memory/count miss), z = fma(S, 2t, (1-a)t^2) + U
+// with U = S^2 - L (sign = cannot beat the running minimum), acc &= z | d2.
+constexpr int32_t kInfI = 1 << 26;  // > any stage sum (< 2^24); 4 of them cannot overflow
+
+template <int KS>
+struct Tables {
+  int32_t vi[KS][KS][kP];   // [stage][multiplicity-1][profile]
+  float tf[KS][kP];         // stage latency (stages 0..KS-2)
+  float a[KS][kP];          // alpha * t^2   (stages 0..KS-2)
+  float t2[kP], cc[kP];     // last stage: 2t and (1 - alpha) t^2
+};
+
+template <int KS>
+__device__ __forceinline__ void build_tables(const SearchState<KS>& c, Tables<KS>& T) {
+  const float one_m_a = 1.f - c.alpha;
+#pragma unroll
+  for (int s = 0; s < KS; ++s) {
+    const uint32_t ra = c.o_pl + (c.row0 + c.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + c.bnd[s + 1]) * kRowW;
+    const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
+    const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
+    const int32_t t[kP] = {(int32_t)(lb.x - la.x), (int32_t)(lb.y - la.y), (int32_t)(lb.z - la.z),
+                           (int32_t)(lb.w - la.w), (int32_t)(c.sm[rb + 4] - c.sm[ra + 4])};
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const bool mem_ok = c.memst[s] <= c.sm[c.o_cap + x];
+      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+#pragma unroll
+      for (int m = 0; m <= s; ++m) T.vi[s][m][x] = (mem_ok && fr > (uint32_t)m) ? t[x] : kInfI;
+      const float f = __int2float_rn(t[x]);
+      if (s < KS - 1) {
+        T.tf[s][x] = f;
+        T.a[s][x] = c.alpha * (f * f);
+      } else {
+        T.t2[x] = f + f;
+        T.cc[x] = one_m_a * (f * f);
+      }
+    }
+  }
+}
+
+__device__ __forceinline__ void cand(float S, float U, int32_t B, int32_t vi, float t2, float cc, uint32_t& acc) {
+  const int32_t d2 = B - vi;               // < 0: SLO, memory or free-slice miss
+  const float z = fmaf(S, t2, cc) + U;     // < 0: cannot beat the running minimum
+  acc &= __float_as_uint(z) | (uint32_t)d2;
+}
+
+// the last two levels (q, p) of one block; prefix digits d0, d1 (KS = 4) / d0 (KS = 3)
+template <int KS, int D0, int D1>
+__device__ __forceinline__ uint32_t block_qp(const Tables<KS>& T, float S, float L, int32_t B) {
+  uint32_t acc = ~0u;
+#pragma unroll
+  for (int q = 0; q < kP; ++q) {
+    const int mq = (KS >= 3 && q == D0) + (KS >= 4 && q == D1);
+    const float S3 = S + T.tf[KS - 2][q];
+    const float L3 = L + T.a[KS - 2][q];
+    const int32_t B3 = B - T.vi[KS - 2][mq][q];
+    const float U = fmaf(S3, S3, -L3);
+#pragma unroll
+    for (int p = 0; p < kP; ++p) {
+      const int mp = (KS >= 3 && p == D0) + (KS >= 4 && p == D1) + (p == q);
+      cand(S3, U, B3, T.vi[KS - 1][mp][p], T.t2[p], T.cc[p], acc);
+    }
+  }
+  return (acc >> 31) ^ 1u;  // 1 if some candidate of the block may win
+}
+
+// KS = 4: stage 0 is a runtime loop over d0 (keeps the unrolled body at P^3 candidates,
+// ~11 KB of SASS, inside the instruction cache); stages 1..3 are unrolled.  The
+// multiplicity of profile x in stages 1..3 is shifted by [x == d0] through
+// per-d0 tables sh[s][m][x] = vi[s][m + (x == d0)][x].
+struct Shift4 {
+  int32_t v1[1][kP], v2[2][kP], v3[3][kP];
+};
+
+__device__ __forceinline__ uint32_t block3(const Tables<4>& T, const Shift4& H, float S1, float L1, int32_t B1) {
+  uint32_t pend = 0;
+#pragma unroll
+  for (int d1 = 0; d1 < kP; ++d1) {
+    const float S2 = S1 + T.tf[1][d1];
+    const float L2 = L1 + T.a[1][d1];
+    const int32_t B2 = B1 - H.v1[0][d1];
+    uint32_t acc = ~0u;
+#pragma unroll
+    for (int q = 0; q < kP; ++q) {
+      const int mq = (q == d1);
+      const float S3 = S2 + T.tf[2][q];
+      const float L3 = L2 + T.a[2][q];
+      const int32_t B3 = B2 - H.v2[mq][q];
+      const float U = fmaf(S3, S3, -L3);
+#pragma unroll
+      for (int p = 0; p < kP; ++p) {
+        const int mp = (p == d1) + (p == q);
+        cand(S3, U, B3, H.v3[mp][p], T.t2[p], T.cc[p], acc);
+      }
+    }
+    pend |= ((acc >> 31) ^ 1u) << d1;
+  }
+  return pend;
+}
+
+template <int KS, bool VERIFY>
+__device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, unsigned long long* misses) {
+  Tables<KS> T;
+  build_tables<KS>(c, T);
+  const int32_t Bl = c.blim_i;
+  uint32_t pend = 0;  // one bit per block of P*P candidates
+  if constexpr (KS == 2) {
+    pend = block_qp<KS, -1, -1>(T, 0.f, 0.f, Bl);
+  } else if constexpr (KS == 3) {
+#define FFS_D0(D0) pend |= block_qp<KS, D0, -1>(T, T.tf[0][D0], T.a[0][D0], Bl - T.vi[0][0][D0]) << D0;
+    FFS_D0(0) FFS_D0(1) FFS_D0(2) FFS_D0(3) FFS_D0(4)
+#undef FFS_D0
+  } else {
+#pragma unroll 1
+    for (int d0 = 0; d0 < kP; ++d0) {
+      Shift4 H;
+#pragma unroll
+      for (int x = 0; x < kP; ++x) {
+        const bool e = (x == d0);
+        H.v1[0][x] = e ? T.vi[1][1][x] : T.vi[1][0][x];
+        H.v2[0][x] = e ? T.vi[2][1][x] : T.vi[2][0][x];
+        H.v2[1][x] = e ? T.vi[2][2][x] : T.vi[2][1][x];
+        H.v3[0][x] = e ? T.vi[3][1][x] : T.vi[3][0][x];
+        H.v3[1][x] = e ? T.vi[3][2][x] : T.vi[3][1][x];
+        H.v3[2][x] = e ? T.vi[3][3][x] : T.vi[3][2][x];
+      }
+      // stage-0 values of digit d0 (runtime index: select from the unrolled tables)
+      float S1 = 0.f, L1 = 0.f;
+      int32_t v0 = 0;
+#pragma unroll
+      for (int x = 0; x < kP; ++x)
+        if (x == d0) {
+          S1 = T.tf[0][x];
+          L1 = T.a[0][x];
+          v0 = T.vi[0][0][x];
+        }
+      pend |= block3(T, H, S1, L1, Bl - v0) << (kP * d0);
+    }
+  }
+  constexpr int NB = KS == 2 ? 1 : (KS == 3 ? kP : kP * kP);
+  const uint32_t all = VERIFY ? ((1u << NB) - 1) : pend;
+  for (uint32_t todo = all; todo;) {
+    const int b = __ffs(todo) - 1;
+    todo &= todo - 1;
+    if constexpr (KS == 3) c.pd[0] = b;
+    if constexpr (KS == 4) {
+      c.pd[0] = b / kP;
+      c.pd[1] = b - kP * (b / kP);
+    }
+    const uint32_t fast = ((pend >> b) & 1u) ? ((1u << (kP * kP)) - 1) : 0u;
+    handle_hits<KS, VERIFY>(c, (1u << (kP * kP)) - 1, fast, misses);
+  }
+}
+
 template <int KS, bool VERIFY>
 __device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, unsigned long long* misses) {
   // stage boundaries: a cut after component j iff bit j is set
@@ -337,7 +498,11 @@ __device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, 
   for (int i = 0; i < KS; ++i) c.memst[i] = c.sm[c.o_pm + c.row0 + c.bnd[i + 1]] - c.sm[c.o_pm + c.row0 + c.bnd[i]];
   // e2e <= B  <=>  sum t <= B - X; exact in float because sum t < 2^24 (R4 bound)
   c.blim_raw = (X <= c.B) ? __uint2float_rd(c.B - X) : -1.f;
-  if constexpr (KS == 1) {
+  c.blim_i_raw = (X <= c.B) ? (int32_t)min(c.B - X, 1u << 24) : -1;
+  if constexpr (KS >= 2 && KS <= 4) {
+    c.blim_i = c.none_can_win ? -1 : c.blim_i_raw;
+    unrolled_mask<KS, VERIFY>(c, misses);
+  } else if constexpr (KS == 1) {
     c.blim = c.blim_raw;
     // 5 candidates per request: evaluate them exactly
     c.pd[0] = 0;
@@ -367,7 +532,7 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
 }
 
 template <int KS, bool VERIFY>
-__global__ void __launch_bounds__(kBlock) k_plan_search(const __grid_constant__ SearchArgs A) {
+__global__ void __launch_bounds__(kBlock, KS == 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
   {  // A0: stage the table image into shared memory (16-byte copies)
     const uint4* src = reinterpret_cast<const uint4*>(A.image);
@@ -415,6 +580,7 @@ __global__ void __launch_bounds__(kBlock) k_plan_search(const __grid_constant__ 
     c.idx_base = img_u64(smem, A.lay.o_offk + 2 * (c.n * 10 + KS)) + rank0 * PK;
     c.best = *reinterpret_cast<volatile const int64_t*>(A.keys + r);  // earlier segments' minimum
     best0 = c.best;
+    if constexpr (KS >= 2) set_threshold(c);
     c.nfeas = 0;
     c.ksum = 0;
     done = 0;

@@ -15,7 +15,7 @@ import numpy as np
 from . import workload as W
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libffs.so")
+LIB_PATH = os.environ.get("FFS_LIB") or os.path.join(_PKG, "libffs.so")  # FFS_LIB: experiment builds
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is not built; run `python -c 'import __graft_entry__ as g; g.build()'`")
 _lib = C.CDLL(LIB_PATH)
