@@ -249,8 +249,8 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
     }
     row += n + 1;
   }
-  if ((size_t)L.words * 4 > 200 * 1024)
-    return fail(c, FFS_ERR_RANGE, "table image %u bytes exceeds the 200 KB shared-memory stage", L.words * 4);
+  if ((size_t)L.words * 4 > kMaxSmem)
+    return fail(c, FFS_ERR_RANGE, "table image %u bytes exceeds the shared-memory stage", L.words * 4);
 
   // ---- per node: free counts (clamped to 8) and the first 8 free slices per profile ----
   const uint32_t NN = cl->n_nodes;
@@ -328,11 +328,14 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
                         c->block_sums.as<uint64_t>(), d_keys, reinterpret_cast<unsigned long long*>(d_checks), st),
      "count/scan kernels");
   const size_t smem = (size_t)c->lay.words * 4;
+  const size_t rows4 = (size_t)20 * kBlock * 16;  // KS = 4 per-thread variant rows
+  if (k_max >= 4 && smem + rows4 > kMaxSmem)
+    return fail(c, FFS_ERR_RANGE, "table image %zu B + %zu B of rows exceeds shared memory", smem, rows4);
   if (c->occ_smem != smem) {
     for (int v = 0; v < 2; ++v)
       for (int k = 1; k <= kMaxK; ++k) {
         int b = 0;
-        CK(search_kernel_config(k, v != 0, smem, &b), "search kernel occupancy");
+        CK(search_kernel_config(k, v != 0, smem + (k == 4 ? rows4 : 0), &b), "search kernel occupancy");
         c->occ[v][k] = std::max(1, b);
       }
     c->occ_smem = smem;
@@ -357,7 +360,7 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
   CK(cudaEventRecord(c->ev[0], st), "event");
   for (uint32_t k = 1; k <= kk; ++k) {
     const int grid = c->sms * c->occ[verify ? 1 : 0][k];
-    CK(launch_search((int)k, verify, a, grid, smem, st), "search kernel");
+    CK(launch_search((int)k, verify, a, grid, smem + (k == 4 ? rows4 : 0), st), "search kernel");
     CK(cudaEventRecord(c->ev[k], st), "event");
   }
   return FFS_OK;

@@ -16,12 +16,13 @@ constexpr int kMaxK = 8;       // max stages
 constexpr int kIdxBits = 41;   // canonical index field of the key
 constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #ifndef FFS_BLOCK
-#define FFS_BLOCK 256
+#define FFS_BLOCK 512
 #endif
 #ifndef FFS_MINB4
 #define FFS_MINB4 1
 #endif
 constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
+constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
 // image into shared memory once per CTA (A0 of DESIGN.md §4); every other kernel reads

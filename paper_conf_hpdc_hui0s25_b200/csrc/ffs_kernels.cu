@@ -159,7 +159,6 @@ struct SearchState {
   uint32_t memst[KS];
   uint32_t X;         // transfer cost of the cuts
   float blim_raw, blim;
-  int32_t blim_i_raw, blim_i;  // e2e bound of the unrolled path: sum t <= blim_i
   // register tables of the last two stages: q = stage KS-2, p = stage KS-1
   float tq[kP], sqq[kP], aq[kP], tp[kP], sqp[kP], ap[kP];
   int pd[KS];         // digits of the outer levels
@@ -183,7 +182,6 @@ __device__ __forceinline__ void set_threshold(SearchState<KS>& c) {
     c.alpha = __fdiv_rd((float)(KS * 65535) * (1.f / 64.f), (float)(1025 + cthr));
   }
   c.blim = c.none_can_win ? -1.f : c.blim_raw;
-  c.blim_i = c.none_can_win ? -1 : c.blim_i_raw;
 #pragma unroll
   for (int p = 0; p < kP; ++p) {
     c.aq[p] = c.alpha * c.sqq[p];
@@ -321,148 +319,184 @@ __device__ __forceinline__ void load_stage(const SearchState<KS>& c, int s, floa
   }
 }
 
-// ---- fully unrolled path for KS = 2..4 ----------------------------
-// Every level is a compile-time loop, so the multiplicity m of a profile within the
-// sequence is a constant and the free-slice check is folded into per-request variant
-// tables vi[s][m][x] = t (stage s on profile x fits memory and the node has > m free
-// slices of x) else kInfI.  Per candidate (p = last stage, prefix sums S, L, B of the
-// group): d2 = B - vi (sign = SLO or memory/count miss), z = fma(S, 2t, (1-a)t^2) + U
-// with U = S^2 - L (sign = cannot beat the running minimum), acc &= z | d2.
-constexpr int32_t kInfI = 1 << 26;  // > any stage sum (< 2^24); 4 of them cannot overflow
-
+// ---- unrolled path for KS = 2..4 -----------------------------------
+// The last three (KS = 4) / all (KS <= 3) levels are compile-time loops, so the
+// multiplicity m of a profile within the sequence is a constant and the free-slice
+// check is folded into variant tables vf[s][m][x] = t (stage s on profile x fits in
+// memory and the node has more than m free slices of x) else +INF.  Per candidate
+// (p = last stage; S, L, B = the group's sum of stage times, alpha * sum t^2 and
+// Blim - S):
+//   d2 = B - vf[p]                 sign set <=> SLO, memory or free-slice miss (exact:
+//                                  every operand is an integer < 2^25 or INF)
+//   z  = fma(S, 2t_p, (1-alpha) t_p^2) + (S^2 - L)
+//                                  sign set <=> (S+t_p)^2 <= alpha (sum t^2): cannot beat
+//                                  the running minimum (conservative, §4.3)
+//   acc &= bits(z) | bits(d2)      sign of acc clear <=> some candidate may win
+// FFMA + FADD + FADD on the full-rate FMA pipe, one LOP3 on the half-rate ALU pipe.
 template <int KS>
 struct Tables {
-  int32_t vi[KS][KS][kP];   // [stage][multiplicity-1][profile]
-  float tf[KS][kP];         // stage latency (stages 0..KS-2)
-  float a[KS][kP];          // alpha * t^2   (stages 0..KS-2)
-  float t2[kP], cc[kP];     // last stage: 2t and (1 - alpha) t^2
+  float vf[KS][KS][kP];  // [stage][multiplicity-1][profile], +INF folded
+  float a[KS][kP];       // alpha * t^2   (stages 0..KS-2)
+  float t2[kP], cc[kP];  // last stage: 2t and (1 - alpha) t^2
 };
 
 template <int KS>
+__device__ __forceinline__ void stage_lat(const SearchState<KS>& c, int s, float (&f)[kP]) {
+  const uint32_t ra = c.o_pl + (c.row0 + c.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + c.bnd[s + 1]) * kRowW;
+  const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
+  const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
+  f[0] = __uint2float_rn(lb.x - la.x);
+  f[1] = __uint2float_rn(lb.y - la.y);
+  f[2] = __uint2float_rn(lb.z - la.z);
+  f[3] = __uint2float_rn(lb.w - la.w);
+  f[4] = __uint2float_rn(c.sm[rb + 4] - c.sm[ra + 4]);
+}
+
+template <int KS>
 __device__ __forceinline__ void build_tables(const SearchState<KS>& c, Tables<KS>& T) {
+  const float INF = __int_as_float(0x7f800000);
   const float one_m_a = 1.f - c.alpha;
 #pragma unroll
   for (int s = 0; s < KS; ++s) {
-    const uint32_t ra = c.o_pl + (c.row0 + c.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + c.bnd[s + 1]) * kRowW;
-    const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
-    const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
-    const int32_t t[kP] = {(int32_t)(lb.x - la.x), (int32_t)(lb.y - la.y), (int32_t)(lb.z - la.z),
-                           (int32_t)(lb.w - la.w), (int32_t)(c.sm[rb + 4] - c.sm[ra + 4])};
+    float f[kP];
+    stage_lat(c, s, f);
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
       const bool mem_ok = c.memst[s] <= c.sm[c.o_cap + x];
       const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
 #pragma unroll
-      for (int m = 0; m <= s; ++m) T.vi[s][m][x] = (mem_ok && fr > (uint32_t)m) ? t[x] : kInfI;
-      const float f = __int2float_rn(t[x]);
+      for (int m = 0; m <= s; ++m) T.vf[s][m][x] = (mem_ok && fr > (uint32_t)m) ? f[x] : INF;
       if (s < KS - 1) {
-        T.tf[s][x] = f;
-        T.a[s][x] = c.alpha * (f * f);
+        T.a[s][x] = c.alpha * (f[x] * f[x]);
       } else {
-        T.t2[x] = f + f;
-        T.cc[x] = one_m_a * (f * f);
+        T.t2[x] = f[x] + f[x];
+        T.cc[x] = one_m_a * (f[x] * f[x]);
       }
     }
   }
 }
 
-__device__ __forceinline__ void cand(float S, float U, int32_t B, int32_t vi, float t2, float cc, uint32_t& acc) {
-  const int32_t d2 = B - vi;               // < 0: SLO, memory or free-slice miss
-  const float z = fmaf(S, t2, cc) + U;     // < 0: cannot beat the running minimum
-  acc &= __float_as_uint(z) | (uint32_t)d2;
+__device__ __forceinline__ void cand(float S, float U, float B, float v, float t2, float cc, uint32_t& acc) {
+  const float d2 = B - v;
+  const float z = fmaf(S, t2, cc) + U;
+  acc &= __float_as_uint(z) | __float_as_uint(d2);
 }
 
-// the last two levels (q, p) of one block; prefix digits d0, d1 (KS = 4) / d0 (KS = 3)
-template <int KS, int D0, int D1>
-__device__ __forceinline__ uint32_t block_qp(const Tables<KS>& T, float S, float L, int32_t B) {
+// one block = the last two levels (q, p): P*P candidates.  vq/vp select the variant
+// tables of the q and p stages by compile-time multiplicity.
+template <class VQ, class VP>
+__device__ __forceinline__ uint32_t block_qp(const float (&aq)[kP], const float (&t2)[kP], const float (&cc)[kP],
+                                             float S, float L, float B, VQ vq, VP vp) {
   uint32_t acc = ~0u;
 #pragma unroll
   for (int q = 0; q < kP; ++q) {
-    const int mq = (KS >= 3 && q == D0) + (KS >= 4 && q == D1);
-    const float S3 = S + T.tf[KS - 2][q];
-    const float L3 = L + T.a[KS - 2][q];
-    const int32_t B3 = B - T.vi[KS - 2][mq][q];
+    const float v = vq(q);
+    const float S3 = S + v;
+    const float B3 = B - v;
+    const float L3 = L + aq[q];
     const float U = fmaf(S3, S3, -L3);
 #pragma unroll
-    for (int p = 0; p < kP; ++p) {
-      const int mp = (KS >= 3 && p == D0) + (KS >= 4 && p == D1) + (p == q);
-      cand(S3, U, B3, T.vi[KS - 1][mp][p], T.t2[p], T.cc[p], acc);
-    }
+    for (int p = 0; p < kP; ++p) cand(S3, U, B3, vp(q, p), t2[p], cc[p], acc);
   }
   return (acc >> 31) ^ 1u;  // 1 if some candidate of the block may win
 }
 
-// KS = 4: stage 0 is a runtime loop over d0 (keeps the unrolled body at P^3 candidates,
-// ~11 KB of SASS, inside the instruction cache); stages 1..3 are unrolled.  The
-// multiplicity of profile x in stages 1..3 is shifted by [x == d0] through
-// per-d0 tables sh[s][m][x] = vi[s][m + (x == d0)][x].
-struct Shift4 {
-  int32_t v1[1][kP], v2[2][kP], v3[3][kP];
+// KS = 4: per-thread shared-memory rows of the stage 1..3 variant tables, two windows
+// per profile x: e = 0 (x is not the stage-0 profile d0) and e = 1 (x == d0, every
+// multiplicity of x shifted by one).  Window e of row x = 8 words:
+//   [vf1[e][x], vf2[e][x], vf2[e+1][x], vf3[e][x], vf3[e+1][x], vf3[e+2][x], w6, w7]
+// with (w6, w7) = (vf0[0][x], a0[x]) in window 1 (the stage-0 values of d0 = x).
+// Layout [x][quad 0..3][thread][4 words]: conflict-free 16-byte accesses.
+struct Win {
+  float s1, s2[2], s3[3];
 };
 
-__device__ __forceinline__ uint32_t block3(const Tables<4>& T, const Shift4& H, float S1, float L1, int32_t B1) {
+template <bool VERIFY>
+__device__ __forceinline__ uint32_t ks4_mask(SearchState<4>& c, float* rows) {
+  const float INF = __int_as_float(0x7f800000);
+  const float one_m_a = 1.f - c.alpha;
+  const int tid = threadIdx.x;
+  float f[4][kP];
+#pragma unroll
+  for (int s = 0; s < 4; ++s) stage_lat(c, s, f[s]);
+  float a1[kP], a2[kP], t2[kP], cc[kP];
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const uint32_t cap = c.sm[c.o_cap + x];
+    float v[4][5];
+#pragma unroll
+    for (int s = 0; s < 4; ++s)
+#pragma unroll
+      for (int m = 0; m <= s + 1 && m < 5; ++m) v[s][m] = (c.memst[s] <= cap && fr > (uint32_t)m) ? f[s][x] : INF;
+    a1[x] = c.alpha * (f[1][x] * f[1][x]);
+    a2[x] = c.alpha * (f[2][x] * f[2][x]);
+    t2[x] = f[3][x] + f[3][x];
+    cc[x] = one_m_a * (f[3][x] * f[3][x]);
+    const float a0 = c.alpha * (f[0][x] * f[0][x]);
+    float4* r = reinterpret_cast<float4*>(rows) + (x * 4) * kBlock + tid;
+    r[0 * kBlock] = make_float4(v[1][0], v[2][0], v[2][1], v[3][0]);
+    r[1 * kBlock] = make_float4(v[3][1], v[3][2], 0.f, 0.f);
+    r[2 * kBlock] = make_float4(v[1][1], v[2][1], v[2][2], v[3][1]);
+    r[3 * kBlock] = make_float4(v[3][2], v[3][3], v[0][0], a0);
+  }
+  const float Bl = c.blim;
   uint32_t pend = 0;
+#pragma unroll 1
+  for (int d0 = 0; d0 < kP; ++d0) {
+    Win W[kP];
+    float S1 = 0.f, L1 = 0.f;
 #pragma unroll
-  for (int d1 = 0; d1 < kP; ++d1) {
-    const float S2 = S1 + T.tf[1][d1];
-    const float L2 = L1 + T.a[1][d1];
-    const int32_t B2 = B1 - H.v1[0][d1];
-    uint32_t acc = ~0u;
-#pragma unroll
-    for (int q = 0; q < kP; ++q) {
-      const int mq = (q == d1);
-      const float S3 = S2 + T.tf[2][q];
-      const float L3 = L2 + T.a[2][q];
-      const int32_t B3 = B2 - H.v2[mq][q];
-      const float U = fmaf(S3, S3, -L3);
-#pragma unroll
-      for (int p = 0; p < kP; ++p) {
-        const int mp = (p == d1) + (p == q);
-        cand(S3, U, B3, H.v3[mp][p], T.t2[p], T.cc[p], acc);
+    for (int x = 0; x < kP; ++x) {
+      const int e = (x == d0) ? 2 : 0;
+      const float4* r = reinterpret_cast<const float4*>(rows) + (x * 4 + e) * kBlock + tid;
+      const float4 q0 = r[0], q1 = r[kBlock];
+      W[x].s1 = q0.x;
+      W[x].s2[0] = q0.y;
+      W[x].s2[1] = q0.z;
+      W[x].s3[0] = q0.w;
+      W[x].s3[1] = q1.x;
+      W[x].s3[2] = q1.y;
+      if (x == d0) {
+        S1 = q1.z;
+        L1 = q1.w;
       }
     }
-    pend |= ((acc >> 31) ^ 1u) << d1;
+    const float B1 = Bl - S1;
+#pragma unroll
+    for (int d1 = 0; d1 < kP; ++d1) {
+      const float v1 = W[d1].s1;
+      const uint32_t hit = block_qp(
+          a2, t2, cc, S1 + v1, L1 + a1[d1], B1 - v1,
+          [&](int q) { return W[q].s2[q == d1]; },
+          [&](int q, int p) { return W[p].s3[(p == d1) + (p == q)]; });
+      pend |= hit << (kP * d0 + d1);
+    }
   }
   return pend;
 }
 
 template <int KS, bool VERIFY>
-__device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, unsigned long long* misses) {
-  Tables<KS> T;
-  build_tables<KS>(c, T);
-  const int32_t Bl = c.blim_i;
+__device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses) {
   uint32_t pend = 0;  // one bit per block of P*P candidates
-  if constexpr (KS == 2) {
-    pend = block_qp<KS, -1, -1>(T, 0.f, 0.f, Bl);
-  } else if constexpr (KS == 3) {
-#define FFS_D0(D0) pend |= block_qp<KS, D0, -1>(T, T.tf[0][D0], T.a[0][D0], Bl - T.vi[0][0][D0]) << D0;
-    FFS_D0(0) FFS_D0(1) FFS_D0(2) FFS_D0(3) FFS_D0(4)
-#undef FFS_D0
+  if constexpr (KS == 4) {
+    pend = ks4_mask<VERIFY>(c, rows);
   } else {
-#pragma unroll 1
-    for (int d0 = 0; d0 < kP; ++d0) {
-      Shift4 H;
+    Tables<KS> T;
+    build_tables<KS>(c, T);
+    const float Bl = c.blim;
+    if constexpr (KS == 2) {
+      pend = block_qp(T.a[0], T.t2, T.cc, 0.f, 0.f, Bl, [&](int q) { return T.vf[0][0][q]; },
+                      [&](int q, int p) { return T.vf[1][p == q][p]; });
+    } else {
 #pragma unroll
-      for (int x = 0; x < kP; ++x) {
-        const bool e = (x == d0);
-        H.v1[0][x] = e ? T.vi[1][1][x] : T.vi[1][0][x];
-        H.v2[0][x] = e ? T.vi[2][1][x] : T.vi[2][0][x];
-        H.v2[1][x] = e ? T.vi[2][2][x] : T.vi[2][1][x];
-        H.v3[0][x] = e ? T.vi[3][1][x] : T.vi[3][0][x];
-        H.v3[1][x] = e ? T.vi[3][2][x] : T.vi[3][1][x];
-        H.v3[2][x] = e ? T.vi[3][3][x] : T.vi[3][2][x];
+      for (int d0 = 0; d0 < kP; ++d0) {
+        const float v0 = T.vf[0][0][d0];
+        pend |= block_qp(T.a[1], T.t2, T.cc, v0, T.a[0][d0], Bl - v0,
+                         [&](int q) { return T.vf[1][q == d0][q]; },
+                         [&](int q, int p) { return T.vf[2][(p == d0) + (p == q)][p]; })
+                << d0;
       }
-      // stage-0 values of digit d0 (runtime index: select from the unrolled tables)
-      float S1 = 0.f, L1 = 0.f;
-      int32_t v0 = 0;
-#pragma unroll
-      for (int x = 0; x < kP; ++x)
-        if (x == d0) {
-          S1 = T.tf[0][x];
-          L1 = T.a[0][x];
-          v0 = T.vi[0][0][x];
-        }
-      pend |= block3(T, H, S1, L1, Bl - v0) << (kP * d0);
     }
   }
   constexpr int NB = KS == 2 ? 1 : (KS == 3 ? kP : kP * kP);
@@ -481,7 +515,8 @@ __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, unsigned long 
 }
 
 template <int KS, bool VERIFY>
-__device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, unsigned long long* misses) {
+__device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, float* rows,
+                                             unsigned long long* misses) {
   // stage boundaries: a cut after component j iff bit j is set
   c.bnd[0] = 0;
   uint32_t m = mask, X = 0;
@@ -498,10 +533,11 @@ __device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, 
   for (int i = 0; i < KS; ++i) c.memst[i] = c.sm[c.o_pm + c.row0 + c.bnd[i + 1]] - c.sm[c.o_pm + c.row0 + c.bnd[i]];
   // e2e <= B  <=>  sum t <= B - X; exact in float because sum t < 2^24 (R4 bound)
   c.blim_raw = (X <= c.B) ? __uint2float_rd(c.B - X) : -1.f;
-  c.blim_i_raw = (X <= c.B) ? (int32_t)min(c.B - X, 1u << 24) : -1;
   if constexpr (KS >= 2 && KS <= 4) {
-    c.blim_i = c.none_can_win ? -1 : c.blim_i_raw;
-    unrolled_mask<KS, VERIFY>(c, misses);
+    // exact in fp32: min(B - X, 2^24) is an integer <= 2^24 and every stage sum is < 2^24
+    c.blim_raw = (X <= c.B) ? (float)min(c.B - X, 1u << 24) : -1.f;
+    c.blim = c.none_can_win ? -1.f : c.blim_raw;
+    unrolled_mask<KS, VERIFY>(c, rows, misses);
   } else if constexpr (KS == 1) {
     c.blim = c.blim_raw;
     // 5 candidates per request: evaluate them exactly
@@ -532,7 +568,7 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
 }
 
 template <int KS, bool VERIFY>
-__global__ void __launch_bounds__(kBlock, KS == 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
+__global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
   {  // A0: stage the table image into shared memory (16-byte copies)
     const uint4* src = reinterpret_cast<const uint4*>(A.image);
@@ -540,6 +576,8 @@ __global__ void __launch_bounds__(kBlock, KS == 4 ? FFS_MINB4 : 1) k_plan_search
     for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += kBlock) dst[i] = src[i];
   }
   __syncthreads();
+  // KS = 4: per-thread rows of the shifted variant tables after the image (ks4_mask)
+  float* rows = reinterpret_cast<float*>(smem + A.lay.words);
 
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint64_t T = pre[A.n_req];
@@ -608,7 +646,7 @@ __global__ void __launch_bounds__(kBlock, KS == 4 ? FFS_MINB4 : 1) k_plan_search
 
   load_request(m);
   while (true) {
-    process_mask<KS, VERIFY>(c, mask, A.misses);
+    process_mask<KS, VERIFY>(c, mask, rows, A.misses);
     ++done;
     if (++task == t1) break;
     if (++m == cnt) {
@@ -627,7 +665,7 @@ __global__ void __launch_bounds__(kBlock, KS == 4 ? FFS_MINB4 : 1) k_plan_search
 
 template <int KS, bool V>
 static cudaError_t set_attr() {
-  return cudaFuncSetAttribute(k_plan_search<KS, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  return cudaFuncSetAttribute(k_plan_search<KS, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
 }
 
 #define FFS_KS_SWITCH(ks, verify, CALL)                  \
