@@ -328,7 +328,7 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
                         c->block_sums.as<uint64_t>(), d_keys, reinterpret_cast<unsigned long long*>(d_checks), st),
      "count/scan kernels");
   const size_t smem = (size_t)c->lay.words * 4;
-  const size_t rows4 = (size_t)20 * kBlock * 16;  // KS = 4 per-thread variant rows
+  const size_t rows4 = (size_t)40 * kBlock * 16;  // KS = 4 per-thread variant windows (ks4_pair)
   if (k_max >= 4 && smem + rows4 > kMaxSmem)
     return fail(c, FFS_ERR_RANGE, "table image %zu B + %zu B of rows exceeds shared memory", smem, rows4);
   if (c->occ_smem != smem) {

@@ -16,7 +16,7 @@ constexpr int kMaxK = 8;       // max stages
 constexpr int kIdxBits = 41;   // canonical index field of the key
 constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #ifndef FFS_BLOCK
-#define FFS_BLOCK 512
+#define FFS_BLOCK 256
 #endif
 #ifndef FFS_MINB4
 #define FFS_MINB4 1

@@ -401,86 +401,204 @@ __device__ __forceinline__ uint32_t block_qp(const float (&aq)[kP], const float 
   return (acc >> 31) ^ 1u;  // 1 if some candidate of the block may win
 }
 
-// KS = 4: per-thread shared-memory rows of the stage 1..3 variant tables, two windows
-// per profile x: e = 0 (x is not the stage-0 profile d0) and e = 1 (x == d0, every
-// multiplicity of x shifted by one).  Window e of row x = 8 words:
-//   [vf1[e][x], vf2[e][x], vf2[e+1][x], vf3[e][x], vf3[e+1][x], vf3[e+2][x], w6, w7]
-// with (w6, w7) = (vf0[0][x], a0[x]) in window 1 (the stage-0 values of d0 = x).
-// Layout [x][quad 0..3][thread][4 words]: conflict-free 16-byte accesses.
-struct Win {
-  float s1, s2[2], s3[3];
+// ---- KS = 4, two cut masks per thread in the two fp32 lanes of FFMA2/FADD2 -----------
+// Mask A (lane lo) and the next mask B of the same request (lane hi) share every
+// control decision (loops, multiplicities) and differ only in data, so one packed
+// instruction scores a candidate of each: per candidate pair FFMA2 + FADD2 + FADD2 on
+// the FMA pipe and two LOP3 on the ALU pipe.
+typedef unsigned long long f2;
+__device__ __forceinline__ f2 f2pack(float lo, float hi) {
+  f2 r;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(lo), "f"(hi));
+  return r;
+}
+__device__ __forceinline__ void f2bits(f2 v, uint32_t& lo, uint32_t& hi) {
+  asm("mov.b64 {%0, %1}, %2;" : "=r"(lo), "=r"(hi) : "l"(v));
+}
+__device__ __forceinline__ f2 f2add(f2 a, f2 b) {
+  f2 d;
+  asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ f2 f2sub(f2 a, f2 b) {
+  f2 d;
+  asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+  return d;
+}
+__device__ __forceinline__ f2 f2fma(f2 a, f2 b, f2 c) {
+  f2 d;
+  asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
+  return d;
+}
+
+struct Geo4 {
+  int bnd[5];
+  uint32_t memst[4];
+  uint32_t X;
+  float blim;
 };
 
-template <bool VERIFY>
-__device__ __forceinline__ uint32_t ks4_mask(SearchState<4>& c, float* rows) {
-  const float INF = __int_as_float(0x7f800000);
-  const float one_m_a = 1.f - c.alpha;
-  const int tid = threadIdx.x;
-  float f[4][kP];
+__device__ __forceinline__ void geo4(const SearchState<4>& c, uint32_t mask, Geo4& g) {
+  g.bnd[0] = 0;
+  uint32_t m = mask, X = 0;
 #pragma unroll
-  for (int s = 0; s < 4; ++s) stage_lat(c, s, f[s]);
-  float a1[kP], a2[kP], t2[kP], cc[kP];
-#pragma unroll
-  for (int x = 0; x < kP; ++x) {
-    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-    const uint32_t cap = c.sm[c.o_cap + x];
-    float v[4][5];
-#pragma unroll
-    for (int s = 0; s < 4; ++s)
-#pragma unroll
-      for (int m = 0; m <= s + 1 && m < 5; ++m) v[s][m] = (c.memst[s] <= cap && fr > (uint32_t)m) ? f[s][x] : INF;
-    a1[x] = c.alpha * (f[1][x] * f[1][x]);
-    a2[x] = c.alpha * (f[2][x] * f[2][x]);
-    t2[x] = f[3][x] + f[3][x];
-    cc[x] = one_m_a * (f[3][x] * f[3][x]);
-    const float a0 = c.alpha * (f[0][x] * f[0][x]);
-    float4* r = reinterpret_cast<float4*>(rows) + (x * 4) * kBlock + tid;
-    r[0 * kBlock] = make_float4(v[1][0], v[2][0], v[2][1], v[3][0]);
-    r[1 * kBlock] = make_float4(v[3][1], v[3][2], 0.f, 0.f);
-    r[2 * kBlock] = make_float4(v[1][1], v[2][1], v[2][2], v[3][1]);
-    r[3 * kBlock] = make_float4(v[3][2], v[3][3], v[0][0], a0);
+  for (int i = 0; i < 3; ++i) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    g.bnd[i + 1] = j + 1;
+    X += c.sm[c.o_xf + c.row0 + j];
   }
-  const float Bl = c.blim;
-  uint32_t pend = 0;
-#pragma unroll 1
-  for (int d0 = 0; d0 < kP; ++d0) {
-    Win W[kP];
-    float S1 = 0.f, L1 = 0.f;
+  g.bnd[4] = c.n;
+  g.X = X;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) g.memst[i] = c.sm[c.o_pm + c.row0 + g.bnd[i + 1]] - c.sm[c.o_pm + c.row0 + g.bnd[i]];
+  g.blim = (X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
+}
+
+__device__ __forceinline__ void geo_lat(const SearchState<4>& c, const Geo4& g, int s, float (&f)[kP]) {
+  const uint32_t ra = c.o_pl + (c.row0 + g.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + g.bnd[s + 1]) * kRowW;
+  const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
+  const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
+  f[0] = __uint2float_rn(lb.x - la.x);
+  f[1] = __uint2float_rn(lb.y - la.y);
+  f[2] = __uint2float_rn(lb.z - la.z);
+  f[3] = __uint2float_rn(lb.w - la.w);
+  f[4] = __uint2float_rn(c.sm[rb + 4] - c.sm[ra + 4]);
+}
+
+struct Win2 {
+  f2 s1, s2[2], s3[3];
+};
+
+// rows: per thread, [x][e][quad 0..3][thread] of 16-byte quads = 2 packed pairs each;
+// window e of profile x = pairs [v1[e], v2[e], v2[e+1], v3[e], v3[e+1], v3[e+2], v0, a0]
+// (v0, a0 = stage-0 value and alpha t0^2 of x, only meaningful in window 1).
+template <bool VERIFY>
+__device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, uint4* rows,
+                                         unsigned long long* misses) {
+  const float INF = __int_as_float(0x7f800000);
+  const int tid = threadIdx.x;
+  Geo4 G[2];
+  geo4(c, maskA, G[0]);
+  geo4(c, maskB, G[1]);
+  if (!haveB) G[1].blim = -1.f;  // dummy lane: nothing passes
+  const float al = c.alpha, one_m_a = 1.f - c.alpha;
+  f2 a1[kP], a2[kP], t2[kP], cc[kP];
+  {
+    float f[2][4][kP];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int s = 0; s < 4; ++s) geo_lat(c, G[h], s, f[h][s]);
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
-      const int e = (x == d0) ? 2 : 0;
-      const float4* r = reinterpret_cast<const float4*>(rows) + (x * 4 + e) * kBlock + tid;
-      const float4 q0 = r[0], q1 = r[kBlock];
-      W[x].s1 = q0.x;
-      W[x].s2[0] = q0.y;
-      W[x].s2[1] = q0.z;
-      W[x].s3[0] = q0.w;
-      W[x].s3[1] = q1.x;
-      W[x].s3[2] = q1.y;
-      if (x == d0) {
-        S1 = q1.z;
-        L1 = q1.w;
+      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+      const uint32_t cap = c.sm[c.o_cap + x];
+      float v[2][4][5];
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 4; ++s)
+#pragma unroll
+          for (int m = 0; m <= s + 1 && m < 5; ++m)
+            v[h][s][m] = (G[h].memst[s] <= cap && fr > (uint32_t)m) ? f[h][s][x] : INF;
+      a1[x] = f2pack(al * (f[0][1][x] * f[0][1][x]), al * (f[1][1][x] * f[1][1][x]));
+      a2[x] = f2pack(al * (f[0][2][x] * f[0][2][x]), al * (f[1][2][x] * f[1][2][x]));
+      t2[x] = f2pack(f[0][3][x] + f[0][3][x], f[1][3][x] + f[1][3][x]);
+      cc[x] = f2pack(one_m_a * (f[0][3][x] * f[0][3][x]), one_m_a * (f[1][3][x] * f[1][3][x]));
+      const float a0A = al * (f[0][0][x] * f[0][0][x]), a0B = al * (f[1][0][x] * f[1][0][x]);
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        uint4* r = rows + ((x * 2 + e) * 4) * kBlock + tid;
+        auto u = [](float f) { return __float_as_uint(f); };
+        r[0 * kBlock] = make_uint4(u(v[0][1][e]), u(v[1][1][e]), u(v[0][2][e]), u(v[1][2][e]));
+        r[1 * kBlock] = make_uint4(u(v[0][2][e + 1]), u(v[1][2][e + 1]), u(v[0][3][e]), u(v[1][3][e]));
+        r[2 * kBlock] = make_uint4(u(v[0][3][e + 1]), u(v[1][3][e + 1]), u(v[0][3][e + 2]), u(v[1][3][e + 2]));
+        r[3 * kBlock] = e ? make_uint4(u(v[0][0][0]), u(v[1][0][0]), u(a0A), u(a0B)) : make_uint4(0, 0, 0, 0);
       }
     }
-    const float B1 = Bl - S1;
+  }
+  const f2 Bl = f2pack(G[0].blim, G[1].blim);
+  uint32_t pendA = 0, pendB = 0;
+#pragma unroll 1
+  for (int d0 = 0; d0 < kP; ++d0) {
+    Win2 W[kP];
+    f2 S1 = 0, L1 = 0;
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const int e = (x == d0);
+      const uint4* r = rows + ((x * 2 + e) * 4) * kBlock + tid;
+      const uint4 q0 = r[0], q1 = r[kBlock], q2 = r[2 * kBlock];
+      W[x].s1 = ((f2)q0.y << 32) | q0.x;
+      W[x].s2[0] = ((f2)q0.w << 32) | q0.z;
+      W[x].s2[1] = ((f2)q1.y << 32) | q1.x;
+      W[x].s3[0] = ((f2)q1.w << 32) | q1.z;
+      W[x].s3[1] = ((f2)q2.y << 32) | q2.x;
+      W[x].s3[2] = ((f2)q2.w << 32) | q2.z;
+    }
+    {
+      const uint4 q3 = rows[((d0 * 2 + 1) * 4 + 3) * kBlock + tid];
+      S1 = ((f2)q3.y << 32) | q3.x;
+      L1 = ((f2)q3.w << 32) | q3.z;
+    }
+    const f2 B1 = f2sub(Bl, S1);
 #pragma unroll
     for (int d1 = 0; d1 < kP; ++d1) {
-      const float v1 = W[d1].s1;
-      const uint32_t hit = block_qp(
-          a2, t2, cc, S1 + v1, L1 + a1[d1], B1 - v1,
-          [&](int q) { return W[q].s2[q == d1]; },
-          [&](int q, int p) { return W[p].s3[(p == d1) + (p == q)]; });
-      pend |= hit << (kP * d0 + d1);
+      const f2 w1 = W[d1].s1;
+      const f2 S2 = f2add(S1, w1), L2 = f2add(L1, a1[d1]), B2 = f2sub(B1, w1);
+      uint32_t accA = ~0u, accB = ~0u;
+#pragma unroll
+      for (int q = 0; q < kP; ++q) {
+        const f2 w2 = W[q].s2[q == d1];
+        const f2 S3 = f2add(S2, w2), B3 = f2sub(B2, w2);
+        const f2 NL3 = f2sub(f2sub(0ull, L2), a2[q]);  // -(L2 + a2)
+        const f2 U = f2fma(S3, S3, NL3);
+#pragma unroll
+        for (int p = 0; p < kP; ++p) {
+          const f2 w3 = W[p].s3[(p == d1) + (p == q)];
+          const f2 z = f2add(f2fma(S3, t2[p], cc[p]), U);
+          const f2 d2 = f2sub(B3, w3);
+          uint32_t zl, zh, dl, dh;
+          f2bits(z, zl, zh);
+          f2bits(d2, dl, dh);
+          accA &= zl | dl;
+          accB &= zh | dh;
+        }
+      }
+      pendA |= ((accA >> 31) ^ 1u) << (kP * d0 + d1);
+      pendB |= ((accB >> 31) ^ 1u) << (kP * d0 + d1);
     }
   }
-  return pend;
+  // rare exact path, one half at a time (geometry copied into the state)
+  constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
+#pragma unroll 1
+  for (int h = 0; h < (haveB ? 2 : 1); ++h) {
+    const uint32_t pend = h ? pendB : pendA;
+    const uint32_t all = VERIFY ? kAll : pend;
+    if (!all) continue;
+#pragma unroll
+    for (int i = 0; i < 5; ++i) c.bnd[i] = G[h].bnd[i];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) c.memst[i] = G[h].memst[i];
+    c.X = G[h].X;
+    if (h) c.idx_base += 625;
+    for (uint32_t todo = all; todo;) {
+      const int b = __ffs(todo) - 1;
+      todo &= todo - 1;
+      c.pd[0] = b / kP;
+      c.pd[1] = b - kP * (b / kP);
+      const uint32_t fast = ((pend >> b) & 1u) ? kAll : 0u;
+      handle_hits<4, VERIFY>(c, kAll, fast, misses);
+    }
+    if (h) c.idx_base -= 625;
+  }
 }
 
 template <int KS, bool VERIFY>
 __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses) {
   uint32_t pend = 0;  // one bit per block of P*P candidates
   if constexpr (KS == 4) {
-    pend = ks4_mask<VERIFY>(c, rows);
+    __trap();  // KS = 4 uses ks4_pair
   } else {
     Tables<KS> T;
     build_tables<KS>(c, T);
@@ -646,10 +764,24 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
 
   load_request(m);
   while (true) {
-    process_mask<KS, VERIFY>(c, mask, rows, A.misses);
-    ++done;
-    if (++task == t1) break;
-    if (++m == cnt) {
+    uint32_t step = 1;
+    if constexpr (KS == 4) {
+      // two consecutive masks of the same request per iteration (ks4_pair)
+      const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
+      const uint32_t maskB = haveB ? gosper_next(mask) : mask;
+      ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<uint4*>(rows), A.misses);
+      if (haveB) {
+        step = 2;
+        mask = maskB;
+      }
+    } else {
+      process_mask<KS, VERIFY>(c, mask, rows, A.misses);
+    }
+    done += step;
+    task += step;
+    if (task >= t1) break;
+    m += step;
+    if (m == cnt) {
       flush();
       r = find_request(pre, A.n_req, task);
       m = 0;
@@ -657,7 +789,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
       load_request(0);
     } else {
       mask = gosper_next(mask);
-      c.idx_base += PK;
+      c.idx_base += step * PK;
     }
   }
   flush();

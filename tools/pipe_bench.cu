@@ -40,6 +40,27 @@ KERNEL(k_core4, {
   asm volatile("sub.s32 %0, %1, %0;" : "+r"(r[i]) : "r"(ia));
   asm volatile("lop3.b32 %0, %0, %1, %2, 0xA8;" : "+r"(r[i]) : "r"(ib), "r"(__float_as_int(f[i])));
 })
+// packed fp32x2 (sm_100): two lanes per instruction
+KERNEL(k_ffma2, {
+  uint64_t v = ((uint64_t)__float_as_uint(f[i]) << 32) | __float_as_uint(f[i] + 1.f);
+  uint64_t A = ((uint64_t)__float_as_uint(a) << 32) | __float_as_uint(a);
+  uint64_t Bv = ((uint64_t)__float_as_uint(b) << 32) | __float_as_uint(b);
+  asm volatile("fma.rn.f32x2 %0, %0, %1, %2;" : "+l"(v) : "l"(A), "l"(Bv));
+  f[i] = __uint_as_float((uint32_t)v) + __uint_as_float((uint32_t)(v >> 32));
+})
+KERNEL(k_fadd2_chain, {
+  uint64_t A = ((uint64_t)__float_as_uint(a) << 32) | __float_as_uint(b);
+  uint64_t v = ((uint64_t)r[i] << 32) | (uint32_t)r[i];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) asm volatile("add.rn.f32x2 %0, %0, %1;" : "+l"(v) : "l"(A));
+  r[i] = (int)(v ^ (v >> 32));
+})
+KERNEL(k_fadd_chain4, {
+  float x = __int_as_float(r[i]);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) asm volatile("add.f32 %0, %0, %1;" : "+f"(x) : "f"(a));
+  r[i] = __float_as_int(x);
+})
 // FFMA + IADD alternating
 KERNEL(k_ffma_iadd, {
   asm volatile("fma.rn.f32 %0, %0, %1, %2;" : "+f"(f[i]) : "f"(a), "f"(b));
@@ -88,12 +109,15 @@ void run(const char* name, K kern, int insts_per_body, int blocks_per_sm, int th
 int main() {
   for (int occ : {2, 4, 8}) {
     run("ffma", k_ffma, 1, occ, 256);
+    run("ffma2", k_ffma2, 1, occ, 256);
     run("fadd", k_fadd, 1, occ, 256);
     run("fmul", k_fmul, 1, occ, 256);
     run("iadd", k_iadd, 1, occ, 256);
     run("lop3", k_lop3, 1, occ, 256);
     run("imad", k_imad, 1, occ, 256);
     run("core4", k_core4, 4, occ, 256);
+    run("fadd2x4", k_fadd2_chain, 4, occ, 256);
+    run("faddx4", k_fadd_chain4, 4, occ, 256);
     run("ffma+iadd", k_ffma_iadd, 2, occ, 256);
     run("fadd+iadd", k_fadd_iadd, 2, occ, 256);
   }
