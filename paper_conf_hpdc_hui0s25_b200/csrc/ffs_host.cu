@@ -327,15 +327,20 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
   CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, c->prefix.as<uint64_t>(),
                         c->block_sums.as<uint64_t>(), d_keys, reinterpret_cast<unsigned long long*>(d_checks), st),
      "count/scan kernels");
+  // dynamic shared memory: the table image (every KS) + the per-thread variant windows
+  // of the KS = 4 kernel (440 B per thread); the KS = 4 CTA shrinks when both do not fit
   const size_t smem = (size_t)c->lay.words * 4;
-  const size_t rows4 = (size_t)40 * kBlock * 16;  // KS = 4 per-thread variant windows (ks4_pair)
-  if (k_max >= 4 && smem + rows4 > kMaxSmem)
-    return fail(c, FFS_ERR_RANGE, "table image %zu B + %zu B of rows exceeds shared memory", smem, rows4);
+  int block4 = kBlock;
+  while (block4 > 32 && smem + (size_t)440 * block4 > kMaxSmem) block4 -= 32;
+  if (k_max >= 4 && c->max_n >= 4 && smem + (size_t)440 * block4 > kMaxSmem)
+    return fail(c, FFS_ERR_RANGE, "table image %zu B leaves no room for the KS=4 windows", smem);
+  auto blk = [&](int k) { return k == 4 ? block4 : kBlock; };
+  auto shm = [&](int k) { return smem + (k == 4 ? (size_t)440 * block4 : 0); };
   if (c->occ_smem != smem) {
     for (int v = 0; v < 2; ++v)
       for (int k = 1; k <= kMaxK; ++k) {
         int b = 0;
-        CK(search_kernel_config(k, v != 0, smem + (k == 4 ? rows4 : 0), &b), "search kernel occupancy");
+        CK(search_kernel_config(k, v != 0, blk(k), shm(k), &b), "search kernel occupancy");
         c->occ[v][k] = std::max(1, b);
       }
     c->occ_smem = smem;
@@ -360,7 +365,7 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
   CK(cudaEventRecord(c->ev[0], st), "event");
   for (uint32_t k = 1; k <= kk; ++k) {
     const int grid = c->sms * c->occ[verify ? 1 : 0][k];
-    CK(launch_search((int)k, verify, a, grid, smem + (k == 4 ? rows4 : 0), st), "search kernel");
+    CK(launch_search((int)k, verify, a, grid, blk((int)k), shm((int)k), st), "search kernel");
     CK(cudaEventRecord(c->ev[k], st), "event");
   }
   return FFS_OK;

@@ -470,14 +470,13 @@ struct Win2 {
   f2 s1, s2[2], s3[3];
 };
 
-// rows: per thread, [x][e][quad 0..3][thread] of 16-byte quads = 2 packed pairs each;
-// window e of profile x = pairs [v1[e], v2[e], v2[e+1], v3[e], v3[e+1], v3[e+2], v0, a0]
-// (v0, a0 = stage-0 value and alpha t0^2 of x, only meaningful in window 1).
+// rows: per thread and profile x, 11 packed pairs in [x][k][thread] order (8-byte,
+// conflict-free); window e (e = 1 when x is the stage-0 profile) is read at offset e.
 template <bool VERIFY>
-__device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, uint4* rows,
+__device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, f2* rows,
                                          unsigned long long* misses) {
   const float INF = __int_as_float(0x7f800000);
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, nb = blockDim.x;  // window stride = threads of the CTA
   Geo4 G[2];
   geo4(c, maskA, G[0]);
   geo4(c, maskB, G[1]);
@@ -507,15 +506,20 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
       t2[x] = f2pack(f[0][3][x] + f[0][3][x], f[1][3][x] + f[1][3][x]);
       cc[x] = f2pack(one_m_a * (f[0][3][x] * f[0][3][x]), one_m_a * (f[1][3][x] * f[1][3][x]));
       const float a0A = al * (f[0][0][x] * f[0][0][x]), a0B = al * (f[1][0][x] * f[1][0][x]);
-#pragma unroll
-      for (int e = 0; e < 2; ++e) {
-        uint4* r = rows + ((x * 2 + e) * 4) * kBlock + tid;
-        auto u = [](float f) { return __float_as_uint(f); };
-        r[0 * kBlock] = make_uint4(u(v[0][1][e]), u(v[1][1][e]), u(v[0][2][e]), u(v[1][2][e]));
-        r[1 * kBlock] = make_uint4(u(v[0][2][e + 1]), u(v[1][2][e + 1]), u(v[0][3][e]), u(v[1][3][e]));
-        r[2 * kBlock] = make_uint4(u(v[0][3][e + 1]), u(v[1][3][e + 1]), u(v[0][3][e + 2]), u(v[1][3][e + 2]));
-        r[3 * kBlock] = e ? make_uint4(u(v[0][0][0]), u(v[1][0][0]), u(a0A), u(a0B)) : make_uint4(0, 0, 0, 0);
-      }
+      // compact per-thread row of profile x: 11 packed pairs
+      //   [v1[0], v1[1], v2[0], v2[1], v2[2], v3[0], v3[1], v3[2], v3[3], v0[0], a0]
+      f2* r = rows + (x * 11) * nb + tid;
+      r[0 * nb] = f2pack(v[0][1][0], v[1][1][0]);
+      r[1 * nb] = f2pack(v[0][1][1], v[1][1][1]);
+      r[2 * nb] = f2pack(v[0][2][0], v[1][2][0]);
+      r[3 * nb] = f2pack(v[0][2][1], v[1][2][1]);
+      r[4 * nb] = f2pack(v[0][2][2], v[1][2][2]);
+      r[5 * nb] = f2pack(v[0][3][0], v[1][3][0]);
+      r[6 * nb] = f2pack(v[0][3][1], v[1][3][1]);
+      r[7 * nb] = f2pack(v[0][3][2], v[1][3][2]);
+      r[8 * nb] = f2pack(v[0][3][3], v[1][3][3]);
+      r[9 * nb] = f2pack(v[0][0][0], v[1][0][0]);
+      r[10 * nb] = f2pack(a0A, a0B);
     }
   }
   const f2 Bl = f2pack(G[0].blim, G[1].blim);
@@ -523,36 +527,34 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
 #pragma unroll 1
   for (int d0 = 0; d0 < kP; ++d0) {
     Win2 W[kP];
-    f2 S1 = 0, L1 = 0;
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
-      const int e = (x == d0);
-      const uint4* r = rows + ((x * 2 + e) * 4) * kBlock + tid;
-      const uint4 q0 = r[0], q1 = r[kBlock], q2 = r[2 * kBlock];
-      W[x].s1 = ((f2)q0.y << 32) | q0.x;
-      W[x].s2[0] = ((f2)q0.w << 32) | q0.z;
-      W[x].s2[1] = ((f2)q1.y << 32) | q1.x;
-      W[x].s3[0] = ((f2)q1.w << 32) | q1.z;
-      W[x].s3[1] = ((f2)q2.y << 32) | q2.x;
-      W[x].s3[2] = ((f2)q2.w << 32) | q2.z;
+      const int e = (x == d0);  // every multiplicity of the stage-0 profile shifted by one
+      const f2* r = rows + (x * 11 + e) * nb + tid;
+      W[x].s1 = r[0];
+      W[x].s2[0] = r[2 * nb];
+      W[x].s2[1] = r[3 * nb];
+      W[x].s3[0] = r[5 * nb];
+      W[x].s3[1] = r[6 * nb];
+      W[x].s3[2] = r[7 * nb];
     }
-    {
-      const uint4 q3 = rows[((d0 * 2 + 1) * 4 + 3) * kBlock + tid];
-      S1 = ((f2)q3.y << 32) | q3.x;
-      L1 = ((f2)q3.w << 32) | q3.z;
-    }
+    const f2 S1 = rows[(d0 * 11 + 9) * nb + tid];
+    const f2 NL1 = f2sub(0ull, rows[(d0 * 11 + 10) * nb + tid]);  // -alpha t0^2
     const f2 B1 = f2sub(Bl, S1);
 #pragma unroll
     for (int d1 = 0; d1 < kP; ++d1) {
       const f2 w1 = W[d1].s1;
-      const f2 S2 = f2add(S1, w1), L2 = f2add(L1, a1[d1]), B2 = f2sub(B1, w1);
-      uint32_t accA = ~0u, accB = ~0u;
+      const f2 S2 = f2add(S1, w1), NL2 = f2sub(NL1, a1[d1]), B2 = f2sub(B1, w1);
+      // independent accumulator chains per q (ILP); merged at the end of the block
+      uint32_t accA[kP], accB[kP];
 #pragma unroll
       for (int q = 0; q < kP; ++q) {
         const f2 w2 = W[q].s2[q == d1];
         const f2 S3 = f2add(S2, w2), B3 = f2sub(B2, w2);
-        const f2 NL3 = f2sub(f2sub(0ull, L2), a2[q]);  // -(L2 + a2)
+        const f2 NL3 = f2sub(NL2, a2[q]);  // -(alpha * sum t^2 of stages 0..2)
         const f2 U = f2fma(S3, S3, NL3);
+        accA[q] = ~0u;
+        accB[q] = ~0u;
 #pragma unroll
         for (int p = 0; p < kP; ++p) {
           const f2 w3 = W[p].s3[(p == d1) + (p == q)];
@@ -561,20 +563,22 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
           uint32_t zl, zh, dl, dh;
           f2bits(z, zl, zh);
           f2bits(d2, dl, dh);
-          accA &= zl | dl;
-          accB &= zh | dh;
+          accA[q] &= zl | dl;
+          accB[q] &= zh | dh;
         }
       }
-      pendA |= ((accA >> 31) ^ 1u) << (kP * d0 + d1);
-      pendB |= ((accB >> 31) ^ 1u) << (kP * d0 + d1);
+      const uint32_t mA = accA[0] & accA[1] & accA[2] & accA[3] & accA[4];
+      const uint32_t mB = accB[0] & accB[1] & accB[2] & accB[3] & accB[4];
+      pendA |= ((mA >> 31) ^ 1u) << (kP * d0 + d1);
+      pendB |= ((mB >> 31) ^ 1u) << (kP * d0 + d1);
     }
   }
   // rare exact path, one half at a time (geometry copied into the state)
   constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
-#pragma unroll 1
-  for (int h = 0; h < (haveB ? 2 : 1); ++h) {
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
     const uint32_t pend = h ? pendB : pendA;
-    const uint32_t all = VERIFY ? kAll : pend;
+    const uint32_t all = (h && !haveB) ? 0u : (VERIFY ? kAll : pend);
     if (!all) continue;
 #pragma unroll
     for (int i = 0; i < 5; ++i) c.bnd[i] = G[h].bnd[i];
@@ -691,7 +695,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
   {  // A0: stage the table image into shared memory (16-byte copies)
     const uint4* src = reinterpret_cast<const uint4*>(A.image);
     uint4* dst = reinterpret_cast<uint4*>(smem);
-    for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += kBlock) dst[i] = src[i];
+    for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += blockDim.x) dst[i] = src[i];
   }
   __syncthreads();
   // KS = 4: per-thread rows of the shifted variant tables after the image (ks4_mask)
@@ -700,7 +704,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint64_t T = pre[A.n_req];
   const uint64_t sb = T * A.rank / A.world, se = T * (A.rank + 1) / A.world;
-  const uint64_t nthr = (uint64_t)gridDim.x * kBlock, g = (uint64_t)blockIdx.x * kBlock + threadIdx.x;
+  const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x, g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const uint64_t len = se - sb;
   const uint64_t t0 = sb + len * g / nthr, t1 = sb + len * (g + 1) / nthr;
   if (t0 >= t1) return;
@@ -769,7 +773,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
       // two consecutive masks of the same request per iteration (ks4_pair)
       const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
       const uint32_t maskB = haveB ? gosper_next(mask) : mask;
-      ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<uint4*>(rows), A.misses);
+      ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<f2*>(rows), A.misses);
       if (haveB) {
         step = 2;
         mask = maskB;
@@ -821,21 +825,22 @@ static cudaError_t set_attr() {
     default: return cudaErrorInvalidValue;               \
   }
 
-cudaError_t search_kernel_config(int ks, bool verify, size_t smem, int* blocks_per_sm) {
+cudaError_t search_kernel_config(int ks, bool verify, int block, size_t smem, int* blocks_per_sm) {
   cudaError_t e = cudaSuccess;
 #define CFG(K, V)                                                                                   \
   do {                                                                                            \
     e = set_attr<K, V>();                                                                         \
     if (e == cudaSuccess)                                                                         \
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_plan_search<K, V>, kBlock, smem); \
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_plan_search<K, V>, block, smem); \
   } while (0)
   FFS_KS_SWITCH(ks, verify, CFG)
 #undef CFG
   return e;
 }
 
-cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, size_t smem, cudaStream_t st) {
-#define LAUNCH(K, V) k_plan_search<K, V><<<grid, kBlock, smem, st>>>(a)
+cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
+                          cudaStream_t st) {
+#define LAUNCH(K, V) k_plan_search<K, V><<<grid, block, smem, st>>>(a)
   FFS_KS_SWITCH(ks, verify, LAUNCH)
 #undef LAUNCH
   return cudaGetLastError();
