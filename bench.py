@@ -176,6 +176,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_hpdc_hui0s25_b200 import ffs
+    from paper_conf_hpdc_hui0s25_b200 import dist as D
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -189,16 +190,13 @@ def main():
     pl.stage(prob)
     req, slo = ffs.to_device(prob)
     keys = torch.empty(R, dtype=torch.int64, device="cuda")
-    lo, hi = R * rank // world, R * (rank + 1) // world
+    lo, hi = D.request_slice(R, rank, world)
     plans = torch.empty((hi - lo, 80), dtype=torch.uint8, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
 
-    def step():
-        pl.plan_keys(req, slo, K, rank, world, keys=keys)
-        if world > 1:
-            dist.all_reduce(keys, op=dist.ReduceOp.MIN)
-        pl.plan_decode(req[lo:hi], slo[lo:hi], keys[lo:hi], K, out=plans)
+    def step():  # keys of this rank's shard -> all_reduce(MIN) over NCCL -> decode own slice
+        D.plan_step(pl, req, slo, K, rank, world, keys, plans)
 
     def barrier():
         if world > 1:
@@ -256,16 +254,11 @@ def main():
         d_slo = torch.empty_like(slo)
 
         def e2e_step():
-            if world == 1:
+            if world == 1:  # the single-GPU public call: ffs_plan_batch_host
                 pl.plan_batch_host(req_np, slo_np, K, out=out_np)
             else:
-                d_req.copy_(h_req.view(-1, 8).cuda(non_blocking=True).view_as(d_req))
-                d_slo.copy_(h_slo.view(torch.int32).cuda(non_blocking=True))
-                pl.plan_keys(d_req, d_slo, K, rank, world, keys=keys)
-                dist.all_reduce(keys, op=dist.ReduceOp.MIN)
-                pl.plan_decode(d_req[lo:hi], d_slo[lo:hi], keys[lo:hi], K, out=plans)
-                h_out.copy_(plans.view(-1), non_blocking=True)
-                torch.cuda.synchronize()
+                D.plan_step_host(pl, h_req.view(-1, 8), h_slo.view(torch.int32), d_req, d_slo, K, rank, world,
+                                 keys, plans, h_out)
 
         for _ in range(2):
             e2e_step()

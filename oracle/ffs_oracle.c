@@ -333,7 +333,9 @@ int oracle_plan(const oracle_plan_args *a, int n_threads) {
  *   pipeline, or busy*100 >= thr*window -> EXCL_HOT (P:358 pipelines; P:370 threshold)
  *   otherwise                          -> TIME_SHARING (utilization below 30%)
  * score = (last_used << 20) | instance index for a resident, idle (not BUSY)
- * time-sharing instance (LRU); every other instance scores INT64_MAX. */
+ * time-sharing instance (LRU); every other instance scores INT64_MAX.  The key
+ * packs last_used into 43 bits and the index into 20 (R20b): an instance with
+ * last_used >= 2^43 or index >= 2^20 cannot be represented and is not evictable. */
 void oracle_evict(int n_inst, const int32_t *inst_slice, const uint8_t *inst_flags, const uint32_t *inst_busy_us,
                   const uint64_t *inst_last_used_us, uint64_t now_us, uint32_t util_thr_pct, uint32_t window_us,
                   uint64_t cold_after_us, int64_t *score, uint8_t *state) {
@@ -351,7 +353,7 @@ void oracle_evict(int n_inst, const int32_t *inst_slice, const uint8_t *inst_fla
         else
             st = ST_TIME_SHARING;
         state[i] = st;
-        if (st == ST_TIME_SHARING && !(inst_flags[i] & FL_BUSY))
+        if (st == ST_TIME_SHARING && !(inst_flags[i] & FL_BUSY) && last < (1ull << 43) && i < (1 << 20))
             score[i] = (int64_t)((last << 20) | (uint64_t)i);
         else
             score[i] = KEY_NONE;

@@ -91,3 +91,38 @@ def brute_plan(prob, r, k_max=None):
                         best_c = dict(k=k, mask=mask, prof=list(seq), t=t, e2e=e2e, gpcs=g, cvq=cvq)
                 idx += 1
     return best, idx, nfeas, ksum, best_c
+
+
+def candidate_keys(prob, r, k_max=None):
+    """Every candidate of request r as (k, cut-mask rank, key or None), canonical order
+    (independent enumeration; used to emulate shards of the task space)."""
+    K = prob.k_max if k_max is None else k_max
+    f, v, B = int(prob.req["func"][r]), int(prob.req["node"][r]), int(prob.slo_us[r])
+    a, b = int(prob.comp_off[f]), int(prob.comp_off[f + 1])
+    n, P = b - a, prob.P
+    lat = prob.lat_us[a:b].astype(int).tolist()
+    mem = prob.mem_mib[a:b].astype(int).tolist()
+    xfer = prob.xfer_us[a:b].astype(int).tolist()
+    sl = prob.slices
+    free = [int(((sl["node"] == v) & (sl["busy"] == 0) & (sl["profile"] == p)).sum()) for p in range(P)]
+    out, idx = [], 0
+    for k in range(1, min(n, K) + 1):
+        masks = sorted(m for m in range(1 << (n - 1)) if bin(m).count("1") == k - 1)
+        for rank, mask in enumerate(masks):
+            cuts = [j for j in range(n - 1) if mask >> j & 1]
+            bounds = [0] + [j + 1 for j in cuts] + [n]
+            stages = [range(bounds[i], bounds[i + 1]) for i in range(k)]
+            for seq in itertools.product(range(P), repeat=k):
+                t = [sum(lat[c][p] for c in st) for st, p in zip(stages, seq)]
+                m = [sum(mem[c] for c in st) for st in stages]
+                ok = all(mi <= int(prob.cap_mib[p]) for mi, p in zip(m, seq))
+                ok = ok and all(seq.count(p) <= free[p] for p in range(P))
+                ok = ok and sum(t) + sum(xfer[j] for j in cuts) <= B
+                key = None
+                if ok:
+                    tf = [Fraction(x) for x in t]
+                    cvq = int(statistics.pvariance(tf) / statistics.mean(tf) ** 2 * 1024)
+                    key = pack_key(cvq, k, sum(int(prob.gpcs[p]) for p in seq), idx)
+                out.append((k, rank, key))
+                idx += 1
+    return out

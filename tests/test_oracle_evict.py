@@ -38,6 +38,14 @@ def test_state_rules_fig8():
             assert score[i] == KEY_NONE
 
 
+def test_lru_key_range_rule():
+    # R20b: last_used must fit the 43-bit field of the packed LRU key
+    rows = [(0, 1, 0, 0, (1 << 43) - 1), (1, 2, 0, 0, 1 << 43)]
+    score, state = oracle.evict(inst(rows), (1 << 43) + 10)
+    assert state.tolist() == [TS, TS]
+    assert score[0] == ((((1 << 43) - 1) << 20) | 0) and score[1] == KEY_NONE
+
+
 def test_lru_order_and_tie_break():
     # evict the least-recently-used time-sharing instance; equal last-use -> lower index
     rows = [(0, 1, 0, 0, NOW - 50), (1, 2, 0, 0, NOW - 500), (2, 3, 0, 0, NOW - 500), (3, 4, 0, 0, NOW - 5)]
