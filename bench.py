@@ -152,6 +152,59 @@ def run_reference(args, prob):
     print(json.dumps(line), flush=True)
 
 
+def run_c4(pl, steps: int, warmup: int, flush, peaks):
+    """C4: hotness-aware eviction over T = 4096 tick snapshots of a 32-node
+    (256-GPU) cluster, 200 warm functions -- one step = ffs_evict_scores_ticks over every
+    instance of every tick (A7) + ffs_evict_victims for every load (A8).  Reported against
+    the HBM roofline (33 algorithmic bytes per score: 24 B record in, 8 B score + 1 B state
+    out)."""
+    import torch
+    wl = W.config4()
+    prob = wl.problem
+    pl.stage(prob)
+    inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
+    toff = torch.from_numpy(wl.tick_off.view(np.int32)).cuda()
+    now = torch.from_numpy(wl.now_us.view(np.int64)).cuda()
+    req = torch.from_numpy(np.ascontiguousarray(prob.req).view(np.uint8).reshape(-1, 8)).cuda()
+    slo = torch.from_numpy(prob.slo_us.view(np.int32)).cuda()
+    rt = torch.from_numpy(wl.req_tick.view(np.int32)).cuda()
+    n = int(wl.inst.shape[0])
+    score = torch.empty(n, dtype=torch.int64, device="cuda")
+    state = torch.empty(n, dtype=torch.uint8, device="cuda")
+    vic = torch.empty(prob.R, dtype=torch.int32, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def step():
+        pl.evict_scores_ticks(inst, toff, now, score=score, state=state, window_us=wl.window_us)
+        pl.evict_victims(req, slo, rt, inst, toff, score, victim=vic)
+
+    for _ in range(warmup):
+        step()
+    torch.cuda.synchronize()
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(steps)]
+    for i in range(steps):
+        flush.fill_(i & 0xFF)
+        ev[i][0].record(stream)
+        pl.evict_scores_ticks(inst, toff, now, score=score, state=state, window_us=wl.window_us)
+        ev[i][1].record(stream)
+        pl.evict_victims(req, slo, rt, inst, toff, score, victim=vic)
+        ev[i][2].record(stream)
+    torch.cuda.synchronize()
+    t_sc = sum(e[0].elapsed_time(e[1]) for e in ev) / steps
+    t_vi = sum(e[1].elapsed_time(e[2]) for e in ev) / steps
+    peak = float(peaks.get("hbm_gbs", 6650.0))
+    achieved = 33.0 * n / (t_sc * 1e-3) / 1e9
+    return {"metric": "eviction_scores_per_s", "value": n / ((t_sc + t_vi) * 1e-3), "unit": "scores/s",
+            "ms_per_step": t_sc + t_vi, "scores_per_step": n, "loads_per_step": int(prob.R),
+            "workload": f"C4: 32 nodes (712 slices), 200 functions, {len(wl.now_us)} ticks x "
+                        f"{n // len(wl.now_us)} instances, victims for {prob.R} loads",
+            "kernels_ms": {"k_evict_ticks": t_sc, "k_victims": t_vi},
+            "roofline": {"bound": "hbm", "kernel": "k_evict_ticks", "achieved": achieved, "peak": peak,
+                         "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "alg_bytes_per_score": 33, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)"},
+            "l2": "flushed between steps"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -161,6 +214,7 @@ def main():
     ap.add_argument("--config", type=int, default=5, choices=[2, 3, 5])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-c4", action="store_true", help="skip the C4 eviction measurement")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference", "timing rules: >= 3 warm-up steps"
 
@@ -277,6 +331,9 @@ def main():
                "h2d_bytes_per_step": int(R * 12), "d2h_bytes_per_step": int((hi - lo) * 80),
                "timer": "host wall clock around the blocking call, max over ranks"}
 
+    c4 = None
+    if world == 1 and not args.no_c4:
+        c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
     if rank == 0:
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
@@ -301,6 +358,7 @@ def main():
             "gpu_launches": launches_per_step * args.steps,
             "e2e": e2e,
             "cpu_baseline": cpu,
+            "eviction_c4": c4,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -480,7 +480,7 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
   Geo4 G[2];
   geo4(c, maskA, G[0]);
   geo4(c, maskB, G[1]);
-  if (!haveB) G[1].blim = -1.f;  // dummy lane: nothing passes
+  if (!haveB) G[1].blim = -1.f;  // dummy lane: nothing passes (every slack < 0)
   const float al = c.alpha, one_m_a = 1.f - c.alpha;
   f2 a1[kP], a2[kP], t2[kP], cc[kP];
   {
@@ -507,22 +507,22 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
       cc[x] = f2pack(one_m_a * (f[0][3][x] * f[0][3][x]), one_m_a * (f[1][3][x] * f[1][3][x]));
       const float a0A = al * (f[0][0][x] * f[0][0][x]), a0B = al * (f[1][0][x] * f[1][0][x]);
       // compact per-thread row of profile x: 11 packed pairs
-      //   [v1[0], v1[1], v2[0], v2[1], v2[2], v3[0], v3[1], v3[2], v3[3], v0[0], a0]
+      //   [v1[0], v1[1], v2[0], v2[1], v2[2], Bl-v3[0..3], v0[0], a0]
+      // (the last stage is stored as SLO slack Blim - v3, so d2 = (Blim - v3) - S3)
       f2* r = rows + (x * 11) * nb + tid;
       r[0 * nb] = f2pack(v[0][1][0], v[1][1][0]);
       r[1 * nb] = f2pack(v[0][1][1], v[1][1][1]);
       r[2 * nb] = f2pack(v[0][2][0], v[1][2][0]);
       r[3 * nb] = f2pack(v[0][2][1], v[1][2][1]);
       r[4 * nb] = f2pack(v[0][2][2], v[1][2][2]);
-      r[5 * nb] = f2pack(v[0][3][0], v[1][3][0]);
-      r[6 * nb] = f2pack(v[0][3][1], v[1][3][1]);
-      r[7 * nb] = f2pack(v[0][3][2], v[1][3][2]);
-      r[8 * nb] = f2pack(v[0][3][3], v[1][3][3]);
+      r[5 * nb] = f2pack(G[0].blim - v[0][3][0], G[1].blim - v[1][3][0]);
+      r[6 * nb] = f2pack(G[0].blim - v[0][3][1], G[1].blim - v[1][3][1]);
+      r[7 * nb] = f2pack(G[0].blim - v[0][3][2], G[1].blim - v[1][3][2]);
+      r[8 * nb] = f2pack(G[0].blim - v[0][3][3], G[1].blim - v[1][3][3]);
       r[9 * nb] = f2pack(v[0][0][0], v[1][0][0]);
       r[10 * nb] = f2pack(a0A, a0B);
     }
   }
-  const f2 Bl = f2pack(G[0].blim, G[1].blim);
   uint32_t pendA = 0, pendB = 0;
 #pragma unroll 1
   for (int d0 = 0; d0 < kP; ++d0) {
@@ -540,17 +540,16 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
     }
     const f2 S1 = rows[(d0 * 11 + 9) * nb + tid];
     const f2 NL1 = f2sub(0ull, rows[(d0 * 11 + 10) * nb + tid]);  // -alpha t0^2
-    const f2 B1 = f2sub(Bl, S1);
 #pragma unroll
     for (int d1 = 0; d1 < kP; ++d1) {
       const f2 w1 = W[d1].s1;
-      const f2 S2 = f2add(S1, w1), NL2 = f2sub(NL1, a1[d1]), B2 = f2sub(B1, w1);
+      const f2 S2 = f2add(S1, w1), NL2 = f2sub(NL1, a1[d1]);
       // independent accumulator chains per q (ILP); merged at the end of the block
       uint32_t accA[kP], accB[kP];
 #pragma unroll
       for (int q = 0; q < kP; ++q) {
         const f2 w2 = W[q].s2[q == d1];
-        const f2 S3 = f2add(S2, w2), B3 = f2sub(B2, w2);
+        const f2 S3 = f2add(S2, w2);
         const f2 NL3 = f2sub(NL2, a2[q]);  // -(alpha * sum t^2 of stages 0..2)
         const f2 U = f2fma(S3, S3, NL3);
         accA[q] = ~0u;
@@ -559,7 +558,7 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
         for (int p = 0; p < kP; ++p) {
           const f2 w3 = W[p].s3[(p == d1) + (p == q)];
           const f2 z = f2add(f2fma(S3, t2[p], cc[p]), U);
-          const f2 d2 = f2sub(B3, w3);
+          const f2 d2 = f2sub(w3, S3);  // (Blim - v3) - S3 < 0: SLO / memory / free miss
           uint32_t zl, zh, dl, dh;
           f2bits(z, zl, zh);
           f2bits(d2, dl, dh);
