@@ -974,17 +974,26 @@ __device__ __forceinline__ void evict_one(const ffs_instance& in, uint32_t i, ui
   state[gi] = st;
 }
 
-// one CTA per tick (blockIdx.y), grid-stride over the tick's instances
-__global__ void __launch_bounds__(256) k_evict_ticks(const ffs_instance* __restrict__ inst,
-                                                      const uint32_t* __restrict__ tick_off,
-                                                      const uint64_t* __restrict__ now_us, ffs_evict_params prm,
-                                                      int64_t* __restrict__ score, uint8_t* __restrict__ state) {
+// one CTA per tick; 4 records in flight per thread (memory-level parallelism).  (A flat
+// persistent grid with a per-record binary search of the tick measured 1.7x slower.)
+constexpr int kEvT = 128, kEvU = 4;
+__global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __restrict__ inst,
+                                                       const uint32_t* __restrict__ tick_off,
+                                                       const uint64_t* __restrict__ now_us, ffs_evict_params prm,
+                                                       int64_t* __restrict__ score, uint8_t* __restrict__ state) {
   const uint32_t t = blockIdx.x;
   const uint32_t b = tick_off[t], e = tick_off[t + 1];
   const uint64_t now = now_us[t];
-  for (uint32_t gi = b + threadIdx.x; gi < e; gi += blockDim.x) {
-    const ffs_instance in = inst[gi];
-    evict_one(in, gi - b, now, prm, score, state, gi);
+  for (uint32_t g0 = b + threadIdx.x; g0 < e; g0 += kEvT * kEvU) {
+    ffs_instance in[kEvU];
+#pragma unroll
+    for (int u = 0; u < kEvU; ++u)
+      if (g0 + u * kEvT < e) in[u] = inst[g0 + u * kEvT];
+#pragma unroll
+    for (int u = 0; u < kEvU; ++u) {
+      const uint32_t gi = g0 + u * kEvT;
+      if (gi < e) evict_one(in[u], gi - b, now, prm, score, state, gi);
+    }
   }
 }
 
@@ -1001,7 +1010,7 @@ cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32
                          uint32_t n_ticks, uint64_t now_single, ffs_evict_params prm, int64_t* score, uint8_t* state,
                          cudaStream_t st) {
   if (tick_off) {
-    if (n_ticks) k_evict_ticks<<<n_ticks, 256, 0, st>>>(inst, tick_off, now_us, prm, score, state);
+    if (n_ticks) k_evict_ticks<<<n_ticks, kEvT, 0, st>>>(inst, tick_off, now_us, prm, score, state);
   } else if (n_inst) {
     int blocks = (int)((n_inst + 255) / 256);
     k_evict_one<<<blocks, 256, 0, st>>>(inst, n_inst, now_single, prm, score, state);
@@ -1012,31 +1021,56 @@ cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32
 // ====================================================================================
 // K4: victims per request over its tick's instances (A8)
 // ====================================================================================
-__global__ void __launch_bounds__(128) k_victims(const uint32_t* __restrict__ img, ImageLayout L,
-                                                  const ffs_request* __restrict__ req, const uint32_t* __restrict__ slo,
-                                                  const uint32_t* __restrict__ req_tick, uint32_t n_req,
-                                                  const ffs_instance* __restrict__ inst,
-                                                  const uint32_t* __restrict__ tick_off,
-                                                  const int64_t* __restrict__ score, const uint16_t* slice_node,
-                                                  const uint8_t* slice_prof, uint32_t n_slices,
-                                                  int32_t* __restrict__ victim) {
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+// Profiles whose slice can host request (f, B) monolithically: the whole function fits
+// the slice memory and latency alone + reload <= B (R19).
+__device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const ImageLayout& L, uint32_t f,
+                                                    uint32_t B) {
+  const uint32_t* fd = img + L.o_fdesc + 4 * f;
+  const uint32_t row0 = fd[0], n = fd[1];
+  uint32_t ok = 0;
+#pragma unroll
+  for (int p = 0; p < kP; ++p) {
+    const uint64_t lat = (uint64_t)img[L.o_pl + (row0 + n) * kRowW + p] - img[L.o_pl + row0 * kRowW + p];
+    if (fd[3] <= img[L.o_cap + p] && lat + fd[2] <= B) ok |= 1u << p;
+  }
+  return ok;
+}
+
+// one warp per load: lanes scan the tick's instances, warp min of the packed score
+constexpr int kViT = 256;
+__global__ void __launch_bounds__(kViT) k_victims(const uint32_t* __restrict__ img, ImageLayout L,
+                                                   const ffs_request* __restrict__ req, const uint32_t* __restrict__ slo,
+                                                   const uint32_t* __restrict__ req_tick, uint32_t n_req,
+                                                   const ffs_instance* __restrict__ inst,
+                                                   const uint32_t* __restrict__ tick_off,
+                                                   const int64_t* __restrict__ score, const uint16_t* slice_node,
+                                                   const uint8_t* slice_prof, uint32_t n_slices,
+                                                   int32_t* __restrict__ victim) {
+  const uint32_t r = (blockIdx.x * kViT + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (r >= n_req) return;
   const ffs_request q = req[r];
-  int32_t best_i = -1;
+  int64_t bs = (int64_t)kKeyNone;
+  uint32_t b = 0, e = 0;
   if (q.func < L.F) {
+    const uint32_t okp = victim_profiles(img, L, q.func, slo[r]);
     const uint32_t t = req_tick[r];
-    const uint32_t b = tick_off[t], e = tick_off[t + 1];
-    int64_t bs = (int64_t)kKeyNone;
-    for (uint32_t i = b; i < e; ++i) {
+    b = tick_off[t];
+    e = tick_off[t + 1];
+    for (uint32_t i = b + lane; i < e; i += 32) {
       const int64_t s = score[i];
-      if (s < bs && victim_ok(img, L, q.func, q.node, slo[r], inst[i], s, slice_node, slice_prof, n_slices)) {
-        bs = s;
-        best_i = (int32_t)(i - b);
-      }
+      if ((uint64_t)s == kKeyNone || s >= bs) continue;
+      const int32_t sl = inst[i].slice;
+      if (sl < 0 || (uint32_t)sl >= n_slices || slice_node[sl] != q.node || !((okp >> slice_prof[sl]) & 1u)) continue;
+      bs = s;
     }
   }
-  victim[r] = best_i;
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const int64_t y = __shfl_xor_sync(0xffffffffu, bs, o);
+    bs = y < bs ? y : bs;
+  }
+  // the packed score's low 20 bits are the index within the tick (R20b)
+  if (lane == 0) victim[r] = (uint64_t)bs == kKeyNone ? -1 : (int32_t)((uint64_t)bs & 0xFFFFFu);
 }
 
 cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const ffs_request* req, const uint32_t* slo,
@@ -1046,8 +1080,10 @@ cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const 
                            int32_t* victim, cudaStream_t st) {
   (void)n_ticks;
   if (n_req == 0) return cudaSuccess;
-  k_victims<<<(n_req + 127) / 128, 128, 0, st>>>(image, lay, req, slo, req_tick, n_req, inst, tick_off, score,
-                                                  slice_node, slice_prof, n_slices, victim);
+  const uint64_t threads = (uint64_t)n_req * 32;
+  k_victims<<<(unsigned)((threads + kViT - 1) / kViT), kViT, 0, st>>>(image, lay, req, slo, req_tick, n_req, inst,
+                                                                       tick_off, score, slice_node, slice_prof,
+                                                                       n_slices, victim);
   return cudaGetLastError();
 }
 
