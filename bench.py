@@ -235,9 +235,14 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = local % torch.cuda.device_count()  # several ranks may share a GPU in smoke runs
     torch.cuda.set_device(local)
+    backend = os.environ.get("FFS_DIST_BACKEND", "nccl")  # gloo: multi-rank smoke on one GPU
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
     K = prob.k_max
     R = prob.R
     pl = ffs.Planner(local)
