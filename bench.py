@@ -351,7 +351,7 @@ def main():
             "data": "synthetic", "plans_per_s": plans_per_s,
             "config": {"workload": prob.meta["workload"], "R": R, "k_max": K, "candidates_per_step": total_cands,
                        "l2": "flushed between steps (256 MiB write, outside the events)",
-                       "parallelism": f"candidate-range shards x{world} + all_reduce(MIN) over NCCL" if world > 1
+                       "parallelism": f"candidate-range shards x{world} + all_reduce(MIN) over {backend}" if world > 1
                        else "single GPU"},
             "roofline": {"bound": "alu", "kernel": f"k_plan_search<{top}>", "achieved": achieved, "peak": peak_ops,
                          "unit": "int lane-ops/s", "frac": achieved / peak_ops, "traffic": traffic,
