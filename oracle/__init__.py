@@ -61,6 +61,8 @@ def lib():
             _lib = C.CDLL(build())
             _lib.oracle_plan.argtypes = [C.POINTER(_PlanArgs), C.c_int]
             _lib.oracle_plan.restype = C.c_int
+            _lib.oracle_plan_ranked.argtypes = [C.POINTER(_PlanArgs), C.c_int, C.c_int]
+            _lib.oracle_plan_ranked.restype = C.c_int
             _lib.oracle_evict.restype = None
             _lib.oracle_victim.restype = None
     return _lib
@@ -128,6 +130,22 @@ def plan(prob, k_max: int | None = None, threads: int | None = None, checks: boo
     rc = lib().oracle_plan(C.byref(h.args), int(threads))
     if rc != 0:
         raise ValueError("oracle_plan rejected its arguments")
+    return h.out
+
+
+def plan_ranked(prob, p_ref: int | None = None, k_max: int | None = None, threads: int | None = None) -> dict:
+    """NEXT-1: the paper's offline CV ranking + first-fit walk (ffs_oracle.c:
+    oracle_plan_ranked).  p_ref = reference profile of the offline CV (default: the
+    profile with the most GPCs).  key = position of the chosen partition in the ranked
+    list.  Same output fields as plan() (no checks)."""
+    k_max = int(prob.k_max if k_max is None else k_max)
+    threads = os.cpu_count() if threads is None else threads
+    if p_ref is None:
+        p_ref = int(np.argmax(np.asarray(prob.gpcs)))
+    h = _Held(prob, k_max, False)
+    rc = lib().oracle_plan_ranked(C.byref(h.args), int(p_ref), int(threads))
+    if rc != 0:
+        raise ValueError("oracle_plan_ranked rejected its arguments")
     return h.out
 
 

@@ -393,3 +393,224 @@ void oracle_victim(const oracle_plan_args *a, const int32_t *status, int n_inst,
         }
     }
 }
+
+/* ---- NEXT-1: the paper's literal offline CV ranking + first-fit walk ------
+ * Offline (per function): every contiguous partition with k <= k_max stages, ranked by
+ * (cvq_ref, k, mask) ascending where cvq_ref = floor(1024 * CV^2) of the stage times on
+ * the reference profile p_ref (R24, R25; "calculating and sorting the CVs for all possible
+ * pipeline configurations ... once and offline").  Online (per request): walk the ranked
+ * list and take the first partition "supported by the available resources":
+ * stages in descending memory (ties: lower stage) each take a distinct free slice of the
+ * smallest-capacity (then fewest-GPC, then lowest-id) profile that holds the stage; the
+ * partition is supported when every stage gets one and the resulting e2e <= B (R26).
+ * Plan fields as in oracle_plan, computed on the assigned profiles; key = position in the
+ * ranked list (R27). */
+typedef struct {
+    uint64_t cvq;
+    int k;
+    uint32_t mask;
+} ranked_entry;
+
+static int cmp_ranked(const void *x, const void *y) {
+    const ranked_entry *a = (const ranked_entry *)x, *b = (const ranked_entry *)y;
+    if (a->cvq != b->cvq) return a->cvq < b->cvq ? -1 : 1;
+    if (a->k != b->k) return a->k < b->k ? -1 : 1;
+    if (a->mask != b->mask) return a->mask < b->mask ? -1 : 1;
+    return 0;
+}
+
+typedef struct {
+    ranked_entry *e;
+    int n, cap;
+    const oracle_plan_args *a;
+    int f, nc, k, p_ref;
+} rank_builder;
+
+static void rank_add(rank_builder *b, uint32_t mask) {
+    const oracle_plan_args *a = b->a;
+    uint64_t t[ORACLE_MAX_STAGES] = {0}, sum = 0;
+    int st = 0;
+    for (int c = 0; c < b->nc; c++) {
+        t[st] += lat_of(a, b->f, c, b->p_ref);
+        if (c < b->nc - 1 && ((mask >> c) & 1u)) st++;
+    }
+    unsigned __int128 sq = 0;
+    for (int i = 0; i < b->k; i++) {
+        sum += t[i];
+        sq += (unsigned __int128)t[i] * t[i];
+    }
+    unsigned __int128 D = (unsigned __int128)sum * sum;
+    unsigned __int128 N = (unsigned __int128)b->k * sq - D;
+    if (b->n == b->cap) {
+        b->cap = b->cap ? 2 * b->cap : 64;
+        b->e = (ranked_entry *)realloc(b->e, sizeof(ranked_entry) * (size_t)b->cap);
+    }
+    b->e[b->n].cvq = (uint64_t)(((unsigned __int128)1024 * N) / D);
+    b->e[b->n].k = b->k;
+    b->e[b->n].mask = mask;
+    b->n++;
+}
+
+static void rank_masks(rank_builder *b, int remaining, int limit, uint32_t mask) {
+    if (remaining == 0) {
+        rank_add(b, mask);
+        return;
+    }
+    for (int j = remaining - 1; j < limit; j++) rank_masks(b, remaining - 1, j, mask | (1u << j));
+}
+
+static void ranked_one(const oracle_plan_args *a, int p_ref, int r) {
+    a->status[r] = PLAN_BAD_REQ;
+    a->key[r] = KEY_NONE;
+    a->k[r] = 0;
+    a->cut_mask[r] = 0;
+    a->e2e_us[r] = 0;
+    a->bottleneck_us[r] = 0;
+    a->gpcs_out[r] = 0;
+    a->cvq[r] = 0;
+    for (int i = 0; i < ORACLE_MAX_STAGES; i++) {
+        a->prof[(size_t)r * 8 + i] = 0xFF;
+        a->slice[(size_t)r * 8 + i] = -1;
+    }
+    if (a->req_func[r] >= (uint32_t)a->F || a->req_node[r] >= (uint32_t)a->n_nodes) return;
+    int f = (int)a->req_func[r], v = (int)a->req_node[r];
+    int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+    uint32_t free_cnt[ORACLE_MAX_P] = {0};
+    for (int i = 0; i < a->n_slices; i++)
+        if (a->sl_node[i] == v && !a->sl_busy[i]) free_cnt[a->sl_prof[i]]++;
+    /* offline ranking of this function's partitions (recomputed here for plainness) */
+    rank_builder b = {0};
+    b.a = a;
+    b.f = f;
+    b.nc = n;
+    b.p_ref = p_ref;
+    int kmax = a->k_max < n ? a->k_max : n;
+    for (int k = 1; k <= kmax; k++) {
+        b.k = k;
+        rank_masks(&b, k - 1, n - 1, 0u);
+    }
+    qsort(b.e, (size_t)b.n, sizeof(ranked_entry), cmp_ranked);
+    /* profiles in (capacity, gpcs, id) order */
+    int order[ORACLE_MAX_P];
+    for (int p = 0; p < a->P; p++) order[p] = p;
+    for (int i = 0; i < a->P; i++)
+        for (int j = i + 1; j < a->P; j++) {
+            int x = order[i], y = order[j];
+            int swap = a->cap_mib[y] < a->cap_mib[x] ||
+                       (a->cap_mib[y] == a->cap_mib[x] && (a->gpcs[y] < a->gpcs[x] || (a->gpcs[y] == a->gpcs[x] && y < x)));
+            if (swap) {
+                order[i] = y;
+                order[j] = x;
+            }
+        }
+    a->status[r] = PLAN_INFEASIBLE;
+    for (int e = 0; e < b.n; e++) {
+        int k = b.e[e].k;
+        uint32_t mask = b.e[e].mask;
+        int first[ORACLE_MAX_STAGES], last[ORACLE_MAX_STAGES], st = 0;
+        first[0] = 0;
+        for (int c = 0; c < n; c++) {
+            int cut = (c < n - 1) && ((mask >> c) & 1u);
+            if (c == n - 1 || cut) {
+                last[st] = c;
+                st++;
+                if (st < k) first[st] = c + 1;
+            }
+        }
+        uint64_t m[ORACLE_MAX_STAGES];
+        for (int i = 0; i < k; i++) {
+            m[i] = 0;
+            for (int c = first[i]; c <= last[i]; c++) m[i] += a->mem_mib[a->comp_off[f] + c];
+        }
+        /* min-resource greedy: stages by descending memory, smallest fitting free profile */
+        uint32_t left[ORACLE_MAX_P];
+        for (int p = 0; p < a->P; p++) left[p] = free_cnt[p];
+        int prof[ORACLE_MAX_STAGES], done[ORACLE_MAX_STAGES] = {0}, ok = 1;
+        for (int step = 0; step < k && ok; step++) {
+            int s = -1;
+            for (int i = 0; i < k; i++)
+                if (!done[i] && (s < 0 || m[i] > m[s])) s = i;
+            done[s] = 1;
+            prof[s] = -1;
+            for (int oi = 0; oi < a->P; oi++) {
+                int p = order[oi];
+                if (left[p] > 0 && m[s] <= a->cap_mib[p]) {
+                    prof[s] = p;
+                    left[p]--;
+                    break;
+                }
+            }
+            if (prof[s] < 0) ok = 0;
+        }
+        if (!ok) continue;
+        uint64_t t[ORACLE_MAX_STAGES], e2e = 0, bott = 0, g = 0;
+        unsigned __int128 sq = 0;
+        uint64_t sum = 0;
+        for (int i = 0; i < k; i++) {
+            t[i] = 0;
+            for (int c = first[i]; c <= last[i]; c++) t[i] += lat_of(a, f, c, prof[i]);
+            sum += t[i];
+            sq += (unsigned __int128)t[i] * t[i];
+            if (t[i] > bott) bott = t[i];
+            g += a->gpcs[prof[i]];
+        }
+        e2e = sum;
+        for (int j = 0; j < n - 1; j++)
+            if ((mask >> j) & 1u) e2e += a->xfer_us[a->comp_off[f] + j];
+        if (e2e > a->req_slo_us[r]) continue;
+        unsigned __int128 D = (unsigned __int128)sum * sum;
+        unsigned __int128 N = (unsigned __int128)k * sq - D;
+        a->status[r] = PLAN_OK;
+        a->key[r] = e;
+        a->k[r] = k;
+        a->cut_mask[r] = mask;
+        a->e2e_us[r] = (uint32_t)e2e;
+        a->bottleneck_us[r] = (uint32_t)bott;
+        a->gpcs_out[r] = (uint32_t)g;
+        a->cvq[r] = (uint32_t)(((unsigned __int128)1024 * N) / D);
+        for (int i = 0; i < k; i++) {
+            a->prof[(size_t)r * 8 + i] = (uint8_t)prof[i];
+            for (int x = 0; x < a->n_slices; x++) {
+                if (a->sl_node[x] != v || a->sl_busy[x] || a->sl_prof[x] != prof[i]) continue;
+                int taken = 0;
+                for (int j = 0; j < i; j++)
+                    if (a->slice[(size_t)r * 8 + j] == x) taken = 1;
+                if (taken) continue;
+                a->slice[(size_t)r * 8 + i] = x;
+                break;
+            }
+        }
+        break;
+    }
+    free(b.e);
+}
+
+typedef struct {
+    const oracle_plan_args *a;
+    int p_ref, tid, nthreads;
+} ranked_worker_arg;
+
+static void *ranked_worker(void *p) {
+    ranked_worker_arg *w = (ranked_worker_arg *)p;
+    for (int r = w->tid; r < w->a->R; r += w->nthreads) ranked_one(w->a, w->p_ref, r);
+    return NULL;
+}
+
+int oracle_plan_ranked(const oracle_plan_args *a, int p_ref, int n_threads) {
+    if (!a || a->P < 1 || a->P > ORACLE_MAX_P || a->k_max < 1 || a->k_max > ORACLE_MAX_STAGES) return -1;
+    if (p_ref < 0 || p_ref >= a->P) return -1;
+    if (n_threads < 1) n_threads = 1;
+    pthread_t *th = (pthread_t *)malloc(sizeof(pthread_t) * (size_t)n_threads);
+    ranked_worker_arg *wa = (ranked_worker_arg *)malloc(sizeof(ranked_worker_arg) * (size_t)n_threads);
+    for (int i = 0; i < n_threads; i++) {
+        wa[i].a = a;
+        wa[i].p_ref = p_ref;
+        wa[i].tid = i;
+        wa[i].nthreads = n_threads;
+        pthread_create(&th[i], NULL, ranked_worker, &wa[i]);
+    }
+    for (int i = 0; i < n_threads; i++) pthread_join(th[i], NULL);
+    free(th);
+    free(wa);
+    return 0;
+}
