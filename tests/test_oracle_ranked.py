@@ -93,8 +93,10 @@ def test_ranked_hand_case():
     assert o["status"][0] == oracle.PLAN_OK and o["k"][0] == 3 and o["cut_mask"][0] == 0b11
     assert list(o["prof"][0, :3]) == [G2, G2, G1] and list(o["slice"][0, :3]) == [0, 1, 2]
     assert o["key"][0] == 2 and o["e2e_us"][0] == 340
-    # budget 339: rank 2 misses the SLO, rank 3 is not supported -> INFEASIBLE
-    assert o["status"][1] == oracle.PLAN_INFEASIBLE
+    # budget 339: rank 2 misses the SLO (340); rank 3 [c0 | c1 c2] = 12 | 18 GB takes the
+    # two 2g slices: e2e = 30 + (30 + 60) + 100 = 220 <= 339 -> chosen
+    assert o["status"][1] == oracle.PLAN_OK and o["key"][1] == 3 and o["cut_mask"][1] == 0b01
+    assert list(o["prof"][1, :2]) == [G2, G2] and o["e2e_us"][1] == 220
 
 
 def test_ranked_prefers_monolithic_when_a_slice_fits():
