@@ -99,12 +99,23 @@ def test_ranked_hand_case():
     assert list(o["prof"][1, :2]) == [G2, G2] and o["e2e_us"][1] == 220
 
 
-def test_ranked_prefers_monolithic_when_a_slice_fits():
-    # the 1-stage partition has CV = 0 and ranks first: with a slice that holds the whole
-    # function and a loose SLO the walk returns the monolithic plan on the smallest fit
+def test_ranked_rank0_is_the_smallest_monolithic_fit():
+    # rank 0 is the 1-stage partition (CV = 0).  When the smallest-capacity free profile
+    # that holds the whole function meets the SLO, the walk stops there (k = 1 on it).
     prob = W.config2(R=256)
     o = oracle.plan_ranked(prob)
-    a = oracle.plan(prob, k_max=1, checks=False)
-    both = (a["status"] == oracle.PLAN_OK) & (o["status"] == oracle.PLAN_OK)
-    assert (o["k"][a["status"] == oracle.PLAN_OK] >= 1).all()
-    assert both.sum() > 0
+    sl = prob.slices
+    hits = 0
+    for r in range(prob.R):
+        f, v, B = int(prob.req["func"][r]), int(prob.req["node"][r]), int(prob.slo_us[r])
+        a, b = int(prob.comp_off[f]), int(prob.comp_off[f + 1])
+        mem = int(prob.mem_mib[a:b].sum())
+        fits = [p for p in range(prob.P)
+                if ((sl["node"] == v) & (sl["busy"] == 0) & (sl["profile"] == p)).any() and mem <= prob.cap_mib[p]]
+        if not fits:
+            continue
+        p = min(fits, key=lambda q: (int(prob.cap_mib[q]), int(prob.gpcs[q]), q))
+        if int(prob.lat_us[a:b, p].sum()) <= B:
+            hits += 1
+            assert o["k"][r] == 1 and o["prof"][r, 0] == p and o["key"][r] == 0
+    assert hits > 0
