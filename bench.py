@@ -205,6 +205,34 @@ def run_c4(pl, steps: int, warmup: int, flush, peaks):
             "l2": "flushed between steps"}
 
 
+def run_ranked(pl, prob, req, slo, steps: int, warmup: int, flush):
+    """NEXT-1 (the paper's literal offline-CV ranked first-fit) on the same batch:
+    plans/s of ffs_plan_ranked (the offline ranking is done once, outside the timing)."""
+    import torch
+    t0 = time.perf_counter()
+    pl.rank_partitions(prob.k_max, int(np.argmax(prob.gpcs)))
+    rank_s = time.perf_counter() - t0
+    out = torch.empty((prob.R, 80), dtype=torch.uint8, device="cuda")
+    for _ in range(warmup):
+        pl.plan_ranked(req, slo, out=out)
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    ms = 0.0
+    for i in range(steps):
+        flush.fill_(i & 0xFF)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        pl.plan_ranked(req, slo, out=out)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ms += a.elapsed_time(b)
+    from paper_conf_hpdc_hui0s25_b200 import ffs
+    p = ffs.plans_to_numpy(out)
+    return {"metric": "ranked_first_fit_plans_per_s", "value": prob.R * steps / (ms * 1e-3), "unit": "plans/s",
+            "ms_per_step": ms / steps, "offline_rank_s": rank_s,
+            "ok_frac": float((p["status"] == 0).mean()), "multi_stage_frac": float(((p["status"] == 0) & (p["k"] > 1)).mean())}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -336,6 +364,9 @@ def main():
                "h2d_bytes_per_step": int(R * 12), "d2h_bytes_per_step": int((hi - lo) * 80),
                "timer": "host wall clock around the blocking call, max over ranks"}
 
+    ranked = None
+    if world == 1 and not args.no_c4:
+        ranked = run_ranked(pl, prob, req, slo, args.steps, args.warmup, flush)
     c4 = None
     if world == 1 and not args.no_c4:
         c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
@@ -364,6 +395,7 @@ def main():
             "e2e": e2e,
             "cpu_baseline": cpu,
             "eviction_c4": c4,
+            "ranked_first_fit": ranked,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -232,6 +232,26 @@ ffs_status ffs_evict_victims(ffs_ctx *ctx, const ffs_request *d_req, const uint3
                              const uint32_t *d_tick_off, const int64_t *d_score, uint32_t n_ticks,
                              int32_t *d_victim, void *stream);
 
+/* ---- NEXT-1: the paper's literal ranked first-fit ---------------------------
+ * "After calculating and sorting the CVs for all possible pipeline configurations, which
+ * is done once and offline for each application ... The pipelines are then evaluated in
+ * order with the profiles, against the available MIG resources".
+ * ffs_rank_partitions: offline step.  For every staged function, every contiguous
+ * partition with k <= k_max stages ranked by (cvq of the stage times on the reference
+ * profile p_ref, k, cut mask) ascending (R24, R25).  Host computation +
+ * upload, synchronous.  FFS_ERR_RANGE: p_ref >= P, k_max not in 1..8, or more than 2^24
+ * ranked partitions in total.  FFS_ERR_STATE: tables not staged.
+ * ffs_plan_ranked: per request, walk its function's ranked list and take the first
+ * partition "supported by the available resources" (R26): stages in descending memory
+ * each take a distinct free slice of the smallest-capacity (then fewest-GPC, then
+ * lowest-id) profile of the request's node that holds the stage, and the resulting
+ * e2e <= budget.  d_out fields as ffs_plan_decode (computed on the assigned profiles,
+ * slices bound in stage order); key = position in the ranked list (R27); INFEASIBLE
+ * when no partition is supported.  Asynchronous on `stream`. */
+ffs_status ffs_rank_partitions(ffs_ctx *ctx, uint32_t k_max, uint32_t p_ref);
+ffs_status ffs_plan_ranked(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                           ffs_plan *d_out, void *stream);
+
 /* ---- measurement / debug helpers ------------------------------------------------------
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
  * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */

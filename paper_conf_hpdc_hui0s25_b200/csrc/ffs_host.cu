@@ -59,6 +59,12 @@ struct ffs_ctx {
   uint32_t P = 0, F = 0, n_nodes = 0, n_slices = 0, max_n = 0, max_gpcs = 0;
   std::vector<uint32_t> fn_len;
   DevBuf image, node_free, free_list, slice_node, slice_prof;
+  std::vector<uint32_t> h_image;  // host copy of the table image (offline ranking)
+  ImageLayout h_lay{};
+  // NEXT-1 ranked partitions
+  DevBuf rank_off, rank_mask;
+  bool ranked = false;
+  uint32_t rank_kmax = 0, prof_order = 0;
   // scratch
   DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses;
   // cached occupancy per (ks, verify, smem)
@@ -128,7 +134,7 @@ void ffs_destroy(ffs_ctx* c) {
     DeviceGuard g(c->device);
     for (auto& e : c->ev)
       if (e) cudaEventDestroy(e);
-    for (DevBuf* b : {&c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
+    for (DevBuf* b : {&c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses})
       b->release();
   }
@@ -284,6 +290,8 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   CK(c->slice_prof.ensure(sprof.size()), "cudaMalloc(slice_prof)");
   CK(cudaMemcpy(c->slice_prof.p, sprof.data(), sprof.size(), cudaMemcpyHostToDevice), "upload slice_prof");
   c->lay = L;
+  c->h_image = img;
+  c->ranked = false;
   c->P = P;
   c->F = F;
   c->n_nodes = NN;
@@ -476,6 +484,107 @@ ffs_status ffs_evict_victims(ffs_ctx* c, const ffs_request* d_req, const uint32_
                     n_ticks, c->slice_node.as<uint16_t>(), c->slice_prof.as<uint8_t>(), c->n_slices, d_victim,
                     (cudaStream_t)stream),
      "victims kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_rank_partitions(ffs_ctx* c, uint32_t k_max, uint32_t p_ref) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  if (k_max < 1 || k_max > (uint32_t)kMaxK) return fail(c, FFS_ERR_RANGE, "k_max %u not in 1..8", k_max);
+  if (p_ref >= c->P) return fail(c, FFS_ERR_RANGE, "p_ref %u >= P", p_ref);
+  const ImageLayout& L = c->lay;
+  const std::vector<uint32_t>& img = c->h_image;
+  uint64_t total = 0;
+  for (uint32_t f = 0; f < c->F; ++f)
+    for (uint32_t k = 1; k <= std::min(k_max, c->fn_len[f]); ++k) total += binom64((int)c->fn_len[f] - 1, (int)k - 1);
+  if (total >= (1ull << 24)) return fail(c, FFS_ERR_RANGE, "%llu ranked partitions > 2^24", (unsigned long long)total);
+  std::vector<uint32_t> off(c->F + 1, 0), masks;
+  masks.reserve((size_t)total);
+  struct E { uint64_t cvq; uint32_t k, mask; };
+  for (uint32_t f = 0; f < c->F; ++f) {
+    const uint32_t row0 = img[L.o_fdesc + 4 * f], n = img[L.o_fdesc + 4 * f + 1];
+    std::vector<E> es;
+    for (uint32_t k = 1; k <= std::min(k_max, n); ++k) {
+      // every (k-1)-subset of the n-1 cut positions in ascending numeric order (Gosper)
+      if (k == 1) {
+        es.push_back({0, 1, 0});
+        continue;
+      }
+      const uint32_t lim = 1u << (n - 1);
+      for (uint32_t m = (1u << (k - 1)) - 1; m < lim;) {
+        uint64_t s = 0, sq = 0;
+        uint32_t a = 0, mm = m;
+        for (uint32_t i = 0; i < k; ++i) {
+          uint32_t b = n;
+          if (i + 1 < k) {
+            b = (uint32_t)__builtin_ctz(mm) + 1;
+            mm &= mm - 1;
+          }
+          const uint64_t t = (uint64_t)img[L.o_pl + (row0 + b) * kRowW + p_ref] - img[L.o_pl + (row0 + a) * kRowW + p_ref];
+          s += t;
+          sq += t * t;
+          a = b;
+        }
+        const uint64_t D = s * s, N = (uint64_t)k * sq - D;  // exact under the R4 bounds
+        es.push_back({(N << 10) / D, k, m});
+        const uint32_t t = m | (m - 1);
+        const uint32_t nm = (uint32_t)((uint64_t)t + 1) | (uint32_t)((((~t & (0u - ~t)) - 1)) >> (__builtin_ctz(m) + 1));
+        if (nm <= m) break;
+        m = nm;
+      }
+    }
+    std::stable_sort(es.begin(), es.end(), [](const E& x, const E& y) {
+      if (x.cvq != y.cvq) return x.cvq < y.cvq;
+      if (x.k != y.k) return x.k < y.k;
+      return x.mask < y.mask;
+    });
+    for (const E& e : es) masks.push_back(e.mask);
+    off[f + 1] = (uint32_t)masks.size();
+  }
+  // profiles ordered by (capacity, gpcs, id) for the min-resource assignment
+  std::vector<uint32_t> ord(c->P);
+  for (uint32_t p = 0; p < c->P; ++p) ord[p] = p;
+  std::sort(ord.begin(), ord.end(), [&](uint32_t x, uint32_t y) {
+    const uint32_t cx = img[L.o_cap + x], cy = img[L.o_cap + y], gx = img[L.o_gpcs + x], gy = img[L.o_gpcs + y];
+    if (cx != cy) return cx < cy;
+    if (gx != gy) return gx < gy;
+    return x < y;
+  });
+  uint32_t po = 0;
+  for (uint32_t i = 0; i < c->P; ++i) po |= ord[i] << (4 * i);
+  DeviceGuard g(c->device);
+  CK(c->rank_off.ensure(off.size() * 4), "cudaMalloc(rank_off)");
+  CK(cudaMemcpy(c->rank_off.p, off.data(), off.size() * 4, cudaMemcpyHostToDevice), "upload rank_off");
+  CK(c->rank_mask.ensure(std::max<size_t>(1, masks.size()) * 4), "cudaMalloc(rank_mask)");
+  if (!masks.empty())
+    CK(cudaMemcpy(c->rank_mask.p, masks.data(), masks.size() * 4, cudaMemcpyHostToDevice), "upload rank_mask");
+  c->prof_order = po;
+  c->rank_kmax = k_max;
+  c->ranked = true;
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_ranked(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                           ffs_plan* d_out, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged || !c->ranked) return fail(c, FFS_ERR_STATE, "call ffs_rank_partitions after staging");
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  RankedArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.req = d_req;
+  a.slo = d_slo;
+  a.n_req = n_req;
+  a.n_nodes = c->n_nodes;
+  a.node_free = c->node_free.as<uint64_t>();
+  a.free_list = c->free_list.as<int32_t>();
+  a.rank_off = c->rank_off.as<uint32_t>();
+  a.rank_mask = c->rank_mask.as<uint32_t>();
+  a.prof_order = c->prof_order;
+  a.out = d_out;
+  CK(launch_ranked(a, (cudaStream_t)stream), "ranked kernel");
   return FFS_OK;
 }
 

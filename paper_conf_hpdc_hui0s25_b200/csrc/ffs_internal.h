@@ -89,4 +89,19 @@ cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const 
                            uint32_t n_slices, int32_t* victim, cudaStream_t st);
 cudaError_t run_int_peak(int sms, double* ops, double* seconds);
 
+struct RankedArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  uint32_t n_req, n_nodes;
+  const uint64_t* node_free;
+  const int32_t* free_list;
+  const uint32_t* rank_off;   // [F+1]
+  const uint32_t* rank_mask;  // ranked cut masks, per function contiguous
+  uint32_t prof_order;        // profiles by (capacity, gpcs, id): 4 bits each, first = low nibble
+  ffs_plan* out;
+};
+cudaError_t launch_ranked(const RankedArgs& a, cudaStream_t st);
+
 }  // namespace ffsk

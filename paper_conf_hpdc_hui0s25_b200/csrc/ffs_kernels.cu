@@ -1088,6 +1088,151 @@ cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const 
 }
 
 // ====================================================================================
+// K6 (NEXT-1): the paper's ranked first-fit walk, one warp per request
+// ====================================================================================
+// Lanes test 32 consecutive ranked partitions at once; the warp stops at the first
+// chunk with a supported partition and takes its lowest rank (ballot + ffs), which is
+// exactly the sequential first fit.
+struct RankedEval {
+  uint32_t k, e2e, bott, gpcs, cvq;
+  int prof[kMaxK];
+};
+
+__device__ __forceinline__ bool ranked_eval(const RankedArgs& A, uint32_t row0, uint32_t n, uint32_t mask,
+                                            uint64_t freeb, uint32_t B, RankedEval& out) {
+  const uint32_t* img = A.image;
+  const ImageLayout& L = A.lay;
+  const uint32_t k = __popc(mask) + 1;
+  uint32_t bnd[kMaxK + 1], mem[kMaxK];
+  bnd[0] = 0;
+  uint32_t m = mask, X = 0;
+  for (uint32_t i = 1; i < k; ++i) {
+    const int j = __ffs(m) - 1;
+    m &= m - 1;
+    bnd[i] = j + 1;
+    X += img[L.o_xf + row0 + j];
+  }
+  bnd[k] = n;
+  for (uint32_t i = 0; i < k; ++i) mem[i] = img[L.o_pm + row0 + bnd[i + 1]] - img[L.o_pm + row0 + bnd[i]];
+  // min-resource greedy: stages by descending memory (ties: lower stage), each takes the
+  // first profile in (capacity, gpcs, id) order with a free slice left that holds it
+  uint32_t left[kP];
+#pragma unroll
+  for (int p = 0; p < kP; ++p) left[p] = (uint32_t)(freeb >> (8 * p)) & 255u;
+  uint32_t done = 0;
+  for (uint32_t step = 0; step < k; ++step) {
+    int s = -1;
+    for (uint32_t i = 0; i < k; ++i)
+      if (!((done >> i) & 1u) && (s < 0 || mem[i] > mem[s])) s = (int)i;
+    done |= 1u << s;
+    int got = -1;
+#pragma unroll
+    for (int oi = 0; oi < kP; ++oi) {
+      const int p = (int)((A.prof_order >> (4 * oi)) & 15u);
+      bool ok = false;
+#pragma unroll
+      for (int q = 0; q < kP; ++q)
+        if (q == p) ok = left[q] > 0;
+      if (got < 0 && ok && mem[s] <= img[L.o_cap + p]) {
+        got = p;
+#pragma unroll
+        for (int q = 0; q < kP; ++q)
+          if (q == p) left[q]--;
+      }
+    }
+    if (got < 0) return false;
+    out.prof[s] = got;
+  }
+  uint64_t St = 0, Sq = 0;
+  uint32_t bott = 0, g = 0;
+  for (uint32_t i = 0; i < k; ++i) {
+    const int p = out.prof[i];
+    const uint32_t t = img[L.o_pl + (row0 + bnd[i + 1]) * kRowW + p] - img[L.o_pl + (row0 + bnd[i]) * kRowW + p];
+    St += t;
+    Sq += (uint64_t)t * t;
+    bott = t > bott ? t : bott;
+    g += img[L.o_gpcs + p];
+  }
+  if (St + X > (uint64_t)B) return false;
+  out.k = k;
+  out.e2e = (uint32_t)(St + X);
+  out.bott = bott;
+  out.gpcs = g;
+  const uint64_t D = St * St, N = (uint64_t)k * Sq - D;
+  out.cvq = (uint32_t)((N << 10) / D);
+  return true;
+}
+
+constexpr int kRkT = 128;
+__global__ void __launch_bounds__(kRkT) k_plan_ranked(const __grid_constant__ RankedArgs A) {
+  const uint32_t r = (blockIdx.x * kRkT + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (r >= A.n_req) return;
+  const uint32_t* img = A.image;
+  const ImageLayout& L = A.lay;
+  const ffs_request q = A.req[r];
+  ffs_plan pl;
+  pl.key = (int64_t)kKeyNone;
+  pl.status = FFS_PLAN_BAD_REQ;
+  pl.k = pl.cut_mask = pl.e2e_us = pl.bottleneck_us = pl.gpcs = pl.cvq = 0;
+#pragma unroll
+  for (int i = 0; i < kMaxK; ++i) {
+    pl.prof[i] = 0xFF;
+    pl.slice[i] = -1;
+  }
+  pl.victim = -1;
+  if (q.func < L.F && q.node < A.n_nodes) {
+    pl.status = FFS_PLAN_INFEASIBLE;
+    const uint32_t* fd = img + L.o_fdesc + 4 * q.func;
+    const uint32_t row0 = fd[0], n = fd[1], B = A.slo[r];
+    const uint64_t freeb = A.node_free[q.node];
+    const uint32_t off = A.rank_off[q.func], cnt = A.rank_off[q.func + 1] - off;
+    for (uint32_t base = 0; base < cnt; base += 32) {
+      const uint32_t j = base + lane;
+      RankedEval ev;
+      uint32_t mask = 0;
+      bool ok = false;
+      if (j < cnt) {
+        mask = A.rank_mask[off + j];
+        ok = ranked_eval(A, row0, n, mask, freeb, B, ev);
+      }
+      const uint32_t bal = __ballot_sync(0xffffffffu, ok);
+      if (bal) {
+        const uint32_t w = __ffs(bal) - 1;
+        if (lane == w) {
+          pl.status = FFS_PLAN_OK;
+          pl.key = (int64_t)(base + w);
+          pl.k = ev.k;
+          pl.cut_mask = mask;
+          pl.e2e_us = ev.e2e;
+          pl.bottleneck_us = ev.bott;
+          pl.gpcs = ev.gpcs;
+          pl.cvq = ev.cvq;
+          uint32_t used[kP] = {0, 0, 0, 0, 0};
+          for (uint32_t i = 0; i < ev.k; ++i) {
+            const int p = ev.prof[i];
+            pl.prof[i] = (uint8_t)p;
+            uint32_t u = 0;
+#pragma unroll
+            for (int x = 0; x < kP; ++x)
+              if (x == p) u = used[x]++;
+            pl.slice[i] = A.free_list[((uint64_t)q.node * 8 + p) * 8 + u];  // R11 binding
+          }
+          A.out[r] = pl;
+        }
+        return;
+      }
+    }
+  }
+  if (lane == 0) A.out[r] = pl;
+}
+
+cudaError_t launch_ranked(const RankedArgs& a, cudaStream_t st) {
+  const uint64_t threads = (uint64_t)a.n_req * 32;
+  k_plan_ranked<<<(unsigned)((threads + kRkT - 1) / kRkT), kRkT, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+// ====================================================================================
 // K5: integer issue-rate microbenchmark (roofline denominator)
 // ====================================================================================
 constexpr int kPeakIters = 4096;

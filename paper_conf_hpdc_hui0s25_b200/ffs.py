@@ -60,6 +60,8 @@ _sig = {
     "ffs_evict_scores": ([_vp, _vp, _u32, _u64, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
+    "ffs_rank_partitions": ([_vp, _u32, _u32], _i32),
+    "ffs_plan_ranked": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
     "ffs_segment_times": ([_vp, C.POINTER(C.c_float)], _i32),
     "ffs_debug_filter_misses": ([_vp, C.POINTER(C.c_uint64)], _i32),
@@ -214,6 +216,18 @@ class Planner:
                                            _ptr(tick_off), _ptr(score), int(tick_off.numel() - 1), _ptr(victim),
                                            _stream(stream)))
         return victim
+
+    # ---- NEXT-1: ranked first-fit -----------------------------------------------
+    def rank_partitions(self, k_max: int, p_ref: int) -> None:
+        self._check(_lib.ffs_rank_partitions(self._h, int(k_max), int(p_ref)))
+
+    def plan_ranked(self, req, slo, out=None, stream=None):
+        import torch
+        n = int(slo.numel())
+        if out is None:
+            out = torch.empty((n, PLAN_DTYPE.itemsize), dtype=torch.uint8, device=slo.device)
+        self._check(_lib.ffs_plan_ranked(self._h, _ptr(req), _ptr(slo), n, _ptr(out), _stream(stream)))
+        return out
 
     # ---- measurement ---------------------------------------------------------------------
     def int_peak(self) -> tuple[float, float]:

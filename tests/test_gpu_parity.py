@@ -249,3 +249,35 @@ def test_decode_victims_single_snapshot(F, planner):
     s_o, _ = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
     v_o = oracle.victim(prob, o["status"], wl.inst, s_o)
     np.testing.assert_array_equal(plans["victim"], v_o)
+
+
+# ---- NEXT-1: ranked first-fit ----------------------------------------------
+def run_ranked(F, planner, prob, p_ref=4):
+    planner.stage(prob)
+    planner.rank_partitions(prob.k_max, p_ref)
+    req, slo = F.to_device(prob)
+    out = planner.plan_ranked(req, slo)
+    torch.cuda.synchronize()
+    return F.plans_to_numpy(out)
+
+
+@pytest.mark.parametrize("seed", range(1000, 1016))
+def test_ranked_tiny_random(F, planner, seed):
+    prob = random_tiny(seed, n_max=5, K=4)
+    for p_ref in (0, 4):
+        p = run_ranked(F, planner, prob, p_ref)
+        assert_plans_equal(p, oracle.plan_ranked(prob, p_ref=p_ref))
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_ranked_configs(F, planner, cfg):
+    prob = {"C1": W.config1, "C2": W.config2, "C3": lambda: W.config3(R=8192)}[cfg]()
+    p = run_ranked(F, planner, prob)
+    assert_plans_equal(p, oracle.plan_ranked(prob))
+
+
+def test_ranked_c5_sample(F, planner):
+    prob = W.config5()
+    p = run_ranked(F, planner, prob)
+    idx = np.arange(0, prob.R, 1021)
+    assert_plans_equal(p, oracle.plan_ranked(prob.subset(idx)), idx)
