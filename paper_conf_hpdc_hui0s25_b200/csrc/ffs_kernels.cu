@@ -431,31 +431,36 @@ __device__ __forceinline__ f2 f2fma(f2 a, f2 b, f2 c) {
   return d;
 }
 
-struct Geo4 {
-  int bnd[5];
-  uint32_t memst[4];
+template <int KS>
+struct Geo {
+  int bnd[KS + 1];
+  uint32_t memst[KS];
   uint32_t X;
   float blim;
 };
+typedef Geo<4> Geo4;
 
-__device__ __forceinline__ void geo4(const SearchState<4>& c, uint32_t mask, Geo4& g) {
+template <int KS>
+__device__ __forceinline__ void geo(const SearchState<KS>& c, uint32_t mask, Geo<KS>& g) {
   g.bnd[0] = 0;
   uint32_t m = mask, X = 0;
 #pragma unroll
-  for (int i = 0; i < 3; ++i) {
+  for (int i = 0; i < KS - 1; ++i) {
     const int j = __ffs(m) - 1;
     m &= m - 1;
     g.bnd[i + 1] = j + 1;
     X += c.sm[c.o_xf + c.row0 + j];
   }
-  g.bnd[4] = c.n;
+  g.bnd[KS] = c.n;
   g.X = X;
 #pragma unroll
-  for (int i = 0; i < 4; ++i) g.memst[i] = c.sm[c.o_pm + c.row0 + g.bnd[i + 1]] - c.sm[c.o_pm + c.row0 + g.bnd[i]];
+  for (int i = 0; i < KS; ++i) g.memst[i] = c.sm[c.o_pm + c.row0 + g.bnd[i + 1]] - c.sm[c.o_pm + c.row0 + g.bnd[i]];
   g.blim = (X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
 }
+__device__ __forceinline__ void geo4(const SearchState<4>& c, uint32_t mask, Geo4& g) { geo<4>(c, mask, g); }
 
-__device__ __forceinline__ void geo_lat(const SearchState<4>& c, const Geo4& g, int s, float (&f)[kP]) {
+template <int KS>
+__device__ __forceinline__ void geo_lat(const SearchState<KS>& c, const Geo<KS>& g, int s, float (&f)[kP]) {
   const uint32_t ra = c.o_pl + (c.row0 + g.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + g.bnd[s + 1]) * kRowW;
   const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
   const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
@@ -464,6 +469,100 @@ __device__ __forceinline__ void geo_lat(const SearchState<4>& c, const Geo4& g, 
   f[2] = __uint2float_rn(lb.z - la.z);
   f[3] = __uint2float_rn(lb.w - la.w);
   f[4] = __uint2float_rn(c.sm[rb + 4] - c.sm[ra + 4]);
+}
+
+// Copy half h's geometry into the state and run the exact path over the flagged blocks.
+template <int KS, bool VERIFY>
+__device__ __forceinline__ void pair_rescan(SearchState<KS>& c, const Geo<KS>& G, uint32_t pend, uint32_t all,
+                                            uint64_t idx_shift, unsigned long long* misses) {
+  constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
+#pragma unroll
+  for (int i = 0; i <= KS; ++i) c.bnd[i] = G.bnd[i];
+#pragma unroll
+  for (int i = 0; i < KS; ++i) c.memst[i] = G.memst[i];
+  c.X = G.X;
+  c.idx_base += idx_shift;
+  for (uint32_t todo = all; todo;) {
+    const int b = __ffs(todo) - 1;
+    todo &= todo - 1;
+    if constexpr (KS == 3) c.pd[0] = b;
+    if constexpr (KS == 4) {
+      c.pd[0] = b / kP;
+      c.pd[1] = b - kP * (b / kP);
+    }
+    const uint32_t fast = ((pend >> b) & 1u) ? kAll : 0u;
+    handle_hits<KS, VERIFY>(c, kAll, fast, misses);
+  }
+  c.idx_base -= idx_shift;
+}
+
+// KS = 3, two consecutive masks per thread in f32x2 lanes, every level unrolled (125
+// candidates per mask, ~8 KB of SASS) and every table in registers.
+template <bool VERIFY>
+__device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint32_t maskB, bool haveB,
+                                         unsigned long long* misses) {
+  const float INF = __int_as_float(0x7f800000);
+  Geo<3> G[2];
+  geo<3>(c, maskA, G[0]);
+  geo<3>(c, maskB, G[1]);
+  if (!haveB) G[1].blim = -1.f;
+  const float al = c.alpha, one_m_a = 1.f - c.alpha;
+  f2 v0[kP], v1[2][kP], sl2[3][kP], na0[kP], a1[kP], t2[kP], cc[kP];
+  {
+    float f[2][3][kP];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int s = 0; s < 3; ++s) geo_lat<3>(c, G[h], s, f[h][s]);
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+      const uint32_t cap = c.sm[c.o_cap + x];
+      float v[2][3][3];
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 3; ++s)
+#pragma unroll
+          for (int m = 0; m <= s; ++m) v[h][s][m] = (G[h].memst[s] <= cap && fr > (uint32_t)m) ? f[h][s][x] : INF;
+      v0[x] = f2pack(v[0][0][0], v[1][0][0]);
+      v1[0][x] = f2pack(v[0][1][0], v[1][1][0]);
+      v1[1][x] = f2pack(v[0][1][1], v[1][1][1]);
+#pragma unroll
+      for (int m = 0; m < 3; ++m) sl2[m][x] = f2pack(G[0].blim - v[0][2][m], G[1].blim - v[1][2][m]);
+      na0[x] = f2pack(-al * (f[0][0][x] * f[0][0][x]), -al * (f[1][0][x] * f[1][0][x]));
+      a1[x] = f2pack(al * (f[0][1][x] * f[0][1][x]), al * (f[1][1][x] * f[1][1][x]));
+      t2[x] = f2pack(f[0][2][x] + f[0][2][x], f[1][2][x] + f[1][2][x]);
+      cc[x] = f2pack(one_m_a * (f[0][2][x] * f[0][2][x]), one_m_a * (f[1][2][x] * f[1][2][x]));
+    }
+  }
+  uint32_t pendA = 0, pendB = 0;
+#pragma unroll
+  for (int d0 = 0; d0 < kP; ++d0) {
+    const f2 S1 = v0[d0], NL1 = na0[d0];
+    uint32_t accA = ~0u, accB = ~0u;
+#pragma unroll
+    for (int q = 0; q < kP; ++q) {
+      const f2 S2 = f2add(S1, v1[q == d0][q]);
+      const f2 NL2 = f2sub(NL1, a1[q]);
+      const f2 U = f2fma(S2, S2, NL2);
+#pragma unroll
+      for (int p = 0; p < kP; ++p) {
+        const f2 z = f2add(f2fma(S2, t2[p], cc[p]), U);
+        const f2 d2 = f2sub(sl2[(p == d0) + (p == q)][p], S2);
+        uint32_t zl, zh, dl, dh;
+        f2bits(z, zl, zh);
+        f2bits(d2, dl, dh);
+        accA &= zl | dl;
+        accB &= zh | dh;
+      }
+    }
+    pendA |= ((accA >> 31) ^ 1u) << d0;
+    pendB |= ((accB >> 31) ^ 1u) << d0;
+  }
+  constexpr uint32_t kAllB = (1u << kP) - 1;
+  pair_rescan<3, VERIFY>(c, G[0], pendA, VERIFY ? kAllB : pendA, 0, misses);
+  if (haveB) pair_rescan<3, VERIFY>(c, G[1], pendB, VERIFY ? kAllB : pendB, 125, misses);
 }
 
 struct Win2 {
@@ -574,27 +673,8 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
   }
   // rare exact path, one half at a time (geometry copied into the state)
   constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
-#pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    const uint32_t pend = h ? pendB : pendA;
-    const uint32_t all = (h && !haveB) ? 0u : (VERIFY ? kAll : pend);
-    if (!all) continue;
-#pragma unroll
-    for (int i = 0; i < 5; ++i) c.bnd[i] = G[h].bnd[i];
-#pragma unroll
-    for (int i = 0; i < 4; ++i) c.memst[i] = G[h].memst[i];
-    c.X = G[h].X;
-    if (h) c.idx_base += 625;
-    for (uint32_t todo = all; todo;) {
-      const int b = __ffs(todo) - 1;
-      todo &= todo - 1;
-      c.pd[0] = b / kP;
-      c.pd[1] = b - kP * (b / kP);
-      const uint32_t fast = ((pend >> b) & 1u) ? kAll : 0u;
-      handle_hits<4, VERIFY>(c, kAll, fast, misses);
-    }
-    if (h) c.idx_base -= 625;
-  }
+  pair_rescan<4, VERIFY>(c, G[0], pendA, VERIFY ? kAll : pendA, 0, misses);
+  if (haveB) pair_rescan<4, VERIFY>(c, G[1], pendB, VERIFY ? kAll : pendB, 625, misses);
 }
 
 template <int KS, bool VERIFY>
@@ -768,11 +848,12 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
   load_request(m);
   while (true) {
     uint32_t step = 1;
-    if constexpr (KS == 4) {
-      // two consecutive masks of the same request per iteration (ks4_pair)
+    if constexpr (KS == 3 || KS == 4) {
+      // two consecutive masks of the same request per iteration (ks3_pair / ks4_pair)
       const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
       const uint32_t maskB = haveB ? gosper_next(mask) : mask;
-      ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<f2*>(rows), A.misses);
+      if constexpr (KS == 4) ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<f2*>(rows), A.misses);
+      else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses);
       if (haveB) {
         step = 2;
         mask = maskB;
