@@ -63,6 +63,8 @@ def lib():
             _lib.oracle_plan.restype = C.c_int
             _lib.oracle_plan_ranked.argtypes = [C.POINTER(_PlanArgs), C.c_int, C.c_int]
             _lib.oracle_plan_ranked.restype = C.c_int
+            _lib.oracle_plan_joint.argtypes = [C.POINTER(_PlanArgs)]
+            _lib.oracle_plan_joint.restype = C.c_int
             _lib.oracle_evict.restype = None
             _lib.oracle_victim.restype = None
     return _lib
@@ -146,6 +148,16 @@ def plan_ranked(prob, p_ref: int | None = None, k_max: int | None = None, thread
     rc = lib().oracle_plan_ranked(C.byref(h.args), int(p_ref), int(threads))
     if rc != 0:
         raise ValueError("oracle_plan_ranked rejected its arguments")
+    return h.out
+
+
+def plan_joint(prob, k_max: int | None = None) -> dict:
+    """NEXT-2: joint commit of the batch, node by node in ascending adjusted deadline,
+    each plan taking its slices (ffs_oracle.c: oracle_plan_joint).  Single-threaded."""
+    h = _Held(prob, int(prob.k_max if k_max is None else k_max), False)
+    rc = lib().oracle_plan_joint(C.byref(h.args))
+    if rc != 0:
+        raise ValueError("oracle_plan_joint rejected its arguments")
     return h.out
 
 

@@ -187,7 +187,11 @@ static uint64_t binom(int n, int r) {
     return c;
 }
 
-static void plan_one(const oracle_plan_args *a, int r) {
+static void plan_one_busy(const oracle_plan_args *a, int r, const uint8_t *busy);
+static void plan_one(const oracle_plan_args *a, int r) { plan_one_busy(a, r, a->sl_busy); }
+
+/* plan request r against the slice states `busy` (free = !busy) */
+static void plan_one_busy(const oracle_plan_args *a, int r, const uint8_t *busy) {
     int64_t *key = &a->key[r];
     a->status[r] = PLAN_BAD_REQ;
     *key = KEY_NONE;
@@ -218,7 +222,7 @@ static void plan_one(const oracle_plan_args *a, int r) {
     s.best = KEY_NONE;
     /* free slices of each profile in the request's node (R10) */
     for (int i = 0; i < a->n_slices; i++)
-        if (a->sl_node[i] == s.v && !a->sl_busy[i]) s.free_cnt[a->sl_prof[i]]++;
+        if (a->sl_node[i] == s.v && !busy[i]) s.free_cnt[a->sl_prof[i]]++;
 
     int kmax = a->k_max < s.n ? a->k_max : s.n;
     for (int k = 1; k <= kmax; k++) {
@@ -271,7 +275,7 @@ static void plan_one(const oracle_plan_args *a, int r) {
     for (int i = 0; i < s.best_k; i++) {
         a->prof[(size_t)r * 8 + i] = (uint8_t)s.best_prof[i];
         for (int x = 0; x < a->n_slices; x++) {
-            if (a->sl_node[x] != s.v || a->sl_busy[x] || a->sl_prof[x] != s.best_prof[i]) continue;
+            if (a->sl_node[x] != s.v || busy[x] || a->sl_prof[x] != s.best_prof[i]) continue;
             int taken = 0;
             for (int j = 0; j < i; j++)
                 if (a->slice[(size_t)r * 8 + j] == x) taken = 1;
@@ -612,5 +616,58 @@ int oracle_plan_ranked(const oracle_plan_args *a, int p_ref, int n_threads) {
     for (int i = 0; i < n_threads; i++) pthread_join(th[i], NULL);
     free(th);
     free(wa);
+    return 0;
+}
+
+/* ---- NEXT-2: joint commit of a batch ----------------------------------
+ * Requests of a node are served one at a time in ascending adjusted deadline
+ * ("deadlines subtracted by estimated execution and instance load times"):
+ * adj_r = B_r - load_f - t_exec_f, t_exec_f = the function's fastest 1-stage latency
+ * (min over profiles of the sum of its component latencies) -- DESIGN.md R28; ties by
+ * request index.  Each request is planned exactly as oracle_plan against the slices
+ * still free, and a plan takes its bound slices (R29).  Sequential, plain. */
+typedef struct {
+    int64_t adj;
+    int node, r;
+} joint_item;
+
+static int cmp_joint(const void *x, const void *y) {
+    const joint_item *a = (const joint_item *)x, *b = (const joint_item *)y;
+    if (a->node != b->node) return a->node < b->node ? -1 : 1;
+    if (a->adj != b->adj) return a->adj < b->adj ? -1 : 1;
+    return a->r < b->r ? -1 : (a->r > b->r);
+}
+
+int oracle_plan_joint(const oracle_plan_args *a) {
+    if (!a || a->P < 1 || a->P > ORACLE_MAX_P || a->k_max < 1 || a->k_max > ORACLE_MAX_STAGES) return -1;
+    uint8_t *busy = (uint8_t *)malloc((size_t)(a->n_slices > 0 ? a->n_slices : 1));
+    for (int i = 0; i < a->n_slices; i++) busy[i] = a->sl_busy[i];
+    joint_item *it = (joint_item *)malloc(sizeof(joint_item) * (size_t)(a->R > 0 ? a->R : 1));
+    for (int r = 0; r < a->R; r++) {
+        int f = (int)a->req_func[r];
+        int64_t adj = (int64_t)a->req_slo_us[r];
+        if (f < a->F) {
+            int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+            uint64_t fast = UINT64_MAX;
+            for (int p = 0; p < a->P; p++) {
+                uint64_t t = 0;
+                for (int c = 0; c < n; c++) t += lat_of(a, f, c, p);
+                if (t < fast) fast = t;
+            }
+            adj -= (int64_t)a->load_us[f] + (int64_t)fast;
+        }
+        it[r].adj = adj;
+        it[r].node = (int)a->req_node[r];
+        it[r].r = r;
+    }
+    qsort(it, (size_t)a->R, sizeof(joint_item), cmp_joint);
+    for (int i = 0; i < a->R; i++) {
+        int r = it[i].r;
+        plan_one_busy(a, r, busy);
+        if (a->status[r] == PLAN_OK)
+            for (int j = 0; j < a->k[r]; j++) busy[a->slice[(size_t)r * 8 + j]] = 1;
+    }
+    free(it);
+    free(busy);
     return 0;
 }

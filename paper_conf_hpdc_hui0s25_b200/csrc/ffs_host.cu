@@ -280,7 +280,14 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
 
   DeviceGuard g(c->device);
   CK(c->image.ensure((size_t)L.words * 4), "cudaMalloc(image)");
-  CK(cudaMemcpy(c->image.p, img.data(), (size_t)L.words * 4, cudaMemcpyHostToDevice), "upload image");
+  {  // device copy: the prefix-latency rows as exact fp32 (every prefix < 2^24, checked above)
+    std::vector<uint32_t> up(img);
+    for (uint32_t i = L.o_pl; i < L.o_pl + rows * kRowW; ++i) {
+      const float f = (float)img[i];
+      std::memcpy(&up[i], &f, 4);
+    }
+    CK(cudaMemcpy(c->image.p, up.data(), (size_t)L.words * 4, cudaMemcpyHostToDevice), "upload image");
+  }
   CK(c->node_free.ensure(NN * 8), "cudaMalloc(node_free)");
   CK(cudaMemcpy(c->node_free.p, node_free.data(), NN * 8, cudaMemcpyHostToDevice), "upload node_free");
   CK(c->free_list.ensure(free_list.size() * 4), "cudaMalloc(free_list)");

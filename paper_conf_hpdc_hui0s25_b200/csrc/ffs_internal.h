@@ -35,7 +35,7 @@ struct ImageLayout {
   uint32_t o_binom;   // [33][8] u32 C(c, i), c <= 32, i <= 7
   uint32_t o_offk;    // [33][10] u64 (word pairs) offk[n][k] = sum_{k'<k} C(n-1,k'-1) P^k'
   uint32_t o_fdesc;   // [F][4] u32 {row0, n, load_us, mem_total}
-  uint32_t o_pl;      // [rows][8] u32 PL[row0+i][p] = sum_{c<i} lat[c][p]  (16-byte aligned)
+  uint32_t o_pl;      // [rows][8] fp32 bits: PL[row0+i][p] = sum_{c<i} lat[c][p], exact (< 2^24), 16-B aligned
   uint32_t o_pm;      // [rows] u32 PM[row0+i] = sum_{c<i} mem[c]
   uint32_t o_xf;      // [rows] u32 xfer cost of a cut after component i (row0+i)
 };

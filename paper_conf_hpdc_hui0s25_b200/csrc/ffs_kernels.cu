@@ -21,6 +21,12 @@ namespace ffsk {
 __device__ __forceinline__ uint64_t img_u64(const uint32_t* w, uint32_t o) {
   return (uint64_t)w[o] | ((uint64_t)w[o + 1] << 32);
 }
+// The prefix-latency table PL is stored as fp32: every prefix is an integer < 2^24 (the
+// ffs_stage_tables bound), so values and differences are exact.  Integer uses convert back.
+__device__ __forceinline__ float plf(const uint32_t* w, uint32_t o) { return __uint_as_float(w[o]); }
+__device__ __forceinline__ uint32_t pl_diff(const uint32_t* w, uint32_t ob, uint32_t oa) {
+  return __float2uint_rn(plf(w, ob) - plf(w, oa));
+}
 __device__ __forceinline__ uint32_t binom(const uint32_t* img, const ImageLayout& L, int c, int i) {
   return img[L.o_binom + c * 8 + i];  // C(c, i), 0 when c < i
 }
@@ -203,7 +209,7 @@ __device__ __forceinline__ void exact_eval(SearchState<KS>& c, int q, int p, boo
   for (int i = 0; i < KS; ++i) {
     const int pr = prof[i];
     const uint32_t a = (c.row0 + c.bnd[i]) * kRowW, b = (c.row0 + c.bnd[i + 1]) * kRowW;
-    const uint32_t t = c.sm[c.o_pl + b + pr] - c.sm[c.o_pl + a + pr];
+    const uint32_t t = pl_diff(c.sm, c.o_pl + b + pr, c.o_pl + a + pr);
     ok &= c.memst[i] <= c.sm[c.o_cap + pr];
     St += t;
     Sq += (uint64_t)t * t;
@@ -293,7 +299,7 @@ __device__ __forceinline__ void outer_level(SearchState<KS>& c, float S, float Q
     const uint32_t a = c.o_pl + (c.row0 + c.bnd[L]) * kRowW, b = c.o_pl + (c.row0 + c.bnd[L + 1]) * kRowW;
 #pragma unroll 1
     for (int p = 0; p < kP; ++p) {
-      const uint32_t t = c.sm[b + p] - c.sm[a + p];
+      const uint32_t t = pl_diff(c.sm, b + p, a + p);
       const uint32_t cw2 = cw - (1u << (5 * p));
       const bool ok = (c.memst[L] <= c.sm[c.o_cap + p]) && ((cw2 >> (5 * p + 4)) & 1u);
       const float tf = ok ? __uint2float_rn(t) : INF;
@@ -308,12 +314,12 @@ template <int KS>
 __device__ __forceinline__ void load_stage(const SearchState<KS>& c, int s, float (&tf)[kP], float (&sq)[kP]) {
   const float INF = __int_as_float(0x7f800000);
   const uint32_t a = c.o_pl + (c.row0 + c.bnd[s]) * kRowW, b = c.o_pl + (c.row0 + c.bnd[s + 1]) * kRowW;
-  const uint4 la = *reinterpret_cast<const uint4*>(c.sm + a);
-  const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + b);
-  const uint32_t t[kP] = {lb.x - la.x, lb.y - la.y, lb.z - la.z, lb.w - la.w, c.sm[b + 4] - c.sm[a + 4]};
+  const float4 la = *reinterpret_cast<const float4*>(c.sm + a);
+  const float4 lb = *reinterpret_cast<const float4*>(c.sm + b);
+  const float t[kP] = {lb.x - la.x, lb.y - la.y, lb.z - la.z, lb.w - la.w, plf(c.sm, b + 4) - plf(c.sm, a + 4)};
 #pragma unroll
   for (int p = 0; p < kP; ++p) {
-    const float f = __uint2float_rn(t[p]);
+    const float f = t[p];
     tf[p] = (c.memst[s] <= c.sm[c.o_cap + p]) ? f : INF;
     sq[p] = f * f;
   }
@@ -343,13 +349,13 @@ struct Tables {
 template <int KS>
 __device__ __forceinline__ void stage_lat(const SearchState<KS>& c, int s, float (&f)[kP]) {
   const uint32_t ra = c.o_pl + (c.row0 + c.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + c.bnd[s + 1]) * kRowW;
-  const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
-  const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
-  f[0] = __uint2float_rn(lb.x - la.x);
-  f[1] = __uint2float_rn(lb.y - la.y);
-  f[2] = __uint2float_rn(lb.z - la.z);
-  f[3] = __uint2float_rn(lb.w - la.w);
-  f[4] = __uint2float_rn(c.sm[rb + 4] - c.sm[ra + 4]);
+  const float4 la = *reinterpret_cast<const float4*>(c.sm + ra);
+  const float4 lb = *reinterpret_cast<const float4*>(c.sm + rb);
+  f[0] = lb.x - la.x;
+  f[1] = lb.y - la.y;
+  f[2] = lb.z - la.z;
+  f[3] = lb.w - la.w;
+  f[4] = plf(c.sm, rb + 4) - plf(c.sm, ra + 4);
 }
 
 template <int KS>
@@ -462,13 +468,13 @@ __device__ __forceinline__ void geo4(const SearchState<4>& c, uint32_t mask, Geo
 template <int KS>
 __device__ __forceinline__ void geo_lat(const SearchState<KS>& c, const Geo<KS>& g, int s, float (&f)[kP]) {
   const uint32_t ra = c.o_pl + (c.row0 + g.bnd[s]) * kRowW, rb = c.o_pl + (c.row0 + g.bnd[s + 1]) * kRowW;
-  const uint4 la = *reinterpret_cast<const uint4*>(c.sm + ra);
-  const uint4 lb = *reinterpret_cast<const uint4*>(c.sm + rb);
-  f[0] = __uint2float_rn(lb.x - la.x);
-  f[1] = __uint2float_rn(lb.y - la.y);
-  f[2] = __uint2float_rn(lb.z - la.z);
-  f[3] = __uint2float_rn(lb.w - la.w);
-  f[4] = __uint2float_rn(c.sm[rb + 4] - c.sm[ra + 4]);
+  const float4 la = *reinterpret_cast<const float4*>(c.sm + ra);
+  const float4 lb = *reinterpret_cast<const float4*>(c.sm + rb);
+  f[0] = lb.x - la.x;
+  f[1] = lb.y - la.y;
+  f[2] = lb.z - la.z;
+  f[3] = lb.w - la.w;
+  f[4] = plf(c.sm, rb + 4) - plf(c.sm, ra + 4);
 }
 
 // Copy half h's geometry into the state and run the exact path over the flagged blocks.
@@ -939,7 +945,7 @@ __device__ __forceinline__ bool victim_ok(const uint32_t* img, const ImageLayout
   const uint32_t* fd = img + L.o_fdesc + 4 * f;
   if (fd[3] > img[L.o_cap + p]) return false;  // time-sharing instances are non-pipeline
   const uint32_t row0 = fd[0], n = fd[1];
-  const uint64_t lat = (uint64_t)img[L.o_pl + (row0 + n) * kRowW + p] - img[L.o_pl + row0 * kRowW + p];
+  const uint64_t lat = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
   return lat + fd[2] <= B;  // execution + reload within the budget
 }
 
@@ -1011,7 +1017,7 @@ __global__ void k_decode(const __grid_constant__ DecodeArgs A) {
           e2e += img[L.o_xf + row0 + j];
         }
         const int p = prof[i];
-        const uint32_t t = img[L.o_pl + (row0 + b) * kRowW + p] - img[L.o_pl + (row0 + a) * kRowW + p];
+        const uint32_t t = pl_diff(img, L.o_pl + (row0 + b) * kRowW + p, L.o_pl + (row0 + a) * kRowW + p);
         e2e += t;
         bott = t > bott ? t : bott;
         g += img[L.o_gpcs + p];
@@ -1111,7 +1117,7 @@ __device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const I
   uint32_t ok = 0;
 #pragma unroll
   for (int p = 0; p < kP; ++p) {
-    const uint64_t lat = (uint64_t)img[L.o_pl + (row0 + n) * kRowW + p] - img[L.o_pl + row0 * kRowW + p];
+    const uint64_t lat = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
     if (fd[3] <= img[L.o_cap + p] && lat + fd[2] <= B) ok |= 1u << p;
   }
   return ok;
@@ -1228,7 +1234,7 @@ __device__ __forceinline__ bool ranked_eval(const RankedArgs& A, uint32_t row0, 
   uint32_t bott = 0, g = 0;
   for (uint32_t i = 0; i < k; ++i) {
     const int p = out.prof[i];
-    const uint32_t t = img[L.o_pl + (row0 + bnd[i + 1]) * kRowW + p] - img[L.o_pl + (row0 + bnd[i]) * kRowW + p];
+    const uint32_t t = pl_diff(img, L.o_pl + (row0 + bnd[i + 1]) * kRowW + p, L.o_pl + (row0 + bnd[i]) * kRowW + p);
     St += t;
     Sq += (uint64_t)t * t;
     bott = t > bott ? t : bott;
