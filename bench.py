@@ -233,6 +233,25 @@ def run_ranked(pl, prob, req, slo, steps: int, warmup: int, flush):
             "ok_frac": float((p["status"] == 0).mean()), "multi_stage_frac": float(((p["status"] == 0) & (p["k"] > 1)).mean())}
 
 
+def run_joint(pl, prob, req, slo):
+    """NEXT-2 (joint commit in adjusted-deadline order) on the same batch:
+    one call, wall/event time, rounds."""
+    import torch
+    out = torch.empty((prob.R, 80), dtype=torch.uint8, device="cuda")
+    pl.plan_joint(req, slo, prob.k_max, out=out)  # warm-up
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    _, rounds = pl.plan_joint(req, slo, prob.k_max, out=out)
+    b.record()
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b)
+    from paper_conf_hpdc_hui0s25_b200 import ffs
+    p = ffs.plans_to_numpy(out)
+    return {"metric": "joint_commit_plans_per_s", "value": prob.R / (ms * 1e-3), "unit": "plans/s", "ms": ms,
+            "rounds": rounds, "ok_frac": float((p["status"] == 0).mean())}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -367,6 +386,9 @@ def main():
     ranked = None
     if world == 1 and not args.no_c4:
         ranked = run_ranked(pl, prob, req, slo, args.steps, args.warmup, flush)
+    joint = None
+    if world == 1 and not args.no_c4:
+        joint = run_joint(pl, prob, req, slo)
     c4 = None
     if world == 1 and not args.no_c4:
         c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
@@ -396,6 +418,7 @@ def main():
             "cpu_baseline": cpu,
             "eviction_c4": c4,
             "ranked_first_fit": ranked,
+            "joint_commit": joint,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

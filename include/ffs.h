@@ -252,6 +252,16 @@ ffs_status ffs_rank_partitions(ffs_ctx *ctx, uint32_t k_max, uint32_t p_ref);
 ffs_status ffs_plan_ranked(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
                            ffs_plan *d_out, void *stream);
 
+/* ---- NEXT-2: joint commit of the batch ---------------------------------
+ * The requests of each node are served one at a time in ascending adjusted deadline
+ * (budget - reload time - fastest 1-stage latency, ties by index; R28), each
+ * planned as ffs_plan_batch would against the slices still free and taking the slices
+ * its plan binds (R29), so the batch's plans are jointly feasible.  Computed in monotone
+ * rounds on the GPU (§4.6).  Uses context scratch; synchronous on `stream` (one host
+ * read of two counters per round).  Errors as ffs_plan_keys. */
+ffs_status ffs_plan_joint(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                          uint32_t k_max, ffs_plan *d_out, uint32_t *rounds, void *stream);
+
 /* ---- measurement / debug helpers ------------------------------------------------------
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
  * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */

@@ -61,6 +61,10 @@ struct ffs_ctx {
   DevBuf image, node_free, free_list, slice_node, slice_prof;
   std::vector<uint32_t> h_image;  // host copy of the table image (offline ranking)
   ImageLayout h_lay{};
+  // NEXT-2 joint commit: staged slice states and per-node slice ranges
+  std::vector<uint8_t> h_busy, h_cnt;
+  std::vector<uint64_t> h_node_free;
+  DevBuf node_off, j_keys, j_state, j_dirty, j_sreq, j_sslo, j_skeys, j_win, j_busy, j_cnt, j_free, j_ctr;
   // NEXT-1 ranked partitions
   DevBuf rank_off, rank_mask;
   bool ranked = false;
@@ -134,6 +138,9 @@ void ffs_destroy(ffs_ctx* c) {
     DeviceGuard g(c->device);
     for (auto& e : c->ev)
       if (e) cudaEventDestroy(e);
+    for (DevBuf* b : {&c->node_off, &c->j_keys, &c->j_state, &c->j_dirty, &c->j_sreq, &c->j_sslo, &c->j_skeys,
+                      &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
+      b->release();
     for (DevBuf* b : {&c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses})
       b->release();
@@ -277,6 +284,13 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   for (uint32_t v = 0; v < NN; ++v)
     for (uint32_t p = 0; p < 8; ++p)
       node_free[v] |= (uint64_t)std::min<uint32_t>(cnt[(size_t)v * 8 + p], 8) << (8 * p);
+  std::vector<uint32_t> noff(NN + 1, 0);
+  std::vector<uint8_t> hbusy(cl->n_slices);
+  for (uint32_t s = 0; s < cl->n_slices; ++s) {
+    noff[cl->slices[s].node + 1]++;
+    hbusy[s] = cl->slices[s].busy ? 1 : 0;
+  }
+  for (uint32_t v = 0; v < NN; ++v) noff[v + 1] += noff[v];
 
   DeviceGuard g(c->device);
   CK(c->image.ensure((size_t)L.words * 4), "cudaMalloc(image)");
@@ -294,6 +308,11 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   CK(cudaMemcpy(c->free_list.p, free_list.data(), free_list.size() * 4, cudaMemcpyHostToDevice), "upload free_list");
   CK(c->slice_node.ensure(snode.size() * 2), "cudaMalloc(slice_node)");
   CK(cudaMemcpy(c->slice_node.p, snode.data(), snode.size() * 2, cudaMemcpyHostToDevice), "upload slice_node");
+  CK(c->node_off.ensure(noff.size() * 4), "cudaMalloc(node_off)");
+  CK(cudaMemcpy(c->node_off.p, noff.data(), noff.size() * 4, cudaMemcpyHostToDevice), "upload node_off");
+  c->h_busy = hbusy;
+  c->h_cnt = cnt;
+  c->h_node_free = node_free;
   CK(c->slice_prof.ensure(sprof.size()), "cudaMalloc(slice_prof)");
   CK(cudaMemcpy(c->slice_prof.p, sprof.data(), sprof.size(), cudaMemcpyHostToDevice), "upload slice_prof");
   c->lay = L;
@@ -325,9 +344,19 @@ static ffs_status check_kmax(ffs_ctx* c, uint32_t k_max) {
   return FFS_OK;
 }
 
+static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                              uint32_t k_max, uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks,
+                              const uint64_t* node_free, void* stream);
+
 ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req, uint32_t k_max,
                          uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks, void* stream) {
   if (!c) return FFS_ERR_ARG;
+  return search_keys(c, d_req, d_slo, n_req, k_max, rank, world, d_keys, d_checks, nullptr, stream);
+}
+
+static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                              uint32_t k_max, uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks,
+                              const uint64_t* node_free, void* stream) {
   ffs_status s = check_kmax(c, k_max);
   if (s != FFS_OK) return s;
   if (world == 0 || rank >= world) return fail(c, FFS_ERR_ARG, "rank %u / world %u", rank, world);
@@ -365,7 +394,7 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
   a.lay = c->lay;
   a.req = d_req;
   a.slo = d_slo;
-  a.node_free = c->node_free.as<uint64_t>();
+  a.node_free = node_free ? node_free : c->node_free.as<uint64_t>();
   a.prefix = c->prefix.as<uint64_t>();
   a.n_req = n_req;
   a.rank = rank;
@@ -592,6 +621,81 @@ ffs_status ffs_plan_ranked(ffs_ctx* c, const ffs_request* d_req, const uint32_t*
   a.prof_order = c->prof_order;
   a.out = d_out;
   CK(launch_ranked(a, (cudaStream_t)stream), "ranked kernel");
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_joint(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req, uint32_t k_max,
+                          ffs_plan* d_out, uint32_t* rounds, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  ffs_status s0 = check_kmax(c, k_max);
+  if (s0 != FFS_OK) return s0;
+  if (rounds) *rounds = 0;
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
+  if (n_req >= (1u << 31)) return fail(c, FFS_ERR_RANGE, "n_req >= 2^31");
+  DeviceGuard g(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t R = n_req, NN = c->n_nodes, S = std::max(1u, c->n_slices);
+  CK(c->j_keys.ensure(R * 8), "cudaMalloc");
+  CK(c->j_state.ensure(R), "cudaMalloc");
+  CK(c->j_dirty.ensure(R * 4), "cudaMalloc");
+  CK(c->j_sreq.ensure(R * sizeof(ffs_request)), "cudaMalloc");
+  CK(c->j_sslo.ensure(R * 4), "cudaMalloc");
+  CK(c->j_skeys.ensure(R * 8), "cudaMalloc");
+  CK(c->j_win.ensure(NN * 8), "cudaMalloc");
+  CK(c->j_busy.ensure(S), "cudaMalloc");
+  CK(c->j_cnt.ensure(NN * 8), "cudaMalloc");
+  CK(c->j_free.ensure(NN * 8), "cudaMalloc");
+  CK(c->j_ctr.ensure(8), "cudaMalloc");
+  if (c->n_slices)
+    CK(cudaMemcpyAsync(c->j_busy.p, c->h_busy.data(), c->n_slices, cudaMemcpyHostToDevice, st), "H2D busy");
+  CK(cudaMemcpyAsync(c->j_cnt.p, c->h_cnt.data(), NN * 8, cudaMemcpyHostToDevice, st), "H2D counts");
+  CK(cudaMemcpyAsync(c->j_free.p, c->h_node_free.data(), NN * 8, cudaMemcpyHostToDevice, st), "H2D free");
+  JointArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.req = d_req;
+  a.slo = d_slo;
+  a.n_req = n_req;
+  a.n_nodes = c->n_nodes;
+  a.k_max = k_max;
+  a.keys = c->j_keys.as<int64_t>();
+  a.state = c->j_state.as<uint8_t>();
+  a.dirty = c->j_dirty.as<uint32_t>();
+  a.sub_req = c->j_sreq.as<ffs_request>();
+  a.sub_slo = c->j_sslo.as<uint32_t>();
+  a.sub_keys = c->j_skeys.as<int64_t>();
+  a.node_win = c->j_win.as<uint64_t>();
+  a.busy = c->j_busy.as<uint8_t>();
+  a.cnt = c->j_cnt.as<uint8_t>();
+  a.node_free = c->j_free.as<uint64_t>();
+  a.node_off = c->node_off.as<uint32_t>();
+  a.slice_prof = c->slice_prof.as<uint8_t>();
+  a.out = d_out;
+  a.n_open = c->j_ctr.as<uint32_t>();
+  a.n_dirty = c->j_ctr.as<uint32_t>() + 1;
+  CK(launch_joint(0, a, 0, st), "joint init");
+  uint32_t n_sub = n_req, nr = 0;
+  for (;;) {
+    ++nr;
+    if (n_sub) {
+      CK(launch_joint(1, a, n_sub, st), "joint gather");
+      ffs_status s = search_keys(c, a.sub_req, a.sub_slo, n_sub, k_max, 0, 1, a.sub_keys, nullptr, a.node_free, stream);
+      if (s != FFS_OK) return s;
+      CK(launch_joint(2, a, n_sub, st), "joint scatter");
+    }
+    CK(cudaMemsetAsync(a.node_win, 0xFF, NN * 8, st), "memset");
+    CK(cudaMemsetAsync(a.n_open, 0, 8, st), "memset");
+    CK(launch_joint(3, a, 0, st), "joint pick");
+    CK(launch_joint(4, a, 0, st), "joint commit");
+    CK(launch_joint(5, a, 0, st), "joint finalize");
+    uint32_t ctr[2];
+    CK(cudaMemcpyAsync(ctr, a.n_open, 8, cudaMemcpyDeviceToHost, st), "D2H counters");
+    CK(cudaStreamSynchronize(st), "sync");
+    if (ctr[0] == 0) break;
+    n_sub = ctr[1];
+  }
+  if (rounds) *rounds = nr;
   return FFS_OK;
 }
 

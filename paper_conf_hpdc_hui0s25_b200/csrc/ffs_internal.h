@@ -104,4 +104,28 @@ struct RankedArgs {
 };
 cudaError_t launch_ranked(const RankedArgs& a, cudaStream_t st);
 
+struct JointArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  uint32_t n_req, n_nodes, k_max;
+  int64_t* keys;               // [n_req] current argmin key of every open request
+  uint8_t* state;              // [n_req] 0 pending, 1 re-plan, 2 final
+  uint32_t* dirty;             // [n_req] requests to (re-)plan next round
+  ffs_request* sub_req;        // gathered dirty requests
+  uint32_t* sub_slo;
+  int64_t* sub_keys;
+  uint64_t* node_win;          // [n_nodes] min (adjusted deadline, index) of feasible open requests
+  uint8_t* busy;               // [n_slices] mutable copy of the slice states
+  uint8_t* cnt;                // [n_nodes][8] free slices per profile (true counts, <= 255)
+  uint64_t* node_free;         // [n_nodes] counts clamped to 8 (search input)
+  const uint32_t* node_off;    // [n_nodes+1] slices of node v
+  const uint8_t* slice_prof;
+  ffs_plan* out;
+  uint32_t* n_open;
+  uint32_t* n_dirty;
+};
+cudaError_t launch_joint(int phase, const JointArgs& a, uint32_t n, cudaStream_t st);
+
 }  // namespace ffsk

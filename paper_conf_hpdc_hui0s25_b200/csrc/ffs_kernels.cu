@@ -949,12 +949,7 @@ __device__ __forceinline__ bool victim_ok(const uint32_t* img, const ImageLayout
   return lat + fd[2] <= B;  // execution + reload within the budget
 }
 
-__global__ void k_decode(const __grid_constant__ DecodeArgs A) {
-  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r >= A.n_req) return;
-  const uint32_t* img = A.image;
-  const ImageLayout& L = A.lay;
-  ffs_plan pl;
+__device__ __forceinline__ void plan_init(ffs_plan& pl) {
   pl.key = (int64_t)kKeyNone;
   pl.status = FFS_PLAN_BAD_REQ;
   pl.k = pl.cut_mask = pl.e2e_us = pl.bottleneck_us = pl.gpcs = pl.cvq = 0;
@@ -964,11 +959,69 @@ __global__ void k_decode(const __grid_constant__ DecodeArgs A) {
     pl.slice[i] = -1;
   }
   pl.victim = -1;
+}
+
+// key -> (k, cut mask, profile digits) -> plan figures; slices are left to the caller.
+__device__ __forceinline__ void plan_from_key(const uint32_t* img, const ImageLayout& L, uint32_t func,
+                                              uint32_t k_max, int64_t key, ffs_plan& pl) {
+  const uint32_t* fd = img + L.o_fdesc + 4 * func;
+  const uint32_t row0 = fd[0], n = fd[1];
+  pl.status = FFS_PLAN_OK;
+  pl.key = key;
+  const uint64_t idx = (uint64_t)key & ((1ull << kIdxBits) - 1);
+  const uint32_t kmax = k_max < n ? k_max : n;
+  uint32_t k = 1;
+  while (k < kmax && img_u64(img, L.o_offk + 2 * (n * 10 + k + 1)) <= idx) ++k;
+  uint64_t PK = 1;
+  for (uint32_t i = 0; i < k; ++i) PK *= kP;
+  const uint64_t rem = idx - img_u64(img, L.o_offk + 2 * (n * 10 + k));
+  uint64_t rank = rem / PK, seq = rem % PK;
+  uint32_t mask = 0;
+  int cc = (int)n - 2;
+  for (int i = (int)k - 1; i >= 1; --i) {
+    while (img[L.o_binom + cc * 8 + i] > rank) --cc;
+    mask |= 1u << cc;
+    rank -= img[L.o_binom + cc * 8 + i];
+    --cc;
+  }
+  for (int i = (int)k - 1; i >= 0; --i) {
+    pl.prof[i] = (uint8_t)(seq % kP);
+    seq /= kP;
+  }
+  uint32_t a = 0, e2e = 0, bott = 0, g = 0, m = mask;
+  for (uint32_t i = 0; i < k; ++i) {
+    uint32_t b = n;
+    if (i + 1 < k) {
+      const int j = __ffs(m) - 1;
+      m &= m - 1;
+      b = j + 1;
+      e2e += img[L.o_xf + row0 + j];
+    }
+    const int p = pl.prof[i];
+    const uint32_t t = pl_diff(img, L.o_pl + (row0 + b) * kRowW + p, L.o_pl + (row0 + a) * kRowW + p);
+    e2e += t;
+    bott = t > bott ? t : bott;
+    g += img[L.o_gpcs + p];
+    a = b;
+  }
+  pl.k = k;
+  pl.cut_mask = mask;
+  pl.e2e_us = e2e;
+  pl.bottleneck_us = bott;  // throughput = 1e6 / bottleneck (R17)
+  pl.gpcs = g;
+  pl.cvq = (uint32_t)((uint64_t)key >> 50);
+}
+
+__global__ void k_decode(const __grid_constant__ DecodeArgs A) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.n_req) return;
+  const uint32_t* img = A.image;
+  const ImageLayout& L = A.lay;
+  ffs_plan pl;
+  plan_init(pl);
   const ffs_request q = A.req[r];
   if (q.func < L.F && q.node < A.n_nodes) {
     const int64_t key = A.keys[r];
-    const uint32_t* fd = img + L.o_fdesc + 4 * q.func;
-    const uint32_t row0 = fd[0], n = fd[1];
     if ((uint64_t)key == kKeyNone) {
       pl.status = FFS_PLAN_INFEASIBLE;
       if (A.inst) {
@@ -983,58 +1036,150 @@ __global__ void k_decode(const __grid_constant__ DecodeArgs A) {
         }
       }
     } else {
-      pl.status = FFS_PLAN_OK;
-      pl.key = key;
-      const uint64_t idx = (uint64_t)key & ((1ull << kIdxBits) - 1);
-      const uint32_t kmax = A.k_max < n ? A.k_max : n;
-      uint32_t k = 1;
-      while (k < kmax && img_u64(img, L.o_offk + 2 * (n * 10 + k + 1)) <= idx) ++k;
-      uint64_t PK = 1;
-      for (uint32_t i = 0; i < k; ++i) PK *= kP;
-      const uint64_t rem = idx - img_u64(img, L.o_offk + 2 * (n * 10 + k));
-      uint64_t rank = rem / PK, seq = rem % PK;
-      uint32_t mask = 0;
-      int cc = (int)n - 2;
-      for (int i = (int)k - 1; i >= 1; --i) {
-        while (img[L.o_binom + cc * 8 + i] > rank) --cc;
-        mask |= 1u << cc;
-        rank -= img[L.o_binom + cc * 8 + i];
-        --cc;
-      }
-      int prof[kMaxK];
-      for (int i = (int)k - 1; i >= 0; --i) {
-        prof[i] = (int)(seq % kP);
-        seq /= kP;
-      }
-      uint32_t a = 0, e2e = 0, bott = 0, g = 0, m = mask;
+      plan_from_key(img, L, q.func, A.k_max, key, pl);
       uint32_t used[kP] = {0, 0, 0, 0, 0};
-      for (uint32_t i = 0; i < k; ++i) {
-        uint32_t b = n;
-        if (i + 1 < k) {
-          const int j = __ffs(m) - 1;
-          m &= m - 1;
-          b = j + 1;
-          e2e += img[L.o_xf + row0 + j];
-        }
-        const int p = prof[i];
-        const uint32_t t = pl_diff(img, L.o_pl + (row0 + b) * kRowW + p, L.o_pl + (row0 + a) * kRowW + p);
-        e2e += t;
-        bott = t > bott ? t : bott;
-        g += img[L.o_gpcs + p];
-        pl.prof[i] = (uint8_t)p;
-        pl.slice[i] = A.free_list[((uint64_t)q.node * 8 + p) * 8 + used[p]];  // R11 binding
-        used[p]++;
-        a = b;
+      for (uint32_t i = 0; i < pl.k; ++i) {
+        const int p = pl.prof[i];
+        uint32_t u = 0;
+#pragma unroll
+        for (int x = 0; x < kP; ++x)
+          if (x == p) u = used[x]++;
+        pl.slice[i] = A.free_list[((uint64_t)q.node * 8 + p) * 8 + u];  // R11 binding
       }
-      pl.k = k;
-      pl.cut_mask = mask;
-      pl.e2e_us = e2e;
-      pl.bottleneck_us = bott;  // throughput = 1e6 / bottleneck (R17)
-      pl.gpcs = g;
-      pl.cvq = (uint32_t)((uint64_t)key >> 50);
     }
   }
   A.out[r] = pl;
+}
+
+// ====================================================================================
+// K7 (NEXT-2): joint commit in monotone rounds
+// ====================================================================================
+// state: 0 pending (key valid for the current free state), 1 dirty (re-plan), 2 final
+__device__ __forceinline__ uint64_t joint_order(const uint32_t* img, const ImageLayout& L, const ffs_request& q,
+                                                uint32_t B, uint32_t r) {
+  // adjusted deadline = B - load - fastest 1-stage latency (R28), biased to be >= 0, then index
+  const uint32_t* fd = img + L.o_fdesc + 4 * q.func;
+  const uint32_t row0 = fd[0], n = fd[1];
+  uint32_t fast = 0xFFFFFFFFu;
+#pragma unroll
+  for (int p = 0; p < kP; ++p) {
+    const uint32_t t = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
+    fast = t < fast ? t : fast;
+  }
+  const int64_t adj = (int64_t)B - (int64_t)fd[2] - (int64_t)fast + (1ll << 26);  // >= 0: load, fast < 2^26
+  return ((uint64_t)adj << 31) | r;
+}
+
+__global__ void k_joint_init(const __grid_constant__ JointArgs A) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.n_req) return;
+  const ffs_request q = A.req[r];
+  if (q.func < A.lay.F && q.node < A.n_nodes) {
+    A.state[r] = 1;  // plan in round 0
+    A.dirty[r] = r;
+  } else {
+    ffs_plan pl;
+    plan_init(pl);
+    A.out[r] = pl;
+    A.state[r] = 2;
+    A.dirty[r] = r;  // planned harmlessly in round 0 (BAD_REQ keys are ignored)
+  }
+}
+
+__global__ void k_joint_gather(const __grid_constant__ JointArgs A, uint32_t n) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t r = A.dirty[i];
+  A.sub_req[i] = A.req[r];
+  A.sub_slo[i] = A.slo[r];
+}
+
+__global__ void k_joint_scatter(const __grid_constant__ JointArgs A, uint32_t n_sub) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n_sub) A.keys[A.dirty[i]] = A.sub_keys[i];  // re-planned keys back to their requests
+}
+
+__global__ void k_joint_pick(const __grid_constant__ JointArgs A) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.n_req || A.state[r] == 2) return;
+  if ((uint64_t)A.keys[r] == kKeyNone) return;
+  const ffs_request q = A.req[r];
+  atomicMin(reinterpret_cast<unsigned long long*>(A.node_win + q.node),
+            (unsigned long long)joint_order(A.image, A.lay, q, A.slo[r], r));
+}
+
+// one thread per node: commit the earliest-deadline feasible request, bind its slices to
+// the lowest-index free slices of its profiles in stage order, take them
+__global__ void k_joint_commit(const __grid_constant__ JointArgs A) {
+  const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+  if (v >= A.n_nodes) return;
+  const uint64_t w = A.node_win[v];
+  if (w == ~0ull) return;
+  const uint32_t r = (uint32_t)(w & 0x7FFFFFFFu);
+  const ffs_request q = A.req[r];
+  ffs_plan pl;
+  plan_init(pl);
+  plan_from_key(A.image, A.lay, q.func, A.k_max, A.keys[r], pl);
+  uint8_t* cnt = A.cnt + (uint64_t)v * 8;
+  for (uint32_t i = 0; i < pl.k; ++i) {
+    const uint32_t p = pl.prof[i];
+    for (uint32_t s = A.node_off[v]; s < A.node_off[v + 1]; ++s)
+      if (!A.busy[s] && A.slice_prof[s] == p) {
+        A.busy[s] = 1;
+        pl.slice[i] = (int32_t)s;
+        cnt[p]--;
+        break;
+      }
+  }
+  uint64_t nf = 0;
+  for (int p = 0; p < 8; ++p) nf |= (uint64_t)(cnt[p] < 8 ? cnt[p] : 8) << (8 * p);
+  A.node_free[v] = nf;
+  A.out[r] = pl;
+  A.state[r] = 2;
+}
+
+// per request: infeasible -> final; a pending plan that no longer fits the node's counts
+// -> dirty (appended to the re-plan list); counts the requests still open
+__global__ void k_joint_finalize(const __grid_constant__ JointArgs A) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.n_req || A.state[r] == 2) return;
+  const ffs_request q = A.req[r];
+  const int64_t key = A.keys[r];
+  if ((uint64_t)key == kKeyNone) {  // the free state only shrinks: stays infeasible
+    ffs_plan pl;
+    plan_init(pl);
+    pl.status = FFS_PLAN_INFEASIBLE;
+    A.out[r] = pl;
+    A.state[r] = 2;
+    return;
+  }
+  uint8_t st = 0;
+  if (A.node_win[q.node] != ~0ull) {  // the node committed this round: does the plan still fit?
+    ffs_plan pl;
+    plan_from_key(A.image, A.lay, q.func, A.k_max, key, pl);
+    uint32_t used[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    for (uint32_t i = 0; i < pl.k; ++i) used[pl.prof[i] & 7]++;
+    const uint8_t* cnt = A.cnt + (uint64_t)q.node * 8;
+    for (int p = 0; p < 8; ++p)
+      if (used[p] > cnt[p]) st = 1;
+  }
+  A.state[r] = st;
+  atomicAdd(A.n_open, 1u);
+  if (st == 1) A.dirty[atomicAdd(A.n_dirty, 1u)] = r;
+}
+
+cudaError_t launch_joint(int phase, const JointArgs& a, uint32_t n, cudaStream_t st) {
+  const uint32_t T = 256;
+  switch (phase) {
+    case 0: k_joint_init<<<(a.n_req + T - 1) / T, T, 0, st>>>(a); break;
+    case 1: if (n) k_joint_gather<<<(n + T - 1) / T, T, 0, st>>>(a, n); break;
+    case 2: if (n) k_joint_scatter<<<(n + T - 1) / T, T, 0, st>>>(a, n); break;
+    case 3: k_joint_pick<<<(a.n_req + T - 1) / T, T, 0, st>>>(a); break;
+    case 4: k_joint_commit<<<(a.n_nodes + T - 1) / T, T, 0, st>>>(a); break;
+    case 5: k_joint_finalize<<<(a.n_req + T - 1) / T, T, 0, st>>>(a); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
 }
 
 cudaError_t launch_decode(const DecodeArgs& a, cudaStream_t st) {

@@ -60,6 +60,7 @@ _sig = {
     "ffs_evict_scores": ([_vp, _vp, _u32, _u64, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
+    "ffs_plan_joint": ([_vp, _vp, _vp, _u32, _u32, _vp, C.POINTER(C.c_uint32), _vp], _i32),
     "ffs_rank_partitions": ([_vp, _u32, _u32], _i32),
     "ffs_plan_ranked": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
@@ -216,6 +217,18 @@ class Planner:
                                            _ptr(tick_off), _ptr(score), int(tick_off.numel() - 1), _ptr(victim),
                                            _stream(stream)))
         return victim
+
+    # ---- NEXT-2: joint commit -------------------------------------------------
+    def plan_joint(self, req, slo, k_max: int, out=None, stream=None):
+        """Jointly feasible plans of the batch; returns (plans, rounds).  Synchronous."""
+        import torch
+        n = int(slo.numel())
+        if out is None:
+            out = torch.empty((n, PLAN_DTYPE.itemsize), dtype=torch.uint8, device=slo.device)
+        rounds = C.c_uint32()
+        self._check(_lib.ffs_plan_joint(self._h, _ptr(req), _ptr(slo), n, int(k_max), _ptr(out), C.byref(rounds),
+                                        _stream(stream)))
+        return out, int(rounds.value)
 
     # ---- NEXT-1: ranked first-fit (P:339-343) -----------------------------------------------
     def rank_partitions(self, k_max: int, p_ref: int) -> None:

@@ -281,3 +281,29 @@ def test_ranked_c5_sample(F, planner):
     p = run_ranked(F, planner, prob)
     idx = np.arange(0, prob.R, 1021)
     assert_plans_equal(p, oracle.plan_ranked(prob.subset(idx)), idx)
+
+
+# ---- NEXT-2: joint commit ------------------------------------------------
+def run_joint(F, planner, prob):
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    out, rounds = planner.plan_joint(req, slo, prob.k_max)
+    return F.plans_to_numpy(out), rounds
+
+
+@pytest.mark.parametrize("seed", range(1000, 1016))
+def test_joint_tiny_random(F, planner, seed):
+    prob = random_tiny(seed)
+    p, _ = run_joint(F, planner, prob)
+    assert_plans_equal(p, oracle.plan_joint(prob))
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3s"])
+def test_joint_configs(F, planner, cfg):
+    prob = {"C1": W.config1, "C2": W.config2, "C3s": lambda: W.config3(R=4096)}[cfg]()
+    p, rounds = run_joint(F, planner, prob)
+    assert_plans_equal(p, oracle.plan_joint(prob))
+    used = p["slice"][p["status"] == 0].ravel()
+    used = used[used >= 0]
+    assert len(used) == len(set(used.tolist()))  # jointly feasible
+    assert rounds >= 1
