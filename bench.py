@@ -252,6 +252,33 @@ def run_joint(pl, prob, req, slo):
             "rounds": rounds, "ok_frac": float((p["status"] == 0).mean())}
 
 
+def run_frontier(pl, prob, req, slo, steps: int, warmup: int, flush):
+    """NEXT-3 (frontier precompute): build every (function, node free-vector) frontier once,
+    then answer the batch by binary search; plans identical to the argmin path."""
+    import torch
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    groups, rounds = pl.frontier_build(prob.k_max)
+    build_s = time.perf_counter() - t0
+    out = torch.empty((prob.R, 80), dtype=torch.uint8, device="cuda")
+    for _ in range(warmup):
+        pl.plan_frontier(req, slo, out=out)
+    stream = torch.cuda.current_stream()
+    ms = 0.0
+    for i in range(steps):
+        flush.fill_(i & 0xFF)
+        a.record(stream)
+        pl.plan_frontier(req, slo, out=out)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ms += a.elapsed_time(b)
+    return {"metric": "frontier_plans_per_s", "value": prob.R * steps / (ms * 1e-3), "unit": "plans/s",
+            "query_ms_per_step": ms / steps, "build_s": build_s, "groups": groups, "rounds": rounds,
+            "note": "plans identical to the argmin path; candidates are scored once per frontier point and group, "
+                    "not per request (not comparable to candidates/s)"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -386,9 +413,10 @@ def main():
     ranked = None
     if world == 1 and not args.no_c4:
         ranked = run_ranked(pl, prob, req, slo, args.steps, args.warmup, flush)
-    joint = None
+    joint = frontier = None
     if world == 1 and not args.no_c4:
         joint = run_joint(pl, prob, req, slo)
+        frontier = run_frontier(pl, prob, req, slo, args.steps, args.warmup, flush)
     c4 = None
     if world == 1 and not args.no_c4:
         c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
@@ -419,6 +447,7 @@ def main():
             "eviction_c4": c4,
             "ranked_first_fit": ranked,
             "joint_commit": joint,
+            "frontier": frontier,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

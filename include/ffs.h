@@ -262,6 +262,20 @@ ffs_status ffs_plan_ranked(ffs_ctx *ctx, const ffs_request *d_req, const uint32_
 ffs_status ffs_plan_joint(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
                           uint32_t k_max, ffs_plan *d_out, uint32_t *rounds, void *stream);
 
+/* ---- NEXT-3: frontier precompute ------------------------------------------------------
+ * For a fixed (function, node free-vector) the feasible set depends on the budget only
+ * through e2e <= B, so the argmin for any B is the lowest-key point of the Pareto
+ * frontier of (key, e2e) with e2e <= B.  ffs_frontier_build computes every frontier of
+ * the staged tables by peeling with the search kernels: point i+1 = the minimum key among
+ * candidates with e2e < e2e(point i).  Synchronous; *n_groups and
+ * *rounds report the work (nullable).  ffs_plan_frontier answers a batch from the
+ * frontiers (binary search by budget + decode/bind): its plans are identical to
+ * ffs_plan_batch's.  Asynchronous.  FFS_ERR_STATE: frontiers not built for these
+ * tables / k_max. */
+ffs_status ffs_frontier_build(ffs_ctx *ctx, uint32_t k_max, uint32_t *n_groups, uint32_t *rounds, void *stream);
+ffs_status ffs_plan_frontier(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                             ffs_plan *d_out, void *stream);
+
 /* ---- measurement / debug helpers ------------------------------------------------------
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
  * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */

@@ -65,6 +65,10 @@ struct ffs_ctx {
   std::vector<uint8_t> h_busy, h_cnt;
   std::vector<uint64_t> h_node_free;
   DevBuf node_off, j_keys, j_state, j_dirty, j_sreq, j_sslo, j_skeys, j_win, j_busy, j_cnt, j_free, j_ctr;
+  // NEXT-3 frontiers
+  DevBuf f_nodefv, f_fvnode, f_act, f_next, f_budget, f_greq, f_gslo, f_gkeys, f_cnt, f_key, f_e2e, f_ctr;
+  bool front_built = false;
+  uint32_t front_kmax = 0, front_groups = 0, front_nfv = 0, front_cap = 0;
   // NEXT-1 ranked partitions
   DevBuf rank_off, rank_mask;
   bool ranked = false;
@@ -138,6 +142,9 @@ void ffs_destroy(ffs_ctx* c) {
     DeviceGuard g(c->device);
     for (auto& e : c->ev)
       if (e) cudaEventDestroy(e);
+    for (DevBuf* b : {&c->f_nodefv, &c->f_fvnode, &c->f_act, &c->f_next, &c->f_budget, &c->f_greq, &c->f_gslo,
+                      &c->f_gkeys, &c->f_cnt, &c->f_key, &c->f_e2e, &c->f_ctr})
+      b->release();
     for (DevBuf* b : {&c->node_off, &c->j_keys, &c->j_state, &c->j_dirty, &c->j_sreq, &c->j_sslo, &c->j_skeys,
                       &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
       b->release();
@@ -318,6 +325,7 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   c->lay = L;
   c->h_image = img;
   c->ranked = false;
+  c->front_built = false;
   c->P = P;
   c->F = F;
   c->n_nodes = NN;
@@ -696,6 +704,133 @@ ffs_status ffs_plan_joint(ffs_ctx* c, const ffs_request* d_req, const uint32_t* 
     n_sub = ctr[1];
   }
   if (rounds) *rounds = nr;
+  return FFS_OK;
+}
+
+ffs_status ffs_frontier_build(ffs_ctx* c, uint32_t k_max, uint32_t* n_groups, uint32_t* rounds, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  ffs_status s0 = check_kmax(c, k_max);
+  if (s0 != FFS_OK) return s0;
+  DeviceGuard g(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  c->front_built = false;
+  // groups = (function, distinct clamped free vector of a node)
+  std::vector<uint32_t> node_fv(c->n_nodes), fv_node;
+  {
+    std::vector<std::pair<uint64_t, uint32_t>> seen;
+    for (uint32_t v = 0; v < c->n_nodes; ++v) {
+      uint32_t id = (uint32_t)seen.size();
+      for (auto& e : seen)
+        if (e.first == c->h_node_free[v]) id = e.second;
+      if (id == seen.size()) {
+        seen.push_back({c->h_node_free[v], id});
+        fv_node.push_back(v);
+      }
+      node_fv[v] = id;
+    }
+  }
+  const uint32_t nfv = (uint32_t)fv_node.size();
+  const uint64_t G64 = (uint64_t)c->F * nfv;
+  if (G64 >= (1ull << 31)) return fail(c, FFS_ERR_RANGE, "too many frontier groups");
+  const uint32_t G = (uint32_t)G64;
+  CK(c->f_nodefv.ensure(node_fv.size() * 4), "cudaMalloc");
+  CK(cudaMemcpy(c->f_nodefv.p, node_fv.data(), node_fv.size() * 4, cudaMemcpyHostToDevice), "H2D");
+  CK(c->f_fvnode.ensure(fv_node.size() * 4), "cudaMalloc");
+  CK(cudaMemcpy(c->f_fvnode.p, fv_node.data(), fv_node.size() * 4, cudaMemcpyHostToDevice), "H2D");
+  for (DevBuf* b : {&c->f_act, &c->f_next, &c->f_budget, &c->f_gslo, &c->f_cnt}) CK(b->ensure((size_t)G * 4), "cudaMalloc");
+  CK(c->f_greq.ensure((size_t)G * sizeof(ffs_request)), "cudaMalloc");
+  CK(c->f_gkeys.ensure((size_t)G * 8), "cudaMalloc");
+  CK(c->f_ctr.ensure(8), "cudaMalloc");
+  std::vector<uint32_t> iota(G);
+  for (uint32_t i = 0; i < G; ++i) iota[i] = i;
+  CK(cudaMemcpyAsync(c->f_act.p, iota.data(), (size_t)G * 4, cudaMemcpyHostToDevice, st), "H2D");
+  CK(cudaMemsetAsync(c->f_budget.p, 0xFF, (size_t)G * 4, st), "memset");
+  CK(cudaMemsetAsync(c->f_cnt.p, 0, (size_t)G * 4, st), "memset");
+  uint32_t cap = 64;
+  CK(c->f_key.ensure((size_t)cap * G * 8), "cudaMalloc");
+  CK(c->f_e2e.ensure((size_t)cap * G * 4), "cudaMalloc");
+  FrontierArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.k_max = k_max;
+  a.n_groups = G;
+  a.n_fv = nfv;
+  a.n_nodes = c->n_nodes;
+  a.node_fv = c->f_nodefv.as<uint32_t>();
+  a.budget = c->f_budget.as<uint32_t>();
+  a.greq = c->f_greq.as<ffs_request>();
+  a.n_next = c->f_ctr.as<uint32_t>();
+  a.fr_cnt = c->f_cnt.as<uint32_t>();
+  uint32_t n_active = G, round = 0;
+  uint32_t *act = c->f_act.as<uint32_t>(), *nxt = c->f_next.as<uint32_t>();
+  while (n_active) {
+    if (round == cap) {  // grow the round-major point arrays
+      DevBuf nk, ne;
+      CK(nk.ensure((size_t)2 * cap * G * 8), "cudaMalloc");
+      CK(ne.ensure((size_t)2 * cap * G * 4), "cudaMalloc");
+      CK(cudaMemcpyAsync(nk.p, c->f_key.p, (size_t)cap * G * 8, cudaMemcpyDeviceToDevice, st), "D2D");
+      CK(cudaMemcpyAsync(ne.p, c->f_e2e.p, (size_t)cap * G * 4, cudaMemcpyDeviceToDevice, st), "D2D");
+      CK(cudaStreamSynchronize(st), "sync");
+      c->f_key.release();
+      c->f_e2e.release();
+      c->f_key = nk;
+      c->f_e2e = ne;
+      nk.p = ne.p = nullptr;
+      cap *= 2;
+    }
+    a.cap = cap;
+    a.fr_key = c->f_key.as<int64_t>();
+    a.fr_e2e = c->f_e2e.as<uint32_t>();
+    a.active = act;
+    a.next_active = nxt;
+    a.keys = c->f_gkeys.as<int64_t>();
+    a.round = round;
+    CK(launch_front_gather(a, n_active, c->f_fvnode.as<uint32_t>(), c->f_gslo.as<uint32_t>(), st), "gather");
+    ffs_status s = search_keys(c, a.greq, c->f_gslo.as<uint32_t>(), n_active, k_max, 0, 1, c->f_gkeys.as<int64_t>(),
+                               nullptr, nullptr, stream);
+    if (s != FFS_OK) return s;
+    CK(cudaMemsetAsync(a.n_next, 0, 4, st), "memset");
+    CK(launch_frontier(1, a, n_active, st), "record");
+    CK(cudaMemcpyAsync(&n_active, a.n_next, 4, cudaMemcpyDeviceToHost, st), "D2H");
+    CK(cudaStreamSynchronize(st), "sync");
+    std::swap(act, nxt);
+    ++round;
+  }
+  c->front_built = true;
+  c->front_kmax = k_max;
+  c->front_groups = G;
+  c->front_nfv = nfv;
+  c->front_cap = cap;
+  if (n_groups) *n_groups = G;
+  if (rounds) *rounds = round;
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_frontier(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                             ffs_plan* d_out, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged || !c->front_built) return fail(c, FFS_ERR_STATE, "call ffs_frontier_build after staging");
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  FrontierArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.k_max = c->front_kmax;
+  a.n_groups = c->front_groups;
+  a.n_fv = c->front_nfv;
+  a.n_nodes = c->n_nodes;
+  a.cap = c->front_cap;
+  a.node_fv = c->f_nodefv.as<uint32_t>();
+  a.fr_key = c->f_key.as<int64_t>();
+  a.fr_e2e = c->f_e2e.as<uint32_t>();
+  a.fr_cnt = c->f_cnt.as<uint32_t>();
+  a.req = d_req;
+  a.slo = d_slo;
+  a.n_req = n_req;
+  a.free_list = c->free_list.as<int32_t>();
+  a.out = d_out;
+  CK(launch_frontier(2, a, 0, (cudaStream_t)stream), "frontier query");
   return FFS_OK;
 }
 

@@ -128,4 +128,32 @@ struct JointArgs {
 };
 cudaError_t launch_joint(int phase, const JointArgs& a, uint32_t n, cudaStream_t st);
 
+struct FrontierArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  uint32_t k_max, n_groups, n_fv, n_nodes, cap;  // cap = rounds allocated
+  const uint32_t* node_fv;      // [n_nodes] free-vector id of each node
+  // build
+  const uint32_t* active;       // [n_active] group ids searched this round
+  const int64_t* keys;          // [n_active] argmin keys of this round
+  uint32_t* next_active;
+  uint32_t* n_next;
+  uint32_t* budget;             // [n_groups] budget of the group's next search (e2e of last point - 1)
+  ffs_request* greq;            // [n_active] synthetic requests of this round
+  uint32_t round;
+  // frontier storage, round-major: point i of group g at [i * n_groups + g]
+  int64_t* fr_key;
+  uint32_t* fr_e2e;
+  uint32_t* fr_cnt;             // [n_groups]
+  // query
+  const ffs_request* req;
+  const uint32_t* slo;
+  uint32_t n_req;
+  const int32_t* free_list;
+  ffs_plan* out;
+};
+cudaError_t launch_frontier(int phase, const FrontierArgs& a, uint32_t n, cudaStream_t st);
+cudaError_t launch_front_gather(const FrontierArgs& a, uint32_t n, const uint32_t* fv_node, uint32_t* gslo,
+                                cudaStream_t st);
+
 }  // namespace ffsk

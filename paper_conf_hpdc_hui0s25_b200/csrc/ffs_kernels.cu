@@ -1465,6 +1465,89 @@ cudaError_t launch_ranked(const RankedArgs& a, cudaStream_t st) {
 }
 
 // ====================================================================================
+// K8 (NEXT-3): frontier build (peeling rounds) and frontier queries
+// ====================================================================================
+// synthetic requests of the active groups: function g / n_fv on a node with free-vector
+// g % n_fv (a representative node), budget = the group's current budget
+__global__ void k_front_gather(const __grid_constant__ FrontierArgs A, uint32_t n_active,
+                               const uint32_t* __restrict__ fv_node, uint32_t* __restrict__ gslo) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n_active) return;
+  const uint32_t g = A.active[i];
+  ffs_request q;
+  q.func = g / A.n_fv;
+  q.node = fv_node[g % A.n_fv];
+  A.greq[i] = q;
+  gslo[i] = A.budget[g];
+}
+
+// record this round's frontier point of every active group; groups with a point stay
+// active with budget e2e - 1
+__global__ void k_front_record(const __grid_constant__ FrontierArgs A, uint32_t n_active) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n_active) return;
+  const uint32_t g = A.active[i];
+  const int64_t key = A.keys[i];
+  if ((uint64_t)key == kKeyNone) return;
+  ffs_plan pl;
+  plan_from_key(A.image, A.lay, g / A.n_fv, A.k_max, key, pl);
+  const uint64_t at = (uint64_t)A.round * A.n_groups + g;
+  A.fr_key[at] = key;
+  A.fr_e2e[at] = pl.e2e_us;
+  A.fr_cnt[g] = A.round + 1;
+  if (pl.e2e_us > 0) {
+    A.budget[g] = pl.e2e_us - 1;
+    A.next_active[atomicAdd(A.n_next, 1u)] = g;
+  }
+}
+
+// one thread per request: the first frontier point (lowest key) with e2e <= B; the
+// points of a group have increasing keys and strictly decreasing e2e
+__global__ void k_front_query(const __grid_constant__ FrontierArgs A) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= A.n_req) return;
+  ffs_plan pl;
+  plan_init(pl);
+  const ffs_request q = A.req[r];
+  if (q.func < A.lay.F && q.node < A.n_nodes) {
+    const uint32_t g = q.func * A.n_fv + A.node_fv[q.node];
+    const uint32_t B = A.slo[r];
+    uint32_t lo = 0, hi = A.fr_cnt[g];  // first i in [lo, hi) with e2e_i <= B
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (A.fr_e2e[(uint64_t)mid * A.n_groups + g] <= B) hi = mid; else lo = mid + 1;
+    }
+    if (lo == A.fr_cnt[g]) {
+      pl.status = FFS_PLAN_INFEASIBLE;
+    } else {
+      plan_from_key(A.image, A.lay, q.func, A.k_max, A.fr_key[(uint64_t)lo * A.n_groups + g], pl);
+      uint32_t used[kP] = {0, 0, 0, 0, 0};
+      for (uint32_t i = 0; i < pl.k; ++i) {
+        const int p = pl.prof[i];
+        uint32_t u = 0;
+#pragma unroll
+        for (int x = 0; x < kP; ++x)
+          if (x == p) u = used[x]++;
+        pl.slice[i] = A.free_list[((uint64_t)q.node * 8 + p) * 8 + u];
+      }
+    }
+  }
+  A.out[r] = pl;
+}
+
+cudaError_t launch_frontier(int phase, const FrontierArgs& a, uint32_t n, cudaStream_t st) {
+  const uint32_t T = 256;
+  if (phase == 1 && n) k_front_record<<<(n + T - 1) / T, T, 0, st>>>(a, n);
+  if (phase == 2 && a.n_req) k_front_query<<<(a.n_req + T - 1) / T, T, 0, st>>>(a);
+  return cudaGetLastError();
+}
+cudaError_t launch_front_gather(const FrontierArgs& a, uint32_t n, const uint32_t* fv_node, uint32_t* gslo,
+                                cudaStream_t st) {
+  if (n) k_front_gather<<<(n + 255) / 256, 256, 0, st>>>(a, n, fv_node, gslo);
+  return cudaGetLastError();
+}
+
+// ====================================================================================
 // K5: integer issue-rate microbenchmark (roofline denominator)
 // ====================================================================================
 constexpr int kPeakIters = 4096;

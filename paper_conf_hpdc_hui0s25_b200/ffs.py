@@ -61,6 +61,8 @@ _sig = {
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_plan_joint": ([_vp, _vp, _vp, _u32, _u32, _vp, C.POINTER(C.c_uint32), _vp], _i32),
+    "ffs_frontier_build": ([_vp, _u32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32), _vp], _i32),
+    "ffs_plan_frontier": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_rank_partitions": ([_vp, _u32, _u32], _i32),
     "ffs_plan_ranked": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
@@ -229,6 +231,21 @@ class Planner:
         self._check(_lib.ffs_plan_joint(self._h, _ptr(req), _ptr(slo), n, int(k_max), _ptr(out), C.byref(rounds),
                                         _stream(stream)))
         return out, int(rounds.value)
+
+    # ---- NEXT-3: frontier precompute ---------------------------------------------------------
+    def frontier_build(self, k_max: int, stream=None) -> tuple[int, int]:
+        """Build every (function, node free-vector) frontier; returns (groups, rounds)."""
+        g, r = C.c_uint32(), C.c_uint32()
+        self._check(_lib.ffs_frontier_build(self._h, int(k_max), C.byref(g), C.byref(r), _stream(stream)))
+        return int(g.value), int(r.value)
+
+    def plan_frontier(self, req, slo, out=None, stream=None):
+        import torch
+        n = int(slo.numel())
+        if out is None:
+            out = torch.empty((n, PLAN_DTYPE.itemsize), dtype=torch.uint8, device=slo.device)
+        self._check(_lib.ffs_plan_frontier(self._h, _ptr(req), _ptr(slo), n, _ptr(out), _stream(stream)))
+        return out
 
     # ---- NEXT-1: ranked first-fit (P:339-343) -----------------------------------------------
     def rank_partitions(self, k_max: int, p_ref: int) -> None:

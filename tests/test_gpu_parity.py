@@ -307,3 +307,29 @@ def test_joint_configs(F, planner, cfg):
     used = used[used >= 0]
     assert len(used) == len(set(used.tolist()))  # jointly feasible
     assert rounds >= 1
+
+
+# ---- NEXT-3: frontier precompute -----------------------------------------------------------
+@pytest.mark.parametrize("cfg", ["tiny", "C1", "C2", "C3s"])
+def test_frontier_plans_equal_argmin_plans(F, planner, cfg):
+    prob = {"tiny": lambda: random_tiny(1003), "C1": W.config1, "C2": W.config2,
+            "C3s": lambda: W.config3(R=8192)}[cfg]()
+    p_arg, _, _ = run_gpu(F, planner, prob, verify=False)
+    groups, rounds = planner.frontier_build(prob.k_max)
+    req, slo = F.to_device(prob)
+    p_fr = F.plans_to_numpy(planner.plan_frontier(req, slo))
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(p_fr.view(np.uint8), p_arg.view(np.uint8))  # identical plans
+    assert rounds >= 1 and groups >= 1
+    if cfg in ("tiny", "C1"):
+        assert_plans_equal(p_fr, oracle.plan(prob, checks=False))
+
+
+def test_frontier_c5_sample(F, planner):
+    prob = W.config5()
+    planner.stage(prob)
+    planner.frontier_build(prob.k_max)
+    req, slo = F.to_device(prob)
+    p = F.plans_to_numpy(planner.plan_frontier(req, slo))
+    idx = np.arange(0, prob.R, 2053)
+    assert_plans_equal(p, oracle.plan(prob.subset(idx), checks=False), idx)
