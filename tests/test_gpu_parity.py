@@ -333,3 +333,24 @@ def test_frontier_c5_sample(F, planner):
     p = F.plans_to_numpy(planner.plan_frontier(req, slo))
     idx = np.arange(0, prob.R, 2053)
     assert_plans_equal(p, oracle.plan(prob.subset(idx), checks=False), idx)
+
+
+def test_next_rows_error_states(F):
+    pl = F.Planner(0)
+    prob = random_tiny(1004)
+    req, slo = F.to_device(prob)
+    for call in (lambda: pl.plan_ranked(req, slo), lambda: pl.plan_frontier(req, slo),
+                 lambda: pl.plan_joint(req, slo, 4)):
+        with pytest.raises(F.FFSError) as e:
+            call()
+        assert e.value.status == F.FFS_ERR_STATE
+    pl.stage(prob)
+    with pytest.raises(F.FFSError) as e:
+        pl.rank_partitions(4, 5)  # p_ref >= P
+    assert e.value.status == F.FFS_ERR_RANGE
+    pl.frontier_build(4)
+    pl.stage(prob)  # re-staging invalidates derived structures
+    with pytest.raises(F.FFSError) as e:
+        pl.plan_frontier(req, slo)
+    assert e.value.status == F.FFS_ERR_STATE
+    pl.close()
