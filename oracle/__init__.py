@@ -65,6 +65,7 @@ def lib():
             _lib.oracle_plan_ranked.restype = C.c_int
             _lib.oracle_plan_joint.argtypes = [C.POINTER(_PlanArgs)]
             _lib.oracle_plan_joint.restype = C.c_int
+            _lib.oracle_route.restype = C.c_int
             _lib.oracle_evict.restype = None
             _lib.oracle_victim.restype = None
     return _lib
@@ -159,6 +160,16 @@ def plan_joint(prob, k_max: int | None = None) -> dict:
     if rc != 0:
         raise ValueError("oracle_plan_joint rejected its arguments")
     return h.out
+
+
+def route(prob, inst_func, inst_state, inst_lat, inst_cap) -> np.ndarray:
+    """NEXT-2 routing (ffs_oracle.c: oracle_route): instance index per request."""
+    h = _Held(prob, prob.k_max, False)
+    fu, st = _c(inst_func, np.uint32), _c(inst_state, np.uint8)
+    la, ca = _c(inst_lat, np.uint32), _c(inst_cap, np.uint32)
+    out = np.full(h.func.shape[0], -1, np.int32)
+    lib().oracle_route(C.byref(h.args), C.c_int(int(fu.shape[0])), _p(fu), _p(st), _p(la), _p(ca), _p(out))
+    return out
 
 
 def evict(inst: np.ndarray, now_us: int, util_thr_pct: int = 30, window_us: int = 10_000_000,

@@ -671,3 +671,84 @@ int oracle_plan_joint(const oracle_plan_args *a) {
     free(busy);
     return 0;
 }
+
+/* ---- NEXT-2 (routing): heterogeneity-aware request routing -------------------
+ * "urgent requests are directed to the instance with the lowest latency until its
+ * serving capacity is reached.  Subsequent requests are routed to the next lowest
+ * latency instance, and so forth.  Then the remaining requests are routed to the time
+ * sharing state instance."  Per function (R30): requests in ascending adjusted
+ * deadline (R28: budget - load - fastest 1-stage latency, ties by index); exclusive-hot
+ * instances of the function (state EXCL_HOT) in ascending (latency, index), each taking
+ * `capacity` requests; every further request goes to the function's time-sharing
+ * instance (the lowest-index instance in state TIME_SHARING or WARM), or -1 if it has
+ * none.  route[r] = instance index; BAD_REQ requests (func >= F) get -1. */
+typedef struct {
+    int64_t a;
+    uint32_t b;
+    int i;
+} route_item;
+
+static int cmp_route(const void *x, const void *y) {
+    const route_item *p = (const route_item *)x, *q = (const route_item *)y;
+    if (p->a != q->a) return p->a < q->a ? -1 : 1;
+    if (p->b != q->b) return p->b < q->b ? -1 : 1;
+    return p->i < q->i ? -1 : (p->i > q->i);
+}
+
+int oracle_route(const oracle_plan_args *a, int n_inst, const uint32_t *inst_func, const uint8_t *inst_state,
+                 const uint32_t *inst_lat, const uint32_t *inst_cap, int32_t *route) {
+    for (int f = 0; f < a->F; f++) {
+        /* requests of f in adjusted-deadline order */
+        int nr = 0;
+        route_item *rq = (route_item *)malloc(sizeof(route_item) * (size_t)(a->R > 0 ? a->R : 1));
+        int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+        uint64_t fast = UINT64_MAX;
+        for (int p = 0; p < a->P; p++) {
+            uint64_t t = 0;
+            for (int c = 0; c < n; c++) t += lat_of(a, f, c, p);
+            if (t < fast) fast = t;
+        }
+        for (int r = 0; r < a->R; r++)
+            if ((int)a->req_func[r] == f) {
+                rq[nr].a = (int64_t)a->req_slo_us[r] - (int64_t)a->load_us[f] - (int64_t)fast;
+                rq[nr].b = (uint32_t)r;
+                rq[nr].i = r;
+                nr++;
+            }
+        qsort(rq, (size_t)nr, sizeof(route_item), cmp_route);
+        /* exclusive-hot instances of f by (latency, index); the time-sharing instance */
+        int nh = 0, ts = -1;
+        route_item *hot = (route_item *)malloc(sizeof(route_item) * (size_t)(n_inst > 0 ? n_inst : 1));
+        for (int i = 0; i < n_inst; i++) {
+            if ((int)inst_func[i] != f) continue;
+            if (inst_state[i] == ST_EXCL_HOT) {
+                hot[nh].a = inst_lat[i];
+                hot[nh].b = (uint32_t)i;
+                hot[nh].i = i;
+                nh++;
+            } else if ((inst_state[i] == ST_TIME_SHARING || inst_state[i] == ST_WARM) && ts < 0) {
+                ts = i;
+            }
+        }
+        qsort(hot, (size_t)nh, sizeof(route_item), cmp_route);
+        int h = 0;
+        uint64_t used = 0;
+        for (int j = 0; j < nr; j++) {
+            while (h < nh && used >= inst_cap[hot[h].i]) {
+                h++;
+                used = 0;
+            }
+            if (h < nh) {
+                route[rq[j].i] = hot[h].i;
+                used++;
+            } else {
+                route[rq[j].i] = ts;
+            }
+        }
+        free(rq);
+        free(hot);
+    }
+    for (int r = 0; r < a->R; r++)
+        if (a->req_func[r] >= (uint32_t)a->F) route[r] = -1;
+    return 0;
+}
