@@ -262,6 +262,19 @@ ffs_status ffs_plan_ranked(ffs_ctx *ctx, const ffs_request *d_req, const uint32_
 ffs_status ffs_plan_joint(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
                           uint32_t k_max, ffs_plan *d_out, uint32_t *rounds, void *stream);
 
+/* ---- NEXT-2 (routing): heterogeneity-aware request routing ---------------------
+ * Per function, requests in ascending adjusted deadline (R28) are directed to the
+ * function's exclusive-hot instances (d_state[i] == FFS_ST_EXCL_HOT, e.g. from
+ * ffs_evict_scores) in ascending (latency d_lat_us[i], index), each taking up to
+ * d_capacity[i] requests; the remaining requests go to the function's time-sharing
+ * instance (lowest index in state TIME_SHARING or WARM), -1 if none (R30).
+ * d_route[r] = instance index or -1 (also for func >= n_funcs).  Uses context scratch
+ * (stable radix sorts); asynchronous.  FFS_ERR_RANGE: n_req or n_inst >= 2^31,
+ * n_funcs >= 2^22. */
+ffs_status ffs_route(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                     const ffs_instance *d_inst, const uint8_t *d_state, const uint32_t *d_lat_us,
+                     const uint32_t *d_capacity, uint32_t n_inst, int32_t *d_route, void *stream);
+
 /* ---- NEXT-3: frontier precompute ------------------------------------------------------
  * For a fixed (function, node free-vector) the feasible set depends on the budget only
  * through e2e <= B, so the argmin for any B is the lowest-key point of the Pareto

@@ -65,6 +65,8 @@ struct ffs_ctx {
   std::vector<uint8_t> h_busy, h_cnt;
   std::vector<uint64_t> h_node_free;
   DevBuf node_off, j_keys, j_state, j_dirty, j_sreq, j_sslo, j_skeys, j_win, j_busy, j_cnt, j_free, j_ctr;
+  // NEXT-2 routing scratch
+  DevBuf r_k, r_k2, r_v, r_v2, i_k, i_k2, i_v, i_v2, i_cum, r_f, r_h, r_n, r_ts, r_hist, r_bsum;
   // NEXT-3 frontiers
   DevBuf f_nodefv, f_fvnode, f_act, f_next, f_budget, f_greq, f_gslo, f_gkeys, f_cnt, f_key, f_e2e, f_ctr;
   bool front_built = false;
@@ -142,6 +144,9 @@ void ffs_destroy(ffs_ctx* c) {
     DeviceGuard g(c->device);
     for (auto& e : c->ev)
       if (e) cudaEventDestroy(e);
+    for (DevBuf* b : {&c->r_k, &c->r_k2, &c->r_v, &c->r_v2, &c->i_k, &c->i_k2, &c->i_v, &c->i_v2, &c->i_cum, &c->r_f,
+                      &c->r_h, &c->r_n, &c->r_ts, &c->r_hist, &c->r_bsum})
+      b->release();
     for (DevBuf* b : {&c->f_nodefv, &c->f_fvnode, &c->f_act, &c->f_next, &c->f_budget, &c->f_greq, &c->f_gslo,
                       &c->f_gkeys, &c->f_cnt, &c->f_key, &c->f_e2e, &c->f_ctr})
       b->release();
@@ -704,6 +709,65 @@ ffs_status ffs_plan_joint(ffs_ctx* c, const ffs_request* d_req, const uint32_t* 
     n_sub = ctr[1];
   }
   if (rounds) *rounds = nr;
+  return FFS_OK;
+}
+
+ffs_status ffs_route(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                     const ffs_instance* d_inst, const uint8_t* d_state, const uint32_t* d_lat, const uint32_t* d_cap,
+                     uint32_t n_inst, int32_t* d_route, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  if (n_req == 0) return FFS_OK;
+  if (n_req >= (1u << 31) || n_inst >= (1u << 31)) return fail(c, FFS_ERR_RANGE, "n_req/n_inst >= 2^31");
+  if (c->F >= (1u << 22)) return fail(c, FFS_ERR_RANGE, "n_funcs >= 2^22");
+  if (!d_req || !d_slo || !d_route || (n_inst && (!d_inst || !d_state || !d_lat || !d_cap)))
+    return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  const size_t R = n_req, I = std::max(1u, n_inst), F1 = c->F + 1;
+  for (DevBuf* b : {&c->r_k, &c->r_k2}) CK(b->ensure(R * 8), "cudaMalloc");
+  for (DevBuf* b : {&c->r_v, &c->r_v2}) CK(b->ensure(R * 4), "cudaMalloc");
+  for (DevBuf* b : {&c->i_k, &c->i_k2}) CK(b->ensure(I * 8), "cudaMalloc");
+  for (DevBuf* b : {&c->i_v, &c->i_v2}) CK(b->ensure(I * 4), "cudaMalloc");
+  CK(c->i_cum.ensure((I + 1) * 8), "cudaMalloc");
+  for (DevBuf* b : {&c->r_f, &c->r_h, &c->r_n, &c->r_ts}) CK(b->ensure(F1 * 4), "cudaMalloc");
+  const size_t nmax = std::max<size_t>(R, I);
+  const size_t hist = 256 * ((nmax + 2047) / 2048) + 1;
+  CK(c->r_hist.ensure(hist * 8), "cudaMalloc");
+  CK(c->r_bsum.ensure(((hist + 2047) / 2048 + 1) * 8), "cudaMalloc");
+  RouteArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.req = d_req;
+  a.slo = d_slo;
+  a.n_req = n_req;
+  a.n_inst = n_inst;
+  a.inst = d_inst;
+  a.state = d_state;
+  a.lat = d_lat;
+  a.cap = d_cap;
+  a.rkey = c->r_k.as<uint64_t>();
+  a.rval = c->r_v.as<uint32_t>();
+  a.ikey = c->i_k.as<uint64_t>();
+  a.ival = c->i_v.as<uint32_t>();
+  a.icum = a.icap = c->i_cum.as<uint64_t>();
+  a.first_req = c->r_f.as<uint32_t>();
+  a.first_hot = c->r_h.as<uint32_t>();
+  a.n_hot = c->r_n.as<uint32_t>();
+  a.ts = c->r_ts.as<int32_t>();
+  a.route = d_route;
+  int fb = 1;
+  while ((1u << fb) <= c->F) ++fb;  // bits of the function id (F means "invalid")
+  CK(launch_route(0, a, st), "route keys");
+  CK(radix_sort_pairs(a.rkey, a.rval, c->r_k2.as<uint64_t>(), c->r_v2.as<uint32_t>(), n_req, 34 + fb,
+                      c->r_hist.as<uint64_t>(), c->r_bsum.as<uint64_t>(), st), "sort requests");
+  if (n_inst)
+    CK(radix_sort_pairs(a.ikey, a.ival, c->i_k2.as<uint64_t>(), c->i_v2.as<uint32_t>(), n_inst, 33 + fb,
+                        c->r_hist.as<uint64_t>(), c->r_bsum.as<uint64_t>(), st), "sort instances");
+  CK(cudaMemsetAsync(a.icum + n_inst, 0, 8, st), "memset");
+  CK(launch_route(1, a, st), "route marks");
+  CK(scan_u64(a.icum, (uint64_t)n_inst + 1, c->r_bsum.as<uint64_t>(), st), "capacity scan");
+  CK(launch_route(2, a, st), "route assign");
   return FFS_OK;
 }
 

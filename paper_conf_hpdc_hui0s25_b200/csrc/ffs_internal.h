@@ -153,6 +153,31 @@ struct FrontierArgs {
   ffs_plan* out;
 };
 cudaError_t launch_frontier(int phase, const FrontierArgs& a, uint32_t n, cudaStream_t st);
+
+struct RouteArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  uint32_t n_req, n_inst;
+  const ffs_instance* inst;
+  const uint8_t* state;
+  const uint32_t* lat;
+  const uint32_t* cap;
+  uint64_t* rkey; uint32_t* rval;   // requests: (func, adjusted deadline) -> index, sorted
+  uint64_t* ikey; uint32_t* ival;   // instances: (func, not-hot, latency) -> index, sorted
+  uint64_t* icum;                   // [n_inst+1] exclusive prefix of hot capacities (sorted order)
+  uint64_t* icap;                   // alias of icum before the scan
+  uint32_t* first_req;              // [F+1]
+  uint32_t* first_hot;              // [F+1]
+  uint32_t* n_hot;                  // [F+1]
+  int32_t* ts;                      // [F+1]
+  int32_t* route;
+};
+cudaError_t launch_route(int phase, const RouteArgs& a, cudaStream_t st);
+cudaError_t radix_sort_pairs(uint64_t* key, uint32_t* val, uint64_t* key2, uint32_t* val2, uint32_t n, int bits,
+                             uint64_t* hist, uint64_t* bsum, cudaStream_t st);
+cudaError_t scan_u64(uint64_t* a, uint64_t len, uint64_t* bsum, cudaStream_t st);
 cudaError_t launch_front_gather(const FrontierArgs& a, uint32_t n, const uint32_t* fv_node, uint32_t* gslo,
                                 cudaStream_t st);
 

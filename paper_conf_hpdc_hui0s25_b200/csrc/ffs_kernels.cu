@@ -12,6 +12,7 @@
 // K5  k_int_peak                 integer issue-rate microbenchmark (roofline denominator)
 //
 // Paper: FluidFaaS, HPDC '25.  P:<line> = line of PAPER.md; R<n> = DESIGN.md §3 reading.
+#include <algorithm>
 #include <cstdio>
 
 #include "ffs_internal.h"
@@ -1544,6 +1545,188 @@ cudaError_t launch_frontier(int phase, const FrontierArgs& a, uint32_t n, cudaSt
 cudaError_t launch_front_gather(const FrontierArgs& a, uint32_t n, const uint32_t* fv_node, uint32_t* gslo,
                                 cudaStream_t st) {
   if (n) k_front_gather<<<(n + 255) / 256, 256, 0, st>>>(a, n, fv_node, gslo);
+  return cudaGetLastError();
+}
+
+// ====================================================================================
+// Stable LSD radix sort of (u64 key, u32 value) pairs, 8-bit digits (NEXT-2 routing)
+// ====================================================================================
+constexpr int kRsT = 256, kRsWarps = kRsT / 32, kRsItems = 8, kRsTile = kRsT * kRsItems;  // 2048
+
+// per (digit, block) counts, digit-major so that one exclusive scan gives stable offsets
+__global__ void __launch_bounds__(kRsT) k_rs_hist(const uint64_t* __restrict__ key, uint32_t n, int shift,
+                                                   uint64_t* __restrict__ hist, uint32_t nb) {
+  __shared__ uint32_t h[256];
+  h[threadIdx.x] = 0;
+  __syncthreads();
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile;
+  for (int i = threadIdx.x; i < kRsTile; i += kRsT)
+    if (base + i < n) atomicAdd(&h[(key[base + i] >> shift) & 255u], 1u);
+  __syncthreads();
+  hist[(uint64_t)threadIdx.x * nb + blockIdx.x] = h[threadIdx.x];
+}
+
+// stable scatter: warp w owns the contiguous quarter-chunk [w*256, (w+1)*256) of the tile
+__global__ void __launch_bounds__(kRsT) k_rs_scatter(const uint64_t* __restrict__ key, const uint32_t* __restrict__ val,
+                                                      uint32_t n, int shift, const uint64_t* __restrict__ off,
+                                                      uint32_t nb, uint64_t* __restrict__ key_out,
+                                                      uint32_t* __restrict__ val_out) {
+  __shared__ uint32_t wh[kRsWarps][256];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int d = threadIdx.x; d < kRsWarps * 256; d += kRsT) (&wh[0][0])[d] = 0;
+  __syncthreads();
+  const uint64_t base = (uint64_t)blockIdx.x * kRsTile + (uint64_t)w * (32 * kRsItems);
+  // pass 1: per-warp digit counts
+  for (int it = 0; it < kRsItems; ++it) {
+    const uint64_t i = base + it * 32 + lane;
+    const bool in = i < n;
+    const uint32_t d = in ? (uint32_t)((key[i] >> shift) & 255u) : 256u + lane;
+    const uint32_t m = __match_any_sync(0xffffffffu, d);
+    if (in && lane == __ffs(m) - 1) wh[w][d] += __popc(m);
+  }
+  __syncthreads();
+  // exclusive prefix over warps per digit, plus the global offset of (digit, block)
+  {
+    const uint32_t d = threadIdx.x;  // kRsT == 256 digits
+    uint32_t run = (uint32_t)off[(uint64_t)d * nb + blockIdx.x];
+    for (int ww = 0; ww < kRsWarps; ++ww) {
+      const uint32_t c = wh[ww][d];
+      wh[ww][d] = run;
+      run += c;
+    }
+  }
+  __syncthreads();
+  // pass 2: scatter in order
+  for (int it = 0; it < kRsItems; ++it) {
+    const uint64_t i = base + it * 32 + lane;
+    const bool in = i < n;
+    const uint64_t k = in ? key[i] : 0;
+    const uint32_t d = in ? (uint32_t)((k >> shift) & 255u) : 256u + lane;
+    const uint32_t m = __match_any_sync(0xffffffffu, d);
+    if (in) {
+      const uint32_t pos = wh[w][d] + __popc(m & ((1u << lane) - 1));
+      key_out[pos] = k;
+      val_out[pos] = val[i];
+    }
+    __syncwarp();
+    if (in && lane == __ffs(m) - 1) wh[w][d] += __popc(m);
+    __syncwarp();
+  }
+}
+
+// sorts (key, val) by the low `bits` bits of key, stably; result in key/val (ping-pong
+// through key2/val2); hist needs 256 * ceil(n / 2048) + 1 entries, bsum scan scratch
+cudaError_t radix_sort_pairs(uint64_t* key, uint32_t* val, uint64_t* key2, uint32_t* val2, uint32_t n, int bits,
+                             uint64_t* hist, uint64_t* bsum, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  const uint32_t nb = (n + kRsTile - 1) / kRsTile;
+  const uint64_t len = (uint64_t)256 * nb;
+  const uint32_t sb = (uint32_t)((len + kScanChunk - 1) / kScanChunk);
+  for (int shift = 0; shift < bits; shift += 8) {
+    k_rs_hist<<<nb, kRsT, 0, st>>>(key, n, shift, hist, nb);
+    k_scan_reduce<<<dim3(sb, 1), kScanT, 0, st>>>(hist, len, bsum, sb);
+    k_scan_top<<<1, kScanT, 0, st>>>(bsum, sb);
+    k_scan_apply<<<dim3(sb, 1), kScanT, 0, st>>>(hist, len, bsum, sb);
+    k_rs_scatter<<<nb, kRsT, 0, st>>>(key, val, n, shift, hist, nb, key2, val2);
+    uint64_t* tk = key; key = key2; key2 = tk;
+    uint32_t* tv = val; val = val2; val2 = tv;
+  }
+  // an odd number of passes leaves the result in the second buffers: copy back
+  if (((bits + 7) / 8) & 1) {
+    cudaMemcpyAsync(key2, key, (size_t)n * 8, cudaMemcpyDeviceToDevice, st);
+    cudaMemcpyAsync(val2, val, (size_t)n * 4, cudaMemcpyDeviceToDevice, st);
+  }
+  return cudaGetLastError();
+}
+
+// ====================================================================================
+// K9 (NEXT-2 routing)
+// ====================================================================================
+__global__ void k_route_keys(const __grid_constant__ RouteArgs A) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < A.n_req) {
+    const ffs_request q = A.req[i];
+    const uint32_t f = q.func < A.lay.F ? q.func : A.lay.F;  // invalid functions sort last
+    const uint64_t adj = q.func < A.lay.F ? (joint_order(A.image, A.lay, q, A.slo[i], 0) >> 31) : 0;
+    A.rkey[i] = ((uint64_t)f << 34) | adj;  // adj < 2^34 (joint_order biases it non-negative)
+    A.rval[i] = i;
+    A.route[i] = -1;
+  }
+  if (i < A.n_inst) {
+    const uint32_t f = A.inst[i].func < A.lay.F ? A.inst[i].func : A.lay.F;
+    const bool hot = A.state[i] == FFS_ST_EXCL_HOT;
+    // non-hot instances sort after every hot one of their function
+    A.ikey[i] = ((uint64_t)f << 33) | ((uint64_t)(hot ? 0u : 1u) << 32) | A.lat[i];
+    A.ival[i] = i;
+  }
+  if (i <= A.lay.F) {
+    A.first_req[i] = 0xFFFFFFFFu;
+    A.first_hot[i] = 0xFFFFFFFFu;
+    A.n_hot[i] = 0;
+    A.ts[i] = 0x7FFFFFFF;
+  }
+}
+
+__global__ void k_route_marks(const __grid_constant__ RouteArgs A) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < A.n_req) atomicMin(A.first_req + (uint32_t)(A.rkey[i] >> 34), i);
+  if (i < A.n_inst) {
+    const uint32_t j = A.ival[i];  // sorted position i holds instance j
+    const uint32_t f = (uint32_t)(A.ikey[i] >> 33);
+    if (f < A.lay.F) {
+      if (A.state[j] == FFS_ST_EXCL_HOT) {
+        atomicMin(A.first_hot + f, i);
+        atomicAdd(A.n_hot + f, 1u);
+        A.icap[i] = A.cap[j];
+      } else {
+        A.icap[i] = 0;
+        if (A.state[j] == FFS_ST_TIME_SHARING || A.state[j] == FFS_ST_WARM) atomicMin(A.ts + f, (int32_t)j);
+      }
+    } else {
+      A.icap[i] = 0;
+    }
+  }
+}
+
+// request at sorted position i with rank j within its function: the instance whose
+// cumulative capacity range covers j, else the time-sharing instance
+__global__ void k_route_assign(const __grid_constant__ RouteArgs A) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= A.n_req) return;
+  const uint32_t f = (uint32_t)(A.rkey[i] >> 34);
+  const uint32_t r = A.rval[i];
+  if (f >= A.lay.F) return;
+  const uint64_t j = i - A.first_req[f];
+  int32_t out = A.ts[f] == 0x7FFFFFFF ? -1 : A.ts[f];
+  const uint32_t h0 = A.first_hot[f], nh = A.n_hot[f];
+  if (nh) {
+    const uint64_t c0 = A.icum[h0];
+    if (j < A.icum[h0 + nh] - c0) {
+      uint32_t lo = 0, hi = nh;  // first l with icum[h0 + l + 1] - c0 > j
+      while (lo < hi) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (A.icum[h0 + mid + 1] - c0 > j) hi = mid; else lo = mid + 1;
+      }
+      out = (int32_t)A.ival[h0 + lo];
+    }
+  }
+  A.route[r] = out;
+}
+
+cudaError_t launch_route(int phase, const RouteArgs& a, cudaStream_t st) {
+  const uint32_t n = std::max(std::max(a.n_req, a.n_inst), a.lay.F + 1);
+  const uint32_t T = 256;
+  if (phase == 0) k_route_keys<<<(n + T - 1) / T, T, 0, st>>>(a);
+  if (phase == 1) k_route_marks<<<(n + T - 1) / T, T, 0, st>>>(a);
+  if (phase == 2 && a.n_req) k_route_assign<<<(a.n_req + T - 1) / T, T, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t scan_u64(uint64_t* a, uint64_t len, uint64_t* bsum, cudaStream_t st) {
+  const uint32_t sb = (uint32_t)((len + kScanChunk - 1) / kScanChunk);
+  k_scan_reduce<<<dim3(sb, 1), kScanT, 0, st>>>(a, len, bsum, sb);
+  k_scan_top<<<1, kScanT, 0, st>>>(bsum, sb);
+  k_scan_apply<<<dim3(sb, 1), kScanT, 0, st>>>(a, len, bsum, sb);
   return cudaGetLastError();
 }
 

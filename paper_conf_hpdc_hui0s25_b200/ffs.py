@@ -61,6 +61,7 @@ _sig = {
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_plan_joint": ([_vp, _vp, _vp, _u32, _u32, _vp, C.POINTER(C.c_uint32), _vp], _i32),
+    "ffs_route": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_frontier_build": ([_vp, _u32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32), _vp], _i32),
     "ffs_plan_frontier": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_rank_partitions": ([_vp, _u32, _u32], _i32),
@@ -231,6 +232,16 @@ class Planner:
         self._check(_lib.ffs_plan_joint(self._h, _ptr(req), _ptr(slo), n, int(k_max), _ptr(out), C.byref(rounds),
                                         _stream(stream)))
         return out, int(rounds.value)
+
+    # ---- NEXT-2: routing ------------------------------------------------------------
+    def route(self, req, slo, inst, state, lat_us, capacity, route=None, stream=None):
+        import torch
+        n = int(slo.numel())
+        n_inst = int(inst.numel() // W.INST_DTYPE.itemsize)
+        route = torch.empty(n, dtype=torch.int32, device=slo.device) if route is None else route
+        self._check(_lib.ffs_route(self._h, _ptr(req), _ptr(slo), n, _ptr(inst), _ptr(state), _ptr(lat_us),
+                                   _ptr(capacity), n_inst, _ptr(route), _stream(stream)))
+        return route
 
     # ---- NEXT-3: frontier precompute ---------------------------------------------------------
     def frontier_build(self, k_max: int, stream=None) -> tuple[int, int]:

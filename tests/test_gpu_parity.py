@@ -354,3 +354,37 @@ def test_next_rows_error_states(F):
         pl.plan_frontier(req, slo)
     assert e.value.status == F.FFS_ERR_STATE
     pl.close()
+
+
+# ---- NEXT-2: routing -------------------------------------------------------------
+def _route_case(prob, n_inst, seed):
+    rng = W.SplitMix64(seed)
+    func = rng.integers(0, prob.F - 1, n_inst).astype(np.uint32)
+    state = rng.integers(0, 3, n_inst).astype(np.uint8)
+    lat = rng.integers(1, 40, n_inst).astype(np.uint32)
+    cap = rng.integers(0, 30, n_inst).astype(np.uint32)
+    inst = np.zeros(n_inst, dtype=W.INST_DTYPE)
+    inst["func"] = func
+    return inst, state, lat, cap
+
+
+@pytest.mark.parametrize("cfg,n_inst", [("tiny", 9), ("C2", 40), ("C3", 3000), ("C4", 0)])
+def test_route_matches_oracle(F, planner, cfg, n_inst):
+    if cfg == "C4":
+        wl = W.config4(T=1)
+        prob = wl.problem
+        inst = wl.inst
+        _, state = oracle.evict(inst, int(wl.now_us[0]), 30, wl.window_us)
+        rng = W.SplitMix64(3)
+        lat = rng.integers(1, 100, len(inst)).astype(np.uint32)
+        cap = rng.integers(0, 3, len(inst)).astype(np.uint32)
+    else:
+        prob = {"tiny": lambda: random_tiny(1009), "C2": W.config2, "C3": W.config3}[cfg]()
+        inst, state, lat, cap = _route_case(prob, n_inst, 11)
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.uint8) if a.dtype == W.INST_DTYPE else a).cuda()
+    route = planner.route(req, slo, t(inst), t(state), t(lat.view(np.int32)), t(cap.view(np.int32)))
+    torch.cuda.synchronize()
+    exp = oracle.route(prob, inst["func"], state, lat, cap)
+    np.testing.assert_array_equal(route.cpu().numpy(), exp)
