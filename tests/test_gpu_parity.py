@@ -388,3 +388,74 @@ def test_route_matches_oracle(F, planner, cfg, n_inst):
     torch.cuda.synchronize()
     exp = oracle.route(prob, inst["func"], state, lat, cap)
     np.testing.assert_array_equal(route.cpu().numpy(), exp)
+
+
+def check_plan_properties(prob, p):
+    """Properties that hold at any size, checked on every request (vectorised numpy):
+    (a) ESG placement when a single free slice holds the function within the budget,
+    (d) e2e / bottleneck / cvq / gpcs recomputed from the tables, slices valid."""
+    R, P = prob.R, prob.P
+    f = prob.req["func"].astype(np.int64)
+    v = prob.req["node"].astype(np.int64)
+    B = prob.slo_us.astype(np.int64)
+    off = prob.comp_off.astype(np.int64)
+    n = off[f + 1] - off[f]
+    lat = prob.lat_us.astype(np.int64)
+    PL = np.zeros((lat.shape[0] + 1, P), np.int64)
+    PL[1:] = np.cumsum(lat, axis=0)
+    PM = np.concatenate([[0], np.cumsum(prob.mem_mib.astype(np.int64))])
+    sl = prob.slices
+    free = np.zeros((prob.n_nodes, P), np.int64)
+    np.add.at(free, (sl["node"][sl["busy"] == 0].astype(np.int64), sl["profile"][sl["busy"] == 0].astype(np.int64)), 1)
+    cap = prob.cap_mib.astype(np.int64)
+    g = prob.gpcs.astype(np.int64)
+    # (a) ESG placement
+    tot_mem = PM[off[f + 1]] - PM[off[f]]
+    tot_lat = PL[off[f + 1]] - PL[off[f]]                     # [R, P]
+    ok1 = (free[v] > 0) & (tot_mem[:, None] <= cap[None, :]) & (tot_lat <= B[:, None])
+    has = ok1.any(axis=1)
+    esg = np.where(ok1, g[None, :] * 16 + np.arange(P)[None, :], 10**9).argmin(axis=1)
+    assert (p["k"][has] == 1).all() and (p["prof"][has, 0] == esg[has]).all()
+    # (d) recompute every OK plan from the tables
+    ok = p["status"] == 0
+    k = p["k"].astype(np.int64)
+    mask = p["cut_mask"].astype(np.int64)
+    St = np.zeros(R, np.int64); Sq = np.zeros(R, np.int64); bott = np.zeros(R, np.int64)
+    X = np.zeros(R, np.int64); gp = np.zeros(R, np.int64)
+    a = np.zeros(R, np.int64); m = mask.copy()
+    used = np.zeros((R, P), np.int64)
+    for i in range(8):
+        live = ok & (i < k)
+        last = live & (i == k - 1)
+        low = m & -m
+        j = np.where(m > 0, np.log2(np.maximum(low, 1)).astype(np.int64), 0)
+        b = np.where(last, n, j + 1)
+        pr = np.where(live, p["prof"][:, i].astype(np.int64), 0)
+        t = np.where(live, PL[off[f] + b, pr] - PL[off[f] + a, pr], 0)
+        mem = np.where(live, PM[off[f] + b] - PM[off[f] + a], 0)
+        assert (mem[live] <= cap[pr[live]]).all()
+        X += np.where(live & ~last, prob.xfer_us[np.minimum(off[f] + j, len(prob.xfer_us) - 1)].astype(np.int64), 0)
+        St += t; Sq += t * t; bott = np.maximum(bott, t); gp += np.where(live, g[pr], 0)
+        np.add.at(used, (np.arange(R)[live], pr[live]), 1)
+        m = np.where(live & ~last, m & (m - 1), m)
+        a = np.where(live, b, a)
+    assert (p["e2e_us"][ok] == (St + X)[ok]).all() and (St + X <= B)[ok].all()
+    assert (p["bottleneck_us"][ok] == bott[ok]).all() and (p["gpcs"][ok] == gp[ok]).all()
+    D = St * St
+    Nn = k * Sq - D
+    cvq = np.where(ok, (Nn << 10) // np.maximum(D, 1), 0)
+    assert (p["cvq"][ok] == cvq[ok]).all() and ((p["key"][ok] >> 50) == cvq[ok]).all()
+    assert (used[ok] <= free[v[ok]]).all()
+    s = p["slice"][ok]
+    live = s >= 0
+    assert (sl["node"][s[live]] == np.repeat(v[ok], (live).sum(axis=1))).all()
+    assert (sl["busy"][s[live]] == 0).all()
+    assert (sl["profile"][s[live]] == p["prof"][ok][live]).all()
+
+
+def test_c5_full_batch_properties(F, planner):
+    prob = W.config5()
+    p, _, _ = run_gpu(F, planner, prob, verify=False)
+    check_plan_properties(prob, p)
+    ok = p["status"] == 0
+    assert ok.mean() > 0.5 and (ok & (p["k"] > 1)).mean() > 0.05 and (~ok).mean() > 0.05
