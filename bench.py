@@ -53,6 +53,15 @@ def segment_candidates(prob, k_max, rank, world):
     return out
 
 
+def _traffic(kernel):
+    """dram read+write bytes per launch of `kernel` from the committed ncu capture, or None."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
+            return json.load(fh).get(kernel)
+    except OSError:
+        return None
+
+
 def measured_peaks():
     try:
         with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
@@ -200,7 +209,7 @@ def run_c4(pl, steps: int, warmup: int, flush, peaks):
                         f"{n // len(wl.now_us)} instances, victims for {prob.R} loads",
             "kernels_ms": {"k_evict_ticks": t_sc, "k_victims": t_vi},
             "roofline": {"bound": "hbm", "kernel": "k_evict_ticks", "achieved": achieved, "peak": peak,
-                         "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "unit": "GB/s", "frac": achieved / peak, "traffic": _traffic("k_evict_ticks"),
                          "alg_bytes_per_score": 33, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)"},
             "l2": "flushed between steps"}
 
@@ -369,10 +378,7 @@ def main():
     max_mhz = float(peaks.get("sm_max_mhz", 1965.0))
     peak_ops = sm_count * 4 * 32 * max_mhz * 1e6  # issue-limited lane-ops/s
     achieved = seg_c[top - 1] * ALG_OPS / (top_ms * 1e-3)
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tpath):
-        traffic = json.load(open(tpath)).get(f"k_plan_search<{top}>")
+    traffic = _traffic(f"k_plan_search<{top}>")
 
     # e2e through the public host-buffer API (N = 1: ffs_plan_batch_host)
     e2e = None
