@@ -599,14 +599,22 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
     for (int x = 0; x < kP; ++x) {
       const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
       const uint32_t cap = c.sm[c.o_cap + x];
-      float v[2][4][5];
+      // memory folded once per (half, stage), then one select per multiplicity; the last
+      // stage is kept as SLO slack Blim - v3 (-INF when folded)
+      float v[2][4][4];
+      bool gate[4];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) gate[m] = fr > (uint32_t)m;
 #pragma unroll
       for (int h = 0; h < 2; ++h)
 #pragma unroll
-        for (int s = 0; s < 4; ++s)
+        for (int s = 0; s < 4; ++s) {
+          const float vm = (G[h].memst[s] <= cap) ? f[h][s][x] : INF;
+          const float base = (s == 3) ? G[h].blim - vm : vm;
+          const float none = (s == 3) ? -INF : INF;
 #pragma unroll
-          for (int m = 0; m <= s + 1 && m < 5; ++m)
-            v[h][s][m] = (G[h].memst[s] <= cap && fr > (uint32_t)m) ? f[h][s][x] : INF;
+          for (int m = 0; m <= s && m < 4; ++m) v[h][s][m] = gate[m] ? base : none;
+        }
       a1[x] = f2pack(al * (f[0][1][x] * f[0][1][x]), al * (f[1][1][x] * f[1][1][x]));
       a2[x] = f2pack(al * (f[0][2][x] * f[0][2][x]), al * (f[1][2][x] * f[1][2][x]));
       t2[x] = f2pack(f[0][3][x] + f[0][3][x], f[1][3][x] + f[1][3][x]);
@@ -621,10 +629,10 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
       r[2 * nb] = f2pack(v[0][2][0], v[1][2][0]);
       r[3 * nb] = f2pack(v[0][2][1], v[1][2][1]);
       r[4 * nb] = f2pack(v[0][2][2], v[1][2][2]);
-      r[5 * nb] = f2pack(G[0].blim - v[0][3][0], G[1].blim - v[1][3][0]);
-      r[6 * nb] = f2pack(G[0].blim - v[0][3][1], G[1].blim - v[1][3][1]);
-      r[7 * nb] = f2pack(G[0].blim - v[0][3][2], G[1].blim - v[1][3][2]);
-      r[8 * nb] = f2pack(G[0].blim - v[0][3][3], G[1].blim - v[1][3][3]);
+      r[5 * nb] = f2pack(v[0][3][0], v[1][3][0]);
+      r[6 * nb] = f2pack(v[0][3][1], v[1][3][1]);
+      r[7 * nb] = f2pack(v[0][3][2], v[1][3][2]);
+      r[8 * nb] = f2pack(v[0][3][3], v[1][3][3]);
       r[9 * nb] = f2pack(v[0][0][0], v[1][0][0]);
       r[10 * nb] = f2pack(a0A, a0B);
     }
