@@ -66,6 +66,7 @@ def lib():
             _lib.oracle_plan_joint.argtypes = [C.POINTER(_PlanArgs)]
             _lib.oracle_plan_joint.restype = C.c_int
             _lib.oracle_route.restype = C.c_int
+            _lib.oracle_sim.restype = C.c_int
             _lib.oracle_evict.restype = None
             _lib.oracle_victim.restype = None
     return _lib
@@ -170,6 +171,22 @@ def route(prob, inst_func, inst_state, inst_lat, inst_cap) -> np.ndarray:
     out = np.full(h.func.shape[0], -1, np.int32)
     lib().oracle_route(C.byref(h.args), C.c_int(int(fu.shape[0])), _p(fu), _p(st), _p(la), _p(ca), _p(out))
     return out
+
+
+def sim(trace, thr_pct: int = 30, cold_after_us: int = 600_000_000):
+    """NEXT-4 time-sharing simulator (ffs_oracle.c: oracle_sim).  Returns (ctr[N, 8],
+    slice[N, F], state[N, F], last_used[N, F], busy[N, F])."""
+    prob = trace.problem
+    h = _Held(prob, prob.k_max, False)
+    N, F = int(prob.n_nodes), int(prob.comp_off.shape[0] - 1)
+    off, fu, bu = _c(trace.req_off, np.uint32), _c(trace.req_func, np.uint32), _c(trace.req_budget, np.uint32)
+    ctr = np.zeros((N, 8), np.uint64)
+    fs, fst = np.zeros((N, F), np.int32), np.zeros((N, F), np.uint8)
+    fl, fb = np.zeros((N, F), np.uint64), np.zeros((N, F), np.uint32)
+    lib().oracle_sim(C.byref(h.args), C.c_int(trace.T), _p(off), _p(fu), _p(bu), C.c_uint64(trace.t0_us),
+                     C.c_uint32(trace.tick_us), C.c_uint32(trace.window_ticks), C.c_uint32(thr_pct),
+                     C.c_uint64(cold_after_us), _p(ctr), _p(fs), _p(fst), _p(fl), _p(fb))
+    return ctr, fs, fst, fl, fb
 
 
 def evict(inst: np.ndarray, now_us: int, util_thr_pct: int = 30, window_us: int = 10_000_000,

@@ -752,3 +752,152 @@ int oracle_route(const oracle_plan_args *a, int n_inst, const uint32_t *inst_fun
         if (a->req_func[r] >= (uint32_t)a->F) route[r] = -1;
     return 0;
 }
+
+/* ---- NEXT-4: time-sharing simulator (Fig. 8) -------------------------------
+ * DESIGN.md R31-R36.  Each node (invoker) is simulated independently; per node every
+ * function has at most one instance (created on its first request there, time-sharing).
+ * Ticks of tick_us; the requests of a tick are served in trace order:
+ *   resident instance            -> served, latency = exec on its slice's profile;
+ *   otherwise (warm / new)       -> placed on the free slice with the smallest (capacity,
+ *     gpcs, id) that holds the function, else on the slice of the least recently used
+ *     (ties: lower slice) time-sharing instance of another function not used in this tick
+ *     whose slice holds the function (the victim goes warm: "selects the least-recently-
+ *     used (LRU) instance for eviction, reloads the pertinent instance, and fulfills the
+ *     request"), latency = load + exec; otherwise unserved.  A served request is an
+ *     SLO hit when its latency <= its budget.
+ *   A served request adds exec to the instance's busy time and sets its last use to now.
+ * At the end of every tick the occupied slices are counted; every window_ticks the
+ * instances whose busy time reached thr% of the window become exclusive hot (exempt from
+ * eviction) for the next window, the others time-sharing, busy resets;
+ * instances idle >= cold_after are terminated.
+ * Slices busy in the staged cluster belong to other tenants and are never used.
+ * ctr[v][8] = requests, served, SLO hits, unserved, reloads, evictions, terminations,
+ * occupied slice-ticks.  Final per (node, function): slice, state, last use, busy. */
+int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const uint32_t *req_func,
+               const uint32_t *req_budget, uint64_t t0_us, uint32_t tick_us, uint32_t window_ticks,
+               uint32_t thr_pct, uint64_t cold_after_us, uint64_t *ctr, int32_t *fin_slice, uint8_t *fin_state,
+               uint64_t *fin_last, uint32_t *fin_busy) {
+    const int F = a->F, P = a->P;
+    /* per function: exec on each profile, total memory, reload */
+    uint64_t *exec = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)F * (size_t)P);
+    uint64_t *memt = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)F);
+    for (int f = 0; f < F; f++) {
+        int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+        memt[f] = 0;
+        for (int c = 0; c < n; c++) memt[f] += a->mem_mib[a->comp_off[f] + c];
+        for (int p = 0; p < P; p++) {
+            uint64_t t = 0;
+            for (int c = 0; c < n; c++) t += lat_of(a, f, c, p);
+            exec[(size_t)f * P + p] = t;
+        }
+    }
+    int *res = (int *)malloc(sizeof(int) * (size_t)(a->n_slices > 0 ? a->n_slices : 1));
+    for (int v = 0; v < a->n_nodes; v++) {
+        uint64_t *C = ctr + (size_t)v * 8;
+        for (int i = 0; i < 8; i++) C[i] = 0;
+        int32_t *sl = fin_slice + (size_t)v * F;
+        uint8_t *st = fin_state + (size_t)v * F;
+        uint64_t *last = fin_last + (size_t)v * F;
+        uint32_t *busy = fin_busy + (size_t)v * F;
+        uint8_t *exists = (uint8_t *)calloc((size_t)F, 1), *hot = (uint8_t *)calloc((size_t)F, 1);
+        for (int f = 0; f < F; f++) {
+            sl[f] = -1;
+            last[f] = 0;
+            busy[f] = 0;
+        }
+        for (int s = 0; s < a->n_slices; s++) res[s] = -1;
+        for (int t = 0; t < T; t++) {
+            uint64_t now = t0_us + (uint64_t)t * tick_us;
+            for (uint32_t j = req_off[(size_t)v * T + t]; j < req_off[(size_t)v * T + t + 1]; j++) {
+                int f = (int)req_func[j];
+                uint64_t B = req_budget[j];
+                C[0]++;
+                if (!exists[f]) {
+                    exists[f] = 1;
+                    sl[f] = -1;
+                    hot[f] = 0;
+                    busy[f] = 0;
+                    last[f] = now;
+                }
+                uint64_t latency = 0, ex = 0;
+                int ok = 0;
+                if (sl[f] >= 0) {
+                    ex = exec[(size_t)f * P + a->sl_prof[sl[f]]];
+                    latency = ex;
+                    ok = 1;
+                } else {
+                    int best = -1;
+                    for (int s = 0; s < a->n_slices; s++) {
+                        if (a->sl_node[s] != v || a->sl_busy[s] || res[s] >= 0) continue;
+                        int p = a->sl_prof[s];
+                        if (memt[f] > a->cap_mib[p]) continue;
+                        if (best < 0) {
+                            best = s;
+                            continue;
+                        }
+                        int q = a->sl_prof[best];
+                        if (a->cap_mib[p] < a->cap_mib[q] || (a->cap_mib[p] == a->cap_mib[q] && a->gpcs[p] < a->gpcs[q]))
+                            best = s;
+                    }
+                    if (best < 0) {
+                        for (int s = 0; s < a->n_slices; s++) {
+                            if (a->sl_node[s] != v || res[s] < 0 || res[s] == f) continue;
+                            int g = res[s], p = a->sl_prof[s];
+                            if (hot[g] || last[g] >= now) continue;
+                            if (memt[f] > a->cap_mib[p]) continue;
+                            if (best < 0 || last[g] < last[res[best]]) best = s;
+                        }
+                        if (best >= 0) {
+                            sl[res[best]] = -1; /* evicted to CPU memory: warm */
+                            res[best] = -1;
+                            C[5]++;
+                        }
+                    }
+                    if (best >= 0) {
+                        res[best] = f;
+                        sl[f] = best;
+                        C[4]++;
+                        ex = exec[(size_t)f * P + a->sl_prof[best]];
+                        latency = a->load_us[f] + ex;
+                        ok = 1;
+                    }
+                }
+                if (ok) {
+                    C[1]++;
+                    if (latency <= B) C[2]++;
+                    busy[f] += (uint32_t)ex;
+                    last[f] = now;
+                } else {
+                    C[3]++;
+                }
+            }
+            for (int s = 0; s < a->n_slices; s++)
+                if (a->sl_node[s] == v && res[s] >= 0) C[7]++;
+            if ((uint32_t)(t + 1) % window_ticks == 0) {
+                uint64_t window_us = (uint64_t)window_ticks * tick_us;
+                for (int f = 0; f < F; f++) {
+                    hot[f] = (uint64_t)busy[f] * 100u >= (uint64_t)thr_pct * window_us;
+                    busy[f] = 0;
+                }
+            }
+            for (int f = 0; f < F; f++) {
+                if (exists[f] && now - last[f] >= cold_after_us) {
+                    if (sl[f] >= 0) res[sl[f]] = -1;
+                    exists[f] = 0;
+                    sl[f] = -1;
+                    hot[f] = 0;
+                    busy[f] = 0;
+                    C[6]++;
+                }
+            }
+        }
+        for (int f = 0; f < F; f++)
+            st[f] = !exists[f] ? ST_COLD : (sl[f] < 0 ? ST_WARM : (hot[f] ? ST_EXCL_HOT : ST_TIME_SHARING));
+        free(exists);
+        free(hot);
+    }
+    free(res);
+    free(exec);
+    free(memt);
+    return 0;
+}

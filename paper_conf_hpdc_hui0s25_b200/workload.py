@@ -422,3 +422,55 @@ def config4(seed: int | None = None, T: int = 4096, n_funcs: int = 200) -> Evict
 
 
 CONFIGS = {1: config1, 2: config2, 3: config3, 5: config5}
+
+
+# ----------------------------------------------------------------------------------
+# NEXT-4: request trace for the time-sharing simulator
+# ----------------------------------------------------------------------------------
+@dataclass
+class SimTrace:
+    problem: Problem           # profile table + cluster (busy slices are other tenants)
+    req_off: np.ndarray        # uint32 [n_nodes * T + 1] CSR: requests of (node, tick)
+    req_func: np.ndarray       # uint32 [n_req]
+    req_budget: np.ndarray     # uint32 [n_req] latency budget (SLO) of the request
+    T: int
+    tick_us: int = 100_000
+    window_ticks: int = 100    # 10 s utilisation window
+    t0_us: int = 1_000_000_000
+
+
+def sim_trace(seed: int | None = None, T: int = 4096, n_funcs: int = 200, nodes=None,
+              rate_scale: float = 1.0) -> SimTrace:
+    """Azure-shaped arrivals: Zipf(1) function popularity, per (node,
+    function) bursty on/off Poisson rates; budgets = SLO_f."""
+    rng = SplitMix64(SEED_BASE + 6 if seed is None else seed)
+    node_parts = NODE_BLOCK * 4 if nodes is None else nodes
+    lengths = rng.sub(9).integers(3, 12, n_funcs)
+    base = _problem("SIM", rng, lengths, node_parts, 1, rho_range=(0.2, 0.6))
+    N = base.n_nodes
+    r = rng.sub(7)
+    pop = (np.arange(1, n_funcs + 1, dtype=np.float64) ** -1.0)
+    pop = pop[np.argsort(r.u64(n_funcs))]
+    lam = 0.05 * rate_scale * pop / pop.max()                       # requests per tick per node
+    on = r.uniform(N * n_funcs).reshape(N, n_funcs) < 0.5
+    # bursty: a function alternates on/off phases of 30..300 ticks per node
+    phase = r.integers(30, 300, N * n_funcs).reshape(N, n_funcs)
+    counts = np.zeros((N, T), dtype=np.int64)
+    funcs_per = [[None] * T for _ in range(N)]
+    u = r.uniform(N * T * n_funcs).reshape(N, T, n_funcs)
+    for t in range(T):
+        flip = (t % phase) == 0
+        on = np.where(flip & (t > 0), ~on, on)
+        p = np.where(on, lam[None, :] * 3.0, lam[None, :] * 0.2)      # on: 3x, off: 0.2x
+        hit = u[:, t, :] < p
+        for v in range(N):
+            fs = np.nonzero(hit[v])[0]
+            funcs_per[v][t] = fs
+            counts[v, t] = fs.shape[0]
+    req_off = np.zeros(N * T + 1, dtype=np.uint32)
+    req_off[1:] = np.cumsum(counts.reshape(-1))
+    req_func = np.concatenate([funcs_per[v][t] for v in range(N) for t in range(T)]).astype(np.uint32) \
+        if req_off[-1] else np.zeros(0, np.uint32)
+    slo_f = base.meta["slo_f"]
+    req_budget = slo_f[req_func].astype(np.uint32)
+    return SimTrace(problem=base, req_off=req_off, req_func=req_func, req_budget=req_budget, T=T)
