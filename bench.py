@@ -288,6 +288,28 @@ def run_frontier(pl, prob, req, slo, steps: int, warmup: int, flush):
                     "not per request (not comparable to candidates/s)"}
 
 
+def run_sim(pl):
+    """NEXT-4: the time-sharing simulator on the C4 cluster, 8192 ticks (13.7 simulated
+    minutes, so 10-minute cold terminations occur); one kernel, device-timed."""
+    import torch
+    tr = W.sim_trace(T=8192)
+    pl.stage(tr.problem)
+    pl.simulate(tr)  # warm-up
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    ctr, *_ = pl.simulate(tr)
+    b.record()
+    torch.cuda.synchronize()
+    ms = a.elapsed_time(b)
+    c = ctr.cpu().numpy().sum(axis=0)
+    return {"metric": "simulated_requests_per_s", "value": float(c[0]) / (ms * 1e-3), "unit": "requests/s",
+            "ms": ms, "ticks": tr.T, "nodes": int(tr.problem.n_nodes), "functions": int(tr.problem.F),
+            "requests": int(c[0]), "served": int(c[1]), "slo_hit_rate": float(c[2]) / max(1, int(c[0])),
+            "reloads": int(c[4]), "evictions": int(c[5]), "cold_terminations": int(c[6]),
+            "slice_ticks_occupied": int(c[7])}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -423,9 +445,10 @@ def main():
     if world == 1 and not args.no_c4:
         joint = run_joint(pl, prob, req, slo)
         frontier = run_frontier(pl, prob, req, slo, args.steps, args.warmup, flush)
-    c4 = None
+    c4 = sim = None
     if world == 1 and not args.no_c4:
         c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
+        sim = run_sim(pl)
     if rank == 0:
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
@@ -454,6 +477,7 @@ def main():
             "ranked_first_fit": ranked,
             "joint_commit": joint,
             "frontier": frontier,
+            "timeshare_sim": sim,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

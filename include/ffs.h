@@ -275,6 +275,26 @@ ffs_status ffs_route(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_s
                      const ffs_instance *d_inst, const uint8_t *d_state, const uint32_t *d_lat_us,
                      const uint32_t *d_capacity, uint32_t n_inst, int32_t *d_route, void *stream);
 
+/* ---- NEXT-4: time-sharing simulator (Fig. 8) --------------------------------
+ * Simulates n_ticks ticks of tick_us on the staged cluster (slices busy in the staged
+ * state belong to other tenants).  Per node every function has at most one instance;
+ * the requests of node v and tick t are d_req_func/d_req_budget[d_req_off[v*n_ticks+t] ..
+ * d_req_off[v*n_ticks+t+1]) and are served in that order: a resident instance serves
+ * (latency = its execution time on its slice); otherwise the instance is loaded on the
+ * free slice of smallest (capacity, gpcs, id) that holds the function, else on the slice
+ * of the least-recently-used time-sharing instance of another function not used in this
+ * tick (evicted to warm), latency = reload + execution; otherwise the request is
+ * unserved.  Every window_ticks an instance becomes exclusive hot (not evictable) iff its
+ * busy time reached thr_pct % of the window; instances idle >= cold_after_us terminate
+ * (R31-R36).  Outputs (device): d_ctr uint64[n_nodes][8] = requests, served,
+ * SLO hits, unserved, reloads, evictions, terminations, occupied slice-ticks; final
+ * per (node, function): d_slice int32, d_state uint8 (FFS_ST_*), d_last uint64,
+ * d_busy uint32 (all [n_nodes][n_funcs]).  Asynchronous. */
+ffs_status ffs_simulate(ffs_ctx *ctx, const uint32_t *d_req_off, const uint32_t *d_req_func,
+                        const uint32_t *d_req_budget, uint32_t n_ticks, uint64_t t0_us, uint32_t tick_us,
+                        uint32_t window_ticks, uint32_t thr_pct, uint64_t cold_after_us, uint64_t *d_ctr,
+                        int32_t *d_slice, uint8_t *d_state, uint64_t *d_last, uint32_t *d_busy, void *stream);
+
 /* ---- NEXT-3: frontier precompute ------------------------------------------------------
  * For a fixed (function, node free-vector) the feasible set depends on the budget only
  * through e2e <= B, so the argmin for any B is the lowest-key point of the Pareto

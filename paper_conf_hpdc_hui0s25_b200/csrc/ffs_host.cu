@@ -67,6 +67,8 @@ struct ffs_ctx {
   DevBuf node_off, j_keys, j_state, j_dirty, j_sreq, j_sslo, j_skeys, j_win, j_busy, j_cnt, j_free, j_ctr;
   // NEXT-2 routing scratch
   DevBuf r_k, r_k2, r_v, r_v2, i_k, i_k2, i_v, i_v2, i_cum, r_f, r_h, r_n, r_ts, r_hist, r_bsum;
+  // NEXT-4 simulator scratch
+  DevBuf s_res, s_flags, s_busy;
   // NEXT-3 frontiers
   DevBuf f_nodefv, f_fvnode, f_act, f_next, f_budget, f_greq, f_gslo, f_gkeys, f_cnt, f_key, f_e2e, f_ctr;
   bool front_built = false;
@@ -144,6 +146,7 @@ void ffs_destroy(ffs_ctx* c) {
     DeviceGuard g(c->device);
     for (auto& e : c->ev)
       if (e) cudaEventDestroy(e);
+    for (DevBuf* b : {&c->s_res, &c->s_flags, &c->s_busy}) b->release();
     for (DevBuf* b : {&c->r_k, &c->r_k2, &c->r_v, &c->r_v2, &c->i_k, &c->i_k2, &c->i_v, &c->i_v2, &c->i_cum, &c->r_f,
                       &c->r_h, &c->r_n, &c->r_ts, &c->r_hist, &c->r_bsum})
       b->release();
@@ -768,6 +771,51 @@ ffs_status ffs_route(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo
   CK(launch_route(1, a, st), "route marks");
   CK(scan_u64(a.icum, (uint64_t)n_inst + 1, c->r_bsum.as<uint64_t>(), st), "capacity scan");
   CK(launch_route(2, a, st), "route assign");
+  return FFS_OK;
+}
+
+ffs_status ffs_simulate(ffs_ctx* c, const uint32_t* d_req_off, const uint32_t* d_req_func,
+                        const uint32_t* d_req_budget, uint32_t n_ticks, uint64_t t0_us, uint32_t tick_us,
+                        uint32_t window_ticks, uint32_t thr_pct, uint64_t cold_after_us, uint64_t* d_ctr,
+                        int32_t* d_slice, uint8_t* d_state, uint64_t* d_last, uint32_t* d_busy, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  if (n_ticks == 0) return FFS_OK;
+  if (!d_req_off || !d_req_func || !d_req_budget || !d_ctr || !d_slice || !d_state || !d_last || !d_busy)
+    return fail(c, FFS_ERR_ARG, "null device pointer");
+  if (window_ticks == 0 || tick_us == 0) return fail(c, FFS_ERR_ARG, "window_ticks and tick_us must be > 0");
+  if (c->n_slices >= (1u << 20)) return fail(c, FFS_ERR_RANGE, "n_slices >= 2^20");
+  DeviceGuard g(c->device);
+  CK(c->s_res.ensure((size_t)std::max(1u, c->n_slices) * 4), "cudaMalloc");
+  CK(c->s_flags.ensure((size_t)c->n_nodes * c->F), "cudaMalloc");
+  CK(c->s_busy.ensure(std::max<size_t>(1, c->n_slices)), "cudaMalloc");
+  if (c->n_slices)
+    CK(cudaMemcpyAsync(c->s_busy.p, c->h_busy.data(), c->n_slices, cudaMemcpyHostToDevice, (cudaStream_t)stream),
+       "H2D busy");
+  SimArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.n_nodes = c->n_nodes;
+  a.n_ticks = n_ticks;
+  a.window_ticks = window_ticks;
+  a.thr_pct = thr_pct;
+  a.tick_us = tick_us;
+  a.t0_us = t0_us;
+  a.cold_after_us = cold_after_us;
+  a.node_off = c->node_off.as<uint32_t>();
+  a.slice_prof = c->slice_prof.as<uint8_t>();
+  a.slice_busy = c->s_busy.as<uint8_t>();
+  a.req_off = d_req_off;
+  a.req_func = d_req_func;
+  a.req_budget = d_req_budget;
+  a.res = c->s_res.as<int32_t>();
+  a.flags = c->s_flags.as<uint8_t>();
+  a.ctr = d_ctr;
+  a.slice = d_slice;
+  a.state = d_state;
+  a.last = d_last;
+  a.busy = d_busy;
+  CK(launch_sim(a, (cudaStream_t)stream), "simulator kernel");
   return FFS_OK;
 }
 

@@ -175,6 +175,27 @@ struct RouteArgs {
   int32_t* route;
 };
 cudaError_t launch_route(int phase, const RouteArgs& a, cudaStream_t st);
+
+struct SimArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  uint32_t n_nodes, n_ticks, window_ticks, thr_pct, tick_us;
+  uint64_t t0_us, cold_after_us;
+  const uint32_t* node_off;     // [n_nodes+1]
+  const uint8_t* slice_prof;
+  const uint8_t* slice_busy;    // staged states (other tenants)
+  const uint32_t* req_off;
+  const uint32_t* req_func;
+  const uint32_t* req_budget;
+  int32_t* res;                 // [n_slices] resident function or -1 (scratch)
+  uint8_t* flags;               // [n_nodes][F] bit0 exists, bit1 hot (scratch)
+  uint64_t* ctr;
+  int32_t* slice;
+  uint8_t* state;
+  uint64_t* last;
+  uint32_t* busy;
+};
+cudaError_t launch_sim(const SimArgs& a, cudaStream_t st);
 cudaError_t radix_sort_pairs(uint64_t* key, uint32_t* val, uint64_t* key2, uint32_t* val2, uint32_t n, int bits,
                              uint64_t* hist, uint64_t* bsum, cudaStream_t st);
 cudaError_t scan_u64(uint64_t* a, uint64_t len, uint64_t* bsum, cudaStream_t st);

@@ -1739,6 +1739,157 @@ cudaError_t scan_u64(uint64_t* a, uint64_t len, uint64_t* bsum, cudaStream_t st)
 }
 
 // ====================================================================================
+// K10 (NEXT-4): time-sharing simulator, one warp per node
+// ====================================================================================
+__device__ __forceinline__ uint64_t warp_min_u64(uint64_t x) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const uint64_t y = __shfl_xor_sync(0xffffffffu, x, o);
+    x = y < x ? y : x;
+  }
+  return x;
+}
+
+__global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArgs A) {
+  const uint32_t v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (v >= A.n_nodes) return;
+  const uint32_t* img = A.image;
+  const ImageLayout& L = A.lay;
+  const uint32_t F = L.F, s0 = A.node_off[v], s1 = A.node_off[v + 1];
+  int32_t* sl = A.slice + (uint64_t)v * F;
+  uint64_t* last = A.last + (uint64_t)v * F;
+  uint32_t* busy = A.busy + (uint64_t)v * F;
+  uint8_t* fl = A.flags + (uint64_t)v * F;
+  for (uint32_t f = lane; f < F; f += 32) {
+    sl[f] = -1;
+    last[f] = 0;
+    busy[f] = 0;
+    fl[f] = 0;
+  }
+  for (uint32_t s = s0 + lane; s < s1; s += 32) A.res[s] = -1;
+  uint64_t c_req = 0, c_srv = 0, c_hit = 0, c_uns = 0, c_rel = 0, c_evi = 0, c_ter = 0, c_occ = 0;
+  const uint64_t window_us = (uint64_t)A.window_ticks * A.tick_us;
+  __syncwarp();
+  for (uint32_t t = 0; t < A.n_ticks; ++t) {
+    const uint64_t now = A.t0_us + (uint64_t)t * A.tick_us;
+    const uint32_t j0 = A.req_off[(uint64_t)v * A.n_ticks + t], j1 = A.req_off[(uint64_t)v * A.n_ticks + t + 1];
+    for (uint32_t j = j0; j < j1; ++j) {
+      const uint32_t f = A.req_func[j];
+      const uint64_t B = A.req_budget[j];
+      const uint32_t* fd = img + L.o_fdesc + 4 * f;
+      const uint32_t row0 = fd[0], n = fd[1], load = fd[2], memt = fd[3];
+      ++c_req;
+      if (lane == 0 && !(fl[f] & 1u)) {  // created on its first request, warm
+        fl[f] = 1;
+        sl[f] = -1;
+        busy[f] = 0;
+        last[f] = now;
+      }
+      __syncwarp();
+      int32_t at = sl[f];
+      uint64_t latency = 0;
+      if (at < 0) {
+        // free slice of smallest (capacity, gpcs, id) holding the function
+        uint64_t best = ~0ull;
+        for (uint32_t s = s0 + lane; s < s1; s += 32) {
+          const uint32_t p = A.slice_prof[s];
+          if (!A.slice_busy[s] && A.res[s] < 0 && memt <= img[L.o_cap + p])
+            best = min(best, ((uint64_t)img[L.o_cap + p] << 40) | ((uint64_t)img[L.o_gpcs + p] << 32) | s);
+        }
+        best = warp_min_u64(best);
+        if (best == ~0ull) {  // LRU time-sharing victim not used in this tick
+          for (uint32_t s = s0 + lane; s < s1; s += 32) {
+            const int32_t g = A.res[s];
+            if (g < 0 || (uint32_t)g == f || (fl[g] & 2u) || last[g] >= now) continue;
+            if (memt > img[L.o_cap + A.slice_prof[s]]) continue;
+            best = min(best, (last[g] << 20) | (s - s0));
+          }
+          best = warp_min_u64(best);
+          if (best != ~0ull) {
+            const uint32_t s = s0 + (uint32_t)(best & 0xFFFFFu);
+            if (lane == 0) {
+              sl[A.res[s]] = -1;  // evicted to CPU memory: warm
+              A.res[s] = -1;
+            }
+            ++c_evi;
+            best = s;
+          }
+        } else {
+          best &= 0xFFFFFFFFull;
+        }
+        if (best != ~0ull) {
+          at = (int32_t)best;
+          if (lane == 0) {
+            A.res[at] = (int32_t)f;
+            sl[f] = at;
+          }
+          ++c_rel;
+          latency = load;
+        }
+      }
+      if (at >= 0) {
+        const uint32_t p = A.slice_prof[at];
+        const uint32_t ex = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
+        latency += ex;
+        ++c_srv;
+        c_hit += latency <= B;
+        if (lane == 0) {
+          busy[f] += ex;
+          last[f] = now;
+        }
+      } else {
+        ++c_uns;
+      }
+      __syncwarp();
+    }
+    // end of tick: occupied slices, utilisation windows, cold terminations
+    uint32_t occ = 0;
+    for (uint32_t s = s0 + lane; s < s1; s += 32) occ += A.res[s] >= 0;
+    uint32_t ter = 0;
+    const bool roll = (t + 1) % A.window_ticks == 0;
+    for (uint32_t f = lane; f < F; f += 32) {
+      uint8_t x = fl[f];
+      if (roll) {
+        x = (uint8_t)((x & 1u) | (((uint64_t)busy[f] * 100u >= (uint64_t)A.thr_pct * window_us) ? 2u : 0u));
+        busy[f] = 0;
+      }
+      if ((x & 1u) && now - last[f] >= A.cold_after_us) {
+        if (sl[f] >= 0) A.res[sl[f]] = -1;
+        sl[f] = -1;
+        busy[f] = 0;
+        x = 0;
+        ++ter;
+      }
+      fl[f] = x;
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+      occ += __shfl_xor_sync(0xffffffffu, occ, o);
+      ter += __shfl_xor_sync(0xffffffffu, ter, o);
+    }
+    c_occ += occ;
+    c_ter += ter;
+    __syncwarp();
+  }
+  for (uint32_t f = lane; f < F; f += 32) {
+    const uint8_t x = fl[f];
+    A.state[(uint64_t)v * F + f] = !(x & 1u) ? FFS_ST_COLD
+                                   : (sl[f] < 0 ? FFS_ST_WARM : ((x & 2u) ? FFS_ST_EXCL_HOT : FFS_ST_TIME_SHARING));
+  }
+  if (lane == 0) {
+    uint64_t* C = A.ctr + (uint64_t)v * 8;
+    C[0] = c_req; C[1] = c_srv; C[2] = c_hit; C[3] = c_uns;
+    C[4] = c_rel; C[5] = c_evi; C[6] = c_ter; C[7] = c_occ;
+  }
+}
+
+cudaError_t launch_sim(const SimArgs& a, cudaStream_t st) {
+  const uint64_t threads = (uint64_t)a.n_nodes * 32;
+  k_simulate<<<(unsigned)((threads + 127) / 128), 128, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+// ====================================================================================
 // K5: integer issue-rate microbenchmark (roofline denominator)
 // ====================================================================================
 constexpr int kPeakIters = 4096;

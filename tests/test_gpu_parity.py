@@ -459,3 +459,24 @@ def test_c5_full_batch_properties(F, planner):
     check_plan_properties(prob, p)
     ok = p["status"] == 0
     assert ok.mean() > 0.5 and (ok & (p["k"] > 1)).mean() > 0.05 and (~ok).mean() > 0.05
+
+
+# ---- NEXT-4: time-sharing simulator ----------------------------------------------------------
+@pytest.mark.parametrize("case", ["small", "c4"])
+def test_simulator_matches_oracle(F, planner, case):
+    if case == "small":
+        tr = W.sim_trace(seed=101, T=600, n_funcs=12, nodes=[W.PART_P1, W.PART_HYBRID, W.PART_P2], rate_scale=8.0)
+        cold = 5_000_000
+    else:
+        tr = W.sim_trace(T=2048)
+        cold = 60_000_000
+    planner.stage(tr.problem)
+    ctr, sl, st, last, busy = planner.simulate(tr, cold_after_us=cold)
+    torch.cuda.synchronize()
+    o = oracle.sim(tr, cold_after_us=cold)
+    np.testing.assert_array_equal(ctr.cpu().numpy().view(np.uint64), o[0])
+    np.testing.assert_array_equal(sl.cpu().numpy(), o[1])
+    np.testing.assert_array_equal(st.cpu().numpy(), o[2])
+    np.testing.assert_array_equal(last.cpu().numpy().view(np.uint64), o[3])
+    np.testing.assert_array_equal(busy.cpu().numpy().view(np.uint32), o[4])
+    assert o[0][:, 5].sum() > 0 and o[0][:, 6].sum() > 0
