@@ -277,8 +277,6 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
     }
     row += n + 1;
   }
-  if ((size_t)L.words * 4 > kMaxSmem)
-    return fail(c, FFS_ERR_RANGE, "table image %u bytes exceeds the shared-memory stage", L.words * 4);
 
   // ---- per node: free counts (clamped to 8) and the first 8 free slices per profile ----
   const uint32_t NN = cl->n_nodes;
@@ -388,22 +386,22 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
                         c->block_sums.as<uint64_t>(), d_keys, reinterpret_cast<unsigned long long*>(d_checks), st),
      "count/scan kernels");
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows
-  // of the KS = 4 kernel (440 B per thread); the KS = 4 CTA shrinks when both do not fit
-  const size_t smem = (size_t)c->lay.words * 4;
+  // of the KS = 4 kernel (440 B per thread); the KS = 4 CTA shrinks when both do not fit.
+  // An image that leaves no room is read from global memory instead (tables_global).
+  const bool tables_global = (size_t)c->lay.words * 4 + (size_t)440 * 64 > kMaxSmem;
+  const size_t smem = tables_global ? 0 : (size_t)c->lay.words * 4;
   int block4 = kBlock;
   while (block4 > 32 && smem + (size_t)440 * block4 > kMaxSmem) block4 -= 32;
-  if (k_max >= 4 && c->max_n >= 4 && smem + (size_t)440 * block4 > kMaxSmem)
-    return fail(c, FFS_ERR_RANGE, "table image %zu B leaves no room for the KS=4 windows", smem);
   auto blk = [&](int k) { return k == 4 ? block4 : kBlock; };
   auto shm = [&](int k) { return smem + (k == 4 ? (size_t)440 * block4 : 0); };
-  if (c->occ_smem != smem) {
+  if (c->occ_smem != smem + 1) {
     for (int v = 0; v < 2; ++v)
       for (int k = 1; k <= kMaxK; ++k) {
         int b = 0;
         CK(search_kernel_config(k, v != 0, blk(k), shm(k), &b), "search kernel occupancy");
         c->occ[v][k] = std::max(1, b);
       }
-    c->occ_smem = smem;
+    c->occ_smem = smem + 1;
   }
   SearchArgs a{};
   a.image = c->image.as<uint32_t>();
@@ -418,6 +416,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   a.keys = d_keys;
   a.checks = reinterpret_cast<unsigned long long*>(d_checks);
   a.misses = c->misses.as<unsigned long long>();
+  a.tables_global = tables_global ? 1u : 0u;
   const bool verify = d_checks != nullptr;
   const uint32_t kk = std::min(k_max, c->max_n);
   c->seg_first = 1;

@@ -52,6 +52,7 @@ struct SearchArgs {
   int64_t* keys;
   unsigned long long* checks;   // [n_req][3] or null
   unsigned long long* misses;   // debug counter (verify mode)
+  uint32_t tables_global;       // 1: read the image from global memory (too large for smem)
 };
 
 struct DecodeArgs {

@@ -786,14 +786,21 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
 template <int KS, bool VERIFY>
 __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
-  {  // A0: stage the table image into shared memory (16-byte copies)
+  // A0: stage the table image into shared memory (16-byte copies); an image too large
+  // for shared memory is read from global memory through L1 instead (A.tables_global)
+  const uint32_t* tbl = smem;
+  uint32_t img_words = A.lay.words;
+  if (A.tables_global) {
+    tbl = A.image;
+    img_words = 0;
+  } else {
     const uint4* src = reinterpret_cast<const uint4*>(A.image);
     uint4* dst = reinterpret_cast<uint4*>(smem);
     for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += blockDim.x) dst[i] = src[i];
   }
   __syncthreads();
-  // KS = 4: per-thread rows of the shifted variant tables after the image (ks4_mask)
-  float* rows = reinterpret_cast<float*>(smem + A.lay.words);
+  // KS = 4: per-thread windows of the shifted variant tables after the image (ks4_pair)
+  float* rows = reinterpret_cast<float*>(smem + img_words);
 
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint64_t T = pre[A.n_req];
@@ -804,7 +811,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
   if (t0 >= t1) return;
 
   SearchState<KS> c;
-  c.sm = smem;
+  c.sm = tbl;
   c.o_pl = A.lay.o_pl;
   c.o_pm = A.lay.o_pm;
   c.o_xf = A.lay.o_xf;
@@ -822,7 +829,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
 
   auto load_request = [&](uint64_t rank0) {
     const ffs_request q = A.req[r];
-    const uint32_t* fd = smem + A.lay.o_fdesc + 4 * q.func;
+    const uint32_t* fd = tbl + A.lay.o_fdesc + 4 * q.func;
     c.row0 = fd[0];
     c.n = fd[1];
     c.B = A.slo[r];
@@ -831,7 +838,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
 #pragma unroll
     for (int p = 0; p < kP; ++p) w |= (16u + (uint32_t)((c.freeb >> (8 * p)) & 255u)) << (5 * p);
     c.free_w = w;
-    c.idx_base = img_u64(smem, A.lay.o_offk + 2 * (c.n * 10 + KS)) + rank0 * PK;
+    c.idx_base = img_u64(tbl, A.lay.o_offk + 2 * (c.n * 10 + KS)) + rank0 * PK;
     c.best = *reinterpret_cast<volatile const int64_t*>(A.keys + r);  // earlier segments' minimum
     best0 = c.best;
     if constexpr (KS >= 2) set_threshold(c);
@@ -844,9 +851,9 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
     int cc = (int)c.n - 2;
 #pragma unroll
     for (int i = KS - 1; i >= 1; --i) {
-      while (binom(smem, A.lay, cc, i) > mm) --cc;
+      while (binom(tbl, A.lay, cc, i) > mm) --cc;
       mk |= 1u << cc;
-      mm -= binom(smem, A.lay, cc, i);
+      mm -= binom(tbl, A.lay, cc, i);
       --cc;
     }
     mask = mk;

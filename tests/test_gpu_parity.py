@@ -480,3 +480,18 @@ def test_simulator_matches_oracle(F, planner, case):
     np.testing.assert_array_equal(last.cpu().numpy().view(np.uint64), o[3])
     np.testing.assert_array_equal(busy.cpu().numpy().view(np.uint32), o[4])
     assert o[0][:, 5].sum() > 0 and o[0][:, 6].sum() > 0
+
+
+def test_large_table_image_reads_tables_from_global(F, planner):
+    """800 functions: the table image no longer fits shared memory; the search reads it
+    from global memory (tables_global) with identical results."""
+    rng = W.SplitMix64(4242)
+    lengths = rng.sub(9).integers(3, 12, 800)
+    prob = W._problem("big", rng, lengths, W.NODE_BLOCK, 2048)
+    p, keys, ch = run_gpu(F, planner, prob)
+    o = oracle.plan(prob)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
+    np.testing.assert_array_equal(keys2, o["key"])
+    assert planner.filter_misses() == 0
