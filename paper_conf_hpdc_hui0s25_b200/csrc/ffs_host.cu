@@ -394,11 +394,11 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   while (block4 > 32 && smem + (size_t)440 * block4 > kMaxSmem) block4 -= 32;
   auto blk = [&](int k) { return k == 4 ? block4 : kBlock; };
   auto shm = [&](int k) { return smem + (k == 4 ? (size_t)440 * block4 : 0); };
-  if (c->occ_smem != smem + 1) {
+  if (c->occ_smem != smem + 1) {  // (smem = 0 <=> tables in global memory)
     for (int v = 0; v < 2; ++v)
       for (int k = 1; k <= kMaxK; ++k) {
         int b = 0;
-        CK(search_kernel_config(k, v != 0, blk(k), shm(k), &b), "search kernel occupancy");
+        CK(search_kernel_config(k, v != 0, tables_global, blk(k), shm(k), &b), "search kernel occupancy");
         c->occ[v][k] = std::max(1, b);
       }
     c->occ_smem = smem + 1;

@@ -78,7 +78,8 @@ cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, co
                                cudaStream_t st);
 cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st);
-cudaError_t search_kernel_config(int ks, bool verify, int block, size_t smem, int* blocks_per_sm);
+cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,
+                                 int* blocks_per_sm);
 cudaError_t launch_decode(const DecodeArgs& a, cudaStream_t st);
 cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32_t* tick_off,
                          const uint64_t* now_us, uint32_t n_ticks, uint64_t now_single,

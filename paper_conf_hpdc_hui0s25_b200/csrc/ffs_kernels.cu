@@ -783,14 +783,15 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
   return lo;
 }
 
-template <int KS, bool VERIFY>
+template <int KS, bool VERIFY, bool TG>
 __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
   // A0: stage the table image into shared memory (16-byte copies); an image too large
   // for shared memory is read from global memory through L1 instead (A.tables_global)
+  // (TG is a template parameter so that the shared-memory variant keeps LDS accesses)
   const uint32_t* tbl = smem;
   uint32_t img_words = A.lay.words;
-  if (A.tables_global) {
+  if constexpr (TG) {
     tbl = A.image;
     img_words = 0;
   } else {
@@ -901,9 +902,9 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
   flush();
 }
 
-template <int KS, bool V>
+template <int KS, bool V, bool TG>
 static cudaError_t set_attr() {
-  return cudaFuncSetAttribute(k_plan_search<KS, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
+  return cudaFuncSetAttribute(k_plan_search<KS, V, TG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
 }
 
 #define FFS_KS_SWITCH(ks, verify, CALL)                  \
@@ -927,25 +928,39 @@ static cudaError_t set_attr() {
     default: return cudaErrorInvalidValue;               \
   }
 
-cudaError_t search_kernel_config(int ks, bool verify, int block, size_t smem, int* blocks_per_sm) {
+template <bool TG>
+static cudaError_t search_config_t(int ks, bool verify, int block, size_t smem, int* blocks_per_sm) {
   cudaError_t e = cudaSuccess;
-#define CFG(K, V)                                                                                   \
-  do {                                                                                            \
-    e = set_attr<K, V>();                                                                         \
-    if (e == cudaSuccess)                                                                         \
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_plan_search<K, V>, block, smem); \
+#define CFG(K, V)                                                                                        \
+  do {                                                                                                 \
+    e = set_attr<K, V, TG>();                                                                          \
+    if (e == cudaSuccess)                                                                              \
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_plan_search<K, V, TG>, block, smem); \
   } while (0)
   FFS_KS_SWITCH(ks, verify, CFG)
 #undef CFG
   return e;
 }
 
-cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
-                          cudaStream_t st) {
-#define LAUNCH(K, V) k_plan_search<K, V><<<grid, block, smem, st>>>(a)
+template <bool TG>
+static cudaError_t launch_search_t(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
+                                   cudaStream_t st) {
+#define LAUNCH(K, V) k_plan_search<K, V, TG><<<grid, block, smem, st>>>(a)
   FFS_KS_SWITCH(ks, verify, LAUNCH)
 #undef LAUNCH
   return cudaGetLastError();
+}
+
+cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,
+                                 int* blocks_per_sm) {
+  return tables_global ? search_config_t<true>(ks, verify, block, smem, blocks_per_sm)
+                       : search_config_t<false>(ks, verify, block, smem, blocks_per_sm);
+}
+
+cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
+                          cudaStream_t st) {
+  return a.tables_global ? launch_search_t<true>(ks, verify, a, grid, block, smem, st)
+                         : launch_search_t<false>(ks, verify, a, grid, block, smem, st);
 }
 
 // ====================================================================================
