@@ -226,7 +226,9 @@ ffs_status ffs_evict_scores_ticks(ffs_ctx *ctx, const ffs_instance *d_inst, cons
 /* A8 batched over ticks: for every request r (tick d_req_tick[r]) the victim among the
  * instances of that tick, by the rule of ffs_plan_decode, regardless of the request's
  * plan (the caller passes the loads that need one).  d_victim[r] = index within the tick
- * or -1.  Async. */
+ * or -1 (also when d_req_tick[r] >= n_ticks or the request's function/node is out of
+ * range).  Scratch: a per-(tick, node, profile) table of n_ticks x nodes x 5 x 8 bytes when
+ * that is <= 256 MiB, else a warp scan of the tick per request.  Async. */
 ffs_status ffs_evict_victims(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us,
                              const uint32_t *d_req_tick, uint32_t n_req, const ffs_instance *d_inst,
                              const uint32_t *d_tick_off, const int64_t *d_score, uint32_t n_ticks,

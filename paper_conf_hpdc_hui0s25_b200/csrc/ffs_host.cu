@@ -78,7 +78,7 @@ struct ffs_ctx {
   bool ranked = false;
   uint32_t rank_kmax = 0, prof_order = 0;
   // scratch
-  DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses;
+  DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses, v_tab;
   // cached occupancy per (ks, verify, smem)
   size_t occ_smem = 0;
   int occ[2][kMaxK + 1] = {};
@@ -157,7 +157,7 @@ void ffs_destroy(ffs_ctx* c) {
                       &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
       b->release();
     for (DevBuf* b : {&c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
-                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses})
+                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab})
       b->release();
   }
   delete c;
@@ -531,9 +531,14 @@ ffs_status ffs_evict_victims(ffs_ctx* c, const ffs_request* d_req, const uint32_
   if (!d_req || !d_slo || !d_req_tick || !d_inst || !d_tick_off || !d_score || !d_victim)
     return fail(c, FFS_ERR_ARG, "null device pointer");
   DeviceGuard g(c->device);
+  // per-(tick, node, profile) minimum table when it stays small, else the warp scan
+  const uint64_t tab_bytes = (uint64_t)n_ticks * c->n_nodes * c->P * 8;
+  unsigned long long* tab = nullptr;
+  if (tab_bytes > 0 && tab_bytes <= (256ull << 20) && c->v_tab.ensure(tab_bytes) == cudaSuccess)
+    tab = c->v_tab.as<unsigned long long>();
   CK(launch_victims(c->image.as<uint32_t>(), c->lay, d_req, d_slo, d_req_tick, n_req, d_inst, d_tick_off, d_score,
-                    n_ticks, c->slice_node.as<uint16_t>(), c->slice_prof.as<uint8_t>(), c->n_slices, d_victim,
-                    (cudaStream_t)stream),
+                    n_ticks, c->slice_node.as<uint16_t>(), c->slice_prof.as<uint8_t>(), c->n_slices, c->n_nodes, tab,
+                    d_victim, (cudaStream_t)stream),
      "victims kernel");
   return FFS_OK;
 }

@@ -88,7 +88,8 @@ cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const 
                            const uint32_t* slo, const uint32_t* req_tick, uint32_t n_req,
                            const ffs_instance* inst, const uint32_t* tick_off, const int64_t* score,
                            uint32_t n_ticks, const uint16_t* slice_node, const uint8_t* slice_prof,
-                           uint32_t n_slices, int32_t* victim, cudaStream_t st);
+                           uint32_t n_slices, uint32_t n_nodes, unsigned long long* tab, int32_t* victim,
+                           cudaStream_t st);
 cudaError_t run_int_peak(int sms, double* ops, double* seconds);
 
 struct RankedArgs {

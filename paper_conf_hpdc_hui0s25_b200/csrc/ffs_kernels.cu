@@ -8,7 +8,8 @@
 //                               to the per-request minimum packed key (A2-A5)
 // K2  k_decode                   key -> plan, recompute figures, bind slices, victims (A6, A8)
 // K3  k_evict                    keep-alive state + LRU eviction key per instance (A7)
-// K4  k_victims                  per-request LRU victim over a tick's instances (A8)
+// K4  k_victim_table/_pick        per-request LRU victim over a tick's instances (A8)
+//     (k_victims: warp-per-load scan, used when the per-tick table would be too large)
 // K5  k_int_peak                 integer issue-rate microbenchmark (roofline denominator)
 //
 // Paper: FluidFaaS, HPDC '25.  P:<line> = line of PAPER.md; R<n> = DESIGN.md §3 reading.
@@ -1304,7 +1305,7 @@ constexpr int kViT = 256;
 __global__ void __launch_bounds__(kViT) k_victims(const uint32_t* __restrict__ img, ImageLayout L,
                                                    const ffs_request* __restrict__ req, const uint32_t* __restrict__ slo,
                                                    const uint32_t* __restrict__ req_tick, uint32_t n_req,
-                                                   const ffs_instance* __restrict__ inst,
+                                                   uint32_t n_ticks, const ffs_instance* __restrict__ inst,
                                                    const uint32_t* __restrict__ tick_off,
                                                    const int64_t* __restrict__ score, const uint16_t* slice_node,
                                                    const uint8_t* slice_prof, uint32_t n_slices,
@@ -1314,9 +1315,9 @@ __global__ void __launch_bounds__(kViT) k_victims(const uint32_t* __restrict__ i
   const ffs_request q = req[r];
   int64_t bs = (int64_t)kKeyNone;
   uint32_t b = 0, e = 0;
-  if (q.func < L.F) {
+  const uint32_t t = req_tick[r];
+  if (q.func < L.F && t < n_ticks) {
     const uint32_t okp = victim_profiles(img, L, q.func, slo[r]);
-    const uint32_t t = req_tick[r];
     b = tick_off[t];
     e = tick_off[t + 1];
     for (uint32_t i = b + lane; i < e; i += 32) {
@@ -1336,16 +1337,67 @@ __global__ void __launch_bounds__(kViT) k_victims(const uint32_t* __restrict__ i
   if (lane == 0) victim[r] = (uint64_t)bs == kKeyNone ? -1 : (int32_t)((uint64_t)bs & 0xFFFFFu);
 }
 
+// Table variant: the minimum packed score per (tick, node, slice profile) is built once
+// per tick (one CTA per tick, 64-bit atomicMin), then each load takes the minimum over its
+// monolithic profiles -- at most 5 reads instead of a scan of the whole tick.  Scores are
+// unique within a tick (low 20 bits = index), so the minimum of the per-profile minima is
+// the same victim.  UINT64_MAX marks an empty cell (FFS_KEY_NONE scores are skipped).
+__global__ void __launch_bounds__(256) k_victim_table(const ffs_instance* __restrict__ inst,
+                                                      const uint32_t* __restrict__ tick_off,
+                                                      const int64_t* __restrict__ score,
+                                                      const uint16_t* __restrict__ slice_node,
+                                                      const uint8_t* __restrict__ slice_prof, uint32_t n_slices,
+                                                      uint32_t n_nodes, unsigned long long* __restrict__ tab) {
+  const uint32_t t = blockIdx.x, b = tick_off[t], e = tick_off[t + 1];
+  unsigned long long* row = tab + (uint64_t)t * n_nodes * kP;
+  for (uint32_t i = b + threadIdx.x; i < e; i += blockDim.x) {
+    const int64_t s = score[i];
+    if ((uint64_t)s == kKeyNone) continue;
+    const int32_t sl = inst[i].slice;
+    if (sl < 0 || (uint32_t)sl >= n_slices) continue;
+    atomicMin(row + (uint32_t)slice_node[sl] * kP + slice_prof[sl], (unsigned long long)s);
+  }
+}
+
+__global__ void __launch_bounds__(256) k_victim_pick(const uint32_t* __restrict__ img, ImageLayout L,
+                                                     const ffs_request* __restrict__ req,
+                                                     const uint32_t* __restrict__ slo,
+                                                     const uint32_t* __restrict__ req_tick, uint32_t n_req,
+                                                     uint32_t n_ticks, uint32_t n_nodes,
+                                                     const unsigned long long* __restrict__ tab,
+                                                     int32_t* __restrict__ victim) {
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= n_req) return;
+  const ffs_request q = req[r];
+  const uint32_t t = req_tick[r];
+  unsigned long long bs = ~0ull;
+  if (q.func < L.F && q.node < n_nodes && t < n_ticks) {
+    const uint32_t okp = victim_profiles(img, L, q.func, slo[r]);
+    const unsigned long long* cell = tab + ((uint64_t)t * n_nodes + q.node) * kP;
+#pragma unroll
+    for (int p = 0; p < kP; ++p)
+      if ((okp >> p) & 1u) bs = min(bs, cell[p]);
+  }
+  victim[r] = bs == ~0ull ? -1 : (int32_t)(bs & 0xFFFFFull);
+}
+
 cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const ffs_request* req, const uint32_t* slo,
                            const uint32_t* req_tick, uint32_t n_req, const ffs_instance* inst,
                            const uint32_t* tick_off, const int64_t* score, uint32_t n_ticks,
                            const uint16_t* slice_node, const uint8_t* slice_prof, uint32_t n_slices,
-                           int32_t* victim, cudaStream_t st) {
-  (void)n_ticks;
+                           uint32_t n_nodes, unsigned long long* tab, int32_t* victim, cudaStream_t st) {
   if (n_req == 0) return cudaSuccess;
+  if (tab && n_ticks > 0) {
+    cudaError_t e = cudaMemsetAsync(tab, 0xFF, (size_t)n_ticks * n_nodes * kP * 8, st);
+    if (e != cudaSuccess) return e;
+    k_victim_table<<<n_ticks, 256, 0, st>>>(inst, tick_off, score, slice_node, slice_prof, n_slices, n_nodes, tab);
+    k_victim_pick<<<(n_req + 255) / 256, 256, 0, st>>>(image, lay, req, slo, req_tick, n_req, n_ticks, n_nodes, tab,
+                                                       victim);
+    return cudaGetLastError();
+  }
   const uint64_t threads = (uint64_t)n_req * 32;
-  k_victims<<<(unsigned)((threads + kViT - 1) / kViT), kViT, 0, st>>>(image, lay, req, slo, req_tick, n_req, inst,
-                                                                       tick_off, score, slice_node, slice_prof,
+  k_victims<<<(unsigned)((threads + kViT - 1) / kViT), kViT, 0, st>>>(image, lay, req, slo, req_tick, n_req, n_ticks,
+                                                                       inst, tick_off, score, slice_node, slice_prof,
                                                                        n_slices, victim);
   return cudaGetLastError();
 }

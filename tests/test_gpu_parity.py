@@ -237,6 +237,32 @@ def test_eviction_scores_and_victims(F, planner):
     assert (vic >= 0).sum() > 0
 
 
+def test_victims_table_and_scan_paths_agree(F, planner):
+    """The per-(tick, node, profile) table path and the warp-scan path (taken when the table
+    would exceed 256 MiB: here forced by appending empty ticks) give the same victims;
+    requests whose tick is out of range get -1 on both."""
+    wl = W.config4(T=32)
+    prob = wl.problem
+    planner.stage(prob)
+    inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
+    toff = torch.from_numpy(wl.tick_off.view(np.int32)).cuda()
+    now = torch.from_numpy(wl.now_us.view(np.int64)).cuda()
+    score, _ = planner.evict_scores_ticks(inst, toff, now, window_us=wl.window_us)
+    req, slo = F.to_device(prob)
+    rt_np = wl.req_tick.astype(np.uint32).copy()
+    rt_np[::7] = len(wl.now_us)  # out of range for the table path
+    rt = torch.from_numpy(rt_np.view(np.int32)).cuda()
+    v_tab = planner.evict_victims(req, slo, rt, inst, toff, score).cpu().numpy()
+    pad = 256 * 2**20 // (prob.n_nodes * 5 * 8) + 1
+    toff_big = np.concatenate([wl.tick_off, np.full(pad, wl.tick_off[-1], wl.tick_off.dtype)])
+    toff_big = torch.from_numpy(toff_big.view(np.int32)).cuda()
+    rt_np[::7] = len(toff_big) + 3  # beyond the padded range too
+    rt = torch.from_numpy(rt_np.view(np.int32)).cuda()
+    v_scan = planner.evict_victims(req, slo, rt, inst, toff_big, score).cpu().numpy()
+    np.testing.assert_array_equal(v_tab, v_scan)
+    assert (v_tab[::7] == -1).all() and (v_tab >= 0).sum() > 0
+
+
 def test_decode_victims_single_snapshot(F, planner):
     wl = W.config4(T=1)
     prob = wl.problem
