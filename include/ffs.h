@@ -180,6 +180,21 @@ ffs_status ffs_plan_keys(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t 
                          uint32_t k_max, uint32_t rank, uint32_t world, int64_t *d_keys, uint64_t *d_checksums,
                          void *stream);
 
+/* Segments k_first..k_last (1 <= k_first <= k_last <= k_max) of ffs_plan_keys, same shard
+ * rule.  k_first == 1 initialises d_keys (FFS_KEY_NONE) and d_checksums (0) like
+ * ffs_plan_keys; k_first > 1 leaves both as given and min-combines / adds into them, so a
+ * caller can all_reduce(MIN) the keys between ranges: every rank then prunes the later
+ * (heavier) segments against the best key of ALL shards of the earlier ones, exactly as
+ * one GPU does, which keeps the shards equal in work.  The result after
+ * the last range and a final MIN is the same as ffs_plan_keys.  Checksums stay per-shard
+ * sums; reduce them with SUM once at the end.  A continuation (k_first > 1) with the same
+ * d_req, n_req and k_max as the previous search call on this context reuses that call's
+ * task prefix: the request batch must not change in between.  FFS_ERR_RANGE: bad segment
+ * range, or as ffs_plan_keys.  Asynchronous on `stream`. */
+ffs_status ffs_plan_keys_range(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                               uint32_t k_max, uint32_t k_first, uint32_t k_last, uint32_t rank, uint32_t world,
+                               int64_t *d_keys, uint64_t *d_checksums, void *stream);
+
 /* ---- A6 (+A8): decode and bind ---------------------------------------------------------
  * Decode the combined keys into plans and bind every stage, in stage order, to the
  * lowest-index free slice of its profile in the request's node not taken by an earlier
@@ -315,9 +330,10 @@ ffs_status ffs_plan_frontier(ffs_ctx *ctx, const ffs_request *d_req, const uint3
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
  * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */
 ffs_status ffs_bench_int_peak(ffs_ctx *ctx, double *ops_per_s, double *seconds);
-/* Device time (ms, CUDA events recorded on the launch stream) of each search-kernel
- * segment of the last ffs_plan_keys call on this context: ms[ks-1] for ks = 1..8 stages,
- * 0 where no segment ran.  Waits for those events.  */
+/* Device time (ms, CUDA events recorded on the launch stream around each launch) of each
+ * search-kernel segment run since the last ffs_plan_keys / ffs_plan_keys_range call with
+ * k_first = 1 on this context: ms[ks-1] for ks = 1..8 stages, 0 where no segment ran.
+ * Waits for those events.  */
 ffs_status ffs_segment_times(ffs_ctx *ctx, float *ms /* [8] */);
 /* Number of candidates, since the context was created, that the fast float filter
  * rejected although their exact key would have beaten the running minimum (verify mode

@@ -78,13 +78,16 @@ struct ffs_ctx {
   bool ranked = false;
   uint32_t rank_kmax = 0, prof_order = 0;
   // scratch
-  DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses, v_tab;
+  DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses, v_tab, work_ctr;
   // cached occupancy per (ks, verify, smem)
   size_t occ_smem = 0;
   int occ[2][kMaxK + 1] = {};
   // per-segment timing of the last plan_keys call
-  cudaEvent_t ev[kMaxK + 1] = {};
-  int seg_first = 0, seg_last = -1;
+  cudaEvent_t ev[kMaxK + 1] = {}, evs[kMaxK + 1] = {};  // per segment: end, start
+  uint32_t seg_mask = 0;                                 // segments timed since the last k_first = 1
+  // task prefix of the last search call (reused by continuation ranges, k_first > 1)
+  const void* pre_req = nullptr;
+  uint32_t pre_n = 0, pre_kmax = 0;
 };
 
 static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
@@ -135,6 +138,7 @@ ffs_status ffs_create(int cuda_device, ffs_ctx** out) {
       return FFS_ERR_CUDA;
     }
     for (auto& e : c->ev) cudaEventCreate(&e);
+    for (auto& e : c->evs) cudaEventCreate(&e);
   }
   *out = c;
   return FFS_OK;
@@ -145,6 +149,8 @@ void ffs_destroy(ffs_ctx* c) {
   {
     DeviceGuard g(c->device);
     for (auto& e : c->ev)
+      if (e) cudaEventDestroy(e);
+    for (auto& e : c->evs)
       if (e) cudaEventDestroy(e);
     for (DevBuf* b : {&c->s_res, &c->s_flags, &c->s_busy}) b->release();
     for (DevBuf* b : {&c->r_k, &c->r_k2, &c->r_v, &c->r_v2, &c->i_k, &c->i_k2, &c->i_v, &c->i_v2, &c->i_cum, &c->r_f,
@@ -157,7 +163,7 @@ void ffs_destroy(ffs_ctx* c) {
                       &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
       b->release();
     for (DevBuf* b : {&c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
-                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab})
+                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr})
       b->release();
   }
   delete c;
@@ -166,6 +172,7 @@ void ffs_destroy(ffs_ctx* c) {
 const char* ffs_last_error(const ffs_ctx* c) { return c ? c->err.c_str() : "null context"; }
 
 ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profile_table* tb, const ffs_cluster* cl) {
+  if (c) c->pre_req = nullptr;  // the task prefix depends on the staged chain lengths
   if (!c) return FFS_ERR_ARG;
   c->staged = false;
   if (!pr || !tb || !cl) return fail(c, FFS_ERR_ARG, "null table pointer");
@@ -360,7 +367,7 @@ static ffs_status check_kmax(ffs_ctx* c, uint32_t k_max) {
 
 static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
                               uint32_t k_max, uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks,
-                              const uint64_t* node_free, void* stream);
+                              const uint64_t* node_free, void* stream, uint32_t k_first = 1, uint32_t k_last = 0);
 
 ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req, uint32_t k_max,
                          uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks, void* stream) {
@@ -368,11 +375,21 @@ ffs_status ffs_plan_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d
   return search_keys(c, d_req, d_slo, n_req, k_max, rank, world, d_keys, d_checks, nullptr, stream);
 }
 
+ffs_status ffs_plan_keys_range(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                               uint32_t k_max, uint32_t k_first, uint32_t k_last, uint32_t rank, uint32_t world,
+                               int64_t* d_keys, uint64_t* d_checks, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (k_first < 1 || k_first > k_last || k_last > k_max)
+    return fail(c, FFS_ERR_RANGE, "segment range %u..%u not within 1..k_max=%u", k_first, k_last, k_max);
+  return search_keys(c, d_req, d_slo, n_req, k_max, rank, world, d_keys, d_checks, nullptr, stream, k_first, k_last);
+}
+
 static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
                               uint32_t k_max, uint32_t rank, uint32_t world, int64_t* d_keys, uint64_t* d_checks,
-                              const uint64_t* node_free, void* stream) {
+                              const uint64_t* node_free, void* stream, uint32_t k_first, uint32_t k_last) {
   ffs_status s = check_kmax(c, k_max);
   if (s != FFS_OK) return s;
+  if (k_last == 0) k_last = k_max;
   if (world == 0 || rank >= world) return fail(c, FFS_ERR_ARG, "rank %u / world %u", rank, world);
   if (n_req == 0) return FFS_OK;
   if (!d_req || !d_slo || !d_keys) return fail(c, FFS_ERR_ARG, "null device pointer");
@@ -382,9 +399,23 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   CK(c->prefix.ensure(len * k_max * 8), "cudaMalloc(prefix)");
   const uint64_t nb = (len + 2047) / 2048;
   CK(c->block_sums.ensure(nb * k_max * 8 + 8), "cudaMalloc(block_sums)");
-  CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, c->prefix.as<uint64_t>(),
-                        c->block_sums.as<uint64_t>(), d_keys, reinterpret_cast<unsigned long long*>(d_checks), st),
-     "count/scan kernels");
+  // keys and checksums are initialised by the first segment only; later ranges continue
+  // from (and prune against) whatever the caller combined into d_keys in between
+  const bool init = k_first == 1;
+  CK(c->work_ctr.ensure((kMaxK + 1) * 8), "cudaMalloc(work_ctr)");
+  if (!init && c->pre_req == d_req && c->pre_n == n_req && c->pre_kmax == k_max) {
+    // continuation of the same batch: the task prefix is still valid; reset the counters
+    CK(cudaMemsetAsync(c->work_ctr.p, 0, (kMaxK + 1) * 8, st), "reset chunk counters");
+  } else {
+    CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, c->prefix.as<uint64_t>(),
+                          c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
+                          init ? reinterpret_cast<unsigned long long*>(d_checks) : nullptr,
+                          c->work_ctr.as<unsigned long long>(), st),
+       "count/scan kernels");
+  }
+  c->pre_req = d_req;
+  c->pre_n = n_req;
+  c->pre_kmax = k_max;
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows
   // of the KS = 4 kernel (440 B per thread); the KS = 4 CTA shrinks when both do not fit.
   // An image that leaves no room is read from global memory instead (tables_global).
@@ -417,15 +448,16 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   a.checks = reinterpret_cast<unsigned long long*>(d_checks);
   a.misses = c->misses.as<unsigned long long>();
   a.tables_global = tables_global ? 1u : 0u;
+  a.work_ctr = c->work_ctr.as<unsigned long long>();
   const bool verify = d_checks != nullptr;
-  const uint32_t kk = std::min(k_max, c->max_n);
-  c->seg_first = 1;
-  c->seg_last = (int)kk;
-  CK(cudaEventRecord(c->ev[0], st), "event");
-  for (uint32_t k = 1; k <= kk; ++k) {
+  const uint32_t kk = std::min(k_last, c->max_n);
+  if (init) c->seg_mask = 0;
+  for (uint32_t k = k_first; k <= kk; ++k) {
     const int grid = c->sms * c->occ[verify ? 1 : 0][k];
+    CK(cudaEventRecord(c->evs[k], st), "event");
     CK(launch_search((int)k, verify, a, grid, blk((int)k), shm((int)k), st), "search kernel");
     CK(cudaEventRecord(c->ev[k], st), "event");
+    c->seg_mask |= 1u << k;
   }
   return FFS_OK;
 }
@@ -961,9 +993,10 @@ ffs_status ffs_segment_times(ffs_ctx* c, float* ms) {
   if (!c || !ms) return FFS_ERR_ARG;
   for (int k = 0; k < kMaxK; ++k) ms[k] = 0.f;
   DeviceGuard g(c->device);
-  for (int k = c->seg_first; k <= c->seg_last; ++k) {
+  for (int k = 1; k <= kMaxK; ++k) {
+    if (!((c->seg_mask >> k) & 1u)) continue;
     CK(cudaEventSynchronize(c->ev[k]), "event sync");
-    CK(cudaEventElapsedTime(&ms[k - 1], c->ev[k - 1], c->ev[k]), "event time");
+    CK(cudaEventElapsedTime(&ms[k - 1], c->evs[k], c->ev[k]), "event time");
   }
   return FFS_OK;
 }

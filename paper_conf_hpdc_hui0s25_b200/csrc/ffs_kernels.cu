@@ -39,14 +39,15 @@ __device__ __forceinline__ uint32_t binom(const uint32_t* img, const ImageLayout
 __global__ void k_count_tasks(const ffs_request* __restrict__ req, const uint32_t* __restrict__ img,
                               ImageLayout lay, uint32_t n_nodes, uint32_t n_req, uint32_t K,
                               uint64_t* __restrict__ prefix, int64_t* __restrict__ keys,
-                              unsigned long long* __restrict__ checks) {
+                              unsigned long long* __restrict__ checks, unsigned long long* __restrict__ work_ctr) {
   uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r <= (uint32_t)kMaxK) work_ctr[r] = 0;  // the search segments' chunk counters
   if (r > n_req) return;
   uint32_t n = 0;
   if (r < n_req) {
     ffs_request q = req[r];
     if (q.func < lay.F && q.node < n_nodes) n = img[lay.o_fdesc + 4 * q.func + 1];
-    keys[r] = (int64_t)kKeyNone;
+    if (keys) keys[r] = (int64_t)kKeyNone;
     if (checks) {
       checks[3ull * r] = 0;
       checks[3ull * r + 1] = 0;
@@ -134,10 +135,10 @@ __global__ void __launch_bounds__(kScanT) k_scan_apply(uint64_t* __restrict__ pr
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, uint64_t* prefix,
                                uint64_t* block_sums, int64_t* keys, unsigned long long* checks,
-                               cudaStream_t st) {
+                               unsigned long long* work_ctr, cudaStream_t st) {
   const uint64_t len = (uint64_t)n_req + 1;
   k_count_tasks<<<(unsigned)((len + 255) / 256), 256, 0, st>>>(req, image, lay, n_nodes, n_req, k_max, prefix,
-                                                                keys, checks);
+                                                                keys, checks, work_ctr);
   const uint32_t nb = (uint32_t)((len + kScanChunk - 1) / kScanChunk);
   dim3 g(nb, k_max);
   k_scan_reduce<<<g, kScanT, 0, st>>>(prefix, len, block_sums, nb);
@@ -806,11 +807,20 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
 
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint64_t T = pre[A.n_req];
-  const uint64_t sb = T * A.rank / A.world, se = T * (A.rank + 1) / A.world;
-  const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x, g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const uint64_t len = se - sb;
-  const uint64_t t0 = sb + len * g / nthr, t1 = sb + len * (g + 1) / nthr;
-  if (t0 >= t1) return;
+  // Work split: the segment's task list is cut into NC = world x (nthr/32) x kDyn chunks
+  // of 32 equal contiguous pieces (one per lane).  Rank `rank` owns chunks
+  // j * world + rank; its warps grab them dynamically (atomic counter, zeroed by the count
+  // kernel), so a warp whose pieces are cheap (skipped stage-0 profiles, no rescans) takes
+  // more of them and the launch ends when the work does, not with the slowest static
+  // share.  Ranks interleave at the grain of one chunk, so each samples the whole batch
+  // (contiguous 1/world ranges measured up to 1.2x apart on C5).  Exact cover needs the
+  // same nthr on every rank (same kernel and device type).  DESIGN.md §4.3, §7.
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t NC = (nthr >> 5) * kDyn * A.world, NT = NC * 32;
+  const uint64_t Tq = T / NT, Tr = T % NT;  // piece u = [Tq u + Tr u / NT, ...): no overflow
+  auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
+  unsigned long long* ctr = A.work_ctr + KS;
 
   SearchState<KS> c;
   c.sm = tbl;
@@ -823,6 +833,14 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
 #pragma unroll
   for (int i = 0; i < KS; ++i) PK *= kP;
 
+  for (;;) {
+  unsigned long long jg = 0;
+  if (lane == 0) jg = atomicAdd(ctr, 1ull);
+  jg = __shfl_sync(0xffffffffu, jg, 0);
+  const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
+  if (chunk >= NC) break;
+  const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
+  if (t0 >= t1) continue;
   uint64_t task = t0;
   uint32_t r = find_request(pre, A.n_req, task);
   uint64_t m = task - pre[r], cnt = pre[r + 1] - pre[r], done = 0;
@@ -901,6 +919,7 @@ __global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search
     }
   }
   flush();
+  }  // grab loop
 }
 
 template <int KS, bool V, bool TG>

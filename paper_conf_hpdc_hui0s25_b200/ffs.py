@@ -54,6 +54,7 @@ _sig = {
     "ffs_last_error": ([_vp], C.c_char_p),
     "ffs_stage_tables": ([_vp, C.POINTER(_Profiles), C.POINTER(_Table), C.POINTER(_Cluster)], _i32),
     "ffs_plan_keys": ([_vp, _vp, _vp, _u32, _u32, _u32, _u32, _vp, _vp, _vp], _i32),
+    "ffs_plan_keys_range": ([_vp, _vp, _vp, _u32, _u32, _u32, _u32, _u32, _u32, _vp, _vp, _vp], _i32),
     "ffs_plan_decode": ([_vp, _vp, _vp, _vp, _u32, _u32, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_plan_batch": ([_vp, _vp, _vp, _u32, _u32, _vp, _vp], _i32),
     "ffs_plan_batch_host": ([_vp, _vp, _vp, _u32, _u32, _vp, _vp], _i32),
@@ -155,6 +156,17 @@ class Planner:
             keys = torch.empty(n, dtype=torch.int64, device=slo.device)
         self._check(_lib.ffs_plan_keys(self._h, _ptr(req), _ptr(slo), n, int(k_max), int(rank), int(world),
                                        _ptr(keys), _ptr(checks), _stream(stream)))
+        return keys
+
+    def plan_keys_range(self, req, slo, k_max: int, k_first: int, k_last: int, rank: int = 0, world: int = 1,
+                        keys=None, checks=None, stream=None):
+        """Segments k_first..k_last; k_first > 1 continues from (and prunes against) `keys`."""
+        import torch
+        n = int(slo.numel())
+        if keys is None:
+            keys = torch.empty(n, dtype=torch.int64, device=slo.device)
+        self._check(_lib.ffs_plan_keys_range(self._h, _ptr(req), _ptr(slo), n, int(k_max), int(k_first), int(k_last),
+                                             int(rank), int(world), _ptr(keys), _ptr(checks), _stream(stream)))
         return keys
 
     # ---- A6 / A8 -------------------------------------------------------------------

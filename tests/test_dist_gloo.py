@@ -15,17 +15,18 @@ import torch.multiprocessing as mp
 from paper_conf_hpdc_hui0s25_b200 import dist as D
 
 KEY_NONE = np.iinfo(np.int64).max
+CHUNKS, GRAIN = 3, 2  # emulated chunks per rank (warps x kDyn) and pieces per chunk (warp)
 
 
-def emulated_shard_keys(prob, rank, world):
-    """Per-request minimum key over the tasks of `rank` in every stage-count segment."""
+def emulated_shard_keys(prob, rank, world, k_first=1, k_last=None):
+    """Per-request minimum key over the tasks of `rank` in stage-count segments
+    k_first..k_last (default: all)."""
     from helpers import candidate_keys
     cands = [candidate_keys(prob, r) for r in range(prob.R)]
     keys = np.full(prob.R, KEY_NONE, dtype=np.int64)
-    for k in range(1, prob.k_max + 1):
+    for k in range(k_first, (k_last or prob.k_max) + 1):
         tasks = [(r, rk) for r in range(prob.R) for rk in sorted({c[1] for c in cands[r] if c[0] == k})]
-        lo, hi = D.task_shard(len(tasks), rank, world)
-        mine = set(tasks[lo:hi])
+        mine = {t for lo, hi in D.task_shard(len(tasks), rank, world, CHUNKS, GRAIN) for t in tasks[lo:hi]}
         for r in range(prob.R):
             for kk, rk, key in cands[r]:
                 if kk == k and key is not None and (r, rk) in mine:
@@ -38,9 +39,18 @@ class FakePlanner:
 
     def __init__(self, prob):
         self.prob = prob
+        self.calls = []
 
     def plan_keys(self, req, slo, k_max, rank, world, keys=None, stream=None):
+        self.calls.append((1, k_max))
         keys.copy_(torch.from_numpy(emulated_shard_keys(self.prob, rank, world)))
+        return keys
+
+    def plan_keys_range(self, req, slo, k_max, k_first, k_last, rank, world, keys=None, stream=None):
+        """ffs_plan_keys_range contract: k_first == 1 overwrites, later ranges min-combine."""
+        self.calls.append((k_first, k_last))
+        part = torch.from_numpy(emulated_shard_keys(self.prob, rank, world, k_first, k_last))
+        keys.copy_(part if k_first == 1 else torch.minimum(keys, part))
         return keys
 
     def plan_decode(self, req, slo, keys, k_max, out=None, stream=None):
@@ -60,7 +70,10 @@ def _worker(rank, world, port, q):
         keys = torch.empty(R, dtype=torch.int64)
         req = torch.zeros((R, 8), dtype=torch.uint8)
         slo = torch.zeros(R, dtype=torch.int32)
-        keys, plans, (lo, hi) = D.plan_step(FakePlanner(prob), req, slo, prob.k_max, rank, world, keys)
+        fp = FakePlanner(prob)
+        keys, plans, (lo, hi) = D.plan_step(fp, req, slo, prob.k_max, rank, world, keys)
+        # one sharded range per segment, an exchange after each
+        assert fp.calls == [(k, k) for k in range(1, prob.k_max + 1)]
         # sentinel survives MIN, and a MIN of partial minima is the global minimum
         t = torch.tensor([KEY_NONE, 5, KEY_NONE], dtype=torch.int64) if rank == 0 else \
             torch.tensor([KEY_NONE, KEY_NONE, 3], dtype=torch.int64)
@@ -107,10 +120,12 @@ def test_sharded_step_matches_oracle_over_gloo(world):
 def test_shard_partitions_are_exact():
     for T in (0, 1, 7, 1000, 2**41 + 3):
         for world in (1, 2, 3, 8):
-            b = [D.task_shard(T, g, world) for g in range(world)]
-            assert b[0][0] == 0 and b[-1][1] == T
-            assert all(x[1] == y[0] for x, y in zip(b, b[1:]))
-            assert max(h - l for l, h in b) - min(h - l for l, h in b) <= 1
+            for chunks, grain in ((1, 1), (3, 2), (1184 * 8, 32)):
+                pieces = sorted(p for g in range(world) for p in D.task_shard(T, g, world, chunks, grain))
+                assert pieces[0][0] == 0 and pieces[-1][1] == T  # exact cover, no overlap
+                assert all(x[1] == y[0] for x, y in zip(pieces, pieces[1:]))
+                sizes = [sum(h - l for l, h in D.task_shard(T, g, world, chunks, grain)) for g in range(world)]
+                assert max(sizes) - min(sizes) <= chunks * grain  # pieces within 1 of each other
 
 
 def test_emulated_shards_cover_every_candidate():

@@ -145,6 +145,38 @@ def test_sharding_invariance(F, planner, world):
     np.testing.assert_array_equal(p1.view(np.uint8), pw.view(np.uint8))
 
 
+@pytest.mark.parametrize("split", [1, 2, 3])
+def test_keys_range_composition(F, planner, split):
+    """ffs_plan_keys_range: segments 1..split then split+1..K continuing from the combined
+    keys give the keys and checksums of one ffs_plan_keys call, on every shard
+    (world 3: each shard's ranges, MIN over shards between and after, as dist.plan_step)."""
+    prob = W.config2(R=2048)
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    K = prob.k_max
+    ref = planner.plan_keys(req, slo, K).cpu().numpy()
+    ck_ref = torch.empty(3 * prob.R, dtype=torch.int64, device="cuda")
+    planner.plan_keys(req, slo, K, checks=ck_ref)
+    keys = torch.empty((3, prob.R), dtype=torch.int64, device="cuda")
+    cks = torch.empty((3, 3 * prob.R), dtype=torch.int64, device="cuda")
+    for g in range(3):
+        planner.plan_keys_range(req, slo, K, 1, split, g, 3, keys=keys[g], checks=cks[g])
+    comb = keys.min(dim=0).values
+    for g in range(3):
+        keys[g].copy_(comb)
+        planner.plan_keys_range(req, slo, K, split + 1, K, g, 3, keys=keys[g], checks=cks[g])
+    np.testing.assert_array_equal(keys.min(dim=0).values.cpu().numpy(), ref)
+    tot = cks.cpu().numpy().view(np.uint64).sum(axis=0, dtype=np.uint64)  # SUM mod 2^64
+    np.testing.assert_array_equal(tot, ck_ref.cpu().numpy().view(np.uint64))
+    ms = planner.segment_times()
+    assert all(ms[k] > 0 for k in range(K)) and all(m == 0 for m in ms[K:])
+    with pytest.raises(F.FFSError) as e:
+        planner.plan_keys_range(req, slo, K, 3, 2, keys=keys[0])
+    assert e.value.status == F.FFS_ERR_RANGE
+    with pytest.raises(F.FFSError):
+        planner.plan_keys_range(req, slo, K, 1, K + 1, keys=keys[0])
+
+
 def test_c5_bench_configuration_sampled(F, planner):
     """C5 at full size in the launch configuration bench.py times (world 1, production
     path), checked on a stratified sample against the oracle."""
