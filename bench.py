@@ -42,7 +42,9 @@ def candidates_per_request(prob, k_max):
 
 
 def segment_candidates(prob, k_max, rank, world):
-    """Candidates of segment ks processed by shard `rank` (same split as the kernel)."""
+    """Candidates of segment ks processed by shard `rank`: T/world tasks (the kernel deals
+    equal pieces round-robin, dist.task_shard; a rank's count is within one task per piece
+    of T/world, < 1e-4 relative at C5)."""
     n = prob.chain_len()[prob.req["func"]]
     out = []
     for ks in range(1, k_max + 1):
