@@ -423,7 +423,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   const size_t smem = tables_global ? 0 : (size_t)c->lay.words * 4;
   int block4 = kBlock;
   while (block4 > 32 && smem + (size_t)440 * block4 > kMaxSmem) block4 -= 32;
-  auto blk = [&](int k) { return k == 4 ? block4 : kBlock; };
+  auto blk = [&](int k) { return k == 4 ? block4 : search_block(k); };
   auto shm = [&](int k) { return smem + (k == 4 ? (size_t)440 * block4 : 0); };
   if (c->occ_smem != smem + 1) {  // (smem = 0 <=> tables in global memory)
     for (int v = 0; v < 2; ++v)

@@ -22,6 +22,10 @@ constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #define FFS_MINB4 1
 #endif
 constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
+// KS = 3 keeps every table in registers; capped at 168 registers it runs 12 warps per SM
+// and is faster (C5: 4.3 -> 3.9 ms); KS = 4 is fastest at 8 warps with 254 registers
+// (DESIGN.md §4.3).  The KS = 4 CTA may shrink further to fit its shared-memory windows.
+constexpr int search_block(int ks) { return ks == 3 ? 384 : kBlock; }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole

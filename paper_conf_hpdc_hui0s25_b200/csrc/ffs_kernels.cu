@@ -786,7 +786,7 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
 }
 
 template <int KS, bool VERIFY, bool TG>
-__global__ void __launch_bounds__(kBlock, KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
+__global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
   // A0: stage the table image into shared memory (16-byte copies); an image too large
   // for shared memory is read from global memory through L1 instead (A.tables_global)
