@@ -41,11 +41,20 @@ def candidates_per_request(prob, k_max):
     return S[prob.req["func"]]
 
 
+def enumerated(prob):
+    """Requests whose candidates the GPU enumerates: a node without any free slice admits
+    no candidate, so its requests are INFEASIBLE without enumeration (R37) and
+    their candidates are not counted as scored."""
+    free = np.zeros(prob.n_nodes, dtype=np.int64)
+    np.add.at(free, prob.slices["node"][prob.slices["busy"] == 0].astype(np.int64), 1)
+    return free[prob.req["node"]] > 0
+
+
 def segment_candidates(prob, k_max, rank, world):
     """Candidates of segment ks processed by shard `rank`: T/world tasks (the kernel deals
     equal pieces round-robin, dist.task_shard; a rank's count is within one task per piece
     of T/world, < 1e-4 relative at C5)."""
-    n = prob.chain_len()[prob.req["func"]]
+    n = prob.chain_len()[prob.req["func"]] * enumerated(prob)
     out = []
     for ks in range(1, k_max + 1):
         tab = np.array([comb(m - 1, ks - 1) if m >= ks else 0 for m in range(33)], dtype=np.int64)
@@ -389,7 +398,7 @@ def main():
         t = torch.tensor([ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
-    total_cands = int(candidates_per_request(prob, K).sum())
+    total_cands = int(candidates_per_request(prob, K)[enumerated(prob)].sum())
     value = total_cands * args.steps / (ms * 1e-3)
     plans_per_s = R * args.steps / (ms * 1e-3)
 

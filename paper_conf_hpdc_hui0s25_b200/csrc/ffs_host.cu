@@ -87,7 +87,9 @@ struct ffs_ctx {
   uint32_t seg_mask = 0;                                 // segments timed since the last k_first = 1
   // task prefix of the last search call (reused by continuation ranges, k_first > 1)
   const void* pre_req = nullptr;
+  const void* pre_nf = nullptr;
   uint32_t pre_n = 0, pre_kmax = 0;
+  bool pre_skip = false;
 };
 
 static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
@@ -403,12 +405,15 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   // from (and prune against) whatever the caller combined into d_keys in between
   const bool init = k_first == 1;
   CK(c->work_ctr.ensure((kMaxK + 1) * 8), "cudaMalloc(work_ctr)");
-  if (!init && c->pre_req == d_req && c->pre_n == n_req && c->pre_kmax == k_max) {
+  const uint64_t* nf = node_free ? node_free : c->node_free.as<uint64_t>();
+  const bool skip_full = d_checks == nullptr;  // verify mode enumerates every request
+  if (!init && c->pre_req == d_req && c->pre_n == n_req && c->pre_kmax == k_max && c->pre_nf == nf &&
+      c->pre_skip == skip_full) {
     // continuation of the same batch: the task prefix is still valid; reset the counters
     CK(cudaMemsetAsync(c->work_ctr.p, 0, (kMaxK + 1) * 8, st), "reset chunk counters");
   } else {
-    CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, c->prefix.as<uint64_t>(),
-                          c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
+    CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, nf, skip_full,
+                          c->prefix.as<uint64_t>(), c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
                           init ? reinterpret_cast<unsigned long long*>(d_checks) : nullptr,
                           c->work_ctr.as<unsigned long long>(), st),
        "count/scan kernels");
@@ -416,6 +421,8 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   c->pre_req = d_req;
   c->pre_n = n_req;
   c->pre_kmax = k_max;
+  c->pre_nf = nf;
+  c->pre_skip = skip_full;
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows
   // of the KS = 4 kernel (440 B per thread); the KS = 4 CTA shrinks when both do not fit.
   // An image that leaves no room is read from global memory instead (tables_global).

@@ -79,9 +79,9 @@ struct DecodeArgs {
 // launchers (ffs_kernels.cu)
 constexpr int kDyn = 8;  // search chunks per warp and rank (dynamic grab, k_plan_search)
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
-                               uint32_t n_nodes, uint32_t n_req, uint32_t k_max, uint64_t* prefix,
-                               uint64_t* block_sums, int64_t* keys, unsigned long long* checks,
-                               unsigned long long* work_ctr, cudaStream_t st);
+                               uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
+                               bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
+                               unsigned long long* checks, unsigned long long* work_ctr, cudaStream_t st);
 cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st);
 cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,

@@ -38,6 +38,7 @@ __device__ __forceinline__ uint32_t binom(const uint32_t* img, const ImageLayout
 // ====================================================================================
 __global__ void k_count_tasks(const ffs_request* __restrict__ req, const uint32_t* __restrict__ img,
                               ImageLayout lay, uint32_t n_nodes, uint32_t n_req, uint32_t K,
+                              const uint64_t* __restrict__ node_free, uint32_t skip_full,
                               uint64_t* __restrict__ prefix, int64_t* __restrict__ keys,
                               unsigned long long* __restrict__ checks, unsigned long long* __restrict__ work_ctr) {
   uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
@@ -47,6 +48,9 @@ __global__ void k_count_tasks(const ffs_request* __restrict__ req, const uint32_
   if (r < n_req) {
     ffs_request q = req[r];
     if (q.func < lay.F && q.node < n_nodes) n = img[lay.o_fdesc + 4 * q.func + 1];
+    // a node without any free slice admits no candidate: no tasks (INFEASIBLE without
+    // enumeration, R37); verify mode enumerates them anyway for the checksums
+    if (skip_full && n && node_free[q.node] == 0) n = 0;
     if (keys) keys[r] = (int64_t)kKeyNone;
     if (checks) {
       checks[3ull * r] = 0;
@@ -133,12 +137,12 @@ __global__ void __launch_bounds__(kScanT) k_scan_apply(uint64_t* __restrict__ pr
 }
 
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
-                               uint32_t n_nodes, uint32_t n_req, uint32_t k_max, uint64_t* prefix,
-                               uint64_t* block_sums, int64_t* keys, unsigned long long* checks,
-                               unsigned long long* work_ctr, cudaStream_t st) {
+                               uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
+                               bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
+                               unsigned long long* checks, unsigned long long* work_ctr, cudaStream_t st) {
   const uint64_t len = (uint64_t)n_req + 1;
-  k_count_tasks<<<(unsigned)((len + 255) / 256), 256, 0, st>>>(req, image, lay, n_nodes, n_req, k_max, prefix,
-                                                                keys, checks, work_ctr);
+  k_count_tasks<<<(unsigned)((len + 255) / 256), 256, 0, st>>>(req, image, lay, n_nodes, n_req, k_max, node_free,
+                                                                skip_full ? 1u : 0u, prefix, keys, checks, work_ctr);
   const uint32_t nb = (uint32_t)((len + kScanChunk - 1) / kScanChunk);
   dim3 g(nb, k_max);
   k_scan_reduce<<<g, kScanT, 0, st>>>(prefix, len, block_sums, nb);
