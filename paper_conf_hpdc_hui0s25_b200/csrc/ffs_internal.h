@@ -21,12 +21,18 @@ constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #ifndef FFS_MINB4
 #define FFS_MINB4 1
 #endif
+#ifndef FFS_KS4_F32
+#define FFS_KS4_F32 0  // 1: the f32x2 KS = 4 body (ks4_pair) instead of the f16x2 pre-filter
+#endif
 constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 // KS = 3 keeps every table in registers; capped at 168 registers it runs 12 warps per SM
-// and is faster (C5: 4.3 -> 3.9 ms); KS = 4 is fastest at 8 warps with 254 registers
-// (DESIGN.md §4.3).  The KS = 4 CTA may shrink further to fit its shared-memory windows.
-constexpr int search_block(int ks) { return ks == 3 ? 384 : kBlock; }
+// and is faster (C5: 4.3 -> 3.9 ms).  The f16x2 KS = 4 kernel needs ~150 registers and
+// also runs 12 warps per SM (C5: 74.2 ms at 8 warps -> 72.0 ms).  The
+// KS = 4 CTA may shrink to fit its shared-memory windows.
+constexpr int search_block(int ks) { return (ks == 3 || (ks == 4 && !FFS_KS4_F32)) ? 384 : kBlock; }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
+// bytes of per-thread shared-memory windows of the KS = 4 kernel: 5 profiles x 11 packed pairs
+constexpr size_t kWin4 = FFS_KS4_F32 ? 440 : 220;
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
 // image into shared memory once per CTA (A0 of DESIGN.md §4); every other kernel reads
@@ -58,6 +64,7 @@ struct SearchArgs {
   unsigned long long* misses;   // debug counter (verify mode)
   uint32_t tables_global;       // 1: read the image from global memory (too large for smem)
   unsigned long long* work_ctr; // [kMaxK + 1] chunk counters, zeroed by the count kernel
+  uint32_t zero;                // always 0: an operand ptxas cannot fold (ks4_pair_h's IADD3)
 };
 
 struct DecodeArgs {

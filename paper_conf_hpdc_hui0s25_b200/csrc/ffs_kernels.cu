@@ -166,6 +166,9 @@ struct SearchState {
   uint64_t idx_base;  // offk[n][KS] + rank * P^KS
   int64_t best;
   float alpha;        // scale of sum t^2 in the balance filter
+  float alpha_h;      // the same with the wider margin of the f16x2 pre-filter (KS = 4)
+  float tmin, tmax;   // KS = 4: sum over the chain of the min / max component latency over
+                      // all profiles (bounds of every candidate's T, for the f16 scale)
   bool none_can_win;  // best's cvq/k already unbeatable by any KS-stage candidate
   // mask
   int bnd[KS + 1];
@@ -181,6 +184,7 @@ struct SearchState {
 
 template <int KS>
 __device__ __forceinline__ void set_threshold(SearchState<KS>& c) {
+  float ap = 0.f;  // alpha' = 1024 KS / (1025 + c*), rounded down; 0 while nothing is known
   if ((uint64_t)c.best == kKeyNone) {
     c.alpha = 0.f;
     c.none_can_win = false;
@@ -193,6 +197,12 @@ __device__ __forceinline__ void set_threshold(SearchState<KS>& c) {
     // filter: (sum t)^2 > alpha * sum t^2 with alpha rounded down by a 2^-16 margin
     // 1024*KS*(1 - 2^-16) = KS*65535/64 is exact in fp32; the quotient is rounded down
     c.alpha = __fdiv_rd((float)(KS * 65535) * (1.f / 64.f), (float)(1025 + cthr));
+    if constexpr (KS == 4) ap = __fdiv_rd((float)(1024 * KS), (float)(1025 + cthr));
+  }
+  if constexpr (KS == 4) {
+    // f16x2 pre-filter (ks4_pair_h): alpha_h = alpha' - 2^-6 (KS + 1 + alpha'), every step
+    // rounded down; the margin covers the f16 rounding (DESIGN.md §4.3 "f16x2 pre-filter")
+    c.alpha_h = __fsub_rd(__fmul_rd(ap, 1.f - 1.f / 64.f), (float)(KS + 1) * (1.f / 64.f));
   }
   c.blim = c.none_can_win ? -1.f : c.blim_raw;
 #pragma unroll
@@ -698,6 +708,176 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
   if (haveB) pair_rescan<4, VERIFY>(c, G[1], pendB, VERIFY ? kAll : pendB, 625, misses);
 }
 
+// ---- KS = 4, f16x2 pre-filter ---------------------------------------
+// The same candidate-pair core in packed half precision: mask A in the low and mask B in
+// the high f16 of one 32-bit register, so one HFMA2/HADD2 scores a candidate of each and
+// one LOP3 folds both sign bits (4 instructions per candidate pair instead of 3 f32x2 +
+// 2 LOP3).  Each half is scaled by its own power of two sigma (exact) so that every
+// feasible candidate's T sigma <= 32: no overflow (T^2, alpha Sigma t^2 < 2^13) and, with
+// T sigma >= 1/8 checked per half, negligible underflow.  The filter is conservative by
+// construction: alpha_h (set_threshold) leaves a 2^-6 (KS + 1 + alpha') Sigma t^2 margin
+// for the f16 rounding and the SLO slack is widened by 2^-7 Blim; a block with a possible
+// winner is always flagged, flagged blocks are re-evaluated exactly (pair_rescan), so the
+// pre-filter decides only how much exact work runs, never a result.
+typedef uint32_t h2;
+__device__ __forceinline__ h2 h2pack(float lo, float hi) {
+  h2 r;
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+__device__ __forceinline__ h2 h2add(h2 a, h2 b) {
+  h2 d;
+  asm("add.rn.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
+__device__ __forceinline__ h2 h2sub(h2 a, h2 b) {
+  h2 d;
+  asm("sub.rn.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
+__device__ __forceinline__ h2 h2fma(h2 a, h2 b, h2 c) {
+  h2 d;
+  asm("fma.rn.f16x2 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
+  return d;
+}
+
+// SLO slack in "guarded" form for the integer SWAR test of the inner loop: per f16 half,
+// bit 15 (guard) | the magnitude bits of slack - v3 when it is >= 0, else the guard alone
+// (magnitude 0).  For S3 >= 0 (a sum of non-negative f16, never NaN), the 32-bit integer
+// difference guarded - bits(S3) keeps the halves apart (every half's minuend >= 2^15 >
+// S3's bits) and its bit 15 / 31 is set iff slack - v3 >= S3 in f16: the same decision as
+// the sign of an f16 subtraction, moved from the FMA pipe to one IADD3 on the ALU pipe.
+__device__ __forceinline__ uint32_t h2guard(h2 w) {
+  const uint32_t neg = w & 0x80008000u;
+  const uint32_t m = neg - (neg >> 15);  // 0x7fff in every half whose sign bit is set
+  return (w & ~m) | 0x80008000u;
+}
+
+// a - b + zero with an opaque zero register: a three-operand add, which only IADD3 (ALU
+// pipe) encodes, so ptxas cannot move the test to an IMAD.IADD on the busier FMA pipe
+__device__ __forceinline__ uint32_t isub(uint32_t a, uint32_t b, uint32_t zero) {
+  uint32_t d;
+  asm("{.reg .u32 t; sub.u32 t, %1, %2; add.u32 %0, t, %3;}" : "=r"(d) : "r"(a), "r"(b), "r"(zero));
+  return d;
+}
+
+struct WinH {
+  h2 s1, s2[2], s3[3];
+};
+
+// rows: per thread and profile x, 11 packed f16 pairs in [x][k][thread] order (4-byte,
+// conflict-free); window e (e = 1 when x is the stage-0 profile) is read at offset e.
+template <bool VERIFY>
+__device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
+                                           unsigned long long* misses, uint32_t zero) {
+  const float INF = __int_as_float(0x7f800000);
+  const int tid = threadIdx.x, nb = blockDim.x;
+  Geo4 G[2];
+  geo4(c, maskA, G[0]);
+  geo4(c, maskB, G[1]);
+  if (!haveB) G[1].blim = -1.f;  // dummy lane: nothing passes
+  const float al = c.alpha_h, one_m_a = 1.f - c.alpha_h;
+  float f[2][4][kP];
+#pragma unroll
+  for (int h = 0; h < 2; ++h)
+#pragma unroll
+    for (int s = 0; s < 4; ++s) geo_lat(c, G[h], s, f[h][s]);
+  // per half: scale sigma = 2^(5 - E) with M = min(Blim, tmax) <= 2^E, so every feasible
+  // candidate (T <= M) has T sigma <= 32; the SLO slack is M sigma (1 + 2^-7) (clamping Blim
+  // to tmax changes no candidate's SLO outcome: T <= tmax always)
+  float sig[2], slack[2];
+  bool wide[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const float bl = G[h].blim;
+    const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+    const uint32_t mb = __float_as_uint(M);
+    const int E = (int)((mb >> 23) & 255u) - 127 + ((mb & 0x7fffffu) != 0u);  // M <= 2^E
+    sig[h] = __int_as_float((127 + 5 - E) << 23);
+    wide[h] = bl >= 0.f && c.tmin * sig[h] < 0.125f;  // f16 underflow could matter: exact path
+    slack[h] = bl >= 0.f ? M * sig[h] * (1.f + 1.f / 128.f) : -INF;
+  }
+  constexpr h2 kInf2 = 0x7c007c00u, kGuard = 0x80008000u;
+  h2 a1[kP], a2[kP], t2[kP], cc[kP];
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const uint32_t cap = c.sm[c.o_cap + x];
+    float fs[2][4], vm[2][4];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int s = 0; s < 4; ++s) {
+        fs[h][s] = f[h][s][x] * sig[h];
+        vm[h][s] = (G[h].memst[s] <= cap) ? fs[h][s] : INF;  // memory folded per half
+      }
+    // the free-slice gates depend only on the node: applied to the packed pair
+    const h2 p0 = h2pack(vm[0][0], vm[1][0]), p1 = h2pack(vm[0][1], vm[1][1]), p2 = h2pack(vm[0][2], vm[1][2]);
+    const h2 p3 = h2guard(h2pack(slack[0] - vm[0][3], slack[1] - vm[1][3]));
+    a1[x] = h2pack(al * (fs[0][1] * fs[0][1]), al * (fs[1][1] * fs[1][1]));
+    a2[x] = h2pack(al * (fs[0][2] * fs[0][2]), al * (fs[1][2] * fs[1][2]));
+    t2[x] = h2pack(fs[0][3] + fs[0][3], fs[1][3] + fs[1][3]);
+    cc[x] = h2pack(one_m_a * (fs[0][3] * fs[0][3]), one_m_a * (fs[1][3] * fs[1][3]));
+    //   [v1[0], v1[1], v2[0], v2[1], v2[2], guarded slack-v3[0..3], v0[0], -alpha t0^2]
+    h2* r = rows + (x * 11) * nb + tid;
+    r[0 * nb] = fr > 0 ? p1 : kInf2;
+    r[1 * nb] = fr > 1 ? p1 : kInf2;
+    r[2 * nb] = fr > 0 ? p2 : kInf2;
+    r[3 * nb] = fr > 1 ? p2 : kInf2;
+    r[4 * nb] = fr > 2 ? p2 : kInf2;
+    r[5 * nb] = fr > 0 ? p3 : kGuard;
+    r[6 * nb] = fr > 1 ? p3 : kGuard;
+    r[7 * nb] = fr > 2 ? p3 : kGuard;
+    r[8 * nb] = fr > 3 ? p3 : kGuard;
+    r[9 * nb] = fr > 0 ? p0 : kInf2;
+    r[10 * nb] = h2pack(-al * (fs[0][0] * fs[0][0]), -al * (fs[1][0] * fs[1][0]));
+  }
+  uint32_t pendA = 0, pendB = 0;
+#pragma unroll 1
+  for (int d0 = 0; d0 < kP; ++d0) {
+    WinH W[kP];
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const int e = (x == d0);
+      const h2* r = rows + (x * 11 + e) * nb + tid;
+      W[x].s1 = r[0];
+      W[x].s2[0] = r[2 * nb];
+      W[x].s2[1] = r[3 * nb];
+      W[x].s3[0] = r[5 * nb];
+      W[x].s3[1] = r[6 * nb];
+      W[x].s3[2] = r[7 * nb];
+    }
+    const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
+    const h2 NL1 = rows[(d0 * 11 + 10) * nb + tid];  // -alpha t0^2
+#pragma unroll
+    for (int d1 = 0; d1 < kP; ++d1) {
+      const h2 S2 = h2add(S1, W[d1].s1), NL2 = h2sub(NL1, a1[d1]);
+      uint32_t acc[kP];
+#pragma unroll
+      for (int q = 0; q < kP; ++q) {
+        const h2 S3 = h2add(S2, W[q].s2[q == d1]);
+        const h2 U = h2fma(S3, S3, h2sub(NL2, a2[q]));
+        acc[q] = ~0u;
+#pragma unroll
+        for (int p = 0; p < kP; ++p) {
+          const h2 z = h2add(h2fma(S3, t2[p], cc[p]), U);
+          // bit 15/31 clear <=> slack - v3 < S3: SLO / memory / free miss (h2guard)
+          const uint32_t ok = isub(W[p].s3[(p == d1) + (p == q)], S3, zero);
+          acc[q] &= z | ~ok;
+        }
+      }
+      const uint32_t m = acc[0] & acc[1] & acc[2] & acc[3] & acc[4];
+      pendA |= (((m >> 15) & 1u) ^ 1u) << (kP * d0 + d1);
+      pendB |= ((m >> 31) ^ 1u) << (kP * d0 + d1);
+    }
+  }
+  constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
+  if (wide[0]) pendA = kAll;  // dynamic range too wide for f16: every block exactly
+  if (wide[1]) pendB = kAll;
+  pair_rescan<4, VERIFY>(c, G[0], pendA, VERIFY ? kAll : pendA, 0, misses);
+  if (haveB) pair_rescan<4, VERIFY>(c, G[1], pendB, VERIFY ? kAll : pendB, 625, misses);
+}
+
 template <int KS, bool VERIFY>
 __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses) {
   uint32_t pend = 0;  // one bit per block of P*P candidates
@@ -866,6 +1046,24 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     c.best = *reinterpret_cast<volatile const int64_t*>(A.keys + r);  // earlier segments' minimum
     best0 = c.best;
     if constexpr (KS >= 2) set_threshold(c);
+    if constexpr (KS == 4) {
+      float tmin = 0.f, tmax = 0.f;
+      const uint32_t* rowp = tbl + A.lay.o_pl + c.row0 * kRowW;
+      float4 la = *reinterpret_cast<const float4*>(rowp);
+      float l4 = __uint_as_float(rowp[4]);
+      for (uint32_t i = 0; i < c.n; ++i) {
+        rowp += kRowW;
+        const float4 lb = *reinterpret_cast<const float4*>(rowp);
+        const float lb4 = __uint_as_float(rowp[4]);
+        const float d0 = lb.x - la.x, d1 = lb.y - la.y, d2 = lb.z - la.z, d3 = lb.w - la.w, d4 = lb4 - l4;
+        tmin += fminf(fminf(fminf(d0, d1), fminf(d2, d3)), d4);
+        tmax += fmaxf(fmaxf(fmaxf(d0, d1), fmaxf(d2, d3)), d4);
+        la = lb;
+        l4 = lb4;
+      }
+      c.tmin = tmin;  // upper/lower bounds; fp32 rounding above 2^24 is covered by the 2^-7 slack margin
+      c.tmax = tmax;
+    }
     c.nfeas = 0;
     c.ksum = 0;
     done = 0;
@@ -903,7 +1101,11 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
       // two consecutive masks of the same request per iteration (ks3_pair / ks4_pair)
       const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
       const uint32_t maskB = haveB ? gosper_next(mask) : mask;
+#if FFS_KS4_F32
       if constexpr (KS == 4) ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<f2*>(rows), A.misses);
+#else
+      if constexpr (KS == 4) ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero);
+#endif
       else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses);
       if (haveB) {
         step = 2;
