@@ -424,12 +424,15 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   c->pre_nf = nf;
   c->pre_skip = skip_full;
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows
-  // of the KS = 4 kernel (kWin4 B per thread); the KS = 4 CTA shrinks when both do not fit.
-  // An image that leaves no room is read from global memory instead (tables_global).
-  const bool tables_global = (size_t)c->lay.words * 4 + kWin4 * 64 > kMaxSmem;
+  // of the KS = 4 kernel (kWin4 B per thread).  The f16x2 kernel's window stride is the
+  // compile-time CTA size (immediate LDS/STS offsets); an image that does not fit next to
+  // its windows is read from global memory instead (tables_global).  The f32x2 variant
+  // shrinks its CTA first.
+  const size_t min_win = FFS_KS4_F32 ? kWin4 * 64 : kWin4 * search_block(4);
+  const bool tables_global = (size_t)c->lay.words * 4 + min_win > kMaxSmem;
   const size_t smem = tables_global ? 0 : (size_t)c->lay.words * 4;
   int block4 = search_block(4);
-  while (block4 > 32 && smem + kWin4 * block4 > kMaxSmem) block4 -= 32;
+  while (FFS_KS4_F32 && block4 > 32 && smem + kWin4 * block4 > kMaxSmem) block4 -= 32;
   auto blk = [&](int k) { return k == 4 ? block4 : search_block(k); };
   auto shm = [&](int k) { return smem + (k == 4 ? kWin4 * block4 : 0); };
   if (c->occ_smem != smem + 1) {  // (smem = 0 <=> tables in global memory)

@@ -771,7 +771,8 @@ template <bool VERIFY>
 __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
                                            unsigned long long* misses, uint32_t zero) {
   const float INF = __int_as_float(0x7f800000);
-  const int tid = threadIdx.x, nb = blockDim.x;
+  constexpr int nb = search_block(4);  // window stride: the CTA size, fixed at compile time
+  const int tid = threadIdx.x;
   Geo4 G[2];
   geo4(c, maskA, G[0]);
   geo4(c, maskB, G[1]);
@@ -849,6 +850,7 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     }
     const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
     const h2 NL1 = rows[(d0 * 11 + 10) * nb + tid];  // -alpha t0^2
+    uint32_t mm[kP];  // per d1: sign bits 15 / 31 clear <=> the (d0, d1) block may hold a winner
 #pragma unroll
     for (int d1 = 0; d1 < kP; ++d1) {
       const h2 S2 = h2add(S1, W[d1].s1), NL2 = h2sub(NL1, a1[d1]);
@@ -866,9 +868,18 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
           acc[q] &= z | ~ok;
         }
       }
-      const uint32_t m = acc[0] & acc[1] & acc[2] & acc[3] & acc[4];
-      pendA |= (((m >> 15) & 1u) ^ 1u) << (kP * d0 + d1);
-      pendB |= ((m >> 31) ^ 1u) << (kP * d0 + d1);
+      mm[d1] = acc[0] & acc[1] & acc[2] & acc[3] & acc[4];
+    }
+    // flagged blocks are rare: the per-block bookkeeping runs only when some block is
+    if ((mm[0] & mm[1] & mm[2] & mm[3] & mm[4] & kGuard) != kGuard) {
+      uint32_t bA = 0, bB = 0;
+#pragma unroll
+      for (int d1 = 0; d1 < kP; ++d1) {
+        bA |= ((mm[d1] >> 15) & 1u) << d1;
+        bB |= (mm[d1] >> 31) << d1;
+      }
+      pendA |= (bA ^ 31u) << (kP * d0);
+      pendB |= (bB ^ 31u) << (kP * d0);
     }
   }
   constexpr uint32_t kAll = (1u << (kP * kP)) - 1;

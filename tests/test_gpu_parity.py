@@ -553,3 +553,51 @@ def test_large_table_image_reads_tables_from_global(F, planner):
     p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
     np.testing.assert_array_equal(keys2, o["key"])
     assert planner.filter_misses() == 0
+
+
+def _f16_stress_problem(seed):
+    """KS = 4 inputs aimed at the f16x2 pre-filter's margins: latencies
+    spanning 1 us .. 2^22 us (underflow / the exact 'wide' path), stages of equal time
+    (CV = 0 ties), budgets exactly at a candidate's e2e (inclusive SLO) and far above the
+    slowest chain (scale clamped to tmax), plus nodes with one free slice per profile."""
+    rng = W.SplitMix64(seed)
+    funcs = []
+    for f in range(6):
+        n = int(rng.integers(4, 11, 1)[0])
+        kind = f % 3
+        if kind == 0:    # extreme dynamic range
+            lat = (2 ** rng.integers(0, 22, n * 5)).reshape(n, 5) + rng.integers(0, 3, n * 5).reshape(n, 5)
+        elif kind == 1:  # equal components: many exact CV ties
+            base = int(rng.integers(1000, 5000, 1)[0])
+            lat = np.tile(np.array([7, 5, 3, 2, 1]) * base, (n, 1))
+        else:            # ordinary, narrow spread
+            lat = rng.integers(900, 1100, n * 5).reshape(n, 5)
+        mem = rng.integers(1000, 9000, n).tolist()
+        xfer = rng.integers(0, 40, n).tolist()
+        funcs.append(dict(lat=np.asarray(lat).tolist(), mem=mem, xfer=xfer, load=10))
+    nodes = [[[0, 1, 2], [3, 4]], [[0, 0, 1, 1], [2, 2, 3]], [[0], [1], [2]]]
+    reqs = []
+    for f, fd in enumerate(funcs):
+        lat = np.asarray(fd["lat"], np.int64)
+        n = lat.shape[0]
+        one_stage = lat.sum(0)
+        for v in range(len(nodes)):
+            # exact e2e of a 4-stage candidate (equal stages, cuts after 0, 1, 2) and budgets around it
+            cut = [0, 1, 2]
+            stages = [lat[0:1, 0].sum(), lat[1:2, 1].sum(), lat[2:3, 2].sum(), lat[3:n, 3].sum()]
+            e2e = int(sum(stages) + sum(fd["xfer"][c] for c in cut))
+            for B in (e2e - 1, e2e, e2e + 1, int(one_stage.min()), int(one_stage.max()) * 4, 2 ** 30):
+                reqs.append((f, v, max(int(B), 1)))
+    return problem(funcs, nodes, reqs, k_max=4)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_f16_prefilter_stress(F, planner, seed):
+    prob = _f16_stress_problem(4200 + seed)
+    p, keys, ch = run_gpu(F, planner, prob)
+    o = oracle.plan(prob)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    assert planner.filter_misses() == 0
+    p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
+    np.testing.assert_array_equal(keys2, o["key"])

@@ -25,6 +25,8 @@ for _ in range(reps):
     ms = pl.segment_times()
     best = ms if best is None else [min(a, b) for a, b in zip(best, ms)]
     assert torch.equal(keys, ref)
+if best is None:
+    best = pl.segment_times()
 lib = os.path.basename(os.environ.get("FFS_LIB", "libffs.so"))
 print(f"{lib}: C{cfg} segment ms " + " ".join(f"KS{k + 1}={t:.2f}" for k, t in enumerate(best) if t > 0)
       + f"  total={sum(best):.2f}")
