@@ -29,7 +29,12 @@ constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 // and is faster (C5: 4.3 -> 3.9 ms).  The f16x2 KS = 4 kernel needs ~150 registers and
 // also runs 12 warps per SM (C5: 74.2 ms at 8 warps -> 72.0 ms).  The
 // KS = 4 CTA may shrink to fit its shared-memory windows.
-__host__ __device__ constexpr int search_block(int ks) { return (ks == 3 || (ks == 4 && !FFS_KS4_F32)) ? 384 : kBlock; }
+#ifndef FFS_BLOCK4
+#define FFS_BLOCK4 384
+#endif
+__host__ __device__ constexpr int search_block(int ks) {
+  return ks == 3 ? 384 : (ks == 4 && !FFS_KS4_F32) ? FFS_BLOCK4 : kBlock;
+}
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
 // bytes of per-thread shared-memory windows of the KS = 4 kernel: 5 profiles x 11 packed pairs
 constexpr size_t kWin4 = FFS_KS4_F32 ? 440 : 220;

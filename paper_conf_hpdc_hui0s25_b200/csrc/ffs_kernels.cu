@@ -834,7 +834,11 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     r[10 * nb] = h2pack(-al * (fs[0][0] * fs[0][0]), -al * (fs[1][0] * fs[1][0]));
   }
   uint32_t pendA = 0, pendB = 0;
+#if FFS_UNROLL_D0
+#pragma unroll
+#else
 #pragma unroll 1
+#endif
   for (int d0 = 0; d0 < kP; ++d0) {
     WinH W[kP];
 #pragma unroll
