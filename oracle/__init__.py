@@ -42,7 +42,7 @@ class _PlanArgs(C.Structure):
     _fields_ = [
         ("P", C.c_int), ("gpcs", C.c_void_p), ("cap_mib", C.c_void_p),
         ("F", C.c_int), ("comp_off", C.c_void_p), ("lat_us", C.c_void_p), ("mem_mib", C.c_void_p),
-        ("xfer_us", C.c_void_p), ("load_us", C.c_void_p),
+        ("xfer_us", C.c_void_p), ("load_us", C.c_void_p), ("max_stage_us", C.c_void_p),
         ("n_nodes", C.c_int), ("n_slices", C.c_int),
         ("sl_node", C.c_void_p), ("sl_gpu", C.c_void_p), ("sl_slice", C.c_void_p), ("sl_prof", C.c_void_p),
         ("sl_busy", C.c_void_p),
@@ -91,6 +91,8 @@ class _Held:
         self.mem = _c(prob.mem_mib, np.uint32)
         self.xfer = _c(prob.xfer_us, np.uint32)
         self.load = _c(prob.load_us, np.uint32)
+        floor = getattr(prob, "max_stage_us", None)  # R38 throughput floor, optional
+        self.floor = None if floor is None else _c(floor, np.uint32)
         sl = prob.slices
         self.sl_node = _c(sl["node"], np.uint16)
         self.sl_gpu = _c(sl["gpu"], np.uint8)
@@ -113,7 +115,7 @@ class _Held:
         self.args = _PlanArgs(
             int(self.gpcs.shape[0]), _p(self.gpcs), _p(self.cap),
             int(self.comp_off.shape[0] - 1), _p(self.comp_off), _p(self.lat), _p(self.mem), _p(self.xfer),
-            _p(self.load), int(prob.n_nodes), int(self.sl_node.shape[0]),
+            _p(self.load), None if self.floor is None else _p(self.floor), int(prob.n_nodes), int(self.sl_node.shape[0]),
             _p(self.sl_node), _p(self.sl_gpu), _p(self.sl_slice), _p(self.sl_prof), _p(self.sl_busy),
             int(R), _p(self.func), _p(self.node), _p(self.slo), int(k_max),
             _p(o["key"]), _p(o["status"]), _p(o["k"]), _p(o["slice"]), _p(o["cut_mask"]), _p(o["e2e_us"]),

@@ -56,6 +56,10 @@ typedef struct {
     /* profile table, one chain per function */
     int F;
     const uint32_t *comp_off, *lat_us /* [C][P] */, *mem_mib, *xfer_us, *load_us;
+    /* throughput floor (R38, NEXT-2): every stage of a plan of f runs in <= max_stage_us[f]
+     * (= 10^6 / lambda_f: an instance sized for the function's load); 0 = none;
+     * nullable */
+    const uint32_t *max_stage_us;
     /* cluster: slices sorted by (node, gpu, slice) */
     int n_nodes, n_slices;
     const uint16_t *sl_node;
@@ -88,6 +92,12 @@ typedef struct {
 
 static uint32_t lat_of(const oracle_plan_args *a, int f, int c, int p) {
     return a->lat_us[(size_t)(a->comp_off[f] + c) * a->P + p];
+}
+
+/* R38: does a stage time t meet function f's throughput floor? */
+static int within_floor(const oracle_plan_args *a, int f, uint64_t t) {
+    if (a->max_stage_us == NULL || a->max_stage_us[f] == 0) return 1;
+    return t <= a->max_stage_us[f];
 }
 
 /* Score every profile sequence for one cut mask (stages = maximal runs of components,
@@ -139,6 +149,8 @@ static void score_mask(req_state *s, uint32_t mask) {
         int feasible = 1;
         for (int i = 0; i < k; i++)
             if (m[i] > a->cap_mib[p[i]]) feasible = 0;
+        for (int i = 0; i < k; i++)
+            if (!within_floor(a, s->f, t[i])) feasible = 0; /* R38 throughput floor */
         for (int q = 0; q < P; q++) {
             uint32_t used = 0;
             for (int i = 0; i < k; i++)
@@ -390,6 +402,7 @@ void oracle_victim(const oracle_plan_args *a, const int32_t *status, int n_inst,
             uint64_t lat = 0;
             for (int c = 0; c < n; c++) lat += lat_of(a, f, c, p);
             if (lat + a->load_us[f] > a->req_slo_us[r]) continue;
+            if (!within_floor(a, f, lat)) continue; /* R38: the monolithic instance meets the floor */
             if (score[i] < best) {
                 best = score[i];
                 victim[r] = i;
@@ -538,7 +551,9 @@ static void ranked_one(const oracle_plan_args *a, int p_ref, int r) {
             prof[s] = -1;
             for (int oi = 0; oi < a->P; oi++) {
                 int p = order[oi];
-                if (left[p] > 0 && m[s] <= a->cap_mib[p]) {
+                uint64_t ts = 0; /* the stage's time on p, for the throughput floor (R38) */
+                for (int c = first[s]; c <= last[s]; c++) ts += lat_of(a, f, c, p);
+                if (left[p] > 0 && m[s] <= a->cap_mib[p] && within_floor(a, f, ts)) {
                     prof[s] = p;
                     left[p]--;
                     break;

@@ -111,6 +111,9 @@ class Problem:
     slo_us: np.ndarray     # uint32 [R] remaining latency budget B_r
     k_max: int = 4
     meta: dict = field(default_factory=dict)
+    # throughput floor per function (R38, NEXT-2): every stage of a plan runs in at most
+    # max_stage_us[f] us (= 10^6 / lambda_f); 0 = none; None = no floors at all
+    max_stage_us: np.ndarray | None = None
 
     @property
     def P(self) -> int:
@@ -474,3 +477,22 @@ def sim_trace(seed: int | None = None, T: int = 4096, n_funcs: int = 200, nodes=
     slo_f = base.meta["slo_f"]
     req_budget = slo_f[req_func].astype(np.uint32)
     return SimTrace(problem=base, req_off=req_off, req_func=req_func, req_budget=req_budget, T=T)
+
+
+def with_throughput_floor(prob: Problem, seed: int = 0x5EEDF100, lo: float = 0.35, hi: float = 1.0,
+                          none_frac: float = 0.25) -> Problem:
+    """A copy of `prob` whose functions carry a throughput floor (R38, NEXT-2): instances
+    sized for the function's load lambda_f ("an instance requiring 4g.40gb"), i.e.
+    max_stage_us[f] = floor(u_f * t_f) with t_f the 1-stage latency on the SLO basis profile
+    and u_f ~ U[lo, hi] -- below 1, only a faster slice or a pipeline (whose bottleneck is a
+    fraction of the chain) serves f.  A fraction `none_frac` of the functions has no floor."""
+    rng = SplitMix64(seed)
+    F = prob.F
+    t_f = np.asarray(prob.meta["t_f"], dtype=np.float64)
+    u = rng.uniform(F, lo, hi)
+    fl = np.floor(u * t_f).astype(np.uint32)
+    fl[rng.sub(1).uniform(F) < none_frac] = 0
+    d = dict(prob.__dict__)
+    d["max_stage_us"] = np.maximum(fl, 0).astype(np.uint32)
+    d["name"] = prob.name + "+floor"
+    return Problem(**d)

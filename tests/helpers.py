@@ -65,6 +65,8 @@ def brute_plan(prob, r, k_max=None):
     xfer = prob.xfer_us[a:b].astype(int).tolist()
     sl = prob.slices
     free = [int(((sl["node"] == v) & (sl["busy"] == 0) & (sl["profile"] == p)).sum()) for p in range(P)]
+    fl = getattr(prob, "max_stage_us", None)
+    floor = 0 if fl is None else int(fl[f])
     best, best_c, idx, nfeas, ksum = KEY_NONE, None, 0, 0, 0
     for k in range(1, min(n, K) + 1):
         masks = sorted(m for m in range(1 << (n - 1)) if bin(m).count("1") == k - 1)
@@ -78,6 +80,7 @@ def brute_plan(prob, r, k_max=None):
                 e2e = sum(t) + sum(xfer[j] for j in cuts)
                 ok = all(mi <= int(prob.cap_mib[p]) for mi, p in zip(m, seq))
                 ok = ok and all(seq.count(p) <= free[p] for p in range(P)) and e2e <= B
+                ok = ok and (floor == 0 or max(t) <= floor)  # R38: throughput floor on the bottleneck
                 if ok:
                     tf = [Fraction(x) for x in t]
                     cv2 = statistics.pvariance(tf) / statistics.mean(tf) ** 2

@@ -28,6 +28,12 @@ def ranked_brute(prob, r, p_ref=None):
     g = [int(x) for x in prob.gpcs]
     sl = prob.slices
     free = [int(((sl["node"] == v) & (sl["busy"] == 0) & (sl["profile"] == p)).sum()) for p in range(P)]
+    fl = getattr(prob, "max_stage_us", None)
+    floor = 0 if fl is None else int(fl[f])  # R38 throughput floor
+
+    def fast_enough(lo, hi, p):
+        return floor == 0 or sum(lat[c][p] for c in range(lo, hi)) <= floor
+
     parts = []
     for mask in range(1 << (n - 1)):
         k = bin(mask).count("1") + 1
@@ -45,7 +51,7 @@ def ranked_brute(prob, r, p_ref=None):
         prof = [None] * k
         for s in sorted(range(k), key=lambda i: (-m[i], i)):
             for p in order:
-                if left[p] > 0 and m[s] <= cap[p]:
+                if left[p] > 0 and m[s] <= cap[p] and fast_enough(bounds[s], bounds[s + 1], p):
                     prof[s] = p
                     left[p] -= 1
                     break
@@ -62,6 +68,23 @@ def ranked_brute(prob, r, p_ref=None):
 @pytest.mark.parametrize("seed", range(1000, 1030))
 def test_ranked_matches_independent_reading(seed):
     prob = random_tiny(seed, n_max=5, K=4)
+    o = oracle.plan_ranked(prob, threads=2)
+    for r in range(prob.R):
+        exp = ranked_brute(prob, r)
+        if exp is None:
+            assert o["status"][r] == oracle.PLAN_INFEASIBLE
+            continue
+        assert o["status"][r] == oracle.PLAN_OK
+        assert o["key"][r] == exp["key"] and o["k"][r] == exp["k"] and o["cut_mask"][r] == exp["mask"]
+        assert list(o["prof"][r, :exp["k"]]) == exp["prof"] and o["e2e_us"][r] == exp["e2e"]
+
+
+@pytest.mark.parametrize("seed", range(3000, 3020))
+def test_ranked_with_floor_matches_independent_reading(seed):
+    prob = random_tiny(seed, n_max=5, K=4)
+    rng = W.SplitMix64(seed ^ 0xF1)
+    fl = rng.integers(0, 160, prob.F).astype(np.uint32)
+    prob = prob.__class__(**{**prob.__dict__, "max_stage_us": fl})
     o = oracle.plan_ranked(prob, threads=2)
     for r in range(prob.R):
         exp = ranked_brute(prob, r)
