@@ -87,6 +87,11 @@ typedef struct {
     const uint32_t *xfer_us;  /* [C] cost of a stage cut after component c (R7); the
                                  last component's entry is ignored                     */
     const uint32_t *load_us;  /* [F] warm -> MIG reload time (victim rule)     */
+    /* [F] throughput floor (NEXT-2, R38), nullable: every stage of a plan of f
+     * -- and the monolithic instance on a time-share victim's slice -- must run in at most
+     * max_stage_us[f] us, i.e. serve >= 10^6 / max_stage_us[f] requests/s (an instance
+     * sized for the function's load); 0 = no floor.  NULL = no floors. */
+    const uint32_t *max_stage_us;
 } ffs_profile_table;
 
 /* One MIG slice of the cluster (12 bytes). */

@@ -249,6 +249,7 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   L.o_pl = take(rows * kRowW, 4);
   L.o_pm = take(rows, 4);
   L.o_xf = take(rows, 4);
+  L.o_thr = take(F, 4);
   L.words = (w + 3) / 4 * 4;
   std::vector<uint32_t> img(L.words, 0);
   for (uint32_t p = 0; p < 8; ++p) {
@@ -275,6 +276,8 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
     img[L.o_fdesc + 4 * f + 1] = n;
     img[L.o_fdesc + 4 * f + 2] = tb->load_us[f];
     img[L.o_fdesc + 4 * f + 3] = (uint32_t)mtot;
+    const uint32_t fl = tb->max_stage_us ? tb->max_stage_us[f] : 0u;
+    img[L.o_thr + f] = fl ? fl : 0xffffffffu;  // R38: 0 = no floor
     for (uint32_t p = 0; p < 8; ++p) img[L.o_pl + row * kRowW + p] = 0;
     img[L.o_pm + row] = 0;
     for (uint32_t i = 0; i < n; ++i) {

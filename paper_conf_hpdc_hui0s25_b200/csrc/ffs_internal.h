@@ -36,7 +36,8 @@ __host__ __device__ constexpr int search_block(int ks) {
   return ks == 3 ? 384 : (ks == 4 && !FFS_KS4_F32) ? FFS_BLOCK4 : kBlock;
 }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
-// bytes of per-thread shared-memory windows of the KS = 4 kernel: 5 profiles x 11 packed pairs
+// bytes of per-thread shared-memory windows of the KS = 4 kernel: 5 profiles x 11 packed
+// pairs of f32 (f32x2 body) or f16 (f16x2 body)
 constexpr size_t kWin4 = FFS_KS4_F32 ? 440 : 220;
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
@@ -53,6 +54,7 @@ struct ImageLayout {
   uint32_t o_pl;      // [rows][8] fp32 bits: PL[row0+i][p] = sum_{c<i} lat[c][p], exact (< 2^24), 16-B aligned
   uint32_t o_pm;      // [rows] u32 PM[row0+i] = sum_{c<i} mem[c]
   uint32_t o_xf;      // [rows] u32 xfer cost of a cut after component i (row0+i)
+  uint32_t o_thr;     // [F] u32 throughput floor: max stage time (R38); 0xffffffff = none
 };
 
 struct SearchArgs {

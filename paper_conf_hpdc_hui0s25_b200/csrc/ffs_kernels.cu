@@ -161,6 +161,8 @@ struct SearchState {
   uint32_t o_pl, o_pm, o_xf, o_cap, o_gpcs;
   // request
   uint32_t row0, n, B;
+  uint32_t thr_u;     // throughput floor: max stage time (R38), 0xffffffff = none
+  float thr;          // the same as an exact fp32 (clamped to 2^24 > every stage time)
   uint64_t freeb;     // 8 x u8 free counts (clamped to 8) of the request's node
   uint32_t free_w;    // 5-bit SWAR lanes 16 + free[p]
   uint64_t idx_base;  // offk[n][KS] + rank * P^KS
@@ -228,6 +230,7 @@ __device__ __forceinline__ void exact_eval(SearchState<KS>& c, int q, int p, boo
     const uint32_t a = (c.row0 + c.bnd[i]) * kRowW, b = (c.row0 + c.bnd[i + 1]) * kRowW;
     const uint32_t t = pl_diff(c.sm, c.o_pl + b + pr, c.o_pl + a + pr);
     ok &= c.memst[i] <= c.sm[c.o_cap + pr];
+    ok &= t <= c.thr_u;  // R38 throughput floor
     St += t;
     Sq += (uint64_t)t * t;
     used += 1u << (4 * pr);
@@ -318,7 +321,7 @@ __device__ __forceinline__ void outer_level(SearchState<KS>& c, float S, float Q
     for (int p = 0; p < kP; ++p) {
       const uint32_t t = pl_diff(c.sm, b + p, a + p);
       const uint32_t cw2 = cw - (1u << (5 * p));
-      const bool ok = (c.memst[L] <= c.sm[c.o_cap + p]) && ((cw2 >> (5 * p + 4)) & 1u);
+      const bool ok = (c.memst[L] <= c.sm[c.o_cap + p]) && t <= c.thr_u && ((cw2 >> (5 * p + 4)) & 1u);
       const float tf = ok ? __uint2float_rn(t) : INF;
       c.pd[L] = p;
       outer_level<L + 1, KS, VERIFY>(c, S + tf, fmaf(tf, tf, Q), cw2, misses);
@@ -337,7 +340,7 @@ __device__ __forceinline__ void load_stage(const SearchState<KS>& c, int s, floa
 #pragma unroll
   for (int p = 0; p < kP; ++p) {
     const float f = t[p];
-    tf[p] = (c.memst[s] <= c.sm[c.o_cap + p]) ? f : INF;
+    tf[p] = (c.memst[s] <= c.sm[c.o_cap + p] && f <= c.thr) ? f : INF;
     sq[p] = f * f;
   }
 }
@@ -385,7 +388,7 @@ __device__ __forceinline__ void build_tables(const SearchState<KS>& c, Tables<KS
     stage_lat(c, s, f);
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
-      const bool mem_ok = c.memst[s] <= c.sm[c.o_cap + x];
+      const bool mem_ok = c.memst[s] <= c.sm[c.o_cap + x] && f[x] <= c.thr;
       const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
 #pragma unroll
       for (int m = 0; m <= s; ++m) T.vf[s][m][x] = (mem_ok && fr > (uint32_t)m) ? f[x] : INF;
@@ -547,7 +550,8 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
 #pragma unroll
         for (int s = 0; s < 3; ++s)
 #pragma unroll
-          for (int m = 0; m <= s; ++m) v[h][s][m] = (G[h].memst[s] <= cap && fr > (uint32_t)m) ? f[h][s][x] : INF;
+          for (int m = 0; m <= s; ++m)
+            v[h][s][m] = (G[h].memst[s] <= cap && f[h][s][x] <= c.thr && fr > (uint32_t)m) ? f[h][s][x] : INF;
       v0[x] = f2pack(v[0][0][0], v[1][0][0]);
       v1[0][x] = f2pack(v[0][1][0], v[1][1][0]);
       v1[1][x] = f2pack(v[0][1][1], v[1][1][1]);
@@ -625,7 +629,7 @@ __device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint
       for (int h = 0; h < 2; ++h)
 #pragma unroll
         for (int s = 0; s < 4; ++s) {
-          const float vm = (G[h].memst[s] <= cap) ? f[h][s][x] : INF;
+          const float vm = (G[h].memst[s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] : INF;
           const float base = (s == 3) ? G[h].blim - vm : vm;
           const float none = (s == 3) ? -INF : INF;
 #pragma unroll
@@ -730,6 +734,11 @@ __device__ __forceinline__ h2 h2add(h2 a, h2 b) {
   asm("add.rn.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
   return d;
 }
+__device__ __forceinline__ h2 h2mul(h2 a, h2 b) {
+  h2 d;
+  asm("mul.rn.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
 __device__ __forceinline__ h2 h2sub(h2 a, h2 b) {
   h2 d;
   asm("sub.rn.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
@@ -766,7 +775,9 @@ struct WinH {
 };
 
 // rows: per thread and profile x, 11 packed f16 pairs in [x][k][thread] order (4-byte,
-// conflict-free); window e (e = 1 when x is the stage-0 profile) is read at offset e.
+// conflict-free, immediate offsets); window e (e = 1 when x is the stage-0 profile: every
+// multiplicity shifted by one) is read at offset e.  (An 8-byte layout with both windows
+// stored -- half the LDS -- measured 2.6 % slower: more registers and smem.)
 template <bool VERIFY>
 __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
                                            unsigned long long* misses, uint32_t zero) {
@@ -799,26 +810,29 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     slack[h] = bl >= 0.f ? M * sig[h] * (1.f + 1.f / 128.f) : -INF;
   }
   constexpr h2 kInf2 = 0x7c007c00u, kGuard = 0x80008000u;
+  const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
   h2 a1[kP], a2[kP], t2[kP], cc[kP];
 #pragma unroll
   for (int x = 0; x < kP; ++x) {
     const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
     const uint32_t cap = c.sm[c.o_cap + x];
-    float fs[2][4], vm[2][4];
+    float vm[2][4];
 #pragma unroll
     for (int h = 0; h < 2; ++h)
 #pragma unroll
-      for (int s = 0; s < 4; ++s) {
-        fs[h][s] = f[h][s][x] * sig[h];
-        vm[h][s] = (G[h].memst[s] <= cap) ? fs[h][s] : INF;  // memory folded per half
-      }
-    // the free-slice gates depend only on the node: applied to the packed pair
+      for (int s = 0; s < 4; ++s)  // memory and the throughput floor (R38) folded
+        vm[h][s] = (G[h].memst[s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * sig[h] : INF;
+    // the stage tables in packed f16 (the squares and alpha products too: two more f16
+    // roundings per entry, inside the margin of DESIGN.md §4.3); a memory-infeasible
+    // stage is INF everywhere, which only an SLO-rejected candidate can see
     const h2 p0 = h2pack(vm[0][0], vm[1][0]), p1 = h2pack(vm[0][1], vm[1][1]), p2 = h2pack(vm[0][2], vm[1][2]);
-    const h2 p3 = h2guard(h2pack(slack[0] - vm[0][3], slack[1] - vm[1][3]));
-    a1[x] = h2pack(al * (fs[0][1] * fs[0][1]), al * (fs[1][1] * fs[1][1]));
-    a2[x] = h2pack(al * (fs[0][2] * fs[0][2]), al * (fs[1][2] * fs[1][2]));
-    t2[x] = h2pack(fs[0][3] + fs[0][3], fs[1][3] + fs[1][3]);
-    cc[x] = h2pack(one_m_a * (fs[0][3] * fs[0][3]), one_m_a * (fs[1][3] * fs[1][3]));
+    const h2 p3 = h2pack(vm[0][3], vm[1][3]);
+    const h2 w3 = h2guard(h2pack(slack[0] - vm[0][3], slack[1] - vm[1][3]));
+    a1[x] = h2mul(h2mul(p1, p1), al2);
+    a2[x] = h2mul(h2mul(p2, p2), al2);
+    t2[x] = h2add(p3, p3);
+    cc[x] = h2mul(h2mul(p3, p3), oma2);
+    const h2 na0 = h2mul(h2mul(p0, p0), nal2);
     //   [v1[0], v1[1], v2[0], v2[1], v2[2], guarded slack-v3[0..3], v0[0], -alpha t0^2]
     h2* r = rows + (x * 11) * nb + tid;
     r[0 * nb] = fr > 0 ? p1 : kInf2;
@@ -826,12 +840,12 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     r[2 * nb] = fr > 0 ? p2 : kInf2;
     r[3 * nb] = fr > 1 ? p2 : kInf2;
     r[4 * nb] = fr > 2 ? p2 : kInf2;
-    r[5 * nb] = fr > 0 ? p3 : kGuard;
-    r[6 * nb] = fr > 1 ? p3 : kGuard;
-    r[7 * nb] = fr > 2 ? p3 : kGuard;
-    r[8 * nb] = fr > 3 ? p3 : kGuard;
+    r[5 * nb] = fr > 0 ? w3 : kGuard;
+    r[6 * nb] = fr > 1 ? w3 : kGuard;
+    r[7 * nb] = fr > 2 ? w3 : kGuard;
+    r[8 * nb] = fr > 3 ? w3 : kGuard;
     r[9 * nb] = fr > 0 ? p0 : kInf2;
-    r[10 * nb] = h2pack(-al * (fs[0][0] * fs[0][0]), -al * (fs[1][0] * fs[1][0]));
+    r[10 * nb] = na0;
   }
   uint32_t pendA = 0, pendB = 0;
 #if FFS_UNROLL_D0
@@ -1053,6 +1067,8 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     c.n = fd[1];
     c.B = A.slo[r];
     c.freeb = A.node_free[q.node];
+    c.thr_u = tbl[A.lay.o_thr + q.func];
+    c.thr = (float)min(c.thr_u, 1u << 24);
     uint32_t w = 0;
 #pragma unroll
     for (int p = 0; p < kP; ++p) w |= (16u + (uint32_t)((c.freeb >> (8 * p)) & 255u)) << (5 * p);
@@ -1225,7 +1241,8 @@ __device__ __forceinline__ bool victim_ok(const uint32_t* img, const ImageLayout
   if (fd[3] > img[L.o_cap + p]) return false;  // time-sharing instances are non-pipeline
   const uint32_t row0 = fd[0], n = fd[1];
   const uint64_t lat = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
-  return lat + fd[2] <= B;  // execution + reload within the budget
+  // execution + reload within the budget; the instance meets the floor (R38)
+  return lat + fd[2] <= B && lat <= img[L.o_thr + f];
 }
 
 __device__ __forceinline__ void plan_init(ffs_plan& pl) {
@@ -1542,7 +1559,7 @@ __device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const I
 #pragma unroll
   for (int p = 0; p < kP; ++p) {
     const uint64_t lat = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
-    if (fd[3] <= img[L.o_cap + p] && lat + fd[2] <= B) ok |= 1u << p;
+    if (fd[3] <= img[L.o_cap + p] && lat + fd[2] <= B && lat <= img[L.o_thr + f]) ok |= 1u << p;
   }
   return ok;
 }
@@ -1661,7 +1678,7 @@ struct RankedEval {
 };
 
 __device__ __forceinline__ bool ranked_eval(const RankedArgs& A, uint32_t row0, uint32_t n, uint32_t mask,
-                                            uint64_t freeb, uint32_t B, RankedEval& out) {
+                                            uint64_t freeb, uint32_t B, uint32_t thr, RankedEval& out) {
   const uint32_t* img = A.image;
   const ImageLayout& L = A.lay;
   const uint32_t k = __popc(mask) + 1;
@@ -1677,7 +1694,8 @@ __device__ __forceinline__ bool ranked_eval(const RankedArgs& A, uint32_t row0, 
   bnd[k] = n;
   for (uint32_t i = 0; i < k; ++i) mem[i] = img[L.o_pm + row0 + bnd[i + 1]] - img[L.o_pm + row0 + bnd[i]];
   // min-resource greedy: stages by descending memory (ties: lower stage), each takes the
-  // first profile in (capacity, gpcs, id) order with a free slice left that holds it
+  // first profile in (capacity, gpcs, id) order with a free slice left that holds it and
+  // runs it within the throughput floor (R38)
   uint32_t left[kP];
 #pragma unroll
   for (int p = 0; p < kP; ++p) left[p] = (uint32_t)(freeb >> (8 * p)) & 255u;
@@ -1695,7 +1713,8 @@ __device__ __forceinline__ bool ranked_eval(const RankedArgs& A, uint32_t row0, 
 #pragma unroll
       for (int q = 0; q < kP; ++q)
         if (q == p) ok = left[q] > 0;
-      if (got < 0 && ok && mem[s] <= img[L.o_cap + p]) {
+      if (got < 0 && ok && mem[s] <= img[L.o_cap + p] &&
+          pl_diff(img, L.o_pl + (row0 + bnd[s + 1]) * kRowW + p, L.o_pl + (row0 + bnd[s]) * kRowW + p) <= thr) {
         got = p;
 #pragma unroll
         for (int q = 0; q < kP; ++q)
@@ -1755,7 +1774,7 @@ __global__ void __launch_bounds__(kRkT) k_plan_ranked(const __grid_constant__ Ra
       bool ok = false;
       if (j < cnt) {
         mask = A.rank_mask[off + j];
-        ok = ranked_eval(A, row0, n, mask, freeb, B, ev);
+        ok = ranked_eval(A, row0, n, mask, freeb, B, img[L.o_thr + q.func], ev);
       }
       const uint32_t bal = __ballot_sync(0xffffffffu, ok);
       if (bal) {

@@ -36,7 +36,7 @@ class _Profiles(C.Structure):
 
 class _Table(C.Structure):
     _fields_ = [("n_funcs", C.c_uint32), ("comp_off", C.c_void_p), ("lat_us", C.c_void_p), ("mem_mib", C.c_void_p),
-                ("xfer_us", C.c_void_p), ("load_us", C.c_void_p)]
+                ("xfer_us", C.c_void_p), ("load_us", C.c_void_p), ("max_stage_us", C.c_void_p)]
 
 
 class _Cluster(C.Structure):
@@ -143,7 +143,12 @@ class Planner:
         keep = [np.ascontiguousarray(prob.comp_off, np.uint32), np.ascontiguousarray(prob.lat_us, np.uint32),
                 np.ascontiguousarray(prob.mem_mib, np.uint32), np.ascontiguousarray(prob.xfer_us, np.uint32),
                 np.ascontiguousarray(prob.load_us, np.uint32)]
+        floor = getattr(prob, "max_stage_us", None)  # R38 throughput floor (optional)
+        if floor is not None:
+            keep.append(np.ascontiguousarray(floor, np.uint32))
         tb = _Table(int(keep[0].shape[0] - 1), *[_host(a) for a in keep])
+        if floor is None:
+            tb.max_stage_us = None
         sl = np.ascontiguousarray(prob.slices, dtype=W.SLICE_DTYPE)
         cl = _Cluster(int(prob.n_nodes), int(sl.shape[0]), _host(sl) if sl.shape[0] else None)
         self._check(_lib.ffs_stage_tables(self._h, C.byref(pr), C.byref(tb), C.byref(cl)))

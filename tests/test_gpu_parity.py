@@ -601,3 +601,58 @@ def test_f16_prefilter_stress(F, planner, seed):
     assert planner.filter_misses() == 0
     p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
     np.testing.assert_array_equal(keys2, o["key"])
+
+
+# ---- NEXT-2 throughput floor (R38) ------------------------------------------
+def _floored(prob, seed=0xF1):
+    rng = W.SplitMix64(seed)
+    fl = rng.integers(0, 160, prob.F).astype(np.uint32)
+    fl[rng.sub(1).uniform(prob.F) < 0.3] = 0
+    return prob.__class__(**{**prob.__dict__, "max_stage_us": fl})
+
+
+@pytest.mark.parametrize("seed", range(2000, 2012))
+def test_floor_tiny_random(F, planner, seed):
+    prob = _floored(random_tiny(seed, n_max=6, K=5), seed)
+    p, keys, ch = run_gpu(F, planner, prob)
+    o = oracle.plan(prob)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    assert planner.filter_misses() == 0
+
+
+@pytest.mark.parametrize("K", [2, 3, 4, 6])
+def test_floor_configs(F, planner, K):
+    # every search template (KS 1..K) with floors that bind on a C2-shaped mix
+    prob = W.with_throughput_floor(W.config2(R=1024 if K <= 4 else 256))
+    p, keys, ch = run_gpu(F, planner, prob, k_max=K)
+    o = oracle.plan(prob, k_max=K)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(ch, o["checks"])
+    assert planner.filter_misses() == 0
+    p2, keys2, _ = run_gpu(F, planner, prob, k_max=K, verify=False)
+    np.testing.assert_array_equal(keys2, o["key"])
+
+
+def test_floor_next_paths(F, planner):
+    """ranked first-fit, joint commit, frontier and victims honour the floor like the oracle."""
+    prob = W.with_throughput_floor(W.config2(R=512))
+    assert_plans_equal(run_ranked(F, planner, prob), oracle.plan_ranked(prob, p_ref=4))
+    pj, _ = run_joint(F, planner, prob)
+    assert_plans_equal(pj, oracle.plan_joint(prob))
+    p_arg, keys, _ = run_gpu(F, planner, prob, verify=False)
+    planner.frontier_build(prob.k_max)
+    req, slo = F.to_device(prob)
+    p_fr = F.plans_to_numpy(planner.plan_frontier(req, slo))
+    np.testing.assert_array_equal(p_fr.view(np.uint8), p_arg.view(np.uint8))
+    # victims of the infeasible requests (single snapshot, decode path)
+    wl = W.config4(T=1)
+    fprob = W.with_throughput_floor(wl.problem)
+    p, keys, _ = run_gpu(F, planner, fprob, verify=False)
+    inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
+    score, _ = planner.evict_scores(inst, int(wl.now_us[0]), window_us=wl.window_us)
+    req, slo = F.to_device(fprob)
+    plans = F.plans_to_numpy(planner.plan_decode(req, slo, torch.from_numpy(keys).cuda(), fprob.k_max, inst, score))
+    o = oracle.plan(fprob, checks=False)
+    s_o, _ = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
+    np.testing.assert_array_equal(plans["victim"], oracle.victim(fprob, o["status"], wl.inst, s_o))
