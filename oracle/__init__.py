@@ -139,6 +139,42 @@ def plan(prob, k_max: int | None = None, threads: int | None = None, checks: boo
     return h.out
 
 
+def plan_any(prob, k_max: int | None = None, threads: int | None = None) -> tuple[dict, np.ndarray]:
+    """NEXT-2 any-invoker (cross-node) planning, R39: a request may be served by
+    any invoker's node (the controller's load balancer sees every invoker); its
+    plan is the argmin over nodes v of the plan against v's free slices (R10 still holds: a
+    pipeline never spans nodes); ties in the key prefer the home node, then the lowest node
+    id.  Plainly: one full oracle.plan per node with every request moved there, then a
+    per-request minimum.  Returns (plans as plan(), node[R]: the serving node or -1)."""
+    R = prob.R
+    best = None
+    node = np.full(R, -1, np.int64)
+    home = np.asarray(prob.req["node"], np.int64)
+    for v in range(int(prob.n_nodes)):
+        req = prob.req.copy()
+        req["node"] = v
+        o = plan(prob.with_requests(req, prob.slo_us), k_max=k_max, threads=threads, checks=False)
+        if best is None:
+            best = {k: a.copy() for k, a in o.items()}
+            node[:] = v
+            continue
+        # (key, not home, node id) lexicographic: v > every earlier node id
+        cur_home = node == home
+        take = (o["key"] < best["key"]) | ((o["key"] == best["key"]) & (home == v) & ~cur_home)
+        for k in best:
+            best[k][take] = o[k][take]
+        node[take] = v
+    node[best["status"] != PLAN_OK] = -1
+    # an out-of-range function or home node stays a bad request (as in plan())
+    bad = np.nonzero((np.asarray(prob.req["func"], np.int64) >= prob.F) | (home >= int(prob.n_nodes)))[0]
+    if len(bad):
+        o = plan(prob.subset(bad), k_max=k_max, threads=threads, checks=False)
+        for k in best:
+            best[k][bad] = o[k]
+        node[bad] = -1
+    return best, node
+
+
 def plan_ranked(prob, p_ref: int | None = None, k_max: int | None = None, threads: int | None = None) -> dict:
     """NEXT-1: the paper's offline CV ranking + first-fit walk (ffs_oracle.c:
     oracle_plan_ranked).  p_ref = reference profile of the offline CV (default: the
