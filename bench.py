@@ -294,10 +294,30 @@ def run_frontier(pl, prob, req, slo, steps: int, warmup: int, flush):
         b.record(stream)
         torch.cuda.synchronize()
         ms += a.elapsed_time(b)
+    # NEXT-2 any-invoker planning (R39) from the same frontiers: every request considers
+    # every node of the cluster (one warp per request over the free-vector classes)
+    node = torch.empty(prob.R, dtype=torch.int32, device="cuda")
+    for _ in range(warmup):
+        pl.plan_frontier_any(req, slo, out=out, node=node)
+    ms_any = 0.0
+    for i in range(steps):
+        flush.fill_(i & 0xFF)
+        a.record(stream)
+        pl.plan_frontier_any(req, slo, out=out, node=node)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ms_any += a.elapsed_time(b)
+    st = out.view(-1, 80)[:, 8:12].contiguous().view(torch.int32)
+    ok_any = int(torch.count_nonzero(st == 0))
+    home = req.view(-1, 8)[:, 4:8].contiguous().view(torch.int32).view(-1)
+    away = int(torch.count_nonzero((node >= 0) & (node != home)))
     return {"metric": "frontier_plans_per_s", "value": prob.R * steps / (ms * 1e-3), "unit": "plans/s",
             "query_ms_per_step": ms / steps, "build_s": build_s, "groups": groups, "rounds": rounds,
             "note": "plans identical to the argmin path; candidates are scored once per frontier point and group, "
-                    "not per request (not comparable to candidates/s)"}
+                    "not per request (not comparable to candidates/s)",
+            "any_invoker": {"metric": "any_invoker_plans_per_s", "value": prob.R * steps / (ms_any * 1e-3),
+                            "unit": "plans/s", "query_ms_per_step": ms_any / steps, "ok": ok_any,
+                            "served_away_from_home": away}}
 
 
 def run_sim(pl):

@@ -330,6 +330,16 @@ ffs_status ffs_simulate(ffs_ctx *ctx, const uint32_t *d_req_off, const uint32_t 
 ffs_status ffs_frontier_build(ffs_ctx *ctx, uint32_t k_max, uint32_t *n_groups, uint32_t *rounds, void *stream);
 ffs_status ffs_plan_frontier(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
                              ffs_plan *d_out, void *stream);
+/* NEXT-2 any-invoker (cross-node) planning from the same frontiers (R39): a
+ * request may be served by any invoker's node -- the controller's load balancer sees every
+ * invoker -- so its plan is the argmin over nodes of the per-node argmin (a
+ * pipeline still never spans nodes, R10); key ties prefer the home node (req.node), then
+ * the lowest node id.  One warp per request scans the function's frontier groups (one per
+ * distinct node free-vector).  d_out: plans bound to the chosen node's slices; d_node
+ * (nullable): int32 serving node per request, -1 when not OK.  An out-of-range func or home
+ * node is FFS_PLAN_BAD_REQ.  Asynchronous.  FFS_ERR_STATE: frontiers not built. */
+ffs_status ffs_plan_frontier_any(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                                 ffs_plan *d_out, int32_t *d_node, void *stream);
 
 /* ---- measurement / debug helpers ------------------------------------------------------
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of

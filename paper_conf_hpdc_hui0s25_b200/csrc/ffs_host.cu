@@ -995,6 +995,36 @@ ffs_status ffs_plan_frontier(ffs_ctx* c, const ffs_request* d_req, const uint32_
   return FFS_OK;
 }
 
+ffs_status ffs_plan_frontier_any(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                                 ffs_plan* d_out, int32_t* d_node, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged || !c->front_built) return fail(c, FFS_ERR_STATE, "call ffs_frontier_build after staging");
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  FrontierArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.k_max = c->front_kmax;
+  a.n_groups = c->front_groups;
+  a.n_fv = c->front_nfv;
+  a.n_nodes = c->n_nodes;
+  a.cap = c->front_cap;
+  a.node_fv = c->f_nodefv.as<uint32_t>();
+  a.fv_node = c->f_fvnode.as<uint32_t>();
+  a.fr_key = c->f_key.as<int64_t>();
+  a.fr_e2e = c->f_e2e.as<uint32_t>();
+  a.fr_cnt = c->f_cnt.as<uint32_t>();
+  a.req = d_req;
+  a.slo = d_slo;
+  a.n_req = n_req;
+  a.free_list = c->free_list.as<int32_t>();
+  a.out = d_out;
+  a.node_out = d_node;
+  CK(launch_frontier(3, a, 0, (cudaStream_t)stream), "frontier any-invoker query");
+  return FFS_OK;
+}
+
 ffs_status ffs_bench_int_peak(ffs_ctx* c, double* ops, double* seconds) {
   if (!c || !ops || !seconds) return FFS_ERR_ARG;
   DeviceGuard g(c->device);

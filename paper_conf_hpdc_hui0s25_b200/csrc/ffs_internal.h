@@ -174,6 +174,8 @@ struct FrontierArgs {
   uint32_t n_req;
   const int32_t* free_list;
   ffs_plan* out;
+  const uint32_t* fv_node;      // [n_fv] lowest node id of each free-vector class (any-invoker)
+  int32_t* node_out;            // [n_req] serving node (any-invoker), nullable
 };
 cudaError_t launch_frontier(int phase, const FrontierArgs& a, uint32_t n, cudaStream_t st);
 

@@ -1884,10 +1884,75 @@ __global__ void k_front_query(const __grid_constant__ FrontierArgs A) {
   A.out[r] = pl;
 }
 
+// first frontier point of group g with e2e <= B (the argmin for budget B), or KEY_NONE
+__device__ __forceinline__ int64_t front_lookup(const FrontierArgs& A, uint32_t g, uint32_t B) {
+  uint32_t lo = 0, hi = A.fr_cnt[g];
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (A.fr_e2e[(uint64_t)mid * A.n_groups + g] <= B) hi = mid; else lo = mid + 1;
+  }
+  return lo == A.fr_cnt[g] ? (int64_t)kKeyNone : A.fr_key[(uint64_t)lo * A.n_groups + g];
+}
+
+// NEXT-2 any-invoker query (R39): one warp per request, lanes over the function's
+// free-vector classes; min of (key, class != home class, lowest node of the class)
+__global__ void __launch_bounds__(256) k_front_query_any(const __grid_constant__ FrontierArgs A) {
+  const uint32_t r = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (r >= A.n_req) return;
+  const ffs_request q = A.req[r];
+  const bool valid = q.func < A.lay.F && q.node < A.n_nodes;
+  int64_t bk = (int64_t)kKeyNone;
+  uint32_t bt = 0xffffffffu;  // tiebreak: (class != home class) << 31 | node
+  if (valid) {
+    const uint32_t home = A.node_fv[q.node], B = A.slo[r];
+    for (uint32_t c = lane; c < A.n_fv; c += 32) {
+      const int64_t k = front_lookup(A, q.func * A.n_fv + c, B);
+      const uint32_t t = (c == home) ? q.node : (0x80000000u | A.fv_node[c]);
+      if (k < bk || (k == bk && t < bt)) {
+        bk = k;
+        bt = t;
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const int64_t k2 = __shfl_xor_sync(0xffffffffu, bk, o);
+    const uint32_t t2 = __shfl_xor_sync(0xffffffffu, bt, o);
+    if (k2 < bk || (k2 == bk && t2 < bt)) {
+      bk = k2;
+      bt = t2;
+    }
+  }
+  if (lane) return;
+  ffs_plan pl;
+  plan_init(pl);
+  int32_t node = -1;
+  if (valid) {
+    if ((uint64_t)bk == kKeyNone) {
+      pl.status = FFS_PLAN_INFEASIBLE;
+    } else {
+      node = (int32_t)(bt & 0x7fffffffu);
+      plan_from_key(A.image, A.lay, q.func, A.k_max, bk, pl);
+      uint32_t used[kP] = {0, 0, 0, 0, 0};
+      for (uint32_t i = 0; i < pl.k; ++i) {
+        const int p = pl.prof[i];
+        uint32_t u = 0;
+#pragma unroll
+        for (int x = 0; x < kP; ++x)
+          if (x == p) u = used[x]++;
+        pl.slice[i] = A.free_list[((uint64_t)node * 8 + p) * 8 + u];
+      }
+    }
+  }
+  A.out[r] = pl;
+  if (A.node_out) A.node_out[r] = node;
+}
+
 cudaError_t launch_frontier(int phase, const FrontierArgs& a, uint32_t n, cudaStream_t st) {
   const uint32_t T = 256;
   if (phase == 1 && n) k_front_record<<<(n + T - 1) / T, T, 0, st>>>(a, n);
   if (phase == 2 && a.n_req) k_front_query<<<(a.n_req + T - 1) / T, T, 0, st>>>(a);
+  if (phase == 3 && a.n_req) k_front_query_any<<<(uint32_t)(((uint64_t)a.n_req * 32 + T - 1) / T), T, 0, st>>>(a);
   return cudaGetLastError();
 }
 cudaError_t launch_front_gather(const FrontierArgs& a, uint32_t n, const uint32_t* fv_node, uint32_t* gslo,

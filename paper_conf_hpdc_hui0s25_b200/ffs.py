@@ -66,6 +66,7 @@ _sig = {
     "ffs_route": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_frontier_build": ([_vp, _u32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32), _vp], _i32),
     "ffs_plan_frontier": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
+    "ffs_plan_frontier_any": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp], _i32),
     "ffs_rank_partitions": ([_vp, _u32, _u32], _i32),
     "ffs_plan_ranked": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
@@ -295,6 +296,18 @@ class Planner:
             out = torch.empty((n, PLAN_DTYPE.itemsize), dtype=torch.uint8, device=slo.device)
         self._check(_lib.ffs_plan_frontier(self._h, _ptr(req), _ptr(slo), n, _ptr(out), _stream(stream)))
         return out
+
+    def plan_frontier_any(self, req, slo, out=None, node=None, stream=None):
+        """NEXT-2 any-invoker planning (R39): (plans, serving node int32 or -1)."""
+        import torch
+        n = int(slo.numel())
+        if out is None:
+            out = torch.empty((n, PLAN_DTYPE.itemsize), dtype=torch.uint8, device=slo.device)
+        if node is None:
+            node = torch.empty(n, dtype=torch.int32, device=slo.device)
+        self._check(_lib.ffs_plan_frontier_any(self._h, _ptr(req), _ptr(slo), n, _ptr(out), _ptr(node),
+                                               _stream(stream)))
+        return out, node
 
     # ---- NEXT-1: ranked first-fit (P:339-343) -----------------------------------------------
     def rank_partitions(self, k_max: int, p_ref: int) -> None:

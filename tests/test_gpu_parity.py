@@ -656,3 +656,49 @@ def test_floor_next_paths(F, planner):
     o = oracle.plan(fprob, checks=False)
     s_o, _ = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
     np.testing.assert_array_equal(plans["victim"], oracle.victim(fprob, o["status"], wl.inst, s_o))
+
+
+# ---- NEXT-2 any-invoker (cross-node) planning (R39) --------------------------
+def _run_any(F, planner, prob):
+    planner.stage(prob)
+    planner.frontier_build(prob.k_max)
+    req, slo = F.to_device(prob)
+    out, node = planner.plan_frontier_any(req, slo)
+    torch.cuda.synchronize()
+    return F.plans_to_numpy(out), node.cpu().numpy()
+
+
+@pytest.mark.parametrize("seed", range(1000, 1008))
+def test_any_invoker_tiny(F, planner, seed):
+    prob = random_tiny(seed)
+    p, node = _run_any(F, planner, prob)
+    o, n_o = oracle.plan_any(prob)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(node, n_o)
+
+
+@pytest.mark.parametrize("floor", [False, True])
+def test_any_invoker_c3_sample(F, planner, floor):
+    prob = W.config3()
+    prob = W.with_throughput_floor(prob) if floor else prob
+    idx = np.arange(0, prob.R, 97)
+    sub = prob.subset(idx)
+    p, node = _run_any(F, planner, sub)
+    o, n_o = oracle.plan_any(sub)
+    assert_plans_equal(p, o)
+    np.testing.assert_array_equal(node, n_o)
+    home = oracle.plan(sub, checks=False)
+    assert (o["key"] <= home["key"]).all() and (o["key"] < home["key"]).any()
+
+
+def test_any_invoker_bad_requests(F, planner):
+    prob = random_tiny(1001)
+    req = prob.req.copy()
+    req["node"][0] = 99
+    req["func"][1] = 77
+    bad = prob.with_requests(req, prob.slo_us)
+    p, node = _run_any(F, planner, bad)
+    assert p["status"][0] == oracle.PLAN_BAD_REQ and p["status"][1] == oracle.PLAN_BAD_REQ
+    assert node[0] == -1 and node[1] == -1
+    o, n_o = oracle.plan_any(bad)
+    assert_plans_equal(p, o)
