@@ -26,11 +26,10 @@ constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #endif
 constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 // KS = 3 keeps every table in registers; capped at 168 registers it runs 12 warps per SM
-// and is faster (C5: 4.3 -> 3.9 ms).  The f16x2 KS = 4 kernel needs ~150 registers and
-// also runs 12 warps per SM (C5: 74.2 ms at 8 warps -> 72.0 ms).  The
-// KS = 4 CTA may shrink to fit its shared-memory windows.
+// and is faster (C5: 4.3 -> 3.9 ms).  The f16x2 KS = 4 kernel fits in 113 registers at
+// 16 warps per SM (C5: 66.3 ms at 8 warps, 61.0 at 12, 60.1 at 16).
 #ifndef FFS_BLOCK4
-#define FFS_BLOCK4 384
+#define FFS_BLOCK4 512
 #endif
 __host__ __device__ constexpr int search_block(int ks) {
   return ks == 3 ? 384 : (ks == 4 && !FFS_KS4_F32) ? FFS_BLOCK4 : kBlock;
