@@ -749,6 +749,12 @@ __device__ __forceinline__ h2 h2fma(h2 a, h2 b, h2 c) {
   asm("fma.rn.f16x2 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c));
   return d;
 }
+// IEEE maxNum per half (a NaN operand loses); ptxas fuses pairs into 3-input VHMNMX
+__device__ __forceinline__ h2 h2max(h2 a, h2 b) {
+  h2 d;
+  asm("max.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
 
 // SLO slack in "guarded" form for the integer SWAR test of the inner loop: per f16 half,
 // bit 15 (guard) | the magnitude bits of slack - v3 when it is >= 0, else the guard alone
@@ -771,7 +777,7 @@ __device__ __forceinline__ uint32_t isub(uint32_t a, uint32_t b, uint32_t zero) 
 }
 
 struct WinH {
-  h2 s1, s2[2], s3[3];
+  h2 s1, s2[2], c3[3];
 };
 
 // rows: per thread and profile x, 11 packed f16 pairs in [x][k][thread] order (4-byte,
@@ -809,9 +815,11 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     wide[h] = bl >= 0.f && c.tmin * sig[h] < 0.125f;  // f16 underflow could matter: exact path
     slack[h] = bl >= 0.f ? M * sig[h] * (1.f + 1.f / 128.f) : -INF;
   }
-  constexpr h2 kInf2 = 0x7c007c00u, kGuard = 0x80008000u;
+  constexpr h2 kInf2 = 0x7c007c00u, kNegInf2 = 0xfc00fc00u, kGuard = 0x80008000u;
   const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
-  h2 a1[kP], a2[kP], t2[kP], cc[kP];
+  h2 a1[kP], a2[kP], t2[kP];
+  // fastest admissible last stage per half (memory, floor, >= 1 free slice of the profile)
+  float v3min[2] = {INF, INF};
 #pragma unroll
   for (int x = 0; x < kP; ++x) {
     const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
@@ -826,27 +834,39 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     // roundings per entry, inside the margin of DESIGN.md §4.3); a memory-infeasible
     // stage is INF everywhere, which only an SLO-rejected candidate can see
     const h2 p0 = h2pack(vm[0][0], vm[1][0]), p1 = h2pack(vm[0][1], vm[1][1]), p2 = h2pack(vm[0][2], vm[1][2]);
-    const h2 p3 = h2pack(vm[0][3], vm[1][3]);
-    const h2 w3 = h2guard(h2pack(slack[0] - vm[0][3], slack[1] - vm[1][3]));
+    // a last stage longer than the (widened) SLO slack on its own is inadmissible too: no
+    // candidate holding it is feasible, and the bound keeps t3 and t3^2 far from overflow
+    const float u0 = vm[0][3] <= slack[0] ? vm[0][3] : INF, u1 = vm[1][3] <= slack[1] ? vm[1][3] : INF;
+    const h2 p3 = h2pack(u0, u1);
+    if (fr > 0) {
+      v3min[0] = fminf(v3min[0], u0);
+      v3min[1] = fminf(v3min[1], u1);
+    }
     a1[x] = h2mul(h2mul(p1, p1), al2);
     a2[x] = h2mul(h2mul(p2, p2), al2);
-    t2[x] = h2add(p3, p3);
-    cc[x] = h2mul(h2mul(p3, p3), oma2);
+    // last stage as (2 t3, (1 - alpha_h) t3^2); an inadmissible one (INF) as (0, -INF), so
+    // its score y = S3 * 2t3 + cc is -INF for every finite S3 (no INF * 0, no INF - INF)
+    const uint32_t inf3 = (u0 == INF ? 0x0000ffffu : 0u) | (u1 == INF ? 0xffff0000u : 0u);
+    t2[x] = h2add(p3, p3) & ~inf3;
+    const h2 cc = (h2mul(h2mul(p3, p3), oma2) & ~inf3) | (kNegInf2 & inf3);
     const h2 na0 = h2mul(h2mul(p0, p0), nal2);
-    //   [v1[0], v1[1], v2[0], v2[1], v2[2], guarded slack-v3[0..3], v0[0], -alpha t0^2]
+    //   [v1[0], v1[1], v2[0], v2[1], v2[2], cc3[0..3], v0[0], -alpha t0^2]
+    // (cc3[k]: the last stage's cc when the node has > k free slices of x, else -INF)
     h2* r = rows + (x * 11) * nb + tid;
     r[0 * nb] = fr > 0 ? p1 : kInf2;
     r[1 * nb] = fr > 1 ? p1 : kInf2;
     r[2 * nb] = fr > 0 ? p2 : kInf2;
     r[3 * nb] = fr > 1 ? p2 : kInf2;
     r[4 * nb] = fr > 2 ? p2 : kInf2;
-    r[5 * nb] = fr > 0 ? w3 : kGuard;
-    r[6 * nb] = fr > 1 ? w3 : kGuard;
-    r[7 * nb] = fr > 2 ? w3 : kGuard;
-    r[8 * nb] = fr > 3 ? w3 : kGuard;
+    r[5 * nb] = fr > 0 ? cc : kNegInf2;
+    r[6 * nb] = fr > 1 ? cc : kNegInf2;
+    r[7 * nb] = fr > 2 ? cc : kNegInf2;
+    r[8 * nb] = fr > 3 ? cc : kNegInf2;
     r[9 * nb] = fr > 0 ? p0 : kInf2;
     r[10 * nb] = na0;
   }
+  // guarded SLO slack of the fastest admissible last stage (h2guard): S3 <= slack - v3min
+  const uint32_t slk = h2guard(h2pack(slack[0] - v3min[0], slack[1] - v3min[1]));
   uint32_t pendA = 0, pendB = 0;
 #if FFS_UNROLL_D0
 #pragma unroll
@@ -862,9 +882,9 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
       W[x].s1 = r[0];
       W[x].s2[0] = r[2 * nb];
       W[x].s2[1] = r[3 * nb];
-      W[x].s3[0] = r[5 * nb];
-      W[x].s3[1] = r[6 * nb];
-      W[x].s3[2] = r[7 * nb];
+      W[x].c3[0] = r[5 * nb];
+      W[x].c3[1] = r[6 * nb];
+      W[x].c3[2] = r[7 * nb];
     }
     const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
     const h2 NL1 = rows[(d0 * 11 + 10) * nb + tid];  // -alpha t0^2
@@ -877,14 +897,16 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
       for (int q = 0; q < kP; ++q) {
         const h2 S3 = h2add(S2, W[q].s2[q == d1]);
         const h2 U = h2fma(S3, S3, h2sub(NL2, a2[q]));
-        acc[q] = ~0u;
+        // y_p = S3 * 2t3 + (1 - alpha_h) t3^2 (-INF for an inadmissible last stage); the
+        // group's best z = max_p y_p + U (rounding is monotone: the same decision as testing
+        // every candidate's own z), two 3-input packed maxima (VHMNMX) per 5 candidates
+        h2 y[kP];
 #pragma unroll
-        for (int p = 0; p < kP; ++p) {
-          const h2 z = h2add(h2fma(S3, t2[p], cc[p]), U);
-          // bit 15/31 clear <=> slack - v3 < S3: SLO / memory / free miss (h2guard)
-          const uint32_t ok = isub(W[p].s3[(p == d1) + (p == q)], S3, zero);
-          acc[q] &= z | ~ok;
-        }
+        for (int p = 0; p < kP; ++p) y[p] = h2fma(S3, t2[p], W[p].c3[(p == d1) + (p == q)]);
+        const h2 z = h2add(h2max(h2max(h2max(y[0], y[1]), y[2]), h2max(y[3], y[4])), U);
+        // group SLO test: bit 15/31 clear <=> S3 + (fastest admissible t3) > slack
+        const uint32_t ok = isub(slk, S3, zero);
+        acc[q] = z | ~ok;
       }
       mm[d1] = acc[0] & acc[1] & acc[2] & acc[3] & acc[4];
     }
