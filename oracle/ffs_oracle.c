@@ -916,3 +916,304 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
     free(memt);
     return 0;
 }
+
+/* ==== NEXT-1 DAG stages (oracle_plan_dag; R40-R43) ======================
+ * The FFS DAG of a function ("represents the components in the function as nodes
+ * and dataflows among them as edges") is read as a series of UNITS: a unit is one
+ * component or a parallel block of 2..4 branches (fork/join), each branch a chain of
+ * components (the expanded image classification app "is extended with two
+ * branches to form a DAG").  Components are numbered unit by unit, branch by branch.
+ *   R40 cuts: only between units -- the dominators of a series-parallel DAG ("based
+ *       on the dominator-based method from ESG"); a stage is a run of consecutive units.
+ *   R41 a stage runs on ONE slice (all its components in sequence: t = sum of their
+ *       latencies, memory = sum), or -- only when the stage is exactly one parallel block --
+ *       SPLIT: branch j on its own slice of profile p_j, t = max_j (branch time) ("If a
+ *       stage involves multiple MIGs running in parallel, we use the maximum execution time
+ *       among them as the stage's execution time"), memory checked per branch slice.
+ *   R42 a cut after a unit moves every branch output: cost = sum over its branches of the
+ *       xfer_us of the branch's last component (one component: its xfer_us, as R7).
+ *   R43 candidate order: k ascending, unit-cut masks ascending, stage options in mixed
+ *       radix (stage 0 most significant); option o < P = one slice of profile o, o = P + w
+ *       = split with branch profiles the base-P digits of w (branch 0 most significant).
+ *       idx = the candidate's position; key, feasibility and binding as R1-R11 with every
+ *       slice of the plan counted (gpcs, free slices), slots in stage then branch order.
+ * A DAG of one-component units is the chain of oracle_plan, candidate for candidate. */
+#define DAG_MAX_UNITS 16
+#define DAG_MAX_BR 4
+#define DAG_MAX_SLOTS 16
+
+typedef struct {
+    const uint32_t *unit_off; /* [F+1] */
+    const uint8_t *unit_nb;   /* [U] branches, 1..4 */
+    const uint8_t *unit_bend; /* [U][4] function-relative exclusive end component of branch j */
+    int64_t *key;
+    int32_t *status, *k, *slice /* [R][16] */;
+    uint32_t *cut_mask, *split_mask, *e2e_us, *bottleneck_us, *gpcs_out, *cvq, *n_slots;
+    uint8_t *prof /* [R][16] */;
+    uint64_t *checks /* [R][3], nullable */;
+} oracle_dag_args;
+
+typedef struct {
+    int nb, c0;               /* branches, first component (function-relative) */
+    int bc0[DAG_MAX_BR], bc1[DAG_MAX_BR]; /* branch j = components [bc0, bc1) */
+} dag_unit;
+
+static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, int r) {
+    const int P = a->P;
+    d->status[r] = PLAN_BAD_REQ;
+    d->key[r] = KEY_NONE;
+    d->k[r] = 0;
+    d->cut_mask[r] = d->split_mask[r] = d->e2e_us[r] = d->bottleneck_us[r] = 0;
+    d->gpcs_out[r] = d->cvq[r] = d->n_slots[r] = 0;
+    for (int i = 0; i < DAG_MAX_SLOTS; i++) {
+        d->prof[(size_t)r * DAG_MAX_SLOTS + i] = 0xFF;
+        d->slice[(size_t)r * DAG_MAX_SLOTS + i] = -1;
+    }
+    if (d->checks)
+        for (int i = 0; i < 3; i++) d->checks[(size_t)r * 3 + i] = 0;
+    if (a->req_func[r] >= (uint32_t)a->F || a->req_node[r] >= (uint32_t)a->n_nodes) return;
+    const int f = (int)a->req_func[r], v = (int)a->req_node[r];
+    const uint32_t base = a->comp_off[f], B = a->req_slo_us[r];
+    const int m = (int)(d->unit_off[f + 1] - d->unit_off[f]);
+    dag_unit U[DAG_MAX_UNITS];
+    int c = 0;
+    for (int u = 0; u < m; u++) {
+        const uint32_t gu = d->unit_off[f] + (uint32_t)u;
+        U[u].nb = d->unit_nb[gu];
+        U[u].c0 = c;
+        for (int j = 0; j < U[u].nb; j++) {
+            U[u].bc0[j] = c;
+            U[u].bc1[j] = d->unit_bend[(size_t)gu * DAG_MAX_BR + j];
+            c = U[u].bc1[j];
+        }
+    }
+    uint32_t free_cnt[ORACLE_MAX_P] = {0};
+    for (int i = 0; i < a->n_slices; i++)
+        if (a->sl_node[i] == v && !a->sl_busy[i]) free_cnt[a->sl_prof[i]]++;
+
+    int64_t best = KEY_NONE;
+    int best_k = 0, best_nsl = 0;
+    uint32_t best_mask = 0, best_split = 0;
+    int best_prof[DAG_MAX_SLOTS];
+    uint64_t idx = 0, nfeas = 0, ksum = 0;
+    const int kmax = a->k_max < m ? a->k_max : m;
+    for (int k = 1; k <= kmax; k++) {
+        for (uint32_t mask = 0; mask < (1u << (m - 1)); mask++) {
+            if (__builtin_popcount(mask) != k - 1) continue;
+            /* stages: runs of units; stage s = units [su0[s], su1[s]] */
+            int su0[ORACLE_MAX_STAGES], su1[ORACLE_MAX_STAGES], st = 0;
+            su0[0] = 0;
+            uint64_t xfer = 0;
+            for (int u = 0; u < m; u++) {
+                const int cut = u < m - 1 && ((mask >> u) & 1u);
+                if (cut) /* R42: every branch output of unit u moves */
+                    for (int j = 0; j < U[u].nb; j++) xfer += a->xfer_us[base + (uint32_t)U[u].bc1[j] - 1];
+                if (u == m - 1 || cut) {
+                    su1[st] = u;
+                    st++;
+                    if (st < k) su0[st] = u + 1;
+                }
+            }
+            uint64_t nopt[ORACLE_MAX_STAGES], total = 1;
+            for (int s = 0; s < k; s++) {
+                const int blk = su0[s] == su1[s] && U[su0[s]].nb >= 2;
+                uint64_t pb = 1;
+                if (blk)
+                    for (int j = 0; j < U[su0[s]].nb; j++) pb *= (uint64_t)P;
+                nopt[s] = (uint64_t)P + (blk ? pb : 0);
+                total *= nopt[s];
+            }
+            for (uint64_t o = 0; o < total; o++, idx++) {
+                uint64_t opt[ORACLE_MAX_STAGES], rest = o;
+                for (int s = k - 1; s >= 0; s--) {
+                    opt[s] = rest % nopt[s];
+                    rest /= nopt[s];
+                }
+                uint64_t t[ORACLE_MAX_STAGES], sum_t = 0, g = 0;
+                int prof[DAG_MAX_SLOTS], nsl = 0, feasible = 1;
+                uint32_t split = 0;
+                for (int s = 0; s < k; s++) {
+                    if (opt[s] < (uint64_t)P) { /* one slice: every component of the stage */
+                        const int p = (int)opt[s];
+                        uint64_t ts = 0, ms = 0;
+                        for (int u = su0[s]; u <= su1[s]; u++)
+                            for (int j = 0; j < U[u].nb; j++)
+                                for (int cc = U[u].bc0[j]; cc < U[u].bc1[j]; cc++) {
+                                    ts += lat_of(a, f, cc, p);
+                                    ms += a->mem_mib[base + (uint32_t)cc];
+                                }
+                        if (ms > a->cap_mib[p]) feasible = 0;
+                        t[s] = ts;
+                        prof[nsl++] = p;
+                    } else { /* split: branch j on its own slice, the stage takes the max */
+                        const dag_unit *un = &U[su0[s]];
+                        int pj[DAG_MAX_BR];
+                        uint64_t w = opt[s] - (uint64_t)P;
+                        for (int j = un->nb - 1; j >= 0; j--) {
+                            pj[j] = (int)(w % (uint64_t)P);
+                            w /= (uint64_t)P;
+                        }
+                        uint64_t ts = 0;
+                        for (int j = 0; j < un->nb; j++) {
+                            uint64_t tb = 0, mb = 0;
+                            for (int cc = un->bc0[j]; cc < un->bc1[j]; cc++) {
+                                tb += lat_of(a, f, cc, pj[j]);
+                                mb += a->mem_mib[base + (uint32_t)cc];
+                            }
+                            if (mb > a->cap_mib[pj[j]]) feasible = 0;
+                            if (tb > ts) ts = tb;
+                            prof[nsl++] = pj[j];
+                        }
+                        t[s] = ts;
+                        split |= 1u << s;
+                    }
+                    if (!within_floor(a, f, t[s])) feasible = 0;
+                    sum_t += t[s];
+                }
+                for (int i = 0; i < nsl; i++) g += a->gpcs[prof[i]];
+                for (int q = 0; q < P; q++) {
+                    uint32_t used = 0;
+                    for (int i = 0; i < nsl; i++) used += prof[i] == q;
+                    if (used > free_cnt[q]) feasible = 0;
+                }
+                if (sum_t + xfer > B) feasible = 0;
+                if (!feasible) continue;
+                unsigned __int128 sum_sq = 0;
+                for (int s = 0; s < k; s++) sum_sq += (unsigned __int128)t[s] * t[s];
+                unsigned __int128 D = (unsigned __int128)sum_t * sum_t;
+                unsigned __int128 N = (unsigned __int128)k * sum_sq - D;
+                uint64_t cvq = (uint64_t)(((unsigned __int128)1024 * N) / D); /* Eq. 1, R3, R4 */
+                int64_t key = (int64_t)((cvq << 50) | ((uint64_t)(k - 1) << 47) | (g << 41) | idx);
+                nfeas++;
+                ksum += (uint64_t)key;
+                if (key < best) {
+                    best = key;
+                    best_k = k;
+                    best_mask = mask;
+                    best_split = split;
+                    best_nsl = nsl;
+                    for (int i = 0; i < nsl; i++) best_prof[i] = prof[i];
+                }
+            }
+        }
+    }
+    if (d->checks) {
+        d->checks[(size_t)r * 3 + 0] = idx;
+        d->checks[(size_t)r * 3 + 1] = nfeas;
+        d->checks[(size_t)r * 3 + 2] = ksum;
+    }
+    if (best == KEY_NONE) {
+        d->status[r] = PLAN_INFEASIBLE;
+        return;
+    }
+    d->status[r] = PLAN_OK;
+    d->key[r] = best;
+    d->k[r] = best_k;
+    d->cut_mask[r] = best_mask;
+    d->split_mask[r] = best_split;
+    d->cvq[r] = (uint32_t)((uint64_t)best >> 50);
+    d->n_slots[r] = (uint32_t)best_nsl;
+    /* the plan's figures, recomputed from the winner (stage times as in the search) */
+    uint64_t e2e = 0, bott = 0, g = 0;
+    int s = 0, slot = 0;
+    uint64_t tcur = 0;
+    for (int u = 0; u < m; u++) {
+        const int cut = u < m - 1 && ((best_mask >> u) & 1u);
+        if ((best_split >> s) & 1u) {
+            for (int j = 0; j < U[u].nb; j++) {
+                uint64_t tb = 0;
+                for (int cc = U[u].bc0[j]; cc < U[u].bc1[j]; cc++) tb += lat_of(a, f, cc, best_prof[slot + j]);
+                if (tb > tcur) tcur = tb;
+            }
+        } else {
+            for (int j = 0; j < U[u].nb; j++)
+                for (int cc = U[u].bc0[j]; cc < U[u].bc1[j]; cc++) tcur += lat_of(a, f, cc, best_prof[slot]);
+        }
+        if (cut)
+            for (int j = 0; j < U[u].nb; j++) e2e += a->xfer_us[base + (uint32_t)U[u].bc1[j] - 1];
+        if (u == m - 1 || cut) {
+            e2e += tcur;
+            if (tcur > bott) bott = tcur;
+            slot += ((best_split >> s) & 1u) ? U[u].nb : 1;
+            tcur = 0;
+            s++;
+        }
+    }
+    for (int i = 0; i < best_nsl; i++) g += a->gpcs[best_prof[i]];
+    d->e2e_us[r] = (uint32_t)e2e;
+    d->bottleneck_us[r] = (uint32_t)bott;
+    d->gpcs_out[r] = (uint32_t)g;
+    /* bind (R11): slot i takes the lowest-index free slice of its profile in node v that
+     * no earlier slot took */
+    for (int i = 0; i < best_nsl; i++) {
+        d->prof[(size_t)r * DAG_MAX_SLOTS + i] = (uint8_t)best_prof[i];
+        for (int x = 0; x < a->n_slices; x++) {
+            if (a->sl_node[x] != v || a->sl_busy[x] || a->sl_prof[x] != best_prof[i]) continue;
+            int taken = 0;
+            for (int j = 0; j < i; j++)
+                if (d->slice[(size_t)r * DAG_MAX_SLOTS + j] == x) taken = 1;
+            if (taken) continue;
+            d->slice[(size_t)r * DAG_MAX_SLOTS + i] = x;
+            break;
+        }
+    }
+}
+
+typedef struct {
+    const oracle_plan_args *a;
+    const oracle_dag_args *d;
+    int tid, nthreads;
+} dag_worker_arg;
+
+static void *dag_worker(void *p) {
+    dag_worker_arg *w = (dag_worker_arg *)p;
+    for (int r = w->tid; r < w->a->R; r += w->nthreads) plan_dag_one(w->a, w->d, r);
+    return NULL;
+}
+
+/* Returns 0, or -1 for a malformed DAG table (units not covering the chain, a branch
+ * count outside 1..4, > 16 units, an empty branch, a one-branch unit of more than one
+ * component) or k_max * (slices per stage) * max gpcs >= 64 (the 6-bit key field). */
+int oracle_plan_dag(const oracle_plan_args *a, const oracle_dag_args *d, int n_threads) {
+    if (a->P < 1 || a->P > ORACLE_MAX_P || a->k_max < 1 || a->k_max > ORACLE_MAX_STAGES) return -1;
+    uint32_t maxg = 0, maxnb = 1;
+    for (int p = 0; p < a->P; p++)
+        if (a->gpcs[p] > maxg) maxg = a->gpcs[p];
+    for (int f = 0; f < a->F; f++) {
+        const int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
+        const int m = (int)(d->unit_off[f + 1] - d->unit_off[f]);
+        if (m < 1 || m > DAG_MAX_UNITS) return -1;
+        int c = 0;
+        for (int u = 0; u < m; u++) {
+            const uint32_t gu = d->unit_off[f] + (uint32_t)u;
+            const int nb = d->unit_nb[gu];
+            if (nb < 1 || nb > DAG_MAX_BR) return -1;
+            if ((uint32_t)nb > maxnb) maxnb = (uint32_t)nb;
+            for (int j = 0; j < nb; j++) {
+                const int e = d->unit_bend[(size_t)gu * DAG_MAX_BR + j];
+                if (e <= c) return -1;
+                c = e;
+            }
+        }
+        if (c != n) return -1;
+        for (int u = 0; u < m; u++) { /* a one-branch unit is one component */
+            const uint32_t gu = d->unit_off[f] + (uint32_t)u;
+            const int start = u == 0 ? 0 : (int)d->unit_bend[(size_t)(gu - 1) * DAG_MAX_BR + d->unit_nb[gu - 1] - 1];
+            if (d->unit_nb[gu] == 1 && d->unit_bend[(size_t)gu * DAG_MAX_BR] != start + 1) return -1;
+        }
+    }
+    if ((uint64_t)a->k_max * maxnb * maxg >= 64) return -1;
+    if (n_threads < 1) n_threads = 1;
+    pthread_t th[256];
+    dag_worker_arg w[256];
+    if (n_threads > 256) n_threads = 256;
+    for (int i = 0; i < n_threads; i++) {
+        w[i].a = a;
+        w[i].d = d;
+        w[i].tid = i;
+        w[i].nthreads = n_threads;
+        pthread_create(&th[i], NULL, dag_worker, &w[i]);
+    }
+    for (int i = 0; i < n_threads; i++) pthread_join(th[i], NULL);
+    return 0;
+}

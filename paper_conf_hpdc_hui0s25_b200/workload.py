@@ -496,3 +496,85 @@ def with_throughput_floor(prob: Problem, seed: int = 0x5EEDF100, lo: float = 0.3
     d["max_stage_us"] = np.maximum(fl, 0).astype(np.uint32)
     d["name"] = prob.name + "+floor"
     return Problem(**d)
+
+
+# ----------------------------------------------------------------------------------
+# NEXT-1 DAG functions (R40-R43): series of units, a unit is one component or
+# a fork/join block of parallel branches (expanded image classification "is
+# extended with two branches to form a DAG")
+# ----------------------------------------------------------------------------------
+@dataclass
+class DagTable:
+    """Unit structure of every function of a Problem (include/ffs.h ffs_dag_table)."""
+    unit_off: np.ndarray   # uint32 [F+1]
+    unit_nb: np.ndarray    # uint8  [U] branches 1..4 (1 = one component)
+    unit_bend: np.ndarray  # uint8  [U, 4] function-relative exclusive end of branch j (0 unused)
+
+    def units(self, f: int) -> list[list[tuple[int, int]]]:
+        """Function f's units as lists of (first, end) component ranges per branch."""
+        out, c = [], 0
+        for u in range(int(self.unit_off[f]), int(self.unit_off[f + 1])):
+            br = []
+            for j in range(int(self.unit_nb[u])):
+                e = int(self.unit_bend[u, j])
+                br.append((c, e))
+                c = e
+            out.append(br)
+        return out
+
+
+def chain_dag(prob: Problem) -> DagTable:
+    """The DAG of a plain chain: every component is its own unit."""
+    n = prob.chain_len()
+    unit_off = np.zeros(prob.F + 1, dtype=np.uint32)
+    unit_off[1:] = np.cumsum(n)
+    bend = np.zeros((int(unit_off[-1]), 4), dtype=np.uint8)
+    bend[:, 0] = np.concatenate([np.arange(1, int(x) + 1) for x in n])
+    return DagTable(unit_off, np.ones(int(unit_off[-1]), dtype=np.uint8), bend)
+
+
+def make_dag_shapes(rng: SplitMix64, F: int, units=(3, 8), p_block=0.35, branches=(2, 2), br_len=(1, 3)):
+    """Per function: a list of units, each a list of branch lengths."""
+    shapes = []
+    for _ in range(F):
+        m = int(rng.integers(units[0], units[1], 1)[0])
+        u_list = []
+        for _ in range(m):
+            if float(rng.uniform(1)[0]) < p_block:
+                nb = int(rng.integers(branches[0], branches[1], 1)[0])
+                u_list.append([int(x) for x in rng.integers(br_len[0], br_len[1], nb)])
+            else:
+                u_list.append([1])
+        shapes.append(u_list)
+    return shapes
+
+
+def dag_table(shapes) -> DagTable:
+    unit_off = np.zeros(len(shapes) + 1, dtype=np.uint32)
+    unit_off[1:] = np.cumsum([len(s) for s in shapes])
+    U = int(unit_off[-1])
+    nb = np.zeros(U, dtype=np.uint8)
+    bend = np.zeros((U, 4), dtype=np.uint8)
+    u = 0
+    for s in shapes:
+        c = 0
+        for br in s:
+            nb[u] = len(br)
+            for j, L in enumerate(br):
+                c += L
+                bend[u, j] = c
+            u += 1
+    return DagTable(unit_off, nb, bend)
+
+
+def dag_config(seed: int | None = None, R: int = 1 << 16, F: int = 32, node_parts=None, k_max: int = 4,
+               p_block: float = 0.35, units=(3, 8), branches=(2, 2)) -> tuple[Problem, DagTable]:
+    """CD: DAG functions (3..8 units, a unit a 2-branch block with probability 0.35,
+    branches of 1..3 components) on the C3 cluster (8 nodes = 64 GPUs), Azure-shaped
+    requests as C3.  Components and budgets follow the chain recipe (make_function,
+    R9 SLO on the summed single-slice latency)."""
+    rng = SplitMix64(SEED_BASE + 6 if seed is None else seed)
+    shapes = make_dag_shapes(rng.sub(8), F, units, p_block, branches)
+    lengths = [sum(sum(br) for br in s) for s in shapes]
+    prob = _problem("CD", rng, lengths, NODE_BLOCK if node_parts is None else node_parts, R, k_max=k_max)
+    return prob, dag_table(shapes)
