@@ -156,17 +156,17 @@ def plan_dag(prob, dag, k_max: int | None = None, threads: int | None = None, ch
     structure ``dag`` (unit_off, unit_nb, unit_bend[U,4]; see ffs_oracle.c:
     oracle_plan_dag, R40-R43).  Returns key, status, k, cut_mask (over unit
     boundaries), split_mask (bit s: stage s runs its branches on separate slices),
-    e2e_us, bottleneck_us, gpcs, cvq, n_slots, prof[R,16], slice[R,16] and checks[R,3]."""
+    e2e_us, bottleneck_us, gpcs, cvq, n_slots, prof[R,8], slice[R,8] and checks[R,3]."""
     k_max = int(prob.k_max if k_max is None else k_max)
     threads = os.cpu_count() if threads is None else threads
     h = _Held(prob, k_max, False)
     R = prob.R
     uo, nb, be = _c(dag.unit_off, np.uint32), _c(dag.unit_nb, np.uint8), _c(dag.unit_bend, np.uint8)
     o = {"key": np.zeros(R, np.int64), "status": np.zeros(R, np.int32), "k": np.zeros(R, np.int32),
-         "slice": np.zeros((R, 16), np.int32), "cut_mask": np.zeros(R, np.uint32),
+         "slice": np.zeros((R, 8), np.int32), "cut_mask": np.zeros(R, np.uint32),
          "split_mask": np.zeros(R, np.uint32), "e2e_us": np.zeros(R, np.uint32),
          "bottleneck_us": np.zeros(R, np.uint32), "gpcs": np.zeros(R, np.uint32), "cvq": np.zeros(R, np.uint32),
-         "n_slots": np.zeros(R, np.uint32), "prof": np.zeros((R, 16), np.uint8)}
+         "n_slots": np.zeros(R, np.uint32), "prof": np.zeros((R, 8), np.uint8)}
     if checks:
         o["checks"] = np.zeros((R, 3), np.uint64)
     d = _DagArgs(_p(uo), _p(nb), _p(be), _p(o["key"]), _p(o["status"]), _p(o["k"]), _p(o["slice"]),

@@ -936,20 +936,21 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
  *       radix (stage 0 most significant); option o < P = one slice of profile o, o = P + w
  *       = split with branch profiles the base-P digits of w (branch 0 most significant).
  *       idx = the candidate's position; key, feasibility and binding as R1-R11 with every
- *       slice of the plan counted (gpcs, free slices), slots in stage then branch order.
+ *       slice of the plan counted (gpcs, free slices), slots in stage then branch order;
+ *       k_max * (max branches) <= 8, so a plan holds at most 8 slices.
  * A DAG of one-component units is the chain of oracle_plan, candidate for candidate. */
 #define DAG_MAX_UNITS 16
 #define DAG_MAX_BR 4
-#define DAG_MAX_SLOTS 16
+#define DAG_MAX_SLOTS 8
 
 typedef struct {
     const uint32_t *unit_off; /* [F+1] */
     const uint8_t *unit_nb;   /* [U] branches, 1..4 */
     const uint8_t *unit_bend; /* [U][4] function-relative exclusive end component of branch j */
     int64_t *key;
-    int32_t *status, *k, *slice /* [R][16] */;
+    int32_t *status, *k, *slice /* [R][8] */;
     uint32_t *cut_mask, *split_mask, *e2e_us, *bottleneck_us, *gpcs_out, *cvq, *n_slots;
-    uint8_t *prof /* [R][16] */;
+    uint8_t *prof /* [R][8] */;
     uint64_t *checks /* [R][3], nullable */;
 } oracle_dag_args;
 
@@ -1173,7 +1174,8 @@ static void *dag_worker(void *p) {
 
 /* Returns 0, or -1 for a malformed DAG table (units not covering the chain, a branch
  * count outside 1..4, > 16 units, an empty branch, a one-branch unit of more than one
- * component) or k_max * (slices per stage) * max gpcs >= 64 (the 6-bit key field). */
+ * component), k_max * (max branches) > 8 (slices per plan) or k_max * (max branches) *
+ * max gpcs >= 64 (the 6-bit key field). */
 int oracle_plan_dag(const oracle_plan_args *a, const oracle_dag_args *d, int n_threads) {
     if (a->P < 1 || a->P > ORACLE_MAX_P || a->k_max < 1 || a->k_max > ORACLE_MAX_STAGES) return -1;
     uint32_t maxg = 0, maxnb = 1;
@@ -1202,7 +1204,7 @@ int oracle_plan_dag(const oracle_plan_args *a, const oracle_dag_args *d, int n_t
             if (d->unit_nb[gu] == 1 && d->unit_bend[(size_t)gu * DAG_MAX_BR] != start + 1) return -1;
         }
     }
-    if ((uint64_t)a->k_max * maxnb * maxg >= 64) return -1;
+    if ((uint64_t)a->k_max * maxnb > DAG_MAX_SLOTS || (uint64_t)a->k_max * maxnb * maxg >= 64) return -1;
     if (n_threads < 1) n_threads = 1;
     pthread_t th[256];
     dag_worker_arg w[256];

@@ -161,7 +161,7 @@ def random_dag(seed, K=3, nb_max=3):
 
 @pytest.mark.parametrize("seed", range(2000, 2030))
 def test_dag_oracle_matches_independent_brute_force(seed):
-    prob, d = random_dag(seed, K=2 if seed % 3 == 0 else 3, nb_max=4 if seed % 3 == 0 else 3)
+    prob, d = random_dag(seed, K=2 if seed % 3 == 0 else 3, nb_max=4 if seed % 3 == 0 else 2)
     o = oracle.plan_dag(prob, d, threads=2)
     for r in range(prob.R):
         best, scored, nfeas, ksum = brute_dag(prob, d, r)
