@@ -254,6 +254,41 @@ def run_ranked(pl, prob, req, slo, steps: int, warmup: int, flush):
             "ok_frac": float((p["status"] == 0).mean()), "multi_stage_frac": float(((p["status"] == 0) & (p["k"] > 1)).mean())}
 
 
+def run_dag(pl, steps: int, warmup: int, flush):
+    """NEXT-1 DAG stages (R40-R43) on the CD workload (32 DAG functions on the C3 cluster,
+    65,536 requests): candidates/s and plans/s of ffs_plan_dag (one warp per request, exact
+    integer scoring).  Stages its own tables; run after the C5 legs."""
+    import torch
+    from paper_conf_hpdc_hui0s25_b200 import ffs
+    prob, dag = W.dag_config()
+    pl.stage(prob)
+    pl.stage_dag(dag, prob.k_max)
+    req, slo = ffs.to_device(prob)
+    out = torch.empty((prob.R, ffs.DAG_PLAN_DTYPE.itemsize), dtype=torch.uint8, device="cuda")
+    checks = torch.zeros((prob.R, 3), dtype=torch.int64, device="cuda")
+    pl.plan_dag(req, slo, out=out, checks=checks)  # candidate count (checksums), untimed
+    torch.cuda.synchronize()
+    cands = int(checks[:, 0].sum().item())
+    for _ in range(warmup):
+        pl.plan_dag(req, slo, out=out)
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    ms = 0.0
+    for i in range(steps):
+        flush.fill_(i & 0xFF)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        pl.plan_dag(req, slo, out=out)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ms += a.elapsed_time(b)
+    p = ffs.dag_plans_to_numpy(out)
+    return {"metric": "dag_candidates_scored_per_s", "value": cands * steps / (ms * 1e-3), "unit": "candidates/s",
+            "plans_per_s": prob.R * steps / (ms * 1e-3), "ms_per_step": ms / steps, "candidates_per_step": cands,
+            "workload": "CD: 32 DAG functions (3-8 units, 2-branch blocks p=0.35), C3 cluster, R=65536, K=4",
+            "ok_frac": float((p["status"] == 0).mean()), "split_frac": float((p["split_mask"] > 0).mean())}
+
+
 def run_joint(pl, prob, req, slo):
     """NEXT-2 (joint commit in adjusted-deadline order) on the same batch:
     one call, wall/event time, rounds."""
@@ -479,10 +514,11 @@ def main():
     if world == 1 and not args.no_c4:
         joint = run_joint(pl, prob, req, slo)
         frontier = run_frontier(pl, prob, req, slo, args.steps, args.warmup, flush)
-    c4 = sim = None
+    c4 = sim = dagr = None
     if world == 1 and not args.no_c4:
         c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
         sim = run_sim(pl)
+        dagr = run_dag(pl, args.steps, args.warmup, flush)
     if rank == 0:
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
@@ -513,6 +549,7 @@ def main():
             "joint_commit": joint,
             "frontier": frontier,
             "timeshare_sim": sim,
+            "dag_stages": dagr,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -274,6 +274,72 @@ ffs_status ffs_rank_partitions(ffs_ctx *ctx, uint32_t k_max, uint32_t p_ref);
 ffs_status ffs_plan_ranked(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
                            ffs_plan *d_out, void *stream);
 
+/* ---- NEXT-1: DAG stages (R40-R43) -----------------------
+ * The FFS DAG of a function is read as a series of UNITS: one component, or a fork/join
+ * block of 2..4 parallel branches, each branch a chain of components (an app "is
+ * extended with two branches to form a DAG").  The staged profile table numbers each
+ * function's components unit by unit, branch by branch.  Stages are runs of consecutive
+ * units (cuts only at unit boundaries -- the dominators, "dominator-based method
+ * from ESG").  A stage runs on one slice (t = sum of all its components' latencies,
+ * memory = sum), or, when the stage is exactly one block, SPLIT: branch j on its own slice
+ * of profile p_j and t = max_j branch time ("If a stage involves multiple MIGs
+ * running in parallel, we use the maximum execution time among them as the stage's
+ * execution time"), memory checked per branch slice.  A cut after a unit costs the sum of
+ * xfer_us of its branches' last components (R42).  Candidate order (R43): k ascending,
+ * unit-cut masks ascending, stage options in mixed radix with stage 0 most significant,
+ * option o < P = one slice of profile o, o = P + w = split with branch profiles the base-P
+ * digits of w (branch 0 most significant); key, feasibility and binding as ffs_plan_keys /
+ * ffs_plan_decode with every slice of the plan counted (gpcs, free slices).
+ * A table of one-component units reproduces ffs_plan_batch's keys exactly. */
+#define FFS_DAG_MAX_UNITS 16
+#define FFS_DAG_MAX_BRANCHES 4
+#define FFS_DAG_MAX_SLOTS 8
+
+/* Unit structure of every staged function.  Host pointers, copied by ffs_dag_stage. */
+typedef struct {
+    uint32_t n_funcs;          /* = n_funcs of the staged profile table                       */
+    const uint32_t *unit_off;  /* [F+1] function f has units unit_off[f] .. unit_off[f+1]-1  */
+    const uint8_t *unit_nb;    /* [U] branches of the unit, 1..4 (1 = exactly one component) */
+    const uint8_t *unit_bend;  /* [U][4] function-relative exclusive end component of branch j
+                                  (branch j starts where branch j-1, or the previous unit,
+                                  ends); entries j >= nb are ignored                         */
+} ffs_dag_table;
+
+/* The plan of one request of a DAG function (88 bytes).  Slots: the plan's slices in
+ * stage order, a split stage's branches in branch order. */
+typedef struct {
+    int64_t key;            /* FFS_KEY_NONE when not OK                                  */
+    uint32_t status;        /* FFS_PLAN_*                                                 */
+    uint32_t k;             /* stages                                                     */
+    uint32_t cut_mask;      /* bit u = stage boundary after unit u                        */
+    uint32_t split_mask;    /* bit s = stage s runs its branches on separate slices       */
+    uint32_t e2e_us;        /* sum of stage times + cut transfers                         */
+    uint32_t bottleneck_us; /* max stage time; throughput = 1e6 / bottleneck_us rps       */
+    uint32_t gpcs;          /* sum of GPCs of every slice of the plan                     */
+    uint32_t cvq;           /* floor(1024 * CV^2) of the k stage times (Eq. 1)            */
+    uint32_t n_slots;       /* slices of the plan                                         */
+    uint32_t pad;
+    uint8_t prof[FFS_DAG_MAX_SLOTS];  /* profile of slot i (0xFF unused)                  */
+    int32_t slice[FFS_DAG_MAX_SLOTS]; /* bound slice (lowest free index of the profile not
+                                         taken by an earlier slot, R11), -1 unused        */
+} ffs_dag_plan;
+
+/* Validate and upload the unit structure for plans with up to k_max stages (host work:
+ * the per-function list of unit-cut masks with candidate offsets).  Synchronous.
+ * FFS_ERR_ARG: n_funcs differs from the staged table, units not covering a chain, a
+ * branch count outside 1..4, an empty branch, a one-branch unit of more than one
+ * component.  FFS_ERR_RANGE: > 16 units, k_max not in 1..8, k_max * max branches > 8,
+ * k_max * max branches * max gpcs >= 64, >= 2^41 candidates for a function.
+ * FFS_ERR_STATE: tables not staged (staging new tables drops the DAG). */
+ffs_status ffs_dag_stage(ffs_ctx *ctx, const ffs_dag_table *dag, uint32_t k_max);
+/* Plan every request against its home node's free slices: one warp per request, lanes
+ * over the function's unit-cut masks, every candidate scored exactly in integers, warp
+ * argmin; the winning lane writes the plan and binds its slices.  d_checksums (nullable):
+ * uint64[3*n_req] = candidates scored, feasible, sum of feasible keys mod 2^64.
+ * Asynchronous on `stream`.  FFS_ERR_STATE: no DAG staged. */
+ffs_status ffs_plan_dag(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
+                        ffs_dag_plan *d_out, uint64_t *d_checksums, void *stream);
+
 /* ---- NEXT-2: joint commit of the batch ---------------------------------
  * The requests of each node are served one at a time in ascending adjusted deadline
  * (budget - reload time - fastest 1-stage latency, ties by index; R28), each

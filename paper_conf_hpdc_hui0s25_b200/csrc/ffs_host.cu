@@ -49,6 +49,8 @@ struct DeviceGuard {
 
 }  // namespace
 
+static_assert(sizeof(ffs_dag_plan) == 88, "ffs_dag_plan layout");
+
 struct ffs_ctx {
   int device = 0;
   int sms = 0;
@@ -75,6 +77,9 @@ struct ffs_ctx {
   uint32_t front_kmax = 0, front_groups = 0, front_nfv = 0, front_cap = 0;
   // NEXT-1 ranked partitions
   DevBuf rank_off, rank_mask;
+  // NEXT-1 DAG stages
+  DevBuf dag_fu, dag_units, dag_xcut, dag_mt_off, dag_mt_mk, dag_mt_cand;
+  bool dag_staged = false;
   bool ranked = false;
   uint32_t rank_kmax = 0, prof_order = 0;
   // scratch
@@ -164,7 +169,8 @@ void ffs_destroy(ffs_ctx* c) {
     for (DevBuf* b : {&c->node_off, &c->j_keys, &c->j_state, &c->j_dirty, &c->j_sreq, &c->j_sslo, &c->j_skeys,
                       &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
       b->release();
-    for (DevBuf* b : {&c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
+    for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand,
+                      &c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr})
       b->release();
   }
@@ -343,6 +349,7 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   c->lay = L;
   c->h_image = img;
   c->ranked = false;
+  c->dag_staged = false;
   c->front_built = false;
   c->P = P;
   c->F = F;
@@ -686,6 +693,127 @@ ffs_status ffs_plan_ranked(ffs_ctx* c, const ffs_request* d_req, const uint32_t*
   a.prof_order = c->prof_order;
   a.out = d_out;
   CK(launch_ranked(a, (cudaStream_t)stream), "ranked kernel");
+  return FFS_OK;
+}
+
+// ---- NEXT-1 DAG stages (R40-R43) ------------------------------------
+ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  c->dag_staged = false;
+  if (!d || !d->unit_off || !d->unit_nb || !d->unit_bend) return fail(c, FFS_ERR_ARG, "null DAG table pointer");
+  if (d->n_funcs != c->F) return fail(c, FFS_ERR_ARG, "DAG n_funcs %u != staged %u", d->n_funcs, c->F);
+  if (k_max < 1 || k_max > (uint32_t)kMaxK) return fail(c, FFS_ERR_RANGE, "k_max %u not in 1..8", k_max);
+  if (d->unit_off[0] != 0) return fail(c, FFS_ERR_ARG, "unit_off[0] != 0");
+  const ImageLayout& L = c->lay;
+  const std::vector<uint32_t>& img = c->h_image;
+  const uint32_t F = c->F, U = d->unit_off[F];
+  std::vector<uint32_t> fu(2 * (size_t)F), units(6 * (size_t)std::max(U, 1u), 0), xcut(std::max(U, 1u), 0);
+  uint32_t maxnb = 1;
+  for (uint32_t f = 0; f < F; ++f) {
+    if (d->unit_off[f + 1] < d->unit_off[f]) return fail(c, FFS_ERR_ARG, "unit_off decreasing at %u", f);
+    const uint32_t m = d->unit_off[f + 1] - d->unit_off[f];
+    if (m < 1) return fail(c, FFS_ERR_ARG, "function %u has no units", f);
+    if (m > FFS_DAG_MAX_UNITS) return fail(c, FFS_ERR_RANGE, "function %u has %u > 16 units", f, m);
+    const uint32_t row0 = img[L.o_fdesc + 4 * f], n = img[L.o_fdesc + 4 * f + 1];
+    fu[2 * f] = d->unit_off[f];
+    fu[2 * f + 1] = m;
+    uint32_t cc = 0;
+    for (uint32_t u = d->unit_off[f]; u < d->unit_off[f + 1]; ++u) {
+      const uint32_t nb = d->unit_nb[u];
+      if (nb < 1 || nb > FFS_DAG_MAX_BRANCHES) return fail(c, FFS_ERR_ARG, "unit %u: %u branches not in 1..4", u, nb);
+      maxnb = std::max(maxnb, nb);
+      units[6 * (size_t)u] = nb;
+      units[6 * (size_t)u + 1] = cc;
+      const uint32_t start = cc;
+      uint32_t x = 0;
+      for (uint32_t j = 0; j < nb; ++j) {
+        const uint32_t e = d->unit_bend[4 * (size_t)u + j];
+        if (e <= cc || e > n) return fail(c, FFS_ERR_ARG, "unit %u branch %u: end %u not in (%u, %u]", u, j, e, cc, n);
+        units[6 * (size_t)u + 2 + j] = e;
+        x += img[L.o_xf + row0 + e - 1];  // R42: every branch output moves at a cut
+        cc = e;
+      }
+      if (nb == 1 && cc != start + 1) return fail(c, FFS_ERR_ARG, "unit %u: one branch of %u components", u, cc - start);
+      xcut[u] = x;
+    }
+    if (cc != n) return fail(c, FFS_ERR_ARG, "function %u: units cover %u of %u components", f, cc, n);
+  }
+  if (k_max * maxnb > FFS_DAG_MAX_SLOTS)
+    return fail(c, FFS_ERR_RANGE, "k_max %u x %u branches > %d slices per plan", k_max, maxnb, FFS_DAG_MAX_SLOTS);
+  if (k_max * maxnb * c->max_gpcs >= 64) return fail(c, FFS_ERR_RANGE, "k_max x branches x max gpcs >= 64");
+  // per function: unit-cut masks in candidate order (k ascending, masks ascending) with
+  // the first candidate index of each (R43)
+  std::vector<uint32_t> mt_off(F + 1, 0), mt_mk;
+  std::vector<unsigned long long> mt_cand;
+  for (uint32_t f = 0; f < F; ++f) {
+    const uint32_t m = fu[2 * f + 1], ub = fu[2 * f];
+    uint64_t cand = 0;
+    for (uint32_t k = 1; k <= std::min(k_max, m); ++k)
+      for (uint32_t mask = 0; mask < (1u << (m - 1)); ++mask) {
+        if ((uint32_t)__builtin_popcount(mask) != k - 1) continue;
+        mt_mk.push_back(mask | (k << 16));
+        mt_cand.push_back(cand);
+        uint64_t tot = 1;
+        uint32_t u0 = 0;
+        for (uint32_t u = 0; u < m; ++u)
+          if (u + 1 == m || ((mask >> u) & 1u)) {
+            const uint32_t nb = units[6 * (size_t)(ub + u0)];
+            uint64_t q = kP;
+            if (u0 == u && nb >= 2) {
+              uint64_t pw = 1;
+              for (uint32_t j = 0; j < nb; ++j) pw *= kP;
+              q += pw;
+            }
+            tot *= q;
+            u0 = u + 1;
+          }
+        cand += tot;
+        if (cand >= (1ull << kIdxBits)) return fail(c, FFS_ERR_RANGE, "function %u: >= 2^41 DAG candidates", f);
+      }
+    mt_off[f + 1] = (uint32_t)mt_mk.size();
+  }
+  DeviceGuard g(c->device);
+  auto up = [&](DevBuf& b, const void* src, size_t bytes) -> cudaError_t {
+    cudaError_t e = b.ensure(std::max<size_t>(bytes, 8));
+    if (e != cudaSuccess || bytes == 0) return e;
+    return cudaMemcpy(b.p, src, bytes, cudaMemcpyHostToDevice);
+  };
+  CK(up(c->dag_fu, fu.data(), fu.size() * 4), "upload dag_fu");
+  CK(up(c->dag_units, units.data(), units.size() * 4), "upload dag_units");
+  CK(up(c->dag_xcut, xcut.data(), xcut.size() * 4), "upload dag_xcut");
+  CK(up(c->dag_mt_off, mt_off.data(), mt_off.size() * 4), "upload dag_mt_off");
+  CK(up(c->dag_mt_mk, mt_mk.data(), mt_mk.size() * 4), "upload dag_mt_mk");
+  CK(up(c->dag_mt_cand, mt_cand.data(), mt_cand.size() * 8), "upload dag_mt_cand");
+  c->dag_staged = true;
+  return FFS_OK;
+}
+
+ffs_status ffs_plan_dag(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo, uint32_t n_req,
+                        ffs_dag_plan* d_out, uint64_t* d_checksums, void* stream) {
+  if (!c) return FFS_ERR_ARG;
+  if (!c->staged || !c->dag_staged) return fail(c, FFS_ERR_STATE, "call ffs_dag_stage after staging");
+  if (n_req == 0) return FFS_OK;
+  if (!d_req || !d_slo || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
+  DeviceGuard g(c->device);
+  DagArgs a{};
+  a.image = c->image.as<uint32_t>();
+  a.lay = c->lay;
+  a.req = d_req;
+  a.slo = d_slo;
+  a.n_req = n_req;
+  a.n_nodes = c->n_nodes;
+  a.node_free = c->node_free.as<uint64_t>();
+  a.free_list = c->free_list.as<int32_t>();
+  a.fu = c->dag_fu.as<uint32_t>();
+  a.units = c->dag_units.as<uint32_t>();
+  a.xcut = c->dag_xcut.as<uint32_t>();
+  a.mt_off = c->dag_mt_off.as<uint32_t>();
+  a.mt_mk = c->dag_mt_mk.as<uint32_t>();
+  a.mt_cand = c->dag_mt_cand.as<unsigned long long>();
+  a.out = d_out;
+  a.checks = reinterpret_cast<unsigned long long*>(d_checksums);
+  CK(launch_dag(a, (cudaStream_t)stream), "dag kernel");
   return FFS_OK;
 }
 

@@ -126,6 +126,26 @@ struct RankedArgs {
 };
 cudaError_t launch_ranked(const RankedArgs& a, cudaStream_t st);
 
+// NEXT-1 DAG stages
+struct DagArgs {
+  const uint32_t* image;
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  uint32_t n_req, n_nodes;
+  const uint64_t* node_free;
+  const int32_t* free_list;
+  const uint32_t* fu;         // [F][2] {first unit, units}
+  const uint32_t* units;      // [U][6] {nb, c0, e0, e1, e2, e3} function-relative components
+  const uint32_t* xcut;       // [U] cost of a cut after the unit (R42)
+  const uint32_t* mt_off;     // [F+1] mask-table entries of f
+  const uint32_t* mt_mk;      // unit-cut mask | k << 16
+  const unsigned long long* mt_cand;  // first candidate index of the entry
+  ffs_dag_plan* out;
+  unsigned long long* checks; // [n_req][3] or null
+};
+cudaError_t launch_dag(const DagArgs& a, cudaStream_t st);
+
 struct JointArgs {
   const uint32_t* image;
   ImageLayout lay;

@@ -345,25 +345,30 @@ __device__ __forceinline__ void load_stage(const SearchState<KS>& c, int s, floa
   }
 }
 
-// ---- unrolled path for KS = 2..4 -----------------------------------
-// The last three (KS = 4) / all (KS <= 3) levels are compile-time loops, so the
-// multiplicity m of a profile within the sequence is a constant and the free-slice
-// check is folded into variant tables vf[s][m][x] = t (stage s on profile x fits in
-// memory and the node has more than m free slices of x) else +INF.  Per candidate
-// (p = last stage; S, L, B = the group's sum of stage times, alpha * sum t^2 and
-// Blim - S):
-//   d2 = B - vf[p]                 sign set <=> SLO, memory or free-slice miss (exact:
-//                                  every operand is an integer < 2^25 or INF)
-//   z  = fma(S, 2t_p, (1-alpha) t_p^2) + (S^2 - L)
-//                                  sign set <=> (S+t_p)^2 <= alpha (sum t^2): cannot beat
-//                                  the running minimum (conservative, §4.3)
+// ---- unrolled path for KS = 2, 3 ------------------------------------
+// All levels are compile-time loops, so the multiplicity m of a profile within the
+// sequence is a constant and the free-slice check is folded into variant tables:
+// vf[s][m][x] = t (stage s on profile x fits in memory and the node has more than m free
+// slices of x) else +INF for the leading stages, and for the last stage the score
+// constant ccv[m][x] = (1 - alpha) t^2 under the same condition else -INF (t2 = 2t, 0 for a
+// stage that fits no slice).  Per group (S, L = the prefix's sum of stage times and
+// alpha * sum t^2, v = the q stage) and its five last-stage profiles p:
+//   y_p = fma(S + v, t2_p, ccv_p)        -INF for an inadmissible last stage
+//   z   = max_p y_p + ((S+v)^2 - L - alpha v^2)
+//                                  sign set <=> no (S+v+t_p)^2 > alpha (sum t^2): no
+//                                  candidate of the group can beat the running minimum
+//                                  (conservative, §4.3; max is exact and rounding monotone)
+//   d2  = (B - vmin) - v           sign set <=> even the fastest admissible last stage
+//                                  misses the SLO (exact: integers < 2^25 or INF)
 //   acc &= bits(z) | bits(d2)      sign of acc clear <=> some candidate may win
-// FFMA + FADD + FADD on the full-rate FMA pipe, one LOP3 on the half-rate ALU pipe.
+// Five FFMA and two 3-input FMNMX3 per five candidates plus a few group operations.
 template <int KS>
 struct Tables {
-  float vf[KS][KS][kP];  // [stage][multiplicity-1][profile], +INF folded
-  float a[KS][kP];       // alpha * t^2   (stages 0..KS-2)
-  float t2[kP], cc[kP];  // last stage: 2t and (1 - alpha) t^2
+  float vf[KS - 1][KS - 1][kP];  // [stage][multiplicity][profile], +INF folded (stages 0..KS-2)
+  float a[KS][kP];               // alpha * t^2   (stages 0..KS-2)
+  float t2[kP];                  // last stage: 2t (0 if it fits no slice)
+  float ccv[KS][kP];             // last stage: (1 - alpha) t^2 by multiplicity, -INF folded
+  float vmin;                    // fastest admissible last stage (>= 1 free slice), else INF
 };
 
 template <int KS>
@@ -382,6 +387,7 @@ template <int KS>
 __device__ __forceinline__ void build_tables(const SearchState<KS>& c, Tables<KS>& T) {
   const float INF = __int_as_float(0x7f800000);
   const float one_m_a = 1.f - c.alpha;
+  T.vmin = INF;
 #pragma unroll
   for (int s = 0; s < KS; ++s) {
     float f[kP];
@@ -390,39 +396,39 @@ __device__ __forceinline__ void build_tables(const SearchState<KS>& c, Tables<KS
     for (int x = 0; x < kP; ++x) {
       const bool mem_ok = c.memst[s] <= c.sm[c.o_cap + x] && f[x] <= c.thr;
       const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-#pragma unroll
-      for (int m = 0; m <= s; ++m) T.vf[s][m][x] = (mem_ok && fr > (uint32_t)m) ? f[x] : INF;
       if (s < KS - 1) {
+#pragma unroll
+        for (int m = 0; m <= s; ++m) T.vf[s][m][x] = (mem_ok && fr > (uint32_t)m) ? f[x] : INF;
         T.a[s][x] = c.alpha * (f[x] * f[x]);
       } else {
-        T.t2[x] = f[x] + f[x];
-        T.cc[x] = one_m_a * (f[x] * f[x]);
+        const float cc = one_m_a * (f[x] * f[x]);
+        T.t2[x] = mem_ok ? f[x] + f[x] : 0.f;
+#pragma unroll
+        for (int m = 0; m <= s; ++m) T.ccv[m][x] = (mem_ok && fr > (uint32_t)m) ? cc : -INF;
+        if (mem_ok && fr > 0) T.vmin = fminf(T.vmin, f[x]);
       }
     }
   }
 }
 
-__device__ __forceinline__ void cand(float S, float U, float B, float v, float t2, float cc, uint32_t& acc) {
-  const float d2 = B - v;
-  const float z = fmaf(S, t2, cc) + U;
-  acc &= __float_as_uint(z) | __float_as_uint(d2);
-}
-
-// one block = the last two levels (q, p): P*P candidates.  vq/vp select the variant
-// tables of the q and p stages by compile-time multiplicity.
-template <class VQ, class VP>
-__device__ __forceinline__ uint32_t block_qp(const float (&aq)[kP], const float (&t2)[kP], const float (&cc)[kP],
-                                             float S, float L, float B, VQ vq, VP vp) {
+// one block = the last two levels (q, p): P*P candidates.  vq selects the q stage's
+// variant table and cp the last stage's score constant by compile-time multiplicity;
+// Bm = Blim - S - vmin.
+template <class VQ, class CP>
+__device__ __forceinline__ uint32_t block_qp(const float (&aq)[kP], const float (&t2)[kP], float S, float L,
+                                             float Bm, VQ vq, CP cp) {
   uint32_t acc = ~0u;
 #pragma unroll
   for (int q = 0; q < kP; ++q) {
     const float v = vq(q);
     const float S3 = S + v;
-    const float B3 = B - v;
-    const float L3 = L + aq[q];
-    const float U = fmaf(S3, S3, -L3);
+    const float d2 = Bm - v;
+    const float U = fmaf(S3, S3, -(L + aq[q]));
+    float y[kP];
 #pragma unroll
-    for (int p = 0; p < kP; ++p) cand(S3, U, B3, vp(q, p), t2[p], cc[p], acc);
+    for (int p = 0; p < kP; ++p) y[p] = fmaf(S3, t2[p], cp(q, p));
+    const float z = fmaxf(fmaxf(fmaxf(y[0], y[1]), y[2]), fmaxf(y[3], y[4])) + U;
+    acc &= __float_as_uint(z) | __float_as_uint(d2);
   }
   return (acc >> 31) ^ 1u;  // 1 if some candidate of the block may win
 }
@@ -939,15 +945,15 @@ __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, u
     build_tables<KS>(c, T);
     const float Bl = c.blim;
     if constexpr (KS == 2) {
-      pend = block_qp(T.a[0], T.t2, T.cc, 0.f, 0.f, Bl, [&](int q) { return T.vf[0][0][q]; },
-                      [&](int q, int p) { return T.vf[1][p == q][p]; });
+      pend = block_qp(T.a[0], T.t2, 0.f, 0.f, Bl - T.vmin, [&](int q) { return T.vf[0][0][q]; },
+                      [&](int q, int p) { return T.ccv[p == q][p]; });
     } else {
 #pragma unroll
       for (int d0 = 0; d0 < kP; ++d0) {
         const float v0 = T.vf[0][0][d0];
-        pend |= block_qp(T.a[1], T.t2, T.cc, v0, T.a[0][d0], Bl - v0,
+        pend |= block_qp(T.a[1], T.t2, v0, T.a[0][d0], (Bl - v0) - T.vmin,
                          [&](int q) { return T.vf[1][q == d0][q]; },
-                         [&](int q, int p) { return T.vf[2][(p == d0) + (p == q)][p]; })
+                         [&](int q, int p) { return T.ccv[(p == d0) + (p == q)][p]; })
                 << d0;
       }
     }
@@ -2366,6 +2372,236 @@ cudaError_t run_int_peak(int sms, double* ops, double* seconds) {
   // 3 ops per chain step; IADD3 with an immediate counts 1, LOP3 1, IMAD 1
   *ops = (double)blocks * 256.0 * kPeakIters * 4 * 8 * 3 / (ms * 1e-3);
   *seconds = ms * 1e-3;
+  return cudaGetLastError();
+}
+
+// ====================================================================================
+// K11 (NEXT-1): DAG stages (R40-R43)
+// ====================================================================================
+// One warp per request; lane l takes the function's mask-table entries l, l+32, ...
+// (unit-cut masks in candidate order with their first candidate index) and scores every
+// stage-option combination of its mask exactly in integers: stage times from the prefix
+// rows of the table image (one slice: the run's component range; split: per branch, max),
+// memory per slice, the throughput floor, free slices as a SWAR byte compare against the
+// node's clamped counts (a plan holds <= 8 slices, so the clamp at 8 is exact), SLO,
+// cvq = floor(1024 (k Q - T^2) / T^2) in u64 (T < 2^24: every stage is at most its
+// one-slice sum).  Warp argmin of the packed keys; the winning lane writes and binds.
+constexpr int kDagT = 128;
+
+__device__ __forceinline__ uint32_t dag_lat(const DagArgs& A, uint32_t row0, uint32_t a, uint32_t b, uint32_t p) {
+  return __float2uint_rn(plf(A.image, A.lay.o_pl + (row0 + b) * kRowW + p) - plf(A.image, A.lay.o_pl + (row0 + a) * kRowW + p));
+}
+
+// options of the stage made of units [u0, u1]: P, plus P^nb splits when it is one block
+__device__ __forceinline__ uint32_t dag_nopt(const uint32_t* uo, uint32_t u0, uint32_t u1) {
+  const uint32_t nb = uo[6 * u0];
+  if (u0 != u1 || nb < 2) return kP;
+  uint32_t q = 1;
+  for (uint32_t j = 0; j < nb; ++j) q *= kP;
+  return kP + q;
+}
+
+// Score option o of the stage [u0, u1] (uo = the function's units): adds its time t,
+// GPCs and per-profile slice counts, clears ok on a memory / floor miss; returns t.
+// A split's branch profiles are the base-P digits of o - P, branch 0 most significant
+// (sums and max are order-free, so the digits are taken least significant first).
+__device__ __forceinline__ uint32_t dag_stage(const DagArgs& A, uint32_t row0, const uint32_t* uo, uint32_t u0,
+                                              uint32_t u1, uint32_t o, uint32_t thr, uint32_t& gp, uint64_t& use,
+                                              bool& ok) {
+  const uint32_t* img = A.image;
+  const uint32_t* U0 = uo + 6 * u0;
+  uint32_t t;
+  if (o < (uint32_t)kP) {
+    const uint32_t* U1 = uo + 6 * u1;
+    const uint32_t c0 = U0[1], c1 = U1[1 + U1[0]];  // end of the last branch of unit u1
+    t = dag_lat(A, row0, c0, c1, o);
+    ok &= img[A.lay.o_pm + row0 + c1] - img[A.lay.o_pm + row0 + c0] <= img[A.lay.o_cap + o];
+    gp += img[A.lay.o_gpcs + o];
+    use += 1ull << (8 * o);
+  } else {
+    const uint32_t nb = U0[0];
+    uint32_t w = o - kP;
+    t = 0;
+    for (uint32_t jj = nb; jj > 0; --jj) {
+      const uint32_t j = jj - 1, p = w % kP;
+      w /= kP;
+      const uint32_t c = U0[1 + j], e = U0[2 + j];  // branch j = [end of branch j-1 (or c0), e)
+      t = max(t, dag_lat(A, row0, c, e, p));
+      ok &= img[A.lay.o_pm + row0 + e] - img[A.lay.o_pm + row0 + c] <= img[A.lay.o_cap + p];
+      gp += img[A.lay.o_gpcs + p];
+      use += 1ull << (8 * p);
+    }
+  }
+  ok &= t <= thr;
+  return t;
+}
+
+// stage s of a mask: units [u0, u1] from the packed last units (4 bits per stage)
+__device__ __forceinline__ void dag_bounds(uint32_t ends, uint32_t s, uint32_t& u0, uint32_t& u1) {
+  u1 = (ends >> (4 * s)) & 15u;
+  u0 = s ? ((ends >> (4 * (s - 1))) & 15u) + 1 : 0;
+}
+
+__global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagArgs A) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t r64 = ((uint64_t)blockIdx.x * kDagT + threadIdx.x) >> 5;
+  if (r64 >= A.n_req) return;
+  const uint32_t r = (uint32_t)r64;
+  const ffs_request q = A.req[r];
+  ffs_dag_plan* out = A.out + r;
+  const bool bad = q.func >= A.lay.F || q.node >= A.n_nodes;
+  const uint32_t f = bad ? 0 : q.func, v = bad ? 0 : q.node;
+  const uint32_t row0 = A.image[A.lay.o_fdesc + 4 * f];
+  const uint32_t thr = A.image[A.lay.o_thr + f];
+  const uint32_t B = A.slo[r];
+  const uint64_t nf = A.node_free[v];
+  const uint32_t* uo = A.units + 6 * A.fu[2 * f];
+  const uint32_t m = A.fu[2 * f + 1];
+  const uint32_t* xc = A.xcut + A.fu[2 * f];
+  uint64_t best = kKeyNone, scored = 0, nfeas = 0, ksum = 0;
+  uint32_t best_mk = 0, best_c = 0;
+  const uint32_t e0 = A.mt_off[f], e1 = bad ? e0 : A.mt_off[f + 1];
+  for (uint32_t e = e0 + lane; e < e1; e += 32) {
+    const uint32_t mk = A.mt_mk[e], mask = mk & 0xffffu, k = mk >> 16;
+    const uint64_t idx0 = A.mt_cand[e];
+    // last unit of every stage (4 bits each), cut costs, option counts
+    uint32_t ends = 0, X = 0, st = 0, total = 1;
+    for (uint32_t u = 0; u < m; ++u) {
+      const bool cut = u + 1 < m && ((mask >> u) & 1u);
+      if (cut) X += xc[u];
+      if (u + 1 == m || cut) {
+        ends |= u << (4 * st);
+        ++st;
+      }
+    }
+    for (uint32_t s = 0; s < k; ++s) {
+      uint32_t u0, u1;
+      dag_bounds(ends, s, u0, u1);
+      total *= dag_nopt(uo, u0, u1);  // <= (5 + 5^4)^2 or 30^4: 32 bits (R43 limits)
+    }
+    for (uint32_t c = 0; c < total; ++c) {
+      // mixed-radix digits of c, the last stage fastest (stage 0 most significant)
+      uint64_t T = 0, Q = 0, use = 0;
+      uint32_t gp = 0, rest = c;
+      bool ok = true;
+      for (uint32_t ss = k; ss > 0; --ss) {
+        uint32_t u0, u1;
+        dag_bounds(ends, ss - 1, u0, u1);
+        const uint32_t no = dag_nopt(uo, u0, u1), os = rest % no;
+        rest /= no;
+        const uint64_t t = dag_stage(A, row0, uo, u0, u1, os, thr, gp, use, ok);
+        T += t;
+        Q += t * t;
+      }
+      // every byte: use <= free (both <= 8), SLO inclusive (R8)
+      ok &= (((nf | 0x8080808080808080ull) - use) & 0x8080808080808080ull) == 0x8080808080808080ull;
+      ok &= T + X <= B;
+      if (ok) {
+        const uint64_t D = T * T, N = (uint64_t)k * Q - D;
+        const uint64_t key = (((N << 10) / D) << 50) | ((uint64_t)(k - 1) << 47) | ((uint64_t)gp << 41) | (idx0 + c);
+        ++nfeas;
+        ksum += key;
+        if (key < best) {
+          best = key;
+          best_mk = mk;
+          best_c = c;
+        }
+      }
+    }
+    scored += total;
+  }
+  // warp argmin (keys are unique: idx is embedded) and checksum sums
+  uint64_t wbest = best;
+#pragma unroll
+  for (int d = 16; d; d >>= 1) wbest = min(wbest, (uint64_t)__shfl_xor_sync(0xffffffffu, (unsigned long long)wbest, d));
+  if (A.checks) {
+#pragma unroll
+    for (int d = 16; d; d >>= 1) {
+      scored += __shfl_xor_sync(0xffffffffu, (unsigned long long)scored, d);
+      nfeas += __shfl_xor_sync(0xffffffffu, (unsigned long long)nfeas, d);
+      ksum += __shfl_xor_sync(0xffffffffu, (unsigned long long)ksum, d);
+    }
+    if (lane == 0) {
+      A.checks[3 * (size_t)r] = scored;
+      A.checks[3 * (size_t)r + 1] = nfeas;
+      A.checks[3 * (size_t)r + 2] = ksum;
+    }
+  }
+  const bool writer = wbest == kKeyNone ? lane == 0 : best == wbest;
+  if (!writer) return;
+  ffs_dag_plan P;
+  P.key = (int64_t)wbest;
+  P.status = bad ? FFS_PLAN_BAD_REQ : (wbest == kKeyNone ? FFS_PLAN_INFEASIBLE : FFS_PLAN_OK);
+  P.k = P.cut_mask = P.split_mask = P.e2e_us = P.bottleneck_us = P.gpcs = P.cvq = P.n_slots = P.pad = 0;
+  for (int i = 0; i < FFS_DAG_MAX_SLOTS; ++i) {
+    P.prof[i] = 0xff;
+    P.slice[i] = -1;
+  }
+  if (P.status == FFS_PLAN_OK) {
+    const uint32_t mask = best_mk & 0xffffu, k = best_mk >> 16;
+    P.k = k;
+    P.cut_mask = mask;
+    P.cvq = (uint32_t)(wbest >> 50);
+    uint32_t ends = 0, X = 0, st = 0;
+    for (uint32_t u = 0; u < m; ++u) {
+      const bool cut = u + 1 < m && ((mask >> u) & 1u);
+      if (cut) X += xc[u];
+      if (u + 1 == m || cut) {
+        ends |= u << (4 * st);
+        ++st;
+      }
+    }
+    // the winner's option of every stage: digits of best_c, stage 0 most significant
+    uint32_t div = 1;
+    for (uint32_t s = 1; s < k; ++s) {
+      uint32_t u0, u1;
+      dag_bounds(ends, s, u0, u1);
+      div *= dag_nopt(uo, u0, u1);
+    }
+    uint32_t rest = best_c, e2e = X, bott = 0, g = 0, ns = 0, taken = 0;  // taken: 4-bit count per profile
+    uint64_t use = 0;
+    bool ok = true;
+    for (uint32_t s = 0; s < k; ++s) {
+      uint32_t u0, u1;
+      dag_bounds(ends, s, u0, u1);
+      const uint32_t os = rest / div;
+      rest -= os * div;
+      if (s + 1 < k) {
+        uint32_t a0, a1;
+        dag_bounds(ends, s + 1, a0, a1);
+        div /= dag_nopt(uo, a0, a1);
+      }
+      const uint32_t t = dag_stage(A, row0, uo, u0, u1, os, 0xffffffffu, g, use, ok);
+      e2e += t;
+      bott = max(bott, t);
+      // slots: one slice, or the branches in order (branch 0 = most significant digit)
+      uint32_t nb = 1, w = os, pw = 1;
+      if (os >= (uint32_t)kP) {
+        P.split_mask |= 1u << s;
+        nb = uo[6 * u0];
+        w = os - kP;
+        for (uint32_t j = 1; j < nb; ++j) pw *= kP;
+      }
+      for (uint32_t j = 0; j < nb; ++j, ++ns) {
+        const uint32_t p = os >= (uint32_t)kP ? (w / pw) % kP : os;
+        pw = pw > 1 ? pw / kP : 1;
+        const uint32_t cnt = (taken >> (4 * p)) & 15u;
+        P.prof[ns] = (uint8_t)p;
+        P.slice[ns] = A.free_list[((size_t)v * 8 + p) * 8 + cnt];
+        taken += 1u << (4 * p);
+      }
+    }
+    P.e2e_us = e2e;
+    P.bottleneck_us = bott;
+    P.gpcs = g;
+    P.n_slots = ns;
+  }
+  *out = P;
+}
+
+cudaError_t launch_dag(const DagArgs& a, cudaStream_t st) {
+  const uint64_t threads = (uint64_t)a.n_req * 32;
+  k_plan_dag<<<(unsigned)((threads + kDagT - 1) / kDagT), kDagT, 0, st>>>(a);
   return cudaGetLastError();
 }
 

@@ -28,6 +28,11 @@ PLAN_DTYPE = np.dtype([("key", "<i8"), ("status", "<u4"), ("k", "<u4"), ("cut_ma
                        ("bottleneck_us", "<u4"), ("gpcs", "<u4"), ("cvq", "<u4"), ("prof", "u1", (8,)),
                        ("slice", "<i4", (8,)), ("victim", "<i4")])
 assert PLAN_DTYPE.itemsize == 80
+# ffs_dag_plan (NEXT-1 DAG stages, R40-R43)
+DAG_PLAN_DTYPE = np.dtype([("key", "<i8"), ("status", "<u4"), ("k", "<u4"), ("cut_mask", "<u4"), ("split_mask", "<u4"),
+                           ("e2e_us", "<u4"), ("bottleneck_us", "<u4"), ("gpcs", "<u4"), ("cvq", "<u4"),
+                           ("n_slots", "<u4"), ("pad", "<u4"), ("prof", "u1", (8,)), ("slice", "<i4", (8,))])
+assert DAG_PLAN_DTYPE.itemsize == 88
 
 
 class _Profiles(C.Structure):
@@ -41,6 +46,10 @@ class _Table(C.Structure):
 
 class _Cluster(C.Structure):
     _fields_ = [("n_nodes", C.c_uint32), ("n_slices", C.c_uint32), ("slices", C.c_void_p)]
+
+
+class _DagTable(C.Structure):
+    _fields_ = [("n_funcs", C.c_uint32), ("unit_off", C.c_void_p), ("unit_nb", C.c_void_p), ("unit_bend", C.c_void_p)]
 
 
 class _EvictParams(C.Structure):
@@ -69,6 +78,8 @@ _sig = {
     "ffs_plan_frontier_any": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp], _i32),
     "ffs_rank_partitions": ([_vp, _u32, _u32], _i32),
     "ffs_plan_ranked": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
+    "ffs_dag_stage": ([_vp, C.POINTER(_DagTable), _u32], _i32),
+    "ffs_plan_dag": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp], _i32),
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
     "ffs_segment_times": ([_vp, C.POINTER(C.c_float)], _i32),
     "ffs_debug_filter_misses": ([_vp, C.POINTER(C.c_uint64)], _i32),
@@ -321,6 +332,24 @@ class Planner:
         self._check(_lib.ffs_plan_ranked(self._h, _ptr(req), _ptr(slo), n, _ptr(out), _stream(stream)))
         return out
 
+    # ---- NEXT-1: DAG stages (R40-R43) ---------------------------------------------------------
+    def stage_dag(self, dag, k_max: int) -> None:
+        """Stage the unit structure (workload.DagTable: unit_off, unit_nb, unit_bend[U, 4])."""
+        uo = np.ascontiguousarray(dag.unit_off, dtype=np.uint32)
+        nb = np.ascontiguousarray(dag.unit_nb, dtype=np.uint8)
+        be = np.ascontiguousarray(dag.unit_bend, dtype=np.uint8)
+        t = _DagTable(int(uo.shape[0] - 1), _host(uo), _host(nb), _host(be))
+        self._check(_lib.ffs_dag_stage(self._h, C.byref(t), int(k_max)))
+
+    def plan_dag(self, req, slo, out=None, checks=None, stream=None):
+        """Plans of DAG functions: (R, 88) uint8 device tensor of ffs_dag_plan records."""
+        import torch
+        n = int(slo.numel())
+        if out is None:
+            out = torch.empty((n, DAG_PLAN_DTYPE.itemsize), dtype=torch.uint8, device=slo.device)
+        self._check(_lib.ffs_plan_dag(self._h, _ptr(req), _ptr(slo), n, _ptr(out), _ptr(checks), _stream(stream)))
+        return out
+
     # ---- measurement ---------------------------------------------------------------------
     def int_peak(self) -> tuple[float, float]:
         ops, sec = C.c_double(), C.c_double()
@@ -343,6 +372,12 @@ def plans_to_numpy(plans) -> np.ndarray:
     """View a (R, 80) uint8 tensor/array of ffs_plan records as a PLAN_DTYPE array."""
     a = plans.cpu().numpy() if hasattr(plans, "cpu") else np.asarray(plans)
     return np.ascontiguousarray(a).view(PLAN_DTYPE).reshape(-1)
+
+
+def dag_plans_to_numpy(plans) -> np.ndarray:
+    """View a (R, 88) uint8 tensor/array of ffs_dag_plan records as a DAG_PLAN_DTYPE array."""
+    a = plans.cpu().numpy() if hasattr(plans, "cpu") else np.asarray(plans)
+    return np.ascontiguousarray(a).view(DAG_PLAN_DTYPE).reshape(-1)
 
 
 def to_device(prob, device="cuda"):
