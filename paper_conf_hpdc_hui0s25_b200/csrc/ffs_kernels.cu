@@ -2460,8 +2460,22 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
   const uint32_t* xc = A.xcut + A.fu[2 * f];
   uint64_t best = kKeyNone, scored = 0, nfeas = 0, ksum = 0;
   uint32_t best_mk = 0, best_c = 0;
+  // the request's candidates [0, Tr) in R43 order are cut into 32 contiguous chunks, one
+  // per lane (a lane walks the masks its chunk covers): every lane gets the same number of
+  // candidates whatever the mask sizes
   const uint32_t e0 = A.mt_off[f], e1 = bad ? e0 : A.mt_off[f + 1];
-  for (uint32_t e = e0 + lane; e < e1; e += 32) {
+  const uint64_t Tr = bad ? 0 : A.ftot[f];
+  const uint64_t chunk = (Tr + 31) / 32, cb = min(Tr, chunk * lane), ce = min(Tr, cb + chunk);
+  uint32_t e = e0;
+  if (cb < ce) {  // last entry with mt_cand[e] <= cb (binary search)
+    uint32_t lo = e0, hi = e1 - 1;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi + 1) >> 1;
+      if (A.mt_cand[mid] <= cb) lo = mid; else hi = mid - 1;
+    }
+    e = lo;
+  }
+  for (uint64_t c = cb; c < ce; ++e) {
     const uint32_t mk = A.mt_mk[e], mask = mk & 0xffffu, k = mk >> 16;
     const uint64_t idx0 = A.mt_cand[e];
     // last unit of every stage (4 bits each), cut costs, option counts
@@ -2479,36 +2493,75 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
       dag_bounds(ends, s, u0, u1);
       total *= dag_nopt(uo, u0, u1);  // <= (5 + 5^4)^2 or 30^4: 32 bits (R43 limits)
     }
-    for (uint32_t c = 0; c < total; ++c) {
-      // mixed-radix digits of c, the last stage fastest (stage 0 most significant)
-      uint64_t T = 0, Q = 0, use = 0;
-      uint32_t gp = 0, rest = c;
-      bool ok = true;
-      for (uint32_t ss = k; ss > 0; --ss) {
+    // this lane's part of the mask: combinations [lo, hi)
+    uint32_t lo = (uint32_t)(c - idx0);
+    const uint32_t hi = (uint32_t)min((uint64_t)total, ce - idx0);
+    scored += hi - lo;
+    c = idx0 + hi;
+    // outer stages (0 .. k-2) decoded once per outer combination, the last stage innermost;
+    // the last stage's five one-slice options do not depend on the outer stages: scored
+    // once per mask into registers
+    uint32_t lu0, lu1;
+    dag_bounds(ends, k - 1, lu0, lu1);
+    const uint32_t nl = dag_nopt(uo, lu0, lu1);
+    uint32_t lt[kP], lg[kP];
+    bool lok[kP];
+#pragma unroll
+    for (int o = 0; o < kP; ++o) {
+      uint64_t us = 0;
+      lg[o] = 0;
+      lok[o] = true;
+      lt[o] = dag_stage(A, row0, uo, lu0, lu1, (uint32_t)o, thr, lg[o], us, lok[o]);
+    }
+    uint32_t co = lo / nl, ol0 = lo - co * nl;
+    while (lo < hi) {
+      uint64_t T0 = 0, Q0 = 0, use0 = 0;
+      uint32_t gp0 = 0, rest = co;
+      bool ok0 = true;
+      for (uint32_t ss = k - 1; ss > 0; --ss) {  // digits of co: stage k-2 fastest
         uint32_t u0, u1;
         dag_bounds(ends, ss - 1, u0, u1);
         const uint32_t no = dag_nopt(uo, u0, u1), os = rest % no;
         rest /= no;
-        const uint64_t t = dag_stage(A, row0, uo, u0, u1, os, thr, gp, use, ok);
-        T += t;
-        Q += t * t;
+        const uint64_t t = dag_stage(A, row0, uo, u0, u1, os, thr, gp0, use0, ok0);
+        T0 += t;
+        Q0 += t * t;
       }
-      // every byte: use <= free (both <= 8), SLO inclusive (R8)
-      ok &= (((nf | 0x8080808080808080ull) - use) & 0x8080808080808080ull) == 0x8080808080808080ull;
-      ok &= T + X <= B;
-      if (ok) {
-        const uint64_t D = T * T, N = (uint64_t)k * Q - D;
-        const uint64_t key = (((N << 10) / D) << 50) | ((uint64_t)(k - 1) << 47) | ((uint64_t)gp << 41) | (idx0 + c);
-        ++nfeas;
-        ksum += key;
-        if (key < best) {
-          best = key;
-          best_mk = mk;
-          best_c = c;
+      const uint32_t cbase = co * nl;  // the combination's index, last stage fastest
+      const uint32_t olEnd = min(nl, ol0 + (hi - lo));
+      auto score = [&](uint64_t t, uint32_t gp, uint64_t use, bool ok, uint32_t ol) {
+        const uint64_t T = T0 + t, Q = Q0 + t * t;
+        // every byte: use <= free (both <= 8), SLO inclusive (R8)
+        ok &= (((nf | 0x8080808080808080ull) - use) & 0x8080808080808080ull) == 0x8080808080808080ull;
+        ok &= T + X <= B;
+        if (ok) {
+          const uint64_t D = T * T, N = (uint64_t)k * Q - D;
+          const uint64_t key =
+              (((N << 10) / D) << 50) | ((uint64_t)(k - 1) << 47) | ((uint64_t)gp << 41) | (idx0 + cbase + ol);
+          ++nfeas;
+          ksum += key;
+          if (key < best) {
+            best = key;
+            best_mk = mk;
+            best_c = cbase + ol;
+          }
         }
+      };
+#pragma unroll
+      for (int o = 0; o < kP; ++o)
+        if ((uint32_t)o >= ol0 && (uint32_t)o < olEnd)
+          score(lt[o], gp0 + lg[o], use0 + (1ull << (8 * o)), ok0 && lok[o], (uint32_t)o);
+      for (uint32_t ol = max(ol0, (uint32_t)kP); ol < olEnd; ++ol) {  // splits of a one-block last stage
+        uint64_t use = use0;
+        uint32_t gp = gp0;
+        bool ok = ok0;
+        const uint64_t t = dag_stage(A, row0, uo, lu0, lu1, ol, thr, gp, use, ok);
+        score(t, gp, use, ok, ol);
       }
+      lo += olEnd - ol0;
+      ++co;
+      ol0 = 0;
     }
-    scored += total;
   }
   // warp argmin (keys are unique: idx is embedded) and checksum sums
   uint64_t wbest = best;
