@@ -2024,6 +2024,7 @@ __global__ void __launch_bounds__(kRsT) k_rs_scatter(const uint64_t* __restrict_
     const uint32_t d = in ? (uint32_t)((key[i] >> shift) & 255u) : 256u + lane;
     const uint32_t m = __match_any_sync(0xffffffffu, d);
     if (in && lane == __ffs(m) - 1) wh[w][d] += __popc(m);
+    __syncwarp();  // the next iteration's leader of the same digit may be another lane
   }
   __syncthreads();
   // exclusive prefix over warps per digit, plus the global offset of (digit, block)
