@@ -529,7 +529,10 @@ __device__ __forceinline__ void pair_rescan(SearchState<KS>& c, const Geo<KS>& G
 }
 
 // KS = 3, two consecutive masks per thread in f32x2 lanes, every level unrolled (125
-// candidates per mask, ~8 KB of SASS) and every table in registers.
+// candidates per mask, ~8 KB of SASS) and every table in registers.  Per group (d0, q)
+// the group maximum of §4.3: y_p = fma(S2, 2t_p, ccw_p) (ccw = -INF for an inadmissible
+// last stage), z = max_p y_p + U, and one exact SLO test against the fastest admissible
+// last stage (blim - v2min - S2, integers < 2^25).
 template <bool VERIFY>
 __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint32_t maskB, bool haveB,
                                          unsigned long long* misses) {
@@ -539,9 +542,9 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
   geo<3>(c, maskB, G[1]);
   if (!haveB) G[1].blim = -1.f;
   const float al = c.alpha, one_m_a = 1.f - c.alpha;
-  f2 v0[kP], v1[2][kP], sl2[3][kP], na0[kP], a1[kP], t2[kP], cc[kP];
+  f2 v0[kP], v1[2][kP], ccw[3][kP], na0[kP], a1[kP], t2[kP], slm;
   {
-    float f[2][3][kP];
+    float f[2][3][kP], vmin[2] = {INF, INF};
 #pragma unroll
     for (int h = 0; h < 2; ++h)
 #pragma unroll
@@ -550,24 +553,31 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
     for (int x = 0; x < kP; ++x) {
       const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
       const uint32_t cap = c.sm[c.o_cap + x];
-      float v[2][3][3];
+      float v[2][2][2], cw[2][3], tw[2];
 #pragma unroll
-      for (int h = 0; h < 2; ++h)
+      for (int h = 0; h < 2; ++h) {
 #pragma unroll
-        for (int s = 0; s < 3; ++s)
+        for (int s = 0; s < 2; ++s)
 #pragma unroll
           for (int m = 0; m <= s; ++m)
             v[h][s][m] = (G[h].memst[s] <= cap && f[h][s][x] <= c.thr && fr > (uint32_t)m) ? f[h][s][x] : INF;
+        const bool ad = G[h].memst[2] <= cap && f[h][2][x] <= c.thr;  // the last stage fits x
+        const float ccx = one_m_a * (f[h][2][x] * f[h][2][x]);
+        tw[h] = ad ? f[h][2][x] + f[h][2][x] : 0.f;
+#pragma unroll
+        for (int m = 0; m < 3; ++m) cw[h][m] = (ad && fr > (uint32_t)m) ? ccx : -INF;
+        if (ad && fr > 0) vmin[h] = fminf(vmin[h], f[h][2][x]);
+      }
       v0[x] = f2pack(v[0][0][0], v[1][0][0]);
       v1[0][x] = f2pack(v[0][1][0], v[1][1][0]);
       v1[1][x] = f2pack(v[0][1][1], v[1][1][1]);
 #pragma unroll
-      for (int m = 0; m < 3; ++m) sl2[m][x] = f2pack(G[0].blim - v[0][2][m], G[1].blim - v[1][2][m]);
+      for (int m = 0; m < 3; ++m) ccw[m][x] = f2pack(cw[0][m], cw[1][m]);
       na0[x] = f2pack(-al * (f[0][0][x] * f[0][0][x]), -al * (f[1][0][x] * f[1][0][x]));
       a1[x] = f2pack(al * (f[0][1][x] * f[0][1][x]), al * (f[1][1][x] * f[1][1][x]));
-      t2[x] = f2pack(f[0][2][x] + f[0][2][x], f[1][2][x] + f[1][2][x]);
-      cc[x] = f2pack(one_m_a * (f[0][2][x] * f[0][2][x]), one_m_a * (f[1][2][x] * f[1][2][x]));
+      t2[x] = f2pack(tw[0], tw[1]);
     }
+    slm = f2pack(G[0].blim - vmin[0], G[1].blim - vmin[1]);  // exact (integers < 2^25 or -INF)
   }
   uint32_t pendA = 0, pendB = 0;
 #pragma unroll
@@ -577,18 +587,24 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
 #pragma unroll
     for (int q = 0; q < kP; ++q) {
       const f2 S2 = f2add(S1, v1[q == d0][q]);
-      const f2 NL2 = f2sub(NL1, a1[q]);
-      const f2 U = f2fma(S2, S2, NL2);
+      const f2 U = f2fma(S2, S2, f2sub(NL1, a1[q]));
+      float ylo[kP], yhi[kP];
 #pragma unroll
       for (int p = 0; p < kP; ++p) {
-        const f2 z = f2add(f2fma(S2, t2[p], cc[p]), U);
-        const f2 d2 = f2sub(sl2[(p == d0) + (p == q)][p], S2);
-        uint32_t zl, zh, dl, dh;
-        f2bits(z, zl, zh);
-        f2bits(d2, dl, dh);
-        accA &= zl | dl;
-        accB &= zh | dh;
+        uint32_t l, h;
+        f2bits(f2fma(S2, t2[p], ccw[(p == d0) + (p == q)][p]), l, h);
+        ylo[p] = __uint_as_float(l);
+        yhi[p] = __uint_as_float(h);
       }
+      const float mlo = fmaxf(fmaxf(fmaxf(ylo[0], ylo[1]), ylo[2]), fmaxf(ylo[3], ylo[4]));
+      const float mhi = fmaxf(fmaxf(fmaxf(yhi[0], yhi[1]), yhi[2]), fmaxf(yhi[3], yhi[4]));
+      const f2 z = f2add(f2pack(mlo, mhi), U);
+      const f2 d2 = f2sub(slm, S2);  // sign set <=> S2 + v2min > blim: no candidate meets the SLO
+      uint32_t zl, zh, dl, dh;
+      f2bits(z, zl, zh);
+      f2bits(d2, dl, dh);
+      accA &= zl | dl;
+      accB &= zh | dh;
     }
     pendA |= ((accA >> 31) ^ 1u) << d0;
     pendB |= ((accB >> 31) ^ 1u) << d0;
