@@ -2459,6 +2459,7 @@ __device__ __forceinline__ void dag_bounds(uint32_t ends, uint32_t s, uint32_t& 
   u0 = s ? ((ends >> (4 * (s - 1))) & 15u) + 1 : 0;
 }
 
+template <bool VERIFY>
 __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagArgs A) {
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t r64 = ((uint64_t)blockIdx.x * kDagT + threadIdx.x) >> 5;
@@ -2553,10 +2554,16 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         ok &= T + X <= B;
         if (ok) {
           const uint64_t D = T * T, N = (uint64_t)k * Q - D;
+          // production: a candidate whose cvq exceeds the running best's cannot win --
+          // decided by one multiply (cvq >= c + 1 <=> 1024 N >= (c + 1) D, < 2^62) before
+          // the 64-bit division (verify mode sums every feasible key)
+          if (!VERIFY && best != kKeyNone && (N << 10) >= ((best >> 50) + 1) * D) return;
           const uint64_t key =
               (((N << 10) / D) << 50) | ((uint64_t)(k - 1) << 47) | ((uint64_t)gp << 41) | (idx0 + cbase + ol);
-          ++nfeas;
-          ksum += key;
+          if (VERIFY) {
+            ++nfeas;
+            ksum += key;
+          }
           if (key < best) {
             best = key;
             best_mk = mk;
@@ -2584,7 +2591,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
   uint64_t wbest = best;
 #pragma unroll
   for (int d = 16; d; d >>= 1) wbest = min(wbest, (uint64_t)__shfl_xor_sync(0xffffffffu, (unsigned long long)wbest, d));
-  if (A.checks) {
+  if (VERIFY) {
 #pragma unroll
     for (int d = 16; d; d >>= 1) {
       scored += __shfl_xor_sync(0xffffffffu, (unsigned long long)scored, d);
@@ -2671,7 +2678,10 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
 
 cudaError_t launch_dag(const DagArgs& a, cudaStream_t st) {
   const uint64_t threads = (uint64_t)a.n_req * 32;
-  k_plan_dag<<<(unsigned)((threads + kDagT - 1) / kDagT), kDagT, 0, st>>>(a);
+  if (a.checks)
+    k_plan_dag<true><<<(unsigned)((threads + kDagT - 1) / kDagT), kDagT, 0, st>>>(a);
+  else
+    k_plan_dag<false><<<(unsigned)((threads + kDagT - 1) / kDagT), kDagT, 0, st>>>(a);
   return cudaGetLastError();
 }
 

@@ -29,13 +29,17 @@ def planner(F):
 
 
 def run_dag(F, planner, prob, dag, k_max=None):
+    """Verify mode (checksums) and production mode (cvq pre-test before the division):
+    both must give the same plans."""
     k_max = prob.k_max if k_max is None else k_max
     planner.stage(prob)
     planner.stage_dag(dag, k_max)
     req, slo = F.to_device(prob)
     checks = torch.zeros((prob.R, 3), dtype=torch.int64, device="cuda")
     out = planner.plan_dag(req, slo, checks=checks)
+    prod = planner.plan_dag(req, slo)
     torch.cuda.synchronize()
+    assert torch.equal(out, prod), "production and verify mode differ"
     return F.dag_plans_to_numpy(out), checks.cpu().numpy().view(np.uint64)
 
 
