@@ -78,7 +78,7 @@ struct ffs_ctx {
   // NEXT-1 ranked partitions
   DevBuf rank_off, rank_mask;
   // NEXT-1 DAG stages
-  DevBuf dag_fu, dag_units, dag_xcut, dag_mt_off, dag_mt_mk, dag_mt_cand, dag_ftot;
+  DevBuf dag_fu, dag_units, dag_xcut, dag_mt_off, dag_mt_mk, dag_mt_cand;
   bool dag_staged = false;
   bool ranked = false;
   uint32_t rank_kmax = 0, prof_order = 0;
@@ -169,7 +169,7 @@ void ffs_destroy(ffs_ctx* c) {
     for (DevBuf* b : {&c->node_off, &c->j_keys, &c->j_state, &c->j_dirty, &c->j_sreq, &c->j_sslo, &c->j_skeys,
                       &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
       b->release();
-    for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand, &c->dag_ftot,
+    for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand,
                       &c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr})
       b->release();
@@ -745,7 +745,7 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
   // per function: unit-cut masks in candidate order (k ascending, masks ascending) with
   // the first candidate index of each (R43)
   std::vector<uint32_t> mt_off(F + 1, 0), mt_mk;
-  std::vector<unsigned long long> mt_cand, ftot(F);
+  std::vector<unsigned long long> mt_cand;
   for (uint32_t f = 0; f < F; ++f) {
     const uint32_t m = fu[2 * f + 1], ub = fu[2 * f];
     uint64_t cand = 0;
@@ -772,7 +772,6 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
         if (cand >= (1ull << kIdxBits)) return fail(c, FFS_ERR_RANGE, "function %u: >= 2^41 DAG candidates", f);
       }
     mt_off[f + 1] = (uint32_t)mt_mk.size();
-    ftot[f] = cand;
   }
   DeviceGuard g(c->device);
   auto up = [&](DevBuf& b, const void* src, size_t bytes) -> cudaError_t {
@@ -786,7 +785,6 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
   CK(up(c->dag_mt_off, mt_off.data(), mt_off.size() * 4), "upload dag_mt_off");
   CK(up(c->dag_mt_mk, mt_mk.data(), mt_mk.size() * 4), "upload dag_mt_mk");
   CK(up(c->dag_mt_cand, mt_cand.data(), mt_cand.size() * 8), "upload dag_mt_cand");
-  CK(up(c->dag_ftot, ftot.data(), ftot.size() * 8), "upload dag_ftot");
   c->dag_staged = true;
   return FFS_OK;
 }
@@ -813,7 +811,6 @@ ffs_status ffs_plan_dag(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_
   a.mt_off = c->dag_mt_off.as<uint32_t>();
   a.mt_mk = c->dag_mt_mk.as<uint32_t>();
   a.mt_cand = c->dag_mt_cand.as<unsigned long long>();
-  a.ftot = c->dag_ftot.as<unsigned long long>();
   a.out = d_out;
   a.checks = reinterpret_cast<unsigned long long*>(d_checksums);
   CK(launch_dag(a, (cudaStream_t)stream), "dag kernel");

@@ -141,7 +141,6 @@ struct DagArgs {
   const uint32_t* mt_off;     // [F+1] mask-table entries of f
   const uint32_t* mt_mk;      // unit-cut mask | k << 16
   const unsigned long long* mt_cand;  // first candidate index of the entry
-  const unsigned long long* ftot;     // [F] candidates of the function
   ffs_dag_plan* out;
   unsigned long long* checks; // [n_req][3] or null
 };

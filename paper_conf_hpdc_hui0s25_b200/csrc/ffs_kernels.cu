@@ -2478,22 +2478,15 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
   const uint32_t* xc = A.xcut + A.fu[2 * f];
   uint64_t best = kKeyNone, scored = 0, nfeas = 0, ksum = 0;
   uint32_t best_mk = 0, best_c = 0;
-  // the request's candidates [0, Tr) in R43 order are cut into 32 contiguous chunks, one
-  // per lane (a lane walks the masks its chunk covers): every lane gets the same number of
-  // candidates whatever the mask sizes
+  uint32_t gpc[kP];
+#pragma unroll
+  for (int x = 0; x < kP; ++x) gpc[x] = A.image[A.lay.o_gpcs + x];
+  // The warp walks the function's masks together (uniform control flow: k, the stage
+  // bounds and option counts are the same on every lane); within a mask the lanes split
+  // the outer combinations (stages 0 .. k-2), and each lane scores the last stage's
+  // options for its outer combination from per-mask tables.
   const uint32_t e0 = A.mt_off[f], e1 = bad ? e0 : A.mt_off[f + 1];
-  const uint64_t Tr = bad ? 0 : A.ftot[f];
-  const uint64_t chunk = (Tr + 31) / 32, cb = min(Tr, chunk * lane), ce = min(Tr, cb + chunk);
-  uint32_t e = e0;
-  if (cb < ce) {  // last entry with mt_cand[e] <= cb (binary search)
-    uint32_t lo = e0, hi = e1 - 1;
-    while (lo < hi) {
-      const uint32_t mid = (lo + hi + 1) >> 1;
-      if (A.mt_cand[mid] <= cb) lo = mid; else hi = mid - 1;
-    }
-    e = lo;
-  }
-  for (uint64_t c = cb; c < ce; ++e) {
+  for (uint32_t e = e0; e < e1; ++e) {
     const uint32_t mk = A.mt_mk[e], mask = mk & 0xffffu, k = mk >> 16;
     const uint64_t idx0 = A.mt_cand[e];
     // last unit of every stage (4 bits each), cut costs, option counts
@@ -2511,17 +2504,12 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
       dag_bounds(ends, s, u0, u1);
       total *= dag_nopt(uo, u0, u1);  // <= (5 + 5^4)^2 or 30^4: 32 bits (R43 limits)
     }
-    // this lane's part of the mask: combinations [lo, hi)
-    uint32_t lo = (uint32_t)(c - idx0);
-    const uint32_t hi = (uint32_t)min((uint64_t)total, ce - idx0);
-    scored += hi - lo;
-    c = idx0 + hi;
-    // outer stages (0 .. k-2) decoded once per outer combination, the last stage innermost;
-    // the last stage's five one-slice options do not depend on the outer stages: scored
-    // once per mask into registers
+    if (lane == 0) scored += total;
     uint32_t lu0, lu1;
     dag_bounds(ends, k - 1, lu0, lu1);
-    const uint32_t nl = dag_nopt(uo, lu0, lu1);
+    const uint32_t nl = dag_nopt(uo, lu0, lu1), nouter = total / nl;
+    // the last stage's one-slice options, and for a two-branch last block each branch's
+    // time and memory fit per profile (a split option is then a max of two table reads)
     uint32_t lt[kP], lg[kP];
     bool lok[kP];
 #pragma unroll
@@ -2531,8 +2519,21 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
       lok[o] = true;
       lt[o] = dag_stage(A, row0, uo, lu0, lu1, (uint32_t)o, thr, lg[o], us, lok[o]);
     }
-    uint32_t co = lo / nl, ol0 = lo - co * nl;
-    while (lo < hi) {
+    const bool split2 = nl == kP + kP * kP;
+    uint32_t bt[2][kP], bok = 0;
+    if (split2) {
+      const uint32_t* U = uo + 6 * lu0;
+#pragma unroll
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int x = 0; x < kP; ++x) {
+          const uint32_t cb0 = U[1 + j], ce0 = U[2 + j];
+          bt[j][x] = dag_lat(A, row0, cb0, ce0, x);
+          if (A.image[A.lay.o_pm + row0 + ce0] - A.image[A.lay.o_pm + row0 + cb0] <= A.image[A.lay.o_cap + x])
+            bok |= 1u << (5 * j + x);
+        }
+    }
+    for (uint32_t co = lane; co < nouter; co += 32) {
       uint64_t T0 = 0, Q0 = 0, use0 = 0;
       uint32_t gp0 = 0, rest = co;
       bool ok0 = true;
@@ -2545,8 +2546,11 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         T0 += t;
         Q0 += t * t;
       }
+      // the outer stages alone already miss memory, the floor, the free slices or the SLO:
+      // no last stage can repair that (times and slice counts only grow)
+      ok0 &= (((nf | 0x8080808080808080ull) - use0) & 0x8080808080808080ull) == 0x8080808080808080ull;
+      if (!ok0 || T0 + X > B) continue;
       const uint32_t cbase = co * nl;  // the combination's index, last stage fastest
-      const uint32_t olEnd = min(nl, ol0 + (hi - lo));
       auto score = [&](uint64_t t, uint32_t gp, uint64_t use, bool ok, uint32_t ol) {
         const uint64_t T = T0 + t, Q = Q0 + t * t;
         // every byte: use <= free (both <= 8), SLO inclusive (R8)
@@ -2572,19 +2576,26 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         }
       };
 #pragma unroll
-      for (int o = 0; o < kP; ++o)
-        if ((uint32_t)o >= ol0 && (uint32_t)o < olEnd)
-          score(lt[o], gp0 + lg[o], use0 + (1ull << (8 * o)), ok0 && lok[o], (uint32_t)o);
-      for (uint32_t ol = max(ol0, (uint32_t)kP); ol < olEnd; ++ol) {  // splits of a one-block last stage
-        uint64_t use = use0;
-        uint32_t gp = gp0;
-        bool ok = ok0;
-        const uint64_t t = dag_stage(A, row0, uo, lu0, lu1, ol, thr, gp, use, ok);
-        score(t, gp, use, ok, ol);
+      for (int o = 0; o < kP; ++o) score(lt[o], gp0 + lg[o], use0 + (1ull << (8 * o)), lok[o], (uint32_t)o);
+      if (split2) {  // splits of a two-branch last block (option kP + 5 p0 + p1)
+#pragma unroll
+        for (int p0 = 0; p0 < kP; ++p0)
+#pragma unroll
+          for (int p1 = 0; p1 < kP; ++p1) {
+            const uint32_t t = max(bt[0][p0], bt[1][p1]);
+            const bool ok = ((bok >> p0) & (bok >> (5 + p1)) & 1u) && t <= thr;
+            score(t, gp0 + gpc[p0] + gpc[p1], use0 + (1ull << (8 * p0)) + (1ull << (8 * p1)), ok,
+                  (uint32_t)(kP + kP * p0 + p1));
+          }
+      } else {
+        for (uint32_t ol = kP; ol < nl; ++ol) {  // splits of a one-block last stage (3-4 branches)
+          uint64_t use = use0;
+          uint32_t gp = gp0;
+          bool ok = true;
+          const uint64_t t = dag_stage(A, row0, uo, lu0, lu1, ol, thr, gp, use, ok);
+          score(t, gp, use, ok, ol);
+        }
       }
-      lo += olEnd - ol0;
-      ++co;
-      ol0 = 0;
     }
   }
   // warp argmin (keys are unique: idx is embedded) and checksum sums
