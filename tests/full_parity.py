@@ -3,7 +3,8 @@
 field.  Writes gpurun_out/full_parity_<cfg>.json.  One-off evidence run (C5 takes ~40 min of
 oracle time on 16 host cores); the sampled versions are in tests/test_gpu_parity.py.
 
-    python tools/full_parity.py 3 5
+    python tests/full_parity.py 3 5   (test infrastructure: the only place besides the test suite
+    that runs the oracle at full size)
 """
 import json
 import os
