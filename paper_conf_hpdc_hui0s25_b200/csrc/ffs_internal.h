@@ -90,7 +90,10 @@ struct DecodeArgs {
 };
 
 // launchers (ffs_kernels.cu)
-constexpr int kDyn = 8;  // search chunks per warp and rank (dynamic grab, k_plan_search)
+#ifndef FFS_KDYN
+#define FFS_KDYN 32  // 8: C5 KS4 41.8 ms, 32: 40.7 (smaller tail of the dynamic grab), 64: 40.5 but a slower step
+#endif
+constexpr int kDyn = FFS_KDYN;  // search chunks per warp and rank (dynamic grab, k_plan_search)
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
