@@ -94,6 +94,10 @@ struct DecodeArgs {
 #define FFS_KDYN 32  // 8: C5 KS4 41.8 ms, 32: 40.7 (smaller tail of the dynamic grab), 64: 40.5 but a slower step
 #endif
 constexpr int kDyn = FFS_KDYN;  // search chunks per warp and rank (dynamic grab, k_plan_search)
+#ifndef FFS_KDYN4
+#define FFS_KDYN4 64  // C5 KS4: 40.58 ms at 32, 40.45 at 64, 40.62 at 128
+#endif
+constexpr int kDyn4 = FFS_KDYN4;  // the same for the KS = 4 segment
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
