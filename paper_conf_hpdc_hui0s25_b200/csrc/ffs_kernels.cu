@@ -1546,9 +1546,15 @@ __device__ __forceinline__ void evict_one(const ffs_instance& in, uint32_t i, ui
   state[gi] = st;
 }
 
-// one CTA per tick; 4 records in flight per thread (memory-level parallelism).  (A flat
+// one CTA per tick; kEvU records in flight per thread (memory-level parallelism).  (A flat
 // persistent grid with a per-record binary search of the tick measured 1.7x slower.)
-constexpr int kEvT = 128, kEvU = 4;
+#ifndef FFS_EVT
+#define FFS_EVT 128
+#endif
+#ifndef FFS_EVU
+#define FFS_EVU 5  // 640 >= the ~582 instances of a C4 tick: one round of loads per CTA (0.545 -> 0.567 of the copy peak)
+#endif
+constexpr int kEvT = FFS_EVT, kEvU = FFS_EVU;
 __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __restrict__ inst,
                                                        const uint32_t* __restrict__ tick_off,
                                                        const uint64_t* __restrict__ now_us, ffs_evict_params prm,
