@@ -332,9 +332,10 @@ typedef struct {
  * k_max * max branches * max gpcs >= 64, >= 2^41 candidates for a function.
  * FFS_ERR_STATE: tables not staged (staging new tables drops the DAG). */
 ffs_status ffs_dag_stage(ffs_ctx *ctx, const ffs_dag_table *dag, uint32_t k_max);
-/* Plan every request against its home node's free slices: one warp per request, lanes
- * over the function's unit-cut masks, every candidate scored exactly in integers, warp
- * argmin; the winning lane writes the plan and binds its slices.  d_checksums (nullable):
+/* Plan every request against its home node's free slices: one warp per request walking
+ * the function's unit-cut masks together, lanes over each mask's stage-option
+ * combinations, every candidate scored exactly in integers, warp argmin; the winning lane
+ * writes the plan and binds its slices (R11).  d_checksums (nullable; verify mode):
  * uint64[3*n_req] = candidates scored, feasible, sum of feasible keys mod 2^64.
  * Asynchronous on `stream`.  FFS_ERR_STATE: no DAG staged. */
 ffs_status ffs_plan_dag(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
