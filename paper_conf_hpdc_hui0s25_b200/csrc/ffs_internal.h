@@ -90,14 +90,11 @@ struct DecodeArgs {
 };
 
 // launchers (ffs_kernels.cu)
-#ifndef FFS_KDYN
-#define FFS_KDYN 32  // 8: C5 KS4 41.8 ms, 32: 40.7 (smaller tail of the dynamic grab), 64: 40.5 but a slower step
-#endif
-constexpr int kDyn = FFS_KDYN;  // search chunks per warp and rank (dynamic grab, k_plan_search)
-#ifndef FFS_KDYN4
-#define FFS_KDYN4 64  // C5 KS4: 40.58 ms at 32, 40.45 at 64, 40.62 at 128
-#endif
-constexpr int kDyn4 = FFS_KDYN4;  // the same for the KS = 4 segment
+// search chunks per warp and rank (dynamic grab, k_plan_search), per stage count: more
+// chunks shorten the tail of the grab, each costs a request lookup.  Measured on C5 (ms of
+// the KS = 1 / 2 / 3 / 4 segments): 1: 0.04 / 1.01 / - / -, 8: 0.06 / 0.92 / 3.14 / 41.8,
+// 16: - / - / 3.04 / -, 32: 0.18 / 0.88 / 3.14 / 40.6, 64: - / - / - / 40.45.
+__host__ __device__ constexpr int kdyn(int ks) { return ks == 1 ? 1 : ks == 2 ? 32 : ks == 3 ? 16 : ks == 4 ? 64 : 32; }
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,

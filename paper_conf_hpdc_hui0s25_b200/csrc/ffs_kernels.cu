@@ -1064,7 +1064,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
 
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint64_t T = pre[A.n_req];
-  // Work split: the segment's task list is cut into NC = world x (nthr/32) x kDyn chunks
+  // Work split: the segment's task list is cut into NC = world x (nthr/32) x kdyn(KS) chunks
   // of 32 equal contiguous pieces (one per lane).  Rank `rank` owns chunks
   // j * world + rank; its warps grab them dynamically (atomic counter, zeroed by the count
   // kernel), so a warp whose pieces are cheap (skipped stage-0 profiles, no rescans) takes
@@ -1074,7 +1074,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   // same nthr on every rank (same kernel and device type).  DESIGN.md §4.3, §7.
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
-  const uint64_t NC = (nthr >> 5) * (KS == 4 ? kDyn4 : kDyn) * A.world, NT = NC * 32;
+  const uint64_t NC = (nthr >> 5) * kdyn(KS) * A.world, NT = NC * 32;
   const uint64_t Tq = T / NT, Tr = T % NT;  // piece u = [Tq u + Tr u / NT, ...): no overflow
   auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
   unsigned long long* ctr = A.work_ctr + KS;
