@@ -468,7 +468,19 @@ def main():
     # issue-limited op rate of the packed f16x2 datapath the KS = 4 filter runs on: one
     # warp-instruction per SMSP per clock, 32 lanes, two 16-bit operations per lane
     peak_ops = sm_count * 4 * 32 * 2 * max_mhz * 1e6
-    achieved = seg_c[top - 1] * ALG_OPS / (top_ms * 1e-3)
+    # algorithmic work the kernel actually scored: for KS = 4, the stage-0 iterations the
+    # pre-filter evaluated (125 candidate pairs = 250 candidate slots each; iterations the
+    # exact stage-0 SLO bound skipped are not counted -- their candidates are decided
+    # infeasible without being scored); other segments score every candidate
+    # Every cut mask (task) of the segment is decided by the mask bound first: KS - 1 transfer
+    # adds and one compare = KS integer ops per mask (counted as one op each although each
+    # takes a full lane-issue of the packed peak: conservative)
+    seg_cov = float(seg_c[top - 1])
+    scored = seg_cov
+    if top == 4:
+        scored = float(pl.ks4_evaluated()) * 250.0  # counter of the last (identical) step
+    seg_tasks = seg_cov / float(P ** top)
+    achieved = (scored * ALG_OPS + seg_tasks * top) / (top_ms * 1e-3)
     traffic = _traffic(f"k_plan_search<{top}>")
 
     # e2e through the public host-buffer API (N = 1: ffs_plan_batch_host)
@@ -537,6 +549,8 @@ def main():
                          "unit": "ops/s (packed f16x2: 2 per lane-issue)", "frac": achieved / peak_ops,
                          "traffic": traffic,
                          "alg_ops_per_candidate": ALG_OPS, "kernel_ms": top_ms,
+                         "candidates_covered_per_launch": seg_cov, "candidates_scored_per_launch": scored,
+                         "masks_per_launch": seg_tasks, "alg_ops_per_mask": top,
                          "kernel_share_of_step": top_ms / (ms / args.steps),
                          "peak_source": f"{sm_count} SMs x 4 SMSP x 32 lanes x 2 (f16x2) x {max_mhz:.0f} MHz "
                                         f"(MEASURED_PEAKS.json sm_max_mhz)"},

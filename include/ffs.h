@@ -421,6 +421,12 @@ ffs_status ffs_segment_times(ffs_ctx *ctx, float *ms /* [8] */);
  * rejected although their exact key would have beaten the running minimum (verify mode
  * only; must be 0).  Synchronous. */
 ffs_status ffs_debug_filter_misses(ffs_ctx *ctx, uint64_t *out);
+/* Number of stage-0 iterations (one iteration = 125 candidate pairs, two masks x 125
+ * profile sequences) that the KS = 4 f16x2 pre-filter scored in the last ffs_plan_keys /
+ * ffs_plan_keys_range call on this context; iterations skipped by the exact stage-0 SLO
+ * bound are not counted.  Measurement only (the roofline's executed work).
+ * *out = 0 before the first call.  Synchronous. */
+ffs_status ffs_debug_ks4_evaluated(ffs_ctx *ctx, uint64_t *out);
 
 #ifdef __cplusplus
 }

@@ -414,13 +414,13 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   // keys and checksums are initialised by the first segment only; later ranges continue
   // from (and prune against) whatever the caller combined into d_keys in between
   const bool init = k_first == 1;
-  CK(c->work_ctr.ensure((kMaxK + 1) * 8), "cudaMalloc(work_ctr)");
+  CK(c->work_ctr.ensure((kMaxK + 2) * 8), "cudaMalloc(work_ctr)");
   const uint64_t* nf = node_free ? node_free : c->node_free.as<uint64_t>();
   const bool skip_full = d_checks == nullptr;  // verify mode enumerates every request
   if (!init && c->pre_req == d_req && c->pre_n == n_req && c->pre_kmax == k_max && c->pre_nf == nf &&
       c->pre_skip == skip_full) {
     // continuation of the same batch: the task prefix is still valid; reset the counters
-    CK(cudaMemsetAsync(c->work_ctr.p, 0, (kMaxK + 1) * 8, st), "reset chunk counters");
+    CK(cudaMemsetAsync(c->work_ctr.p, 0, (kMaxK + 2) * 8, st), "reset chunk counters");
   } else {
     CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, nf, skip_full,
                           c->prefix.as<uint64_t>(), c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
@@ -1169,6 +1169,16 @@ ffs_status ffs_segment_times(ffs_ctx* c, float* ms) {
     CK(cudaEventSynchronize(c->ev[k]), "event sync");
     CK(cudaEventElapsedTime(&ms[k - 1], c->evs[k], c->ev[k]), "event time");
   }
+  return FFS_OK;
+}
+
+ffs_status ffs_debug_ks4_evaluated(ffs_ctx* c, uint64_t* out) {
+  if (!c || !out) return FFS_ERR_ARG;
+  *out = 0;
+  if (!c->work_ctr.p) return FFS_OK;
+  DeviceGuard g(c->device);
+  CK(cudaDeviceSynchronize(), "sync");
+  CK(cudaMemcpy(out, c->work_ctr.as<unsigned long long>() + kMaxK + 1, 8, cudaMemcpyDeviceToHost), "read count");
   return FFS_OK;
 }
 

@@ -42,7 +42,7 @@ __global__ void k_count_tasks(const ffs_request* __restrict__ req, const uint32_
                               uint64_t* __restrict__ prefix, int64_t* __restrict__ keys,
                               unsigned long long* __restrict__ checks, unsigned long long* __restrict__ work_ctr) {
   uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r <= (uint32_t)kMaxK) work_ctr[r] = 0;  // the search segments' chunk counters
+  if (r <= (uint32_t)kMaxK + 1) work_ctr[r] = 0;  // chunk counters + the KS = 4 evaluated-iteration count
   if (r > n_req) return;
   uint32_t n = 0;
   if (r < n_req) {
@@ -169,6 +169,7 @@ struct SearchState {
   int64_t best;
   float alpha;        // scale of sum t^2 in the balance filter
   float alpha_h;      // the same with the wider margin of the f16x2 pre-filter (KS = 4)
+  uint32_t n_eval;    // KS = 4: stage-0 iterations the pre-filter evaluated (not bound-skipped)
   float tmin, tmax;   // KS = 4: sum over the chain of the min / max component latency over
                       // all profiles (bounds of every candidate's T, for the f16 scale)
   bool none_can_win;  // best's cvq/k already unbeatable by any KS-stage candidate
@@ -438,6 +439,10 @@ __device__ __forceinline__ uint32_t block_qp(const float (&aq)[kP], const float 
 // control decision (loops, multiplicities) and differ only in data, so one packed
 // instruction scores a candidate of each: per candidate pair FFMA2 + FADD2 + FADD2 on
 // the FMA pipe and two LOP3 on the ALU pipe.
+// stage-0 SLO bound of the KS = 3 / KS = 4 cores; 0 = only the +INF skip (KS = 4)
+#ifndef FFS_D0_BOUND
+#define FFS_D0_BOUND 1
+#endif
 typedef unsigned long long f2;
 __device__ __forceinline__ f2 f2pack(float lo, float hi) {
   f2 r;
@@ -579,10 +584,30 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
     }
     slm = f2pack(G[0].blim - vmin[0], G[1].blim - vmin[1]);  // exact (integers < 2^25 or -INF)
   }
+  // fastest admissible stage 1 per half (the unshifted window; a shifted entry is the same
+  // value or +INF), for the stage-0 bound below
+  float v1lo = INF, v1hi = INF;
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    uint32_t l, h;
+    f2bits(v1[0][x], l, h);
+    v1lo = fminf(v1lo, __uint_as_float(l));
+    v1hi = fminf(v1hi, __uint_as_float(h));
+  }
+  const f2 v1min = f2pack(v1lo, v1hi);
   uint32_t pendA = 0, pendB = 0;
 #pragma unroll
   for (int d0 = 0; d0 < kP; ++d0) {
     const f2 S1 = v0[d0], NL1 = na0[d0];
+#if FFS_D0_BOUND
+    {  // stage-0 bound: every group has S2 >= S1 + v1min (monotone fp32
+       // rounding) and its SLO test d2 = slm - S2 is monotone in S2, so when slm -
+       // (S1 + v1min) < 0 in every live half the iteration can flag nothing
+      uint32_t bl, bh;
+      f2bits(f2sub(slm, f2add(S1, v1min)), bl, bh);
+      if ((bl >> 31) && (!haveB || (bh >> 31))) continue;
+    }
+#endif
     uint32_t accA = ~0u, accB = ~0u;
 #pragma unroll
     for (int q = 0; q < kP; ++q) {
@@ -778,6 +803,12 @@ __device__ __forceinline__ h2 h2max(h2 a, h2 b) {
   return d;
 }
 
+__device__ __forceinline__ h2 h2min(h2 a, h2 b) {
+  h2 d;
+  asm("min.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
+
 // SLO slack in "guarded" form for the integer SWAR test of the inner loop: per f16 half,
 // bit 15 (guard) | the magnitude bits of slack - v3 when it is >= 0, else the guard alone
 // (magnitude 0).  For S3 >= 0 (a sum of non-negative f16, never NaN), the 32-bit integer
@@ -842,6 +873,8 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   h2 a1[kP], a2[kP], t2[kP];
   // fastest admissible last stage per half (memory, floor, >= 1 free slice of the profile)
   float v3min[2] = {INF, INF};
+  // fastest admissible stage 1 / stage 2 per half (>= 1 free slice), for the d0 bound
+  h2 v1min = kInf2, v2min = kInf2;
 #pragma unroll
   for (int x = 0; x < kP; ++x) {
     const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
@@ -875,6 +908,10 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     //   [v1[0], v1[1], v2[0], v2[1], v2[2], cc3[0..3], v0[0], -alpha t0^2]
     // (cc3[k]: the last stage's cc when the node has > k free slices of x, else -INF)
     h2* r = rows + (x * 11) * nb + tid;
+    if (fr > 0) {
+      v1min = h2min(v1min, p1);
+      v2min = h2min(v2min, p2);
+    }
     r[0 * nb] = fr > 0 ? p1 : kInf2;
     r[1 * nb] = fr > 1 ? p1 : kInf2;
     r[2 * nb] = fr > 0 ? p2 : kInf2;
@@ -896,6 +933,20 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
 #pragma unroll 1
 #endif
   for (int d0 = 0; d0 < kP; ++d0) {
+    // d0 bound: every group of the iteration has S3 = (S1 + w1) + w2 >= (S1 + v1min) +
+    // v2min (f16 addition rounds monotonically, and a window entry is its profile's value
+    // or +INF), and the group SLO test below is monotone in S3, so when the bound already
+    // fails it in every live half the iteration can flag nothing: skip it.  This covers a
+    // stage-0 profile with no free slice on the node (S1 = +INF; on C5 the large profiles
+    // are fully busy on most nodes) and stage-0 prefixes that leave too little budget.
+    const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
+#if FFS_D0_BOUND
+    const uint32_t okb = isub(slk, h2add(h2add(S1, v1min), v2min), zero);
+    if (!(okb & 0x8000u) && (!haveB || !(okb & 0x80000000u))) continue;
+#else
+    if ((S1 & 0xffffu) == 0x7c00u && (!haveB || (S1 >> 16) == 0x7c00u)) continue;
+#endif
+    ++c.n_eval;  // 125 candidate pairs scored by the pre-filter
     WinH W[kP];
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
@@ -908,7 +959,6 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
       W[x].c3[1] = r[6 * nb];
       W[x].c3[2] = r[7 * nb];
     }
-    const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
     const h2 NL1 = rows[(d0 * 11 + 10) * nb + tid];  // -alpha t0^2
     uint32_t mm[kP];  // per d1: sign bits 15 / 31 clear <=> the (d0, d1) block may hold a winner
 #pragma unroll
@@ -1080,6 +1130,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   unsigned long long* ctr = A.work_ctr + KS;
 
   SearchState<KS> c;
+  c.n_eval = 0;
   c.sm = tbl;
   c.o_pl = A.lay.o_pl;
   c.o_pm = A.lay.o_pm;
@@ -1208,6 +1259,10 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   }
   flush();
   }  // grab loop
+  if constexpr (KS == 4) {  // measurement: evaluated stage-0 iterations (ffs_debug_ks4_evaluated)
+    const unsigned long long e = __reduce_add_sync(0xffffffffu, c.n_eval);
+    if ((threadIdx.x & 31) == 0 && e) atomicAdd(A.work_ctr + kMaxK + 1, e);
+  }
 }
 
 template <int KS, bool V, bool TG>

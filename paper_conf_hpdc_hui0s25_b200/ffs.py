@@ -83,6 +83,7 @@ _sig = {
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
     "ffs_segment_times": ([_vp, C.POINTER(C.c_float)], _i32),
     "ffs_debug_filter_misses": ([_vp, C.POINTER(C.c_uint64)], _i32),
+    "ffs_debug_ks4_evaluated": ([_vp, C.POINTER(C.c_uint64)], _i32),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_lib, _name)
@@ -361,6 +362,13 @@ class Planner:
         ms = (C.c_float * 8)()
         self._check(_lib.ffs_segment_times(self._h, ms))
         return [float(x) for x in ms]
+
+    def ks4_evaluated(self) -> int:
+        """Stage-0 iterations (125 candidate pairs each) the KS = 4 pre-filter scored in the
+        last plan_keys call (bound-skipped iterations excluded)."""
+        v = C.c_uint64()
+        self._check(_lib.ffs_debug_ks4_evaluated(self._h, C.byref(v)))
+        return int(v.value)
 
     def filter_misses(self) -> int:
         v = C.c_uint64()

@@ -191,6 +191,13 @@ def test_c5_bench_configuration_sampled(F, planner):
     ok = p["status"] == 0
     assert (p["key"][~ok] == np.iinfo(np.int64).max).all()
     assert (p["e2e_us"][ok] <= prob.slo_us[ok]).all()
+    # the KS = 4 pre-filter's stage-0 SLO bound skips work on C5 (large
+    # profiles busy on most nodes): evaluated iterations lie in (0, 5 x KS = 4 masks]
+    from math import comb
+    n = prob.chain_len()[prob.req["func"]]
+    masks = sum(comb(int(m) - 1, 3) for m in n if m >= 4)
+    ev = planner.ks4_evaluated()
+    assert 0 < ev <= 5 * masks
 
 
 def test_bad_requests_and_empty(F, planner):
