@@ -870,7 +870,8 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   }
   constexpr h2 kInf2 = 0x7c007c00u, kNegInf2 = 0xfc00fc00u, kGuard = 0x80008000u;
   const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
-  h2 a1[kP], a2[kP], t2[kP];
+  // pass 1: the packed stage tables and the per-half minima the stage-0 bound needs
+  h2 P0[kP], P1[kP], P2[kP], P3[kP];
   // fastest admissible last stage per half (memory, floor, >= 1 free slice of the profile)
   float v3min[2] = {INF, INF};
   // fastest admissible stage 1 / stage 2 per half (>= 1 free slice), for the d0 bound
@@ -888,30 +889,61 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     // the stage tables in packed f16 (the squares and alpha products too: two more f16
     // roundings per entry, inside the margin of DESIGN.md §4.3); a memory-infeasible
     // stage is INF everywhere, which only an SLO-rejected candidate can see
-    const h2 p0 = h2pack(vm[0][0], vm[1][0]), p1 = h2pack(vm[0][1], vm[1][1]), p2 = h2pack(vm[0][2], vm[1][2]);
+    P0[x] = h2pack(vm[0][0], vm[1][0]);
+    P1[x] = h2pack(vm[0][1], vm[1][1]);
+    P2[x] = h2pack(vm[0][2], vm[1][2]);
     // a last stage longer than the (widened) SLO slack on its own is inadmissible too: no
     // candidate holding it is feasible, and the bound keeps t3 and t3^2 far from overflow
+    // (an admissible t3 sigma <= slack < 33 never packs to the f16 INF pattern)
     const float u0 = vm[0][3] <= slack[0] ? vm[0][3] : INF, u1 = vm[1][3] <= slack[1] ? vm[1][3] : INF;
-    const h2 p3 = h2pack(u0, u1);
+    P3[x] = h2pack(u0, u1);
     if (fr > 0) {
       v3min[0] = fminf(v3min[0], u0);
       v3min[1] = fminf(v3min[1], u1);
+      v1min = h2min(v1min, P1[x]);
+      v2min = h2min(v2min, P2[x]);
     }
+  }
+  // guarded SLO slack of the fastest admissible last stage (h2guard): S3 <= slack - v3min
+  const uint32_t slk = h2guard(h2pack(slack[0] - v3min[0], slack[1] - v3min[1]));
+  // d0 bound: every group of stage-0 iteration d0 has S3 = (S1 + w1) + w2 >= (S1 + v1min)
+  // + v2min (f16 addition rounds monotonically, and a window entry is its profile's value
+  // or +INF), and the group SLO test is monotone in S3, so when the bound already fails it
+  // in every live half the iteration can flag nothing: it is skipped.  This covers a
+  // stage-0 profile with no free slice on the node (S1 = +INF; on C5 the large profiles
+  // are fully busy on most nodes) and stage-0 prefixes that leave too little budget.
+  uint32_t live = 0;
+#pragma unroll
+  for (int d0 = 0; d0 < kP; ++d0) {
+    const h2 S1 = ((c.freeb >> (8 * d0)) & 255u) ? P0[d0] : kInf2;
+#if FFS_D0_BOUND
+    const uint32_t okb = isub(slk, h2add(h2add(S1, v1min), v2min), zero);
+    const bool on = (okb & 0x8000u) || (haveB && (okb & 0x80000000u));
+#else
+    const bool on = (S1 & 0xffffu) != 0x7c00u || (haveB && (S1 >> 16) != 0x7c00u);
+#endif
+    live |= (on ? 1u : 0u) << d0;
+  }
+  // no live iteration (the common case on C5): the windows are never read, so the rest of
+  // the setup is skipped too (verify mode and too-wide halves still rescan exactly below)
+  if (!VERIFY && live == 0 && !wide[0] && !wide[1]) return;
+  // pass 2: the per-thread windows and the register tables of the scoring core
+  h2 a1[kP], a2[kP], t2[kP];
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const h2 p0 = P0[x], p1 = P1[x], p2 = P2[x], p3 = P3[x];
     a1[x] = h2mul(h2mul(p1, p1), al2);
     a2[x] = h2mul(h2mul(p2, p2), al2);
     // last stage as (2 t3, (1 - alpha_h) t3^2); an inadmissible one (INF) as (0, -INF), so
     // its score y = S3 * 2t3 + cc is -INF for every finite S3 (no INF * 0, no INF - INF)
-    const uint32_t inf3 = (u0 == INF ? 0x0000ffffu : 0u) | (u1 == INF ? 0xffff0000u : 0u);
+    const uint32_t inf3 = ((p3 & 0xffffu) == 0x7c00u ? 0x0000ffffu : 0u) | ((p3 >> 16) == 0x7c00u ? 0xffff0000u : 0u);
     t2[x] = h2add(p3, p3) & ~inf3;
     const h2 cc = (h2mul(h2mul(p3, p3), oma2) & ~inf3) | (kNegInf2 & inf3);
     const h2 na0 = h2mul(h2mul(p0, p0), nal2);
     //   [v1[0], v1[1], v2[0], v2[1], v2[2], cc3[0..3], v0[0], -alpha t0^2]
     // (cc3[k]: the last stage's cc when the node has > k free slices of x, else -INF)
     h2* r = rows + (x * 11) * nb + tid;
-    if (fr > 0) {
-      v1min = h2min(v1min, p1);
-      v2min = h2min(v2min, p2);
-    }
     r[0 * nb] = fr > 0 ? p1 : kInf2;
     r[1 * nb] = fr > 1 ? p1 : kInf2;
     r[2 * nb] = fr > 0 ? p2 : kInf2;
@@ -924,8 +956,6 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     r[9 * nb] = fr > 0 ? p0 : kInf2;
     r[10 * nb] = na0;
   }
-  // guarded SLO slack of the fastest admissible last stage (h2guard): S3 <= slack - v3min
-  const uint32_t slk = h2guard(h2pack(slack[0] - v3min[0], slack[1] - v3min[1]));
   uint32_t pendA = 0, pendB = 0;
 #if FFS_UNROLL_D0
 #pragma unroll
@@ -933,19 +963,8 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
 #pragma unroll 1
 #endif
   for (int d0 = 0; d0 < kP; ++d0) {
-    // d0 bound: every group of the iteration has S3 = (S1 + w1) + w2 >= (S1 + v1min) +
-    // v2min (f16 addition rounds monotonically, and a window entry is its profile's value
-    // or +INF), and the group SLO test below is monotone in S3, so when the bound already
-    // fails it in every live half the iteration can flag nothing: skip it.  This covers a
-    // stage-0 profile with no free slice on the node (S1 = +INF; on C5 the large profiles
-    // are fully busy on most nodes) and stage-0 prefixes that leave too little budget.
+    if (!((live >> d0) & 1u)) continue;
     const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
-#if FFS_D0_BOUND
-    const uint32_t okb = isub(slk, h2add(h2add(S1, v1min), v2min), zero);
-    if (!(okb & 0x8000u) && (!haveB || !(okb & 0x80000000u))) continue;
-#else
-    if ((S1 & 0xffffu) == 0x7c00u && (!haveB || (S1 >> 16) == 0x7c00u)) continue;
-#endif
     ++c.n_eval;  // 125 candidate pairs scored by the pre-filter
     WinH W[kP];
 #pragma unroll
