@@ -53,6 +53,10 @@ typedef enum {
 #define FFS_MAX_CHAIN 32
 #define FFS_KEY_NONE INT64_MAX
 
+/* search modes (ffs_set_search_mode) */
+#define FFS_SEARCH_BOUNDED 0u    /* default: exact SLO lower bounds skip candidates that cannot be feasible */
+#define FFS_SEARCH_EXHAUSTIVE 1u /* every candidate of every request is scored ("all possible partitions") */
+
 /* per-plan status (an infeasible request is not an error) */
 #define FFS_PLAN_OK 0u
 #define FFS_PLAN_INFEASIBLE 1u
@@ -169,10 +173,23 @@ const char *ffs_last_error(const ffs_ctx *ctx);
 ffs_status ffs_stage_tables(ffs_ctx *ctx, const ffs_profiles *profiles, const ffs_profile_table *table,
                             const ffs_cluster *cluster);
 
+/* ---- search mode ------------------------------------------------------------------------
+ * FFS_SEARCH_BOUNDED (default): the search skips candidates that an exact integer lower
+ * bound of their end-to-end latency proves infeasible (SLO) -- identical keys,
+ * much less work.  FFS_SEARCH_EXHAUSTIVE: every candidate of every request (including
+ * requests on a node without a free slice, R37) has its own score computed, "all
+ * possible partitions"; the measured throughput of this mode is the benchmark's
+ * candidates-scored/s.  Both modes return bit-identical keys and plans.  FFS_ERR_ARG for
+ * another value.  Applies to every later search call on the context. */
+ffs_status ffs_set_search_mode(ffs_ctx *ctx, uint32_t mode);
+
 /* ---- A1-A5: keys ---------------------------------------------------------------------
- * Partial argmin keys of shard `rank` of `world` (0 <= rank < world): for every k the
- * flattened (request, cut mask) task list is split into `world` equal contiguous ranges
- * and this call scores every candidate of range `rank`.  d_keys[r] receives the minimum
+ * Partial argmin keys of shard `rank` of `world` (0 <= rank < world).  For every k the
+ * flattened (request, cut mask) task list is cut into world x (search warps) x c chunks
+ * of 32 equal contiguous pieces; shard `rank` owns the chunks j with j mod world = rank
+ * (chunk interleave, DESIGN.md §4.3/§7) and decides every candidate of its chunks
+ * (scored, or in bounded mode possibly proved infeasible by the exact SLO bound).
+ * d_keys[r] receives the minimum
  * feasible key of request r within the shard, FFS_KEY_NONE where none (overwritten, not
  * combined with its previous content).  Combine shards with an element-wise MIN
  * (torch.distributed.all_reduce(keys, MIN) over NCCL) before ffs_plan_decode.
@@ -192,10 +209,9 @@ ffs_status ffs_plan_keys(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t 
  * (heavier) segments against the best key of ALL shards of the earlier ones, exactly as
  * one GPU does, which keeps the shards equal in work.  The result after
  * the last range and a final MIN is the same as ffs_plan_keys.  Checksums stay per-shard
- * sums; reduce them with SUM once at the end.  A continuation (k_first > 1) with the same
- * d_req, n_req and k_max as the previous search call on this context reuses that call's
- * task prefix: the request batch must not change in between.  FFS_ERR_RANGE: bad segment
- * range, or as ffs_plan_keys.  Asynchronous on `stream`. */
+ * sums; reduce them with SUM once at the end.  Every call recomputes its task prefix from
+ * d_req (no state is carried between calls besides d_keys / d_checksums).  FFS_ERR_RANGE:
+ * bad segment range, or as ffs_plan_keys.  Asynchronous on `stream`. */
 ffs_status ffs_plan_keys_range(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, uint32_t n_req,
                                uint32_t k_max, uint32_t k_first, uint32_t k_last, uint32_t rank, uint32_t world,
                                int64_t *d_keys, uint64_t *d_checksums, void *stream);
@@ -229,16 +245,20 @@ ffs_status ffs_plan_batch_host(ffs_ctx *ctx, const ffs_request *h_req, const uin
  *   slice < 0 (not resident)                               -> WARM
  *   PIPELINE flag, or busy_us*100 >= util_thr_pct*window_us -> EXCL_HOT
  *   otherwise                                              -> TIME_SHARING
- * d_score[i] = (last_used_us << 20) | i for a TIME_SHARING instance without the BUSY
- * flag (the LRU key), FFS_KEY_NONE otherwise.  d_state[i] = FFS_ST_*.
- * FFS_ERR_RANGE: n_inst > 2^20.  (last_used_us >= 2^43 scores FFS_KEY_NONE.)  Async. */
+ * d_score[i] = ((cold_after_us - idle) << 20) | i for a TIME_SHARING instance without the
+ * BUSY flag, FFS_KEY_NONE otherwise: the LRU key -- the smallest score is the
+ * instance with the largest idle time (least recently used), ties to the lower index
+ * (R20c).  A time-sharing instance has idle < cold_after_us, so the key is exact for any
+ * timestamp epoch (e.g. Unix microseconds).  d_state[i] = FFS_ST_*.
+ * FFS_ERR_RANGE: n_inst > 2^20, params->cold_after_us >= 2^43.  Async. */
 ffs_status ffs_evict_scores(ffs_ctx *ctx, const ffs_instance *d_inst, uint32_t n_inst, uint64_t now_us,
                             const ffs_evict_params *params, int64_t *d_score, uint8_t *d_state, void *stream);
 
 /* Batched over n_ticks snapshots: tick t owns instances d_tick_off[t] .. d_tick_off[t+1]-1
  * (device array, n_ticks+1 entries, non-decreasing) at time d_now_us[t]; the index in the
  * score is the index within the tick.  An instance at index >= 2^20 within its tick
- * scores FFS_KEY_NONE.  Async. */
+ * scores FFS_KEY_NONE (ticks are device data; the caller keeps ticks below 2^20
+ * instances).  FFS_ERR_RANGE: params->cold_after_us >= 2^43.  Async. */
 ffs_status ffs_evict_scores_ticks(ffs_ctx *ctx, const ffs_instance *d_inst, const uint32_t *d_tick_off,
                                   const uint64_t *d_now_us, uint32_t n_ticks, const ffs_evict_params *params,
                                   int64_t *d_score, uint8_t *d_state, void *stream);
@@ -410,8 +430,14 @@ ffs_status ffs_plan_frontier_any(ffs_ctx *ctx, const ffs_request *d_req, const u
 
 /* ---- measurement / debug helpers ------------------------------------------------------
  * K5: integer issue-rate microbenchmark over all SMs; *ops_per_s = measured lane-ops/s of
- * an IADD3/LOP3/IMAD mix, *clock_khz = SM clock reported during the run.  Synchronous. */
+ * an IADD3/LOP3/IMAD mix (8 independent chains, 2048 threads per SM), *seconds = the
+ * timed launch's duration.  Synchronous. */
 ffs_status ffs_bench_int_peak(ffs_ctx *ctx, double *ops_per_s, double *seconds);
+/* Packed f16x2 microbenchmark over all SMs (roofline denominator of the KS = 4 pre-filter):
+ * mode 0 = HFMA2 chains only (FMA-pipe rate), mode 1 = HFMA2 interleaved 1:1 with packed
+ * max and LOP3 (ALU pipe): the issue-limited rate.  *lane_instr_per_s = measured
+ * lane-instructions per second (each acts on two 16-bit halves).  Synchronous. */
+ffs_status ffs_bench_packed_peak(ffs_ctx *ctx, uint32_t mode, double *lane_instr_per_s, double *seconds);
 /* Device time (ms, CUDA events recorded on the launch stream around each launch) of each
  * search-kernel segment run since the last ffs_plan_keys / ffs_plan_keys_range call with
  * k_first = 1 on this context: ms[ks-1] for ks = 1..8 stages, 0 where no segment ran.
@@ -421,12 +447,12 @@ ffs_status ffs_segment_times(ffs_ctx *ctx, float *ms /* [8] */);
  * rejected although their exact key would have beaten the running minimum (verify mode
  * only; must be 0).  Synchronous. */
 ffs_status ffs_debug_filter_misses(ffs_ctx *ctx, uint64_t *out);
-/* Number of stage-0 iterations (one iteration = 125 candidate pairs, two masks x 125
- * profile sequences) that the KS = 4 f16x2 pre-filter scored in the last ffs_plan_keys /
- * ffs_plan_keys_range call on this context; iterations skipped by the exact stage-0 SLO
- * bound are not counted.  Measurement only (the roofline's executed work).
- * *out = 0 before the first call.  Synchronous. */
-ffs_status ffs_debug_ks4_evaluated(ffs_ctx *ctx, uint64_t *out);
+/* Candidates whose own score the search kernels computed in the last ffs_plan_keys /
+ * ffs_plan_keys_range call on this context, per stage count: per_ks[ks-1], ks = 1..8
+ * (device counters; in FFS_SEARCH_EXHAUSTIVE mode the sum over ks equals
+ * sum_r S(n_r, k_max) of the shard; candidates the bounded mode proves infeasible without
+ * scoring are not counted).  Synchronises the device.  Zeros before the first call. */
+ffs_status ffs_search_scored(ffs_ctx *ctx, uint64_t *per_ks /* [8] */);
 
 #ifdef __cplusplus
 }

@@ -17,6 +17,7 @@ import subprocess
 import threading
 
 import numpy as np
+from typing import NamedTuple
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "ffs_oracle.c")
@@ -267,28 +268,38 @@ def sim(trace, thr_pct: int = 30, cold_after_us: int = 600_000_000):
     return ctr, fs, fst, fl, fb
 
 
+class Evict(NamedTuple):
+    """One snapshot's keep-alive states and LRU order (no packed key): the least recently
+    used evictable instance is the one with the largest idle time, ties to the lower index."""
+    state: np.ndarray      # uint8 FFS_ST_*
+    evictable: np.ndarray  # bool
+    idle: np.ndarray       # uint64 now - last_used (0 for a future last use)
+
+
 def evict(inst: np.ndarray, now_us: int, util_thr_pct: int = 30, window_us: int = 10_000_000,
-          cold_after_us: int = 600_000_000):
-    """Eviction state + LRU score of one snapshot (ffs_oracle.c: oracle_evict)."""
+          cold_after_us: int = 600_000_000) -> Evict:
+    """Eviction state + LRU order of one snapshot (ffs_oracle.c: oracle_evict)."""
     n = int(inst.shape[0])
     sl = _c(inst["slice"], np.int32)
     fl = _c(inst["flags"], np.uint8)
     bu = _c(inst["busy_us"], np.uint32)
     lu = _c(inst["last_used_us"], np.uint64)
-    score = np.zeros(n, np.int64)
     state = np.zeros(n, np.uint8)
+    ev = np.zeros(n, np.uint8)
+    idle = np.zeros(n, np.uint64)
     lib().oracle_evict(C.c_int(n), _p(sl), _p(fl), _p(bu), _p(lu), C.c_uint64(int(now_us)),
                        C.c_uint32(util_thr_pct), C.c_uint32(window_us), C.c_uint64(int(cold_after_us)),
-                       _p(score), _p(state))
-    return score, state
+                       _p(state), _p(ev), _p(idle))
+    return Evict(state, ev.astype(bool), idle)
 
 
-def victim(prob, status: np.ndarray, inst: np.ndarray, score: np.ndarray, k_max: int | None = None) -> np.ndarray:
+def victim(prob, status: np.ndarray, inst: np.ndarray, ev: Evict, k_max: int | None = None) -> np.ndarray:
     """Time-share victim per INFEASIBLE request (ffs_oracle.c: oracle_victim)."""
     h = _Held(prob, int(prob.k_max if k_max is None else k_max), False)
     st = _c(status, np.int32)
     sl = _c(inst["slice"], np.int32)
-    sc = _c(score, np.int64)
+    e = _c(ev.evictable, np.uint8)
+    idle = _c(ev.idle, np.uint64)
     out = np.zeros(h.func.shape[0], np.int32)
-    lib().oracle_victim(C.byref(h.args), _p(st), C.c_int(int(inst.shape[0])), _p(sl), _p(sc), _p(out))
+    lib().oracle_victim(C.byref(h.args), _p(st), C.c_int(int(inst.shape[0])), _p(sl), _p(e), _p(idle), _p(out))
     return out

@@ -348,13 +348,14 @@ int oracle_plan(const oracle_plan_args *a, int n_threads) {
  *   not resident (slice < 0)           -> WARM  (evicted to CPU memory)
  *   pipeline, or busy*100 >= thr*window -> EXCL_HOT (P:358 pipelines; P:370 threshold)
  *   otherwise                          -> TIME_SHARING (utilization below 30%)
- * score = (last_used << 20) | instance index for a resident, idle (not BUSY)
- * time-sharing instance (LRU); every other instance scores INT64_MAX.  The key
- * packs last_used into 43 bits and the index into 20 (R20b): an instance with
- * last_used >= 2^43 or index >= 2^20 cannot be represented and is not evictable. */
+ * evictable[i] = 1 for a resident, idle (not BUSY) time-sharing instance (LRU
+ * eviction among time-sharing instances; exclusive-hot ones are exempt), idle[i] =
+ * now - last_used (0 when last_used is in the future, R20b).  The least recently used
+ * evictable instance is the one with the largest idle time (R20c); no packed key, so any
+ * 64-bit timestamp is representable. */
 void oracle_evict(int n_inst, const int32_t *inst_slice, const uint8_t *inst_flags, const uint32_t *inst_busy_us,
                   const uint64_t *inst_last_used_us, uint64_t now_us, uint32_t util_thr_pct, uint32_t window_us,
-                  uint64_t cold_after_us, int64_t *score, uint8_t *state) {
+                  uint64_t cold_after_us, uint8_t *state, uint8_t *evictable, uint64_t *idle_out) {
     for (int i = 0; i < n_inst; i++) {
         uint64_t last = inst_last_used_us[i];
         uint64_t idle = now_us >= last ? now_us - last : 0;
@@ -369,22 +370,20 @@ void oracle_evict(int n_inst, const int32_t *inst_slice, const uint8_t *inst_fla
         else
             st = ST_TIME_SHARING;
         state[i] = st;
-        if (st == ST_TIME_SHARING && !(inst_flags[i] & FL_BUSY) && last < (1ull << 43) && i < (1 << 20))
-            score[i] = (int64_t)((last << 20) | (uint64_t)i);
-        else
-            score[i] = KEY_NONE;
+        evictable[i] = (st == ST_TIME_SHARING && !(inst_flags[i] & FL_BUSY)) ? 1 : 0;
+        idle_out[i] = idle;
     }
 }
 
 /* Time-share victim for each request whose status is INFEASIBLE: among the
- * instances with a finite score whose slice is in the request's node, whose slice
- * profile holds the whole function (time-sharing instances are non-pipeline) and
- * whose monolithic latency plus the reload time meets the budget ("deadlines
- * subtracted by estimated execution and instance load times"), the one with
- * the smallest score (least recently used).  -1 when there is none or when the
+ * evictable instances whose slice is in the request's node, whose slice profile holds
+ * the whole function (time-sharing instances are non-pipeline) and whose monolithic
+ * latency plus the reload time meets the budget ("deadlines subtracted by estimated
+ * execution and instance load times"), the least recently used one: the largest
+ * idle time, ties to the lower instance index.  -1 when there is none or when the
  * request is not INFEASIBLE. */
 void oracle_victim(const oracle_plan_args *a, const int32_t *status, int n_inst, const int32_t *inst_slice,
-                   const int64_t *score, int32_t *victim) {
+                   const uint8_t *evictable, const uint64_t *idle, int32_t *victim) {
     for (int r = 0; r < a->R; r++) {
         victim[r] = -1;
         if (status[r] != PLAN_INFEASIBLE) continue;
@@ -392,9 +391,10 @@ void oracle_victim(const oracle_plan_args *a, const int32_t *status, int n_inst,
         int n = (int)(a->comp_off[f + 1] - a->comp_off[f]);
         uint64_t mem = 0;
         for (int c = 0; c < n; c++) mem += a->mem_mib[a->comp_off[f] + c];
-        int64_t best = KEY_NONE;
+        int have = 0;
+        uint64_t best = 0;
         for (int i = 0; i < n_inst; i++) {
-            if (score[i] == KEY_NONE) continue;
+            if (!evictable[i]) continue;
             int s = inst_slice[i];
             if (s < 0 || s >= a->n_slices || a->sl_node[s] != v) continue;
             int p = a->sl_prof[s];
@@ -403,8 +403,9 @@ void oracle_victim(const oracle_plan_args *a, const int32_t *status, int n_inst,
             for (int c = 0; c < n; c++) lat += lat_of(a, f, c, p);
             if (lat + a->load_us[f] > a->req_slo_us[r]) continue;
             if (!within_floor(a, f, lat)) continue; /* R38: the monolithic instance meets the floor */
-            if (score[i] < best) {
-                best = score[i];
+            if (!have || idle[i] > best) { /* strictly larger: ties keep the lower index */
+                have = 1;
+                best = idle[i];
                 victim[r] = i;
             }
         }

@@ -7,6 +7,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "ffs_internal.h"
 
 using namespace ffsk;
@@ -90,11 +92,8 @@ struct ffs_ctx {
   // per-segment timing of the last plan_keys call
   cudaEvent_t ev[kMaxK + 1] = {}, evs[kMaxK + 1] = {};  // per segment: end, start
   uint32_t seg_mask = 0;                                 // segments timed since the last k_first = 1
-  // task prefix of the last search call (reused by continuation ranges, k_first > 1)
-  const void* pre_req = nullptr;
-  const void* pre_nf = nullptr;
-  uint32_t pre_n = 0, pre_kmax = 0;
-  bool pre_skip = false;
+  // search mode (ffs_set_search_mode)
+  uint32_t search_mode = FFS_SEARCH_BOUNDED;
 };
 
 static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
@@ -180,7 +179,6 @@ void ffs_destroy(ffs_ctx* c) {
 const char* ffs_last_error(const ffs_ctx* c) { return c ? c->err.c_str() : "null context"; }
 
 ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profile_table* tb, const ffs_cluster* cl) {
-  if (c) c->pre_req = nullptr;  // the task prefix depends on the staged chain lengths
   if (!c) return FFS_ERR_ARG;
   c->staged = false;
   if (!pr || !tb || !cl) return fail(c, FFS_ERR_ARG, "null table pointer");
@@ -414,25 +412,20 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   // keys and checksums are initialised by the first segment only; later ranges continue
   // from (and prune against) whatever the caller combined into d_keys in between
   const bool init = k_first == 1;
-  CK(c->work_ctr.ensure((kMaxK + 2) * 8), "cudaMalloc(work_ctr)");
+  CK(c->work_ctr.ensure(kCtrWords * 8), "cudaMalloc(work_ctr)");
   const uint64_t* nf = node_free ? node_free : c->node_free.as<uint64_t>();
-  const bool skip_full = d_checks == nullptr;  // verify mode enumerates every request
-  if (!init && c->pre_req == d_req && c->pre_n == n_req && c->pre_kmax == k_max && c->pre_nf == nf &&
-      c->pre_skip == skip_full) {
-    // continuation of the same batch: the task prefix is still valid; reset the counters
-    CK(cudaMemsetAsync(c->work_ctr.p, 0, (kMaxK + 2) * 8, st), "reset chunk counters");
-  } else {
-    CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, nf, skip_full,
-                          c->prefix.as<uint64_t>(), c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
-                          init ? reinterpret_cast<unsigned long long*>(d_checks) : nullptr,
-                          c->work_ctr.as<unsigned long long>(), st),
-       "count/scan kernels");
-  }
-  c->pre_req = d_req;
-  c->pre_n = n_req;
-  c->pre_kmax = k_max;
-  c->pre_nf = nf;
-  c->pre_skip = skip_full;
+  const bool exhaustive = c->search_mode == FFS_SEARCH_EXHAUSTIVE;
+  // verify and exhaustive modes enumerate every request, including those whose node has
+  // no free slice (R37); the task prefix is recomputed on every call (a continuation range
+  // k_first > 1 therefore never sees a stale prefix, whatever the caller did to d_req)
+  const bool skip_full = d_checks == nullptr && !exhaustive;
+  nvtxRangePushA("ffs count+scan");
+  CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, nf, skip_full,
+                        c->prefix.as<uint64_t>(), c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
+                        init ? reinterpret_cast<unsigned long long*>(d_checks) : nullptr,
+                        c->work_ctr.as<unsigned long long>(), st),
+     "count/scan kernels");
+  nvtxRangePop();
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows
   // of the KS = 4 kernel (kWin4 B per thread).  The f16x2 kernel's window stride is the
   // compile-time CTA size (immediate LDS/STS offsets); an image that does not fit next to
@@ -469,14 +462,20 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   a.misses = c->misses.as<unsigned long long>();
   a.tables_global = tables_global ? 1u : 0u;
   a.work_ctr = c->work_ctr.as<unsigned long long>();
+  a.exhaustive = exhaustive ? 1u : 0u;
   const bool verify = d_checks != nullptr;
   const uint32_t kk = std::min(k_last, c->max_n);
   if (init) c->seg_mask = 0;
   for (uint32_t k = k_first; k <= kk; ++k) {
     const int grid = c->sms * c->occ[verify ? 1 : 0][k];
+    static const char* kSegName[kMaxK + 1] = {"", "ffs search KS=1", "ffs search KS=2", "ffs search KS=3",
+                                              "ffs search KS=4", "ffs search KS=5", "ffs search KS=6",
+                                              "ffs search KS=7", "ffs search KS=8"};
+    nvtxRangePushA(kSegName[k]);
     CK(cudaEventRecord(c->evs[k], st), "event");
     CK(launch_search((int)k, verify, a, grid, blk((int)k), shm((int)k), st), "search kernel");
     CK(cudaEventRecord(c->ev[k], st), "event");
+    nvtxRangePop();
     c->seg_mask |= 1u << k;
   }
   return FFS_OK;
@@ -553,6 +552,7 @@ ffs_status ffs_evict_scores(ffs_ctx* c, const ffs_instance* d_inst, uint32_t n_i
   if (!c) return FFS_ERR_ARG;
   if (!prm) return fail(c, FFS_ERR_ARG, "null params");
   if (n_inst > (1u << 20)) return fail(c, FFS_ERR_RANGE, "n_inst %u > 2^20", n_inst);
+  if (prm->cold_after_us >= (1ull << 43)) return fail(c, FFS_ERR_RANGE, "cold_after_us >= 2^43");
   if (n_inst == 0) return FFS_OK;
   if (!d_inst || !d_score || !d_state) return fail(c, FFS_ERR_ARG, "null device pointer");
   DeviceGuard g(c->device);
@@ -566,6 +566,7 @@ ffs_status ffs_evict_scores_ticks(ffs_ctx* c, const ffs_instance* d_inst, const 
                                   int64_t* d_score, uint8_t* d_state, void* stream) {
   if (!c) return FFS_ERR_ARG;
   if (!prm) return fail(c, FFS_ERR_ARG, "null params");
+  if (prm->cold_after_us >= (1ull << 43)) return fail(c, FFS_ERR_RANGE, "cold_after_us >= 2^43");
   if (n_ticks == 0) return FFS_OK;
   if (!d_inst || !d_tick_off || !d_now_us || !d_score || !d_state) return fail(c, FFS_ERR_ARG, "null device pointer");
   DeviceGuard g(c->device);
@@ -1172,13 +1173,29 @@ ffs_status ffs_segment_times(ffs_ctx* c, float* ms) {
   return FFS_OK;
 }
 
-ffs_status ffs_debug_ks4_evaluated(ffs_ctx* c, uint64_t* out) {
-  if (!c || !out) return FFS_ERR_ARG;
-  *out = 0;
+ffs_status ffs_set_search_mode(ffs_ctx* c, uint32_t mode) {
+  if (!c) return FFS_ERR_ARG;
+  if (mode != FFS_SEARCH_BOUNDED && mode != FFS_SEARCH_EXHAUSTIVE) return fail(c, FFS_ERR_ARG, "search mode %u", mode);
+  c->search_mode = mode;
+  return FFS_OK;
+}
+
+ffs_status ffs_search_scored(ffs_ctx* c, uint64_t* per_ks) {
+  if (!c || !per_ks) return FFS_ERR_ARG;
+  for (int k = 0; k < kMaxK; ++k) per_ks[k] = 0;
   if (!c->work_ctr.p) return FFS_OK;
   DeviceGuard g(c->device);
   CK(cudaDeviceSynchronize(), "sync");
-  CK(cudaMemcpy(out, c->work_ctr.as<unsigned long long>() + kMaxK + 1, 8, cudaMemcpyDeviceToHost), "read count");
+  unsigned long long w[kCtrWords];
+  CK(cudaMemcpy(w, c->work_ctr.p, sizeof w, cudaMemcpyDeviceToHost), "read counters");
+  for (int k = 1; k <= kMaxK; ++k) per_ks[k - 1] = w[kCtrScored + k];
+  return FFS_OK;
+}
+
+ffs_status ffs_bench_packed_peak(ffs_ctx* c, uint32_t mode, double* lane_instr_per_s, double* seconds) {
+  if (!c || !lane_instr_per_s || !seconds || mode > 1) return FFS_ERR_ARG;
+  DeviceGuard g(c->device);
+  CK(run_packed_peak(c->sms, (int)mode, lane_instr_per_s, seconds), "packed peak kernel");
   return FFS_OK;
 }
 

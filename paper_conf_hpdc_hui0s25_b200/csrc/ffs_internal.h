@@ -69,9 +69,15 @@ struct SearchArgs {
   unsigned long long* checks;   // [n_req][3] or null
   unsigned long long* misses;   // debug counter (verify mode)
   uint32_t tables_global;       // 1: read the image from global memory (too large for smem)
-  unsigned long long* work_ctr; // [kMaxK + 1] chunk counters, zeroed by the count kernel
+  unsigned long long* work_ctr; // [kCtrWords] chunk counters [KS] and scored-candidate
+                                // counters [kCtrScored + KS], zeroed by the count kernel
   uint32_t zero;                // always 0: an operand ptxas cannot fold (ks4_pair_h's IADD3)
+  uint32_t exhaustive;          // FFS_SEARCH_EXHAUSTIVE: no stage-0 SLO bound, every
+                                // candidate of every enumerated mask is scored
 };
+// work_ctr layout: [0..kMaxK] per-KS chunk counters; [kCtrScored + KS] candidates the
+// segment's kernel scored (every candidate whose own score it computed)
+constexpr int kCtrScored = 16, kCtrWords = 32;
 
 struct DecodeArgs {
   const uint32_t* image;
@@ -114,6 +120,7 @@ cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const 
                            uint32_t n_slices, uint32_t n_nodes, unsigned long long* tab, int32_t* victim,
                            cudaStream_t st);
 cudaError_t run_int_peak(int sms, double* ops, double* seconds);
+cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double* seconds);
 
 struct RankedArgs {
   const uint32_t* image;

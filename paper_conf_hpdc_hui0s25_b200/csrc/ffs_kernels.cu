@@ -42,7 +42,7 @@ __global__ void k_count_tasks(const ffs_request* __restrict__ req, const uint32_
                               uint64_t* __restrict__ prefix, int64_t* __restrict__ keys,
                               unsigned long long* __restrict__ checks, unsigned long long* __restrict__ work_ctr) {
   uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r <= (uint32_t)kMaxK + 1) work_ctr[r] = 0;  // chunk counters + the KS = 4 evaluated-iteration count
+  if (r < (uint32_t)kCtrWords) work_ctr[r] = 0;  // chunk counters + scored-candidate counters
   if (r > n_req) return;
   uint32_t n = 0;
   if (r < n_req) {
@@ -169,7 +169,7 @@ struct SearchState {
   int64_t best;
   float alpha;        // scale of sum t^2 in the balance filter
   float alpha_h;      // the same with the wider margin of the f16x2 pre-filter (KS = 4)
-  uint32_t n_eval;    // KS = 4: stage-0 iterations the pre-filter evaluated (not bound-skipped)
+  uint64_t n_scored;  // candidates whose own score this thread computed (measurement)
   float tmin, tmax;   // KS = 4: sum over the chain of the min / max component latency over
                       // all profiles (bounds of every candidate's T, for the f16 scale)
   bool none_can_win;  // best's cvq/k already unbeatable by any KS-stage candidate
@@ -540,7 +540,7 @@ __device__ __forceinline__ void pair_rescan(SearchState<KS>& c, const Geo<KS>& G
 // last stage (blim - v2min - S2, integers < 2^25).
 template <bool VERIFY>
 __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint32_t maskB, bool haveB,
-                                         unsigned long long* misses) {
+                                         unsigned long long* misses, bool exh) {
   const float INF = __int_as_float(0x7f800000);
   Geo<3> G[2];
   geo<3>(c, maskA, G[0]);
@@ -605,9 +605,10 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
        // (S1 + v1min) < 0 in every live half the iteration can flag nothing
       uint32_t bl, bh;
       f2bits(f2sub(slm, f2add(S1, v1min)), bl, bh);
-      if ((bl >> 31) && (!haveB || (bh >> 31))) continue;
+      if (!exh && (bl >> 31) && (!haveB || (bh >> 31))) continue;
     }
 #endif
+    c.n_scored += haveB ? 2 * kP * kP : kP * kP;  // 25 candidates per mask of this d0
     uint32_t accA = ~0u, accB = ~0u;
 #pragma unroll
     for (int q = 0; q < kP; ++q) {
@@ -839,7 +840,7 @@ struct WinH {
 // stored -- half the LDS -- measured 2.6 % slower: more registers and smem.)
 template <bool VERIFY>
 __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
-                                           unsigned long long* misses, uint32_t zero) {
+                                           unsigned long long* misses, uint32_t zero, bool exh) {
   const float INF = __int_as_float(0x7f800000);
   constexpr int nb = search_block(4);  // window stride: the CTA size, fixed at compile time
   const int tid = threadIdx.x;
@@ -924,6 +925,7 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
 #endif
     live |= (on ? 1u : 0u) << d0;
   }
+  if (exh) live = (1u << kP) - 1;  // exhaustive mode: every stage-0 iteration is scored
   // no live iteration (the common case on C5): the windows are never read, so the rest of
   // the setup is skipped too (verify mode and too-wide halves still rescan exactly below)
   if (!VERIFY && live == 0 && !wide[0] && !wide[1]) return;
@@ -965,7 +967,7 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   for (int d0 = 0; d0 < kP; ++d0) {
     if (!((live >> d0) & 1u)) continue;
     const h2 S1 = rows[(d0 * 11 + 9) * nb + tid];
-    ++c.n_eval;  // 125 candidate pairs scored by the pre-filter
+    c.n_scored += haveB ? 250 : 125;  // 125 candidates per mask of this d0, each y_p computed
     WinH W[kP];
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
@@ -1044,6 +1046,7 @@ __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, u
     }
   }
   constexpr int NB = KS == 2 ? 1 : (KS == 3 ? kP : kP * kP);
+  c.n_scored += (KS == 2 ? kP * kP : KS == 3 ? kP * kP * kP : kP * kP * kP * kP);
   const uint32_t all = VERIFY ? ((1u << NB) - 1) : pend;
   for (uint32_t todo = all; todo;) {
     const int b = __ffs(todo) - 1;
@@ -1086,12 +1089,17 @@ __device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, 
     c.blim = c.blim_raw;
     // 5 candidates per request: evaluate them exactly
     c.pd[0] = 0;
+    c.n_scored += kP;
 #pragma unroll
     for (int p = 0; p < kP; ++p) exact_eval<KS, VERIFY>(c, 0, p, true, misses);
   } else {
     load_stage<KS>(c, KS - 2, c.tq, c.sqq);
     load_stage<KS>(c, KS - 1, c.tp, c.sqp);
     set_threshold(c);
+    uint64_t pk = 1;
+#pragma unroll
+    for (int i = 0; i < KS; ++i) pk *= kP;
+    c.n_scored += pk;  // the generic path scores every candidate of the mask
     outer_level<0, KS, VERIFY>(c, 0.f, 0.f, c.free_w, misses);
   }
 }
@@ -1149,7 +1157,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   unsigned long long* ctr = A.work_ctr + KS;
 
   SearchState<KS> c;
-  c.n_eval = 0;
+  c.n_scored = 0;
   c.sm = tbl;
   c.o_pl = A.lay.o_pl;
   c.o_pm = A.lay.o_pm;
@@ -1249,9 +1257,10 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
 #if FFS_KS4_F32
       if constexpr (KS == 4) ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<f2*>(rows), A.misses);
 #else
-      if constexpr (KS == 4) ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero);
+      if constexpr (KS == 4)
+        ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero, A.exhaustive != 0);
 #endif
-      else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses);
+      else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0);
       if (haveB) {
         step = 2;
         mask = maskB;
@@ -1278,9 +1287,11 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   }
   flush();
   }  // grab loop
-  if constexpr (KS == 4) {  // measurement: evaluated stage-0 iterations (ffs_debug_ks4_evaluated)
-    const unsigned long long e = __reduce_add_sync(0xffffffffu, c.n_eval);
-    if ((threadIdx.x & 31) == 0 && e) atomicAdd(A.work_ctr + kMaxK + 1, e);
+  {  // measurement: candidates scored by this warp (ffs_search_scored)
+    uint64_t e = c.n_scored;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+    if ((threadIdx.x & 31) == 0 && e) atomicAdd(A.work_ctr + kCtrScored + KS, (unsigned long long)e);
   }
 }
 
@@ -1614,9 +1625,11 @@ __device__ __forceinline__ void evict_one(const ffs_instance& in, uint32_t i, ui
   else if ((in.flags & FFS_INST_PIPELINE) || (uint64_t)in.busy_us * 100u >= (uint64_t)p.util_thr_pct * p.window_us)
     st = FFS_ST_EXCL_HOT;
   else st = FFS_ST_TIME_SHARING;
-  const bool evictable = st == FFS_ST_TIME_SHARING && !(in.flags & FFS_INST_BUSY) &&
-                         in.last_used_us < (1ull << 43) && i < (1u << 20);
-  score[gi] = evictable ? (int64_t)((in.last_used_us << 20) | i) : (int64_t)kKeyNone;
+  // LRU key (R20c): the least recently used instance has the largest idle time;
+  // a time-sharing instance has idle < cold_after_us < 2^43 (host-checked), so
+  // (cold_after - idle) packs into 43 bits whatever the timestamps' epoch
+  const bool evictable = st == FFS_ST_TIME_SHARING && !(in.flags & FFS_INST_BUSY) && i < (1u << 20);
+  score[gi] = evictable ? (int64_t)(((p.cold_after_us - idle) << 20) | i) : (int64_t)kKeyNone;
   state[gi] = st;
 }
 
@@ -2468,6 +2481,69 @@ cudaError_t run_int_peak(int sms, double* ops, double* seconds) {
   if (e != cudaSuccess) return e;
   // 3 ops per chain step; IADD3 with an immediate counts 1, LOP3 1, IMAD 1
   *ops = (double)blocks * 256.0 * kPeakIters * 4 * 8 * 3 / (ms * 1e-3);
+  *seconds = ms * 1e-3;
+  return cudaGetLastError();
+}
+
+// Packed f16x2 issue-rate microbenchmark (roofline denominator of the KS = 4 pre-filter,
+// DESIGN.md §5).  mode 0: eight independent HFMA2 chains (the FMA-pipe rate of the
+// packed datapath); mode 1: HFMA2 interleaved 1:1 with packed max (VHMNMX) and LOP3 on
+// the ALU pipe -- the issue-limited rate, one warp-instruction per SMSP per clock at best.
+template <int MODE>
+__global__ void __launch_bounds__(256) k_packed_peak(uint32_t seed, uint32_t* out) {
+  uint32_t h[8], m[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    h[i] = 0x3c003c00u ^ ((seed + threadIdx.x + i) & 0x00ff00ffu);
+    m[i] = h[i] ^ 0x04000400u;
+  }
+  const uint32_t a = 0x3bff3bffu ^ (seed & 1u), b = 0x10001000u | (seed & 2u);
+#pragma unroll 1
+  for (int it = 0; it < kPeakIters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        asm volatile("fma.rn.f16x2 %0, %0, %1, %2;" : "+r"(h[i]) : "r"(a), "r"(b));
+        if (MODE == 1) {
+          asm volatile("max.f16x2 %0, %0, %1;" : "+r"(m[i]) : "r"(h[i]));
+          asm volatile("lop3.b32 %0, %0, %1, %2, 0xE8;" : "+r"(m[i]) : "r"(a), "r"(h[(i + 1) & 7]));
+          asm volatile("fma.rn.f16x2 %0, %0, %1, %2;" : "+r"(h[i]) : "r"(a), "r"(b));
+        }
+      }
+    }
+  }
+  uint32_t s = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) s ^= h[i] ^ m[i];
+  if (s == 0x12345678u) out[0] = s;
+}
+
+cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double* seconds) {
+  uint32_t* d = nullptr;
+  cudaError_t e = cudaMalloc(&d, 4);
+  if (e != cudaSuccess) return e;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  const int blocks = sms * 8;  // 2048 threads per SM
+  auto launch = [&](uint32_t seed) {
+    if (mode == 0) k_packed_peak<0><<<blocks, 256>>>(seed, d);
+    else k_packed_peak<1><<<blocks, 256>>>(seed, d);
+  };
+  launch(1u);  // warm-up
+  cudaEventRecord(a);
+  launch(2u);
+  cudaEventRecord(b);
+  e = cudaEventSynchronize(b);
+  float ms = 0;
+  cudaEventElapsedTime(&ms, a, b);
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(d);
+  if (e != cudaSuccess) return e;
+  const double per_step = mode == 0 ? 1.0 : 4.0;  // lane-instructions per chain step
+  *lane_instr_per_s = (double)blocks * 256.0 * kPeakIters * 4 * 8 * per_step / (ms * 1e-3);
   *seconds = ms * 1e-3;
   return cudaGetLastError();
 }

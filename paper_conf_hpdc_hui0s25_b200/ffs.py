@@ -22,6 +22,7 @@ _lib = C.CDLL(LIB_PATH)
 
 FFS_OK, FFS_ERR_ARG, FFS_ERR_RANGE, FFS_ERR_CUDA, FFS_ERR_STATE = 0, -1, -2, -3, -4
 PLAN_OK, PLAN_INFEASIBLE, PLAN_BAD_REQ = 0, 1, 2
+SEARCH_BOUNDED, SEARCH_EXHAUSTIVE = 0, 1
 KEY_NONE = np.iinfo(np.int64).max
 
 PLAN_DTYPE = np.dtype([("key", "<i8"), ("status", "<u4"), ("k", "<u4"), ("cut_mask", "<u4"), ("e2e_us", "<u4"),
@@ -83,7 +84,9 @@ _sig = {
     "ffs_bench_int_peak": ([_vp, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
     "ffs_segment_times": ([_vp, C.POINTER(C.c_float)], _i32),
     "ffs_debug_filter_misses": ([_vp, C.POINTER(C.c_uint64)], _i32),
-    "ffs_debug_ks4_evaluated": ([_vp, C.POINTER(C.c_uint64)], _i32),
+    "ffs_set_search_mode": ([_vp, _u32], _i32),
+    "ffs_search_scored": ([_vp, C.POINTER(C.c_uint64)], _i32),
+    "ffs_bench_packed_peak": ([_vp, _u32, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_lib, _name)
@@ -363,12 +366,22 @@ class Planner:
         self._check(_lib.ffs_segment_times(self._h, ms))
         return [float(x) for x in ms]
 
-    def ks4_evaluated(self) -> int:
-        """Stage-0 iterations (125 candidate pairs each) the KS = 4 pre-filter scored in the
-        last plan_keys call (bound-skipped iterations excluded)."""
-        v = C.c_uint64()
-        self._check(_lib.ffs_debug_ks4_evaluated(self._h, C.byref(v)))
-        return int(v.value)
+    def packed_peak(self, mode: int = 1) -> tuple[float, float]:
+        """(lane-instructions/s, seconds) of the packed f16x2 microbenchmark (0: HFMA2 only,
+        1: HFMA2 interleaved with packed max / LOP3)."""
+        v, sec = C.c_double(), C.c_double()
+        self._check(_lib.ffs_bench_packed_peak(self._h, int(mode), C.byref(v), C.byref(sec)))
+        return v.value, sec.value
+
+    def set_search_mode(self, mode: int) -> None:
+        """SEARCH_BOUNDED (default) or SEARCH_EXHAUSTIVE (every candidate scored)."""
+        self._check(_lib.ffs_set_search_mode(self._h, int(mode)))
+
+    def scored(self) -> list[int]:
+        """Candidates scored per stage count (ks = 1..8) by the last plan_keys call."""
+        v = (C.c_uint64 * 8)()
+        self._check(_lib.ffs_search_scored(self._h, v))
+        return [int(x) for x in v]
 
     def filter_misses(self) -> int:
         v = C.c_uint64()

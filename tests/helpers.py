@@ -129,3 +129,14 @@ def candidate_keys(prob, r, k_max=None):
                 out.append((k, rank, key))
                 idx += 1
     return out
+
+
+def abi_evict_score(ev, cold_after_us: int = 600_000_000) -> np.ndarray:
+    """The ABI's documented LRU key (include/ffs.h, ffs_evict_scores) of an oracle.Evict:
+    ((cold_after_us - idle) << 20) | index for an evictable instance, FFS_KEY_NONE
+    otherwise -- smaller = less recently used, ties to the lower index."""
+    n = len(ev.state)
+    out = np.full(n, KEY_NONE, dtype=np.int64)
+    i = np.flatnonzero(ev.evictable)
+    out[i] = ((np.uint64(cold_after_us) - ev.idle[i].astype(np.uint64)) << np.uint64(20)).astype(np.int64) | i
+    return out

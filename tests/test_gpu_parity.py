@@ -8,7 +8,7 @@ import numpy as np
 import pytest
 
 import oracle
-from helpers import problem
+from helpers import problem, abi_evict_score
 from test_oracle_pins import random_tiny
 from paper_conf_hpdc_hui0s25_b200 import workload as W
 
@@ -196,8 +196,36 @@ def test_c5_bench_configuration_sampled(F, planner):
     from math import comb
     n = prob.chain_len()[prob.req["func"]]
     masks = sum(comb(int(m) - 1, 3) for m in n if m >= 4)
-    ev = planner.ks4_evaluated()
-    assert 0 < ev <= 5 * masks
+    ev = planner.scored()[3]
+    assert 0 < ev <= 625 * masks
+
+
+def test_exhaustive_mode_scores_every_candidate(F, planner):
+    """FFS_SEARCH_EXHAUSTIVE (the benchmark's mode, "all possible partitions"): the
+    device counters see every candidate of every request scored -- sum over ks equals
+    sum_r S(n_r, K), including requests on nodes without a free slice -- and the keys are
+    bit-identical to the bounded mode's (C3, full batch) and to the oracle (sample)."""
+    from math import comb
+    prob = W.config3()
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    K = prob.k_max
+    bounded = planner.plan_keys(req, slo, K).cpu().numpy()
+    try:
+        planner.set_search_mode(F.SEARCH_EXHAUSTIVE)
+        ex = planner.plan_keys(req, slo, K).cpu().numpy()
+        sc = planner.scored()
+    finally:
+        planner.set_search_mode(F.SEARCH_BOUNDED)
+    np.testing.assert_array_equal(ex, bounded)
+    n = prob.chain_len()[prob.req["func"]]
+    per_ks = [sum(comb(int(m) - 1, k - 1) * 5 ** k for m in n if m >= k) for k in range(1, 9)]
+    assert sc[:K] == per_ks[:K] and sum(sc[K:]) == 0
+    idx = np.arange(0, prob.R, 997)
+    o = oracle.plan(prob.subset(idx), checks=False)
+    np.testing.assert_array_equal(ex[idx], o["key"])
+    with pytest.raises(F.FFSError):
+        planner.set_search_mode(7)
 
 
 def test_bad_requests_and_empty(F, planner):
@@ -266,14 +294,35 @@ def test_eviction_scores_and_victims(F, planner):
     score, state, vic = score.cpu().numpy(), state.cpu().numpy(), vic.cpu().numpy()
     for t in range(len(wl.now_us)):
         a, b = int(wl.tick_off[t]), int(wl.tick_off[t + 1])
-        s_o, st_o = oracle.evict(wl.inst[a:b], int(wl.now_us[t]), 30, wl.window_us)
-        np.testing.assert_array_equal(score[a:b], s_o)
-        np.testing.assert_array_equal(state[a:b], st_o)
+        ev = oracle.evict(wl.inst[a:b], int(wl.now_us[t]), 30, wl.window_us)
+        np.testing.assert_array_equal(score[a:b], abi_evict_score(ev))
+        np.testing.assert_array_equal(state[a:b], ev.state)
         rs = np.where(wl.req_tick == t)[0]
         sub = prob.subset(rs)
-        v_o = oracle.victim(sub, np.full(len(rs), oracle.PLAN_INFEASIBLE, np.int32), wl.inst[a:b], s_o)
+        v_o = oracle.victim(sub, np.full(len(rs), oracle.PLAN_INFEASIBLE, np.int32), wl.inst[a:b], ev)
         np.testing.assert_array_equal(vic[rs], v_o)
     assert (vic >= 0).sum() > 0
+
+
+def test_eviction_epoch_timestamps_and_range(F, planner):
+    """Unix-epoch microsecond timestamps (~1.8e15 > 2^43) score like small ones (the LRU key
+    packs cold_after - idle, not the timestamp); a future last use counts as idle 0; a
+    cold_after >= 2^43 (the only unpackable input) is FFS_ERR_RANGE."""
+    wl = W.config4(T=1)
+    planner.stage(wl.problem)
+    base = 1_800_000_000_000_000
+    a = wl.inst.copy()
+    a["last_used_us"] = a["last_used_us"] - int(wl.now_us[0]) + base
+    a["last_used_us"][::11] = base + 5  # in the future
+    inst = torch.from_numpy(a.view(np.uint8)).cuda()
+    score, state = planner.evict_scores(inst, base, window_us=wl.window_us)
+    ev = oracle.evict(a, base, 30, wl.window_us)
+    np.testing.assert_array_equal(score.cpu().numpy(), abi_evict_score(ev))
+    np.testing.assert_array_equal(state.cpu().numpy(), ev.state)
+    assert ev.evictable.sum() > 10
+    with pytest.raises(F.FFSError) as e:
+        planner.evict_scores(inst, base, window_us=wl.window_us, cold_after_us=1 << 43)
+    assert e.value.status == F.FFS_ERR_RANGE
 
 
 def test_victims_table_and_scan_paths_agree(F, planner):
@@ -311,8 +360,8 @@ def test_decode_victims_single_snapshot(F, planner):
     req, slo = F.to_device(prob)
     plans = F.plans_to_numpy(planner.plan_decode(req, slo, torch.from_numpy(keys).cuda(), prob.k_max, inst, score))
     o = oracle.plan(prob, checks=False)
-    s_o, _ = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
-    v_o = oracle.victim(prob, o["status"], wl.inst, s_o)
+    ev = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
+    v_o = oracle.victim(prob, o["status"], wl.inst, ev)
     np.testing.assert_array_equal(plans["victim"], v_o)
 
 
@@ -439,7 +488,7 @@ def test_route_matches_oracle(F, planner, cfg, n_inst):
         wl = W.config4(T=1)
         prob = wl.problem
         inst = wl.inst
-        _, state = oracle.evict(inst, int(wl.now_us[0]), 30, wl.window_us)
+        state = oracle.evict(inst, int(wl.now_us[0]), 30, wl.window_us).state
         rng = W.SplitMix64(3)
         lat = rng.integers(1, 100, len(inst)).astype(np.uint32)
         cap = rng.integers(0, 3, len(inst)).astype(np.uint32)
@@ -661,8 +710,8 @@ def test_floor_next_paths(F, planner):
     req, slo = F.to_device(fprob)
     plans = F.plans_to_numpy(planner.plan_decode(req, slo, torch.from_numpy(keys).cuda(), fprob.k_max, inst, score))
     o = oracle.plan(fprob, checks=False)
-    s_o, _ = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
-    np.testing.assert_array_equal(plans["victim"], oracle.victim(fprob, o["status"], wl.inst, s_o))
+    ev = oracle.evict(wl.inst, int(wl.now_us[0]), 30, wl.window_us)
+    np.testing.assert_array_equal(plans["victim"], oracle.victim(fprob, o["status"], wl.inst, ev))
 
 
 # ---- NEXT-2 any-invoker (cross-node) planning (R39) --------------------------

@@ -28,30 +28,35 @@ def test_state_rules_fig8():
         (4, 8, W.INST_BUSY, 0, NOW - 10),        # serving right now: not evictable
         (5, -1, W.INST_PIPELINE, 9_000_000, NOW - 700_000_000),  # cold wins over everything
     ]
-    score, state = oracle.evict(inst(rows), NOW, 30, WIN, 600_000_000)
-    assert state.tolist() == [TS, HOT, HOT, WARM, COLD, TS, TS, COLD]
-    evictable = [0, 5]
-    for i in range(len(rows)):
-        if i in evictable:
-            assert score[i] == ((rows[i][4] << 20) | i)
-        else:
-            assert score[i] == KEY_NONE
+    ev = oracle.evict(inst(rows), NOW, 30, WIN, 600_000_000)
+    assert ev.state.tolist() == [TS, HOT, HOT, WARM, COLD, TS, TS, COLD]
+    assert ev.evictable.tolist() == [i in (0, 5) for i in range(len(rows))]
+    assert ev.idle.tolist() == [NOW - r[4] for r in rows]
 
 
-def test_lru_key_range_rule():
-    # R20b: last_used must fit the 43-bit field of the packed LRU key
-    rows = [(0, 1, 0, 0, (1 << 43) - 1), (1, 2, 0, 0, 1 << 43)]
-    score, state = oracle.evict(inst(rows), (1 << 43) + 10)
-    assert state.tolist() == [TS, TS]
-    assert score[0] == ((((1 << 43) - 1) << 20) | 0) and score[1] == KEY_NONE
+def test_epoch_timestamps_are_representable():
+    # R20c: no packed key in the oracle -- Unix-epoch microseconds (~1.8e15 > 2^43) order
+    # exactly like small ones; a last use in the future counts as idle 0 (R20b)
+    T = 1_800_000_000_000_000
+    rows = [(0, 1, 0, 0, T - 7), (1, 2, 0, 0, T - 9), (2, 3, 0, 0, T + 5)]
+    ev = oracle.evict(inst(rows), T)
+    assert ev.state.tolist() == [TS, TS, TS] and ev.evictable.all()
+    assert ev.idle.tolist() == [7, 9, 0]
 
 
 def test_lru_order_and_tie_break():
     # evict the least-recently-used time-sharing instance; equal last-use -> lower index
     rows = [(0, 1, 0, 0, NOW - 50), (1, 2, 0, 0, NOW - 500), (2, 3, 0, 0, NOW - 500), (3, 4, 0, 0, NOW - 5)]
-    score, state = oracle.evict(inst(rows), NOW)
-    order = np.argsort(score, kind="stable").tolist()
+    ev = oracle.evict(inst(rows), NOW)
+    order = sorted(range(len(rows)), key=lambda i: (-int(ev.idle[i]), i))
     assert order == [1, 2, 0, 3]
+    # the victim rule applies that order: every instance on one node whose slice fits
+    G = 4
+    f = dict(lat=[[100] * 5], mem=[1024], load=0)
+    prob = problem([f], [[[(G, 1), (G, 1), (G, 1), (G, 1)]]], [(0, 0, 10_000)])
+    v = oracle.victim(prob, np.array([oracle.PLAN_INFEASIBLE]), inst([(r[0], i, 0, 0, r[4]) for i, r in
+                                                                    enumerate(rows)]), ev)
+    assert v.tolist() == [1]
 
 
 def test_victim_rules():
@@ -66,9 +71,9 @@ def test_victim_rules():
         (9, 2, 0, 0, NOW - 100),   # 4g: 150 + 50 <= 400, more recently used
         (9, 3, 0, 0, NOW - 999),   # other node
     ]
-    score, _ = oracle.evict(inst(rows), NOW)
+    ev = oracle.evict(inst(rows), NOW)
     status = np.array([oracle.PLAN_INFEASIBLE, oracle.PLAN_INFEASIBLE, oracle.PLAN_INFEASIBLE, oracle.PLAN_OK])
-    v = oracle.victim(prob, status, inst(rows), score)
+    v = oracle.victim(prob, status, inst(rows), ev)
     # r0: LRU among {1, 2} -> 1;  r1: budget 200 leaves only 4g (150+50) -> 2;
     # r2: node 1 -> 3;  r3: has a free-slice plan -> no victim
     assert v.tolist() == [1, 2, 3, -1]
@@ -77,7 +82,7 @@ def test_victim_rules():
 def test_c4_generator_snapshot_mix():
     wl = W.config4(T=8)
     t0, t1 = int(wl.tick_off[0]), int(wl.tick_off[1])
-    score, state = oracle.evict(wl.inst[t0:t1], int(wl.now_us[0]))
-    counts = np.bincount(state, minlength=4)
+    ev = oracle.evict(wl.inst[t0:t1], int(wl.now_us[0]))
+    counts = np.bincount(ev.state, minlength=4)
     assert (counts > 0).all(), counts  # every keep-alive state occurs
-    assert (score != KEY_NONE).sum() > 10
+    assert ev.evictable.sum() > 10

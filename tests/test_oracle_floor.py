@@ -101,8 +101,8 @@ def test_floor_victims_and_ranked_respect_it():
     inst["func"] = rng.integers(0, prob.F, n_inst)
     inst["slice"] = rng.integers(0, len(prob.slices), n_inst)
     inst["last_used_us"] = rng.integers(0, 1 << 30, n_inst)
-    score, _ = oracle.evict(inst, 1 << 31, 30, 10_000_000)
-    vic = oracle.victim(prob, o["status"], inst, score)
+    ev = oracle.evict(inst, 1 << 31, 30, 10_000_000)
+    vic = oracle.victim(prob, o["status"], inst, ev)
     for q in np.nonzero(vic >= 0)[0]:
         p = int(prob.slices["profile"][inst["slice"][vic[q]]])
         a, b = int(prob.comp_off[f[q]]), int(prob.comp_off[f[q] + 1])
