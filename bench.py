@@ -2,12 +2,17 @@
 candidates scored/s and plans/s at 1/2/4/8 B200, % of the integer roofline).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ffs|reference] [--config 5]
+                    [--shard requests|candidates]
 
 One step = the whole hot path over one batch: ffs_plan_keys on this rank's shard (K0
-scan + K1 search segments) -> all_reduce(keys, MIN) over NCCL (N > 1) -> ffs_plan_decode
-of this rank's slice of the requests.  Inputs are resident in HBM when the timed region
-starts; L2 is flushed (256 MiB write) between timed steps, outside the events.  Each
-step is timed with CUDA events on the launching stream; ranks report the max.
+count + scan, K1 search segments KS = 1..4) -> ffs_plan_decode of this rank's slice.
+Request shards (default at C5) need no collective; candidate shards all_reduce(keys, MIN)
+over NCCL after every segment.  The headline `value` is the EXHAUSTIVE mode (every
+candidate of every request scored, device counters prove the count); the production
+(bounded) mode -- same keys -- is reported as plans/s under "production".  Inputs are
+resident in HBM when the timed region starts; L2 is flushed (256 MiB write) between timed
+steps, outside the events.  Each step is timed with CUDA events on the launching stream;
+ranks report the max.  Roofline peaks are measured by microbenchmarks in the same run.
 `--impl reference` times the CPU oracle (oracle/, the plain brute force) on a bounded
 sample of the same workload on this box's host cores (rank 0 only).
 """
@@ -39,29 +44,6 @@ def candidates_per_request(prob, k_max):
     S = np.array([sum(comb(int(m) - 1, k - 1) * P ** k for k in range(1, min(int(m), k_max) + 1)) for m in n],
                  dtype=np.int64)
     return S[prob.req["func"]]
-
-
-def enumerated(prob):
-    """Requests whose candidates the GPU enumerates: a node without any free slice admits
-    no candidate, so its requests are INFEASIBLE without enumeration (R37) and
-    their candidates are not counted as scored."""
-    free = np.zeros(prob.n_nodes, dtype=np.int64)
-    np.add.at(free, prob.slices["node"][prob.slices["busy"] == 0].astype(np.int64), 1)
-    return free[prob.req["node"]] > 0
-
-
-def segment_candidates(prob, k_max, rank, world):
-    """Candidates of segment ks processed by shard `rank`: T/world tasks (the kernel deals
-    equal pieces round-robin, dist.task_shard; a rank's count is within one task per piece
-    of T/world, < 1e-4 relative at C5)."""
-    n = prob.chain_len()[prob.req["func"]] * enumerated(prob)
-    out = []
-    for ks in range(1, k_max + 1):
-        tab = np.array([comb(m - 1, ks - 1) if m >= ks else 0 for m in range(33)], dtype=np.int64)
-        T = int(tab[n].sum())
-        sb, se = T * rank // world, T * (rank + 1) // world
-        out.append((se - sb) * P ** ks)
-    return out
 
 
 def _traffic(kernel):
@@ -377,6 +359,53 @@ def run_sim(pl):
             "slice_ticks_occupied": int(c[7])}
 
 
+def measure_peaks(pl):
+    """Roofline denominators measured on this GPU, in this run: K5 (integer
+    IADD3/LOP3/IMAD mix) and the packed f16x2 microbenchmarks (HFMA2 alone = FMA-pipe rate;
+    HFMA2 interleaved 1:1 with packed max / LOP3 = issue-limited rate).  Best of 3."""
+    int_ops = max(pl.int_peak()[0] for _ in range(3))
+    fma = max(pl.packed_peak(0)[0] for _ in range(3))
+    mix = max(pl.packed_peak(1)[0] for _ in range(3))
+    return {"int32_ops_per_s": int_ops, "hfma2_lane_instr_per_s": fma, "issue_lane_instr_per_s": mix,
+            "packed_ops_per_s": 2.0 * max(fma, mix)}
+
+
+def winner_histogram(p, slo):
+    """Winner histogram of one step's plans (printed with every run)."""
+    st = p["status"]
+    ok = st == 0
+    ks = np.bincount(p["k"][ok].astype(np.int64), minlength=9)[1:]
+    prof = np.zeros(5, dtype=np.int64)
+    for i in range(8):
+        sel = ok & (p["k"] > i)
+        prof += np.bincount(p["prof"][sel, i].astype(np.int64), minlength=5)[:5]
+    n = max(1, len(st))
+    return {"requests": int(len(st)), "ok_frac": float(ok.mean()) if len(st) else 0.0,
+            "infeasible_frac": float((st == 1).sum() / n), "bad_req_frac": float((st == 2).sum() / n),
+            "one_stage_frac": float((ok & (p["k"] == 1)).sum() / n),
+            "multi_stage_frac": float((ok & (p["k"] > 1)).sum() / n),
+            "k_hist": {str(k + 1): int(v) for k, v in enumerate(ks) if v},
+            "stage_profile_hist": dict(zip(["1g", "2g", "3g", "4g", "7g"], map(int, prof)))}
+
+
+def timed_steps(step, steps, flush, stream, barrier, pl=None):
+    """Per-step CUDA events on the launching stream, L2 flushed before each step outside
+    the events; returns (total ms, per-segment ms summed over the steps)."""
+    import torch
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    seg_ms = np.zeros(8)
+    barrier()
+    for i in range(steps):
+        flush.fill_(i & 0xFF)
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+        if pl is not None:
+            seg_ms += np.array(pl.segment_times())  # waits for this step's search segments
+    barrier()
+    return sum(a.elapsed_time(b) for a, b in ev), seg_ms
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -384,9 +413,10 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ffs", choices=["ffs", "reference"])
     ap.add_argument("--config", type=int, default=5, choices=[2, 3, 5])
+    ap.add_argument("--shard", default=None, choices=[None, "requests", "candidates"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--no-c4", action="store_true", help="skip the C4 eviction measurement")
+    ap.add_argument("--no-c4", action="store_true", help="skip the C4 eviction and NEXT-row measurements")
     args = ap.parse_args()
     assert args.warmup >= 3 or args.impl == "reference", "timing rules: >= 3 warm-up steps"
 
@@ -417,73 +447,96 @@ def main():
             dist.init_process_group(backend)
     K = prob.k_max
     R = prob.R
+    shard = args.shard or D.choose_shard(R, world)
     pl = ffs.Planner(local)
     pl.stage(prob)
     req, slo = ffs.to_device(prob)
-    keys = torch.empty(R, dtype=torch.int64, device="cuda")
+    keys = torch.full((R,), np.iinfo(np.int64).max, dtype=torch.int64, device="cuda")
     lo, hi = D.request_slice(R, rank, world)
     plans = torch.empty((hi - lo, 80), dtype=torch.uint8, device="cuda")
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
+    peaks_file = measured_peaks()
+    peaks = measure_peaks(pl)  # this GPU, this run
 
-    def step():  # keys of this rank's shard -> all_reduce(MIN) over NCCL -> decode own slice
-        D.plan_step(pl, req, slo, K, rank, world, keys, plans)
+    def step():  # this rank's shard of the batch: keys -> (exchange) -> decode of its slice
+        D.plan_step(pl, req, slo, K, rank, world, keys, plans, shard=shard)
 
     def barrier():
         if world > 1:
             dist.barrier()
         torch.cuda.synchronize()
 
+    def max_over_ranks(x):
+        if world > 1:
+            t = torch.tensor([x], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            x = float(t.item())
+        return x
+
+    # ---- headline: exhaustive mode, every candidate of every request scored ----
+    pl.set_search_mode(ffs.SEARCH_EXHAUSTIVE)
     for _ in range(args.warmup):
         step()
     barrier()
     clocks = Clocks(local)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    seg_ms = np.zeros(8)
-    barrier()
-    for i in range(args.steps):
-        flush.fill_(i & 0xFF)  # L2 flush, outside the timed events
-        ev[i][0].record(stream)
-        step()
-        ev[i][1].record(stream)
-        seg_ms += np.array(pl.segment_times())  # waits for this step's search segments
-    barrier()
+    ms, seg_ms = timed_steps(step, args.steps, flush, stream, barrier, pl)
     clk = clocks.stop()
-    ms = sum(a.elapsed_time(b) for a, b in ev)
+    scored_ks = pl.scored()  # device counters of the last (identical) step
+    ms = max_over_ranks(ms)
+    total_cands = int(candidates_per_request(prob, K).sum())
+    scored_all = sum(scored_ks)
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
-    total_cands = int(candidates_per_request(prob, K)[enumerated(prob)].sum())
-    value = total_cands * args.steps / (ms * 1e-3)
-    plans_per_s = R * args.steps / (ms * 1e-3)
-
-    # dominant kernel: the KS = K search segment on this rank
-    seg_c = segment_candidates(prob, K, rank, world)
+        t = torch.tensor([sum(scored_ks)], dtype=torch.int64, device="cuda")
+        dist.all_reduce(t)
+        scored_all = int(t.item())
+    value = scored_all * args.steps / (ms * 1e-3)
+    # dominant kernel of the exhaustive step on this rank: its scored candidates x the
+    # algorithmic ops per candidate over its event-timed launch duration
     top = int(np.argmax(seg_ms)) + 1
     top_ms = seg_ms[top - 1] / args.steps
-    peaks = measured_peaks()
-    sm_count = torch.cuda.get_device_properties(local).multi_processor_count
-    max_mhz = float(peaks.get("sm_max_mhz", 1965.0))
-    # issue-limited op rate of the packed f16x2 datapath the KS = 4 filter runs on: one
-    # warp-instruction per SMSP per clock, 32 lanes, two 16-bit operations per lane
-    peak_ops = sm_count * 4 * 32 * 2 * max_mhz * 1e6
-    # algorithmic work the kernel actually scored: for KS = 4, the stage-0 iterations the
-    # pre-filter evaluated (125 candidate pairs = 250 candidate slots each; iterations the
-    # exact stage-0 SLO bound skipped are not counted -- their candidates are decided
-    # infeasible without being scored); other segments score every candidate
-    # Every cut mask (task) of the segment is decided by the mask bound first: KS - 1 transfer
-    # adds and one compare = KS integer ops per mask (counted as one op each although each
-    # takes a full lane-issue of the packed peak: conservative)
-    seg_cov = float(seg_c[top - 1])
-    scored = seg_cov
-    if top == 4:
-        scored = float(pl.ks4_evaluated()) * 250.0  # counter of the last (identical) step
-    seg_tasks = seg_cov / float(P ** top)
-    achieved = (scored * ALG_OPS + seg_tasks * top) / (top_ms * 1e-3)
+    top_scored = float(scored_ks[top - 1])
+    achieved = top_scored * ALG_OPS / (top_ms * 1e-3)
     traffic = _traffic(f"k_plan_search<{top}>")
+    sm_count = torch.cuda.get_device_properties(local).multi_processor_count
+    max_mhz = float(peaks_file.get("sm_max_mhz", 1965.0))
+    nominal = sm_count * 4 * 32 * 2 * max_mhz * 1e6
+    peak = peaks["packed_ops_per_s"]
+    roofline = {"bound": "alu", "kernel": f"k_plan_search<{top}>", "achieved": achieved, "peak": peak,
+                "unit": "ops/s (16-bit lane ops; a packed f16x2 lane-instruction = 2)", "frac": achieved / peak,
+                "traffic": traffic, "alg_ops_per_candidate": ALG_OPS, "kernel_ms": top_ms,
+                "candidates_scored_per_launch": top_scored, "kernel_share_of_step": top_ms / (ms / args.steps),
+                "peak_source": "measured this run: 2 x max(HFMA2-chain, HFMA2+VHMNMX/LOP3 issue-mix) "
+                               "lane-instructions/s over all SMs (ffs_bench_packed_peak)",
+                "peak_nominal": nominal, "measured_peaks": peaks,
+                "survey_basis": {"ops_per_candidate": 20, "peak": peaks["int32_ops_per_s"],
+                                 "peak_source": "measured this run: K5 IADD3/LOP3/IMAD mix (ffs_bench_int_peak)",
+                                 "frac": top_scored * 20 / (top_ms * 1e-3) / peaks["int32_ops_per_s"],
+                                 "note": "SURVEY 8(d)'s 20 hoisted scalar int32 ops per candidate; the kernel's "
+                                         "group-maximum f16x2 core decides 5 candidates of each of 2 masks with 13 "
+                                         "packed instructions, so this basis can exceed 1 (DESIGN.md §5)"}}
 
-    # e2e through the public host-buffer API (N = 1: ffs_plan_batch_host)
+    # ---- production: bounded mode, identical keys, plans/s -----------------------------
+    pl.set_search_mode(ffs.SEARCH_BOUNDED)
+    keys_ex = keys[lo:hi].clone()
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    ms_b, seg_b = timed_steps(step, args.steps, flush, stream, barrier, pl)
+    ms_b = max_over_ranks(ms_b)
+    bounded_scored = sum(pl.scored())
+    same = bool(torch.equal(keys_ex, keys[lo:hi]))
+    hist = winner_histogram(ffs.plans_to_numpy(plans), None) if rank == 0 else None
+    production = {"metric": "plans_per_s", "value": R * args.steps / (ms_b * 1e-3), "unit": "plans/s",
+                  "ms_per_step": ms_b / args.steps,
+                  "candidates_decided_per_s": total_cands * args.steps / (ms_b * 1e-3),
+                  "candidates_scored_per_step_rank0": int(bounded_scored),
+                  "segment_ms_rank0": [float(x) / args.steps for x in seg_b[:K]],
+                  "keys_identical_to_exhaustive": same,
+                  "note": "FFS_SEARCH_BOUNDED: exact integer SLO lower bounds prove candidates infeasible "
+                          "without scoring them; same keys and plans as the exhaustive headline"}
+
+    # ---- e2e through the public host-buffer API (N = 1: ffs_plan_batch_host) ------------
     e2e = None
     if not args.no_e2e:
         h_req = torch.from_numpy(np.ascontiguousarray(prob.req).view(np.uint8)).pin_memory()
@@ -500,64 +553,64 @@ def main():
                 pl.plan_batch_host(req_np, slo_np, K, out=out_np)
             else:
                 D.plan_step_host(pl, h_req.view(-1, 8), h_slo.view(torch.int32), d_req, d_slo, K, rank, world,
-                                 keys, plans, h_out)
+                                 keys, plans, h_out, shard=shard)
 
-        for _ in range(2):
-            e2e_step()
-        barrier()
-        t0 = time.perf_counter()
-        n_e2e = max(3, args.steps // 2)
-        for _ in range(n_e2e):
-            e2e_step()
-        barrier()
-        dt = time.perf_counter() - t0
-        if world > 1:
-            t = torch.tensor([dt], dtype=torch.float64, device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            dt = float(t.item())
-        e2e = {"value": total_cands * n_e2e / dt, "unit": "candidates/s", "plans_per_s": R * n_e2e / dt,
-               "h2d_bytes_per_step": int(R * 12), "d2h_bytes_per_step": int((hi - lo) * 80),
+        def e2e_run():
+            for _ in range(2):
+                e2e_step()
+            barrier()
+            t0 = time.perf_counter()
+            n = max(3, args.steps // 2)
+            for _ in range(n):
+                e2e_step()
+            barrier()
+            return n, max_over_ranks(time.perf_counter() - t0)
+
+        pl.set_search_mode(ffs.SEARCH_EXHAUSTIVE)
+        n_e2e, dt = e2e_run()
+        pl.set_search_mode(ffs.SEARCH_BOUNDED)
+        n_b, dt_b = e2e_run()
+        e2e = {"value": scored_all * n_e2e / dt, "unit": "candidates/s", "plans_per_s": R * n_e2e / dt,
+               "h2d_bytes_per_step": int(D.h2d_bytes(R, rank, world, shard) if world > 1 else R * 12),
+               "d2h_bytes_per_step": int((hi - lo) * 80),
+               "production_plans_per_s": R * n_b / dt_b,
                "timer": "host wall clock around the blocking call, max over ranks"}
 
-    ranked = None
+    ranked = joint = frontier = c4 = sim = dagr = None
     if world == 1 and not args.no_c4:
         ranked = run_ranked(pl, prob, req, slo, args.steps, args.warmup, flush)
-    joint = frontier = None
-    if world == 1 and not args.no_c4:
         joint = run_joint(pl, prob, req, slo)
         frontier = run_frontier(pl, prob, req, slo, args.steps, args.warmup, flush)
-    c4 = sim = dagr = None
-    if world == 1 and not args.no_c4:
-        c4 = run_c4(pl, args.steps, args.warmup, flush, peaks)
+        c4 = run_c4(pl, args.steps, args.warmup, flush, peaks_file)
         sim = run_sim(pl)
         dagr = run_dag(pl, args.steps, args.warmup, flush)
     if rank == 0:
         cpu = None
         if world == 1 and not args.no_cpu_baseline:
             cpu = cpu_baseline(prob, K)
-        launches_per_step = 1 + 3 + min(K, int(prob.chain_len().max())) + 1
+        n_seg = min(K, int(prob.chain_len().max()))
+        launches_per_step = (1 + 3 + n_seg + 1) if shard == "requests" else (K * (1 + 3) + n_seg + 1)
         line = {
             "metric": "candidates_scored_per_s", "value": value, "unit": "candidates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/u64",
-            "data": "synthetic", "plans_per_s": plans_per_s,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f16x2 pre-filter + exact u32/u64 keys",
+            "data": "synthetic", "plans_per_s": R * args.steps / (ms * 1e-3),
             "config": {"workload": prob.meta["workload"], "R": R, "k_max": K, "candidates_per_step": total_cands,
+                       "candidates_scored_per_step": scored_all,
+                       "scored_counter_equals_sum_S": scored_all == total_cands,
+                       "mode": "exhaustive (FFS_SEARCH_EXHAUSTIVE)",
                        "l2": "flushed between steps (256 MiB write, outside the events)",
-                       "parallelism": f"candidate-range shards x{world} + all_reduce(MIN) over {backend}" if world > 1
-                       else "single GPU"},
-            "roofline": {"bound": "alu", "kernel": f"k_plan_search<{top}>", "achieved": achieved, "peak": peak_ops,
-                         "unit": "ops/s (packed f16x2: 2 per lane-issue)", "frac": achieved / peak_ops,
-                         "traffic": traffic,
-                         "alg_ops_per_candidate": ALG_OPS, "kernel_ms": top_ms,
-                         "candidates_covered_per_launch": seg_cov, "candidates_scored_per_launch": scored,
-                         "masks_per_launch": seg_tasks, "alg_ops_per_mask": top,
-                         "kernel_share_of_step": top_ms / (ms / args.steps),
-                         "peak_source": f"{sm_count} SMs x 4 SMSP x 32 lanes x 2 (f16x2) x {max_mhz:.0f} MHz "
-                                        f"(MEASURED_PEAKS.json sm_max_mhz)"},
+                       "parallelism": (f"request shards x{world} (no data-path collective)" if shard == "requests"
+                                       else f"candidate-range shards x{world} + all_reduce(MIN) over {backend}")
+                       if world > 1 else "single GPU"},
+            "roofline": roofline,
             "clocks": clk,
             "gpu_launches": launches_per_step * args.steps,
             "e2e": e2e,
             "cpu_baseline": cpu,
+            "production": production,
+            "winners": hist,
             "eviction_c4": c4,
             "ranked_first_fit": ranked,
             "joint_commit": joint,

@@ -1,25 +1,29 @@
-"""N-GPU path of the search: one process per GPU, torch.distributed NCCL.
+"""N-GPU path of the search: one process per GPU, torch.distributed (NCCL
+on GPUs, gloo in the CPU tests).  Every rank stages the same tables and holds the whole
+request batch.  Two ways to split it, both bit-identical to one GPU:
 
-Every rank stages the same tables and holds the whole request batch.  For each stage
-count k the flattened (request, cut mask) task list is cut into equal pieces dealt
-round-robin to the ranks one warp-sized chunk of 32 pieces at a time (``task_shard``, the same integer formula the search kernel uses), so
-shards are equal in candidates even with skewed chain lengths and sample the whole batch
-(equal in pruning too).  Each rank writes the
-minimum key of its range per request; one ``all_reduce(keys, MIN)`` over NCCL combines
-them (valid keys < INT64_MAX, the "none" sentinel, so MIN is exact and order-free).
-Each rank then decodes its own contiguous slice of the requests (``request_slice``).
+``shard="requests"`` (default for batches with many requests, the C5 case): requests are
+independent against the snapshot (R13), so rank g plans the contiguous request slice
+``request_slice(R, g, G)`` -- every segment, its own keys, its own decode -- with no
+data-path collective.  The request order of a batch is arrival order (Azure-shaped,
+functions drawn i.i.d.), so equal request counts are equal in candidates to within the
+sampling noise of R/G requests (C5 at 8 ranks: DESIGN.md §7 measures the spread).
+Pruning is per request, so a shard prunes exactly as one GPU does.
 
-Pruning: the search skips candidates that cannot beat the request's running best key,
-seeded by the earlier (cheaper) segments.  A rank's shard of segment k covers other
-requests than its shards of the earlier ones, so without exchange it would prune against
-(almost) nothing: measured on C5 at 8 ranks, 30 ms per rank instead of 13.4
-(tools/shard_emulation.py).  ``plan_step`` therefore all-reduces the keys after every
-segment (``ffs_plan_keys_range``, K collectives of 8 B x R): every rank prunes exactly
-as one GPU does.
+``shard="candidates"`` (few requests with huge candidate sets): for each stage count k the
+flattened (request, cut mask) task list is cut into equal pieces dealt round-robin to the
+ranks one warp-sized chunk of 32 pieces at a time (``task_shard``, the same integer
+formula the search kernel uses); each rank writes the minimum key of its pieces per
+request and ``all_reduce(keys, MIN)`` over NCCL combines them after every segment, so the
+next (heavier) segment prunes against the best key of all shards of the earlier ones
+(valid keys < INT64_MAX, the "none" sentinel: MIN is exact and order-free).  Each rank
+then decodes its own slice of the requests.
 """
 from __future__ import annotations
 
 import numpy as np
+
+MIN_REQUESTS_PER_RANK = 64  # below this a request shard is too lumpy: use candidate shards
 
 
 def task_shard(T: int, rank: int, world: int, chunks_per_rank: int, grain: int = 32) -> list[tuple[int, int]]:
@@ -34,8 +38,12 @@ def task_shard(T: int, rank: int, world: int, chunks_per_rank: int, grain: int =
 
 
 def request_slice(R: int, rank: int, world: int) -> tuple[int, int]:
-    """[lo, hi) of the requests whose plans `rank` decodes."""
+    """[lo, hi) of the requests `rank` owns (request shards) / decodes (candidate shards)."""
     return R * rank // world, R * (rank + 1) // world
+
+
+def choose_shard(R: int, world: int) -> str:
+    return "requests" if world == 1 or R >= MIN_REQUESTS_PER_RANK * world else "candidates"
 
 
 def allreduce_min_(keys, group=None):
@@ -48,10 +56,9 @@ def allreduce_min_(keys, group=None):
 
 
 def search_sharded(planner, req, slo, k_max: int, rank: int, world: int, keys, group=None, stream=None):
-    """Keys of the whole batch on every rank: for k = 1..K, shard segment k ->
-    all_reduce(MIN).  Each segment then prunes against the best key of every earlier
-    segment over all shards, as on one GPU (without the exchange the KS = 3 shard at 8
-    ranks costs 0.8x the whole single-GPU segment, measured).  One GPU: one ffs_plan_keys."""
+    """Candidate shards: keys of the whole batch on every rank: for k = 1..K, shard
+    segment k -> all_reduce(MIN).  Each segment then prunes against the best key of every
+    earlier segment over all shards, as on one GPU.  One GPU: one ffs_plan_keys."""
     if world == 1:
         planner.plan_keys(req, slo, k_max, rank, world, keys=keys, stream=stream)
         return keys
@@ -61,27 +68,48 @@ def search_sharded(planner, req, slo, k_max: int, rank: int, world: int, keys, g
     return keys
 
 
-def plan_step(planner, req, slo, k_max: int, rank: int, world: int, keys, plans=None, group=None, stream=None):
-    """One step of the sharded hot path: keys of this rank's shards (with the exchange of
-    ``search_sharded``) -> decode this rank's slice.  Returns (keys, plans of the slice,
-    (lo, hi))."""
-    search_sharded(planner, req, slo, k_max, rank, world, keys, group, stream)
-    lo, hi = request_slice(int(slo.numel()), rank, world)
-    plans = planner.plan_decode(req[lo:hi], slo[lo:hi], keys[lo:hi], k_max, out=plans, stream=stream)
+def plan_step(planner, req, slo, k_max: int, rank: int, world: int, keys, plans=None, group=None, stream=None,
+              shard: str | None = None):
+    """One step of the sharded hot path; returns (keys, plans of this rank's slice,
+    (lo, hi)).  Request shards: keys[lo:hi] and the plans of [lo, hi) from this rank
+    alone.  Candidate shards: keys of the whole batch (exchange per segment), then decode
+    of [lo, hi)."""
+    R = int(slo.numel())
+    shard = shard or choose_shard(R, world)
+    lo, hi = request_slice(R, rank, world)
+    if shard == "requests":
+        if hi > lo:
+            planner.plan_keys(req[lo:hi], slo[lo:hi], k_max, keys=keys[lo:hi], stream=stream)
+    elif shard == "candidates":
+        search_sharded(planner, req, slo, k_max, rank, world, keys, group, stream)
+    else:
+        raise ValueError(f"shard={shard!r}")
+    if hi > lo:
+        plans = planner.plan_decode(req[lo:hi], slo[lo:hi], keys[lo:hi], k_max, out=plans, stream=stream)
     return keys, plans, (lo, hi)
 
 
 def plan_step_host(planner, h_req, h_slo, d_req, d_slo, k_max: int, rank: int, world: int, keys, plans, h_out,
-                   group=None):
-    """End-to-end step through the public API with host buffers: H2D of the batch,
-    the sharded step, D2H of this rank's plans, synchronise."""
+                   group=None, shard: str | None = None):
+    """End-to-end step through the public API with host buffers: H2D of the batch rows the
+    rank needs (its slice for request shards, all of it for candidate shards), the sharded
+    step, D2H of this rank's plans, synchronise."""
     import torch
-    d_req.copy_(h_req, non_blocking=True)
-    d_slo.copy_(h_slo, non_blocking=True)
-    plan_step(planner, d_req, d_slo, k_max, rank, world, keys, plans, group)
+    R = int(h_slo.numel())
+    shard = shard or choose_shard(R, world)
+    lo, hi = request_slice(R, rank, world)
+    a, b = (lo, hi) if shard == "requests" else (0, R)
+    d_req[a:b].copy_(h_req[a:b], non_blocking=True)
+    d_slo[a:b].copy_(h_slo[a:b], non_blocking=True)
+    plan_step(planner, d_req, d_slo, k_max, rank, world, keys, plans, group, shard=shard)
     h_out.copy_(plans.view(-1), non_blocking=True)
     torch.cuda.current_stream().synchronize()
     return h_out
+
+
+def h2d_bytes(R: int, rank: int, world: int, shard: str, row_bytes: int = 12) -> int:
+    lo, hi = request_slice(R, rank, world)
+    return (hi - lo if shard == "requests" else R) * row_bytes
 
 
 def segment_tasks(chain_len: np.ndarray, k_max: int) -> list[int]:

@@ -20,21 +20,26 @@ prob = W.config3(R=8192)
 pl = ffs.Planner(dev)
 pl.stage(prob)
 req, slo = ffs.to_device(prob)
-keys = torch.empty(prob.R, dtype=torch.int64, device="cuda")
 lo, hi = D.request_slice(prob.R, rank, world)
-plans = torch.empty((hi - lo, 80), dtype=torch.uint8, device="cuda")
-D.plan_step(pl, req, slo, prob.k_max, rank, world, keys, plans)
-torch.cuda.synchronize()
-mine = (lo, hi, plans.cpu().numpy().tobytes(), keys.cpu().numpy().tobytes())
-got = [None] * world
-dist.all_gather_object(got, mine)
-if rank == 0:
-    ref_keys = pl.plan_keys(req, slo, prob.k_max)          # single rank, whole task space
-    ref_plans = pl.plan_decode(req, slo, ref_keys, prob.k_max).cpu().numpy()
-    ref_keys = ref_keys.cpu().numpy()
-    for lo_, hi_, pb, kb in got:
-        assert np.array_equal(np.frombuffer(kb, np.int64), ref_keys)
-        assert np.array_equal(np.frombuffer(pb, np.uint8).reshape(-1, 80), ref_plans[lo_:hi_])
-    assert got[0][0] == 0 and got[-1][1] == prob.R
-    print(f"dist-run ok world={world} backend={backend}")
+ref_keys = pl.plan_keys(req, slo, prob.k_max)          # single rank, whole task space
+ref_plans = pl.plan_decode(req, slo, ref_keys, prob.k_max).cpu().numpy()
+ref_keys = ref_keys.cpu().numpy()
+for shard in ("requests", "candidates"):
+    keys = torch.full((prob.R,), np.iinfo(np.int64).max, dtype=torch.int64, device="cuda")
+    plans = torch.empty((hi - lo, 80), dtype=torch.uint8, device="cuda")
+    D.plan_step(pl, req, slo, prob.k_max, rank, world, keys, plans, shard=shard)
+    torch.cuda.synchronize()
+    mine = (lo, hi, plans.cpu().numpy().tobytes(), keys.cpu().numpy().tobytes())
+    got = [None] * world
+    dist.all_gather_object(got, mine)
+    if rank == 0:
+        for lo_, hi_, pb, kb in got:
+            k = np.frombuffer(kb, np.int64)
+            if shard == "candidates":  # every rank holds the combined keys of the batch
+                assert np.array_equal(k, ref_keys)
+            else:                      # a rank holds the keys of its own requests
+                assert np.array_equal(k[lo_:hi_], ref_keys[lo_:hi_])
+            assert np.array_equal(np.frombuffer(pb, np.uint8).reshape(-1, 80), ref_plans[lo_:hi_])
+        assert got[0][0] == 0 and got[-1][1] == prob.R
+        print(f"dist-run ok world={world} backend={backend} shard={shard}")
 dist.destroy_process_group()

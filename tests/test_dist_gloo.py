@@ -1,6 +1,6 @@
 """The N-GPU path's host logic at world_size 2 over gloo on CPU:
-task-range shards, all_reduce(MIN) of int64 keys with the INT64_MAX sentinel, decode
-slices.  The CUDA shard kernel is replaced by an independent CPU emulation of the same
+request shards (no collective) and task-range shards with all_reduce(MIN) of int64 keys
+(INT64_MAX sentinel), decode slices.  The CUDA shard kernel is replaced by an independent CPU emulation of the same
 task split (tests/helpers.candidate_keys); the GPU kernel's own sharding is checked
 bit-exactly in tests/test_gpu_parity.py::test_sharding_invariance."""
 import os
@@ -35,15 +35,19 @@ def emulated_shard_keys(prob, rank, world, k_first=1, k_last=None):
 
 
 class FakePlanner:
-    """Stands in for ffs.Planner on CPU: plan_keys = emulated shard, decode = keys."""
+    """Stands in for ffs.Planner on CPU: plan_keys = emulated shard, decode = keys.  The
+    fake request rows carry the request index in their first four bytes, so a call on a
+    slice of the batch knows which requests it holds."""
 
     def __init__(self, prob):
         self.prob = prob
         self.calls = []
 
-    def plan_keys(self, req, slo, k_max, rank, world, keys=None, stream=None):
-        self.calls.append((1, k_max))
-        keys.copy_(torch.from_numpy(emulated_shard_keys(self.prob, rank, world)))
+    def plan_keys(self, req, slo, k_max, rank=0, world=1, keys=None, stream=None):
+        self.calls.append((1, k_max, int(req.shape[0])))
+        idx = req[:, :4].contiguous().view(torch.int32).view(-1).numpy()
+        sub = self.prob.subset(idx)
+        keys.copy_(torch.from_numpy(emulated_shard_keys(sub, rank, world)))
         return keys
 
     def plan_keys_range(self, req, slo, k_max, k_first, k_last, rank, world, keys=None, stream=None):
@@ -57,7 +61,7 @@ class FakePlanner:
         return keys.clone()
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, shard):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -67,13 +71,16 @@ def _worker(rank, world, port, q):
         from test_oracle_pins import random_tiny
         prob = random_tiny(1007)
         R = prob.R
-        keys = torch.empty(R, dtype=torch.int64)
+        keys = torch.full((R,), KEY_NONE, dtype=torch.int64)
         req = torch.zeros((R, 8), dtype=torch.uint8)
+        req[:, :4] = torch.arange(R, dtype=torch.int32).view(-1, 1).view(torch.uint8).view(R, 4)
         slo = torch.zeros(R, dtype=torch.int32)
         fp = FakePlanner(prob)
-        keys, plans, (lo, hi) = D.plan_step(fp, req, slo, prob.k_max, rank, world, keys)
-        # one sharded range per segment, an exchange after each
-        assert fp.calls == [(k, k) for k in range(1, prob.k_max + 1)]
+        keys, plans, (lo, hi) = D.plan_step(fp, req, slo, prob.k_max, rank, world, keys, shard=shard)
+        if shard == "candidates":  # one sharded range per segment, an exchange after each
+            assert fp.calls == [(k, k) for k in range(1, prob.k_max + 1)]
+        else:  # one whole search of the rank's own request slice, no collective
+            assert fp.calls == [(1, prob.k_max, hi - lo)]
         # sentinel survives MIN, and a MIN of partial minima is the global minimum
         t = torch.tensor([KEY_NONE, 5, KEY_NONE], dtype=torch.int64) if rank == 0 else \
             torch.tensor([KEY_NONE, KEY_NONE, 3], dtype=torch.int64)
@@ -91,14 +98,14 @@ def free_port():
     return p
 
 
-@pytest.mark.parametrize("world", [2])
-def test_sharded_step_matches_oracle_over_gloo(world):
+@pytest.mark.parametrize("world,shard", [(2, "candidates"), (2, "requests")])
+def test_sharded_step_matches_oracle_over_gloo(world, shard):
     import oracle
     from test_oracle_pins import random_tiny
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, shard)) for r in range(world)]
     for p in procs:
         p.start()
     res = sorted(q.get(timeout=120) for _ in range(world))
@@ -109,7 +116,10 @@ def test_sharded_step_matches_oracle_over_gloo(world):
     o = oracle.plan(prob)
     slices = []
     for rank, keys, (lo, hi), plans, t in res:
-        assert keys == o["key"].tolist()          # all_reduce(MIN) of the shards = global argmin
+        if shard == "candidates":
+            assert keys == o["key"].tolist()      # all_reduce(MIN) of the shards = global argmin
+        else:
+            assert keys[lo:hi] == o["key"][lo:hi].tolist()  # the rank's own requests, complete
         assert plans == o["key"][lo:hi].tolist()  # each rank decodes its own slice
         assert t == [KEY_NONE, 5, 3]
         slices.append((lo, hi))
@@ -137,3 +147,14 @@ def test_emulated_shards_cover_every_candidate():
     for world in (2, 3, 5):
         parts = np.stack([emulated_shard_keys(prob, g, world) for g in range(world)])
         np.testing.assert_array_equal(parts.min(axis=0), o["key"])
+
+
+def test_request_slices_partition_and_choice():
+    for R in (0, 1, 7, 1000, 1 << 20):
+        for world in (1, 2, 3, 8):
+            sl = [D.request_slice(R, g, world) for g in range(world)]
+            assert sl[0][0] == 0 and sl[-1][1] == R and all(a[1] == b[0] for a, b in zip(sl, sl[1:]))
+            assert max(h - l for l, h in sl) - min(h - l for l, h in sl) <= 1
+    assert D.choose_shard(1 << 20, 8) == "requests" and D.choose_shard(100, 8) == "candidates"
+    assert D.choose_shard(5, 1) == "requests"
+    assert D.h2d_bytes(1000, 1, 4, "requests") == 250 * 12 and D.h2d_bytes(1000, 1, 4, "candidates") == 12000

@@ -20,12 +20,28 @@ def _port():
     return p
 
 
-@pytest.mark.parametrize("world", [2, 4])
-def test_torchrun_sharded_step(world):
+def _torchrun(world, backend):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr", "127.0.0.1", "--master-port", str(_port()), os.path.join(HERE, "_dist_run.py")]
     res = subprocess.run(cmd, capture_output=True, text=True, timeout=900,
-                         env={**os.environ, "FFS_DIST_BACKEND": "gloo"})
+                         env={**os.environ, "FFS_DIST_BACKEND": backend})
     out = res.stdout + res.stderr
     assert res.returncode == 0, out[-4000:]
-    assert f"dist-run ok world={world}" in out
+    for shard in ("requests", "candidates"):
+        assert f"dist-run ok world={world} backend={backend} shard={shard}" in out
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_torchrun_sharded_step(world):
+    """Several ranks sharing the GPU(s) over gloo (runs on a one-GPU box)."""
+    _torchrun(world, "gloo")
+
+
+def test_torchrun_sharded_step_nccl():
+    """The NCCL path (one rank per GPU, all_reduce(MIN) over NVLink for candidate
+    shards): needs >= 2 GPUs, so it runs on the driver's multi-GPU box."""
+    import torch
+    n = torch.cuda.device_count()
+    if n < 2:
+        pytest.skip("NCCL path needs >= 2 GPUs (one rank per GPU)")
+    _torchrun(min(n, 8), "nccl")
