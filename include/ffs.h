@@ -453,6 +453,11 @@ ffs_status ffs_debug_filter_misses(ffs_ctx *ctx, uint64_t *out);
  * sum_r S(n_r, k_max) of the shard; candidates the bounded mode proves infeasible without
  * scoring are not counted).  Synchronises the device.  Zeros before the first call. */
 ffs_status ffs_search_scored(ffs_ctx *ctx, uint64_t *per_ks /* [8] */);
+/* Live (request, mask pair) records the bounded mode's compaction kernel wrote per stage
+ * count in the last search call (per_ks[ks-1]; 0 for segments that did not compact:
+ * ks = 1, ks > 4, exhaustive / verify modes).  A count above the context's list capacity
+ * means that segment ran on the task ranges instead.  Synchronises the device. */
+ffs_status ffs_search_live_records(ffs_ctx *ctx, uint64_t *per_ks /* [8] */);
 
 #ifdef __cplusplus
 }

@@ -3,6 +3,7 @@
 #include <algorithm>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -94,6 +95,11 @@ struct ffs_ctx {
   uint32_t seg_mask = 0;                                 // segments timed since the last k_first = 1
   // search mode (ffs_set_search_mode)
   uint32_t search_mode = FFS_SEARCH_BOUNDED;
+  // bounded mode: group tables (per function x availability pattern) and live-record lists
+  DevBuf gofs, grp, live_list;
+  bool grp_ok = false;
+  uint32_t list_cap = 0;
+  uint64_t list_cap_max = 1ull << 28;  // FFS_LIST_CAP (tests: force the task-range fallback)
 };
 
 static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
@@ -137,6 +143,7 @@ ffs_status ffs_create(int cuda_device, ffs_ctx** out) {
   ffs_ctx* c = new ffs_ctx;
   c->device = cuda_device;
   c->sms = prop.multiProcessorCount;
+  if (const char* e = std::getenv("FFS_LIST_CAP")) c->list_cap_max = std::strtoull(e, nullptr, 10);
   {
     DeviceGuard g(c->device);
     if (c->misses.ensure(8) != cudaSuccess || cudaMemset(c->misses.p, 0, 8) != cudaSuccess) {
@@ -170,7 +177,8 @@ void ffs_destroy(ffs_ctx* c) {
       b->release();
     for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand,
                       &c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
-                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr})
+                      &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr,
+                      &c->gofs, &c->grp, &c->live_list})
       b->release();
   }
   delete c;
@@ -254,6 +262,7 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   L.o_pm = take(rows, 4);
   L.o_xf = take(rows, 4);
   L.o_thr = take(F, 4);
+  L.o_tmm = take(2 * F, 4);
   L.words = (w + 3) / 4 * 4;
   std::vector<uint32_t> img(L.words, 0);
   for (uint32_t p = 0; p < 8; ++p) {
@@ -282,6 +291,21 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
     img[L.o_fdesc + 4 * f + 3] = (uint32_t)mtot;
     const uint32_t fl = tb->max_stage_us ? tb->max_stage_us[f] : 0u;
     img[L.o_thr + f] = fl ? fl : 0xffffffffu;  // R38: 0 = no floor
+    {  // KS = 4 f16 scale bounds, fp32 in chain order (as the kernel used to sum them)
+      float tmin = 0.f, tmax = 0.f;
+      for (uint32_t i = 0; i < n; ++i) {
+        float lo = 0.f, hi = 0.f;
+        for (uint32_t p = 0; p < P; ++p) {
+          const float l = (float)tb->lat_us[(uint64_t)(c0 + i) * P + p];
+          lo = p ? std::min(lo, l) : l;
+          hi = p ? std::max(hi, l) : l;
+        }
+        tmin += lo;
+        tmax += hi;
+      }
+      std::memcpy(&img[L.o_tmm + 2 * f], &tmin, 4);
+      std::memcpy(&img[L.o_tmm + 2 * f + 1], &tmax, 4);
+    }
     for (uint32_t p = 0; p < 8; ++p) img[L.o_pl + row * kRowW + p] = 0;
     img[L.o_pm + row] = 0;
     for (uint32_t i = 0; i < n; ++i) {
@@ -344,6 +368,25 @@ ffs_status ffs_stage_tables(ffs_ctx* c, const ffs_profiles* pr, const ffs_profil
   c->h_node_free = node_free;
   CK(c->slice_prof.ensure(sprof.size()), "cudaMalloc(slice_prof)");
   CK(cudaMemcpy(c->slice_prof.p, sprof.data(), sprof.size(), cudaMemcpyHostToDevice), "upload slice_prof");
+  // bounded-mode group tables: 32 availability patterns per function,
+  // built on the device from the image; skipped (task-range search only) above 1 GiB
+  {
+    std::vector<uint32_t> gofs(F);
+    uint64_t tot = 0;
+    for (uint32_t f = 0; f < F; ++f) {
+      gofs[f] = (uint32_t)tot;
+      tot += 32ull * grp_stride(len[f]);
+    }
+    c->grp_ok = tot * 4 <= (1ull << 30);
+    if (c->grp_ok) {
+      CK(c->gofs.ensure((size_t)F * 4), "cudaMalloc(gofs)");
+      CK(cudaMemcpy(c->gofs.p, gofs.data(), (size_t)F * 4, cudaMemcpyHostToDevice), "upload gofs");
+      CK(c->grp.ensure((size_t)tot * 4), "cudaMalloc(group tables)");
+      CK(launch_group_tables(c->image.as<uint32_t>(), L, c->gofs.as<uint32_t>(), c->grp.as<uint32_t>(), 0),
+         "group tables kernel");
+      CK(cudaDeviceSynchronize(), "group tables");
+    }
+  }
   c->lay = L;
   c->h_image = img;
   c->ranked = false;
@@ -429,13 +472,11 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows
   // of the KS = 4 kernel (kWin4 B per thread).  The f16x2 kernel's window stride is the
   // compile-time CTA size (immediate LDS/STS offsets); an image that does not fit next to
-  // its windows is read from global memory instead (tables_global).  The f32x2 variant
-  // shrinks its CTA first.
-  const size_t min_win = FFS_KS4_F32 ? kWin4 * 64 : kWin4 * search_block(4);
+  // its windows is read from global memory instead (tables_global).
+  const size_t min_win = kWin4 * search_block(4);
   const bool tables_global = (size_t)c->lay.words * 4 + min_win > kMaxSmem;
   const size_t smem = tables_global ? 0 : (size_t)c->lay.words * 4;
-  int block4 = search_block(4);
-  while (FFS_KS4_F32 && block4 > 32 && smem + kWin4 * block4 > kMaxSmem) block4 -= 32;
+  const int block4 = search_block(4);
   auto blk = [&](int k) { return k == 4 ? block4 : search_block(k); };
   auto shm = [&](int k) { return smem + (k == 4 ? kWin4 * block4 : 0); };
   if (c->occ_smem != smem + 1) {  // (smem = 0 <=> tables in global memory)
@@ -465,6 +506,34 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   a.exhaustive = exhaustive ? 1u : 0u;
   const bool verify = d_checks != nullptr;
   const uint32_t kk = std::min(k_last, c->max_n);
+  // bounded mode, KS = 2..4: live-mask compaction (k_live) before the search, which then
+  // walks the compacted records.  The list holds up to list_cap records;
+  // a segment with more live records falls back to the task ranges inside the search
+  // kernel (same result), so the capacity only bounds memory, never correctness.
+  const bool use_live = !verify && !exhaustive && c->grp_ok;
+  LiveArgs la{};
+  if (use_live) {
+    const uint64_t want = std::min<uint64_t>(16ull * n_req + (1ull << 20), c->list_cap_max);
+    if (c->list_cap != want) {
+      CK(c->live_list.ensure(std::max<uint64_t>(want, 1) * 16), "cudaMalloc(live list)");
+      c->list_cap = (uint32_t)want;
+    }
+    la.image = c->image.as<uint32_t>();
+    la.lay = c->lay;
+    la.req = d_req;
+    la.slo = d_slo;
+    la.node_free = a.node_free;
+    la.prefix = a.prefix;
+    la.n_req = n_req;
+    la.rank = rank;
+    la.world = world;
+    la.gofs = c->gofs.as<uint32_t>();
+    la.grp = c->grp.as<uint32_t>();
+    la.list = c->live_list.as<uint4>();
+    la.list_cap = c->list_cap;
+    la.work_ctr = a.work_ctr;
+    la.warps_total = (uint32_t)c->sms * 64;
+  }
   if (init) c->seg_mask = 0;
   for (uint32_t k = k_first; k <= kk; ++k) {
     const int grid = c->sms * c->occ[verify ? 1 : 0][k];
@@ -473,6 +542,13 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
                                               "ffs search KS=7", "ffs search KS=8"};
     nvtxRangePushA(kSegName[k]);
     CK(cudaEventRecord(c->evs[k], st), "event");
+    a.list = nullptr;
+    a.list_cap = 0;
+    if (use_live && k >= 2 && k <= 4) {
+      CK(launch_live((int)k, la, c->sms * 8, st), "live-mask kernel");
+      a.list = c->live_list.as<uint4>();
+      a.list_cap = c->list_cap;
+    }
     CK(launch_search((int)k, verify, a, grid, blk((int)k), shm((int)k), st), "search kernel");
     CK(cudaEventRecord(c->ev[k], st), "event");
     nvtxRangePop();
@@ -1189,6 +1265,18 @@ ffs_status ffs_search_scored(ffs_ctx* c, uint64_t* per_ks) {
   unsigned long long w[kCtrWords];
   CK(cudaMemcpy(w, c->work_ctr.p, sizeof w, cudaMemcpyDeviceToHost), "read counters");
   for (int k = 1; k <= kMaxK; ++k) per_ks[k - 1] = w[kCtrScored + k];
+  return FFS_OK;
+}
+
+ffs_status ffs_search_live_records(ffs_ctx* c, uint64_t* per_ks) {
+  if (!c || !per_ks) return FFS_ERR_ARG;
+  for (int k = 0; k < kMaxK; ++k) per_ks[k] = 0;
+  if (!c->work_ctr.p) return FFS_OK;
+  DeviceGuard g(c->device);
+  CK(cudaDeviceSynchronize(), "sync");
+  unsigned long long w[kCtrWords];
+  CK(cudaMemcpy(w, c->work_ctr.p, sizeof w, cudaMemcpyDeviceToHost), "read counters");
+  for (int k = 1; k <= kMaxK; ++k) per_ks[k - 1] = w[kCtrListCount + k];
   return FFS_OK;
 }
 

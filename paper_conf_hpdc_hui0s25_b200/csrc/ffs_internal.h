@@ -21,9 +21,6 @@ constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #ifndef FFS_MINB4
 #define FFS_MINB4 1
 #endif
-#ifndef FFS_KS4_F32
-#define FFS_KS4_F32 0  // 1: the f32x2 KS = 4 body (ks4_pair) instead of the f16x2 pre-filter
-#endif
 constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 // KS = 3 keeps every table in registers; capped at 168 registers it runs 12 warps per SM
 // and is faster (C5: 4.3 -> 3.9 ms).  The f16x2 KS = 4 kernel fits in 113 registers at
@@ -32,12 +29,12 @@ constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 #define FFS_BLOCK4 512
 #endif
 __host__ __device__ constexpr int search_block(int ks) {
-  return ks == 3 ? 384 : (ks == 4 && !FFS_KS4_F32) ? FFS_BLOCK4 : kBlock;
+  return ks == 3 ? 384 : ks == 4 ? FFS_BLOCK4 : kBlock;
 }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
 // bytes of per-thread shared-memory windows of the KS = 4 kernel: 5 profiles x 11 packed
-// pairs of f32 (f32x2 body) or f16 (f16x2 body)
-constexpr size_t kWin4 = FFS_KS4_F32 ? 440 : 220;
+// f16x2 pairs
+constexpr size_t kWin4 = 220;
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
 // image into shared memory once per CTA (A0 of DESIGN.md §4); every other kernel reads
@@ -54,6 +51,8 @@ struct ImageLayout {
   uint32_t o_pm;      // [rows] u32 PM[row0+i] = sum_{c<i} mem[c]
   uint32_t o_xf;      // [rows] u32 xfer cost of a cut after component i (row0+i)
   uint32_t o_thr;     // [F] u32 throughput floor: max stage time (R38); 0xffffffff = none
+  uint32_t o_tmm;     // [F][2] fp32 {tmin, tmax}: sum over the chain of the min / max component
+                      // latency over all profiles (KS = 4 f16 scale bounds), fp32 in chain order
 };
 
 struct SearchArgs {
@@ -74,10 +73,44 @@ struct SearchArgs {
   uint32_t zero;                // always 0: an operand ptxas cannot fold (ks4_pair_h's IADD3)
   uint32_t exhaustive;          // FFS_SEARCH_EXHAUSTIVE: no stage-0 SLO bound, every
                                 // candidate of every enumerated mask is scored
+  // bounded mode, KS = 2..4: the live (request, mask pair) records k_live wrote; when set
+  // and the segment's record count fits list_cap, the search walks the list instead of
+  // the task ranges (DESIGN.md §4.3 "live-mask compaction")
+  const uint4* list;            // {request, maskA, maskB (0 = none), 0}
+  uint32_t list_cap;
 };
-// work_ctr layout: [0..kMaxK] per-KS chunk counters; [kCtrScored + KS] candidates the
-// segment's kernel scored (every candidate whose own score it computed)
-constexpr int kCtrScored = 16, kCtrWords = 32;
+// work_ctr layout: [0..kMaxK] per-KS task-chunk grab counters; [kCtrScored + KS]
+// candidates the segment's kernel scored (every candidate whose own score it computed);
+// [kCtrListGrab + KS] record-chunk grab counters and [kCtrListCount + KS] live records
+// written by k_live (bounded mode)
+constexpr int kCtrScored = 16, kCtrListGrab = 24, kCtrListCount = 32, kCtrWords = 48;
+
+// Group tables of the bounded mode: per function f and availability
+// pattern a (bit p = the node has >= 1 free slice of profile p), with W(i, j) = the fastest
+// admissible time of stage [i, j) (profile in a, stage memory <= capacity, time <= floor;
+// kGInf if none) and X(j) the cost of the cut at boundary j:
+//   H0[j] = W(0, j) + X(j), T3[i] = W(i, n), Mt[j][i] = W(i, j) + X(j) (i < j < n),
+//   R2[j] = min_i H0[i] + Mt[j][i], R3[j] = min_i R2[i] + Mt[j][i]
+// every value clamped to kGInf.  An e2e lower bound of a KS-stage mask is then a sum of
+// <= 4 table entries, exact in u32.
+constexpr uint32_t kGInf = 1u << 29;
+__host__ __device__ constexpr uint32_t grp_stride(uint32_t n) { return 4 * (n + 1) + (n + 1) * (n + 1); }
+
+struct LiveArgs {
+  const uint32_t* image;        // global copy (read through L1)
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  const uint64_t* node_free;
+  const uint64_t* prefix;
+  uint32_t n_req, rank, world;
+  const uint32_t* gofs;         // [F] word offset of function f's group tables
+  const uint32_t* grp;
+  uint4* list;
+  uint32_t list_cap;
+  unsigned long long* work_ctr;
+  uint32_t warps_total;         // warps per search launch (the task split must match k_plan_search)
+};
 
 struct DecodeArgs {
   const uint32_t* image;
@@ -121,6 +154,9 @@ cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const 
                            cudaStream_t st);
 cudaError_t run_int_peak(int sms, double* ops, double* seconds);
 cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double* seconds);
+cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, const uint32_t* gofs, uint32_t* grp,
+                                cudaStream_t st);
+cudaError_t launch_live(int ks, const LiveArgs& a, int grid, cudaStream_t st);
 
 struct RankedArgs {
   const uint32_t* image;

@@ -540,7 +540,7 @@ __device__ __forceinline__ void pair_rescan(SearchState<KS>& c, const Geo<KS>& G
 // last stage (blim - v2min - S2, integers < 2^25).
 template <bool VERIFY>
 __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint32_t maskB, bool haveB,
-                                         unsigned long long* misses, bool exh) {
+                                         unsigned long long* misses, bool exh, uint64_t shiftB) {
   const float INF = __int_as_float(0x7f800000);
   Geo<3> G[2];
   geo<3>(c, maskA, G[0]);
@@ -637,127 +637,7 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
   }
   constexpr uint32_t kAllB = (1u << kP) - 1;
   pair_rescan<3, VERIFY>(c, G[0], pendA, VERIFY ? kAllB : pendA, 0, misses);
-  if (haveB) pair_rescan<3, VERIFY>(c, G[1], pendB, VERIFY ? kAllB : pendB, 125, misses);
-}
-
-struct Win2 {
-  f2 s1, s2[2], s3[3];
-};
-
-// rows: per thread and profile x, 11 packed pairs in [x][k][thread] order (8-byte,
-// conflict-free); window e (e = 1 when x is the stage-0 profile) is read at offset e.
-template <bool VERIFY>
-__device__ __forceinline__ void ks4_pair(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, f2* rows,
-                                         unsigned long long* misses) {
-  const float INF = __int_as_float(0x7f800000);
-  const int tid = threadIdx.x, nb = blockDim.x;  // window stride = threads of the CTA
-  Geo4 G[2];
-  geo4(c, maskA, G[0]);
-  geo4(c, maskB, G[1]);
-  if (!haveB) G[1].blim = -1.f;  // dummy lane: nothing passes (every slack < 0)
-  const float al = c.alpha, one_m_a = 1.f - c.alpha;
-  f2 a1[kP], a2[kP], t2[kP], cc[kP];
-  {
-    float f[2][4][kP];
-#pragma unroll
-    for (int h = 0; h < 2; ++h)
-#pragma unroll
-      for (int s = 0; s < 4; ++s) geo_lat(c, G[h], s, f[h][s]);
-#pragma unroll
-    for (int x = 0; x < kP; ++x) {
-      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-      const uint32_t cap = c.sm[c.o_cap + x];
-      // memory folded once per (half, stage), then one select per multiplicity; the last
-      // stage is kept as SLO slack Blim - v3 (-INF when folded)
-      float v[2][4][4];
-      bool gate[4];
-#pragma unroll
-      for (int m = 0; m < 4; ++m) gate[m] = fr > (uint32_t)m;
-#pragma unroll
-      for (int h = 0; h < 2; ++h)
-#pragma unroll
-        for (int s = 0; s < 4; ++s) {
-          const float vm = (G[h].memst[s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] : INF;
-          const float base = (s == 3) ? G[h].blim - vm : vm;
-          const float none = (s == 3) ? -INF : INF;
-#pragma unroll
-          for (int m = 0; m <= s && m < 4; ++m) v[h][s][m] = gate[m] ? base : none;
-        }
-      a1[x] = f2pack(al * (f[0][1][x] * f[0][1][x]), al * (f[1][1][x] * f[1][1][x]));
-      a2[x] = f2pack(al * (f[0][2][x] * f[0][2][x]), al * (f[1][2][x] * f[1][2][x]));
-      t2[x] = f2pack(f[0][3][x] + f[0][3][x], f[1][3][x] + f[1][3][x]);
-      cc[x] = f2pack(one_m_a * (f[0][3][x] * f[0][3][x]), one_m_a * (f[1][3][x] * f[1][3][x]));
-      const float a0A = al * (f[0][0][x] * f[0][0][x]), a0B = al * (f[1][0][x] * f[1][0][x]);
-      // compact per-thread row of profile x: 11 packed pairs
-      //   [v1[0], v1[1], v2[0], v2[1], v2[2], Bl-v3[0..3], v0[0], a0]
-      // (the last stage is stored as SLO slack Blim - v3, so d2 = (Blim - v3) - S3)
-      f2* r = rows + (x * 11) * nb + tid;
-      r[0 * nb] = f2pack(v[0][1][0], v[1][1][0]);
-      r[1 * nb] = f2pack(v[0][1][1], v[1][1][1]);
-      r[2 * nb] = f2pack(v[0][2][0], v[1][2][0]);
-      r[3 * nb] = f2pack(v[0][2][1], v[1][2][1]);
-      r[4 * nb] = f2pack(v[0][2][2], v[1][2][2]);
-      r[5 * nb] = f2pack(v[0][3][0], v[1][3][0]);
-      r[6 * nb] = f2pack(v[0][3][1], v[1][3][1]);
-      r[7 * nb] = f2pack(v[0][3][2], v[1][3][2]);
-      r[8 * nb] = f2pack(v[0][3][3], v[1][3][3]);
-      r[9 * nb] = f2pack(v[0][0][0], v[1][0][0]);
-      r[10 * nb] = f2pack(a0A, a0B);
-    }
-  }
-  uint32_t pendA = 0, pendB = 0;
-#pragma unroll 1
-  for (int d0 = 0; d0 < kP; ++d0) {
-    Win2 W[kP];
-#pragma unroll
-    for (int x = 0; x < kP; ++x) {
-      const int e = (x == d0);  // every multiplicity of the stage-0 profile shifted by one
-      const f2* r = rows + (x * 11 + e) * nb + tid;
-      W[x].s1 = r[0];
-      W[x].s2[0] = r[2 * nb];
-      W[x].s2[1] = r[3 * nb];
-      W[x].s3[0] = r[5 * nb];
-      W[x].s3[1] = r[6 * nb];
-      W[x].s3[2] = r[7 * nb];
-    }
-    const f2 S1 = rows[(d0 * 11 + 9) * nb + tid];
-    const f2 NL1 = f2sub(0ull, rows[(d0 * 11 + 10) * nb + tid]);  // -alpha t0^2
-#pragma unroll
-    for (int d1 = 0; d1 < kP; ++d1) {
-      const f2 w1 = W[d1].s1;
-      const f2 S2 = f2add(S1, w1), NL2 = f2sub(NL1, a1[d1]);
-      // independent accumulator chains per q (ILP); merged at the end of the block
-      uint32_t accA[kP], accB[kP];
-#pragma unroll
-      for (int q = 0; q < kP; ++q) {
-        const f2 w2 = W[q].s2[q == d1];
-        const f2 S3 = f2add(S2, w2);
-        const f2 NL3 = f2sub(NL2, a2[q]);  // -(alpha * sum t^2 of stages 0..2)
-        const f2 U = f2fma(S3, S3, NL3);
-        accA[q] = ~0u;
-        accB[q] = ~0u;
-#pragma unroll
-        for (int p = 0; p < kP; ++p) {
-          const f2 w3 = W[p].s3[(p == d1) + (p == q)];
-          const f2 z = f2add(f2fma(S3, t2[p], cc[p]), U);
-          const f2 d2 = f2sub(w3, S3);  // (Blim - v3) - S3 < 0: SLO / memory / free miss
-          uint32_t zl, zh, dl, dh;
-          f2bits(z, zl, zh);
-          f2bits(d2, dl, dh);
-          accA[q] &= zl | dl;
-          accB[q] &= zh | dh;
-        }
-      }
-      const uint32_t mA = accA[0] & accA[1] & accA[2] & accA[3] & accA[4];
-      const uint32_t mB = accB[0] & accB[1] & accB[2] & accB[3] & accB[4];
-      pendA |= ((mA >> 31) ^ 1u) << (kP * d0 + d1);
-      pendB |= ((mB >> 31) ^ 1u) << (kP * d0 + d1);
-    }
-  }
-  // rare exact path, one half at a time (geometry copied into the state)
-  constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
-  pair_rescan<4, VERIFY>(c, G[0], pendA, VERIFY ? kAll : pendA, 0, misses);
-  if (haveB) pair_rescan<4, VERIFY>(c, G[1], pendB, VERIFY ? kAll : pendB, 625, misses);
+  if (haveB) pair_rescan<3, VERIFY>(c, G[1], pendB, VERIFY ? kAllB : pendB, shiftB, misses);
 }
 
 // ---- KS = 4, f16x2 pre-filter ---------------------------------------
@@ -840,7 +720,7 @@ struct WinH {
 // stored -- half the LDS -- measured 2.6 % slower: more registers and smem.)
 template <bool VERIFY>
 __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
-                                           unsigned long long* misses, uint32_t zero, bool exh) {
+                                           unsigned long long* misses, uint32_t zero, bool exh, uint64_t shiftB) {
   const float INF = __int_as_float(0x7f800000);
   constexpr int nb = search_block(4);  // window stride: the CTA size, fixed at compile time
   const int tid = threadIdx.x;
@@ -1019,7 +899,7 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   if (wide[0]) pendA = kAll;  // dynamic range too wide for f16: every block exactly
   if (wide[1]) pendB = kAll;
   pair_rescan<4, VERIFY>(c, G[0], pendA, VERIFY ? kAll : pendA, 0, misses);
-  if (haveB) pair_rescan<4, VERIFY>(c, G[1], pendB, VERIFY ? kAll : pendB, 625, misses);
+  if (haveB) pair_rescan<4, VERIFY>(c, G[1], pendB, VERIFY ? kAll : pendB, shiftB, misses);
 }
 
 template <int KS, bool VERIFY>
@@ -1119,6 +999,19 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
   return lo;
 }
 
+// colex rank of a cut mask among the (KS-1)-subsets of the cut positions: sum C(j_i, i)
+template <int KS>
+__device__ __forceinline__ uint64_t colex_rank(const uint32_t* img, const ImageLayout& L, uint32_t mask) {
+  uint64_t rk = 0;
+#pragma unroll
+  for (int i = 1; i < KS; ++i) {
+    const int j = __ffs(mask) - 1;
+    mask &= mask - 1;
+    rk += binom(img, L, j, i);
+  }
+  return rk;
+}
+
 template <int KS, bool VERIFY, bool TG>
 __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
@@ -1136,25 +1029,14 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += blockDim.x) dst[i] = src[i];
   }
   __syncthreads();
-  // KS = 4: per-thread windows of the shifted variant tables after the image (ks4_pair)
+  // KS = 4: per-thread windows of the shifted variant tables after the image (ks4_pair_h)
   float* rows = reinterpret_cast<float*>(smem + img_words);
 
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
-  const uint64_t T = pre[A.n_req];
-  // Work split: the segment's task list is cut into NC = world x (nthr/32) x kdyn(KS) chunks
-  // of 32 equal contiguous pieces (one per lane).  Rank `rank` owns chunks
-  // j * world + rank; its warps grab them dynamically (atomic counter, zeroed by the count
-  // kernel), so a warp whose pieces are cheap (skipped stage-0 profiles, no rescans) takes
-  // more of them and the launch ends when the work does, not with the slowest static
-  // share.  Ranks interleave at the grain of one chunk, so each samples the whole batch
-  // (contiguous 1/world ranges measured up to 1.2x apart on C5).  Exact cover needs the
-  // same nthr on every rank (same kernel and device type).  DESIGN.md §4.3, §7.
   const uint32_t lane = threadIdx.x & 31;
-  const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
-  const uint64_t NC = (nthr >> 5) * kdyn(KS) * A.world, NT = NC * 32;
-  const uint64_t Tq = T / NT, Tr = T % NT;  // piece u = [Tq u + Tr u / NT, ...): no overflow
-  auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
-  unsigned long long* ctr = A.work_ctr + KS;
+  uint64_t PK = 1;
+#pragma unroll
+  for (int i = 0; i < KS; ++i) PK *= kP;
 
   SearchState<KS> c;
   c.n_scored = 0;
@@ -1164,24 +1046,10 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   c.o_xf = A.lay.o_xf;
   c.o_cap = A.lay.o_cap;
   c.o_gpcs = A.lay.o_gpcs;
-  uint64_t PK = 1;
-#pragma unroll
-  for (int i = 0; i < KS; ++i) PK *= kP;
-
-  for (;;) {
-  unsigned long long jg = 0;
-  if (lane == 0) jg = atomicAdd(ctr, 1ull);
-  jg = __shfl_sync(0xffffffffu, jg, 0);
-  const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
-  if (chunk >= NC) break;
-  const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
-  if (t0 >= t1) continue;
-  uint64_t task = t0;
-  uint32_t r = find_request(pre, A.n_req, task);
-  uint64_t m = task - pre[r], cnt = pre[r + 1] - pre[r], done = 0;
+  uint32_t r = 0;
   int64_t best0 = 0;
-  uint32_t mask = 0;
 
+  // request r's state; idx_base = the index of the rank0-th mask's first candidate
   auto load_request = [&](uint64_t rank0) {
     const ffs_request q = A.req[r];
     const uint32_t* fd = tbl + A.lay.o_fdesc + 4 * q.func;
@@ -1199,46 +1067,14 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     c.best = *reinterpret_cast<volatile const int64_t*>(A.keys + r);  // earlier segments' minimum
     best0 = c.best;
     if constexpr (KS >= 2) set_threshold(c);
-    if constexpr (KS == 4) {
-      float tmin = 0.f, tmax = 0.f;
-      const uint32_t* rowp = tbl + A.lay.o_pl + c.row0 * kRowW;
-      float4 la = *reinterpret_cast<const float4*>(rowp);
-      float l4 = __uint_as_float(rowp[4]);
-      for (uint32_t i = 0; i < c.n; ++i) {
-        rowp += kRowW;
-        const float4 lb = *reinterpret_cast<const float4*>(rowp);
-        const float lb4 = __uint_as_float(rowp[4]);
-        const float d0 = lb.x - la.x, d1 = lb.y - la.y, d2 = lb.z - la.z, d3 = lb.w - la.w, d4 = lb4 - l4;
-        tmin += fminf(fminf(fminf(d0, d1), fminf(d2, d3)), d4);
-        tmax += fmaxf(fmaxf(fmaxf(d0, d1), fmaxf(d2, d3)), d4);
-        la = lb;
-        l4 = lb4;
-      }
-      c.tmin = tmin;  // upper/lower bounds; fp32 rounding above 2^24 is covered by the 2^-7 slack margin
-      c.tmax = tmax;
+    if constexpr (KS == 4) {  // f16 scale bounds; fp32 rounding above 2^24 is covered by the 2^-7 slack margin
+      c.tmin = __uint_as_float(tbl[A.lay.o_tmm + 2 * q.func]);
+      c.tmax = __uint_as_float(tbl[A.lay.o_tmm + 2 * q.func + 1]);
     }
     c.nfeas = 0;
     c.ksum = 0;
-    done = 0;
-    // colex unrank of rank0 among the (KS-1)-subsets of the n-1 cut positions.  Rank 0
-    // (a request entered at its first task) is the lowest KS-1 bits: a shortcut worth it
-    // where requests are short (KS <= 3); for KS = 4 the extra branch measured 1% slower.
-    uint32_t mk = (1u << (KS - 1)) - 1;
-    if (KS >= 4 || rank0 != 0) {
-      mk = 0;
-      uint64_t mm = rank0;
-      int cc = (int)c.n - 2;
-#pragma unroll
-      for (int i = KS - 1; i >= 1; --i) {
-        while (binom(tbl, A.lay, cc, i) > mm) --cc;
-        mk |= 1u << cc;
-        mm -= binom(tbl, A.lay, cc, i);
-        --cc;
-      }
-    }
-    mask = mk;
   };
-  auto flush = [&]() {
+  auto flush = [&](uint64_t done) {
     if (c.best < best0) atomicMin(reinterpret_cast<long long*>(A.keys + r), (long long)c.best);
     if (VERIFY) {
       atomicAdd(A.checks + 3ull * r, (unsigned long long)(done * PK));
@@ -1247,46 +1083,130 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     }
   };
 
-  load_request(m);
-  while (true) {
-    uint32_t step = 1;
-    if constexpr (KS == 3 || KS == 4) {
-      // two consecutive masks of the same request per iteration (ks3_pair / ks4_pair)
-      const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
-      const uint32_t maskB = haveB ? gosper_next(mask) : mask;
-#if FFS_KS4_F32
-      if constexpr (KS == 4) ks4_pair<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<f2*>(rows), A.misses);
-#else
-      if constexpr (KS == 4)
-        ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero, A.exhaustive != 0);
-#endif
-      else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0);
-      if (haveB) {
-        step = 2;
-        mask = maskB;
+  uint64_t n_list = ~0ull;
+  if (!VERIFY && KS >= 2 && KS <= 4 && A.list != nullptr)
+    n_list = *reinterpret_cast<volatile const unsigned long long*>(A.work_ctr + kCtrListCount + KS);
+  if (n_list <= A.list_cap) {
+    // ---- bounded mode: the live (request, mask pair) records of k_live ----------------
+    // A warp takes 32 consecutive records (one per lane) at a time; every record carries
+    // its request, so a lane loads the request's state per record.
+    unsigned long long* lctr = A.work_ctr + kCtrListGrab + KS;
+    for (;;) {
+      unsigned long long jg = 0;
+      if (lane == 0) jg = atomicAdd(lctr, 1ull);
+      jg = __shfl_sync(0xffffffffu, jg, 0);
+      if (jg * 32 >= n_list) break;
+      const uint64_t i = jg * 32 + lane;
+      if (i >= n_list) continue;
+      const uint4 rec = A.list[i];
+      r = rec.x;
+      const uint32_t maskA = rec.y, maskB = rec.z;
+      const bool haveB = maskB != 0u;
+      const uint64_t rkA = colex_rank<KS>(tbl, A.lay, maskA);
+      const uint64_t shiftB = haveB ? (colex_rank<KS>(tbl, A.lay, maskB) - rkA) * PK : 0ull;
+      load_request(rkA);
+      if constexpr (KS == 4) {
+        ks4_pair_h<false>(c, maskA, haveB ? maskB : maskA, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
+                          false, shiftB);
+      } else if constexpr (KS == 3) {
+        ks3_pair<false>(c, maskA, haveB ? maskB : maskA, haveB, A.misses, false, shiftB);
+      } else if constexpr (KS == 2) {
+        process_mask<KS, false>(c, maskA, rows, A.misses);
+        if (haveB) {
+          c.idx_base += shiftB;
+          process_mask<KS, false>(c, maskB, rows, A.misses);
+        }
       }
-    } else {
-      process_mask<KS, VERIFY>(c, mask, rows, A.misses);
+      flush(0);
     }
-    done += step;
-    task += step;
-    if (task >= t1) break;
-    m += step;
-    if (m == cnt) {
-      flush();
-      // tasks are consecutive: the next one belongs to the next request with tasks
-      // (requests without tasks of this KS have pre[r + 1] == pre[r]); no binary search
-      do ++r; while (pre[r + 1] <= task);
-      m = 0;
-      cnt = pre[r + 1] - pre[r];
-      load_request(0);
-    } else {
-      mask = gosper_next(mask);
-      c.idx_base += step * PK;
-    }
+  } else {
+    // ---- task ranges (exhaustive and verify modes; bounded mode's fallback) -------------
+    const uint64_t T = pre[A.n_req];
+    // Work split: the segment's task list is cut into NC = world x (nthr/32) x kdyn(KS) chunks
+    // of 32 equal contiguous pieces (one per lane).  Rank `rank` owns chunks
+    // j * world + rank; its warps grab them dynamically (atomic counter, zeroed by the count
+    // kernel), so a warp whose pieces are cheap (skipped stage-0 profiles, no rescans) takes
+    // more of them and the launch ends when the work does, not with the slowest static
+    // share.  Ranks interleave at the grain of one chunk, so each samples the whole batch
+    // (contiguous 1/world ranges measured up to 1.2x apart on C5).  Exact cover needs the
+    // same nthr on every rank (same kernel and device type).  DESIGN.md §4.3, §7.
+    const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t NC = (nthr >> 5) * kdyn(KS) * A.world, NT = NC * 32;
+    const uint64_t Tq = T / NT, Tr = T % NT;  // piece u = [Tq u + Tr u / NT, ...): no overflow
+    auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
+    unsigned long long* ctr = A.work_ctr + KS;
+    for (;;) {
+      unsigned long long jg = 0;
+      if (lane == 0) jg = atomicAdd(ctr, 1ull);
+      jg = __shfl_sync(0xffffffffu, jg, 0);
+      const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
+      if (chunk >= NC) break;
+      const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
+      if (t0 >= t1) continue;
+      uint64_t task = t0;
+      r = find_request(pre, A.n_req, task);
+      uint64_t m = task - pre[r], cnt = pre[r + 1] - pre[r], done = 0;
+      uint32_t mask = 0;
+      // colex unrank of rank0 among the (KS-1)-subsets of the n-1 cut positions.  Rank 0
+      // (a request entered at its first task) is the lowest KS-1 bits: a shortcut worth it
+      // where requests are short (KS <= 3); for KS = 4 the extra branch measured 1% slower.
+      auto unrank = [&](uint64_t rank0) {
+        uint32_t mk = (1u << (KS - 1)) - 1;
+        if (KS >= 4 || rank0 != 0) {
+          mk = 0;
+          uint64_t mm = rank0;
+          int cc = (int)c.n - 2;
+#pragma unroll
+          for (int i = KS - 1; i >= 1; --i) {
+            while (binom(tbl, A.lay, cc, i) > mm) --cc;
+            mk |= 1u << cc;
+            mm -= binom(tbl, A.lay, cc, i);
+            --cc;
+          }
+        }
+        mask = mk;
+      };
+      load_request(m);
+      unrank(m);
+      while (true) {
+        uint32_t step = 1;
+        if constexpr (KS == 3 || KS == 4) {
+          // two consecutive masks of the same request per iteration (ks3_pair / ks4_pair_h)
+          const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
+          const uint32_t maskB = haveB ? gosper_next(mask) : mask;
+          if constexpr (KS == 4)
+            ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
+                               A.exhaustive != 0, PK);
+          else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0, PK);
+          if (haveB) {
+            step = 2;
+            mask = maskB;
+          }
+        } else {
+          process_mask<KS, VERIFY>(c, mask, rows, A.misses);
+        }
+        done += step;
+        task += step;
+        if (task >= t1) break;
+        m += step;
+        if (m == cnt) {
+          flush(done);
+          done = 0;
+          // tasks are consecutive: the next one belongs to the next request with tasks
+          // (requests without tasks of this KS have pre[r + 1] == pre[r]); no binary search
+          do ++r; while (pre[r + 1] <= task);
+          m = 0;
+          cnt = pre[r + 1] - pre[r];
+          load_request(0);
+          unrank(0);
+        } else {
+          mask = gosper_next(mask);
+          c.idx_base += step * PK;
+        }
+      }
+      flush(done);
+    }  // grab loop
   }
-  flush();
-  }  // grab loop
   {  // measurement: candidates scored by this warp (ffs_search_scored)
     uint64_t e = c.n_scored;
 #pragma unroll
@@ -1354,6 +1274,240 @@ cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, in
                           cudaStream_t st) {
   return a.tables_global ? launch_search_t<true>(ks, verify, a, grid, block, smem, st)
                          : launch_search_t<false>(ks, verify, a, grid, block, smem, st);
+}
+
+// ====================================================================================
+// K1b: bounded mode -- group tables and live-mask compaction
+// ====================================================================================
+// One CTA per (function, availability pattern).  W(i, j) = the fastest admissible time of
+// stage [i, j): over the profiles p of the pattern with stage memory <= cap_p and time <=
+// the throughput floor (R38); a candidate's stage on p needs p admissible, so every
+// candidate's stage time is >= W (the multiplicity of p is ignored: still a lower bound).
+__global__ void __launch_bounds__(128) k_group_tables(const uint32_t* __restrict__ img, ImageLayout L,
+                                                      const uint32_t* __restrict__ gofs, uint32_t* __restrict__ grp) {
+  __shared__ uint32_t Wm[33 * 33];  // W(i, j) at [j * 33 + i]
+  __shared__ uint32_t h0[33], r2[33];
+  const uint32_t f = blockIdx.x, a = blockIdx.y;
+  const uint32_t row0 = img[L.o_fdesc + 4 * f], n = img[L.o_fdesc + 4 * f + 1], N1 = n + 1;
+  const uint32_t thr = img[L.o_thr + f];
+  uint32_t* g = grp + gofs[f] + a * grp_stride(n);
+  uint32_t *H0 = g, *T3 = g + N1, *R2 = g + 2 * N1, *R3 = g + 3 * N1, *Mt = g + 4 * N1;
+  auto X = [&](uint32_t j) { return img[L.o_xf + row0 + j - 1]; };  // cut at boundary j (after component j-1)
+  auto sat = [](uint64_t v) { return (uint32_t)(v < kGInf ? v : kGInf); };
+  for (uint32_t idx = threadIdx.x; idx < N1 * N1; idx += blockDim.x) {
+    const uint32_t i = idx % N1, j = idx / N1;
+    uint32_t w = kGInf;
+    if (i < j) {
+      const uint32_t mem = img[L.o_pm + row0 + j] - img[L.o_pm + row0 + i];
+      for (int p = 0; p < kP; ++p) {
+        if (!((a >> p) & 1u) || mem > img[L.o_cap + p]) continue;
+        const uint32_t t = pl_diff(img, L.o_pl + (row0 + j) * kRowW + p, L.o_pl + (row0 + i) * kRowW + p);
+        if (t <= thr) w = min(w, t);
+      }
+    }
+    Wm[j * 33 + i] = w;
+  }
+  __syncthreads();
+  for (uint32_t idx = threadIdx.x; idx < N1 * N1; idx += blockDim.x) {
+    const uint32_t i = idx % N1, j = idx / N1;
+    Mt[j * N1 + i] = (i < j && j < n && i >= 1) ? sat((uint64_t)Wm[j * 33 + i] + X(j)) : kGInf;
+  }
+  for (uint32_t j = threadIdx.x; j < N1; j += blockDim.x) {
+    const uint32_t h = (j >= 1 && j < n) ? sat((uint64_t)Wm[j * 33] + X(j)) : kGInf;
+    H0[j] = h;
+    h0[j] = h;
+    T3[j] = (j >= 1 && j < n) ? Wm[n * 33 + j] : kGInf;
+  }
+  __syncthreads();
+  for (uint32_t j = threadIdx.x; j < N1; j += blockDim.x) {
+    uint32_t m = kGInf;
+    if (j < n)
+      for (uint32_t i = 1; i < j; ++i) m = min(m, sat((uint64_t)h0[i] + Wm[j * 33 + i] + X(j)));
+    R2[j] = m;
+    r2[j] = m;
+  }
+  __syncthreads();
+  for (uint32_t j = threadIdx.x; j < N1; j += blockDim.x) {
+    uint32_t m = kGInf;
+    if (j < n)
+      for (uint32_t i = 2; i < j; ++i) m = min(m, sat((uint64_t)r2[i] + Wm[j * 33 + i] + X(j)));
+    R3[j] = m;
+  }
+}
+
+cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, const uint32_t* gofs, uint32_t* grp,
+                                cudaStream_t st) {
+  k_group_tables<<<dim3(lay.F, 32), 128, 0, st>>>(image, lay, gofs, grp);
+  return cudaGetLastError();
+}
+
+// colex rank of a (KS-1)-subset {j_1 < ... < j_{KS-1}} of the cut positions: sum C(j_i, i)
+__host__ __device__ __forceinline__ uint32_t c2(uint32_t x) { return x * (x - 1) / 2; }
+__host__ __device__ __forceinline__ uint32_t c3(uint32_t x) { return x * (x - 1) * (x - 2) / 6; }
+
+// K1b: live-mask compaction.  The segment's (request, cut mask) tasks are split exactly as
+// k_plan_search splits them (same chunks, same rank interleave); each lane walks its
+// piece in colex order and keeps the masks whose e2e lower bound
+//   LB = W(0,b1) + X(b1) + W(b1,b2) + X(b2) + ... + W(b_{KS-1}, n) <= B   (exact integers)
+// skipping a whole block of masks (fixed highest cut) or row (fixed two highest cuts) when
+// its best-case bound (R3 / R2 of the group tables) already exceeds the budget.  A mask
+// with LB > B holds no feasible candidate, so dropping it is exact.  Consecutive live masks
+// of one request are paired into one record {r, maskA, maskB, 0} (maskB = 0: single).
+// Lockstep: every lane takes one action per iteration (a block test, a row test, a mask
+// test, a request change or the end), so the warp stays converged at the emission point.
+template <int KS>
+__global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A) {
+  static_assert(KS >= 2 && KS <= 4, "k_live: KS = 2..4");
+  enum { kBlock = 0, kRow = 1, kMask = 2, kNext = 3, kEnd = 4 };
+  const uint32_t* img = A.image;
+  const ImageLayout& L = A.lay;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
+  const uint64_t T = pre[A.n_req];
+  const uint64_t NC = (uint64_t)A.warps_total * kdyn(KS) * A.world, NT = NC * 32;
+  const uint64_t Tq = T / NT, Tr = T % NT;
+  auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
+  unsigned long long* ctr = A.work_ctr + KS;
+  unsigned long long* lcount = A.work_ctr + kCtrListCount + KS;
+
+  for (;;) {
+    unsigned long long jg = 0;
+    if (lane == 0) jg = atomicAdd(ctr, 1ull);
+    jg = __shfl_sync(0xffffffffu, jg, 0);
+    const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
+    if (chunk >= NC) break;
+    const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
+    bool active = t0 < t1;
+    uint64_t task = t0;
+    uint32_t r = 0, m = 0, cnt = 0, n = 0, N1 = 0, B = 0, j1 = 0, j2 = 0, j3 = 0, rowc = 0, pend = 0, recR = 0;
+    const uint32_t* gp = nullptr;
+    int need = kEnd;
+    auto load = [&](uint32_t mm) {  // request r, rank mm within it
+      const ffs_request q = A.req[r];
+      n = img[L.o_fdesc + 4 * q.func + 1];
+      N1 = n + 1;
+      B = A.slo[r];
+      const uint64_t fb = A.node_free[q.node];
+      uint32_t av = 0;
+#pragma unroll
+      for (int p = 0; p < kP; ++p) av |= (((fb >> (8 * p)) & 255u) != 0u ? 1u : 0u) << p;
+      gp = A.grp + A.gofs[q.func] + av * grp_stride(n);
+      cnt = (uint32_t)(pre[r + 1] - pre[r]);
+      m = mm;
+      // colex unrank of mm
+      uint32_t x = n - 1;
+      if constexpr (KS == 4) {
+        while (c3(x) > mm) --x;
+        j3 = x;
+        mm -= c3(x);
+      }
+      if constexpr (KS >= 3) {
+        x = (KS == 4) ? j3 - 1 : n - 1;
+        while (c2(x) > mm) --x;
+        j2 = x;
+        mm -= c2(x);
+      }
+      j1 = mm;
+      need = KS == 4 ? kBlock : KS == 3 ? kRow : kMask;
+      pend = 0;
+    };
+    if (active) {
+      r = find_request(pre, A.n_req, task);
+      load((uint32_t)(task - pre[r]));
+    }
+    // move to rank mm (> m) of the current request; the caller sets the state for mm
+    auto jump = [&](uint32_t mm) {
+      task += mm - m;
+      m = mm;
+      if (task >= t1) need = kEnd;
+      else if (m == cnt) need = kNext;
+    };
+    while (__any_sync(0xffffffffu, active)) {
+      uint32_t recA = 0, recB = 0;
+      bool has = false;
+      if (active) {
+        recR = r;
+        const uint32_t b1 = j1 + 1, b2 = j2 + 1, b3 = j3 + 1;
+        if (need == kEnd || need == kNext) {
+          if (pend) {  // the request's last live mask has no partner
+            has = true;
+            recA = pend;
+            pend = 0;
+          }
+          if (need == kEnd) {
+            active = false;
+          } else {
+            do ++r; while (pre[r + 1] <= task);
+            load(0);
+          }
+        } else if (KS == 4 && need == kBlock) {
+          if ((uint64_t)gp[3 * N1 + b3] + gp[N1 + b3] > B) {  // R3[b3] + T3[b3]
+            jump(c3(j3 + 1));
+            if (need == kBlock) { j1 = 0; j2 = 1; j3 += 1; }
+          } else {
+            need = kRow;
+          }
+        } else if (KS >= 3 && need == kRow) {
+          // KS = 4: R2[b2] + Mt[b3][b2] + T3[b3];  KS = 3: R2[b2] + T3[b2]
+          rowc = KS == 4 ? gp[4 * N1 + b3 * N1 + b2] + gp[N1 + b3] : gp[N1 + b2];
+          if ((uint64_t)gp[2 * N1 + b2] + rowc > B) {
+            const uint32_t base = KS == 4 ? c3(j3) : 0u;
+            if (KS == 4 && j2 + 1 == j3) {  // last row of the block
+              jump(c3(j3 + 1));
+              if (need == kRow) { j1 = 0; j2 = 1; j3 += 1; need = kBlock; }
+            } else {
+              jump(base + c2(j2 + 1));
+              if (need == kRow) { j1 = 0; j2 += 1; }
+            }
+          } else {
+            need = kMask;
+          }
+        } else {  // kMask
+          uint64_t lb;
+          if constexpr (KS == 2) lb = (uint64_t)gp[b1] + gp[N1 + b1];  // H0 + T3
+          else lb = (uint64_t)gp[b1] + gp[4 * N1 + b2 * N1 + b1] + rowc;
+          if (lb <= B) {
+            const uint32_t mk = (1u << j1) | (KS >= 3 ? 1u << j2 : 0u) | (KS == 4 ? 1u << j3 : 0u);
+            if (pend) {
+              has = true;
+              recA = pend;
+              recB = mk;
+              pend = 0;
+            } else {
+              pend = mk;
+            }
+          }
+          jump(m + 1);
+          if (need == kMask) {  // colex successor
+            if (KS == 2 || j1 + 1 < j2) {
+              ++j1;
+            } else if (KS == 4 && j2 + 1 == j3) {
+              j1 = 0; j2 = 1; j3 += 1; need = kBlock;
+            } else {
+              j1 = 0; j2 += 1; need = kRow;
+            }
+          }
+        }
+      }
+      // warp-aggregated append
+      const uint32_t bal = __ballot_sync(0xffffffffu, has);
+      if (bal) {
+        uint32_t base = 0;
+        if (lane == 0) base = (uint32_t)atomicAdd(lcount, (unsigned long long)__popc(bal));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        const uint32_t slot = base + __popc(bal & ((1u << lane) - 1u));
+        if (has && slot < A.list_cap) A.list[slot] = make_uint4(recR, recA, recB, 0u);
+      }
+    }
+  }
+}
+
+cudaError_t launch_live(int ks, const LiveArgs& a, int grid, cudaStream_t st) {
+  if (ks == 2) k_live<2><<<grid, 256, 0, st>>>(a);
+  else if (ks == 3) k_live<3><<<grid, 256, 0, st>>>(a);
+  else if (ks == 4) k_live<4><<<grid, 256, 0, st>>>(a);
+  else return cudaErrorInvalidValue;
+  return cudaGetLastError();
 }
 
 // ====================================================================================

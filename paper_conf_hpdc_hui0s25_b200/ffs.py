@@ -86,6 +86,7 @@ _sig = {
     "ffs_debug_filter_misses": ([_vp, C.POINTER(C.c_uint64)], _i32),
     "ffs_set_search_mode": ([_vp, _u32], _i32),
     "ffs_search_scored": ([_vp, C.POINTER(C.c_uint64)], _i32),
+    "ffs_search_live_records": ([_vp, C.POINTER(C.c_uint64)], _i32),
     "ffs_bench_packed_peak": ([_vp, _u32, C.POINTER(C.c_double), C.POINTER(C.c_double)], _i32),
 }
 for _name, (_args, _res) in _sig.items():
@@ -376,6 +377,12 @@ class Planner:
     def set_search_mode(self, mode: int) -> None:
         """SEARCH_BOUNDED (default) or SEARCH_EXHAUSTIVE (every candidate scored)."""
         self._check(_lib.ffs_set_search_mode(self._h, int(mode)))
+
+    def live_records(self) -> list[int]:
+        """Live (request, mask pair) records of the bounded mode's compaction per ks."""
+        v = (C.c_uint64 * 8)()
+        self._check(_lib.ffs_search_live_records(self._h, v))
+        return [int(x) for x in v]
 
     def scored(self) -> list[int]:
         """Candidates scored per stage count (ks = 1..8) by the last plan_keys call."""

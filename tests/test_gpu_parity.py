@@ -228,6 +228,59 @@ def test_exhaustive_mode_scores_every_candidate(F, planner):
         planner.set_search_mode(7)
 
 
+@pytest.mark.parametrize("seed", range(16))
+def test_bounded_list_mode_chains(F, planner, seed):
+    """Production mode (exact SLO lower bounds: live-mask compaction + list search,
+    DESIGN.md §4.3) on random 4-7 component chains, K = 4, budgets from infeasible to
+    loose: keys and plans equal the oracle and the exhaustive mode."""
+    from test_bound_tables import random_chain_problem
+    prob = random_chain_problem(seed)
+    rng = W.SplitMix64(seed + 77)
+    reqs = np.repeat(prob.req, 6)
+    slo = rng.integers(20, 400, len(reqs)).astype(np.uint32)
+    prob = prob.with_requests(reqs, slo)
+    p, keys, _ = run_gpu(F, planner, prob, verify=False)
+    o = oracle.plan(prob, checks=False)
+    assert_plans_equal(p, o)
+    req, slo_d = F.to_device(prob)
+    planner.set_search_mode(F.SEARCH_EXHAUSTIVE)
+    try:
+        ex = planner.plan_keys(req, slo_d, prob.k_max).cpu().numpy()
+    finally:
+        planner.set_search_mode(F.SEARCH_BOUNDED)
+    np.testing.assert_array_equal(ex, o["key"])
+
+
+def test_bounded_list_path_and_fallback(F, planner):
+    """The bounded mode compacts live masks for KS = 2..4 and walks the records; a context
+    whose list is too small for a segment falls back to the task ranges inside the search
+    kernel -- same keys either way (C3 subset)."""
+    import os
+    prob = W.config3(R=16384)
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    K = prob.k_max
+    keys = planner.plan_keys(req, slo, K).cpu().numpy()
+    live = planner.live_records()
+    assert all(live[k] > 0 for k in (1, 2, 3)) and live[0] == 0 and sum(live[4:]) == 0
+    planner.set_search_mode(F.SEARCH_EXHAUSTIVE)
+    try:
+        ex = planner.plan_keys(req, slo, K).cpu().numpy()
+    finally:
+        planner.set_search_mode(F.SEARCH_BOUNDED)
+    np.testing.assert_array_equal(keys, ex)
+    os.environ["FFS_LIST_CAP"] = "16"
+    try:
+        small = F.Planner(0)
+    finally:
+        del os.environ["FFS_LIST_CAP"]
+    small.stage(prob)
+    k2 = small.plan_keys(req, slo, K).cpu().numpy()
+    assert small.live_records()[3] > 16  # KS = 4 overflowed: task-range fallback
+    np.testing.assert_array_equal(k2, ex)
+    small.close()
+
+
 def test_bad_requests_and_empty(F, planner):
     prob = random_tiny(1001)
     req = prob.req.copy()
