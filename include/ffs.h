@@ -434,9 +434,10 @@ ffs_status ffs_plan_frontier_any(ffs_ctx *ctx, const ffs_request *d_req, const u
  * timed launch's duration.  Synchronous. */
 ffs_status ffs_bench_int_peak(ffs_ctx *ctx, double *ops_per_s, double *seconds);
 /* Packed f16x2 microbenchmark over all SMs (roofline denominator of the KS = 4 pre-filter):
- * mode 0 = HFMA2 chains only (FMA-pipe rate), mode 1 = HFMA2 interleaved 1:1 with packed
- * max and LOP3 (ALU pipe): the issue-limited rate.  *lane_instr_per_s = measured
- * lane-instructions per second (each acts on two 16-bit halves).  Synchronous. */
+ * mode 0 = HFMA2 chains only (FMA-pipe rate), mode 1 = HFMA2 chains interleaved 1:1 with
+ * independent LOP3 chains, mode 2 = the same with packed max (HMNMX2): the issue-limited
+ * rate.  *lane_instr_per_s = measured lane-instructions per second (each acts on two 16-bit
+ * halves).  FFS_ERR_ARG for mode > 2.  Synchronous. */
 ffs_status ffs_bench_packed_peak(ffs_ctx *ctx, uint32_t mode, double *lane_instr_per_s, double *seconds);
 /* Device time (ms, CUDA events recorded on the launch stream around each launch) of each
  * search-kernel segment run since the last ffs_plan_keys / ffs_plan_keys_range call with

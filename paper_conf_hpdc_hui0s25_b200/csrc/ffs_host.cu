@@ -527,6 +527,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     la.n_req = n_req;
     la.rank = rank;
     la.world = world;
+    la.keys = d_keys;
     la.gofs = c->gofs.as<uint32_t>();
     la.grp = c->grp.as<uint32_t>();
     la.list = c->live_list.as<uint4>();
@@ -1281,7 +1282,7 @@ ffs_status ffs_search_live_records(ffs_ctx* c, uint64_t* per_ks) {
 }
 
 ffs_status ffs_bench_packed_peak(ffs_ctx* c, uint32_t mode, double* lane_instr_per_s, double* seconds) {
-  if (!c || !lane_instr_per_s || !seconds || mode > 1) return FFS_ERR_ARG;
+  if (!c || !lane_instr_per_s || !seconds || mode > 2) return FFS_ERR_ARG;
   DeviceGuard g(c->device);
   CK(run_packed_peak(c->sms, (int)mode, lane_instr_per_s, seconds), "packed peak kernel");
   return FFS_OK;

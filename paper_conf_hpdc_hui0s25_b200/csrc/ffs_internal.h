@@ -81,9 +81,10 @@ struct SearchArgs {
 };
 // work_ctr layout: [0..kMaxK] per-KS task-chunk grab counters; [kCtrScored + KS]
 // candidates the segment's kernel scored (every candidate whose own score it computed);
-// [kCtrListGrab + KS] record-chunk grab counters and [kCtrListCount + KS] live records
-// written by k_live (bounded mode)
-constexpr int kCtrScored = 16, kCtrListGrab = 24, kCtrListCount = 32, kCtrWords = 48;
+// [kCtrListGrab + KS] record-chunk grab counters, [kCtrListCount + KS] live records
+// written by k_live and [kCtrLiveGrab + KS] k_live's own task-chunk grab counters (bounded
+// mode)
+constexpr int kCtrScored = 16, kCtrListGrab = 24, kCtrListCount = 32, kCtrLiveGrab = 40, kCtrWords = 48;
 
 // Group tables of the bounded mode: per function f and availability
 // pattern a (bit p = the node has >= 1 free slice of profile p), with W(i, j) = the fastest
@@ -104,6 +105,7 @@ struct LiveArgs {
   const uint64_t* node_free;
   const uint64_t* prefix;
   uint32_t n_req, rank, world;
+  const int64_t* keys;          // best keys of the earlier segments (request-level CV test)
   const uint32_t* gofs;         // [F] word offset of function f's group tables
   const uint32_t* grp;
   uint4* list;

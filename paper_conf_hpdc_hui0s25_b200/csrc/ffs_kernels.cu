@@ -1367,7 +1367,7 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
   const uint64_t NC = (uint64_t)A.warps_total * kdyn(KS) * A.world, NT = NC * 32;
   const uint64_t Tq = T / NT, Tr = T % NT;
   auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
-  unsigned long long* ctr = A.work_ctr + KS;
+  unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;
   unsigned long long* lcount = A.work_ctr + kCtrListCount + KS;
 
   for (;;) {
@@ -1382,6 +1382,7 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
     uint32_t r = 0, m = 0, cnt = 0, n = 0, N1 = 0, B = 0, j1 = 0, j2 = 0, j3 = 0, rowc = 0, pend = 0, recR = 0;
     const uint32_t* gp = nullptr;
     int need = kEnd;
+    bool jump_dead = false;
     auto load = [&](uint32_t mm) {  // request r, rank mm within it
       const ffs_request q = A.req[r];
       n = img[L.o_fdesc + 4 * q.func + 1];
@@ -1394,6 +1395,12 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
       gp = A.grp + A.gofs[q.func] + av * grp_stride(n);
       cnt = (uint32_t)(pre[r + 1] - pre[r]);
       m = mm;
+      // request-level CV test (set_threshold's none_can_win): a best key of the earlier
+      // segments with cvq = 0 and fewer than KS stages cannot be beaten by any KS-stage
+      // candidate (R1: cvq, then k) -- every 1-stage plan has CV = 0 -- so the request's
+      // remaining masks are all dead
+      const uint64_t bk = (uint64_t)A.keys[r];
+      const bool dead = bk != kKeyNone && (bk >> 50) == 0 && (int)((bk >> 47) & 7) + 1 < KS;
       // colex unrank of mm
       uint32_t x = n - 1;
       if constexpr (KS == 4) {
@@ -1410,6 +1417,7 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
       j1 = mm;
       need = KS == 4 ? kBlock : KS == 3 ? kRow : kMask;
       pend = 0;
+      if (dead) jump_dead = true;
     };
     if (active) {
       r = find_request(pre, A.n_req, task);
@@ -1422,6 +1430,10 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
       if (task >= t1) need = kEnd;
       else if (m == cnt) need = kNext;
     };
+    if (jump_dead) {  // the first request of the piece is dead: skip to its end
+      jump_dead = false;
+      jump(cnt);
+    }
     while (__any_sync(0xffffffffu, active)) {
       uint32_t recA = 0, recB = 0;
       bool has = false;
@@ -1439,6 +1451,10 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
           } else {
             do ++r; while (pre[r + 1] <= task);
             load(0);
+            if (jump_dead) {
+              jump_dead = false;
+              jump(cnt);
+            }
           }
         } else if (KS == 4 && need == kBlock) {
           if ((uint64_t)gp[3 * N1 + b3] + gp[N1 + b3] > B) {  // R3[b3] + T3[b3]
@@ -2589,7 +2605,7 @@ cudaError_t launch_sim(const SimArgs& a, cudaStream_t st) {
 // ====================================================================================
 // K5: integer issue-rate microbenchmark (roofline denominator)
 // ====================================================================================
-constexpr int kPeakIters = 4096;
+constexpr int kPeakIters = 4096, kPeakReps = 16;
 __global__ void __launch_bounds__(256) k_int_peak(uint32_t seed, uint32_t* out) {
   // 8 independent chains of IADD3 / LOP3 / IMAD: 3 integer lane-ops per chain step.
   uint32_t a[8];
@@ -2622,9 +2638,10 @@ cudaError_t run_int_peak(int sms, double* ops, double* seconds) {
   cudaEventCreate(&a);
   cudaEventCreate(&b);
   const int blocks = sms * 8;  // 2048 threads per SM
-  k_int_peak<<<blocks, 256>>>(1u, d);  // warm-up
+  // ~100 ms of warm-up so the SM clock has ramped from idle, then 16 timed launches
+  for (int i = 0; i < 32; ++i) k_int_peak<<<blocks, 256>>>(1u, d);
   cudaEventRecord(a);
-  k_int_peak<<<blocks, 256>>>(2u, d);
+  for (int i = 0; i < kPeakReps; ++i) k_int_peak<<<blocks, 256>>>(2u, d);
   cudaEventRecord(b);
   e = cudaEventSynchronize(b);
   float ms = 0;
@@ -2634,15 +2651,16 @@ cudaError_t run_int_peak(int sms, double* ops, double* seconds) {
   cudaFree(d);
   if (e != cudaSuccess) return e;
   // 3 ops per chain step; IADD3 with an immediate counts 1, LOP3 1, IMAD 1
-  *ops = (double)blocks * 256.0 * kPeakIters * 4 * 8 * 3 / (ms * 1e-3);
+  *ops = (double)kPeakReps * blocks * 256.0 * kPeakIters * 4 * 8 * 3 / (ms * 1e-3);
   *seconds = ms * 1e-3;
   return cudaGetLastError();
 }
 
 // Packed f16x2 issue-rate microbenchmark (roofline denominator of the KS = 4 pre-filter,
-// DESIGN.md §5).  mode 0: eight independent HFMA2 chains (the FMA-pipe rate of the
-// packed datapath); mode 1: HFMA2 interleaved 1:1 with packed max (VHMNMX) and LOP3 on
-// the ALU pipe -- the issue-limited rate, one warp-instruction per SMSP per clock at best.
+// DESIGN.md §5).  mode 0: eight independent HFMA2 chains (the FMA-pipe rate of the packed
+// datapath); mode 1: eight HFMA2 chains interleaved with eight independent LOP3 chains (ALU
+// pipe); mode 2: the same with packed max (HMNMX2) on the ALU side -- modes 1 and 2 measure
+// the issue-limited rate, one warp-instruction per SMSP per clock at best.
 template <int MODE>
 __global__ void __launch_bounds__(256) k_packed_peak(uint32_t seed, uint32_t* out) {
   uint32_t h[8], m[8];
@@ -2651,7 +2669,7 @@ __global__ void __launch_bounds__(256) k_packed_peak(uint32_t seed, uint32_t* ou
     h[i] = 0x3c003c00u ^ ((seed + threadIdx.x + i) & 0x00ff00ffu);
     m[i] = h[i] ^ 0x04000400u;
   }
-  const uint32_t a = 0x3bff3bffu ^ (seed & 1u), b = 0x10001000u | (seed & 2u);
+  const uint32_t a = 0x3bff3bffu ^ (seed & 1u), b = 0x10001000u | (seed & 2u), c = 0x12340000u ^ seed;
 #pragma unroll 1
   for (int it = 0; it < kPeakIters; ++it) {
 #pragma unroll
@@ -2659,11 +2677,8 @@ __global__ void __launch_bounds__(256) k_packed_peak(uint32_t seed, uint32_t* ou
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         asm volatile("fma.rn.f16x2 %0, %0, %1, %2;" : "+r"(h[i]) : "r"(a), "r"(b));
-        if (MODE == 1) {
-          asm volatile("max.f16x2 %0, %0, %1;" : "+r"(m[i]) : "r"(h[i]));
-          asm volatile("lop3.b32 %0, %0, %1, %2, 0xE8;" : "+r"(m[i]) : "r"(a), "r"(h[(i + 1) & 7]));
-          asm volatile("fma.rn.f16x2 %0, %0, %1, %2;" : "+r"(h[i]) : "r"(a), "r"(b));
-        }
+        if (MODE == 1) asm volatile("lop3.b32 %0, %0, %1, %2, 0x96;" : "+r"(m[i]) : "r"(a), "r"(c));
+        if (MODE == 2) asm volatile("max.f16x2 %0, %0, %1;" : "+r"(m[i]) : "r"(c));
       }
     }
   }
@@ -2683,11 +2698,12 @@ cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double*
   const int blocks = sms * 8;  // 2048 threads per SM
   auto launch = [&](uint32_t seed) {
     if (mode == 0) k_packed_peak<0><<<blocks, 256>>>(seed, d);
-    else k_packed_peak<1><<<blocks, 256>>>(seed, d);
+    else if (mode == 1) k_packed_peak<1><<<blocks, 256>>>(seed, d);
+    else k_packed_peak<2><<<blocks, 256>>>(seed, d);
   };
-  launch(1u);  // warm-up
+  for (int i = 0; i < 32; ++i) launch(1u);  // ~100 ms warm-up: clocks ramped from idle
   cudaEventRecord(a);
-  launch(2u);
+  for (int i = 0; i < kPeakReps; ++i) launch(2u);
   cudaEventRecord(b);
   e = cudaEventSynchronize(b);
   float ms = 0;
@@ -2696,8 +2712,8 @@ cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double*
   cudaEventDestroy(b);
   cudaFree(d);
   if (e != cudaSuccess) return e;
-  const double per_step = mode == 0 ? 1.0 : 4.0;  // lane-instructions per chain step
-  *lane_instr_per_s = (double)blocks * 256.0 * kPeakIters * 4 * 8 * per_step / (ms * 1e-3);
+  const double per_step = mode == 0 ? 1.0 : 2.0;  // lane-instructions per chain step
+  *lane_instr_per_s = (double)kPeakReps * blocks * 256.0 * kPeakIters * 4 * 8 * per_step / (ms * 1e-3);
   *seconds = ms * 1e-3;
   return cudaGetLastError();
 }

@@ -138,9 +138,9 @@ class Planner:
         self.k_max = None
 
     def close(self):
-        if getattr(self, "_h", None):
+        if getattr(self, "_h", None) and _lib is not None:  # (module globals may be gone at exit)
             _lib.ffs_destroy(self._h)
-            self._h = None
+        self._h = None
 
     __del__ = close
 

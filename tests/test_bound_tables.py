@@ -62,11 +62,11 @@ def random_chain_problem(seed):
     rng = W.SplitMix64(seed)
     funcs = []
     for _ in range(2):
-        n = int(rng.integers(4, 8, 1)[0])
+        n = int(rng.integers(4, 7, 1)[0])
         funcs.append(dict(lat=rng.integers(1, 80, n * 5).reshape(n, 5).tolist(),
                           mem=rng.integers(1000, 30000, n).tolist(),
                           xfer=rng.integers(0, 40, n).tolist(), load=0))
-    nodes = [[[int(p) for p in rng.integers(0, 5, 3)], [(int(rng.integers(0, 5, 1)[0]), 1)]] for _ in range(2)]
+    nodes = [[[int(p) for p in rng.integers(0, 4, 3)], [(int(rng.integers(0, 4, 1)[0]), 1)]] for _ in range(2)]
     reqs = [(f, v, 10 ** 6) for f in range(2) for v in range(2)]
     return problem(funcs, nodes, reqs, k_max=4)
 
