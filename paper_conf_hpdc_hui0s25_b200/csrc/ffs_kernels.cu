@@ -1890,8 +1890,8 @@ cudaError_t launch_decode(const DecodeArgs& a, cudaStream_t st) {
 // ====================================================================================
 // K3: hotness-aware eviction score (A7)
 // ====================================================================================
-__device__ __forceinline__ void evict_one(const ffs_instance& in, uint32_t i, uint64_t now,
-                                          const ffs_evict_params& p, int64_t* score, uint8_t* state, uint64_t gi) {
+__device__ __forceinline__ int64_t evict_one(const ffs_instance& in, uint32_t i, uint64_t now,
+                                             const ffs_evict_params& p, int64_t* score, uint8_t* state, uint64_t gi) {
   const uint64_t idle = now >= in.last_used_us ? now - in.last_used_us : 0;
   uint8_t st;
   if (idle >= p.cold_after_us) st = FFS_ST_COLD;
@@ -1903,8 +1903,10 @@ __device__ __forceinline__ void evict_one(const ffs_instance& in, uint32_t i, ui
   // a time-sharing instance has idle < cold_after_us < 2^43 (host-checked), so
   // (cold_after - idle) packs into 43 bits whatever the timestamps' epoch
   const bool evictable = st == FFS_ST_TIME_SHARING && !(in.flags & FFS_INST_BUSY) && i < (1u << 20);
-  score[gi] = evictable ? (int64_t)(((p.cold_after_us - idle) << 20) | i) : (int64_t)kKeyNone;
+  const int64_t sc = evictable ? (int64_t)(((p.cold_after_us - idle) << 20) | i) : (int64_t)kKeyNone;
+  score[gi] = sc;
   state[gi] = st;
+  return sc;
 }
 
 // one CTA per tick; kEvU records in flight per thread (memory-level parallelism).  (A flat
@@ -1916,13 +1918,27 @@ __device__ __forceinline__ void evict_one(const ffs_instance& in, uint32_t i, ui
 #define FFS_EVU 5  // 640 >= the ~582 instances of a C4 tick: one round of loads per CTA (0.545 -> 0.567 of the copy peak)
 #endif
 constexpr int kEvT = FFS_EVT, kEvU = FFS_EVU;
+// TAB (ffs_evict_step): the CTA also folds every scored instance into the tick's
+// (node, slice profile) minima in shared memory (64-bit atomicMin) and writes that row of
+// the victim table once -- the victim pass then reads <= 5 cells per load instead of
+// re-reading the tick's scores and records.  ~0 marks an empty cell.
+template <bool TAB>
 __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __restrict__ inst,
                                                        const uint32_t* __restrict__ tick_off,
                                                        const uint64_t* __restrict__ now_us, ffs_evict_params prm,
-                                                       int64_t* __restrict__ score, uint8_t* __restrict__ state) {
+                                                       int64_t* __restrict__ score, uint8_t* __restrict__ state,
+                                                       const uint16_t* __restrict__ slice_node,
+                                                       const uint8_t* __restrict__ slice_prof, uint32_t n_slices,
+                                                       uint32_t n_nodes, unsigned long long* __restrict__ tab) {
+  extern __shared__ unsigned long long cell[];
   const uint32_t t = blockIdx.x;
   const uint32_t b = tick_off[t], e = tick_off[t + 1];
   const uint64_t now = now_us[t];
+  const uint32_t ncell = n_nodes * kP;
+  if constexpr (TAB) {
+    for (uint32_t i = threadIdx.x; i < ncell; i += kEvT) cell[i] = ~0ull;
+    __syncthreads();
+  }
   for (uint32_t g0 = b + threadIdx.x; g0 < e; g0 += kEvT * kEvU) {
     ffs_instance in[kEvU];
 #pragma unroll
@@ -1931,8 +1947,20 @@ __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __rest
 #pragma unroll
     for (int u = 0; u < kEvU; ++u) {
       const uint32_t gi = g0 + u * kEvT;
-      if (gi < e) evict_one(in[u], gi - b, now, prm, score, state, gi);
+      if (gi < e) {
+        const int64_t sc = evict_one(in[u], gi - b, now, prm, score, state, gi);
+        if (TAB && (uint64_t)sc != kKeyNone) {
+          const int32_t sl = in[u].slice;
+          if (sl >= 0 && (uint32_t)sl < n_slices)
+            atomicMin(cell + (uint32_t)slice_node[sl] * kP + slice_prof[sl], (unsigned long long)sc);
+        }
+      }
     }
+  }
+  if constexpr (TAB) {
+    __syncthreads();
+    unsigned long long* row = tab + (uint64_t)t * ncell;
+    for (uint32_t i = threadIdx.x; i < ncell; i += kEvT) row[i] = cell[i];
   }
 }
 
@@ -1949,7 +1977,9 @@ cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32
                          uint32_t n_ticks, uint64_t now_single, ffs_evict_params prm, int64_t* score, uint8_t* state,
                          cudaStream_t st) {
   if (tick_off) {
-    if (n_ticks) k_evict_ticks<<<n_ticks, kEvT, 0, st>>>(inst, tick_off, now_us, prm, score, state);
+    if (n_ticks)
+      k_evict_ticks<false><<<n_ticks, kEvT, 0, st>>>(inst, tick_off, now_us, prm, score, state, nullptr, nullptr, 0,
+                                                     0, nullptr);
   } else if (n_inst) {
     int blocks = (int)((n_inst + 255) / 256);
     k_evict_one<<<blocks, 256, 0, st>>>(inst, n_inst, now_single, prm, score, state);
@@ -2054,6 +2084,28 @@ __global__ void __launch_bounds__(256) k_victim_pick(const uint32_t* __restrict_
       if ((okp >> p) & 1u) bs = min(bs, cell[p]);
   }
   victim[r] = bs == ~0ull ? -1 : (int32_t)(bs & 0xFFFFFull);
+}
+
+// ffs_evict_step: scores + states + the per-tick victim table in one pass, then the picks
+cudaError_t launch_evict_step(const uint32_t* image, const ImageLayout& lay, const ffs_instance* inst,
+                              const uint32_t* tick_off, const uint64_t* now_us, uint32_t n_ticks, ffs_evict_params prm,
+                              int64_t* score, uint8_t* state, const uint16_t* slice_node, const uint8_t* slice_prof,
+                              uint32_t n_slices, uint32_t n_nodes, unsigned long long* tab, const ffs_request* req,
+                              const uint32_t* slo, const uint32_t* req_tick, uint32_t n_req, int32_t* victim,
+                              cudaStream_t st) {
+  if (n_ticks) {
+    const size_t sm = (size_t)n_nodes * kP * 8;
+    if (sm > 48 * 1024) {
+      cudaError_t e = cudaFuncSetAttribute(k_evict_ticks<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+      if (e != cudaSuccess) return e;
+    }
+    k_evict_ticks<true><<<n_ticks, kEvT, sm, st>>>(inst, tick_off, now_us, prm, score, state, slice_node, slice_prof,
+                                                   n_slices, n_nodes, tab);
+  }
+  if (n_req)
+    k_victim_pick<<<(n_req + 255) / 256, 256, 0, st>>>(image, lay, req, slo, req_tick, n_req, n_ticks, n_nodes, tab,
+                                                       victim);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_victims(const uint32_t* image, const ImageLayout& lay, const ffs_request* req, const uint32_t* slo,

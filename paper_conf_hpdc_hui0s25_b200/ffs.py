@@ -71,6 +71,8 @@ _sig = {
     "ffs_evict_scores": ([_vp, _vp, _u32, _u64, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
+    "ffs_evict_step": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp, _vp, _vp, _u32, _vp, _vp],
+                       _i32),
     "ffs_plan_joint": ([_vp, _vp, _vp, _u32, _u32, _vp, C.POINTER(C.c_uint32), _vp], _i32),
     "ffs_simulate": ([_vp, _vp, _vp, _vp, _u32, _u64, _u32, _u32, _u32, _u64, _vp, _vp, _vp, _vp, _vp, _vp], _i32),
     "ffs_route": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
@@ -255,6 +257,21 @@ class Planner:
                                            _ptr(tick_off), _ptr(score), int(tick_off.numel() - 1), _ptr(victim),
                                            _stream(stream)))
         return victim
+
+    def evict_step(self, inst, tick_off, now_us, req, slo, req_tick, score=None, state=None, victim=None, stream=None,
+                   **params):
+        """Scores + states of every tick's instances and the victims of the loads, fused."""
+        import torch
+        n = int(inst.numel() // W.INST_DTYPE.itemsize)
+        nr = int(slo.numel())
+        score = torch.empty(n, dtype=torch.int64, device=inst.device) if score is None else score
+        state = torch.empty(n, dtype=torch.uint8, device=inst.device) if state is None else state
+        victim = torch.empty(nr, dtype=torch.int32, device=inst.device) if victim is None else victim
+        prm = self._params(**params)
+        self._check(_lib.ffs_evict_step(self._h, _ptr(inst), _ptr(tick_off), _ptr(now_us), int(now_us.numel()),
+                                        C.byref(prm), _ptr(score), _ptr(state), _ptr(req), _ptr(slo), _ptr(req_tick),
+                                        nr, _ptr(victim), _stream(stream)))
+        return score, state, victim
 
     # ---- NEXT-2: joint commit (P:364, P:374) -------------------------------------------------
     def plan_joint(self, req, slo, k_max: int, out=None, stream=None):

@@ -3,8 +3,8 @@
 field.  Writes gpurun_out/full_parity_<cfg>.json.  One-off evidence run (C5 takes ~40 min of
 oracle time on 16 host cores); the sampled versions are in tests/test_gpu_parity.py.
 
-    python tests/full_parity.py 3 5   (test infrastructure: the only place besides the test suite
-    that runs the oracle at full size)
+    python tests/full_parity.py 3 5 [--exhaustive]   (test infrastructure: the only place
+    besides the test suite that runs the oracle at full size; tools/run_full_parity.sh)
 """
 import json
 import os
@@ -24,7 +24,10 @@ def main():
     import torch
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
     pl = ffs.Planner(0)
-    for cfg in [int(x) for x in sys.argv[1:]] or [3]:
+    exhaustive = "--exhaustive" in sys.argv
+    if exhaustive:
+        pl.set_search_mode(ffs.SEARCH_EXHAUSTIVE)
+    for cfg in [int(x) for x in sys.argv[1:] if not x.startswith("--")] or [3]:
         prob = W.CONFIGS[cfg]()
         pl.stage(prob)
         req, slo = ffs.to_device(prob)
@@ -49,7 +52,8 @@ def main():
                   flush=True)
         cpu_s = time.perf_counter() - t
         st = p["status"]
-        res = {"config": f"C{cfg}", "requests": prob.R, "mismatched_fields": mism,
+        res = {"config": f"C{cfg}", "mode": "exhaustive" if exhaustive else "bounded", "requests": prob.R,
+               "mismatched_fields": mism,
                "bit_exact": all(v == 0 for v in mism.values()), "gpu_s": gpu_s, "oracle_s": cpu_s,
                "oracle_threads": os.cpu_count(), "ok": int((st == 0).sum()), "infeasible": int((st == 1).sum()),
                "multi_stage": int(((st == 0) & (p["k"] > 1)).sum())}

@@ -333,7 +333,10 @@ def test_host_entry_point_matches(F, planner):
 
 
 def test_eviction_scores_and_victims(F, planner):
-    wl = W.config4(T=64)
+    """C4 at full size: every instance score and state of all 4096 ticks and the victim
+    of every load, against the oracle."""
+    wl = W.config4()
+    assert len(wl.now_us) == 4096
     prob = wl.problem
     planner.stage(prob)
     inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
@@ -355,6 +358,29 @@ def test_eviction_scores_and_victims(F, planner):
         v_o = oracle.victim(sub, np.full(len(rs), oracle.PLAN_INFEASIBLE, np.int32), wl.inst[a:b], ev)
         np.testing.assert_array_equal(vic[rs], v_o)
     assert (vic >= 0).sum() > 0
+
+
+def test_evict_step_fused_matches_separate_calls(F, planner):
+    """ffs_evict_step (scores + per-tick victim table in one pass, then picks) equals
+    ffs_evict_scores_ticks + ffs_evict_victims bit for bit on C4 (all 4096 ticks), also
+    with loads whose tick is out of range and with no loads at all."""
+    wl = W.config4()
+    prob = wl.problem
+    planner.stage(prob)
+    inst = torch.from_numpy(wl.inst.view(np.uint8)).cuda()
+    toff = torch.from_numpy(wl.tick_off.view(np.int32)).cuda()
+    now = torch.from_numpy(wl.now_us.view(np.int64)).cuda()
+    req, slo = F.to_device(prob)
+    rt_np = wl.req_tick.astype(np.uint32).copy()
+    rt_np[::13] = len(wl.now_us) + 1
+    rt = torch.from_numpy(rt_np.view(np.int32)).cuda()
+    s1, st1 = planner.evict_scores_ticks(inst, toff, now, window_us=wl.window_us)
+    v1 = planner.evict_victims(req, slo, rt, inst, toff, s1)
+    s2, st2, v2 = planner.evict_step(inst, toff, now, req, slo, rt, window_us=wl.window_us)
+    assert torch.equal(s1, s2) and torch.equal(st1, st2) and torch.equal(v1, v2)
+    assert int((v2 >= 0).sum()) > 0 and bool((v2[::13] == -1).all())
+    s3, st3, _ = planner.evict_step(inst, toff, now, req[:0], slo[:0], rt[:0], window_us=wl.window_us)
+    assert torch.equal(s1, s3) and torch.equal(st1, st3)
 
 
 def test_eviction_epoch_timestamps_and_range(F, planner):
