@@ -359,11 +359,17 @@ def run_sim(pl):
     torch.cuda.synchronize()
     ms = a.elapsed_time(b)
     c = ctr.cpu().numpy().sum(axis=0)
+    # the same trace with monolithic instances only (no pipelines, R44-R46 off): the
+    # FluidFaaS mechanism's effect on the simulated SLO hit rate
+    c0 = pl.simulate(tr, k_max=0)[0].cpu().numpy().sum(axis=0)
     return {"metric": "simulated_requests_per_s", "value": float(c[0]) / (ms * 1e-3), "unit": "requests/s",
             "ms": ms, "ticks": tr.T, "nodes": int(tr.problem.n_nodes), "functions": int(tr.problem.F),
             "requests": int(c[0]), "served": int(c[1]), "slo_hit_rate": float(c[2]) / max(1, int(c[0])),
             "reloads": int(c[4]), "evictions": int(c[5]), "cold_terminations": int(c[6]),
-            "slice_ticks_occupied": int(c[7])}
+            "slice_ticks_occupied": int(c[7]), "pipelines_placed": int(c[8]), "pipeline_migrations": int(c[9]),
+            "served_by_pipelines": int(c[10]), "pipeline_slice_ticks": int(c[11]),
+            "monolithic_only": {"served": int(c0[1]), "slo_hit_rate": float(c0[2]) / max(1, int(c0[0])),
+                                "evictions": int(c0[5])}}
 
 
 def measure_peaks(pl):

@@ -400,20 +400,30 @@ ffs_status ffs_route(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_s
  * state belong to other tenants).  Per node every function has at most one instance;
  * the requests of node v and tick t are d_req_func/d_req_budget[d_req_off[v*n_ticks+t] ..
  * d_req_off[v*n_ticks+t+1]) and are served in that order: a resident instance serves
- * (latency = its execution time on its slice); otherwise the instance is loaded on the
- * free slice of smallest (capacity, gpcs, id) that holds the function, else on the slice
- * of the least-recently-used time-sharing instance of another function not used in this
- * tick (evicted to warm), latency = reload + execution; otherwise the request is
- * unserved.  Every window_ticks an instance becomes exclusive hot (not evictable) iff its
- * busy time reached thr_pct % of the window; instances idle >= cold_after_us terminate
- * (R31-R36).  Outputs (device): d_ctr uint64[n_nodes][8] = requests, served,
- * SLO hits, unserved, reloads, evictions, terminations, occupied slice-ticks; final
- * per (node, function): d_slice int32, d_state uint8 (FFS_ST_*), d_last uint64,
- * d_busy uint32 (all [n_nodes][n_funcs]).  Asynchronous. */
+ * (latency = its execution time on its slice, or its plan's e2e for a pipeline);
+ * otherwise the instance is built "adaptive based on available resources": on the
+ * free slice of smallest (capacity, gpcs, id) that holds the function; else, when k_max >=
+ * 2, as a PIPELINE over the node's free slices -- the argmin plan of ffs_plan_keys for the
+ * request's budget, slices bound as ffs_plan_decode, exclusive hot and never evicted
+ * (P:358); else on the slice of the least-recently-used time-sharing instance of another
+ * function not used in this tick (evicted to warm); latency = reload + execution
+ * (e2e); otherwise the request is unserved.  Every window_ticks an instance becomes
+ * exclusive hot (not evictable) iff its busy time reached thr_pct % of the window;
+ * instances idle >= cold_after_us terminate; then every pipeline for which a free slice
+ * holds the whole function migrates to a non-pipeline instance on the smallest such slice
+ * (a reload) and releases its slices (R31-R36, R44-R46).  k_max = 0
+ * simulates monolithic instances only.  Outputs (device): d_ctr uint64[n_nodes][12] =
+ * requests, served, SLO hits, unserved, reloads, evictions, terminations, occupied
+ * slice-ticks, pipelines placed, migrations, requests served by pipelines, pipeline
+ * slice-ticks; final per (node, function): d_slice int32 (a pipeline's stage-0 slice),
+ * d_state uint8 (FFS_ST_*), d_last uint64, d_busy uint32, d_stages uint8 (0 none, 1
+ * monolithic, k pipeline; all [n_nodes][n_funcs]).  FFS_ERR_RANGE: k_max > 8 or as
+ * ffs_plan_keys for k_max >= 2.  Asynchronous. */
 ffs_status ffs_simulate(ffs_ctx *ctx, const uint32_t *d_req_off, const uint32_t *d_req_func,
                         const uint32_t *d_req_budget, uint32_t n_ticks, uint64_t t0_us, uint32_t tick_us,
-                        uint32_t window_ticks, uint32_t thr_pct, uint64_t cold_after_us, uint64_t *d_ctr,
-                        int32_t *d_slice, uint8_t *d_state, uint64_t *d_last, uint32_t *d_busy, void *stream);
+                        uint32_t window_ticks, uint32_t thr_pct, uint64_t cold_after_us, uint32_t k_max,
+                        uint64_t *d_ctr, int32_t *d_slice, uint8_t *d_state, uint64_t *d_last, uint32_t *d_busy,
+                        uint8_t *d_stages, void *stream);
 
 /* ---- NEXT-3: frontier precompute ------------------------------------------------------
  * For a fixed (function, node free-vector) the feasible set depends on the budget only

@@ -252,20 +252,23 @@ def route(prob, inst_func, inst_state, inst_lat, inst_cap) -> np.ndarray:
     return out
 
 
-def sim(trace, thr_pct: int = 30, cold_after_us: int = 600_000_000):
-    """NEXT-4 time-sharing simulator (ffs_oracle.c: oracle_sim).  Returns (ctr[N, 8],
-    slice[N, F], state[N, F], last_used[N, F], busy[N, F])."""
+def sim(trace, thr_pct: int = 30, cold_after_us: int = 600_000_000, k_max: int | None = None):
+    """NEXT-4 time-sharing simulator with pipeline instances and migration (ffs_oracle.c:
+    oracle_sim).  Returns (ctr[N, 12], slice[N, F], state[N, F], last_used[N, F], busy[N, F],
+    stages[N, F]).  k_max = pipeline search depth (default the problem's; 0: monolithic
+    instances only -- the search then has no candidate)."""
     prob = trace.problem
-    h = _Held(prob, prob.k_max, False)
+    h = _Held(prob, int(prob.k_max if k_max is None else k_max), False)
     N, F = int(prob.n_nodes), int(prob.comp_off.shape[0] - 1)
     off, fu, bu = _c(trace.req_off, np.uint32), _c(trace.req_func, np.uint32), _c(trace.req_budget, np.uint32)
-    ctr = np.zeros((N, 8), np.uint64)
+    ctr = np.zeros((N, 12), np.uint64)
     fs, fst = np.zeros((N, F), np.int32), np.zeros((N, F), np.uint8)
     fl, fb = np.zeros((N, F), np.uint64), np.zeros((N, F), np.uint32)
+    fk = np.zeros((N, F), np.uint8)
     lib().oracle_sim(C.byref(h.args), C.c_int(trace.T), _p(off), _p(fu), _p(bu), C.c_uint64(trace.t0_us),
                      C.c_uint32(trace.tick_us), C.c_uint32(trace.window_ticks), C.c_uint32(thr_pct),
-                     C.c_uint64(cold_after_us), _p(ctr), _p(fs), _p(fst), _p(fl), _p(fb))
-    return ctr, fs, fst, fl, fb
+                     C.c_uint64(cold_after_us), _p(ctr), _p(fs), _p(fst), _p(fl), _p(fb), _p(fk))
+    return ctr, fs, fst, fl, fb, fk
 
 
 class Evict(NamedTuple):

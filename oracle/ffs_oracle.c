@@ -770,29 +770,45 @@ int oracle_route(const oracle_plan_args *a, int n_inst, const uint32_t *inst_fun
 }
 
 /* ---- NEXT-4: time-sharing simulator (Fig. 8) -------------------------------
- * DESIGN.md R31-R36.  Each node (invoker) is simulated independently; per node every
- * function has at most one instance (created on its first request there, time-sharing).
- * Ticks of tick_us; the requests of a tick are served in trace order:
- *   resident instance            -> served, latency = exec on its slice's profile;
- *   otherwise (warm / new)       -> placed on the free slice with the smallest (capacity,
- *     gpcs, id) that holds the function, else on the slice of the least recently used
- *     (ties: lower slice) time-sharing instance of another function not used in this tick
- *     whose slice holds the function (the victim goes warm: "selects the least-recently-
- *     used (LRU) instance for eviction, reloads the pertinent instance, and fulfills the
- *     request"), latency = load + exec; otherwise unserved.  A served request is an
- *     SLO hit when its latency <= its budget.
- *   A served request adds exec to the instance's busy time and sets its last use to now.
+ * DESIGN.md R31-R36, R44-R46.  Each node (invoker) is simulated independently; per node
+ * every function has at most one instance (created on its first request there).  Ticks of
+ * tick_us; the requests of a tick are served in trace order:
+ *   resident monolithic instance -> served, latency = exec on its slice's profile;
+ *   resident pipeline instance   -> served, latency = the plan's e2e (R45);
+ *   otherwise (warm / new): "the construction of that instance should be flexible and
+ *     adaptive based on available resources ... a two-stage or three-stage pipeline, or ...
+ *     a non-pipeline process":
+ *     (1) the free slice with the smallest (capacity, gpcs, id) that holds the function
+ *         (monolithic, time-sharing), latency = load + exec (R33);
+ *     (2) else a PIPELINE over the node's free slices: the argmin plan of the search
+ *         (oracle_plan, R1) with the request's budget, slices bound per R11; pipeline
+ *         instances are exclusive hot and never evicted ("All pipeline instances are in the
+ *         exclusive hot state"), latency = load + e2e (R44);
+ *     (3) else the slice of the least recently used (ties: lower slice) time-sharing
+ *         instance of another function not used in this tick whose slice holds the
+ *         function (the victim goes warm: P:364), latency = load + exec (R33);
+ *     otherwise unserved.  A served request is an SLO hit when its latency <= its budget.
+ *   A served request adds its service time (exec, or e2e for a pipeline) to the instance's
+ *   busy time and sets its last use to now.
  * At the end of every tick the occupied slices are counted; every window_ticks the
  * instances whose busy time reached thr% of the window become exclusive hot (exempt from
  * eviction) for the next window, the others time-sharing, busy resets;
- * instances idle >= cold_after are terminated.
+ * instances idle >= cold_after are terminated, releasing their slices; then
+ * every pipeline instance (function order) for which a free slice now holds the whole
+ * function migrates to a new non-pipeline instance on the smallest such slice and releases
+ * its slices ("migrates pipeline instances to non-pipeline instances when large MIG
+ * slices become available"); the new instance loads its model (a reload) and keeps the
+ * function's hotness (R46).
  * Slices busy in the staged cluster belong to other tenants and are never used.
- * ctr[v][8] = requests, served, SLO hits, unserved, reloads, evictions, terminations,
- * occupied slice-ticks.  Final per (node, function): slice, state, last use, busy. */
+ * ctr[v][12] = requests, served, SLO hits, unserved, reloads, evictions, terminations,
+ * occupied slice-ticks, pipelines placed, migrations, requests served by a pipeline
+ * (including the one that placed it), pipeline slice-ticks.  Final per (node, function): slice (a pipeline: its stage-0
+ * slice), state, last use, busy, stages (0 none, 1 monolithic, k >= 2 pipeline). */
+#define SIM_CTR 12
 int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const uint32_t *req_func,
                const uint32_t *req_budget, uint64_t t0_us, uint32_t tick_us, uint32_t window_ticks,
                uint32_t thr_pct, uint64_t cold_after_us, uint64_t *ctr, int32_t *fin_slice, uint8_t *fin_state,
-               uint64_t *fin_last, uint32_t *fin_busy) {
+               uint64_t *fin_last, uint32_t *fin_busy, uint8_t *fin_k) {
     const int F = a->F, P = a->P;
     /* per function: exec on each profile, total memory, reload */
     uint64_t *exec = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)F * (size_t)P);
@@ -807,15 +823,43 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
             exec[(size_t)f * P + p] = t;
         }
     }
-    int *res = (int *)malloc(sizeof(int) * (size_t)(a->n_slices > 0 ? a->n_slices : 1));
+    const int NS = a->n_slices > 0 ? a->n_slices : 1;
+    int *res = (int *)malloc(sizeof(int) * (size_t)NS);
+    uint8_t *occ = (uint8_t *)malloc((size_t)NS);
+    /* one-request plan arguments for the pipeline search (R44): the staged tables, the
+     * simulated slice occupancy as "busy" */
+    oracle_plan_args b = *a;
+    uint32_t q_func = 0, q_node = 0, q_slo = 0;
+    int64_t o_key;
+    int32_t o_status, o_k, o_slice[8];
+    uint32_t o_cut, o_e2e, o_bott, o_g, o_cvq;
+    uint8_t o_prof[8];
+    b.R = 1;
+    b.req_func = &q_func;
+    b.req_node = &q_node;
+    b.req_slo_us = &q_slo;
+    b.key = &o_key;
+    b.status = &o_status;
+    b.k = &o_k;
+    b.slice = o_slice;
+    b.cut_mask = &o_cut;
+    b.e2e_us = &o_e2e;
+    b.bottleneck_us = &o_bott;
+    b.gpcs_out = &o_g;
+    b.cvq = &o_cvq;
+    b.prof = o_prof;
+    b.checks = NULL;
     for (int v = 0; v < a->n_nodes; v++) {
-        uint64_t *C = ctr + (size_t)v * 8;
-        for (int i = 0; i < 8; i++) C[i] = 0;
+        uint64_t *C = ctr + (size_t)v * SIM_CTR;
+        for (int i = 0; i < SIM_CTR; i++) C[i] = 0;
         int32_t *sl = fin_slice + (size_t)v * F;
         uint8_t *st = fin_state + (size_t)v * F;
         uint64_t *last = fin_last + (size_t)v * F;
         uint32_t *busy = fin_busy + (size_t)v * F;
         uint8_t *exists = (uint8_t *)calloc((size_t)F, 1), *hot = (uint8_t *)calloc((size_t)F, 1);
+        uint8_t *pk = (uint8_t *)calloc((size_t)F, 1); /* pipeline stages, 0 = no pipeline */
+        int32_t *psl = (int32_t *)malloc(sizeof(int32_t) * (size_t)F * 8);
+        uint64_t *pe2e = (uint64_t *)calloc((size_t)F, sizeof(uint64_t));
         for (int f = 0; f < F; f++) {
             sl[f] = -1;
             last[f] = 0;
@@ -841,7 +885,13 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
                     ex = exec[(size_t)f * P + a->sl_prof[sl[f]]];
                     latency = ex;
                     ok = 1;
+                } else if (pk[f] >= 2) {
+                    ex = pe2e[f];
+                    latency = ex;
+                    ok = 1;
+                    C[10]++;
                 } else {
+                    /* (1) smallest free slice that holds the function */
                     int best = -1;
                     for (int s = 0; s < a->n_slices; s++) {
                         if (a->sl_node[s] != v || a->sl_busy[s] || res[s] >= 0) continue;
@@ -856,10 +906,39 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
                             best = s;
                     }
                     if (best < 0) {
+                        /* (2) a pipeline over the free slices: the plan search's argmin */
+                        int any_free = 0;
+                        for (int s = 0; s < a->n_slices; s++) {
+                            occ[s] = (uint8_t)(a->sl_busy[s] || res[s] >= 0);
+                            if (a->sl_node[s] == v && !occ[s]) any_free = 1;
+                        }
+                        if (any_free) {
+                            q_func = (uint32_t)f;
+                            q_node = (uint32_t)v;
+                            q_slo = (uint32_t)(B > 0xffffffffull ? 0xffffffffull : B);
+                            plan_one_busy(&b, 0, occ);
+                            if (o_status == PLAN_OK) {
+                                pk[f] = (uint8_t)o_k;
+                                for (int i = 0; i < o_k; i++) {
+                                    psl[(size_t)f * 8 + i] = o_slice[i];
+                                    res[o_slice[i]] = f;
+                                }
+                                pe2e[f] = o_e2e;
+                                C[8]++;
+                                C[4]++;
+                                C[10]++;
+                                ex = o_e2e;
+                                latency = a->load_us[f] + ex;
+                                ok = 1;
+                            }
+                        }
+                    }
+                    if (!ok && best < 0) {
+                        /* (3) evict the LRU time-sharing instance of another function */
                         for (int s = 0; s < a->n_slices; s++) {
                             if (a->sl_node[s] != v || res[s] < 0 || res[s] == f) continue;
                             int g = res[s], p = a->sl_prof[s];
-                            if (hot[g] || last[g] >= now) continue;
+                            if (pk[g] >= 2 || hot[g] || last[g] >= now) continue;
                             if (memt[f] > a->cap_mib[p]) continue;
                             if (best < 0 || last[g] < last[res[best]]) best = s;
                         }
@@ -869,7 +948,7 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
                             C[5]++;
                         }
                     }
-                    if (best >= 0) {
+                    if (!ok && best >= 0) {
                         res[best] = f;
                         sl[f] = best;
                         C[4]++;
@@ -888,7 +967,10 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
                 }
             }
             for (int s = 0; s < a->n_slices; s++)
-                if (a->sl_node[s] == v && res[s] >= 0) C[7]++;
+                if (a->sl_node[s] == v && res[s] >= 0) {
+                    C[7]++;
+                    if (pk[res[s]] >= 2) C[11]++;
+                }
             if ((uint32_t)(t + 1) % window_ticks == 0) {
                 uint64_t window_us = (uint64_t)window_ticks * tick_us;
                 for (int f = 0; f < F; f++) {
@@ -899,6 +981,8 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
             for (int f = 0; f < F; f++) {
                 if (exists[f] && now - last[f] >= cold_after_us) {
                     if (sl[f] >= 0) res[sl[f]] = -1;
+                    for (int i = 0; i < pk[f]; i++) res[psl[(size_t)f * 8 + i]] = -1;
+                    pk[f] = 0;
                     exists[f] = 0;
                     sl[f] = -1;
                     hot[f] = 0;
@@ -906,13 +990,45 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
                     C[6]++;
                 }
             }
+            /* pipeline migration (R46) */
+            for (int f = 0; f < F; f++) {
+                if (pk[f] < 2) continue;
+                int best = -1;
+                for (int s = 0; s < a->n_slices; s++) {
+                    if (a->sl_node[s] != v || a->sl_busy[s] || res[s] >= 0) continue;
+                    int p = a->sl_prof[s];
+                    if (memt[f] > a->cap_mib[p]) continue;
+                    if (best < 0) {
+                        best = s;
+                        continue;
+                    }
+                    int q = a->sl_prof[best];
+                    if (a->cap_mib[p] < a->cap_mib[q] || (a->cap_mib[p] == a->cap_mib[q] && a->gpcs[p] < a->gpcs[q]))
+                        best = s;
+                }
+                if (best < 0) continue;
+                for (int i = 0; i < pk[f]; i++) res[psl[(size_t)f * 8 + i]] = -1;
+                pk[f] = 0;
+                res[best] = f;
+                sl[f] = best;
+                C[9]++;
+                C[4]++;
+            }
         }
-        for (int f = 0; f < F; f++)
-            st[f] = !exists[f] ? ST_COLD : (sl[f] < 0 ? ST_WARM : (hot[f] ? ST_EXCL_HOT : ST_TIME_SHARING));
+        for (int f = 0; f < F; f++) {
+            st[f] = !exists[f] ? ST_COLD
+                               : (pk[f] >= 2 ? ST_EXCL_HOT : (sl[f] < 0 ? ST_WARM : (hot[f] ? ST_EXCL_HOT : ST_TIME_SHARING)));
+            fin_k[(size_t)v * F + f] = pk[f] >= 2 ? pk[f] : (sl[f] >= 0 ? 1 : 0);
+            if (pk[f] >= 2) sl[f] = psl[(size_t)f * 8];
+        }
         free(exists);
         free(hot);
+        free(pk);
+        free(psl);
+        free(pe2e);
     }
     free(res);
+    free(occ);
     free(exec);
     free(memt);
     return 0;

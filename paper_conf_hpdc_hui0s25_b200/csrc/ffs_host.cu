@@ -73,7 +73,7 @@ struct ffs_ctx {
   // NEXT-2 routing scratch
   DevBuf r_k, r_k2, r_v, r_v2, i_k, i_k2, i_v, i_v2, i_cum, r_f, r_h, r_n, r_ts, r_hist, r_bsum;
   // NEXT-4 simulator scratch
-  DevBuf s_res, s_flags, s_busy;
+  DevBuf s_res, s_flags, s_busy, s_psl, s_pe2e, s_pk;
   // NEXT-3 frontiers
   DevBuf f_nodefv, f_fvnode, f_act, f_next, f_budget, f_greq, f_gslo, f_gkeys, f_cnt, f_key, f_e2e, f_ctr;
   bool front_built = false;
@@ -165,7 +165,7 @@ void ffs_destroy(ffs_ctx* c) {
       if (e) cudaEventDestroy(e);
     for (auto& e : c->evs)
       if (e) cudaEventDestroy(e);
-    for (DevBuf* b : {&c->s_res, &c->s_flags, &c->s_busy}) b->release();
+    for (DevBuf* b : {&c->s_res, &c->s_flags, &c->s_busy, &c->s_psl, &c->s_pe2e, &c->s_pk}) b->release();
     for (DevBuf* b : {&c->r_k, &c->r_k2, &c->r_v, &c->r_v2, &c->i_k, &c->i_k2, &c->i_v, &c->i_v2, &c->i_cum, &c->r_f,
                       &c->r_h, &c->r_n, &c->r_ts, &c->r_hist, &c->r_bsum})
       b->release();
@@ -1061,12 +1061,19 @@ ffs_status ffs_route(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_slo
 
 ffs_status ffs_simulate(ffs_ctx* c, const uint32_t* d_req_off, const uint32_t* d_req_func,
                         const uint32_t* d_req_budget, uint32_t n_ticks, uint64_t t0_us, uint32_t tick_us,
-                        uint32_t window_ticks, uint32_t thr_pct, uint64_t cold_after_us, uint64_t* d_ctr,
-                        int32_t* d_slice, uint8_t* d_state, uint64_t* d_last, uint32_t* d_busy, void* stream) {
+                        uint32_t window_ticks, uint32_t thr_pct, uint64_t cold_after_us, uint32_t k_max,
+                        uint64_t* d_ctr, int32_t* d_slice, uint8_t* d_state, uint64_t* d_last, uint32_t* d_busy,
+                        uint8_t* d_stages, void* stream) {
   if (!c) return FFS_ERR_ARG;
   if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
+  if (k_max > (uint32_t)kMaxK) return fail(c, FFS_ERR_RANGE, "k_max %u > 8", k_max);
+  if (k_max >= 2) {
+    ffs_status s = check_kmax(c, k_max);
+    if (s != FFS_OK) return s;
+  }
   if (n_ticks == 0) return FFS_OK;
-  if (!d_req_off || !d_req_func || !d_req_budget || !d_ctr || !d_slice || !d_state || !d_last || !d_busy)
+  if (!d_req_off || !d_req_func || !d_req_budget || !d_ctr || !d_slice || !d_state || !d_last || !d_busy ||
+      !d_stages)
     return fail(c, FFS_ERR_ARG, "null device pointer");
   if (window_ticks == 0 || tick_us == 0) return fail(c, FFS_ERR_ARG, "window_ticks and tick_us must be > 0");
   if (c->n_slices >= (1u << 20)) return fail(c, FFS_ERR_RANGE, "n_slices >= 2^20");
@@ -1074,6 +1081,9 @@ ffs_status ffs_simulate(ffs_ctx* c, const uint32_t* d_req_off, const uint32_t* d
   CK(c->s_res.ensure((size_t)std::max(1u, c->n_slices) * 4), "cudaMalloc");
   CK(c->s_flags.ensure((size_t)c->n_nodes * c->F), "cudaMalloc");
   CK(c->s_busy.ensure(std::max<size_t>(1, c->n_slices)), "cudaMalloc");
+  CK(c->s_psl.ensure((size_t)c->n_nodes * c->F * 8 * 4), "cudaMalloc");
+  CK(c->s_pe2e.ensure((size_t)c->n_nodes * c->F * 4), "cudaMalloc");
+  CK(c->s_pk.ensure((size_t)c->n_nodes * c->F), "cudaMalloc");
   if (c->n_slices)
     CK(cudaMemcpyAsync(c->s_busy.p, c->h_busy.data(), c->n_slices, cudaMemcpyHostToDevice, (cudaStream_t)stream),
        "H2D busy");
@@ -1100,6 +1110,11 @@ ffs_status ffs_simulate(ffs_ctx* c, const uint32_t* d_req_off, const uint32_t* d
   a.state = d_state;
   a.last = d_last;
   a.busy = d_busy;
+  a.stages = d_stages;
+  a.k_max = k_max;
+  a.psl = c->s_psl.as<int32_t>();
+  a.pe2e = c->s_pe2e.as<uint32_t>();
+  a.pk = c->s_pk.as<uint8_t>();
   CK(launch_sim(a, (cudaStream_t)stream), "simulator kernel");
   return FFS_OK;
 }

@@ -288,11 +288,16 @@ struct SimArgs {
   const uint32_t* req_budget;
   int32_t* res;                 // [n_slices] resident function or -1 (scratch)
   uint8_t* flags;               // [n_nodes][F] bit0 exists, bit1 hot (scratch)
-  uint64_t* ctr;
+  uint64_t* ctr;                // [n_nodes][12]
   int32_t* slice;
   uint8_t* state;
   uint64_t* last;
   uint32_t* busy;
+  uint8_t* stages;              // [n_nodes][F] 0 none, 1 monolithic, k pipeline
+  uint32_t k_max;               // pipeline search depth (0: monolithic instances only)
+  int32_t* psl;                 // [n_nodes][F][8] pipeline slices (scratch)
+  uint32_t* pe2e;               // [n_nodes][F] pipeline e2e (scratch)
+  uint8_t* pk;                  // [n_nodes][F] pipeline stages (scratch)
 };
 cudaError_t launch_sim(const SimArgs& a, cudaStream_t st);
 cudaError_t radix_sort_pairs(uint64_t* key, uint32_t* val, uint64_t* key2, uint32_t* val2, uint32_t n, int bits,

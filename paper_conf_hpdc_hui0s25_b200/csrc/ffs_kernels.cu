@@ -2619,6 +2619,65 @@ __device__ __forceinline__ uint64_t warp_min_u64(uint64_t x) {
   return x;
 }
 
+// Warp-wide exact argmin of function f's candidates against free counts `freeb` (8 x u8)
+// and budget B (R44: the pipeline a new instance is built as): the masks walked in colex
+// order by the whole warp, the lanes over the profile sequences; exact integer scoring as
+// exact_eval (memory, floor, free slices, SLO, cvq), packed key (R1).  Returns the key.
+__device__ int64_t warp_plan_argmin(const uint32_t* img, const ImageLayout& L, uint32_t f, uint64_t freeb,
+                                    uint32_t B, uint32_t K, uint32_t lane) {
+  const uint32_t* fd = img + L.o_fdesc + 4 * f;
+  const uint32_t row0 = fd[0], n = fd[1];
+  const uint32_t thr = img[L.o_thr + f];
+  int64_t best = (int64_t)kKeyNone;
+  const uint32_t kk = min(K, n);
+  for (uint32_t k = 1; k <= kk; ++k) {
+    uint32_t pk = 1;
+    for (uint32_t i = 0; i < k; ++i) pk *= kP;
+    const uint64_t off = img_u64(img, L.o_offk + 2 * (n * 10 + k));
+    const uint32_t nm = binom(img, L, n - 1, k - 1);
+    uint32_t mask = (1u << (k - 1)) - 1;
+    for (uint32_t rk = 0; rk < nm; ++rk, mask = (k > 1 ? gosper_next(mask) : 0u)) {
+      // stage bounds of the mask (warp-uniform)
+      uint32_t bnd[kMaxK + 1];
+      bnd[0] = 0;
+      uint32_t m = mask, X = 0;
+      for (uint32_t i = 1; i < k; ++i) {
+        const uint32_t j = __ffs(m) - 1;
+        m &= m - 1;
+        bnd[i] = j + 1;
+        X += img[L.o_xf + row0 + j];
+      }
+      bnd[k] = n;
+      if (X > B) continue;
+      for (uint32_t seq = lane; seq < pk; seq += 32) {
+        uint32_t rest = seq, used = 0, g = 0;
+        uint64_t St = 0, Sq = 0;
+        bool ok = true;
+        for (int i = (int)k - 1; i >= 0; --i) {  // digits, stage 0 most significant
+          const uint32_t pr = rest % kP;
+          rest /= kP;
+          const uint32_t t = pl_diff(img, L.o_pl + (row0 + bnd[i + 1]) * kRowW + pr, L.o_pl + (row0 + bnd[i]) * kRowW + pr);
+          ok &= img[L.o_pm + row0 + bnd[i + 1]] - img[L.o_pm + row0 + bnd[i]] <= img[L.o_cap + pr];
+          ok &= t <= thr;
+          St += t;
+          Sq += (uint64_t)t * t;
+          used += 1u << (4 * pr);
+          g += img[L.o_gpcs + pr];
+        }
+#pragma unroll
+        for (int pp = 0; pp < kP; ++pp) ok &= ((used >> (4 * pp)) & 15u) <= ((freeb >> (8 * pp)) & 255u);
+        ok &= St + X <= (uint64_t)B;
+        if (!ok) continue;
+        const uint64_t D = St * St, N = (uint64_t)k * Sq - D;
+        const uint64_t cvq = (N << 10) / D;  // floor(1024 CV^2), exact (R4)
+        const int64_t key = (int64_t)((cvq << 50) | ((uint64_t)(k - 1) << 47) | ((uint64_t)g << 41) | (off + rk * pk + seq));
+        best = key < best ? key : best;
+      }
+    }
+  }
+  return (int64_t)warp_min_u64((uint64_t)best);
+}
+
 __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArgs A) {
   const uint32_t v = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (v >= A.n_nodes) return;
@@ -2629,16 +2688,31 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
   uint64_t* last = A.last + (uint64_t)v * F;
   uint32_t* busy = A.busy + (uint64_t)v * F;
   uint8_t* fl = A.flags + (uint64_t)v * F;
+  uint8_t* pk = A.pk + (uint64_t)v * F;
+  int32_t* psl = A.psl + (uint64_t)v * F * 8;
+  uint32_t* pe2e = A.pe2e + (uint64_t)v * F;
   for (uint32_t f = lane; f < F; f += 32) {
     sl[f] = -1;
     last[f] = 0;
     busy[f] = 0;
     fl[f] = 0;
+    pk[f] = 0;
   }
   for (uint32_t s = s0 + lane; s < s1; s += 32) A.res[s] = -1;
   uint64_t c_req = 0, c_srv = 0, c_hit = 0, c_uns = 0, c_rel = 0, c_evi = 0, c_ter = 0, c_occ = 0;
+  uint64_t c_pip = 0, c_mig = 0, c_psrv = 0, c_pocc = 0;
   const uint64_t window_us = (uint64_t)A.window_ticks * A.tick_us;
   __syncwarp();
+  // smallest (capacity, gpcs, id) free slice of the node holding memt MiB, ~0 if none
+  auto free_fit = [&](uint32_t memt) {
+    uint64_t best = ~0ull;
+    for (uint32_t s = s0 + lane; s < s1; s += 32) {
+      const uint32_t p = A.slice_prof[s];
+      if (!A.slice_busy[s] && A.res[s] < 0 && memt <= img[L.o_cap + p])
+        best = min(best, ((uint64_t)img[L.o_cap + p] << 40) | ((uint64_t)img[L.o_gpcs + p] << 32) | s);
+    }
+    return warp_min_u64(best);
+  };
   for (uint32_t t = 0; t < A.n_ticks; ++t) {
     const uint64_t now = A.t0_us + (uint64_t)t * A.tick_us;
     const uint32_t j0 = A.req_off[(uint64_t)v * A.n_ticks + t], j1 = A.req_off[(uint64_t)v * A.n_ticks + t + 1];
@@ -2656,20 +2730,87 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
       }
       __syncwarp();
       int32_t at = sl[f];
-      uint64_t latency = 0;
-      if (at < 0) {
-        // free slice of smallest (capacity, gpcs, id) holding the function
-        uint64_t best = ~0ull;
-        for (uint32_t s = s0 + lane; s < s1; s += 32) {
-          const uint32_t p = A.slice_prof[s];
-          if (!A.slice_busy[s] && A.res[s] < 0 && memt <= img[L.o_cap + p])
-            best = min(best, ((uint64_t)img[L.o_cap + p] << 40) | ((uint64_t)img[L.o_gpcs + p] << 32) | s);
+      uint64_t latency = 0, ex = 0;
+      bool served = false;
+      if (at < 0 && pk[f] >= 2) {  // resident pipeline (R45)
+        ex = pe2e[f];
+        latency = ex;
+        served = true;
+        ++c_psrv;
+      } else if (at < 0) {
+        uint64_t best = free_fit(memt);
+        if (best == ~0ull && A.k_max >= 2) {
+          // a pipeline over the node's free slices: the argmin plan for this budget (R44)
+          uint32_t cnt[kP] = {0, 0, 0, 0, 0};
+          for (uint32_t s = s0; s < s1; ++s)
+            if (!A.slice_busy[s] && A.res[s] < 0) ++cnt[A.slice_prof[s]];
+          uint64_t freeb = 0;
+#pragma unroll
+          for (int p = 0; p < kP; ++p) freeb |= (uint64_t)min(cnt[p], 8u) << (8 * p);
+          if (freeb) {
+            const int64_t key = warp_plan_argmin(img, L, f, freeb, (uint32_t)min(B, (uint64_t)0xffffffffull), A.k_max, lane);
+            if ((uint64_t)key != kKeyNone) {
+              // decode (as k_decode): k, mask rank, profile digits; bind stage i to the
+              // lowest-index free slice of its profile not taken by an earlier stage (R11)
+              const uint64_t idx = (uint64_t)key & ((1ull << kIdxBits) - 1);
+              const uint32_t k = (uint32_t)(((uint64_t)key >> 47) & 7) + 1;
+              uint32_t pkk = 1;
+              for (uint32_t i = 0; i < k; ++i) pkk *= kP;
+              const uint64_t rel = idx - img_u64(img, L.o_offk + 2 * (n * 10 + k));
+              uint64_t rk = rel / pkk;
+              uint32_t seq = (uint32_t)(rel % pkk);
+              uint32_t mask = 0;
+              int cc = (int)n - 2;
+              for (int i = (int)k - 1; i >= 1; --i) {  // colex unrank
+                while (binom(img, L, cc, i) > rk) --cc;
+                mask |= 1u << cc;
+                rk -= binom(img, L, cc, i);
+                --cc;
+              }
+              uint32_t prof[kMaxK];
+              for (int i = (int)k - 1; i >= 0; --i) {
+                prof[i] = seq % kP;
+                seq /= kP;
+              }
+              uint32_t e2e = 0, a0 = 0;
+              uint32_t mm = mask;
+              for (uint32_t i = 0; i < k; ++i) {
+                uint32_t b1 = n;
+                if (i + 1 < k) {
+                  const uint32_t jj = __ffs(mm) - 1;
+                  mm &= mm - 1;
+                  b1 = jj + 1;
+                  e2e += img[L.o_xf + row0 + jj];
+                }
+                e2e += pl_diff(img, L.o_pl + (row0 + b1) * kRowW + prof[i], L.o_pl + (row0 + a0) * kRowW + prof[i]);
+                a0 = b1;
+              }
+              if (lane == 0) {
+                for (uint32_t i = 0; i < k; ++i) {
+                  for (uint32_t s = s0; s < s1; ++s) {
+                    if (A.slice_busy[s] || A.res[s] >= 0 || A.slice_prof[s] != prof[i]) continue;
+                    A.res[s] = (int32_t)f;  // taken: later stages skip it
+                    psl[f * 8 + i] = (int32_t)s;
+                    break;
+                  }
+                }
+                pk[f] = (uint8_t)k;
+                pe2e[f] = e2e;
+              }
+              __syncwarp();
+              ++c_pip;
+              ++c_rel;
+              ++c_psrv;
+              ex = e2e;
+              latency = (uint64_t)load + e2e;
+              served = true;
+            }
+          }
         }
-        best = warp_min_u64(best);
-        if (best == ~0ull) {  // LRU time-sharing victim not used in this tick
+        if (!served && best == ~0ull) {  // LRU time-sharing victim not used in this tick
           for (uint32_t s = s0 + lane; s < s1; s += 32) {
             const int32_t g = A.res[s];
-            if (g < 0 || (uint32_t)g == f || (fl[g] & 2u) || last[g] >= now) continue;
+            if (g < 0 || (uint32_t)g == f || pk[g] >= 2 || (fl[g] & 2u) || last[g] >= now) continue;
             if (memt > img[L.o_cap + A.slice_prof[s]]) continue;
             best = min(best, (last[g] << 20) | (s - s0));
           }
@@ -2683,10 +2824,10 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
             ++c_evi;
             best = s;
           }
-        } else {
+        } else if (!served) {
           best &= 0xFFFFFFFFull;
         }
-        if (best != ~0ull) {
+        if (!served && best != ~0ull) {
           at = (int32_t)best;
           if (lane == 0) {
             A.res[at] = (int32_t)f;
@@ -2696,14 +2837,17 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
           latency = load;
         }
       }
-      if (at >= 0) {
+      if (!served && at >= 0) {
         const uint32_t p = A.slice_prof[at];
-        const uint32_t ex = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
+        ex = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
         latency += ex;
+        served = true;
+      }
+      if (served) {
         ++c_srv;
         c_hit += latency <= B;
         if (lane == 0) {
-          busy[f] += ex;
+          busy[f] += (uint32_t)ex;
           last[f] = now;
         }
       } else {
@@ -2711,9 +2855,13 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
       }
       __syncwarp();
     }
-    // end of tick: occupied slices, utilisation windows, cold terminations
-    uint32_t occ = 0;
-    for (uint32_t s = s0 + lane; s < s1; s += 32) occ += A.res[s] >= 0;
+    // end of tick: occupied slices, utilisation windows, cold terminations, migrations
+    uint32_t occ = 0, pocc = 0;
+    for (uint32_t s = s0 + lane; s < s1; s += 32) {
+      const int32_t g = A.res[s];
+      occ += g >= 0;
+      pocc += g >= 0 && pk[g] >= 2;
+    }
     uint32_t ter = 0;
     const bool roll = (t + 1) % A.window_ticks == 0;
     for (uint32_t f = lane; f < F; f += 32) {
@@ -2724,6 +2872,8 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
       }
       if ((x & 1u) && now - last[f] >= A.cold_after_us) {
         if (sl[f] >= 0) A.res[sl[f]] = -1;
+        for (uint32_t i = 0; i < pk[f]; ++i) A.res[psl[f * 8 + i]] = -1;
+        pk[f] = 0;
         sl[f] = -1;
         busy[f] = 0;
         x = 0;
@@ -2734,21 +2884,47 @@ __global__ void __launch_bounds__(128) k_simulate(const __grid_constant__ SimArg
 #pragma unroll
     for (int o = 16; o; o >>= 1) {
       occ += __shfl_xor_sync(0xffffffffu, occ, o);
+      pocc += __shfl_xor_sync(0xffffffffu, pocc, o);
       ter += __shfl_xor_sync(0xffffffffu, ter, o);
     }
     c_occ += occ;
+    c_pocc += pocc;
     c_ter += ter;
     __syncwarp();
+    // pipeline migration (R46), function order
+    for (uint32_t f0 = 0; f0 < F; f0 += 32) {
+      uint32_t has = __ballot_sync(0xffffffffu, f0 + lane < F && pk[f0 + lane] >= 2);
+      while (has) {
+        const uint32_t f = f0 + __ffs(has) - 1;
+        has &= has - 1;
+        const uint64_t best = free_fit(img[L.o_fdesc + 4 * f + 3]);
+        if (best == ~0ull) continue;
+        if (lane == 0) {
+          for (uint32_t i = 0; i < pk[f]; ++i) A.res[psl[f * 8 + i]] = -1;
+          pk[f] = 0;
+          A.res[(uint32_t)best] = (int32_t)f;
+          sl[f] = (int32_t)(uint32_t)best;
+        }
+        __syncwarp();
+        ++c_mig;
+        ++c_rel;
+      }
+    }
   }
   for (uint32_t f = lane; f < F; f += 32) {
     const uint8_t x = fl[f];
+    const bool pipe = pk[f] >= 2;
     A.state[(uint64_t)v * F + f] = !(x & 1u) ? FFS_ST_COLD
+                                   : pipe ? FFS_ST_EXCL_HOT
                                    : (sl[f] < 0 ? FFS_ST_WARM : ((x & 2u) ? FFS_ST_EXCL_HOT : FFS_ST_TIME_SHARING));
+    A.stages[(uint64_t)v * F + f] = pipe ? pk[f] : (sl[f] >= 0 ? 1 : 0);
+    if (pipe) sl[f] = psl[f * 8];
   }
   if (lane == 0) {
-    uint64_t* C = A.ctr + (uint64_t)v * 8;
+    uint64_t* C = A.ctr + (uint64_t)v * 12;
     C[0] = c_req; C[1] = c_srv; C[2] = c_hit; C[3] = c_uns;
     C[4] = c_rel; C[5] = c_evi; C[6] = c_ter; C[7] = c_occ;
+    C[8] = c_pip; C[9] = c_mig; C[10] = c_psrv; C[11] = c_pocc;
   }
 }
 

@@ -74,7 +74,8 @@ _sig = {
     "ffs_evict_step": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp, _vp, _vp, _u32, _vp, _vp],
                        _i32),
     "ffs_plan_joint": ([_vp, _vp, _vp, _u32, _u32, _vp, C.POINTER(C.c_uint32), _vp], _i32),
-    "ffs_simulate": ([_vp, _vp, _vp, _vp, _u32, _u64, _u32, _u32, _u32, _u64, _vp, _vp, _vp, _vp, _vp, _vp], _i32),
+    "ffs_simulate": ([_vp, _vp, _vp, _vp, _u32, _u64, _u32, _u32, _u32, _u64, _u32, _vp, _vp, _vp, _vp, _vp, _vp, _vp],
+                     _i32),
     "ffs_route": ([_vp, _vp, _vp, _u32, _vp, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
     "ffs_frontier_build": ([_vp, _u32, C.POINTER(C.c_uint32), C.POINTER(C.c_uint32), _vp], _i32),
     "ffs_plan_frontier": ([_vp, _vp, _vp, _u32, _vp, _vp], _i32),
@@ -286,24 +287,29 @@ class Planner:
         return out, int(rounds.value)
 
     # ---- NEXT-4: time-sharing simulator ------------------------------------------
-    def simulate(self, trace, thr_pct: int = 30, cold_after_us: int = 600_000_000, stream=None):
-        """Run the simulator on a workload.SimTrace whose problem is staged.  Returns device
-        tensors (ctr[N, 8], slice[N, F], state[N, F], last_used[N, F], busy[N, F])."""
+    def simulate(self, trace, thr_pct: int = 30, cold_after_us: int = 600_000_000, k_max: int | None = None,
+                 stream=None):
+        """Run the simulator on a workload.SimTrace whose problem is staged; k_max = pipeline
+        search depth (default the problem's; 0 = monolithic instances only).  Returns device
+        tensors (ctr[N, 12], slice[N, F], state[N, F], last_used[N, F], busy[N, F], stages[N, F])."""
         import torch
         prob = trace.problem
         N, F = int(prob.n_nodes), int(prob.comp_off.shape[0] - 1)
+        K = int(prob.k_max if k_max is None else k_max)
         dev = torch.device("cuda", self.device)
         t = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).to(dev)
         off, fu, bu = t(trace.req_off), t(trace.req_func), t(trace.req_budget)
-        ctr = torch.zeros((N, 8), dtype=torch.int64, device=dev)
+        ctr = torch.zeros((N, 12), dtype=torch.int64, device=dev)
         sl = torch.empty((N, F), dtype=torch.int32, device=dev)
         st = torch.empty((N, F), dtype=torch.uint8, device=dev)
         last = torch.empty((N, F), dtype=torch.int64, device=dev)
         busy = torch.empty((N, F), dtype=torch.int32, device=dev)
+        stages = torch.empty((N, F), dtype=torch.uint8, device=dev)
         self._check(_lib.ffs_simulate(self._h, _ptr(off), _ptr(fu), _ptr(bu), int(trace.T), int(trace.t0_us),
                                       int(trace.tick_us), int(trace.window_ticks), int(thr_pct), int(cold_after_us),
-                                      _ptr(ctr), _ptr(sl), _ptr(st), _ptr(last), _ptr(busy), _stream(stream)))
-        return ctr, sl, st, last, busy
+                                      K, _ptr(ctr), _ptr(sl), _ptr(st), _ptr(last), _ptr(busy), _ptr(stages),
+                                      _stream(stream)))
+        return ctr, sl, st, last, busy, stages
 
     # ---- NEXT-2: routing (P:374) ------------------------------------------------------------
     def route(self, req, slo, inst, state, lat_us, capacity, route=None, stream=None):

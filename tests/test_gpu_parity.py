@@ -664,15 +664,43 @@ def test_simulator_matches_oracle(F, planner, case):
         tr = W.sim_trace(T=2048)
         cold = 60_000_000
     planner.stage(tr.problem)
-    ctr, sl, st, last, busy = planner.simulate(tr, cold_after_us=cold)
-    torch.cuda.synchronize()
-    o = oracle.sim(tr, cold_after_us=cold)
+    for K in (tr.problem.k_max, 0):  # with pipeline instances (R44-R46), and monolithic only
+        out = planner.simulate(tr, cold_after_us=cold, k_max=K)
+        torch.cuda.synchronize()
+        o = oracle.sim(tr, cold_after_us=cold, k_max=K)
+        _assert_sim_equal(out, o)
+        assert o[0][:, 5].sum() > 0 and o[0][:, 6].sum() > 0
+        assert (o[0][:, 8].sum() > 0) == (K > 0)  # pipelines are placed exactly when enabled
+
+
+def _assert_sim_equal(out, o):
+    ctr, sl, st, last, busy, stages = out
     np.testing.assert_array_equal(ctr.cpu().numpy().view(np.uint64), o[0])
     np.testing.assert_array_equal(sl.cpu().numpy(), o[1])
     np.testing.assert_array_equal(st.cpu().numpy(), o[2])
     np.testing.assert_array_equal(last.cpu().numpy().view(np.uint64), o[3])
     np.testing.assert_array_equal(busy.cpu().numpy().view(np.uint32), o[4])
-    assert o[0][:, 5].sum() > 0 and o[0][:, 6].sum() > 0
+    np.testing.assert_array_equal(stages.cpu().numpy(), o[5])
+
+
+@pytest.mark.parametrize("case", ["fragmented", "never_evicted", "migration"])
+def test_simulator_pipeline_hand_cases(F, planner, case):
+    """The oracle's hand-worked pipeline scenarios (tests/test_oracle_sim.py) on the GPU."""
+    from test_oracle_sim import pipe_funcs, make_trace, G1, G2
+    if case == "fragmented":
+        prob = pipe_funcs([[[G1, G1, (G2, 1)]]])
+        tr, cold = make_trace(prob, 3, [(0, 0, 0, 300), (1, 0, 0, 106), (2, 0, 0, 107)], window_ticks=100), 600_000_000
+    elif case == "never_evicted":
+        prob = pipe_funcs([[[G1, G1]]], mem_h=5 * 1024)
+        tr, cold = make_trace(prob, 2, [(0, 0, 0, 10**6), (1, 0, 1, 10**6)], window_ticks=100), 600_000_000
+    else:
+        prob = pipe_funcs([[[G2, G1, G1]]])
+        ev = [(0, 0, 1, 10**6), (1, 0, 0, 10**6), (2, 0, 0, 10**6), (3, 0, 0, 10**6), (4, 0, 0, 75)]
+        tr, cold = make_trace(prob, 5, ev, window_ticks=100), 300
+    planner.stage(prob)
+    o = oracle.sim(tr, cold_after_us=cold)
+    _assert_sim_equal(planner.simulate(tr, cold_after_us=cold), o)
+    assert o[0][0, 8] == 1
 
 
 def test_large_table_image_reads_tables_from_global(F, planner):
