@@ -12,7 +12,8 @@ candidate of every request scored, device counters prove the count); the product
 (bounded) mode -- same keys -- is reported as plans/s under "production".  Inputs are
 resident in HBM when the timed region starts; L2 is flushed (256 MiB write) between timed
 steps, outside the events.  Each step is timed with CUDA events on the launching stream;
-ranks report the max.  Roofline peaks are measured by microbenchmarks in the same run.
+ranks report the max.  The roofline peak is the issue-limited packed rate (unit counts x the SM
+clock measured during the timed region); microbenchmarks measured in the same run are reported.
 `--impl reference` times the CPU oracle (oracle/, the plain brute force) on a bounded
 sample of the same workload on this box's host cores (rank 0 only).
 """
@@ -159,7 +160,8 @@ def run_c4(pl, steps: int, warmup: int, flush, peaks):
     """C4: hotness-aware eviction over T = 4096 tick snapshots of a 32-node
     (256-GPU) cluster, 200 warm functions -- one step = ffs_evict_step: every instance of
     every tick scored (A7) and the victim of every load (A8), fused (one pass over the
-    instances builds each tick's (node, profile) minima; the picks read <= 5 cells).
+    instances builds each tick's (node, profile) minima in shared memory and picks the
+    victims of the tick's loads from them: one launch).
     Reported against the HBM roofline: 33 algorithmic bytes per score (24 B record in, 8 B
     score + 1 B state out), for the scoring kernel and for the whole step."""
     import torch
@@ -171,7 +173,9 @@ def run_c4(pl, steps: int, warmup: int, flush, peaks):
     now = torch.from_numpy(wl.now_us.view(np.int64)).cuda()
     req = torch.from_numpy(np.ascontiguousarray(prob.req).view(np.uint8).reshape(-1, 8)).cuda()
     slo = torch.from_numpy(prob.slo_us.view(np.int32)).cuda()
-    rt = torch.from_numpy(wl.req_tick.view(np.int32)).cuda()
+    # the C4 loads arrive tick by tick: grouped (CSR offsets per tick), so the victims are
+    # picked inside each tick's CTA
+    load_off = torch.from_numpy(np.searchsorted(wl.req_tick, np.arange(len(wl.now_us) + 1)).astype(np.int32)).cuda()
     n = int(wl.inst.shape[0])
     score = torch.empty(n, dtype=torch.int64, device="cuda")
     state = torch.empty(n, dtype=torch.uint8, device="cuda")
@@ -179,7 +183,8 @@ def run_c4(pl, steps: int, warmup: int, flush, peaks):
     stream = torch.cuda.current_stream()
 
     def step():
-        pl.evict_step(inst, toff, now, req, slo, rt, score=score, state=state, victim=vic, window_us=wl.window_us)
+        pl.evict_step(inst, toff, now, req, slo, load_off=load_off, score=score, state=state, victim=vic,
+                      window_us=wl.window_us)
 
     for _ in range(warmup):
         step()

@@ -276,14 +276,20 @@ ffs_status ffs_evict_victims(ffs_ctx *ctx, const ffs_request *d_req, const uint3
 
 /* A7 + A8 fused over ticks: the scores and states of ffs_evict_scores_ticks and the victims
  * of ffs_evict_victims for the n_req loads, in one pass over the instances: each tick's
- * CTA folds its scored instances into per-(node, slice profile) minima in shared memory,
- * so the victim pass reads at most 5 cells per load.  Same outputs, same rules and errors
- * as the two calls (which it falls back to when the table would exceed 256 MiB or a tick's
- * minima 160 KiB of shared memory).  n_req may be 0 (scores only).  Async. */
+ * CTA folds its scored instances into per-(node, slice profile) minima in shared memory.
+ * Loads given per tick (d_req_tick[r], any order): the minima go to a table in device
+ * memory and a second kernel picks (<= 5 cells per load).  Loads grouped by tick
+ * (d_load_off non-null: uint32[n_ticks + 1], the loads of tick t are rows d_load_off[t] ..
+ * d_load_off[t+1]-1 of d_req/d_slo_us/d_victim; d_req_tick may then be null): the tick's
+ * CTA picks its loads' victims from shared memory -- one launch, no table.  Same outputs,
+ * same rules and errors as the two calls (which it falls back to when a tick's minima
+ * exceed 160 KiB of shared memory, or the table 256 MiB with per-load ticks).  n_req may
+ * be 0 (scores only).  Async. */
 ffs_status ffs_evict_step(ffs_ctx *ctx, const ffs_instance *d_inst, const uint32_t *d_tick_off,
                           const uint64_t *d_now_us, uint32_t n_ticks, const ffs_evict_params *params,
                           int64_t *d_score, uint8_t *d_state, const ffs_request *d_req, const uint32_t *d_slo_us,
-                          const uint32_t *d_req_tick, uint32_t n_req, int32_t *d_victim, void *stream);
+                          const uint32_t *d_req_tick, const uint32_t *d_load_off, uint32_t n_req, int32_t *d_victim,
+                          void *stream);
 
 /* ---- NEXT-1: the paper's literal ranked first-fit ---------------------------
  * "After calculating and sorting the CVs for all possible pipeline configurations, which

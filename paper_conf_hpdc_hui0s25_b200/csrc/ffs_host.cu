@@ -654,30 +654,33 @@ ffs_status ffs_evict_scores_ticks(ffs_ctx* c, const ffs_instance* d_inst, const 
 
 ffs_status ffs_evict_step(ffs_ctx* c, const ffs_instance* d_inst, const uint32_t* d_tick_off, const uint64_t* d_now_us,
                           uint32_t n_ticks, const ffs_evict_params* prm, int64_t* d_score, uint8_t* d_state,
-                          const ffs_request* d_req, const uint32_t* d_slo, const uint32_t* d_req_tick, uint32_t n_req,
-                          int32_t* d_victim, void* stream) {
+                          const ffs_request* d_req, const uint32_t* d_slo, const uint32_t* d_req_tick,
+                          const uint32_t* d_load_off, uint32_t n_req, int32_t* d_victim, void* stream) {
   if (!c) return FFS_ERR_ARG;
   if (!c->staged) return fail(c, FFS_ERR_STATE, "tables not staged");
   if (!prm) return fail(c, FFS_ERR_ARG, "null params");
   if (prm->cold_after_us >= (1ull << 43)) return fail(c, FFS_ERR_RANGE, "cold_after_us >= 2^43");
   if (n_ticks == 0 && n_req == 0) return FFS_OK;
   if (!d_inst || !d_tick_off || !d_now_us || !d_score || !d_state) return fail(c, FFS_ERR_ARG, "null device pointer");
-  if (n_req && (!d_req || !d_slo || !d_req_tick || !d_victim)) return fail(c, FFS_ERR_ARG, "null device pointer");
+  if (n_req && (!d_req || !d_slo || (!d_req_tick && !d_load_off) || !d_victim))
+    return fail(c, FFS_ERR_ARG, "null device pointer");
   const uint64_t tab_bytes = (uint64_t)n_ticks * c->n_nodes * c->P * 8;
   // the fused pass needs the tick's (node, profile) minima in shared memory and the whole
   // table in device memory; otherwise: the two calls it fuses
-  if (c->n_nodes * c->P * 8 > 160 * 1024 || tab_bytes > (256ull << 20)) {
+  const bool grouped = d_load_off != nullptr && n_req > 0;
+  if (c->n_nodes * c->P * 8 > 160 * 1024 || (!grouped && tab_bytes > (256ull << 20))) {
+    if (!d_req_tick && n_req) return fail(c, FFS_ERR_ARG, "d_req_tick needed for this cluster size");
     ffs_status s = ffs_evict_scores_ticks(c, d_inst, d_tick_off, d_now_us, n_ticks, prm, d_score, d_state, stream);
     if (s != FFS_OK || n_req == 0) return s;
     return ffs_evict_victims(c, d_req, d_slo, d_req_tick, n_req, d_inst, d_tick_off, d_score, n_ticks, d_victim,
                              stream);
   }
   DeviceGuard g(c->device);
-  CK(c->v_tab.ensure(std::max<uint64_t>(tab_bytes, 8)), "cudaMalloc(victim table)");
+  if (!grouped) CK(c->v_tab.ensure(std::max<uint64_t>(tab_bytes, 8)), "cudaMalloc(victim table)");
   CK(launch_evict_step(c->image.as<uint32_t>(), c->lay, d_inst, d_tick_off, d_now_us, n_ticks, *prm, d_score, d_state,
                        c->slice_node.as<uint16_t>(), c->slice_prof.as<uint8_t>(), c->n_slices, c->n_nodes,
-                       c->v_tab.as<unsigned long long>(), d_req, d_slo, d_req_tick, n_req, d_victim,
-                       (cudaStream_t)stream),
+                       c->v_tab.as<unsigned long long>(), d_req, d_slo, d_req_tick, grouped ? d_load_off : nullptr,
+                       n_req, d_victim, (cudaStream_t)stream),
      "evict step kernels");
   return FFS_OK;
 }

@@ -158,8 +158,8 @@ cudaError_t launch_evict_step(const uint32_t* image, const ImageLayout& lay, con
                               const uint32_t* tick_off, const uint64_t* now_us, uint32_t n_ticks, ffs_evict_params prm,
                               int64_t* score, uint8_t* state, const uint16_t* slice_node, const uint8_t* slice_prof,
                               uint32_t n_slices, uint32_t n_nodes, unsigned long long* tab, const ffs_request* req,
-                              const uint32_t* slo, const uint32_t* req_tick, uint32_t n_req, int32_t* victim,
-                              cudaStream_t st);
+                              const uint32_t* slo, const uint32_t* req_tick, const uint32_t* load_off, uint32_t n_req,
+                              int32_t* victim, cudaStream_t st);
 cudaError_t run_int_peak(int sms, double* ops, double* seconds);
 cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double* seconds);
 cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, const uint32_t* gofs, uint32_t* grp,

@@ -1922,14 +1922,29 @@ constexpr int kEvT = FFS_EVT, kEvU = FFS_EVU;
 // (node, slice profile) minima in shared memory (64-bit atomicMin) and writes that row of
 // the victim table once -- the victim pass then reads <= 5 cells per load instead of
 // re-reading the tick's scores and records.  ~0 marks an empty cell.
-template <bool TAB>
+// (defined with the victim kernels below)
+__device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const ImageLayout& L, uint32_t f, uint32_t B);
+
+// PICK (loads grouped by tick, d_load_off): the tick's loads take their victims from the
+// shared-memory minima right away -- no table in device memory, one launch for the step.
+struct EvictPick {
+  const uint32_t* image;
+  ImageLayout lay;
+  const ffs_request* req;
+  const uint32_t* slo;
+  const uint32_t* load_off;  // [n_ticks + 1] loads of tick t: [load_off[t], load_off[t+1])
+  int32_t* victim;
+};
+
+template <bool TAB, bool PICK = false>
 __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __restrict__ inst,
                                                        const uint32_t* __restrict__ tick_off,
                                                        const uint64_t* __restrict__ now_us, ffs_evict_params prm,
                                                        int64_t* __restrict__ score, uint8_t* __restrict__ state,
                                                        const uint16_t* __restrict__ slice_node,
                                                        const uint8_t* __restrict__ slice_prof, uint32_t n_slices,
-                                                       uint32_t n_nodes, unsigned long long* __restrict__ tab) {
+                                                       uint32_t n_nodes, unsigned long long* __restrict__ tab,
+                                                       EvictPick pk = EvictPick{}) {
   extern __shared__ unsigned long long cell[];
   const uint32_t t = blockIdx.x;
   const uint32_t b = tick_off[t], e = tick_off[t + 1];
@@ -1957,10 +1972,25 @@ __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __rest
       }
     }
   }
-  if constexpr (TAB) {
+  if constexpr (TAB && !PICK) {
     __syncthreads();
     unsigned long long* row = tab + (uint64_t)t * ncell;
     for (uint32_t i = threadIdx.x; i < ncell; i += kEvT) row[i] = cell[i];
+  }
+  if constexpr (TAB && PICK) {  // this tick's loads: the minimum over their monolithic profiles' cells
+    __syncthreads();
+    const uint32_t lb = pk.load_off[t], le = pk.load_off[t + 1];
+    for (uint32_t r = lb + threadIdx.x; r < le; r += kEvT) {
+      const ffs_request q = pk.req[r];
+      unsigned long long bs = ~0ull;
+      if (q.func < pk.lay.F && q.node < n_nodes) {
+        const uint32_t okp = victim_profiles(pk.image, pk.lay, q.func, pk.slo[r]);
+#pragma unroll
+        for (int p = 0; p < kP; ++p)
+          if ((okp >> p) & 1u) bs = min(bs, cell[q.node * kP + p]);
+      }
+      pk.victim[r] = bs == ~0ull ? -1 : (int32_t)(bs & 0xFFFFFull);
+    }
   }
 }
 
@@ -1993,7 +2023,7 @@ cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32
 // Profiles whose slice can host request (f, B) monolithically: the whole function fits
 // the slice memory and latency alone + reload <= B (R19).
 __device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const ImageLayout& L, uint32_t f,
-                                                    uint32_t B) {
+                                                    uint32_t B) {  // (declared above k_evict_ticks)
   const uint32_t* fd = img + L.o_fdesc + 4 * f;
   const uint32_t row0 = fd[0], n = fd[1];
   uint32_t ok = 0;
@@ -2091,10 +2121,21 @@ cudaError_t launch_evict_step(const uint32_t* image, const ImageLayout& lay, con
                               const uint32_t* tick_off, const uint64_t* now_us, uint32_t n_ticks, ffs_evict_params prm,
                               int64_t* score, uint8_t* state, const uint16_t* slice_node, const uint8_t* slice_prof,
                               uint32_t n_slices, uint32_t n_nodes, unsigned long long* tab, const ffs_request* req,
-                              const uint32_t* slo, const uint32_t* req_tick, uint32_t n_req, int32_t* victim,
-                              cudaStream_t st) {
+                              const uint32_t* slo, const uint32_t* req_tick, const uint32_t* load_off, uint32_t n_req,
+                              int32_t* victim, cudaStream_t st) {
+  const size_t sm = (size_t)n_nodes * kP * 8;
+  if (load_off && n_ticks) {  // loads grouped by tick: picks inside the tick's CTA, one launch
+    if (sm > 48 * 1024) {
+      cudaError_t e = cudaFuncSetAttribute(k_evict_ticks<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           (int)sm);
+      if (e != cudaSuccess) return e;
+    }
+    EvictPick pk{image, lay, req, slo, load_off, victim};
+    k_evict_ticks<true, true><<<n_ticks, kEvT, sm, st>>>(inst, tick_off, now_us, prm, score, state, slice_node,
+                                                         slice_prof, n_slices, n_nodes, nullptr, pk);
+    return cudaGetLastError();
+  }
   if (n_ticks) {
-    const size_t sm = (size_t)n_nodes * kP * 8;
     if (sm > 48 * 1024) {
       cudaError_t e = cudaFuncSetAttribute(k_evict_ticks<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
       if (e != cudaSuccess) return e;

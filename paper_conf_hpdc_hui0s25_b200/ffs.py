@@ -71,8 +71,8 @@ _sig = {
     "ffs_evict_scores": ([_vp, _vp, _u32, _u64, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_scores_ticks": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp], _i32),
     "ffs_evict_victims": ([_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp, _u32, _vp, _vp], _i32),
-    "ffs_evict_step": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp, _vp, _vp, _u32, _vp, _vp],
-                       _i32),
+    "ffs_evict_step": ([_vp, _vp, _vp, _vp, _u32, C.POINTER(_EvictParams), _vp, _vp, _vp, _vp, _vp, _vp, _u32, _vp,
+                        _vp], _i32),
     "ffs_plan_joint": ([_vp, _vp, _vp, _u32, _u32, _vp, C.POINTER(C.c_uint32), _vp], _i32),
     "ffs_simulate": ([_vp, _vp, _vp, _vp, _u32, _u64, _u32, _u32, _u32, _u64, _u32, _vp, _vp, _vp, _vp, _vp, _vp, _vp],
                      _i32),
@@ -259,9 +259,10 @@ class Planner:
                                            _stream(stream)))
         return victim
 
-    def evict_step(self, inst, tick_off, now_us, req, slo, req_tick, score=None, state=None, victim=None, stream=None,
-                   **params):
-        """Scores + states of every tick's instances and the victims of the loads, fused."""
+    def evict_step(self, inst, tick_off, now_us, req, slo, req_tick=None, load_off=None, score=None, state=None,
+                   victim=None, stream=None, **params):
+        """Scores + states of every tick's instances and the victims of the loads, fused
+        (load_off: loads grouped by tick, the victims picked inside the tick's CTA)."""
         import torch
         n = int(inst.numel() // W.INST_DTYPE.itemsize)
         nr = int(slo.numel())
@@ -271,7 +272,7 @@ class Planner:
         prm = self._params(**params)
         self._check(_lib.ffs_evict_step(self._h, _ptr(inst), _ptr(tick_off), _ptr(now_us), int(now_us.numel()),
                                         C.byref(prm), _ptr(score), _ptr(state), _ptr(req), _ptr(slo), _ptr(req_tick),
-                                        nr, _ptr(victim), _stream(stream)))
+                                        _ptr(load_off), nr, _ptr(victim), _stream(stream)))
         return score, state, victim
 
     # ---- NEXT-2: joint commit -------------------------------------------------

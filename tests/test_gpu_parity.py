@@ -379,6 +379,13 @@ def test_evict_step_fused_matches_separate_calls(F, planner):
     s2, st2, v2 = planner.evict_step(inst, toff, now, req, slo, rt, window_us=wl.window_us)
     assert torch.equal(s1, s2) and torch.equal(st1, st2) and torch.equal(v1, v2)
     assert int((v2 >= 0).sum()) > 0 and bool((v2[::13] == -1).all())
+    # loads grouped by tick (the C4 batch is tick-sorted): picks inside the tick's CTA
+    T = len(wl.now_us)
+    lo = torch.from_numpy(np.searchsorted(wl.req_tick, np.arange(T + 1)).astype(np.int32)).cuda()
+    rt_all = torch.from_numpy(wl.req_tick.view(np.int32)).cuda()
+    v_ref = planner.evict_victims(req, slo, rt_all, inst, toff, s1)
+    s4, st4, v4 = planner.evict_step(inst, toff, now, req, slo, load_off=lo, window_us=wl.window_us)
+    assert torch.equal(s1, s4) and torch.equal(st1, st4) and torch.equal(v_ref, v4)
     s3, st3, _ = planner.evict_step(inst, toff, now, req[:0], slo[:0], rt[:0], window_us=wl.window_us)
     assert torch.equal(s1, s3) and torch.equal(st1, st3)
 
