@@ -136,6 +136,10 @@ struct DecodeArgs {
 // the KS = 1 / 2 / 3 / 4 segments): 1: 0.04 / 1.01 / - / -, 8: 0.06 / 0.92 / 3.14 / 41.8,
 // 16: - / - / 3.04 / -, 32: 0.18 / 0.88 / 3.14 / 40.6, 64: - / - / - / 40.45.
 __host__ __device__ constexpr int kdyn(int ks) { return ks == 1 ? 1 : ks == 2 ? 32 : ks == 3 ? 16 : ks == 4 ? 64 : 32; }
+// minimum tasks per lane piece of the search's task ranges (a piece costs a request
+// lookup; a KS = 1/2 task is ~5 / ~100 instructions, a KS = 4 mask pair ~3000) and of k_live
+__host__ __device__ constexpr int kMinPiece(int ks) { return ks == 1 ? 64 : ks == 2 ? 16 : ks == 3 ? 2 : 1; }
+constexpr int kLiveMinPiece = 64;
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,

@@ -1235,7 +1235,12 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     // (contiguous 1/world ranges measured up to 1.2x apart on C5).  Exact cover needs the
     // same nthr on every rank (same kernel and device type).  DESIGN.md §4.3, §7.
     const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
-    const uint64_t NC = (nthr >> 5) * kdyn(KS) * A.world, NT = NC * 32;
+    // at most warps x kdyn chunks per rank, pieces of at least kMinPiece(KS) tasks (short
+    // segments -- a request shard's -- would otherwise pay a request lookup per task)
+    uint64_t NC = (nthr >> 5) * kdyn(KS) * A.world;
+    const uint64_t want = T / (32ull * kMinPiece(KS));
+    if (want < NC) NC = max((uint64_t)A.world, (want + A.world - 1) / A.world * A.world);
+    const uint64_t NT = NC * 32;
     const uint64_t Tq = T / NT, Tr = T % NT;  // piece u = [Tq u + Tr u / NT, ...): no overflow
     auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
     unsigned long long* ctr = A.work_ctr + KS;
@@ -1468,7 +1473,14 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint64_t T = pre[A.n_req];
-  const uint64_t NC = (uint64_t)A.warps_total * kdyn(KS) * A.world, NT = NC * 32;
+  // chunks of 32 pieces, at most warps x kdyn per rank and no smaller than kLiveMinPiece
+  // tasks per piece: a piece costs a request lookup and an unrank, a task ~20
+  // instructions, so small segments (a request shard's) use fewer, longer pieces.  The
+  // count depends only on T, so every rank of a candidate-shard split agrees on it.
+  uint64_t NC = (uint64_t)A.warps_total * kdyn(KS) * A.world;
+  const uint64_t want = T / (32ull * kLiveMinPiece);
+  if (want < NC) NC = max((uint64_t)A.world, (want + A.world - 1) / A.world * A.world);
+  const uint64_t NT = NC * 32;
   const uint64_t Tq = T / NT, Tr = T % NT;
   auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
   unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;

@@ -30,8 +30,9 @@ def task_shard(T: int, rank: int, world: int, chunks_per_rank: int, grain: int =
     """[lo, hi) pieces of a segment of T tasks owned by `rank`: the list is cut into
     NC = world * chunks_per_rank chunks of `grain` (the warp) equal contiguous pieces
     (floor(T*u/(NC*grain)) boundaries) and rank g owns chunks j*world + g (the rule of
-    k_plan_search, where chunks_per_rank = warps per launch x kDyn and the rank's warps
-    grab its chunks dynamically)."""
+    k_plan_search, where chunks_per_rank = warps per launch x kDyn -- fewer for short
+    segments, whose pieces are clamped to a minimum length -- and the rank's warps grab its
+    chunks dynamically)."""
     NT = world * chunks_per_rank * grain
     us = [(j * world + rank) * grain + i for j in range(chunks_per_rank) for i in range(grain)]
     return [(T * u // NT, T * (u + 1) // NT) for u in us]
