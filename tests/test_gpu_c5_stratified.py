@@ -25,7 +25,7 @@ def F():
 
 def chunk_straddlers(prob, sms, world, ks=4, kdyn=64, limit=1000):
     """Requests whose KS-segment task range contains a chunk boundary of the k_live split
-    (NC = sms*64 warps x kdyn x world chunks of 32 pieces, clamped to >= 64 tasks per piece;
+    (NC = sms*64 warps x kdyn x world chunks of 32 pieces, clamped to >= 8 tasks per piece;
     bounded mode:
     requests on a node without a free slice have no tasks).  Evenly spaced subset."""
     n = prob.chain_len()[prob.req["func"]].astype(np.int64)
@@ -36,7 +36,7 @@ def chunk_straddlers(prob, sms, world, ks=4, kdyn=64, limit=1000):
     pre = np.concatenate([[0], np.cumsum(t)])
     T = int(pre[-1])
     NC = sms * 64 * kdyn * world
-    want = T // (32 * 64)  # k_live's minimum piece (kLiveMinPiece = 64 tasks)
+    want = T // (32 * 8)  # k_live's minimum piece (kLiveMinPiece = 8 tasks)
     if want < NC:
         NC = max(world, -(-want // world) * world)
     NT = NC * 32
