@@ -33,8 +33,8 @@ __host__ __device__ constexpr int search_block(int ks) {
 }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
 // bytes of per-thread shared memory of the KS = 4 kernel: 5 profiles x 11 packed f16x2
-// windows + the 21-word row cache (ks4_pair_h)
-constexpr size_t kWin4 = 76 * 4;
+// windows (ks4_pair_h)
+constexpr size_t kWin4 = 55 * 4;
 
 // Layout of the staged "table image" (32-bit words).  The search kernel copies the whole
 // image into shared memory once per CTA (A0 of DESIGN.md §4); every other kernel reads

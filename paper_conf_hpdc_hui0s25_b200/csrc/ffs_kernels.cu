@@ -714,22 +714,13 @@ struct WinH {
   h2 s1, s2[2], c3[3];
 };
 
-// Per-thread shared-memory slots of the KS = 4 kernel, [slot][thread] (4-byte,
-// conflict-free, immediate offsets: the stride is the compile-time CTA size):
-//   x * 11 + k  windows of profile x: k = 0-1 s1 (stage 1 gated by > 0 / > 1 free slices),
-//               2-4 s2 (> 0, > 1, > 2), 5-8 cc3 (> 0 .. > 3), 9 v0 (> 0), 10 -alpha t0^2;
-//               window e (e = 1 when x is the stage-0 profile: every multiplicity shifted
-//               by one) is read at offset e
-//   55 + x      a2[x] = alpha t2^2      \  the row cache: every value that depends only on
-//   60 + x      t2[x] = 2 t3 (0: none)   |  the request, the last two stages [b2, b3), [b3, n)
-//   65          v2min (packed)           |  and alpha -- shared by all masks with the same
-//   66, 67      v3min per half (f32)     |  two highest cuts (a "row"), so a lane walking
-//   68, 69      sigma per half (f32)     |  consecutive masks rebuilds them once per row
-//   70, 71      row slack per half (f32) |
-//   72          wide flags               |
-//   73, 74, 75  tag: request, j2 | j3 << 8, alpha_h bits (request ~0 = invalid)
-//   (kWin4 = 76 words = 304 B per thread)
-constexpr int kSlotRow = 55, kSlotTag = 73;
+// Per-thread shared-memory windows of the KS = 4 kernel, [slot][thread] (4-byte,
+// conflict-free, immediate offsets: the stride is the compile-time CTA size): x * 11 + k,
+// x = profile, k = 0-1 s1 (stage 1 gated by > 0 / > 1 free slices), 2-4 s2 (> 0, > 1, > 2),
+// 5-8 cc3 (> 0 .. > 3), 9 v0 (> 0), 10 -alpha t0^2; window e (e = 1 when x is the stage-0
+// profile: every multiplicity shifted by one) is read at offset e.  (A per-thread cache of
+// the stage-2/3 tables across the masks of a row measured 4 % slower: SIMT rebuilds it
+// whenever any lane of the warp leaves its row.)
 
 __device__ __forceinline__ void ks4_cuts(uint32_t m, int& j1, int& j2, int& j3) {
   j1 = __ffs(m) - 1;
@@ -739,166 +730,89 @@ __device__ __forceinline__ void ks4_cuts(uint32_t m, int& j1, int& j2, int& j3) 
   j3 = __ffs(m) - 1;
 }
 
-// per half: scale sigma = 2^(5 - E) with M <= 2^E, M = max(min(bl, tmax), 1)
-__device__ __forceinline__ float ks4_sigma(float bl, float tmax) {
-  const float M = fmaxf(fminf(bl, tmax), 1.f);
-  const uint32_t mb = __float_as_uint(M);
-  const int E = (int)((mb >> 23) & 255u) - 127 + ((mb & 0x7fffffu) != 0u);  // M <= 2^E
-  return __int_as_float((127 + 5 - E) << 23);
-}
-
 template <bool VERIFY>
 __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
-                                           unsigned long long* misses, uint32_t zero, bool exh, uint64_t shiftB,
-                                           uint32_t req) {
+                                           unsigned long long* misses, uint32_t zero, bool exh, uint64_t shiftB) {
   const float INF = __int_as_float(0x7f800000);
   constexpr int nb = search_block(4);  // slot stride: the CTA size, fixed at compile time
-  const int tid = threadIdx.x;
-  h2* slot = rows + tid;
+  h2* slot = rows + threadIdx.x;
   constexpr h2 kInf2 = 0x7c007c00u, kNegInf2 = 0xfc00fc00u, kGuard = 0x80008000u;
   const float al = c.alpha_h, one_m_a = 1.f - c.alpha_h;
   const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
   const uint32_t* PL = c.sm + c.o_pl + c.row0 * kRowW;  // prefix rows of the request's chain
   const uint32_t* PM = c.sm + c.o_pm + c.row0;
   const uint32_t* XF = c.sm + c.o_xf + c.row0;          // XF[j]: cut after component j
-  int j1[2], j2[2], j3[2];
-  ks4_cuts(maskA, j1[0], j2[0], j3[0]);
-  ks4_cuts(maskB, j1[1], j2[1], j3[1]);
-  const bool same_row = j2[0] == j2[1] && j3[0] == j3[1];
-  const uint32_t tag_row = (uint32_t)j2[0] | ((uint32_t)j3[0] << 8);
-  const bool hit = same_row && slot[kSlotTag * nb] == req && slot[(kSlotTag + 1) * nb] == tag_row &&
-                   slot[(kSlotTag + 2) * nb] == __float_as_uint(al);
-  // X23: cost of the two highest cuts per half (the per-row part of the mask's transfer cost)
-  uint32_t X23[2];
-#pragma unroll
-  for (int h = 0; h < 2; ++h) X23[h] = XF[j2[h]] + XF[j3[h]];
-  if (!hit) {
-    // ---- row part: stages 2 = [b2, b3) and 3 = [b3, n) --------------------------------
-    // sigma from the row's largest budget (the mask's own X1 >= 0 only lowers it), so
-    // every feasible candidate of every mask of the row has T sigma <= 32
-    float sig[2], slr[2], v3m[2] = {INF, INF};
-    uint32_t wide = 0;
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const float bl = (X23[h] <= c.B && !c.none_can_win) ? (float)min(c.B - X23[h], 1u << 24) : -1.f;
-      sig[h] = ks4_sigma(bl, c.tmax);
-      slr[h] = bl >= 0.f ? fmaxf(fminf(bl, c.tmax), 1.f) * sig[h] * (1.f + 1.f / 128.f) : -INF;
-      if (bl >= 0.f && c.tmin * sig[h] < 0.125f) wide |= 1u << h;  // f16 underflow could matter
-    }
-    h2 P2[kP], P3[kP], v2min = kInf2;
-    {
-      float t2f[2][kP], t3f[2][kP];
-      uint32_t m2[2], m3[2];
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const uint32_t b2 = j2[h] + 1, b3 = j3[h] + 1;
-        const float4 l2 = *reinterpret_cast<const float4*>(PL + b2 * kRowW);
-        const float4 l3 = *reinterpret_cast<const float4*>(PL + b3 * kRowW);
-        const float4 ln = *reinterpret_cast<const float4*>(PL + c.n * kRowW);
-        const float e2 = __uint_as_float(PL[b2 * kRowW + 4]), e3 = __uint_as_float(PL[b3 * kRowW + 4]);
-        const float en = __uint_as_float(PL[c.n * kRowW + 4]);
-        t2f[h][0] = l3.x - l2.x; t2f[h][1] = l3.y - l2.y; t2f[h][2] = l3.z - l2.z; t2f[h][3] = l3.w - l2.w;
-        t2f[h][4] = e3 - e2;
-        t3f[h][0] = ln.x - l3.x; t3f[h][1] = ln.y - l3.y; t3f[h][2] = ln.z - l3.z; t3f[h][3] = ln.w - l3.w;
-        t3f[h][4] = en - e3;
-        m2[h] = PM[b3] - PM[b2];
-        m3[h] = PM[c.n] - PM[b3];
-      }
-#pragma unroll
-      for (int x = 0; x < kP; ++x) {
-        const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-        const uint32_t cap = c.sm[c.o_cap + x];
-        float v2[2], u3[2];
-#pragma unroll
-        for (int h = 0; h < 2; ++h) {  // memory and the throughput floor (R38) folded
-          v2[h] = (m2[h] <= cap && t2f[h][x] <= c.thr) ? t2f[h][x] * sig[h] : INF;
-          const float v3 = (m3[h] <= cap && t3f[h][x] <= c.thr) ? t3f[h][x] * sig[h] : INF;
-          // a last stage longer than the (widened) row slack on its own is inadmissible: no
-          // candidate holding it is feasible, and t3 sigma <= slack < 33 stays far from the
-          // f16 INF pattern (no overflow in t3^2)
-          u3[h] = v3 <= slr[h] ? v3 : INF;
-          if (fr > 0) v3m[h] = fminf(v3m[h], u3[h]);
-        }
-        P2[x] = h2pack(v2[0], v2[1]);
-        P3[x] = h2pack(u3[0], u3[1]);
-        if (fr > 0) v2min = h2min(v2min, P2[x]);
-      }
-    }
-#pragma unroll
-    for (int x = 0; x < kP; ++x) {
-      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-      const h2 p2 = P2[x], p3 = P3[x];
-      // last stage as (2 t3, (1 - alpha_h) t3^2); an inadmissible one (INF) as (0, -INF), so
-      // its score y = S3 * 2t3 + cc is -INF for every finite S3 (no INF * 0, no INF - INF)
-      const uint32_t inf3 = ((p3 & 0xffffu) == 0x7c00u ? 0x0000ffffu : 0u) | ((p3 >> 16) == 0x7c00u ? 0xffff0000u : 0u);
-      const h2 cc = (h2mul(h2mul(p3, p3), oma2) & ~inf3) | (kNegInf2 & inf3);
-      h2* r = slot + (x * 11) * nb;
-      r[2 * nb] = fr > 0 ? p2 : kInf2;
-      r[3 * nb] = fr > 1 ? p2 : kInf2;
-      r[4 * nb] = fr > 2 ? p2 : kInf2;
-      r[5 * nb] = fr > 0 ? cc : kNegInf2;
-      r[6 * nb] = fr > 1 ? cc : kNegInf2;
-      r[7 * nb] = fr > 2 ? cc : kNegInf2;
-      r[8 * nb] = fr > 3 ? cc : kNegInf2;
-      slot[(kSlotRow + x) * nb] = h2mul(h2mul(p2, p2), al2);
-      slot[(kSlotRow + 5 + x) * nb] = h2add(p3, p3) & ~inf3;
-    }
-    slot[(kSlotRow + 10) * nb] = v2min;
-    slot[(kSlotRow + 11) * nb] = __float_as_uint(v3m[0]);
-    slot[(kSlotRow + 12) * nb] = __float_as_uint(v3m[1]);
-    slot[(kSlotRow + 13) * nb] = __float_as_uint(sig[0]);
-    slot[(kSlotRow + 14) * nb] = __float_as_uint(sig[1]);
-    slot[(kSlotRow + 15) * nb] = __float_as_uint(slr[0]);
-    slot[(kSlotRow + 16) * nb] = __float_as_uint(slr[1]);
-    slot[(kSlotRow + 17) * nb] = wide;
-    slot[kSlotTag * nb] = same_row ? req : ~0u;
-    slot[(kSlotTag + 1) * nb] = tag_row;
-    slot[(kSlotTag + 2) * nb] = __float_as_uint(al);
-  }
-  // ---- mask part: stages 0 = [0, b1) and 1 = [b1, b2) ---------------------------------
-  const h2 v2min = slot[(kSlotRow + 10) * nb];
-  const float v3m[2] = {__uint_as_float(slot[(kSlotRow + 11) * nb]), __uint_as_float(slot[(kSlotRow + 12) * nb])};
-  const float sig[2] = {__uint_as_float(slot[(kSlotRow + 13) * nb]), __uint_as_float(slot[(kSlotRow + 14) * nb])};
-  const uint32_t wide = slot[(kSlotRow + 17) * nb];
-  float slack[2];
+  // per half: the stage times of its four stages from the five prefix rows 0 (= 0), b1,
+  // b2, b3, n (shared by adjacent stages), the stage memories, the budget
+  float f[2][4][kP], sig[2], slack[2];
+  uint32_t ms[2][4];
+  bool wide[2];
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
-    const uint32_t X = XF[j1[h]] + X23[h];
-    const bool live_h = h == 0 || haveB;  // the B half of a single mask is a dummy: nothing passes
-    const float bl = (live_h && X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
-    // SLO slack M sigma (1 + 2^-7) (clamping Blim to tmax changes no candidate's SLO outcome:
-    // T <= tmax always)
-    slack[h] = bl >= 0.f ? fmaxf(fminf(bl, c.tmax), 1.f) * sig[h] * (1.f + 1.f / 128.f) : -INF;
-  }
-  h2 P0[kP], P1[kP], v1min = kInf2;
-  {
-    float t0f[2][kP], t1f[2][kP];
-    uint32_t m0[2], m1[2];
+    int j1, j2, j3;
+    ks4_cuts(h ? maskB : maskA, j1, j2, j3);
+    const uint32_t b[5] = {0u, (uint32_t)j1 + 1, (uint32_t)j2 + 1, (uint32_t)j3 + 1, c.n};
+    float pr[5][kP];
 #pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const uint32_t b1 = j1[h] + 1, b2 = j2[h] + 1;
-      const float4 l1 = *reinterpret_cast<const float4*>(PL + b1 * kRowW);
-      const float4 l2 = *reinterpret_cast<const float4*>(PL + b2 * kRowW);
-      const float e1 = __uint_as_float(PL[b1 * kRowW + 4]), e2 = __uint_as_float(PL[b2 * kRowW + 4]);
-      t0f[h][0] = l1.x; t0f[h][1] = l1.y; t0f[h][2] = l1.z; t0f[h][3] = l1.w; t0f[h][4] = e1;  // PL[0] = 0
-      t1f[h][0] = l2.x - l1.x; t1f[h][1] = l2.y - l1.y; t1f[h][2] = l2.z - l1.z; t1f[h][3] = l2.w - l1.w;
-      t1f[h][4] = e2 - e1;
-      m0[h] = PM[b1];
-      m1[h] = PM[b2] - PM[b1];
+    for (int i = 0; i < 5; ++i) {
+      if (i == 0) {
+#pragma unroll
+        for (int x = 0; x < kP; ++x) pr[0][x] = 0.f;
+        continue;
+      }
+      const float4 l = *reinterpret_cast<const float4*>(PL + b[i] * kRowW);
+      pr[i][0] = l.x;
+      pr[i][1] = l.y;
+      pr[i][2] = l.z;
+      pr[i][3] = l.w;
+      pr[i][4] = __uint_as_float(PL[b[i] * kRowW + 4]);
     }
 #pragma unroll
-    for (int x = 0; x < kP; ++x) {
-      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-      const uint32_t cap = c.sm[c.o_cap + x];
-      float v0[2], v1[2];
+    for (int s = 0; s < 4; ++s) {
 #pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        v0[h] = (m0[h] <= cap && t0f[h][x] <= c.thr) ? t0f[h][x] * sig[h] : INF;
-        v1[h] = (m1[h] <= cap && t1f[h][x] <= c.thr) ? t1f[h][x] * sig[h] : INF;
-      }
-      P0[x] = h2pack(v0[0], v0[1]);
-      P1[x] = h2pack(v1[0], v1[1]);
-      if (fr > 0) v1min = h2min(v1min, P1[x]);
+      for (int x = 0; x < kP; ++x) f[h][s][x] = pr[s + 1][x] - pr[s][x];
+      ms[h][s] = PM[b[s + 1]] - PM[b[s]];
+    }
+    const uint32_t X = XF[j1] + XF[j2] + XF[j3];
+    const bool live_h = h == 0 || haveB;  // the B half of a single mask is a dummy: nothing passes
+    const float bl = (live_h && X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
+    // scale sigma = 2^(5 - E) with M = min(Blim, tmax) <= 2^E, so every feasible candidate
+    // (T <= M) has T sigma <= 32; the SLO slack is M sigma (1 + 2^-7) (clamping Blim to tmax
+    // changes no candidate's SLO outcome: T <= tmax always)
+    const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+    const uint32_t mb = __float_as_uint(M);
+    const int E = (int)((mb >> 23) & 255u) - 127 + ((mb & 0x7fffffu) != 0u);  // M <= 2^E
+    sig[h] = __int_as_float((127 + 5 - E) << 23);
+    wide[h] = bl >= 0.f && c.tmin * sig[h] < 0.125f;  // f16 underflow could matter: exact path
+    slack[h] = bl >= 0.f ? M * sig[h] * (1.f + 1.f / 128.f) : -INF;
+  }
+  // the packed stage tables and the per-half minima the stage-0 bound needs
+  h2 P0[kP], P1[kP], P2[kP], P3[kP];
+  float v3m[2] = {INF, INF};  // fastest admissible last stage per half (>= 1 free slice)
+  h2 v1min = kInf2, v2min = kInf2;
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const uint32_t cap = c.sm[c.o_cap + x];
+    float vm[2][4];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int s = 0; s < 4; ++s)  // memory and the throughput floor (R38) folded
+        vm[h][s] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * sig[h] : INF;
+    P0[x] = h2pack(vm[0][0], vm[1][0]);
+    P1[x] = h2pack(vm[0][1], vm[1][1]);
+    P2[x] = h2pack(vm[0][2], vm[1][2]);
+    // a last stage longer than the (widened) SLO slack on its own is inadmissible too: no
+    // candidate holding it is feasible, and the bound keeps t3 and t3^2 far from overflow
+    // (an admissible t3 sigma <= slack < 33 never packs to the f16 INF pattern)
+    const float u0 = vm[0][3] <= slack[0] ? vm[0][3] : INF, u1 = vm[1][3] <= slack[1] ? vm[1][3] : INF;
+    P3[x] = h2pack(u0, u1);
+    if (fr > 0) {
+      v3m[0] = fminf(v3m[0], u0);
+      v3m[1] = fminf(v3m[1], u1);
+      v1min = h2min(v1min, P1[x]);
+      v2min = h2min(v2min, P2[x]);
     }
   }
   // guarded SLO slack of the fastest admissible last stage (h2guard): S3 <= slack - v3min
@@ -921,18 +835,29 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   uint32_t pendA = 0, pendB = 0;
   // no live iteration (the common case in bounded mode): nothing else to set up
   if (VERIFY || live != 0) {
-    // the stage-0/1 windows and the register tables of the scoring core
+    // the per-thread windows and the register tables of the scoring core
     h2 a1[kP], a2[kP], t2[kP];
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
       const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-      const h2 p0 = P0[x], p1 = P1[x];
+      const h2 p0 = P0[x], p1 = P1[x], p2 = P2[x], p3 = P3[x];
       a1[x] = h2mul(h2mul(p1, p1), al2);
-      a2[x] = slot[(kSlotRow + x) * nb];
-      t2[x] = slot[(kSlotRow + 5 + x) * nb];
+      a2[x] = h2mul(h2mul(p2, p2), al2);
+      // last stage as (2 t3, (1 - alpha_h) t3^2); an inadmissible one (INF) as (0, -INF), so
+      // its score y = S3 * 2t3 + cc is -INF for every finite S3 (no INF * 0, no INF - INF)
+      const uint32_t inf3 = ((p3 & 0xffffu) == 0x7c00u ? 0x0000ffffu : 0u) | ((p3 >> 16) == 0x7c00u ? 0xffff0000u : 0u);
+      t2[x] = h2add(p3, p3) & ~inf3;
+      const h2 cc = (h2mul(h2mul(p3, p3), oma2) & ~inf3) | (kNegInf2 & inf3);
       h2* r = slot + (x * 11) * nb;
       r[0 * nb] = fr > 0 ? p1 : kInf2;
       r[1 * nb] = fr > 1 ? p1 : kInf2;
+      r[2 * nb] = fr > 0 ? p2 : kInf2;
+      r[3 * nb] = fr > 1 ? p2 : kInf2;
+      r[4 * nb] = fr > 2 ? p2 : kInf2;
+      r[5 * nb] = fr > 0 ? cc : kNegInf2;
+      r[6 * nb] = fr > 1 ? cc : kNegInf2;
+      r[7 * nb] = fr > 2 ? cc : kNegInf2;
+      r[8 * nb] = fr > 3 ? cc : kNegInf2;
       r[9 * nb] = fr > 0 ? p0 : kInf2;
       r[10 * nb] = h2mul(h2mul(p0, p0), nal2);
     }
@@ -990,8 +915,8 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     }
   }
   constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
-  if (wide & 1u) pendA = kAll;  // dynamic range too wide for f16: every block exactly
-  if (wide & 2u) pendB = kAll;
+  if (wide[0]) pendA = kAll;  // dynamic range too wide for f16: every block exactly
+  if (wide[1]) pendB = kAll;
   if (VERIFY || pendA) {
     Geo4 G;
     geo4(c, maskA, G);
@@ -1131,10 +1056,8 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += blockDim.x) dst[i] = src[i];
   }
   __syncthreads();
-  // KS = 4: per-thread windows of the shifted variant tables after the image (ks4_pair_h);
-  // the row cache starts invalid
+  // KS = 4: per-thread windows of the shifted variant tables after the image (ks4_pair_h)
   float* rows = reinterpret_cast<float*>(smem + img_words);
-  if constexpr (KS == 4) reinterpret_cast<uint32_t*>(rows)[kSlotTag * search_block(4) + threadIdx.x] = ~0u;
 
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
   const uint32_t lane = threadIdx.x & 31;
@@ -1211,7 +1134,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
       load_request(rkA);
       if constexpr (KS == 4) {
         ks4_pair_h<false>(c, maskA, haveB ? maskB : maskA, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
-                          false, shiftB, r);
+                          false, shiftB);
       } else if constexpr (KS == 3) {
         ks3_pair<false>(c, maskA, haveB ? maskB : maskA, haveB, A.misses, false, shiftB);
       } else if constexpr (KS == 2) {
@@ -1285,7 +1208,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
           const uint32_t maskB = haveB ? gosper_next(mask) : mask;
           if constexpr (KS == 4)
             ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
-                               A.exhaustive != 0, PK, r);
+                               A.exhaustive != 0, PK);
           else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0, PK);
           if (haveB) {
             step = 2;
