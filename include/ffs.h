@@ -327,7 +327,9 @@ ffs_status ffs_plan_ranked(ffs_ctx *ctx, const ffs_request *d_req, const uint32_
  * option o < P = one slice of profile o, o = P + w = split with branch profiles the base-P
  * digits of w (branch 0 most significant); key, feasibility and binding as ffs_plan_keys /
  * ffs_plan_decode with every slice of the plan counted (gpcs, free slices).
- * A table of one-component units reproduces ffs_plan_batch's keys exactly. */
+ * Conditional units (unit_cond, R48) contribute their slowest alternative to a one-slice
+ * stage and offer no split.  A table of one-component units reproduces ffs_plan_batch's
+ * keys exactly. */
 #define FFS_DAG_MAX_UNITS 16
 #define FFS_DAG_MAX_BRANCHES 4
 #define FFS_DAG_MAX_SLOTS 8
@@ -340,6 +342,12 @@ typedef struct {
     const uint8_t *unit_bend;  /* [U][4] function-relative exclusive end component of branch j
                                   (branch j starts where branch j-1, or the previous unit,
                                   ends); entries j >= nb are ignored                         */
+    const uint8_t *unit_cond;  /* [U] nullable: 1 = CONDITIONAL unit (R48, App 3): 2..4
+                                  alternative branches, exactly one runs per request, an empty
+                                  branch is "pass"; the slice hosts every branch, the unit's
+                                  time is its slowest branch, it never splits, a cut after it
+                                  costs the largest branch output (an empty branch: the
+                                  previous component's)                                      */
 } ffs_dag_table;
 
 /* The plan of one request of a DAG function (88 bytes).  Slots: the plan's slices in
@@ -364,7 +372,8 @@ typedef struct {
 /* Validate and upload the unit structure for plans with up to k_max stages (host work:
  * the per-function list of unit-cut masks with candidate offsets).  Synchronous.
  * FFS_ERR_ARG: n_funcs differs from the staged table, units not covering a chain, a
- * branch count outside 1..4, an empty branch, a one-branch unit of more than one
+ * branch count outside 1..4 (2..4 for a conditional unit), an empty branch outside a
+ * conditional unit, a unit without components, a one-branch unit of more than one
  * component.  FFS_ERR_RANGE: > 16 units, k_max not in 1..8, k_max * max branches > 8,
  * k_max * max branches * max gpcs >= 64, >= 2^41 candidates for a function.
  * FFS_ERR_STATE: tables not staged (staging new tables drops the DAG). */

@@ -57,7 +57,7 @@ class _PlanArgs(C.Structure):
 
 class _DagArgs(C.Structure):
     _fields_ = [
-        ("unit_off", C.c_void_p), ("unit_nb", C.c_void_p), ("unit_bend", C.c_void_p),
+        ("unit_off", C.c_void_p), ("unit_nb", C.c_void_p), ("unit_bend", C.c_void_p), ("unit_cond", C.c_void_p),
         ("key", C.c_void_p), ("status", C.c_void_p), ("k", C.c_void_p), ("slice", C.c_void_p),
         ("cut_mask", C.c_void_p), ("split_mask", C.c_void_p), ("e2e_us", C.c_void_p),
         ("bottleneck_us", C.c_void_p), ("gpcs_out", C.c_void_p), ("cvq", C.c_void_p), ("n_slots", C.c_void_p),
@@ -155,7 +155,7 @@ def plan(prob, k_max: int | None = None, threads: int | None = None, checks: boo
 def plan_dag(prob, dag, k_max: int | None = None, threads: int | None = None, checks: bool = True) -> dict:
     """Brute-force plan of every request of ``prob`` whose functions have the unit
     structure ``dag`` (unit_off, unit_nb, unit_bend[U,4]; see ffs_oracle.c:
-    oracle_plan_dag, R40-R43).  Returns key, status, k, cut_mask (over unit
+    oracle_plan_dag, R40-R43, R48 for conditional units).  Returns key, status, k, cut_mask (over unit
     boundaries), split_mask (bit s: stage s runs its branches on separate slices),
     e2e_us, bottleneck_us, gpcs, cvq, n_slots, prof[R,8], slice[R,8] and checks[R,3]."""
     k_max = int(prob.k_max if k_max is None else k_max)
@@ -163,6 +163,8 @@ def plan_dag(prob, dag, k_max: int | None = None, threads: int | None = None, ch
     h = _Held(prob, k_max, False)
     R = prob.R
     uo, nb, be = _c(dag.unit_off, np.uint32), _c(dag.unit_nb, np.uint8), _c(dag.unit_bend, np.uint8)
+    cond = getattr(dag, "unit_cond", None)
+    cd = None if cond is None else _c(cond, np.uint8)  # R48 conditional units (nullable)
     o = {"key": np.zeros(R, np.int64), "status": np.zeros(R, np.int32), "k": np.zeros(R, np.int32),
          "slice": np.zeros((R, 8), np.int32), "cut_mask": np.zeros(R, np.uint32),
          "split_mask": np.zeros(R, np.uint32), "e2e_us": np.zeros(R, np.uint32),
@@ -170,7 +172,7 @@ def plan_dag(prob, dag, k_max: int | None = None, threads: int | None = None, ch
          "n_slots": np.zeros(R, np.uint32), "prof": np.zeros((R, 8), np.uint8)}
     if checks:
         o["checks"] = np.zeros((R, 3), np.uint64)
-    d = _DagArgs(_p(uo), _p(nb), _p(be), _p(o["key"]), _p(o["status"]), _p(o["k"]), _p(o["slice"]),
+    d = _DagArgs(_p(uo), _p(nb), _p(be), _p(cd) if cd is not None else None, _p(o["key"]), _p(o["status"]), _p(o["k"]), _p(o["slice"]),
                  _p(o["cut_mask"]), _p(o["split_mask"]), _p(o["e2e_us"]), _p(o["bottleneck_us"]),
                  _p(o["gpcs"]), _p(o["cvq"]), _p(o["n_slots"]), _p(o["prof"]),
                  _p(o["checks"]) if checks else None)

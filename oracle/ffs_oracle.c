@@ -1055,6 +1055,15 @@ int oracle_sim(const oracle_plan_args *a, int T, const uint32_t *req_off, const 
  *       idx = the candidate's position; key, feasibility and binding as R1-R11 with every
  *       slice of the plan counted (gpcs, free slices), slots in stage then branch order;
  *       k_max * (max branches) <= 8, so a plan holds at most 8 slices.
+ *   R48 a CONDITIONAL unit (App 3, Table 4: "Deblur -> (if low resolution: -> Super
+ *       resolution; else: pass) -> ...") holds 2..4 alternative branches of which exactly
+ *       one runs per request (a branch may be empty: "pass"): the instance hosts all of
+ *       them (memory = every branch's components), the unit's time on a slice is its
+ *       slowest branch (the SLO must hold whichever branch a request takes; the profile
+ *       table carries no branch probabilities), alternatives are never split over slices,
+ *       and a cut after the unit moves the output of the branch that ran: the largest of
+ *       the branches' last-component xfer_us (an empty branch passes the previous
+ *       component's output; nothing before the first component).
  * A DAG of one-component units is the chain of oracle_plan, candidate for candidate. */
 #define DAG_MAX_UNITS 16
 #define DAG_MAX_BR 4
@@ -1064,6 +1073,7 @@ typedef struct {
     const uint32_t *unit_off; /* [F+1] */
     const uint8_t *unit_nb;   /* [U] branches, 1..4 */
     const uint8_t *unit_bend; /* [U][4] function-relative exclusive end component of branch j */
+    const uint8_t *unit_cond; /* [U] nullable: 1 = conditional unit (R48) */
     int64_t *key;
     int32_t *status, *k, *slice /* [R][8] */;
     uint32_t *cut_mask, *split_mask, *e2e_us, *bottleneck_us, *gpcs_out, *cvq, *n_slots;
@@ -1072,9 +1082,22 @@ typedef struct {
 } oracle_dag_args;
 
 typedef struct {
-    int nb, c0;               /* branches, first component (function-relative) */
+    int nb, c0, cond;         /* branches, first component (function-relative), R48 */
     int bc0[DAG_MAX_BR], bc1[DAG_MAX_BR]; /* branch j = components [bc0, bc1) */
 } dag_unit;
+
+/* cost of a cut right after unit un (R42; R48 for a conditional unit) */
+static uint64_t dag_cut_cost(const oracle_plan_args *a, uint32_t base, const dag_unit *un) {
+    uint64_t x = 0;
+    for (int j = 0; j < un->nb; j++) {
+        uint64_t xb = 0;
+        if (un->bc1[j] > un->bc0[j]) xb = a->xfer_us[base + (uint32_t)un->bc1[j] - 1];
+        else if (un->c0 > 0) xb = a->xfer_us[base + (uint32_t)un->c0 - 1]; /* "pass" */
+        if (un->cond) x = xb > x ? xb : x;
+        else x += xb;
+    }
+    return x;
+}
 
 static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, int r) {
     const int P = a->P;
@@ -1099,6 +1122,7 @@ static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, in
         const uint32_t gu = d->unit_off[f] + (uint32_t)u;
         U[u].nb = d->unit_nb[gu];
         U[u].c0 = c;
+        U[u].cond = d->unit_cond ? d->unit_cond[gu] : 0;
         for (int j = 0; j < U[u].nb; j++) {
             U[u].bc0[j] = c;
             U[u].bc1[j] = d->unit_bend[(size_t)gu * DAG_MAX_BR + j];
@@ -1124,8 +1148,7 @@ static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, in
             uint64_t xfer = 0;
             for (int u = 0; u < m; u++) {
                 const int cut = u < m - 1 && ((mask >> u) & 1u);
-                if (cut) /* R42: every branch output of unit u moves */
-                    for (int j = 0; j < U[u].nb; j++) xfer += a->xfer_us[base + (uint32_t)U[u].bc1[j] - 1];
+                if (cut) xfer += dag_cut_cost(a, base, &U[u]);
                 if (u == m - 1 || cut) {
                     su1[st] = u;
                     st++;
@@ -1134,7 +1157,7 @@ static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, in
             }
             uint64_t nopt[ORACLE_MAX_STAGES], total = 1;
             for (int s = 0; s < k; s++) {
-                const int blk = su0[s] == su1[s] && U[su0[s]].nb >= 2;
+                const int blk = su0[s] == su1[s] && U[su0[s]].nb >= 2 && !U[su0[s]].cond;
                 uint64_t pb = 1;
                 if (blk)
                     for (int j = 0; j < U[su0[s]].nb; j++) pb *= (uint64_t)P;
@@ -1154,12 +1177,19 @@ static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, in
                     if (opt[s] < (uint64_t)P) { /* one slice: every component of the stage */
                         const int p = (int)opt[s];
                         uint64_t ts = 0, ms = 0;
-                        for (int u = su0[s]; u <= su1[s]; u++)
-                            for (int j = 0; j < U[u].nb; j++)
+                        for (int u = su0[s]; u <= su1[s]; u++) {
+                            uint64_t tu = 0; /* the unit's time: sum, or the slowest alternative (R48) */
+                            for (int j = 0; j < U[u].nb; j++) {
+                                uint64_t tb = 0;
                                 for (int cc = U[u].bc0[j]; cc < U[u].bc1[j]; cc++) {
-                                    ts += lat_of(a, f, cc, p);
+                                    tb += lat_of(a, f, cc, p);
                                     ms += a->mem_mib[base + (uint32_t)cc];
                                 }
+                                if (U[u].cond) tu = tb > tu ? tb : tu;
+                                else tu += tb;
+                            }
+                            ts += tu;
+                        }
                         if (ms > a->cap_mib[p]) feasible = 0;
                         t[s] = ts;
                         prof[nsl++] = p;
@@ -1244,11 +1274,16 @@ static void plan_dag_one(const oracle_plan_args *a, const oracle_dag_args *d, in
                 if (tb > tcur) tcur = tb;
             }
         } else {
-            for (int j = 0; j < U[u].nb; j++)
-                for (int cc = U[u].bc0[j]; cc < U[u].bc1[j]; cc++) tcur += lat_of(a, f, cc, best_prof[slot]);
+            uint64_t tu = 0;
+            for (int j = 0; j < U[u].nb; j++) {
+                uint64_t tb = 0;
+                for (int cc = U[u].bc0[j]; cc < U[u].bc1[j]; cc++) tb += lat_of(a, f, cc, best_prof[slot]);
+                if (U[u].cond) tu = tb > tu ? tb : tu;
+                else tu += tb;
+            }
+            tcur += tu;
         }
-        if (cut)
-            for (int j = 0; j < U[u].nb; j++) e2e += a->xfer_us[base + (uint32_t)U[u].bc1[j] - 1];
+        if (cut) e2e += dag_cut_cost(a, base, &U[u]);
         if (u == m - 1 || cut) {
             e2e += tcur;
             if (tcur > bott) bott = tcur;
@@ -1306,13 +1341,16 @@ int oracle_plan_dag(const oracle_plan_args *a, const oracle_dag_args *d, int n_t
         for (int u = 0; u < m; u++) {
             const uint32_t gu = d->unit_off[f] + (uint32_t)u;
             const int nb = d->unit_nb[gu];
-            if (nb < 1 || nb > DAG_MAX_BR) return -1;
-            if ((uint32_t)nb > maxnb) maxnb = (uint32_t)nb;
+            const int cond = d->unit_cond ? d->unit_cond[gu] : 0;
+            if (nb < 1 || nb > DAG_MAX_BR || (cond && nb < 2)) return -1;
+            if (!cond && (uint32_t)nb > maxnb) maxnb = (uint32_t)nb; /* alternatives never split */
+            const int start = c;
             for (int j = 0; j < nb; j++) {
                 const int e = d->unit_bend[(size_t)gu * DAG_MAX_BR + j];
-                if (e <= c) return -1;
+                if (cond ? e < c : e <= c) return -1; /* an alternative may be empty ("pass") */
                 c = e;
             }
+            if (c == start) return -1; /* a unit holds at least one component */
         }
         if (c != n) return -1;
         for (int u = 0; u < m; u++) { /* a one-branch unit is one component */

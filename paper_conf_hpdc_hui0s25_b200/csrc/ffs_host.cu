@@ -81,7 +81,7 @@ struct ffs_ctx {
   // NEXT-1 ranked partitions
   DevBuf rank_off, rank_mask;
   // NEXT-1 DAG stages
-  DevBuf dag_fu, dag_units, dag_xcut, dag_mt_off, dag_mt_mk, dag_mt_cand;
+  DevBuf dag_fu, dag_units, dag_xcut, dag_mt_off, dag_mt_mk, dag_mt_cand, dag_sv;
   bool dag_staged = false;
   bool ranked = false;
   uint32_t rank_kmax = 0, prof_order = 0;
@@ -175,7 +175,7 @@ void ffs_destroy(ffs_ctx* c) {
     for (DevBuf* b : {&c->node_off, &c->j_keys, &c->j_state, &c->j_dirty, &c->j_sreq, &c->j_sslo, &c->j_skeys,
                       &c->j_win, &c->j_busy, &c->j_cnt, &c->j_free, &c->j_ctr})
       b->release();
-    for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand,
+    for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand, &c->dag_sv,
                       &c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr,
                       &c->gofs, &c->grp, &c->live_list})
@@ -820,6 +820,10 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
   const std::vector<uint32_t>& img = c->h_image;
   const uint32_t F = c->F, U = d->unit_off[F];
   std::vector<uint32_t> fu(2 * (size_t)F), units(6 * (size_t)std::max(U, 1u), 0), xcut(std::max(U, 1u), 0);
+  // per function m + 1 rows of 8: prefix over its units of the conditional units'
+  // one-slice saving (sum of the alternatives' times - the slowest), R48
+  std::vector<uint32_t> sv(8 * ((size_t)U + F), 0);
+  auto plat = [&](uint32_t row, uint32_t p) { return img[L.o_pl + row * kRowW + p]; };  // host copy: integers
   uint32_t maxnb = 1;
   for (uint32_t f = 0; f < F; ++f) {
     if (d->unit_off[f + 1] < d->unit_off[f]) return fail(c, FFS_ERR_ARG, "unit_off decreasing at %u", f);
@@ -830,23 +834,39 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
     fu[2 * f] = d->unit_off[f];
     fu[2 * f + 1] = m;
     uint32_t cc = 0;
+    uint32_t* svf = sv.data() + 8 * ((size_t)d->unit_off[f] + f);
     for (uint32_t u = d->unit_off[f]; u < d->unit_off[f + 1]; ++u) {
       const uint32_t nb = d->unit_nb[u];
+      const bool cond = d->unit_cond && d->unit_cond[u];
       if (nb < 1 || nb > FFS_DAG_MAX_BRANCHES) return fail(c, FFS_ERR_ARG, "unit %u: %u branches not in 1..4", u, nb);
-      maxnb = std::max(maxnb, nb);
-      units[6 * (size_t)u] = nb;
+      if (cond && nb < 2) return fail(c, FFS_ERR_ARG, "conditional unit %u: %u alternatives", u, nb);
+      if (!cond) maxnb = std::max(maxnb, nb);  // alternatives never split (R48)
+      units[6 * (size_t)u] = nb | (cond ? 1u << 8 : 0u);
       units[6 * (size_t)u + 1] = cc;
       const uint32_t start = cc;
-      uint32_t x = 0;
+      uint32_t x = 0, tsum[kP] = {0, 0, 0, 0, 0}, tmax[kP] = {0, 0, 0, 0, 0};
       for (uint32_t j = 0; j < nb; ++j) {
         const uint32_t e = d->unit_bend[4 * (size_t)u + j];
-        if (e <= cc || e > n) return fail(c, FFS_ERR_ARG, "unit %u branch %u: end %u not in (%u, %u]", u, j, e, cc, n);
+        if ((cond ? e < cc : e <= cc) || e > n)
+          return fail(c, FFS_ERR_ARG, "unit %u branch %u: end %u not in (%u, %u]", u, j, e, cc, n);
         units[6 * (size_t)u + 2 + j] = e;
-        x += img[L.o_xf + row0 + e - 1];  // R42: every branch output moves at a cut
+        // R42: every branch output moves at a cut; R48: the alternative that ran (worst
+        // case), an empty one passing the previous component's output
+        const uint32_t xb = e > cc ? img[L.o_xf + row0 + e - 1] : (start > 0 ? img[L.o_xf + row0 + start - 1] : 0u);
+        x = cond ? std::max(x, xb) : x + xb;
+        for (uint32_t p = 0; p < (uint32_t)kP; ++p) {
+          const uint32_t tb = plat(row0 + e, p) - plat(row0 + cc, p);
+          tsum[p] += tb;
+          tmax[p] = std::max(tmax[p], tb);
+        }
         cc = e;
       }
+      if (cc == start) return fail(c, FFS_ERR_ARG, "unit %u has no components", u);
       if (nb == 1 && cc != start + 1) return fail(c, FFS_ERR_ARG, "unit %u: one branch of %u components", u, cc - start);
       xcut[u] = x;
+      const uint32_t lu = u - d->unit_off[f];
+      for (uint32_t p = 0; p < 8; ++p)
+        svf[8 * (lu + 1) + p] = svf[8 * lu + p] + (cond && p < (uint32_t)kP ? tsum[p] - tmax[p] : 0u);
     }
     if (cc != n) return fail(c, FFS_ERR_ARG, "function %u: units cover %u of %u components", f, cc, n);
   }
@@ -869,9 +889,10 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
         uint32_t u0 = 0;
         for (uint32_t u = 0; u < m; ++u)
           if (u + 1 == m || ((mask >> u) & 1u)) {
-            const uint32_t nb = units[6 * (size_t)(ub + u0)];
+            const uint32_t nb = units[6 * (size_t)(ub + u0)] & 0xffu;
+            const bool cond = (units[6 * (size_t)(ub + u0)] >> 8) != 0;
             uint64_t q = kP;
-            if (u0 == u && nb >= 2) {
+            if (u0 == u && nb >= 2 && !cond) {
               uint64_t pw = 1;
               for (uint32_t j = 0; j < nb; ++j) pw *= kP;
               q += pw;
@@ -893,6 +914,7 @@ ffs_status ffs_dag_stage(ffs_ctx* c, const ffs_dag_table* d, uint32_t k_max) {
   CK(up(c->dag_fu, fu.data(), fu.size() * 4), "upload dag_fu");
   CK(up(c->dag_units, units.data(), units.size() * 4), "upload dag_units");
   CK(up(c->dag_xcut, xcut.data(), xcut.size() * 4), "upload dag_xcut");
+  CK(up(c->dag_sv, sv.data(), sv.size() * 4), "upload dag_sv");
   CK(up(c->dag_mt_off, mt_off.data(), mt_off.size() * 4), "upload dag_mt_off");
   CK(up(c->dag_mt_mk, mt_mk.data(), mt_mk.size() * 4), "upload dag_mt_mk");
   CK(up(c->dag_mt_cand, mt_cand.data(), mt_cand.size() * 8), "upload dag_mt_cand");
@@ -919,6 +941,7 @@ ffs_status ffs_plan_dag(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_
   a.fu = c->dag_fu.as<uint32_t>();
   a.units = c->dag_units.as<uint32_t>();
   a.xcut = c->dag_xcut.as<uint32_t>();
+  a.sv = c->dag_sv.as<uint32_t>();
   a.mt_off = c->dag_mt_off.as<uint32_t>();
   a.mt_mk = c->dag_mt_mk.as<uint32_t>();
   a.mt_cand = c->dag_mt_cand.as<unsigned long long>();

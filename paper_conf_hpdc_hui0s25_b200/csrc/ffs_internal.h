@@ -198,7 +198,9 @@ struct DagArgs {
   const int32_t* free_list;
   const uint32_t* fu;         // [F][2] {first unit, units}
   const uint32_t* units;      // [U][6] {nb, c0, e0, e1, e2, e3} function-relative components
-  const uint32_t* xcut;       // [U] cost of a cut after the unit (R42)
+  const uint32_t* xcut;       // [U] cost of a cut after the unit (R42, R48)
+  const uint32_t* sv;         // [U + F][8] per function (rows fu[2f] + f ..): prefix over its units
+                              // of the conditional units' one-slice saving sum - max (R48)
   const uint32_t* mt_off;     // [F+1] mask-table entries of f
   const uint32_t* mt_mk;      // unit-cut mask | k << 16
   const unsigned long long* mt_cand;  // first candidate index of the entry

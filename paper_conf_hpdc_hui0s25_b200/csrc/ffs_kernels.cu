@@ -3043,10 +3043,12 @@ __device__ __forceinline__ uint32_t dag_lat(const DagArgs& A, uint32_t row0, uin
   return __float2uint_rn(plf(A.image, A.lay.o_pl + (row0 + b) * kRowW + p) - plf(A.image, A.lay.o_pl + (row0 + a) * kRowW + p));
 }
 
-// options of the stage made of units [u0, u1]: P, plus P^nb splits when it is one block
+// options of the stage made of units [u0, u1]: P, plus P^nb splits when it is one
+// fork/join block (a conditional unit's alternatives never split, R48; uo[6u] = nb |
+// cond << 8)
 __device__ __forceinline__ uint32_t dag_nopt(const uint32_t* uo, uint32_t u0, uint32_t u1) {
-  const uint32_t nb = uo[6 * u0];
-  if (u0 != u1 || nb < 2) return kP;
+  const uint32_t nb = uo[6 * u0] & 0xffu;
+  if (u0 != u1 || nb < 2 || (uo[6 * u0] >> 8)) return kP;
   uint32_t q = 1;
   for (uint32_t j = 0; j < nb; ++j) q *= kP;
   return kP + q;
@@ -3058,19 +3060,20 @@ __device__ __forceinline__ uint32_t dag_nopt(const uint32_t* uo, uint32_t u0, ui
 // (sums and max are order-free, so the digits are taken least significant first).
 __device__ __forceinline__ uint32_t dag_stage(const DagArgs& A, uint32_t row0, const uint32_t* uo, uint32_t u0,
                                               uint32_t u1, uint32_t o, uint32_t thr, uint32_t& gp, uint64_t& use,
-                                              bool& ok) {
+                                              bool& ok, const uint32_t* sv) {
   const uint32_t* img = A.image;
   const uint32_t* U0 = uo + 6 * u0;
   uint32_t t;
   if (o < (uint32_t)kP) {
     const uint32_t* U1 = uo + 6 * u1;
-    const uint32_t c0 = U0[1], c1 = U1[1 + U1[0]];  // end of the last branch of unit u1
-    t = dag_lat(A, row0, c0, c1, o);
+    const uint32_t c0 = U0[1], c1 = U1[1 + (U1[0] & 0xffu)];  // end of the last branch of unit u1
+    // every component in sequence, minus the conditional units' sum - max (R48)
+    t = dag_lat(A, row0, c0, c1, o) - (sv[8 * (u1 + 1) + o] - sv[8 * u0 + o]);
     ok &= img[A.lay.o_pm + row0 + c1] - img[A.lay.o_pm + row0 + c0] <= img[A.lay.o_cap + o];
     gp += img[A.lay.o_gpcs + o];
     use += 1ull << (8 * o);
   } else {
-    const uint32_t nb = U0[0];
+    const uint32_t nb = U0[0] & 0xffu;
     uint32_t w = o - kP;
     t = 0;
     for (uint32_t jj = nb; jj > 0; --jj) {
@@ -3110,6 +3113,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
   const uint32_t* uo = A.units + 6 * A.fu[2 * f];
   const uint32_t m = A.fu[2 * f + 1];
   const uint32_t* xc = A.xcut + A.fu[2 * f];
+  const uint32_t* sv = A.sv + 8 * (A.fu[2 * f] + f);
   uint64_t best = kKeyNone, scored = 0, nfeas = 0, ksum = 0;
   uint32_t best_mk = 0, best_c = 0;
   uint32_t gpc[kP];
@@ -3151,7 +3155,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
       uint64_t us = 0;
       lg[o] = 0;
       lok[o] = true;
-      lt[o] = dag_stage(A, row0, uo, lu0, lu1, (uint32_t)o, thr, lg[o], us, lok[o]);
+      lt[o] = dag_stage(A, row0, uo, lu0, lu1, (uint32_t)o, thr, lg[o], us, lok[o], sv);
     }
     const bool split2 = nl == kP + kP * kP;
     uint32_t bt[2][kP], bok = 0;
@@ -3176,7 +3180,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         dag_bounds(ends, ss - 1, u0, u1);
         const uint32_t no = dag_nopt(uo, u0, u1), os = rest % no;
         rest /= no;
-        const uint64_t t = dag_stage(A, row0, uo, u0, u1, os, thr, gp0, use0, ok0);
+        const uint64_t t = dag_stage(A, row0, uo, u0, u1, os, thr, gp0, use0, ok0, sv);
         T0 += t;
         Q0 += t * t;
       }
@@ -3226,7 +3230,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
           uint64_t use = use0;
           uint32_t gp = gp0;
           bool ok = true;
-          const uint64_t t = dag_stage(A, row0, uo, lu0, lu1, ol, thr, gp, use, ok);
+          const uint64_t t = dag_stage(A, row0, uo, lu0, lu1, ol, thr, gp, use, ok, sv);
           score(t, gp, use, ok, ol);
         }
       }
@@ -3293,14 +3297,14 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         dag_bounds(ends, s + 1, a0, a1);
         div /= dag_nopt(uo, a0, a1);
       }
-      const uint32_t t = dag_stage(A, row0, uo, u0, u1, os, 0xffffffffu, g, use, ok);
+      const uint32_t t = dag_stage(A, row0, uo, u0, u1, os, 0xffffffffu, g, use, ok, sv);
       e2e += t;
       bott = max(bott, t);
       // slots: one slice, or the branches in order (branch 0 = most significant digit)
       uint32_t nb = 1, w = os, pw = 1;
       if (os >= (uint32_t)kP) {
         P.split_mask |= 1u << s;
-        nb = uo[6 * u0];
+        nb = uo[6 * u0] & 0xffu;
         w = os - kP;
         for (uint32_t j = 1; j < nb; ++j) pw *= kP;
       }

@@ -50,7 +50,8 @@ class _Cluster(C.Structure):
 
 
 class _DagTable(C.Structure):
-    _fields_ = [("n_funcs", C.c_uint32), ("unit_off", C.c_void_p), ("unit_nb", C.c_void_p), ("unit_bend", C.c_void_p)]
+    _fields_ = [("n_funcs", C.c_uint32), ("unit_off", C.c_void_p), ("unit_nb", C.c_void_p), ("unit_bend", C.c_void_p),
+                ("unit_cond", C.c_void_p)]
 
 
 class _EvictParams(C.Structure):
@@ -367,7 +368,9 @@ class Planner:
         uo = np.ascontiguousarray(dag.unit_off, dtype=np.uint32)
         nb = np.ascontiguousarray(dag.unit_nb, dtype=np.uint8)
         be = np.ascontiguousarray(dag.unit_bend, dtype=np.uint8)
-        t = _DagTable(int(uo.shape[0] - 1), _host(uo), _host(nb), _host(be))
+        cond = getattr(dag, "unit_cond", None)
+        cd = None if cond is None else np.ascontiguousarray(cond, dtype=np.uint8)
+        t = _DagTable(int(uo.shape[0] - 1), _host(uo), _host(nb), _host(be), _host(cd) if cd is not None else None)
         self._check(_lib.ffs_dag_stage(self._h, C.byref(t), int(k_max)))
 
     def plan_dag(self, req, slo, out=None, checks=None, stream=None):

@@ -503,12 +503,19 @@ def with_throughput_floor(prob: Problem, seed: int = 0x5EEDF100, lo: float = 0.3
 # a fork/join block of parallel branches (expanded image classification "is
 # extended with two branches to form a DAG")
 # ----------------------------------------------------------------------------------
+class Cond(list):
+    """A conditional unit in a DAG shape (R48, App 3): alternative branches, exactly
+    one runs per request; a branch of length 0 is "pass"."""
+
+
 @dataclass
 class DagTable:
     """Unit structure of every function of a Problem (include/ffs.h ffs_dag_table)."""
     unit_off: np.ndarray   # uint32 [F+1]
     unit_nb: np.ndarray    # uint8  [U] branches 1..4 (1 = one component)
     unit_bend: np.ndarray  # uint8  [U, 4] function-relative exclusive end of branch j (0 unused)
+    unit_cond: np.ndarray | None = None  # uint8 [U] 1 = conditional unit (R48), None = none
+
 
     def units(self, f: int) -> list[list[tuple[int, int]]]:
         """Function f's units as lists of (first, end) component ranges per branch."""
@@ -533,9 +540,13 @@ def chain_dag(prob: Problem) -> DagTable:
     return DagTable(unit_off, np.ones(int(unit_off[-1]), dtype=np.uint8), bend)
 
 
-def make_dag_shapes(rng: SplitMix64, F: int, units=(3, 8), p_block=0.35, branches=(2, 2), br_len=(1, 3)):
-    """Per function: a list of units, each a list of branch lengths."""
+def make_dag_shapes(rng: SplitMix64, F: int, units=(3, 8), p_block=0.35, branches=(2, 2), br_len=(1, 3),
+                    p_cond: float = 0.0):
+    """Per function: a list of units, each a list of branch lengths; with probability
+    p_cond a unit is conditional (App 3's "if low resolution: super resolution; else:
+    pass", P:403): a Cond of one 1..2-component branch and a pass."""
     shapes = []
+    c_rng = rng.sub(17)  # separate stream: p_cond = 0 reproduces the round-1 shapes
     for _ in range(F):
         m = int(rng.integers(units[0], units[1], 1)[0])
         u_list = []
@@ -545,36 +556,42 @@ def make_dag_shapes(rng: SplitMix64, F: int, units=(3, 8), p_block=0.35, branche
                 u_list.append([int(x) for x in rng.integers(br_len[0], br_len[1], nb)])
             else:
                 u_list.append([1])
+            if p_cond and float(c_rng.uniform(1)[0]) < p_cond and len(u_list[-1]) == 1:
+                u_list[-1] = Cond([int(c_rng.integers(1, 2, 1)[0]), 0])
         shapes.append(u_list)
     return shapes
 
 
 def dag_table(shapes) -> DagTable:
+    """Shapes: per function a list of units, each a list of branch lengths (a fork/join
+    block when > 1) or a Cond of alternative branch lengths (0 = pass)."""
     unit_off = np.zeros(len(shapes) + 1, dtype=np.uint32)
     unit_off[1:] = np.cumsum([len(s) for s in shapes])
     U = int(unit_off[-1])
     nb = np.zeros(U, dtype=np.uint8)
     bend = np.zeros((U, 4), dtype=np.uint8)
+    cond = np.zeros(U, dtype=np.uint8)
     u = 0
     for s in shapes:
         c = 0
         for br in s:
             nb[u] = len(br)
+            cond[u] = isinstance(br, Cond)
             for j, L in enumerate(br):
                 c += L
                 bend[u, j] = c
             u += 1
-    return DagTable(unit_off, nb, bend)
+    return DagTable(unit_off, nb, bend, cond if cond.any() else None)
 
 
 def dag_config(seed: int | None = None, R: int = 1 << 16, F: int = 32, node_parts=None, k_max: int = 4,
-               p_block: float = 0.35, units=(3, 8), branches=(2, 2)) -> tuple[Problem, DagTable]:
+               p_block: float = 0.35, units=(3, 8), branches=(2, 2), p_cond: float = 0.0) -> tuple[Problem, DagTable]:
     """CD: DAG functions (3..8 units, a unit a 2-branch block with probability 0.35,
     branches of 1..3 components) on the C3 cluster (8 nodes = 64 GPUs), Azure-shaped
     requests as C3.  Components and budgets follow the chain recipe (make_function,
     R9 SLO on the summed single-slice latency)."""
     rng = SplitMix64(SEED_BASE + 6 if seed is None else seed)
-    shapes = make_dag_shapes(rng.sub(8), F, units, p_block, branches)
+    shapes = make_dag_shapes(rng.sub(8), F, units, p_block, branches, p_cond=p_cond)
     lengths = [sum(sum(br) for br in s) for s in shapes]
     prob = _problem("CD", rng, lengths, NODE_BLOCK if node_parts is None else node_parts, R, k_max=k_max)
     return prob, dag_table(shapes)

@@ -141,3 +141,42 @@ def test_dag_bad_requests_and_errors(F, planner):
         p3, d3 = W.dag_config(R=8, F=4, branches=(4, 4), p_block=1.0)
         planner.stage(p3)
         planner.stage_dag(d3, 4)
+
+
+# ---- R48 conditional units (App 3, Table 4) --------------------------------------
+def app3_5(budget, mem, branch_y, k_max):
+    """test_oracle_dag.app3_like on the P = 5 build: four free 4g.40gb slices; mem MiB per
+    component (12000: the whole function does not fit one slice, [D, X|Y] does)."""
+    lat = [[10] * 5, [20] * 5] + ([[15] * 5] if branch_y else []) + [[30] * 5]
+    xfer = [1, 2] + ([3] if branch_y else []) + [0]
+    f = dict(lat=lat, mem=[mem] * len(lat), xfer=xfer)
+    prob = problem([f], [[[3] * 4]], [(0, 0, budget)], k_max=k_max)
+    return prob, W.dag_table([[[1], W.Cond([1, branch_y]), [1]]])
+
+
+@pytest.mark.parametrize("budget,mem,branch_y,k_max", [(1000, 1000, 1, 2), (1000, 12000, 1, 2), (62, 12000, 1, 2),
+                                                        (1000, 1000, 1, 3), (1000, 12000, 0, 2)])
+def test_dag_conditional_units_hand(F, planner, budget, mem, branch_y, k_max):
+    prob, d = app3_5(budget, mem, branch_y, k_max)
+    g, c = run_dag(F, planner, prob, d)
+    o = oracle.plan_dag(prob, d)
+    assert_dag_equal(g, o, c)
+    assert (g["split_mask"] == 0).all()
+
+
+@pytest.mark.parametrize("seed", range(2030, 2040))
+def test_dag_random_tiny_conditional(F, planner, seed):
+    prob, d = random_dag(seed, K=2 if seed % 3 == 0 else 3, nb_max=4 if seed % 3 == 0 else 2, p_cond=0.4)
+    assert d.unit_cond is not None
+    g, c = run_dag(F, planner, prob, d)
+    assert_dag_equal(g, oracle.plan_dag(prob, d), c)
+
+
+def test_dag_config_with_conditional_units(F, planner):
+    """The CD recipe with App-3-like conditional units ("super resolution | pass")."""
+    prob, d = W.dag_config(R=4096, p_cond=0.2)
+    assert d.unit_cond is not None and d.unit_cond.sum() > 0
+    g, c = run_dag(F, planner, prob, d)
+    o = oracle.plan_dag(prob, d)
+    assert_dag_equal(g, o, c)
+    assert (o["status"] == 0).mean() > 0.3

@@ -82,6 +82,8 @@ def brute_dag(prob, dag, r):
     base = int(prob.comp_off[f])
     units = dag.units(f)
     m = len(units)
+    cu = [False] * m if dag.unit_cond is None else \
+        [bool(dag.unit_cond[int(dag.unit_off[f]) + u]) for u in range(m)]  # R48 conditional units
     lat = lambda c, p: int(prob.lat_us[base + c, p])  # noqa: E731
     mem = lambda c: int(prob.mem_mib[base + c])  # noqa: E731
     xf = lambda c: int(prob.xfer_us[base + c])  # noqa: E731
@@ -96,20 +98,29 @@ def brute_dag(prob, dag, r):
         for cuts in cuts_list:
             bounds = [0] + [c + 1 for c in cuts] + [m]
             stages = [units[bounds[i]:bounds[i + 1]] for i in range(k)]
+            conds = [cu[bounds[i]:bounds[i + 1]] for i in range(k)]
             opts = []
-            for st in stages:
+            for st, cs in zip(stages, conds):
                 o = [("one", (p,)) for p in range(P)]
-                if len(st) == 1 and len(st[0]) >= 2:
+                if len(st) == 1 and len(st[0]) >= 2 and not cs[0]:
                     o += [("split", ps) for ps in itertools.product(range(P), repeat=len(st[0]))]
                 opts.append(o)
-            xfer = sum(sum(xf(e - 1) for (_, e) in units[c]) for c in cuts)
+
+            def cut_cost(u):  # R42; R48: the output of the alternative that ran (worst case)
+                xs = [xf(e - 1) if e > a else (xf(units[u][0][0] - 1) if units[u][0][0] > 0 else 0)
+                      for (a, e) in units[u]]
+                return max(xs) if cu[u] else sum(xs)
+            xfer = sum(cut_cost(c) for c in cuts)
             for choice in itertools.product(*opts):
                 t, used, ok = [], [0] * P, True
-                for st, (kind, ps) in zip(stages, choice):
+                for st, cs, (kind, ps) in zip(stages, conds, choice):
                     comps = [c for u in st for (a, e) in u for c in range(a, e)]
                     if kind == "one":
                         p = ps[0]
-                        t.append(sum(lat(c, p) for c in comps))
+                        # a unit's time: its components in sequence, or its slowest alternative
+                        t.append(sum(max(sum(lat(c, p) for c in range(a, e)) for (a, e) in u) if cnd
+                                     else sum(lat(c, p) for (a, e) in u for c in range(a, e))
+                                     for u, cnd in zip(st, cs)))
                         ok &= sum(mem(c) for c in comps) <= int(prob.cap_mib[p])
                         used[p] += 1
                     else:
@@ -137,8 +148,9 @@ def brute_dag(prob, dag, r):
     return best, idx, nfeas, ksum
 
 
-def random_dag(seed, K=3, nb_max=3):
+def random_dag(seed, K=3, nb_max=3, p_cond=0.0):
     rng = W.SplitMix64(seed)
+    c_rng = rng.sub(5)
     shapes, funcs = [], []
     for _ in range(3):
         m = int(rng.integers(1, 4, 1)[0])
@@ -148,6 +160,8 @@ def random_dag(seed, K=3, nb_max=3):
                 units.append([int(x) for x in rng.integers(1, 2, int(rng.integers(2, nb_max, 1)[0]))])
             else:
                 units.append([1])
+            if p_cond and float(c_rng.uniform(1)[0]) < p_cond:  # R48: alternatives, maybe a "pass"
+                units[-1] = W.Cond([int(c_rng.integers(1, 2, 1)[0]), int(c_rng.integers(0, 1, 1)[0])])
         n = sum(sum(u) for u in units)
         shapes.append(units)
         funcs.append(dict(lat=rng.integers(1, 60, n * 5).reshape(n, 5).tolist(),
@@ -159,9 +173,12 @@ def random_dag(seed, K=3, nb_max=3):
     return problem(funcs, nodes, reqs, k_max=K), dag_of(shapes)
 
 
-@pytest.mark.parametrize("seed", range(2000, 2030))
+@pytest.mark.parametrize("seed", range(2000, 2040))
 def test_dag_oracle_matches_independent_brute_force(seed):
-    prob, d = random_dag(seed, K=2 if seed % 3 == 0 else 3, nb_max=4 if seed % 3 == 0 else 2)
+    prob, d = random_dag(seed, K=2 if seed % 3 == 0 else 3, nb_max=4 if seed % 3 == 0 else 2,
+                         p_cond=0.4 if seed >= 2030 else 0.0)
+    if seed >= 2030:
+        assert d.unit_cond is not None
     o = oracle.plan_dag(prob, d, threads=2)
     for r in range(prob.R):
         best, scored, nfeas, ksum = brute_dag(prob, d, r)
@@ -211,3 +228,39 @@ def test_dag_table_validation():
     p2, d2 = W.dag_config(R=8, F=4, branches=(4, 4), p_block=1.0)
     with pytest.raises(ValueError):
         oracle.plan_dag(p2, d2, k_max=4)
+
+
+# ---- R48 conditional units (App 3, Table 4) --------------------------------------
+def app3_like(budget, cap=100, k_max=2, branch_y=1):
+    """Units [D], Cond[X | Y] (Y empty when branch_y = 0: "pass"), [E] on one profile:
+    lat D=10, X=20, Y=15, E=30; mem 10 each; xfer D=1, X=2, Y=3."""
+    lat = [[10], [20]] + ([[15]] if branch_y else []) + [[30]]
+    xfer = [1, 2] + ([3] if branch_y else []) + [0]
+    f = dict(lat=lat, mem=[10] * len(lat), xfer=xfer)
+    prob = problem([f], [[[0] * 4]], [(0, 0, budget)], k_max=k_max, gpcs=[1], cap=[cap])
+    return prob, W.dag_table([[[1], W.Cond([1, branch_y]), [1]]])
+
+
+def test_conditional_unit_takes_the_slowest_alternative():
+    # one slice: 10 + max(20, 15) + 30 = 60 (a fork/join block on one slice would be 75)
+    o = oracle.plan_dag(*app3_like(1000))
+    assert o["status"][0] == 0 and o["key"][0] == pack_key(0, 1, 1, 0) and o["e2e_us"][0] == 60
+    # every alternative is hosted: memory 40 > cap 35 makes the one-stage plan infeasible
+    o = oracle.plan_dag(*app3_like(1000, cap=35))
+    # cut after the conditional unit: [D, X|Y] = 30 | [E] = 30 (CV 0), the cut moves the
+    # output of whichever alternative ran: max(2, 3) = 3 -> e2e 63
+    assert o["key"][0] == pack_key(0, 2, 2, 2) and o["e2e_us"][0] == 63 and o["cut_mask"][0] == 0b10
+    # budget 62: that plan misses the SLO; the cut after D (10 | 50, cvq 455, e2e 61) wins
+    o = oracle.plan_dag(*app3_like(62, cap=35))
+    assert o["key"][0] == pack_key(455, 2, 2, 1) and o["e2e_us"][0] == 61
+
+
+def test_conditional_unit_is_never_split_and_pass_moves_the_previous_output():
+    # k_max 3: the mask with the conditional unit alone in a stage has 1 option (P = 1),
+    # not P + P^2 = 2 as a fork/join block would: 1 + 2 + 1 candidates
+    o = oracle.plan_dag(*app3_like(1000, k_max=3))
+    assert o["checks"][0][0] == 4 and (o["split_mask"] == 0).all()
+    # "pass" (empty alternative): one slice = 10 + max(20, 0) + 30; a cut after the unit
+    # moves max(X's output 2, D's output passed through 1) = 2
+    o = oracle.plan_dag(*app3_like(1000, cap=25, branch_y=0))
+    assert o["e2e_us"][0] == 60 + 2 and o["cut_mask"][0] == 0b10
