@@ -466,7 +466,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   CK(launch_count_tasks(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, k_max, nf, skip_full,
                         c->prefix.as<uint64_t>(), c->block_sums.as<uint64_t>(), init ? d_keys : nullptr,
                         init ? reinterpret_cast<unsigned long long*>(d_checks) : nullptr,
-                        c->work_ctr.as<unsigned long long>(), st),
+                        c->work_ctr.as<unsigned long long>(), k_first, k_last, st),
      "count/scan kernels");
   nvtxRangePop();
   // dynamic shared memory: the table image (every KS) + the per-thread variant windows

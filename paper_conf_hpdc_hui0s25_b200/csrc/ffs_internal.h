@@ -79,12 +79,15 @@ struct SearchArgs {
   const uint4* list;            // {request, maskA, maskB (0 = none), 0}
   uint32_t list_cap;
 };
-// work_ctr layout: [0..kMaxK] per-KS task-chunk grab counters; [kCtrScored + KS]
-// candidates the segment's kernel scored (every candidate whose own score it computed);
-// [kCtrListGrab + KS] record-chunk grab counters, [kCtrListCount + KS] live records
-// written by k_live and [kCtrLiveGrab + KS] k_live's own task-chunk grab counters (bounded
-// mode)
-constexpr int kCtrScored = 16, kCtrListGrab = 24, kCtrListCount = 32, kCtrLiveGrab = 40, kCtrWords = 48;
+// work_ctr layout: blocks of kCtrBlock words indexed by KS: [KS] task-chunk grab
+// counters; [kCtrScored + KS] candidates the segment's kernel scored (every candidate whose
+// own score it computed); [kCtrListGrab + KS] record-chunk grab counters, [kCtrListCount +
+// KS] live records written by k_live and [kCtrLiveGrab + KS] k_live's own task-chunk grab
+// counters (bounded mode).  A search call zeroes the slots of the segments it runs (all of
+// them when k_first = 1), so a caller running the segments range by range (candidate
+// shards) still reads every segment's counters after the last range.
+constexpr int kCtrBlock = 12, kCtrScored = 12, kCtrListGrab = 24, kCtrListCount = 36, kCtrLiveGrab = 48,
+              kCtrWords = 60;
 
 // Group tables of the bounded mode: per function f and availability
 // pattern a (bit p = the node has >= 1 free slice of profile p), with W(i, j) = the fastest
@@ -145,7 +148,8 @@ constexpr int kLiveMinPiece = 8;
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
-                               unsigned long long* checks, unsigned long long* work_ctr, cudaStream_t st);
+                               unsigned long long* checks, unsigned long long* work_ctr, uint32_t k_first,
+                               uint32_t k_last, cudaStream_t st);
 cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st);
 cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,

@@ -40,9 +40,13 @@ __global__ void k_count_tasks(const ffs_request* __restrict__ req, const uint32_
                               ImageLayout lay, uint32_t n_nodes, uint32_t n_req, uint32_t K,
                               const uint64_t* __restrict__ node_free, uint32_t skip_full,
                               uint64_t* __restrict__ prefix, int64_t* __restrict__ keys,
-                              unsigned long long* __restrict__ checks, unsigned long long* __restrict__ work_ctr) {
+                              unsigned long long* __restrict__ checks, unsigned long long* __restrict__ work_ctr,
+                              uint32_t k_first, uint32_t k_last) {
   uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
-  if (r < (uint32_t)kCtrWords) work_ctr[r] = 0;  // chunk counters + scored-candidate counters
+  if (r < (uint32_t)kCtrWords) {  // the counters of the segments this call runs (all on k_first = 1)
+    const uint32_t ks = r % kCtrBlock;
+    if (k_first <= 1 || (ks >= k_first && ks <= k_last)) work_ctr[r] = 0;
+  }
   if (r > n_req) return;
   uint32_t n = 0;
   if (r < n_req) {
@@ -139,10 +143,12 @@ __global__ void __launch_bounds__(kScanT) k_scan_apply(uint64_t* __restrict__ pr
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
-                               unsigned long long* checks, unsigned long long* work_ctr, cudaStream_t st) {
+                               unsigned long long* checks, unsigned long long* work_ctr, uint32_t k_first,
+                               uint32_t k_last, cudaStream_t st) {
   const uint64_t len = (uint64_t)n_req + 1;
   k_count_tasks<<<(unsigned)((len + 255) / 256), 256, 0, st>>>(req, image, lay, n_nodes, n_req, k_max, node_free,
-                                                                skip_full ? 1u : 0u, prefix, keys, checks, work_ctr);
+                                                                skip_full ? 1u : 0u, prefix, keys, checks, work_ctr,
+                                                                k_first, k_last);
   const uint32_t nb = (uint32_t)((len + kScanChunk - 1) / kScanChunk);
   dim3 g(nb, k_max);
   k_scan_reduce<<<g, kScanT, 0, st>>>(prefix, len, block_sums, nb);
@@ -861,9 +867,11 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
       r[9 * nb] = fr > 0 ? p0 : kInf2;
       r[10 * nb] = h2mul(h2mul(p0, p0), nal2);
     }
+    // each lane walks its own live stage-0 profiles: a warp runs max(popcount) iterations,
+    // not the union of its lanes' sets (records of the bounded list mode differ per lane)
 #pragma unroll 1
-    for (int d0 = 0; d0 < kP; ++d0) {
-      if (!((live >> d0) & 1u)) continue;
+    for (uint32_t todo = live; todo; todo &= todo - 1) {
+      const int d0 = __ffs(todo) - 1;
       const h2 S1 = slot[(d0 * 11 + 9) * nb];
       c.n_scored += haveB ? 250 : 125;  // 125 candidates per mask of this d0, each y_p computed
       WinH W[kP];
