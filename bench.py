@@ -147,7 +147,7 @@ def run_reference(args, prob):
     v = cands / tot
     line = {"metric": "candidates_scored_per_s", "value": v, "unit": "candidates/s", "impl": "reference",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / len(times),
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32/u64",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "exact u64/u128 integers (oracle)",
             "data": "synthetic", "plans_per_s": plans / tot,
             "config": {"workload": prob.meta["workload"], "R": prob.R, "k_max": prob.k_max},
             "cpu_baseline": {"value": v, "unit": "candidates/s", "cores": cores, "kind": "oracle",
