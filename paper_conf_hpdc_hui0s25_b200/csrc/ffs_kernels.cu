@@ -792,6 +792,25 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     wide[h] = bl >= 0.f && c.tmin * sig[h] < 0.125f;  // f16 underflow could matter: exact path
     slack[h] = bl >= 0.f ? M * sig[h] * (1.f + 1.f / 128.f) : -INF;
   }
+  // the scaled stage times with memory and the throughput floor (R38) folded: +INF where
+  // the stage does not fit the profile; a function without a floor (the common case) skips
+  // the floor compare (uniform per request)
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t cap = c.sm[c.o_cap + x];
+    if (c.thr_u == 0xffffffffu) {
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 4; ++s) f[h][s][x] = ms[h][s] <= cap ? f[h][s][x] * sig[h] : INF;
+    } else {
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 4; ++s)
+          f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * sig[h] : INF;
+    }
+  }
   // the packed stage tables and the per-half minima the stage-0 bound needs
   h2 P0[kP], P1[kP], P2[kP], P3[kP];
   float v3m[2] = {INF, INF};  // fastest admissible last stage per half (>= 1 free slice)
@@ -799,13 +818,11 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
 #pragma unroll
   for (int x = 0; x < kP; ++x) {
     const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
-    const uint32_t cap = c.sm[c.o_cap + x];
     float vm[2][4];
 #pragma unroll
     for (int h = 0; h < 2; ++h)
 #pragma unroll
-      for (int s = 0; s < 4; ++s)  // memory and the throughput floor (R38) folded
-        vm[h][s] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * sig[h] : INF;
+      for (int s = 0; s < 4; ++s) vm[h][s] = f[h][s][x];
     P0[x] = h2pack(vm[0][0], vm[1][0]);
     P1[x] = h2pack(vm[0][1], vm[1][1]);
     P2[x] = h2pack(vm[0][2], vm[1][2]);
