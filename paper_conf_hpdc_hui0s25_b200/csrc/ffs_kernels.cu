@@ -29,6 +29,15 @@ __device__ __forceinline__ float plf(const uint32_t* w, uint32_t o) { return __u
 __device__ __forceinline__ uint32_t pl_diff(const uint32_t* w, uint32_t ob, uint32_t oa) {
   return __float2uint_rn(plf(w, ob) - plf(w, oa));
 }
+__device__ __forceinline__ uint64_t warp_min_u64(uint64_t x) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) {
+    const uint64_t y = __shfl_xor_sync(0xffffffffu, x, o);
+    x = y < x ? y : x;
+  }
+  return x;
+}
+
 __device__ __forceinline__ uint32_t binom(const uint32_t* img, const ImageLayout& L, int c, int i) {
   return img[L.o_binom + c * 8 + i];  // C(c, i), 0 when c < i
 }
@@ -546,7 +555,8 @@ __device__ __forceinline__ void pair_rescan(SearchState<KS>& c, const Geo<KS>& G
 // last stage (blim - v2min - S2, integers < 2^25).
 template <bool VERIFY>
 __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint32_t maskB, bool haveB,
-                                         unsigned long long* misses, bool exh, uint64_t shiftB) {
+                                         unsigned long long* misses, bool exh, uint64_t shiftB,
+                                         uint32_t* defer = nullptr) {
   const float INF = __int_as_float(0x7f800000);
   Geo<3> G[2];
   geo<3>(c, maskA, G[0]);
@@ -642,6 +652,11 @@ __device__ __forceinline__ void ks3_pair(SearchState<3>& c, uint32_t maskA, uint
     pendB |= ((accB >> 31) ^ 1u) << d0;
   }
   constexpr uint32_t kAllB = (1u << kP) - 1;
+  if (!VERIFY && defer) {  // the caller rescans the flagged blocks warp-cooperatively
+    defer[0] = pendA;
+    defer[1] = haveB ? pendB : 0u;
+    return;
+  }
   pair_rescan<3, VERIFY>(c, G[0], pendA, VERIFY ? kAllB : pendA, 0, misses);
   if (haveB) pair_rescan<3, VERIFY>(c, G[1], pendB, VERIFY ? kAllB : pendB, shiftB, misses);
 }
@@ -738,7 +753,8 @@ __device__ __forceinline__ void ks4_cuts(uint32_t m, int& j1, int& j2, int& j3) 
 
 template <bool VERIFY>
 __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, uint32_t maskB, bool haveB, h2* rows,
-                                           unsigned long long* misses, uint32_t zero, bool exh, uint64_t shiftB) {
+                                           unsigned long long* misses, uint32_t zero, bool exh, uint64_t shiftB,
+                                           uint32_t* defer = nullptr) {
   const float INF = __int_as_float(0x7f800000);
   constexpr int nb = search_block(4);  // slot stride: the CTA size, fixed at compile time
   h2* slot = rows + threadIdx.x;
@@ -942,6 +958,11 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
   if (wide[0]) pendA = kAll;  // dynamic range too wide for f16: every block exactly
   if (wide[1]) pendB = kAll;
+  if (!VERIFY && defer) {  // the caller rescans the flagged blocks warp-cooperatively
+    defer[0] = pendA;
+    defer[1] = haveB ? pendB : 0u;
+    return;
+  }
   if (VERIFY || pendA) {
     Geo4 G;
     geo4(c, maskA, G);
@@ -1051,6 +1072,94 @@ __device__ __forceinline__ uint32_t find_request(const uint64_t* __restrict__ pr
   return lo;
 }
 
+// Exact key of one candidate (as exact_eval): request state broadcast from the lane that
+// owns the block, cut mask, profile digits; FFS_KEY_NONE when infeasible.
+template <int KS>
+__device__ __forceinline__ int64_t exact_key(const SearchState<KS>& c, uint32_t row0, uint32_t n, uint32_t B,
+                                             uint32_t thr_u, uint64_t freeb, uint32_t mask, uint64_t idx,
+                                             const int (&prof)[KS]) {
+  uint32_t bnd[KS + 1];
+  bnd[0] = 0;
+  uint32_t m = mask, X = 0;
+#pragma unroll
+  for (int i = 1; i < KS; ++i) {
+    const uint32_t j = __ffs(m) - 1;
+    m &= m - 1;
+    bnd[i] = j + 1;
+    X += c.sm[c.o_xf + row0 + j];
+  }
+  bnd[KS] = n;
+  uint64_t St = 0, Sq = 0;
+  uint32_t used = 0, g = 0;
+  bool ok = true;
+#pragma unroll
+  for (int i = 0; i < KS; ++i) {
+    const int pr = prof[i];
+    const uint32_t a = (row0 + bnd[i]) * kRowW, b = (row0 + bnd[i + 1]) * kRowW;
+    const uint32_t t = pl_diff(c.sm, c.o_pl + b + pr, c.o_pl + a + pr);
+    ok &= c.sm[c.o_pm + row0 + bnd[i + 1]] - c.sm[c.o_pm + row0 + bnd[i]] <= c.sm[c.o_cap + pr];
+    ok &= t <= thr_u;  // R38 throughput floor
+    St += t;
+    Sq += (uint64_t)t * t;
+    used += 1u << (4 * pr);
+    g += c.sm[c.o_gpcs + pr];
+  }
+#pragma unroll
+  for (int pp = 0; pp < kP; ++pp) ok &= ((used >> (4 * pp)) & 15u) <= ((freeb >> (8 * pp)) & 255u);
+  ok &= St + X <= (uint64_t)B;
+  if (!ok) return (int64_t)kKeyNone;
+  const uint64_t D = St * St, N = (uint64_t)KS * Sq - D;
+  const uint64_t cvq = (N << 10) / D;  // floor(1024 * CV^2), exact (R4)
+  return (int64_t)((cvq << 50) | ((uint64_t)(KS - 1) << 47) | ((uint64_t)g << 41) | idx);
+}
+
+// Warp-cooperative exact rescan of the flagged blocks (KS = 4: block = stage-0/1 profiles
+// (d0, d1); KS = 3: block = d0), each a block of 25 candidates (the last two stages' q, p):
+// the block's owner lane broadcasts its request state, 25 lanes evaluate one candidate
+// each, the warp minimum goes back to the owner.  In the bounded list mode the flags are
+// frequent and sparse across lanes -- rescanned lane by lane they ran at ~2 active threads
+// per instruction.  All 32 lanes must call it.
+template <int KS>
+__device__ __forceinline__ void coop_rescan(SearchState<KS>& c, uint32_t mask, uint32_t pend, uint64_t idx0) {
+  const uint32_t lane = threadIdx.x & 31;
+  for (;;) {
+    const uint32_t who = __ballot_sync(0xffffffffu, pend != 0u);
+    if (!who) break;
+    const int L = __ffs(who) - 1;
+    const int b = __shfl_sync(0xffffffffu, __ffs(pend) - 1, L);
+    if ((int)lane == L) pend &= pend - 1;
+    const uint32_t row0 = __shfl_sync(0xffffffffu, c.row0, L), n = __shfl_sync(0xffffffffu, c.n, L);
+    const uint32_t B = __shfl_sync(0xffffffffu, c.B, L), thr = __shfl_sync(0xffffffffu, c.thr_u, L);
+    const uint32_t mk = __shfl_sync(0xffffffffu, mask, L);
+    const uint64_t freeb = __shfl_sync(0xffffffffu, c.freeb, L);
+    const uint64_t i0 = __shfl_sync(0xffffffffu, idx0, L);
+    int64_t key = (int64_t)kKeyNone;
+    if (lane < (uint32_t)(kP * kP)) {
+      const int q = (int)lane / kP, p = (int)lane - kP * q;
+      int prof[KS];
+      uint64_t seq;
+      if constexpr (KS == 4) {
+        prof[0] = b / kP;
+        prof[1] = b - kP * (b / kP);
+        prof[2] = q;
+        prof[3] = p;
+        seq = (uint64_t)b * (kP * kP) + lane;
+      } else {
+        prof[0] = b;
+        prof[1] = q;
+        prof[2] = p;
+        seq = (uint64_t)b * (kP * kP) + lane;
+      }
+      key = exact_key<KS>(c, row0, n, B, thr, freeb, mk, i0 + seq, prof);
+    }
+    const int64_t kmin = (int64_t)warp_min_u64((uint64_t)key);
+    if ((int)lane == L && kmin < c.best) {
+      c.best = kmin;
+      set_threshold(c);
+    }
+  }
+}
+
 // colex rank of a cut mask among the (KS-1)-subsets of the cut positions: sum C(j_i, i)
 template <int KS>
 __device__ __forceinline__ uint64_t colex_rank(const uint32_t* img, const ImageLayout& L, uint32_t mask) {
@@ -1142,6 +1251,8 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     // ---- bounded mode: the live (request, mask pair) records of k_live ----------------
     // A warp takes 32 consecutive records (one per lane) at a time; every record carries
     // its request, so a lane loads the request's state per record.
+    // The loop stays warp-converged (a lane without a record idles) so the flagged blocks
+    // of all lanes are rescanned cooperatively (coop_rescan).
     unsigned long long* lctr = A.work_ctr + kCtrListGrab + KS;
     for (;;) {
       unsigned long long jg = 0;
@@ -1149,27 +1260,37 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
       jg = __shfl_sync(0xffffffffu, jg, 0);
       if (jg * 32 >= n_list) break;
       const uint64_t i = jg * 32 + lane;
-      if (i >= n_list) continue;
-      const uint4 rec = A.list[i];
-      r = rec.x;
-      const uint32_t maskA = rec.y, maskB = rec.z;
-      const bool haveB = maskB != 0u;
-      const uint64_t rkA = colex_rank<KS>(tbl, A.lay, maskA);
-      const uint64_t shiftB = haveB ? (colex_rank<KS>(tbl, A.lay, maskB) - rkA) * PK : 0ull;
-      load_request(rkA);
-      if constexpr (KS == 4) {
-        ks4_pair_h<false>(c, maskA, haveB ? maskB : maskA, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
-                          false, shiftB);
-      } else if constexpr (KS == 3) {
-        ks3_pair<false>(c, maskA, haveB ? maskB : maskA, haveB, A.misses, false, shiftB);
-      } else if constexpr (KS == 2) {
-        process_mask<KS, false>(c, maskA, rows, A.misses);
-        if (haveB) {
-          c.idx_base += shiftB;
-          process_mask<KS, false>(c, maskB, rows, A.misses);
+      const bool has = i < n_list;
+      uint32_t maskA = 0, maskB = 0, pend[2] = {0u, 0u};
+      uint64_t shiftB = 0;
+      if (has) {
+        const uint4 rec = A.list[i];
+        r = rec.x;
+        maskA = rec.y;
+        maskB = rec.z;
+        const bool haveB = maskB != 0u;
+        const uint64_t rkA = colex_rank<KS>(tbl, A.lay, maskA);
+        shiftB = haveB ? (colex_rank<KS>(tbl, A.lay, maskB) - rkA) * PK : 0ull;
+        load_request(rkA);
+        if constexpr (KS == 4) {
+          ks4_pair_h<false>(c, maskA, haveB ? maskB : maskA, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
+                            false, shiftB, pend);
+        } else if constexpr (KS == 3) {
+          ks3_pair<false>(c, maskA, haveB ? maskB : maskA, haveB, A.misses, false, shiftB, pend);
+        } else if constexpr (KS == 2) {
+          process_mask<KS, false>(c, maskA, rows, A.misses);
+          if (haveB) {
+            c.idx_base += shiftB;
+            process_mask<KS, false>(c, maskB, rows, A.misses);
+          }
         }
       }
-      flush(0);
+      if constexpr (KS == 3 || KS == 4) {
+        __syncwarp();
+        coop_rescan<KS>(c, maskA, pend[0], c.idx_base);
+        coop_rescan<KS>(c, maskB, pend[1], c.idx_base + shiftB);
+      }
+      if (has) flush(0);
     }
   } else {
     // ---- task ranges (exhaustive and verify modes; bounded mode's fallback) -------------
@@ -1199,10 +1320,11 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
       const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
       if (chunk >= NC) break;
       const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
-      if (t0 >= t1) continue;
-      uint64_t task = t0;
-      r = find_request(pre, A.n_req, task);
-      uint64_t m = task - pre[r], cnt = pre[r + 1] - pre[r], done = 0;
+      // the lanes walk their pieces in lockstep (pieces differ by at most one task), so the
+      // flagged blocks of KS = 3/4 pairs are rescanned warp-cooperatively (coop_rescan);
+      // verify mode rescans every block per lane
+      bool active = t0 < t1;
+      uint64_t task = t0, m = 0, cnt = 0, done = 0;
       uint32_t mask = 0;
       // colex unrank of rank0 among the (KS-1)-subsets of the n-1 cut positions.  Rank 0
       // (a request entered at its first task) is the lowest KS-1 bits: a shortcut worth it
@@ -1223,45 +1345,63 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
         }
         mask = mk;
       };
-      load_request(m);
-      unrank(m);
-      while (true) {
-        uint32_t step = 1;
-        if constexpr (KS == 3 || KS == 4) {
-          // two consecutive masks of the same request per iteration (ks3_pair / ks4_pair_h)
-          const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
-          const uint32_t maskB = haveB ? gosper_next(mask) : mask;
-          if constexpr (KS == 4)
-            ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
-                               A.exhaustive != 0, PK);
-          else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0, PK);
-          if (haveB) {
-            step = 2;
-            mask = maskB;
+      if (active) {
+        r = find_request(pre, A.n_req, task);
+        m = task - pre[r];
+        cnt = pre[r + 1] - pre[r];
+        load_request(m);
+        unrank(m);
+      }
+      while (__any_sync(0xffffffffu, active)) {
+        uint32_t step = 1, pend[2] = {0u, 0u}, mA = 0, mB = 0;
+        const uint64_t i0 = c.idx_base;
+        if (active) {
+          if constexpr (KS == 3 || KS == 4) {
+            // two consecutive masks of the same request per iteration (ks3_pair / ks4_pair_h)
+            const bool haveB = (m + 1 < cnt) && (task + 1 < t1);
+            const uint32_t maskB = haveB ? gosper_next(mask) : mask;
+            if constexpr (KS == 4)
+              ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
+                                 A.exhaustive != 0, PK, VERIFY ? nullptr : pend);
+            else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0, PK, VERIFY ? nullptr : pend);
+            mA = mask;
+            mB = maskB;
+            if (haveB) step = 2;
+          } else {
+            process_mask<KS, VERIFY>(c, mask, rows, A.misses);
           }
-        } else {
-          process_mask<KS, VERIFY>(c, mask, rows, A.misses);
         }
-        done += step;
-        task += step;
-        if (task >= t1) break;
-        m += step;
-        if (m == cnt) {
-          flush(done);
-          done = 0;
-          // tasks are consecutive: the next one belongs to the next request with tasks
-          // (requests without tasks of this KS have pre[r + 1] == pre[r]); no binary search
-          do ++r; while (pre[r + 1] <= task);
-          m = 0;
-          cnt = pre[r + 1] - pre[r];
-          load_request(0);
-          unrank(0);
-        } else {
-          mask = gosper_next(mask);
-          c.idx_base += step * PK;
+        if constexpr (!VERIFY && (KS == 3 || KS == 4)) {
+          __syncwarp();
+          coop_rescan<KS>(c, mA, pend[0], i0);  // before the lane moves on to another request
+          coop_rescan<KS>(c, mB, pend[1], i0 + PK);
+        }
+        if (active) {
+          if (step == 2) mask = mB;
+          done += step;
+          task += step;
+          if (task >= t1) {
+            flush(done);
+            active = false;
+          } else {
+            m += step;
+            if (m == cnt) {
+              flush(done);
+              done = 0;
+              // tasks are consecutive: the next one belongs to the next request with tasks
+              // (requests without tasks of this KS have pre[r + 1] == pre[r]); no binary search
+              do ++r; while (pre[r + 1] <= task);
+              m = 0;
+              cnt = pre[r + 1] - pre[r];
+              load_request(0);
+              unrank(0);
+            } else {
+              mask = gosper_next(mask);
+              c.idx_base += step * PK;
+            }
+          }
         }
       }
-      flush(done);
     }  // grab loop
   }
   {  // measurement: candidates scored by this warp (ffs_search_scored)
@@ -2611,14 +2751,6 @@ cudaError_t scan_u64(uint64_t* a, uint64_t len, uint64_t* bsum, cudaStream_t st)
 // ====================================================================================
 // K10 (NEXT-4): time-sharing simulator, one warp per node
 // ====================================================================================
-__device__ __forceinline__ uint64_t warp_min_u64(uint64_t x) {
-#pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    const uint64_t y = __shfl_xor_sync(0xffffffffu, x, o);
-    x = y < x ? y : x;
-  }
-  return x;
-}
 
 // Warp-wide exact argmin of function f's candidates against free counts `freeb` (8 x u8)
 // and budget B (R44: the pipeline a new instance is built as): the masks walked in colex
