@@ -222,8 +222,11 @@ ffs_status ffs_plan_keys_range(ffs_ctx *ctx, const ffs_request *d_req, const uin
  * stage (R11).  When d_inst and d_evict_scores are non-null, an INFEASIBLE request gets
  * the time-share victim of A8: the instance with the smallest eviction score
  * (from ffs_evict_scores on the same snapshot) resident in the request's node on a slice
- * that holds the whole function and meets lat + load <= budget; -1 if none.
- * Asynchronous on `stream`.  k_max must equal the one given to ffs_plan_keys. */
+ * that holds the whole function and meets lat + load <= budget; -1 if none.  The victims
+ * cost O(n_inst + n_req): one pass folds the scores into per-(node, slice profile) minima
+ * (context scratch), each INFEASIBLE request reads at most 5 of them.
+ * Asynchronous on `stream`.  k_max must equal the one given to ffs_plan_keys.
+ * FFS_ERR_RANGE: n_inst > 2^20 (the scores' index field). */
 ffs_status ffs_plan_decode(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t *d_slo_us, const int64_t *d_keys,
                            uint32_t n_req, uint32_t k_max, const ffs_instance *d_inst,
                            const int64_t *d_evict_scores, uint32_t n_inst, ffs_plan *d_out, void *stream);

@@ -96,7 +96,7 @@ struct ffs_ctx {
   // search mode (ffs_set_search_mode)
   uint32_t search_mode = FFS_SEARCH_BOUNDED;
   // bounded mode: group tables (per function x availability pattern) and live-record lists
-  DevBuf gofs, grp, live_list;
+  DevBuf gofs, grp, live_list, d_vtab;
   bool grp_ok = false;
   uint32_t list_cap = 0;
   uint64_t list_cap_max = 1ull << 28;  // FFS_LIST_CAP (tests: force the task-range fallback)
@@ -178,7 +178,7 @@ void ffs_destroy(ffs_ctx* c) {
     for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand, &c->dag_sv,
                       &c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr,
-                      &c->gofs, &c->grp, &c->live_list})
+                      &c->gofs, &c->grp, &c->live_list, &c->d_vtab})
       b->release();
   }
   delete c;
@@ -567,6 +567,7 @@ ffs_status ffs_plan_decode(ffs_ctx* c, const ffs_request* d_req, const uint32_t*
   if (n_req == 0) return FFS_OK;
   if (!d_req || !d_slo || !d_keys || !d_out) return fail(c, FFS_ERR_ARG, "null device pointer");
   if ((d_inst == nullptr) != (d_scores == nullptr)) return fail(c, FFS_ERR_ARG, "d_inst and d_evict_scores must both be set");
+  if (d_inst && n_inst > (1u << 20)) return fail(c, FFS_ERR_RANGE, "n_inst %u > 2^20", n_inst);
   DeviceGuard g(c->device);
   DecodeArgs a{};
   a.image = c->image.as<uint32_t>();
@@ -585,7 +586,8 @@ ffs_status ffs_plan_decode(ffs_ctx* c, const ffs_request* d_req, const uint32_t*
   a.score = d_scores;
   a.n_inst = d_inst ? n_inst : 0;
   a.out = d_out;
-  CK(launch_decode(a, (cudaStream_t)stream), "decode kernel");
+  if (d_inst) CK(c->d_vtab.ensure((size_t)c->n_nodes * c->P * 8), "cudaMalloc(decode victim table)");
+  CK(launch_decode(a, c->d_vtab.as<unsigned long long>(), (cudaStream_t)stream), "decode kernel");
   return FFS_OK;
 }
 

@@ -131,6 +131,7 @@ struct DecodeArgs {
   const int64_t* score;
   uint32_t n_inst;
   ffs_plan* out;
+  const unsigned long long* vtab;  // [n_nodes][kP] minimum LRU score per (node, slice profile), ~0 empty
 };
 
 // launchers (ffs_kernels.cu)
@@ -154,7 +155,7 @@ cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, in
                           cudaStream_t st);
 cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,
                                  int* blocks_per_sm);
-cudaError_t launch_decode(const DecodeArgs& a, cudaStream_t st);
+cudaError_t launch_decode(const DecodeArgs& a, unsigned long long* vtab, cudaStream_t st);
 cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32_t* tick_off,
                          const uint64_t* now_us, uint32_t n_ticks, uint64_t now_single,
                          ffs_evict_params prm, int64_t* score, uint8_t* state, cudaStream_t st);

@@ -38,6 +38,10 @@ __device__ __forceinline__ uint64_t warp_min_u64(uint64_t x) {
   return x;
 }
 
+// profiles whose slice can host function f monolithically within budget B (defined with
+// the victim kernels, K4)
+__device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const ImageLayout& L, uint32_t f, uint32_t B);
+
 __device__ __forceinline__ uint32_t binom(const uint32_t* img, const ImageLayout& L, int c, int i) {
   return img[L.o_binom + c * 8 + i];  // C(c, i), 0 when c < i
 }
@@ -1733,19 +1737,20 @@ cudaError_t launch_live(int ks, const LiveArgs& a, int grid, cudaStream_t st) {
 // ====================================================================================
 // K2: decode + bind (A6) and time-share victim (A8)
 // ====================================================================================
-__device__ __forceinline__ bool victim_ok(const uint32_t* img, const ImageLayout& L, uint32_t f, uint32_t v,
-                                          uint32_t B, const ffs_instance& in, int64_t score,
-                                          const uint16_t* slice_node, const uint8_t* slice_prof,
-                                          uint32_t n_slices) {
-  if ((uint64_t)score == kKeyNone) return false;
-  if (in.slice < 0 || (uint32_t)in.slice >= n_slices || slice_node[in.slice] != v) return false;
-  const uint32_t p = slice_prof[in.slice];
-  const uint32_t* fd = img + L.o_fdesc + 4 * f;
-  if (fd[3] > img[L.o_cap + p]) return false;  // time-sharing instances are non-pipeline
-  const uint32_t row0 = fd[0], n = fd[1];
-  const uint64_t lat = pl_diff(img, L.o_pl + (row0 + n) * kRowW + p, L.o_pl + row0 * kRowW + p);
-  // execution + reload within the budget; the instance meets the floor (R38)
-  return lat + fd[2] <= B && lat <= img[L.o_thr + f];
+// per-(node, slice profile) minimum LRU score of one snapshot (A8 in ffs_plan_decode):
+// a flat grid over the instances, 64-bit atomicMin into the table (~0 = empty)
+__global__ void __launch_bounds__(256) k_vtab_snapshot(const ffs_instance* __restrict__ inst,
+                                                       const int64_t* __restrict__ score, uint32_t n,
+                                                       const uint16_t* __restrict__ slice_node,
+                                                       const uint8_t* __restrict__ slice_prof, uint32_t n_slices,
+                                                       unsigned long long* __restrict__ tab) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int64_t s = score[i];
+    if ((uint64_t)s == kKeyNone) continue;
+    const int32_t sl = inst[i].slice;
+    if (sl < 0 || (uint32_t)sl >= n_slices) continue;
+    atomicMin(tab + (uint32_t)slice_node[sl] * kP + slice_prof[sl], (unsigned long long)s);
+  }
 }
 
 __device__ __forceinline__ void plan_init(ffs_plan& pl) {
@@ -1824,15 +1829,16 @@ __global__ void k_decode(const __grid_constant__ DecodeArgs A) {
     if ((uint64_t)key == kKeyNone) {
       pl.status = FFS_PLAN_INFEASIBLE;
       if (A.inst) {
-        int64_t bs = (int64_t)kKeyNone;
-        for (uint32_t i = 0; i < A.n_inst; ++i) {
-          const int64_t s = A.score[i];
-          if (s < bs && victim_ok(img, L, q.func, q.node, A.slo[r], A.inst[i], s, A.slice_node, A.slice_prof,
-                                  A.n_slices)) {
-            bs = s;
-            pl.victim = (int32_t)i;
-          }
-        }
+        // A8: the least recently used evictable instance on the node whose slice can
+        // host the function monolithically within the budget: the minimum over the request's
+        // admissible profiles of the per-(node, profile) minima (k_vtab_snapshot; the score's
+        // low 20 bits are the instance index)
+        const uint32_t okp = victim_profiles(img, L, q.func, A.slo[r]);
+        unsigned long long bs = ~0ull;
+#pragma unroll
+        for (int p = 0; p < kP; ++p)
+          if ((okp >> p) & 1u) bs = min(bs, A.vtab[(uint64_t)q.node * kP + p]);
+        pl.victim = bs == ~0ull ? -1 : (int32_t)(bs & 0xFFFFFull);
       }
     } else {
       plan_from_key(img, L, q.func, A.k_max, key, pl);
@@ -1981,9 +1987,18 @@ cudaError_t launch_joint(int phase, const JointArgs& a, uint32_t n, cudaStream_t
   return cudaGetLastError();
 }
 
-cudaError_t launch_decode(const DecodeArgs& a, cudaStream_t st) {
+cudaError_t launch_decode(const DecodeArgs& a, unsigned long long* vtab, cudaStream_t st) {
   if (a.n_req == 0) return cudaSuccess;
-  k_decode<<<(a.n_req + 127) / 128, 128, 0, st>>>(a);
+  DecodeArgs b = a;
+  if (a.inst) {  // victims: the snapshot's per-(node, profile) minima first (O(n_inst + n_req))
+    cudaError_t e = cudaMemsetAsync(vtab, 0xFF, (size_t)a.n_nodes * kP * 8, st);
+    if (e != cudaSuccess) return e;
+    if (a.n_inst)
+      k_vtab_snapshot<<<(a.n_inst + 255) / 256, 256, 0, st>>>(a.inst, a.score, a.n_inst, a.slice_node, a.slice_prof,
+                                                             a.n_slices, vtab);
+    b.vtab = vtab;
+  }
+  k_decode<<<(a.n_req + 127) / 128, 128, 0, st>>>(b);
   return cudaGetLastError();
 }
 
@@ -2022,8 +2037,6 @@ constexpr int kEvT = FFS_EVT, kEvU = FFS_EVU;
 // (node, slice profile) minima in shared memory (64-bit atomicMin) and writes that row of
 // the victim table once -- the victim pass then reads <= 5 cells per load instead of
 // re-reading the tick's scores and records.  ~0 marks an empty cell.
-// (defined with the victim kernels below)
-__device__ __forceinline__ uint32_t victim_profiles(const uint32_t* img, const ImageLayout& L, uint32_t f, uint32_t B);
 
 // PICK (loads grouped by tick, d_load_off): the tick's loads take their victims from the
 // shared-memory minima right away -- no table in device memory, one launch for the step.

@@ -451,6 +451,32 @@ def test_decode_victims_single_snapshot(F, planner):
     np.testing.assert_array_equal(plans["victim"], v_o)
 
 
+def test_decode_victims_many_instances(F, planner):
+    """Victims in ffs_plan_decode with 50,000 instances on the C3 cluster (the per-(node,
+    profile) minima path, O(n_inst + n_req)) against the oracle's direct LRU scan."""
+    prob = W.config3(R=4096)
+    planner.stage(prob)
+    rng = W.SplitMix64(808)
+    n = 50_000
+    inst = np.zeros(n, dtype=W.INST_DTYPE)
+    inst["func"] = rng.integers(0, prob.F - 1, n)
+    inst["slice"] = rng.integers(-1, len(prob.slices) - 1, n)
+    inst["flags"] = np.where(rng.uniform(n) < 0.1, W.INST_BUSY, 0)
+    inst["busy_us"] = rng.integers(0, 4_000_000, n)
+    now = 10**12
+    inst["last_used_us"] = now - rng.integers(0, 700_000_000, n).astype(np.uint64)
+    d_inst = torch.from_numpy(inst.view(np.uint8)).cuda()
+    score, _ = planner.evict_scores(d_inst, now, window_us=10_000_000)
+    req, slo = F.to_device(prob)
+    keys = planner.plan_keys(req, slo, prob.k_max)
+    plans = F.plans_to_numpy(planner.plan_decode(req, slo, keys, prob.k_max, d_inst, score))
+    o = oracle.plan(prob, checks=False)
+    ev = oracle.evict(inst, now, 30, 10_000_000)
+    v_o = oracle.victim(prob, o["status"], inst, ev)
+    np.testing.assert_array_equal(plans["victim"], v_o)
+    assert (v_o >= 0).sum() > 20
+
+
 # ---- NEXT-1: ranked first-fit (P:339-343) ----------------------------------------------
 def run_ranked(F, planner, prob, p_ref=4):
     planner.stage(prob)
