@@ -854,8 +854,10 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
     if (fr > 0) {
       v3m[0] = fminf(v3m[0], u0);
       v3m[1] = fminf(v3m[1], u1);
-      v1min = h2min(v1min, P1[x]);
-      v2min = h2min(v2min, P2[x]);
+      if (!exh) {  // only the stage-0 bound needs them
+        v1min = h2min(v1min, P1[x]);
+        v2min = h2min(v2min, P2[x]);
+      }
     }
   }
   // guarded SLO slack of the fastest admissible last stage (h2guard): S3 <= slack - v3min
@@ -866,15 +868,17 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   // in every live half the iteration can flag nothing: it is skipped.  This covers a
   // stage-0 profile with no free slice on the node (S1 = +INF) and stage-0 prefixes that
   // leave too little budget.
-  uint32_t live = 0;
+  uint32_t live = (1u << kP) - 1;  // exhaustive mode: every stage-0 iteration is scored
+  if (!exh) {  // (uniform: a kernel argument)
+    live = 0;
 #pragma unroll
-  for (int d0 = 0; d0 < kP; ++d0) {
-    const h2 S1 = ((c.freeb >> (8 * d0)) & 255u) ? P0[d0] : kInf2;
-    const uint32_t okb = isub(slk, h2add(h2add(S1, v1min), v2min), zero);
-    const bool on = (okb & 0x8000u) || (haveB && (okb & 0x80000000u));
-    live |= (on ? 1u : 0u) << d0;
+    for (int d0 = 0; d0 < kP; ++d0) {
+      const h2 S1 = ((c.freeb >> (8 * d0)) & 255u) ? P0[d0] : kInf2;
+      const uint32_t okb = isub(slk, h2add(h2add(S1, v1min), v2min), zero);
+      const bool on = (okb & 0x8000u) || (haveB && (okb & 0x80000000u));
+      live |= (on ? 1u : 0u) << d0;
+    }
   }
-  if (exh) live = (1u << kP) - 1;  // exhaustive mode: every stage-0 iteration is scored
   uint32_t pendA = 0, pendB = 0;
   // no live iteration (the common case in bounded mode): nothing else to set up
   if (VERIFY || live != 0) {
@@ -912,10 +916,10 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
       const h2 S1 = slot[(d0 * 11 + 9) * nb];
       c.n_scored += haveB ? 250 : 125;  // 125 candidates per mask of this d0, each y_p computed
       WinH W[kP];
+      const h2* shifted = slot + nb;  // the d0 profile's windows are read one slot later
 #pragma unroll
       for (int x = 0; x < kP; ++x) {
-        const int e = (x == d0);
-        const h2* r = slot + (x * 11 + e) * nb;
+        const h2* r = (x == d0 ? shifted : slot) + x * 11 * nb;  // a select + immediate offsets
         W[x].s1 = r[0];
         W[x].s2[0] = r[2 * nb];
         W[x].s2[1] = r[3 * nb];
