@@ -533,7 +533,6 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     la.list = c->live_list.as<uint4>();
     la.list_cap = c->list_cap;
     la.work_ctr = a.work_ctr;
-    la.warps_total = (uint32_t)c->sms * 64;
   }
   if (init) c->seg_mask = 0;
   for (uint32_t k = k_first; k <= kk; ++k) {

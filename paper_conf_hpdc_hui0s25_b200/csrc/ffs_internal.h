@@ -114,7 +114,6 @@ struct LiveArgs {
   uint4* list;
   uint32_t list_cap;
   unsigned long long* work_ctr;
-  uint32_t warps_total;         // warps per search launch (the task split must match k_plan_search)
 };
 
 struct DecodeArgs {
@@ -141,11 +140,10 @@ struct DecodeArgs {
 // 16: - / - / 3.04 / -, 32: 0.18 / 0.88 / 3.14 / 40.6, 64: - / - / - / 40.45.
 __host__ __device__ constexpr int kdyn(int ks) { return ks == 1 ? 1 : ks == 2 ? 32 : ks == 3 ? 16 : ks == 4 ? 64 : 32; }
 // minimum tasks per lane piece of the search's task ranges (a piece costs a request
-// lookup; a KS = 1/2 task is ~5 / ~100 instructions, a KS = 4 mask pair ~3000) and of k_live
+// lookup; a KS = 1/2 task is ~5 / ~100 instructions, a KS = 4 mask pair ~3000)
 // (measured on C5 slices of 1/1 .. 1/16 of the batch: shorter pieces leave more of the
 // per-piece lookups, longer ones more imbalance)
 __host__ __device__ constexpr int kMinPiece(int ks) { return ks == 1 ? 4 : ks == 2 ? 8 : ks == 3 ? 2 : 1; }
-constexpr int kLiveMinPiece = 8;
 cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, const ImageLayout& lay,
                                uint32_t n_nodes, uint32_t n_req, uint32_t k_max, const uint64_t* node_free,
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,

@@ -1303,6 +1303,11 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   } else {
     // ---- task ranges (exhaustive and verify modes; bounded mode's fallback) -------------
     const uint64_t T = pre[A.n_req];
+    // bounded mode whose live list overflowed: k_live partitioned the masks over the ranks
+    // by row, not by these chunks, so this rank covers the whole segment (redundant with
+    // the other ranks but complete; the MIN of the keys is idempotent)
+    const bool whole = A.list != nullptr;
+    const uint32_t world = whole ? 1u : A.world, rank = whole ? 0u : A.rank;
     // Work split: the segment's task list is cut into NC = world x (nthr/32) x kdyn(KS) chunks
     // of 32 equal contiguous pieces (one per lane).  Rank `rank` owns chunks
     // j * world + rank; its warps grab them dynamically (atomic counter, zeroed by the count
@@ -1314,9 +1319,9 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     const uint64_t nthr = (uint64_t)gridDim.x * blockDim.x;
     // at most warps x kdyn chunks per rank, pieces of at least kMinPiece(KS) tasks (short
     // segments -- a request shard's -- would otherwise pay a request lookup per task)
-    uint64_t NC = (nthr >> 5) * kdyn(KS) * A.world;
+    uint64_t NC = (nthr >> 5) * kdyn(KS) * world;
     const uint64_t want = T / (32ull * kMinPiece(KS));
-    if (want < NC) NC = max((uint64_t)A.world, (want + A.world - 1) / A.world * A.world);
+    if (want < NC) NC = max((uint64_t)world, (want + world - 1) / world * world);
     const uint64_t NT = NC * 32;
     const uint64_t Tq = T / NT, Tr = T % NT;  // piece u = [Tq u + Tr u / NT, ...): no overflow
     auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
@@ -1325,7 +1330,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
       unsigned long long jg = 0;
       if (lane == 0) jg = atomicAdd(ctr, 1ull);
       jg = __shfl_sync(0xffffffffu, jg, 0);
-      const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
+      const uint64_t chunk = (uint64_t)jg * world + rank;
       if (chunk >= NC) break;
       const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
       // the lanes walk their pieces in lockstep (pieces differ by at most one task), so the
@@ -1546,185 +1551,117 @@ cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, c
   return cudaGetLastError();
 }
 
-// colex rank of a (KS-1)-subset {j_1 < ... < j_{KS-1}} of the cut positions: sum C(j_i, i)
-__host__ __device__ __forceinline__ uint32_t c2(uint32_t x) { return x * (x - 1) / 2; }
-__host__ __device__ __forceinline__ uint32_t c3(uint32_t x) { return x * (x - 1) * (x - 2) / 6; }
+// K1b: live-mask compaction, one warp per request (warps grab 4 requests at a time).  A
+// mask (j1 < j2 < j3: cut positions) is kept iff its exact e2e lower bound
+//   LB = W(0,b1) + X(b1) + W(b1,b2) + X(b2) + ... + W(b_{KS-1}, n) <= B   (b = j + 1)
+// -- a mask with LB > B holds no feasible candidate, so dropping it is exact.  The warp
+// tests the request's blocks (fixed highest cut j3: R3[b3] + T3[b3], lanes over j3), then
+// the rows of every live block (fixed j2, j3: R2[b2] + Mt[b3][b2] + T3[b3], lanes over j2),
+// then the masks of every live row (H0[b1] + Mt[b2][b1] + row constant, lanes over j1) --
+// n <= 32, so each level is one warp instruction stream, with no per-lane walk and no
+// divergence between lanes.  Requests whose best key of the earlier segments has cvq = 0
+// and fewer stages are dropped whole (no KS-stage candidate can beat it, R1).  Live masks
+// of a row are paired in order into records {r, maskA, maskB (0 = single), 0}; one
+// warp-aggregated atomic per row reserves their slots.  Candidate shards (world > 1): rank
+// g keeps the rows whose (request, j3, j2) hash is g mod world -- a partition of the masks.
+__device__ __forceinline__ bool live_owned(uint32_t r, uint32_t j3, uint32_t j2, uint32_t rank, uint32_t world) {
+  if (world == 1) return true;
+  const uint32_t h = (r * 0x9E3779B1u) ^ ((j3 << 5 | j2) * 0x85EBCA6Bu);
+  return (h ^ (h >> 15)) % world == rank;
+}
 
-// K1b: live-mask compaction.  The segment's (request, cut mask) tasks are split exactly as
-// k_plan_search splits them (same chunks, same rank interleave); each lane walks its
-// piece in colex order and keeps the masks whose e2e lower bound
-//   LB = W(0,b1) + X(b1) + W(b1,b2) + X(b2) + ... + W(b_{KS-1}, n) <= B   (exact integers)
-// skipping a whole block of masks (fixed highest cut) or row (fixed two highest cuts) when
-// its best-case bound (R3 / R2 of the group tables) already exceeds the budget.  A mask
-// with LB > B holds no feasible candidate, so dropping it is exact.  Consecutive live masks
-// of one request are paired into one record {r, maskA, maskB, 0} (maskB = 0: single).
-// Lockstep: every lane takes one action per iteration (a block test, a row test, a mask
-// test, a request change or the end), so the warp stays converged at the emission point.
 template <int KS>
 __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A) {
   static_assert(KS >= 2 && KS <= 4, "k_live: KS = 2..4");
-  enum { kBlock = 0, kRow = 1, kMask = 2, kNext = 3, kEnd = 4 };
+  constexpr uint32_t kReqPerGrab = 4;
   const uint32_t* img = A.image;
   const ImageLayout& L = A.lay;
   const uint32_t lane = threadIdx.x & 31;
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
-  const uint64_t T = pre[A.n_req];
-  // chunks of 32 pieces, at most warps x kdyn per rank and no smaller than kLiveMinPiece
-  // tasks per piece: a piece costs a request lookup and an unrank, a task ~20
-  // instructions, so small segments (a request shard's) use fewer, longer pieces.  The
-  // count depends only on T, so every rank of a candidate-shard split agrees on it.
-  uint64_t NC = (uint64_t)A.warps_total * kdyn(KS) * A.world;
-  const uint64_t want = T / (32ull * kLiveMinPiece);
-  if (want < NC) NC = max((uint64_t)A.world, (want + A.world - 1) / A.world * A.world);
-  const uint64_t NT = NC * 32;
-  const uint64_t Tq = T / NT, Tr = T % NT;
-  auto piece = [&](uint64_t u) { return Tq * u + Tr * u / NT; };
   unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;
   unsigned long long* lcount = A.work_ctr + kCtrListCount + KS;
-
+  const uint32_t lt_mask = (1u << lane) - 1u;
+  uint32_t r = 0;
+  // pair the live masks of one row (bit j1 of `bal`, the row's other cuts in `hi`) and
+  // append them; every lane of the warp calls it
+  auto emit_row = [&](uint32_t bal, uint32_t hi) {
+    if (!bal) return;
+    const uint32_t np = (__popc(bal) + 1) >> 1;
+    uint32_t base = 0;
+    if (lane == 0) base = (uint32_t)atomicAdd(lcount, (unsigned long long)np);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    const uint32_t rk = __popc(bal & lt_mask);
+    if (((bal >> lane) & 1u) && !(rk & 1u)) {
+      const uint32_t above = lane == 31 ? 0u : bal & ~((2u << lane) - 1u);
+      const uint32_t mB = above ? ((1u << (__ffs(above) - 1)) | hi) : 0u;
+      const uint32_t slot = base + (rk >> 1);
+      if (slot < A.list_cap) A.list[slot] = make_uint4(r, (1u << lane) | hi, mB, 0u);
+    }
+  };
   for (;;) {
     unsigned long long jg = 0;
     if (lane == 0) jg = atomicAdd(ctr, 1ull);
     jg = __shfl_sync(0xffffffffu, jg, 0);
-    const uint64_t chunk = (uint64_t)jg * A.world + A.rank;
-    if (chunk >= NC) break;
-    const uint64_t t0 = piece(chunk * 32 + lane), t1 = piece(chunk * 32 + lane + 1);
-    bool active = t0 < t1;
-    uint64_t task = t0;
-    uint32_t r = 0, m = 0, cnt = 0, n = 0, N1 = 0, B = 0, j1 = 0, j2 = 0, j3 = 0, rowc = 0, pend = 0, recR = 0;
-    const uint32_t* gp = nullptr;
-    int need = kEnd;
-    bool jump_dead = false;
-    auto load = [&](uint32_t mm) {  // request r, rank mm within it
+    const uint64_t r0 = jg * kReqPerGrab;
+    if (r0 >= A.n_req) break;
+    const uint32_t r1 = (uint32_t)min(r0 + kReqPerGrab, (uint64_t)A.n_req);
+    for (r = (uint32_t)r0; r < r1; ++r) {
+      if (pre[r + 1] == pre[r]) continue;  // no tasks of this KS (short chain, full node, bad request)
+      const uint64_t bk = (uint64_t)A.keys[r];
+      if (bk != kKeyNone && (bk >> 50) == 0 && (int)((bk >> 47) & 7) + 1 < KS) continue;
       const ffs_request q = A.req[r];
-      n = img[L.o_fdesc + 4 * q.func + 1];
-      N1 = n + 1;
-      B = A.slo[r];
+      const uint32_t n = img[L.o_fdesc + 4 * q.func + 1], N1 = n + 1;
+      const uint32_t B = A.slo[r];
       const uint64_t fb = A.node_free[q.node];
       uint32_t av = 0;
 #pragma unroll
       for (int p = 0; p < kP; ++p) av |= (((fb >> (8 * p)) & 255u) != 0u ? 1u : 0u) << p;
-      gp = A.grp + A.gofs[q.func] + av * grp_stride(n);
-      cnt = (uint32_t)(pre[r + 1] - pre[r]);
-      m = mm;
-      // request-level CV test (set_threshold's none_can_win): a best key of the earlier
-      // segments with cvq = 0 and fewer than KS stages cannot be beaten by any KS-stage
-      // candidate (R1: cvq, then k) -- every 1-stage plan has CV = 0 -- so the request's
-      // remaining masks are all dead
-      const uint64_t bk = (uint64_t)A.keys[r];
-      const bool dead = bk != kKeyNone && (bk >> 50) == 0 && (int)((bk >> 47) & 7) + 1 < KS;
-      // colex unrank of mm
-      uint32_t x = n - 1;
-      if constexpr (KS == 4) {
-        while (c3(x) > mm) --x;
-        j3 = x;
-        mm -= c3(x);
-      }
-      if constexpr (KS >= 3) {
-        x = (KS == 4) ? j3 - 1 : n - 1;
-        while (c2(x) > mm) --x;
-        j2 = x;
-        mm -= c2(x);
-      }
-      j1 = mm;
-      need = KS == 4 ? kBlock : KS == 3 ? kRow : kMask;
-      pend = 0;
-      if (dead) jump_dead = true;
-    };
-    if (active) {
-      r = find_request(pre, A.n_req, task);
-      load((uint32_t)(task - pre[r]));
-    }
-    // move to rank mm (> m) of the current request; the caller sets the state for mm
-    auto jump = [&](uint32_t mm) {
-      task += mm - m;
-      m = mm;
-      if (task >= t1) need = kEnd;
-      else if (m == cnt) need = kNext;
-    };
-    if (jump_dead) {  // the first request of the piece is dead: skip to its end
-      jump_dead = false;
-      jump(cnt);
-    }
-    while (__any_sync(0xffffffffu, active)) {
-      uint32_t recA = 0, recB = 0;
-      bool has = false;
-      if (active) {
-        recR = r;
-        const uint32_t b1 = j1 + 1, b2 = j2 + 1, b3 = j3 + 1;
-        if (need == kEnd || need == kNext) {
-          if (pend) {  // the request's last live mask has no partner
-            has = true;
-            recA = pend;
-            pend = 0;
-          }
-          if (need == kEnd) {
-            active = false;
-          } else {
-            do ++r; while (pre[r + 1] <= task);
-            load(0);
-            if (jump_dead) {
-              jump_dead = false;
-              jump(cnt);
-            }
-          }
-        } else if (KS == 4 && need == kBlock) {
-          if ((uint64_t)gp[3 * N1 + b3] + gp[N1 + b3] > B) {  // R3[b3] + T3[b3]
-            jump(c3(j3 + 1));
-            if (need == kBlock) { j1 = 0; j2 = 1; j3 += 1; }
-          } else {
-            need = kRow;
-          }
-        } else if (KS >= 3 && need == kRow) {
-          // KS = 4: R2[b2] + Mt[b3][b2] + T3[b3];  KS = 3: R2[b2] + T3[b2]
-          rowc = KS == 4 ? gp[4 * N1 + b3 * N1 + b2] + gp[N1 + b3] : gp[N1 + b2];
-          if ((uint64_t)gp[2 * N1 + b2] + rowc > B) {
-            const uint32_t base = KS == 4 ? c3(j3) : 0u;
-            if (KS == 4 && j2 + 1 == j3) {  // last row of the block
-              jump(c3(j3 + 1));
-              if (need == kRow) { j1 = 0; j2 = 1; j3 += 1; need = kBlock; }
-            } else {
-              jump(base + c2(j2 + 1));
-              if (need == kRow) { j1 = 0; j2 += 1; }
-            }
-          } else {
-            need = kMask;
-          }
-        } else {  // kMask
-          uint64_t lb;
-          if constexpr (KS == 2) lb = (uint64_t)gp[b1] + gp[N1 + b1];  // H0 + T3
-          else lb = (uint64_t)gp[b1] + gp[4 * N1 + b2 * N1 + b1] + rowc;
-          if (lb <= B) {
-            const uint32_t mk = (1u << j1) | (KS >= 3 ? 1u << j2 : 0u) | (KS == 4 ? 1u << j3 : 0u);
-            if (pend) {
-              has = true;
-              recA = pend;
-              recB = mk;
-              pend = 0;
-            } else {
-              pend = mk;
-            }
-          }
-          jump(m + 1);
-          if (need == kMask) {  // colex successor
-            if (KS == 2 || j1 + 1 < j2) {
-              ++j1;
-            } else if (KS == 4 && j2 + 1 == j3) {
-              j1 = 0; j2 = 1; j3 += 1; need = kBlock;
-            } else {
-              j1 = 0; j2 += 1; need = kRow;
-            }
+      const uint32_t* gp = A.grp + A.gofs[q.func] + av * grp_stride(n);
+      const uint32_t* H0 = gp;
+      const uint32_t* T3 = gp + N1;
+      const uint32_t* R2 = gp + 2 * N1;
+      const uint32_t* R3 = gp + 3 * N1;
+      const uint32_t* Mt = gp + 4 * N1;
+      // mask test for row (j2, row constant rc): lanes over j1 < j2
+      auto row_masks = [&](uint32_t j2, uint32_t rc) {
+        const bool live = lane < j2 && (uint64_t)H0[lane + 1] + Mt[(j2 + 1) * N1 + lane + 1] + rc <= B;
+        return __ballot_sync(0xffffffffu, live);
+      };
+      if constexpr (KS == 2) {
+        const uint32_t j1 = lane;
+        const bool live = j1 + 2 <= n && live_owned(r, 0, j1, A.rank, A.world) &&
+                          (uint64_t)H0[j1 + 1] + T3[j1 + 1] <= B;
+        emit_row(__ballot_sync(0xffffffffu, live), 0u);
+      } else if constexpr (KS == 3) {
+        const uint32_t j2 = lane + 1;
+        const bool valid = j2 + 2 <= n && live_owned(r, 0, j2, A.rank, A.world);
+        const uint32_t rc = valid ? T3[j2 + 1] : 0u;
+        uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= B);
+        while (rows) {
+          const uint32_t b = __ffs(rows) - 1;
+          rows &= rows - 1;
+          const uint32_t jr = b + 1, rcb = __shfl_sync(0xffffffffu, rc, b);
+          emit_row(row_masks(jr, rcb), 1u << jr);
+        }
+      } else {
+        const uint32_t j3 = lane + 2;
+        const bool bvalid = j3 + 2 <= n;
+        uint32_t blocks = __ballot_sync(0xffffffffu, bvalid && (uint64_t)R3[j3 + 1] + T3[j3 + 1] <= B);
+        while (blocks) {
+          const uint32_t jb = __ffs(blocks) - 1 + 2;
+          blocks &= blocks - 1;
+          const uint32_t b3 = jb + 1, t3 = T3[b3];
+          const uint32_t j2 = lane + 1;
+          const bool valid = j2 < jb && live_owned(r, jb, j2, A.rank, A.world);
+          const uint32_t rc = valid ? Mt[b3 * N1 + j2 + 1] + t3 : 0u;
+          uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= B);
+          while (rows) {
+            const uint32_t b = __ffs(rows) - 1;
+            rows &= rows - 1;
+            const uint32_t jr = b + 1, rcb = __shfl_sync(0xffffffffu, rc, b);
+            emit_row(row_masks(jr, rcb), (1u << jr) | (1u << jb));
           }
         }
-      }
-      // warp-aggregated append
-      const uint32_t bal = __ballot_sync(0xffffffffu, has);
-      if (bal) {
-        uint32_t base = 0;
-        if (lane == 0) base = (uint32_t)atomicAdd(lcount, (unsigned long long)__popc(bal));
-        base = __shfl_sync(0xffffffffu, base, 0);
-        const uint32_t slot = base + __popc(bal & ((1u << lane) - 1u));
-        if (has && slot < A.list_cap) A.list[slot] = make_uint4(recR, recA, recB, 0u);
       }
     }
   }

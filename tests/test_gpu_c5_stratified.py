@@ -23,20 +23,17 @@ def F():
     return ffs
 
 
-def chunk_straddlers(prob, sms, world, ks=4, kdyn=64, limit=1000):
-    """Requests whose KS-segment task range contains a chunk boundary of the k_live split
-    (NC = sms*64 warps x kdyn x world chunks of 32 pieces, clamped to >= 8 tasks per piece;
-    bounded mode:
-    requests on a node without a free slice have no tasks).  Evenly spaced subset."""
+def chunk_straddlers(prob, sms, world, ks=4, warps_per_sm=16, kdyn=64, limit=1000):
+    """Requests whose KS-segment task range contains a chunk boundary of the search
+    kernel's task split in exhaustive mode (every request enumerated; NC = sms x 16 warps x
+    kdyn x world chunks of 32 pieces, at least 1 task per piece for KS = 4), at world 1 or 8
+    (candidate shards).  Evenly spaced subset."""
     n = prob.chain_len()[prob.req["func"]].astype(np.int64)
-    free = np.zeros(prob.n_nodes, np.int64)
-    np.add.at(free, prob.slices["node"][prob.slices["busy"] == 0].astype(np.int64), 1)
     tab = np.array([comb(m - 1, ks - 1) if m >= ks else 0 for m in range(33)], np.int64)
-    t = tab[n] * (free[prob.req["node"]] > 0)
-    pre = np.concatenate([[0], np.cumsum(t)])
+    pre = np.concatenate([[0], np.cumsum(tab[n])])
     T = int(pre[-1])
-    NC = sms * 64 * kdyn * world
-    want = T // (32 * 8)  # k_live's minimum piece (kLiveMinPiece = 8 tasks)
+    NC = sms * warps_per_sm * kdyn * world
+    want = T // 32
     if want < NC:
         NC = max(world, -(-want // world) * world)
     NT = NC * 32
