@@ -1561,9 +1561,9 @@ cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, c
 // n <= 32, so each level is one warp instruction stream, with no per-lane walk and no
 // divergence between lanes.  Requests whose best key of the earlier segments has cvq = 0
 // and fewer stages are dropped whole (no KS-stage candidate can beat it, R1).  Live masks
-// of a row are paired in order into records {r, maskA, maskB (0 = single), 0}; one
-// warp-aggregated atomic per row reserves their slots.  Candidate shards (world > 1): rank
-// g keeps the rows whose (request, j3, j2) hash is g mod world -- a partition of the masks.
+// of a request are paired in order into records {r, maskA, maskB (0 = single), 0}, staged
+// per warp in shared memory and appended 32 at a time (one atomic per 32 records).
+// Candidate shards (world > 1): rank g keeps the rows whose (request, j3, j2) hash is g mod world -- a partition of the masks.
 __device__ __forceinline__ bool live_owned(uint32_t r, uint32_t j3, uint32_t j2, uint32_t rank, uint32_t world) {
   if (world == 1) return true;
   const uint32_t h = (r * 0x9E3779B1u) ^ ((j3 << 5 | j2) * 0x85EBCA6Bu);
@@ -1581,22 +1581,54 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
   unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;
   unsigned long long* lcount = A.work_ctr + kCtrListCount + KS;
   const uint32_t lt_mask = (1u << lane) - 1u;
-  uint32_t r = 0;
-  // pair the live masks of one row (bit j1 of `bal`, the row's other cuts in `hi`) and
-  // append them; every lane of the warp calls it
+  // per-warp staging of records: flushed 32 at a time with one atomic (a row yields a few
+  // records; an atomic per row serialised the warp on the list counter)
+  __shared__ uint4 stage_all[8][64];
+  uint4* stage = stage_all[threadIdx.x >> 5];
+  uint32_t r = 0, cnt = 0, pend = 0;  // warp-uniform: staged records, unpaired live mask
+  auto flush = [&](uint32_t upto) {  // write stage[0, upto) to the list
+    uint32_t base = 0;
+    if (lane == 0) base = (uint32_t)atomicAdd(lcount, (unsigned long long)upto);
+    base = __shfl_sync(0xffffffffu, base, 0);
+    if (lane < upto && base + lane < A.list_cap) A.list[base + lane] = stage[lane];
+  };
+  auto stage_push = [&](bool has, uint4 rec) {  // lanes with `has` append one record each
+    const uint32_t bal = __ballot_sync(0xffffffffu, has);
+    if (has) stage[cnt + __popc(bal & lt_mask)] = rec;
+    cnt += __popc(bal);
+    __syncwarp();
+    if (cnt >= 32) {
+      flush(32);
+      __syncwarp();
+      if (lane < cnt - 32) stage[lane] = stage[32 + lane];
+      __syncwarp();
+      cnt -= 32;
+    }
+  };
+  // the live masks of one row (bit j1 of `bal`, the row's other cuts in `hi`) continue
+  // the request's sequence after `pend`; consecutive masks are paired, an unpaired last
+  // one stays in `pend`.  Every lane of the warp calls it.
   auto emit_row = [&](uint32_t bal, uint32_t hi) {
     if (!bal) return;
-    const uint32_t np = (__popc(bal) + 1) >> 1;
-    uint32_t base = 0;
-    if (lane == 0) base = (uint32_t)atomicAdd(lcount, (unsigned long long)np);
-    base = __shfl_sync(0xffffffffu, base, 0);
-    const uint32_t rk = __popc(bal & lt_mask);
-    if (((bal >> lane) & 1u) && !(rk & 1u)) {
-      const uint32_t above = lane == 31 ? 0u : bal & ~((2u << lane) - 1u);
-      const uint32_t mB = above ? ((1u << (__ffs(above) - 1)) | hi) : 0u;
-      const uint32_t slot = base + (rk >> 1);
-      if (slot < A.list_cap) A.list[slot] = make_uint4(r, (1u << lane) | hi, mB, 0u);
+    const uint32_t hp = pend ? 1u : 0u;
+    const uint32_t i = __popc(bal & lt_mask) + hp;  // index of this lane's mask
+    const bool mine = (bal >> lane) & 1u;
+    bool has = false;
+    uint4 rec = make_uint4(r, 0u, 0u, 0u);
+    if (mine && (i & 1u)) {  // second of a pair: the previous mask is pend or the bit below
+      const uint32_t below = bal & lt_mask;
+      rec.y = below ? ((1u << (31 - __clz(below))) | hi) : pend;
+      rec.z = (1u << lane) | hi;
+      has = true;
     }
+    const uint32_t tot = __popc(bal) + hp;
+    const uint32_t last = 31 - __clz(bal);
+    pend = (tot & 1u) ? ((1u << last) | hi) : 0u;
+    stage_push(has, rec);
+  };
+  auto end_request = [&]() {
+    if (pend) stage_push(lane == 0, make_uint4(r, pend, 0u, 0u));
+    pend = 0;
   };
   for (;;) {
     unsigned long long jg = 0;
@@ -1663,8 +1695,10 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
           }
         }
       }
+      end_request();
     }
   }
+  if (cnt) flush(cnt);
 }
 
 cudaError_t launch_live(int ks, const LiveArgs& a, int grid, cudaStream_t st) {
