@@ -514,8 +514,8 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   LiveArgs la{};
   if (use_live) {
     const uint64_t want = std::min<uint64_t>(16ull * n_req + (1ull << 20), c->list_cap_max);
-    if (c->list_cap != want) {
-      CK(c->live_list.ensure(std::max<uint64_t>(want, 1) * 16), "cudaMalloc(live list)");
+    if (c->list_cap != want) {  // one list per segment KS = 2..4
+      CK(c->live_list.ensure(std::max<uint64_t>(want, 1) * 16 * 3), "cudaMalloc(live lists)");
       c->list_cap = (uint32_t)want;
     }
     la.image = c->image.as<uint32_t>();
@@ -530,7 +530,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     la.keys = d_keys;
     la.gofs = c->gofs.as<uint32_t>();
     la.grp = c->grp.as<uint32_t>();
-    la.list = c->live_list.as<uint4>();
+    for (int j = 0; j < 3; ++j) la.list[j] = c->live_list.as<uint4>() + (size_t)j * c->list_cap;
     la.list_cap = c->list_cap;
     la.work_ctr = a.work_ctr;
   }
@@ -545,8 +545,17 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     a.list = nullptr;
     a.list_cap = 0;
     if (use_live && k >= 2 && k <= 4) {
-      CK(launch_live((int)k, la, c->sms * 8, st), "live-mask kernel");
-      a.list = c->live_list.as<uint4>();
+      // compaction right before the segment: the keys of all earlier segments drop the
+      // requests already settled with cvq = 0 (a 2- or 3-stage winner with CV^2 < 1/1024
+      // is common; one pass for KS = 2..4 after KS = 1 measured 6x the records at KS = 4)
+      la.ks = k;
+      // requests per warp grab: 32 (one header per lane, loaded in parallel) for the light
+      // KS = 2 pass; fewer for the heavy segments, whose per-request mask work would
+      // otherwise leave the last grabs of a small batch (a request shard) on a few warps
+      const uint64_t warps = (uint64_t)c->sms * 8 * 8, div = k == 2 ? 1 : k == 3 ? 4 : 16;
+      la.per_grab = k == 2 ? 32u : (uint32_t)std::min<uint64_t>(32, std::max<uint64_t>(1, n_req / (warps * div)));
+      CK(launch_live(la, c->sms * 8, st), "live-mask kernel");
+      a.list = la.list[k - 2];
       a.list_cap = c->list_cap;
     }
     CK(launch_search((int)k, verify, a, grid, blk((int)k), shm((int)k), st), "search kernel");

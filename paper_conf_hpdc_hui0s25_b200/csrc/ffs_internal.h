@@ -111,8 +111,9 @@ struct LiveArgs {
   const int64_t* keys;          // best keys of the earlier segments (request-level CV test)
   const uint32_t* gofs;         // [F] word offset of function f's group tables
   const uint32_t* grp;
-  uint4* list;
-  uint32_t list_cap;
+  uint4* list[3];               // record lists of KS = 2, 3, 4 (list_cap records each)
+  uint32_t list_cap, ks;        // the segment this launch compacts (2..4)
+  uint32_t per_grab;            // requests a warp takes per grab (1..32, one per lane)
   unsigned long long* work_ctr;
 };
 
@@ -173,7 +174,7 @@ cudaError_t run_int_peak(int sms, double* ops, double* seconds);
 cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double* seconds);
 cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, const uint32_t* gofs, uint32_t* grp,
                                 cudaStream_t st);
-cudaError_t launch_live(int ks, const LiveArgs& a, int grid, cudaStream_t st);
+cudaError_t launch_live(const LiveArgs& a, int grid, cudaStream_t st);
 
 struct RankedArgs {
   const uint32_t* image;

@@ -1551,134 +1551,167 @@ cudaError_t launch_group_tables(const uint32_t* image, const ImageLayout& lay, c
   return cudaGetLastError();
 }
 
-// K1b: live-mask compaction, one warp per request (warps grab 4 requests at a time).  A
+// K1b: live-mask compaction of segment KS (2..4), launched right before its search.  A
 // mask (j1 < j2 < j3: cut positions) is kept iff its exact e2e lower bound
 //   LB = W(0,b1) + X(b1) + W(b1,b2) + X(b2) + ... + W(b_{KS-1}, n) <= B   (b = j + 1)
-// -- a mask with LB > B holds no feasible candidate, so dropping it is exact.  The warp
-// tests the request's blocks (fixed highest cut j3: R3[b3] + T3[b3], lanes over j3), then
-// the rows of every live block (fixed j2, j3: R2[b2] + Mt[b3][b2] + T3[b3], lanes over j2),
-// then the masks of every live row (H0[b1] + Mt[b2][b1] + row constant, lanes over j1) --
-// n <= 32, so each level is one warp instruction stream, with no per-lane walk and no
-// divergence between lanes.  Requests whose best key of the earlier segments has cvq = 0
-// and fewer stages are dropped whole (no KS-stage candidate can beat it, R1).  Live masks
-// of a request are paired in order into records {r, maskA, maskB (0 = single), 0}, staged
-// per warp in shared memory and appended 32 at a time (one atomic per 32 records).
-// Candidate shards (world > 1): rank g keeps the rows whose (request, j3, j2) hash is g mod world -- a partition of the masks.
+// -- a mask with LB > B holds no feasible candidate, so dropping it is exact.  A warp takes
+// per_grab (<= 32) requests at a time, one per lane: each lane loads its request's header (task counts,
+// best key, function, budget, node availability) in parallel, and the requests that still
+// have work are visited one after another by the whole warp (n <= 32, so each colex level
+// fits the lanes): KS = 4 tests the blocks (fixed highest cut j3: R3[b3] + T3[b3], lanes over
+// j3), the rows of every live block (fixed j2, j3: R2[b2] + Mt[b3][b2] + T3[b3], lanes over
+// j2) and the masks of every live row (H0[b1] + Mt[b2][b1] + row constant, lanes over j1);
+// KS = 3 and 2 are the same with one and two levels fewer.  A request is skipped for a
+// segment when it has no tasks there (short chain, full node, bad request) or when its best
+// key so far has cvq = 0 with fewer stages (no KS-stage candidate can beat it, R1 -- every
+// 1-stage plan has CV = 0: 71 % of C5 after KS = 1, and many 2- and 3-stage winners).
+// Live masks of a request are paired in order into records {r, maskA, maskB (0 = single), 0},
+// staged per warp and segment in shared memory and appended 32 at a time (one atomic per
+// 32 records).  Candidate shards (world > 1): rank g keeps the rows whose (request, j3, j2)
+// hash is g mod world -- a partition of the masks.
 __device__ __forceinline__ bool live_owned(uint32_t r, uint32_t j3, uint32_t j2, uint32_t rank, uint32_t world) {
   if (world == 1) return true;
   const uint32_t h = (r * 0x9E3779B1u) ^ ((j3 << 5 | j2) * 0x85EBCA6Bu);
   return (h ^ (h >> 15)) % world == rank;
 }
 
-template <int KS>
-__global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A) {
-  static_assert(KS >= 2 && KS <= 4, "k_live: KS = 2..4");
-  constexpr uint32_t kReqPerGrab = 4;
-  const uint32_t* img = A.image;
-  const ImageLayout& L = A.lay;
-  const uint32_t lane = threadIdx.x & 31;
-  const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (A.n_req + 1);
-  unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;
-  unsigned long long* lcount = A.work_ctr + kCtrListCount + KS;
-  const uint32_t lt_mask = (1u << lane) - 1u;
-  // per-warp staging of records: flushed 32 at a time with one atomic (a row yields a few
-  // records; an atomic per row serialised the warp on the list counter)
-  __shared__ uint4 stage_all[8][64];
-  uint4* stage = stage_all[threadIdx.x >> 5];
-  uint32_t r = 0, cnt = 0, pend = 0;  // warp-uniform: staged records, unpaired live mask
-  auto flush = [&](uint32_t upto) {  // write stage[0, upto) to the list
+// one segment's record stream of a warp: shared staging, flushed 32 records at a time
+struct LiveStage {
+  uint4* stage;                 // this warp's 64 staging slots
+  uint4* list;
+  unsigned long long* lcount;   // records appended so far (the segment's list length)
+  uint32_t cap, cnt, pend;      // warp-uniform: staged records, unpaired live mask
+
+  __device__ __forceinline__ void flush(uint32_t upto, uint32_t lane) {  // stage[0, upto) -> list
     uint32_t base = 0;
     if (lane == 0) base = (uint32_t)atomicAdd(lcount, (unsigned long long)upto);
     base = __shfl_sync(0xffffffffu, base, 0);
-    if (lane < upto && base + lane < A.list_cap) A.list[base + lane] = stage[lane];
-  };
-  auto stage_push = [&](bool has, uint4 rec) {  // lanes with `has` append one record each
+    if (lane < upto && base + lane < cap) list[base + lane] = stage[lane];
+  }
+  __device__ __forceinline__ void push(bool has, uint4 rec, uint32_t lane) {  // one record per lane with `has`
     const uint32_t bal = __ballot_sync(0xffffffffu, has);
-    if (has) stage[cnt + __popc(bal & lt_mask)] = rec;
+    if (has) stage[cnt + __popc(bal & ((1u << lane) - 1u))] = rec;
     cnt += __popc(bal);
     __syncwarp();
     if (cnt >= 32) {
-      flush(32);
+      flush(32, lane);
       __syncwarp();
       if (lane < cnt - 32) stage[lane] = stage[32 + lane];
       __syncwarp();
       cnt -= 32;
     }
-  };
-  // the live masks of one row (bit j1 of `bal`, the row's other cuts in `hi`) continue
-  // the request's sequence after `pend`; consecutive masks are paired, an unpaired last
-  // one stays in `pend`.  Every lane of the warp calls it.
-  auto emit_row = [&](uint32_t bal, uint32_t hi) {
+  }
+  // the live masks of one row of request r (bit j1 of `bal`, the row's other cuts in `hi`)
+  // continue the request's sequence after `pend`: consecutive masks are paired, an unpaired
+  // last one stays in `pend`.  Every lane of the warp calls it.
+  __device__ __forceinline__ void row(uint32_t bal, uint32_t hi, uint32_t r, uint32_t lane) {
     if (!bal) return;
-    const uint32_t hp = pend ? 1u : 0u;
-    const uint32_t i = __popc(bal & lt_mask) + hp;  // index of this lane's mask
-    const bool mine = (bal >> lane) & 1u;
+    const uint32_t lt = (1u << lane) - 1u, hp = pend ? 1u : 0u;
+    const uint32_t i = __popc(bal & lt) + hp;  // index of this lane's mask in the sequence
     bool has = false;
     uint4 rec = make_uint4(r, 0u, 0u, 0u);
-    if (mine && (i & 1u)) {  // second of a pair: the previous mask is pend or the bit below
-      const uint32_t below = bal & lt_mask;
+    if (((bal >> lane) & 1u) && (i & 1u)) {  // second of a pair: the previous mask is pend or the bit below
+      const uint32_t below = bal & lt;
       rec.y = below ? ((1u << (31 - __clz(below))) | hi) : pend;
       rec.z = (1u << lane) | hi;
       has = true;
     }
-    const uint32_t tot = __popc(bal) + hp;
-    const uint32_t last = 31 - __clz(bal);
-    pend = (tot & 1u) ? ((1u << last) | hi) : 0u;
-    stage_push(has, rec);
-  };
-  auto end_request = [&]() {
-    if (pend) stage_push(lane == 0, make_uint4(r, pend, 0u, 0u));
+    pend = ((__popc(bal) + hp) & 1u) ? ((1u << (31 - __clz(bal))) | hi) : 0u;
+    push(has, rec, lane);
+  }
+  __device__ __forceinline__ void end_request(uint32_t r, uint32_t lane) {
+    if (pend) push(lane == 0, make_uint4(r, pend, 0u, 0u), lane);
     pend = 0;
-  };
+  }
+};
+
+template <int KS>
+__global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A) {
+  static_assert(KS >= 2 && KS <= 4, "k_live: KS = 2..4");
+  constexpr uint32_t kTabWords = 4 * 33 + 33 * 33;  // grp_stride(32)
+  const uint32_t* img = A.image;
+  const ImageLayout& L = A.lay;
+  const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const uint32_t NR = A.n_req;
+  __shared__ uint4 stage_all[8][64];
+  // KS = 3, 4: the visited request's group tables, copied once per request -- the row and
+  // mask tests are a dependent chain per row (ballot -> row constant -> mask loads), so
+  // they run at shared-memory rather than L2 latency
+  __shared__ uint32_t tab_all[KS >= 3 ? 8 : 1][KS >= 3 ? kTabWords : 1];
+  LiveStage sg{stage_all[warp], A.list[KS - 2], A.work_ctr + kCtrListCount + KS, A.list_cap, 0u, 0u};
+  const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (NR + 1);
+  unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;
   for (;;) {
     unsigned long long jg = 0;
     if (lane == 0) jg = atomicAdd(ctr, 1ull);
     jg = __shfl_sync(0xffffffffu, jg, 0);
-    const uint64_t r0 = jg * kReqPerGrab;
-    if (r0 >= A.n_req) break;
-    const uint32_t r1 = (uint32_t)min(r0 + kReqPerGrab, (uint64_t)A.n_req);
-    for (r = (uint32_t)r0; r < r1; ++r) {
-      if (pre[r + 1] == pre[r]) continue;  // no tasks of this KS (short chain, full node, bad request)
-      const uint64_t bk = (uint64_t)A.keys[r];
-      if (bk != kKeyNone && (bk >> 50) == 0 && (int)((bk >> 47) & 7) + 1 < KS) continue;
-      const ffs_request q = A.req[r];
-      const uint32_t n = img[L.o_fdesc + 4 * q.func + 1], N1 = n + 1;
-      const uint32_t B = A.slo[r];
-      const uint64_t fb = A.node_free[q.node];
-      uint32_t av = 0;
+    const uint64_t r0 = jg * A.per_grab;
+    if (r0 >= NR) break;
+    // this lane's request: does the segment need it, its chain length, budget, group tables
+    const uint32_t rl = (uint32_t)r0 + lane;
+    uint32_t n = 0, B = 0, go = 0;
+    bool need = false;
+    if (lane < A.per_grab && rl < NR && pre[rl + 1] != pre[rl]) {
+      const uint64_t bk = (uint64_t)A.keys[rl];
+      need = !(bk != kKeyNone && (bk >> 50) == 0 && (uint32_t)((bk >> 47) & 7) + 1u < (uint32_t)KS);
+      if (need) {
+        const ffs_request q = A.req[rl];
+        n = img[L.o_fdesc + 4 * q.func + 1];
+        B = A.slo[rl];
+        const uint64_t fb = A.node_free[q.node];
+        uint32_t av = 0;
 #pragma unroll
-      for (int p = 0; p < kP; ++p) av |= (((fb >> (8 * p)) & 255u) != 0u ? 1u : 0u) << p;
-      const uint32_t* gp = A.grp + A.gofs[q.func] + av * grp_stride(n);
+        for (int p = 0; p < kP; ++p) av |= (((fb >> (8 * p)) & 255u) != 0u ? 1u : 0u) << p;
+        go = A.gofs[q.func] + av * grp_stride(n);
+      }
+    }
+    uint32_t todo = __ballot_sync(0xffffffffu, need);
+    while (todo) {
+      const int Lr = __ffs(todo) - 1;
+      todo &= todo - 1;
+      const uint32_t r = (uint32_t)r0 + Lr;
+      const uint32_t nr = __shfl_sync(0xffffffffu, n, Lr), N1 = nr + 1;
+      const uint32_t Br = __shfl_sync(0xffffffffu, B, Lr);
+      const uint32_t* gp = A.grp + __shfl_sync(0xffffffffu, go, Lr);
+      if constexpr (KS >= 3) {
+        uint32_t* t = tab_all[warp];
+        const uint32_t words = grp_stride(nr);
+        __syncwarp();  // the previous request's readers are done
+        for (uint32_t i = lane; i < words; i += 32) t[i] = gp[i];
+        __syncwarp();
+        gp = t;
+      }
       const uint32_t* H0 = gp;
       const uint32_t* T3 = gp + N1;
       const uint32_t* R2 = gp + 2 * N1;
       const uint32_t* R3 = gp + 3 * N1;
       const uint32_t* Mt = gp + 4 * N1;
+      const uint32_t h0 = lane + 1 < N1 ? H0[lane + 1] : 0u;  // W(0, b1) + X(b1) of j1 = lane
       // mask test for row (j2, row constant rc): lanes over j1 < j2
       auto row_masks = [&](uint32_t j2, uint32_t rc) {
-        const bool live = lane < j2 && (uint64_t)H0[lane + 1] + Mt[(j2 + 1) * N1 + lane + 1] + rc <= B;
+        const bool live = lane < j2 && (uint64_t)h0 + Mt[(j2 + 1) * N1 + lane + 1] + rc <= Br;
         return __ballot_sync(0xffffffffu, live);
       };
-      if constexpr (KS == 2) {
+      if constexpr (KS == 2) {  // one row, masks j1 (b1 = j1 + 1): H0[b1] + T3[b1]
         const uint32_t j1 = lane;
-        const bool live = j1 + 2 <= n && live_owned(r, 0, j1, A.rank, A.world) &&
-                          (uint64_t)H0[j1 + 1] + T3[j1 + 1] <= B;
-        emit_row(__ballot_sync(0xffffffffu, live), 0u);
-      } else if constexpr (KS == 3) {
+        const bool live = j1 + 2 <= nr && live_owned(r, 0, j1, A.rank, A.world) &&
+                          (uint64_t)h0 + T3[j1 + 1] <= Br;
+        sg.row(__ballot_sync(0xffffffffu, live), 0u, r, lane);
+      } else if constexpr (KS == 3) {  // rows j2 (R2[b2] + T3[b2]), then their masks
         const uint32_t j2 = lane + 1;
-        const bool valid = j2 + 2 <= n && live_owned(r, 0, j2, A.rank, A.world);
+        const bool valid = j2 + 2 <= nr && live_owned(r, 0, j2, A.rank, A.world);
         const uint32_t rc = valid ? T3[j2 + 1] : 0u;
-        uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= B);
+        uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= Br);
         while (rows) {
           const uint32_t b = __ffs(rows) - 1;
           rows &= rows - 1;
           const uint32_t jr = b + 1, rcb = __shfl_sync(0xffffffffu, rc, b);
-          emit_row(row_masks(jr, rcb), 1u << jr);
+          sg.row(row_masks(jr, rcb), 1u << jr, r, lane);
         }
-      } else {
+      } else {  // blocks j3, rows j2 < j3, masks j1 < j2
         const uint32_t j3 = lane + 2;
-        const bool bvalid = j3 + 2 <= n;
-        uint32_t blocks = __ballot_sync(0xffffffffu, bvalid && (uint64_t)R3[j3 + 1] + T3[j3 + 1] <= B);
+        uint32_t blocks = __ballot_sync(0xffffffffu, j3 + 2 <= nr && (uint64_t)R3[j3 + 1] + T3[j3 + 1] <= Br);
+        const uint32_t r2 = lane + 2 < N1 ? R2[lane + 2] : 0u;  // R2[b2] of j2 = lane + 1
         while (blocks) {
           const uint32_t jb = __ffs(blocks) - 1 + 2;
           blocks &= blocks - 1;
@@ -1686,25 +1719,26 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
           const uint32_t j2 = lane + 1;
           const bool valid = j2 < jb && live_owned(r, jb, j2, A.rank, A.world);
           const uint32_t rc = valid ? Mt[b3 * N1 + j2 + 1] + t3 : 0u;
-          uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= B);
+          uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)r2 + rc <= Br);
           while (rows) {
             const uint32_t b = __ffs(rows) - 1;
             rows &= rows - 1;
             const uint32_t jr = b + 1, rcb = __shfl_sync(0xffffffffu, rc, b);
-            emit_row(row_masks(jr, rcb), (1u << jr) | (1u << jb));
+            sg.row(row_masks(jr, rcb), (1u << jr) | (1u << jb), r, lane);
           }
         }
       }
-      end_request();
+      sg.end_request(r, lane);
     }
   }
-  if (cnt) flush(cnt);
+  if (sg.cnt) sg.flush(sg.cnt, lane);
 }
 
-cudaError_t launch_live(int ks, const LiveArgs& a, int grid, cudaStream_t st) {
-  if (ks == 2) k_live<2><<<grid, 256, 0, st>>>(a);
-  else if (ks == 3) k_live<3><<<grid, 256, 0, st>>>(a);
-  else if (ks == 4) k_live<4><<<grid, 256, 0, st>>>(a);
+cudaError_t launch_live(const LiveArgs& a, int grid, cudaStream_t st) {
+  if (a.per_grab < 1 || a.per_grab > 32) return cudaErrorInvalidValue;
+  if (a.ks == 2) k_live<2><<<grid, 256, 0, st>>>(a);
+  else if (a.ks == 3) k_live<3><<<grid, 256, 0, st>>>(a);
+  else if (a.ks == 4) k_live<4><<<grid, 256, 0, st>>>(a);
   else return cudaErrorInvalidValue;
   return cudaGetLastError();
 }

@@ -108,6 +108,23 @@ def plan_step_host(planner, h_req, h_slo, d_req, d_slo, k_max: int, rank: int, w
     return h_out
 
 
+def capture_graph(step):
+    """A rank's whole step (count + scan, every segment, decode: ~12 library calls)
+    captured once into a CUDA graph; ``g.replay()`` then issues it as one launch.  The
+    library allocates its scratch on the first call, so `step` is run once on the capture
+    stream before capturing.  Only collective-free steps (request shards) are captured."""
+    import torch
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        step()
+    torch.cuda.current_stream().wait_stream(side)
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        step()
+    return g
+
+
 def h2d_bytes(R: int, rank: int, world: int, shard: str, row_bytes: int = 12) -> int:
     lo, hi = request_slice(R, rank, world)
     return (hi - lo if shard == "requests" else R) * row_bytes

@@ -8,7 +8,8 @@ import subprocess
 import sys
 
 rep, cands = sys.argv[1], float(sys.argv[2])
-raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+flt = ["-k", "regex:" + sys.argv[3]] if len(sys.argv) > 3 else []  # kernel filter
+raw = subprocess.run(["ncu", "-i", rep, *flt, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(raw)))
 h, v = rows[0], rows[2]
 for w in ["Kernel Name", "gpu__time_duration.sum", "launch__registers_per_thread", "launch__block_size",
@@ -26,7 +27,7 @@ st = sorted(((float(v[i]), n) for i, n in enumerate(h)
             reverse=True)
 tot = sum(x for x, _ in st)
 print("stall samples:", ", ".join(f"{n.split('stalled_')[1]} {x / tot:.2f}" for x, n in st[:8]))
-src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass"],
+src = subprocess.run(["ncu", "-i", rep, *flt, "--page", "source", "--csv", "--print-source", "sass"],
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(src)))
 h = rows[1]
@@ -34,7 +35,9 @@ iA, iE = h.index("Source"), h.index("Instructions Executed")
 ops = collections.Counter()
 tot = 0
 for r in rows[2:]:
-    e = int(r[iE] or 0)
+    if len(r) <= max(iA, iE) or not r[iE].isdigit():
+        continue
+    e = int(r[iE])
     m = re.match(r"(@!?U?P\w+\s+)?([A-Z0-9_]+)", r[iA].strip())
     ops[m.group(2) if m else "?"] += e
     tot += e

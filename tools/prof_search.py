@@ -19,13 +19,15 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", type=int, default=5)
 ap.add_argument("--mode", default="exhaustive", choices=["exhaustive", "bounded"])
 ap.add_argument("--calls", type=int, default=1)
+ap.add_argument("--slice", type=int, default=1, help="plan the first 1/SLICE of the requests (a request shard)")
 a = ap.parse_args()
 prob = W.CONFIGS[a.config]()
 pl = ffs.Planner(0)
 pl.stage(prob)
 pl.set_search_mode(ffs.SEARCH_EXHAUSTIVE if a.mode == "exhaustive" else ffs.SEARCH_BOUNDED)
 req, slo = ffs.to_device(prob)
+hi = prob.R // a.slice
 for _ in range(a.calls):
-    keys = pl.plan_keys(req, slo, prob.k_max)
+    keys = pl.plan_keys(req[:hi], slo[:hi], prob.k_max)
 torch.cuda.synchronize()
 print("segments ms", pl.segment_times()[:prob.k_max], "scored", pl.scored()[:prob.k_max])

@@ -10,7 +10,8 @@ regions), then decode of slice g; the projection adds K all-reduces of the 8 MiB
 modelled at the guide's measured 8-rank NVLink bus bandwidth (725 GB/s,
 B200_PROFILING.md): t = 2 (N-1)/N x bytes / busbw per all-reduce.
 
-Both search modes: exhaustive (the benchmark headline) and bounded (production).
+Both search modes: exhaustive (the benchmark headline) and bounded (production); the
+bounded request shards also replayed from a CUDA graph per rank (dist.capture_graph).
 Output: gpurun_out/shard_emulation.json.
 
     python tools/shard_emulation.py
@@ -35,6 +36,7 @@ def main():
     req, slo = ffs.to_device(prob)
     R, K = prob.R, prob.k_max
     keys = torch.empty(R, dtype=torch.int64, device="cuda")
+    plans = torch.empty((R, 80), dtype=torch.uint8, device="cuda")
     flush = torch.empty(256 * 2**20, dtype=torch.uint8, device="cuda")
     out = {"workload": "C5", "R": R, "busbw_model_Bps": BUSBW, "runs": {}}
 
@@ -54,20 +56,24 @@ def main():
 
     for mode_name, mode in (("exhaustive", ffs.SEARCH_EXHAUSTIVE), ("bounded", ffs.SEARCH_BOUNDED)):
         pl.set_search_mode(mode)
-        for shard in ("requests", "candidates"):
-            if shard == "candidates" and mode_name == "exhaustive":
+        for shard in ("requests", "requests+graph", "candidates"):
+            if shard != "requests" and mode_name == "exhaustive":
                 continue
             res, base = {}, None
             for G in (1, 2, 4, 8):
                 times = []
-                if shard == "requests" or G == 1:
+                if shard.startswith("requests") or G == 1:
                     for g in range(G):
                         lo, hi = dist.request_slice(R, g, G)
 
                         def fn():
                             pl.plan_keys(req[lo:hi], slo[lo:hi], K, keys=keys[lo:hi])
-                            pl.plan_decode(req[lo:hi], slo[lo:hi], keys[lo:hi], K)
-                        times.append(median3(fn))
+                            pl.plan_decode(req[lo:hi], slo[lo:hi], keys[lo:hi], K, out=plans[lo:hi])
+                        if shard == "requests+graph":  # the rank's step replayed from a CUDA graph
+                            graph = dist.capture_graph(fn)
+                            times.append(median3(graph.replay))
+                        else:
+                            times.append(median3(fn))
                     coll = 0.0
                 else:
                     combs = []  # keys after segments 1..k combined over all shards
