@@ -1619,6 +1619,20 @@ struct LiveStage {
     pend = ((__popc(bal) + hp) & 1u) ? ((1u << (31 - __clz(bal))) | hi) : 0u;
     push(has, rec, lane);
   }
+  // the same for live masks held one per lane (lane order = colex order): `bal` = lanes
+  // with a live mask, `mk` = this lane's mask.  Every lane of the warp calls it.
+  __device__ __forceinline__ void masks(uint32_t bal, uint32_t mk, uint32_t r, uint32_t lane) {
+    if (!bal) return;
+    const uint32_t lt = (1u << lane) - 1u, hp = pend ? 1u : 0u;
+    const uint32_t below = bal & lt;
+    const uint32_t prev = __shfl_sync(0xffffffffu, mk, below ? 31 - __clz(below) : lane);
+    const uint32_t i = __popc(below) + hp;
+    const bool has = ((bal >> lane) & 1u) && (i & 1u);  // second of a pair
+    const uint4 rec = make_uint4(r, below ? prev : pend, mk, 0u);
+    const uint32_t last = __shfl_sync(0xffffffffu, mk, 31 - __clz(bal));
+    pend = ((__popc(bal) + hp) & 1u) ? last : 0u;
+    push(has, rec, lane);
+  }
   __device__ __forceinline__ void end_request(uint32_t r, uint32_t lane) {
     if (pend) push(lane == 0, make_uint4(r, pend, 0u, 0u), lane);
     pend = 0;
@@ -1638,6 +1652,16 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
   // mask tests are a dependent chain per row (ballot -> row constant -> mask loads), so
   // they run at shared-memory rather than L2 latency
   __shared__ uint32_t tab_all[KS >= 3 ? 8 : 1][KS >= 3 ? kTabWords : 1];
+  // colex order of the pairs j1 < j2 (< 32): tri[C(j2, 2) + j1] = j2 << 8 | j1
+  __shared__ uint16_t tri[KS >= 3 ? 496 : 1];
+  if constexpr (KS >= 3) {
+    for (uint32_t t = threadIdx.x; t < 496; t += blockDim.x) {
+      uint32_t j2 = 1;
+      while ((j2 + 1) * j2 / 2 <= t) ++j2;
+      tri[t] = (uint16_t)(j2 << 8 | (t - j2 * (j2 - 1) / 2));
+    }
+    __syncthreads();
+  }
   LiveStage sg{stage_all[warp], A.list[KS - 2], A.work_ctr + kCtrListCount + KS, A.list_cap, 0u, 0u};
   const uint64_t* pre = A.prefix + (uint64_t)(KS - 1) * (NR + 1);
   unsigned long long* ctr = A.work_ctr + kCtrLiveGrab + KS;
@@ -1687,28 +1711,37 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
       const uint32_t* R3 = gp + 3 * N1;
       const uint32_t* Mt = gp + 4 * N1;
       const uint32_t h0 = lane + 1 < N1 ? H0[lane + 1] : 0u;  // W(0, b1) + X(b1) of j1 = lane
-      // mask test for row (j2, row constant rc): lanes over j1 < j2
-      auto row_masks = [&](uint32_t j2, uint32_t rc) {
-        const bool live = lane < j2 && (uint64_t)h0 + Mt[(j2 + 1) * N1 + lane + 1] + rc <= Br;
-        return __ballot_sync(0xffffffffu, live);
-      };
       if constexpr (KS == 2) {  // one row, masks j1 (b1 = j1 + 1): H0[b1] + T3[b1]
         const uint32_t j1 = lane;
         const bool live = j1 + 2 <= nr && live_owned(r, 0, j1, A.rank, A.world) &&
                           (uint64_t)h0 + T3[j1 + 1] <= Br;
         sg.row(__ballot_sync(0xffffffffu, live), 0u, r, lane);
-      } else if constexpr (KS == 3) {  // rows j2 (R2[b2] + T3[b2]), then their masks
+      } else if constexpr (KS == 3) {
+        // rows j2 (R2[b2] + T3[b2] <= B, lanes over j2), then the masks (j2, j1) of all
+        // rows flattened over the lanes in colex order, 32 per step (a row-by-row walk
+        // was a serial chain of up to 30 short steps per request)
         const uint32_t j2 = lane + 1;
         const bool valid = j2 + 2 <= nr && live_owned(r, 0, j2, A.rank, A.world);
         const uint32_t rc = valid ? T3[j2 + 1] : 0u;
-        uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= Br);
-        while (rows) {
-          const uint32_t b = __ffs(rows) - 1;
-          rows &= rows - 1;
-          const uint32_t jr = b + 1, rcb = __shfl_sync(0xffffffffu, rc, b);
-          sg.row(row_masks(jr, rcb), 1u << jr, r, lane);
+        const uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)R2[j2 + 1] + rc <= Br);
+        if (rows) {
+          // masks of the live rows' span j2 = jlo..jtop (rows bit b = j2 - 1)
+          const uint32_t jlo = __ffs(rows), jtop = 32 - __clz(rows);
+          const uint32_t tot = jtop * (jtop + 1) / 2;
+          for (uint32_t t0 = jlo * (jlo - 1) / 2; t0 < tot; t0 += 32) {
+            const uint32_t t = t0 + lane;
+            const uint32_t tj = t < tot ? tri[t] : 0x0100u;
+            const uint32_t m2 = tj >> 8, m1 = tj & 255u;  // (j2, j1), j1 < j2
+            const uint32_t rcm = __shfl_sync(0xffffffffu, rc, (m2 - 1) & 31);
+            const bool live = t < tot && ((rows >> (m2 - 1)) & 1u) &&
+                              (uint64_t)H0[m1 + 1] + Mt[(m2 + 1) * N1 + m1 + 1] + rcm <= Br;
+            sg.masks(__ballot_sync(0xffffffffu, live), (1u << m1) | (1u << m2), r, lane);
+          }
         }
-      } else {  // blocks j3, rows j2 < j3, masks j1 < j2
+      } else {
+        // blocks j3 (R3[b3] + T3[b3] <= B, lanes over j3); per live block its rows j2
+        // (R2[b2] + Mt[b3][b2] + T3[b3] <= B, lanes over j2), then the block's masks
+        // (j2, j1) flattened over the lanes in colex order, 32 per step
         const uint32_t j3 = lane + 2;
         uint32_t blocks = __ballot_sync(0xffffffffu, j3 + 2 <= nr && (uint64_t)R3[j3 + 1] + T3[j3 + 1] <= Br);
         const uint32_t r2 = lane + 2 < N1 ? R2[lane + 2] : 0u;  // R2[b2] of j2 = lane + 1
@@ -1719,12 +1752,18 @@ __global__ void __launch_bounds__(256) k_live(const __grid_constant__ LiveArgs A
           const uint32_t j2 = lane + 1;
           const bool valid = j2 < jb && live_owned(r, jb, j2, A.rank, A.world);
           const uint32_t rc = valid ? Mt[b3 * N1 + j2 + 1] + t3 : 0u;
-          uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)r2 + rc <= Br);
-          while (rows) {
-            const uint32_t b = __ffs(rows) - 1;
-            rows &= rows - 1;
-            const uint32_t jr = b + 1, rcb = __shfl_sync(0xffffffffu, rc, b);
-            sg.row(row_masks(jr, rcb), (1u << jr) | (1u << jb), r, lane);
+          const uint32_t rows = __ballot_sync(0xffffffffu, valid && (uint64_t)r2 + rc <= Br);
+          if (!rows) continue;
+          const uint32_t jlo = __ffs(rows), jtop = 32 - __clz(rows);
+          const uint32_t tot = jtop * (jtop + 1) / 2;
+          for (uint32_t t0 = jlo * (jlo - 1) / 2; t0 < tot; t0 += 32) {
+            const uint32_t t = t0 + lane;
+            const uint32_t tj = t < tot ? tri[t] : 0x0100u;
+            const uint32_t m2 = tj >> 8, m1 = tj & 255u;
+            const uint32_t rcm = __shfl_sync(0xffffffffu, rc, (m2 - 1) & 31);
+            const bool live = t < tot && ((rows >> (m2 - 1)) & 1u) &&
+                              (uint64_t)H0[m1 + 1] + Mt[(m2 + 1) * N1 + m1 + 1] + rcm <= Br;
+            sg.masks(__ballot_sync(0xffffffffu, live), (1u << m1) | (1u << m2) | (1u << jb), r, lane);
           }
         }
       }
