@@ -188,8 +188,13 @@ ffs_status ffs_set_search_mode(ffs_ctx *ctx, uint32_t mode);
  * flattened (request, cut mask) task list is cut into world x (search warps) x c chunks
  * of 32 equal contiguous pieces; shard `rank` owns the chunks j with j mod world = rank
  * (chunk interleave, DESIGN.md §4.3/§7) and decides every candidate of its chunks
- * (scored, or in bounded mode possibly proved infeasible by the exact SLO bound).
- * d_keys[r] receives the minimum
+ * (scored, or in bounded mode possibly proved infeasible by the exact SLO bound).  In
+ * bounded mode the segments k = 2..4 are instead partitioned by a hash of (request, two
+ * highest cut positions) -- either way the shards partition the candidates.  Bounded mode
+ * keeps three device lists of live (request, mask pair) records, 16 B each, capacity
+ * 16 n_req + 2^20 records per list (0.85 GB at n_req = 2^20; the environment variable
+ * FFS_LIST_CAP lowers it); a segment whose records exceed it runs on the task ranges
+ * instead, with the same result.  d_keys[r] receives the minimum
  * feasible key of request r within the shard, FFS_KEY_NONE where none (overwritten, not
  * combined with its previous content).  Combine shards with an element-wise MIN
  * (torch.distributed.all_reduce(keys, MIN) over NCCL) before ffs_plan_decode.

@@ -29,13 +29,13 @@ __device__ __forceinline__ float plf(const uint32_t* w, uint32_t o) { return __u
 __device__ __forceinline__ uint32_t pl_diff(const uint32_t* w, uint32_t ob, uint32_t oa) {
   return __float2uint_rn(plf(w, ob) - plf(w, oa));
 }
+// minimum over the (full) warp of a 64-bit value: the minimum high word, then the minimum
+// low word among the lanes holding it -- two REDUX.MIN instead of five shuffle rounds
 __device__ __forceinline__ uint64_t warp_min_u64(uint64_t x) {
-#pragma unroll
-  for (int o = 16; o; o >>= 1) {
-    const uint64_t y = __shfl_xor_sync(0xffffffffu, x, o);
-    x = y < x ? y : x;
-  }
-  return x;
+  const uint32_t hi = (uint32_t)(x >> 32), lo = (uint32_t)x;
+  const uint32_t mh = __reduce_min_sync(0xffffffffu, hi);
+  const uint32_t ml = __reduce_min_sync(0xffffffffu, hi == mh ? lo : 0xffffffffu);
+  return (uint64_t)mh << 32 | ml;
 }
 
 // profiles whose slice can host function f monolithically within budget B (defined with
