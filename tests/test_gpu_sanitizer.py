@@ -1,4 +1,9 @@
-"""compute-sanitizer memcheck / racecheck / synccheck over every kernel (small inputs)."""
+"""compute-sanitizer memcheck / racecheck / synccheck over every kernel (small inputs).
+
+Opt-in (FFS_RUN_SANITIZER=1): the GPU pool closed compute-sanitizer in round 2 (runs under
+it left GPUs needing a reset), so the default GPU suite runs the same small workload
+without the tool (every kernel, exit status and oracle parity) instead; the round-1
+sanitizer runs were clean."""
 import os
 import subprocess
 import sys
@@ -12,6 +17,8 @@ SAN = "/usr/local/cuda/bin/compute-sanitizer"
 
 @pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
 def test_sanitizer_clean(tool):
+    if os.environ.get("FFS_RUN_SANITIZER") != "1":
+        pytest.skip("compute-sanitizer is opt-in (FFS_RUN_SANITIZER=1): closed on the GPU pool")
     if not os.path.exists(SAN):
         pytest.skip("compute-sanitizer not installed")
     cmd = [SAN, "--tool", tool, "--error-exitcode", "3", "--target-processes", "all",
@@ -21,3 +28,12 @@ def test_sanitizer_clean(tool):
     assert res.returncode == 0, out[-4000:]
     assert "sanitize-run ok" in out
     assert "ERROR SUMMARY: 0 errors" in out or "RACECHECK SUMMARY: 0 hazards" in out, out[-2000:]
+
+
+def test_sanitize_workload_without_tool():
+    """The sanitizer's workload (every kernel on small inputs) runs clean without the tool."""
+    res = subprocess.run([sys.executable, os.path.join(HERE, "_sanitize_run.py")], capture_output=True, text=True,
+                         timeout=600)
+    out = res.stdout + res.stderr
+    assert res.returncode == 0, out[-4000:]
+    assert "sanitize-run ok" in out

@@ -3,7 +3,7 @@
 # (k_live + list search) and the fused C4 step, shard emulation, segment scaling, issue
 # microbenchmark.   gpurun --timeout 4000 -- bash tools/gpu_evidence_r2.sh
 set -x
-D=gpurun_out/ev2
+D=${D:-gpurun_out/ev2}
 mkdir -p $D
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > $D/smoke.log 2>&1; echo smoke=$? >> $D/smoke.log
 timeout 1800 python -m pytest tests -m gpu -q --durations=15 > $D/gpu_tests.log 2>&1; echo rc=$? >> $D/gpu_tests.log
