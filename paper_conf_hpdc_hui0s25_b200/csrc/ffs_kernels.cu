@@ -984,7 +984,8 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
 }
 
 template <int KS, bool VERIFY>
-__device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses) {
+__device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses,
+                                              uint32_t* defer = nullptr) {
   uint32_t pend = 0;  // one bit per block of P*P candidates
   if constexpr (KS == 4) {
     __trap();  // KS = 4 uses ks4_pair
@@ -1008,6 +1009,10 @@ __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, u
   }
   constexpr int NB = KS == 2 ? 1 : (KS == 3 ? kP : kP * kP);
   c.n_scored += (KS == 2 ? kP * kP : KS == 3 ? kP * kP * kP : kP * kP * kP * kP);
+  if (!VERIFY && defer) {  // the caller rescans the flagged block warp-cooperatively (KS = 2)
+    *defer = pend;
+    return;
+  }
   const uint32_t all = VERIFY ? ((1u << NB) - 1) : pend;
   for (uint32_t todo = all; todo;) {
     const int b = __ffs(todo) - 1;
@@ -1024,7 +1029,7 @@ __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, u
 
 template <int KS, bool VERIFY>
 __device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, float* rows,
-                                             unsigned long long* misses) {
+                                             unsigned long long* misses, uint32_t* defer = nullptr) {
   // stage boundaries: a cut after component j iff bit j is set
   c.bnd[0] = 0;
   uint32_t m = mask, X = 0;
@@ -1045,7 +1050,7 @@ __device__ __forceinline__ void process_mask(SearchState<KS>& c, uint32_t mask, 
     // exact in fp32: min(B - X, 2^24) is an integer <= 2^24 and every stage sum is < 2^24
     c.blim_raw = (X <= c.B) ? (float)min(c.B - X, 1u << 24) : -1.f;
     c.blim = c.none_can_win ? -1.f : c.blim_raw;
-    unrolled_mask<KS, VERIFY>(c, rows, misses);
+    unrolled_mask<KS, VERIFY>(c, rows, misses, defer);
   } else if constexpr (KS == 1) {
     c.blim = c.blim_raw;
     // 5 candidates per request: evaluate them exactly
@@ -1122,7 +1127,8 @@ __device__ __forceinline__ int64_t exact_key(const SearchState<KS>& c, uint32_t 
 }
 
 // Warp-cooperative exact rescan of the flagged blocks (KS = 4: block = stage-0/1 profiles
-// (d0, d1); KS = 3: block = d0), each a block of 25 candidates (the last two stages' q, p):
+// (d0, d1); KS = 3: block = d0; KS = 2: the mask), each a block of 25 candidates (the last
+// two stages' q, p):
 // the block's owner lane broadcasts its request state, 25 lanes evaluate one candidate
 // each, the warp minimum goes back to the owner.  In the bounded list mode the flags are
 // frequent and sparse across lanes -- rescanned lane by lane they ran at ~2 active threads
@@ -1152,6 +1158,10 @@ __device__ __forceinline__ void coop_rescan(SearchState<KS>& c, uint32_t mask, u
         prof[2] = q;
         prof[3] = p;
         seq = (uint64_t)b * (kP * kP) + lane;
+      } else if constexpr (KS == 2) {  // one block per mask (b = 0)
+        prof[0] = q;
+        prof[1] = p;
+        seq = lane;
       } else {
         prof[0] = b;
         prof[1] = q;
@@ -1286,6 +1296,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
         } else if constexpr (KS == 3) {
           ks3_pair<false>(c, maskA, haveB ? maskB : maskA, haveB, A.misses, false, shiftB, pend);
         } else if constexpr (KS == 2) {
+          // (flags are dense among live records: each lane rescans its own, in parallel)
           process_mask<KS, false>(c, maskA, rows, A.misses);
           if (haveB) {
             c.idx_base += shiftB;
@@ -1381,13 +1392,17 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
             mB = maskB;
             if (haveB) step = 2;
           } else {
-            process_mask<KS, VERIFY>(c, mask, rows, A.misses);
+            process_mask<KS, VERIFY>(c, mask, rows, A.misses, (KS == 2 && !VERIFY) ? pend : nullptr);
+            mA = mask;
           }
         }
         if constexpr (!VERIFY && (KS == 3 || KS == 4)) {
           __syncwarp();
           coop_rescan<KS>(c, mA, pend[0], i0);  // before the lane moves on to another request
           coop_rescan<KS>(c, mB, pend[1], i0 + PK);
+        } else if constexpr (!VERIFY && KS == 2) {
+          __syncwarp();  // (flags are sparse over task ranges: cooperative, ~2x over per lane)
+          coop_rescan<KS>(c, mA, pend[0], i0);
         }
         if (active) {
           if (step == 2) mask = mB;

@@ -6,7 +6,10 @@ import sys
 
 rep = sys.argv[1]
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 40
-flt = ["-k", "regex:" + sys.argv[3]] if len(sys.argv) > 3 else []
+flt = []
+if len(sys.argv) > 3:  # a kernel-name regex, or the index of the launch in the report
+    a = sys.argv[3]
+    flt = ["--launch-skip", a, "--launch-count", "1"] if a.isdigit() else ["-k", "regex:" + a]
 out = subprocess.run(["ncu", "-i", rep, *flt, "--page", "source", "--csv", "--print-source", "cuda,sass"],
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(out.splitlines()))
