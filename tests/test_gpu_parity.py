@@ -679,6 +679,25 @@ def check_plan_properties(prob, p):
     assert (sl["profile"][s[live]] == p["prof"][ok][live]).all()
 
 
+@pytest.mark.parametrize("cfg", ["C3", "C5"])
+def test_host_entry_point_large(F, planner, cfg):
+    """ffs_plan_batch_host at C3 / C5 size: byte-identical to ffs_plan_batch on the
+    device-resident batch, with pinned and with pageable host buffers."""
+    import torch
+    prob = W.config3() if cfg == "C3" else W.config5()
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    ref = F.plans_to_numpy(planner.plan_batch(req, slo, prob.k_max))
+    h_req = torch.from_numpy(np.ascontiguousarray(prob.req).view(np.uint8)).pin_memory()
+    h_slo = torch.from_numpy(np.ascontiguousarray(prob.slo_us).view(np.uint8)).pin_memory()
+    h_out = torch.zeros(prob.R * 80, dtype=torch.uint8).pin_memory()
+    out = h_out.numpy().view(F.PLAN_DTYPE)
+    planner.plan_batch_host(h_req.numpy().view(W.REQ_DTYPE), h_slo.numpy().view(np.uint32), prob.k_max, out=out)
+    np.testing.assert_array_equal(out.view(np.uint8), ref.view(np.uint8))
+    pageable = planner.plan_batch_host(np.ascontiguousarray(prob.req), np.ascontiguousarray(prob.slo_us), prob.k_max)
+    np.testing.assert_array_equal(pageable.view(np.uint8), ref.view(np.uint8))
+
+
 def test_c5_full_batch_properties(F, planner):
     prob = W.config5()
     p, _, _ = run_gpu(F, planner, prob, verify=False)
