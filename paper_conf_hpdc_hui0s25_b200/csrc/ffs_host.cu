@@ -89,7 +89,7 @@ struct ffs_ctx {
   DevBuf prefix, block_sums, keys, req_dev, slo_dev, plans_dev, misses, v_tab, work_ctr;
   // cached occupancy per (ks, verify, smem)
   size_t occ_smem = 0;
-  int occ[2][kMaxK + 1] = {};
+  int occ[3][kMaxK + 1] = {};  // [task ranges | verify | bounded list kernel][KS]
   // per-segment timing of the last plan_keys call
   cudaEvent_t ev[kMaxK + 1] = {}, evs[kMaxK + 1] = {};  // per segment: end, start
   uint32_t seg_mask = 0;                                 // segments timed since the last k_first = 1
@@ -477,13 +477,15 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   const bool tables_global = (size_t)c->lay.words * 4 + min_win > kMaxSmem;
   const size_t smem = tables_global ? 0 : (size_t)c->lay.words * 4;
   const int block4 = search_block(4);
-  auto blk = [&](int k) { return k == 4 ? block4 : search_block(k); };
+  // kernel variants: v = 0 task ranges, 1 verify, 2 the bounded mode's list kernel (KS = 2..4)
+  auto blk = [&](int k, int v) { return k == 4 ? block4 : search_block(k, v == 2); };
   auto shm = [&](int k) { return smem + (k == 4 ? kWin4 * block4 : 0); };
   if (c->occ_smem != smem + 1) {  // (smem = 0 <=> tables in global memory)
-    for (int v = 0; v < 2; ++v)
+    for (int v = 0; v < 3; ++v)
       for (int k = 1; k <= kMaxK; ++k) {
+        if (v == 2 && (k < 2 || k > 4)) continue;
         int b = 0;
-        CK(search_kernel_config(k, v != 0, tables_global, blk(k), shm(k), &b), "search kernel occupancy");
+        CK(search_kernel_config(k, v == 1, v == 2, tables_global, blk(k, v), shm(k), &b), "search kernel occupancy");
         c->occ[v][k] = std::max(1, b);
       }
     c->occ_smem = smem + 1;
@@ -536,7 +538,9 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
   }
   if (init) c->seg_mask = 0;
   for (uint32_t k = k_first; k <= kk; ++k) {
-    const int grid = c->sms * c->occ[verify ? 1 : 0][k];
+    const bool list = use_live && k >= 2 && k <= 4;
+    const int var = verify ? 1 : list ? 2 : 0;
+    const int grid = c->sms * c->occ[var][k];
     static const char* kSegName[kMaxK + 1] = {"", "ffs search KS=1", "ffs search KS=2", "ffs search KS=3",
                                               "ffs search KS=4", "ffs search KS=5", "ffs search KS=6",
                                               "ffs search KS=7", "ffs search KS=8"};
@@ -544,7 +548,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     CK(cudaEventRecord(c->evs[k], st), "event");
     a.list = nullptr;
     a.list_cap = 0;
-    if (use_live && k >= 2 && k <= 4) {
+    if (list) {
       // compaction right before the segment: the keys of all earlier segments drop the
       // requests already settled with cvq = 0 (a 2- or 3-stage winner with CV^2 < 1/1024
       // is common; one pass for KS = 2..4 after KS = 1 measured 6x the records at KS = 4)
@@ -558,7 +562,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
       a.list = la.list[k - 2];
       a.list_cap = c->list_cap;
     }
-    CK(launch_search((int)k, verify, a, grid, blk((int)k), shm((int)k), st), "search kernel");
+    CK(launch_search((int)k, verify, list, a, grid, blk((int)k, var), shm((int)k), st), "search kernel");
     CK(cudaEventRecord(c->ev[k], st), "event");
     nvtxRangePop();
     c->seg_mask |= 1u << k;

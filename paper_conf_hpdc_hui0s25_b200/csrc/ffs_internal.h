@@ -28,8 +28,14 @@ constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
 #ifndef FFS_BLOCK4
 #define FFS_BLOCK4 512
 #endif
-__host__ __device__ constexpr int search_block(int ks) {
-  return ks == 3 ? 384 : ks == 4 ? FFS_BLOCK4 : kBlock;
+// KS = 3: the f16x2 core of the task-range kernel (exhaustive / verify modes, 127-136
+// registers) runs 16 warps per SM; the list kernel of the bounded mode keeps the fp32 core
+// (tighter filter margin: fewer rescans of its near-winning records, 168 registers, 12 warps)
+#ifndef FFS_BLOCK3
+#define FFS_BLOCK3 512
+#endif
+__host__ __device__ constexpr int search_block(int ks, bool list = false) {
+  return ks == 3 ? (list ? 384 : FFS_BLOCK3) : ks == 4 ? FFS_BLOCK4 : kBlock;
 }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
 // bytes of per-thread shared memory of the KS = 4 kernel: 5 profiles x 11 packed f16x2
@@ -150,9 +156,9 @@ cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, co
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
                                unsigned long long* checks, unsigned long long* work_ctr, uint32_t k_first,
                                uint32_t k_last, cudaStream_t st);
-cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
+cudaError_t launch_search(int ks, bool verify, bool list, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st);
-cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,
+cudaError_t search_kernel_config(int ks, bool verify, bool list, bool tables_global, int block, size_t smem,
                                  int* blocks_per_sm);
 cudaError_t launch_decode(const DecodeArgs& a, unsigned long long* vtab, cudaStream_t st);
 cudaError_t launch_evict(const ffs_instance* inst, uint32_t n_inst, const uint32_t* tick_off,

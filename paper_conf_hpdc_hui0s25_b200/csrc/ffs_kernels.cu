@@ -219,11 +219,12 @@ __device__ __forceinline__ void set_threshold(SearchState<KS>& c) {
     // filter: (sum t)^2 > alpha * sum t^2 with alpha rounded down by a 2^-16 margin
     // 1024*KS*(1 - 2^-16) = KS*65535/64 is exact in fp32; the quotient is rounded down
     c.alpha = __fdiv_rd((float)(KS * 65535) * (1.f / 64.f), (float)(1025 + cthr));
-    if constexpr (KS == 4) ap = __fdiv_rd((float)(1024 * KS), (float)(1025 + cthr));
+    if constexpr (KS == 3 || KS == 4) ap = __fdiv_rd((float)(1024 * KS), (float)(1025 + cthr));
   }
-  if constexpr (KS == 4) {
-    // f16x2 pre-filter (ks4_pair_h): alpha_h = alpha' - 2^-6 (KS + 1 + alpha'), every step
-    // rounded down; the margin covers the f16 rounding (DESIGN.md §4.3 "f16x2 pre-filter")
+  if constexpr (KS == 3 || KS == 4) {
+    // f16x2 pre-filter (ks3_pair_h, ks4_pair_h): alpha_h = alpha' - 2^-6 (KS + 1 + alpha'),
+    // every step rounded down; the margin covers the f16 rounding (DESIGN.md §4.3 "f16x2
+    // pre-filter"; KS = 3 sums fewer terms, so the KS = 4 bound covers it)
     c.alpha_h = __fsub_rd(__fmul_rd(ap, 1.f - 1.f / 64.f), (float)(KS + 1) * (1.f / 64.f));
   }
   c.blim = c.none_can_win ? -1.f : c.blim_raw;
@@ -983,6 +984,155 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   }
 }
 
+// ---- KS = 3, f16x2 pre-filter ---------------------------------------------------------
+// ks4_pair_h with one stage fewer: masks A / B in the low / high f16 halves, each half
+// scaled by its own power of two sigma, memory / floor / an over-long last stage folded in
+// as +INF, group maximum over the last stage (p) per (d0, q): 13 instructions per 10
+// candidates.  Every table fits in registers (no windows in shared memory): stage 1 by
+// multiplicity {> 0, > 1}, the last stage's cc by {> 0, > 1, > 2}; d0 is unrolled so the
+// multiplicity selects are compile-time.  Conservative as ks4_pair_h (same alpha_h margin,
+// same guarded SLO test); flagged blocks (one per d0) are rescanned exactly.
+template <bool VERIFY>
+__device__ __forceinline__ void ks3_pair_h(SearchState<3>& c, uint32_t maskA, uint32_t maskB, bool haveB,
+                                           unsigned long long* misses, uint32_t zero, bool exh, uint64_t shiftB,
+                                           uint32_t* defer = nullptr) {
+  const float INF = __int_as_float(0x7f800000);
+  constexpr h2 kInf2 = 0x7c007c00u, kNegInf2 = 0xfc00fc00u;
+  const float al = c.alpha_h, one_m_a = 1.f - c.alpha_h;
+  const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
+  const uint32_t* PL = c.sm + c.o_pl + c.row0 * kRowW;
+  const uint32_t* PM = c.sm + c.o_pm + c.row0;
+  const uint32_t* XF = c.sm + c.o_xf + c.row0;
+  float f[2][3][kP], sig[2], slack[2];
+  uint32_t ms[2][3];
+  bool wide[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    uint32_t m = h ? maskB : maskA;
+    const int j1 = __ffs(m) - 1;
+    m &= m - 1;
+    const int j2 = __ffs(m) - 1;
+    const uint32_t b[4] = {0u, (uint32_t)j1 + 1, (uint32_t)j2 + 1, c.n};
+    float pr[4][kP];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      if (i == 0) {
+#pragma unroll
+        for (int x = 0; x < kP; ++x) pr[0][x] = 0.f;
+        continue;
+      }
+      const float4 l = *reinterpret_cast<const float4*>(PL + b[i] * kRowW);
+      pr[i][0] = l.x;
+      pr[i][1] = l.y;
+      pr[i][2] = l.z;
+      pr[i][3] = l.w;
+      pr[i][4] = __uint_as_float(PL[b[i] * kRowW + 4]);
+    }
+#pragma unroll
+    for (int st = 0; st < 3; ++st) {
+#pragma unroll
+      for (int x = 0; x < kP; ++x) f[h][st][x] = pr[st + 1][x] - pr[st][x];
+      ms[h][st] = PM[b[st + 1]] - PM[b[st]];
+    }
+    const uint32_t X = XF[j1] + XF[j2];
+    const bool live_h = h == 0 || haveB;  // the B half of a single mask is a dummy: nothing passes
+    const float bl = (live_h && X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
+    // sigma = 2^(5 - E) with M = min(Blim, tmax) <= 2^E (as ks4_pair_h)
+    const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+    const uint32_t mb = __float_as_uint(M);
+    const int E = (int)((mb >> 23) & 255u) - 127 + ((mb & 0x7fffffu) != 0u);
+    sig[h] = __int_as_float((127 + 5 - E) << 23);
+    wide[h] = bl >= 0.f && c.tmin * sig[h] < 0.125f;
+    slack[h] = bl >= 0.f ? M * sig[h] * (1.f + 1.f / 128.f) : -INF;
+  }
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t cap = c.sm[c.o_cap + x];
+    if (c.thr_u == 0xffffffffu) {
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int st = 0; st < 3; ++st) f[h][st][x] = ms[h][st] <= cap ? f[h][st][x] * sig[h] : INF;
+    } else {
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int st = 0; st < 3; ++st)
+          f[h][st][x] = (ms[h][st] <= cap && f[h][st][x] <= c.thr) ? f[h][st][x] * sig[h] : INF;
+    }
+  }
+  h2 v0[kP], nl0[kP], s1w[2][kP], a1[kP], t2[kP], c2w[3][kP];
+  float v2m[2] = {INF, INF};  // fastest admissible last stage per half (>= 1 free slice)
+  h2 v1min = kInf2;
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const h2 p0 = h2pack(f[0][0][x], f[1][0][x]), p1 = h2pack(f[0][1][x], f[1][1][x]);
+    // an over-long last stage is inadmissible (keeps t2 and t2^2 far from overflow)
+    const float u0 = f[0][2][x] <= slack[0] ? f[0][2][x] : INF, u1 = f[1][2][x] <= slack[1] ? f[1][2][x] : INF;
+    const h2 p2 = h2pack(u0, u1);
+    if (fr > 0) {
+      v2m[0] = fminf(v2m[0], u0);
+      v2m[1] = fminf(v2m[1], u1);
+      v1min = h2min(v1min, p1);
+    }
+    v0[x] = fr > 0 ? p0 : kInf2;
+    nl0[x] = h2mul(h2mul(p0, p0), nal2);
+    s1w[0][x] = fr > 0 ? p1 : kInf2;
+    s1w[1][x] = fr > 1 ? p1 : kInf2;
+    a1[x] = h2mul(h2mul(p1, p1), al2);
+    const uint32_t inf2 = ((p2 & 0xffffu) == 0x7c00u ? 0x0000ffffu : 0u) | ((p2 >> 16) == 0x7c00u ? 0xffff0000u : 0u);
+    t2[x] = h2add(p2, p2) & ~inf2;
+    const h2 cc = (h2mul(h2mul(p2, p2), oma2) & ~inf2) | (kNegInf2 & inf2);
+    c2w[0][x] = fr > 0 ? cc : kNegInf2;
+    c2w[1][x] = fr > 1 ? cc : kNegInf2;
+    c2w[2][x] = fr > 2 ? cc : kNegInf2;
+  }
+  const uint32_t slk = h2guard(h2pack(slack[0] - v2m[0], slack[1] - v2m[1]));
+  uint32_t pendA = 0, pendB = 0;
+#pragma unroll
+  for (int d0 = 0; d0 < kP; ++d0) {
+    const h2 S1 = v0[d0], NL1 = nl0[d0];
+    if (!exh) {  // stage-0 bound (bounded mode): every group has S2 >= S1 + v1min
+      const uint32_t okb = isub(slk, h2add(S1, v1min), zero);
+      if (!((okb & 0x8000u) || (haveB && (okb & 0x80000000u)))) continue;
+    }
+    c.n_scored += haveB ? 2 * kP * kP : kP * kP;  // 25 candidates per mask of this d0
+    uint32_t acc = ~0u;
+#pragma unroll
+    for (int q = 0; q < kP; ++q) {
+      const h2 S2 = h2add(S1, s1w[q == d0][q]);
+      const h2 U = h2fma(S2, S2, h2sub(NL1, a1[q]));
+      h2 y[kP];
+#pragma unroll
+      for (int p = 0; p < kP; ++p) y[p] = h2fma(S2, t2[p], c2w[(p == d0) + (p == q)][p]);
+      const h2 z = h2add(h2max(h2max(h2max(y[0], y[1]), y[2]), h2max(y[3], y[4])), U);
+      const uint32_t ok = isub(slk, S2, zero);
+      acc &= z | ~ok;
+    }
+    pendA |= (((acc >> 15) & 1u) ^ 1u) << d0;
+    pendB |= ((acc >> 31) ^ 1u) << d0;
+  }
+  constexpr uint32_t kAllB = (1u << kP) - 1;
+  if (wide[0]) pendA = kAllB;  // dynamic range too wide for f16: every block exactly
+  if (wide[1]) pendB = kAllB;
+  if (!VERIFY && defer) {  // the caller rescans the flagged blocks warp-cooperatively
+    defer[0] = pendA;
+    defer[1] = haveB ? pendB : 0u;
+    return;
+  }
+  if (VERIFY || pendA) {
+    Geo<3> G;
+    geo<3>(c, maskA, G);
+    pair_rescan<3, VERIFY>(c, G, pendA, VERIFY ? kAllB : pendA, 0, misses);
+  }
+  if (haveB && (VERIFY || pendB)) {
+    Geo<3> G;
+    geo<3>(c, maskB, G);
+    pair_rescan<3, VERIFY>(c, G, pendB, VERIFY ? kAllB : pendB, shiftB, misses);
+  }
+}
+
 template <int KS, bool VERIFY>
 __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses,
                                               uint32_t* defer = nullptr) {
@@ -1191,8 +1341,10 @@ __device__ __forceinline__ uint64_t colex_rank(const uint32_t* img, const ImageL
   return rk;
 }
 
-template <int KS, bool VERIFY, bool TG>
-__global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
+// LIST: the bounded mode's kernel (walks k_live's records, task ranges only as the
+// overflow fallback); !LIST: task ranges only (exhaustive and verify modes, or no lists)
+template <int KS, bool VERIFY, bool TG, bool LIST>
+__global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 1) k_plan_search(const __grid_constant__ SearchArgs A) {
   extern __shared__ __align__(16) uint32_t smem[];
   // A0: stage the table image into shared memory (16-byte copies); an image too large
   // for shared memory is read from global memory through L1 instead (A.tables_global)
@@ -1246,7 +1398,7 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
     c.best = *reinterpret_cast<volatile const int64_t*>(A.keys + r);  // earlier segments' minimum
     best0 = c.best;
     if constexpr (KS >= 2) set_threshold(c);
-    if constexpr (KS == 4) {  // f16 scale bounds; fp32 rounding above 2^24 is covered by the 2^-7 slack margin
+    if constexpr (KS == 3 || KS == 4) {  // f16 scale bounds; fp32 rounding above 2^24 is covered by the 2^-7 slack margin
       c.tmin = __uint_as_float(tbl[A.lay.o_tmm + 2 * q.func]);
       c.tmax = __uint_as_float(tbl[A.lay.o_tmm + 2 * q.func + 1]);
     }
@@ -1263,9 +1415,9 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   };
 
   uint64_t n_list = ~0ull;
-  if (!VERIFY && KS >= 2 && KS <= 4 && A.list != nullptr)
+  if (LIST && !VERIFY && KS >= 2 && KS <= 4 && A.list != nullptr)
     n_list = *reinterpret_cast<volatile const unsigned long long*>(A.work_ctr + kCtrListCount + KS);
-  if (n_list <= A.list_cap) {
+  if (LIST && n_list <= A.list_cap) {
     // ---- bounded mode: the live (request, mask pair) records of k_live ----------------
     // A warp takes 32 consecutive records (one per lane) at a time; every record carries
     // its request, so a lane loads the request's state per record.
@@ -1387,7 +1539,11 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
             if constexpr (KS == 4)
               ks4_pair_h<VERIFY>(c, mask, maskB, haveB, reinterpret_cast<h2*>(rows), A.misses, A.zero,
                                  A.exhaustive != 0, PK, VERIFY ? nullptr : pend);
-            else ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0, PK, VERIFY ? nullptr : pend);
+            else if constexpr (LIST)
+              ks3_pair<VERIFY>(c, mask, maskB, haveB, A.misses, A.exhaustive != 0, PK, VERIFY ? nullptr : pend);
+            else
+              ks3_pair_h<VERIFY>(c, mask, maskB, haveB, A.misses, A.zero, A.exhaustive != 0, PK,
+                                 VERIFY ? nullptr : pend);
             mA = mask;
             mB = maskB;
             if (haveB) step = 2;
@@ -1440,65 +1596,71 @@ __global__ void __launch_bounds__(search_block(KS), KS <= 4 ? FFS_MINB4 : 1) k_p
   }
 }
 
-template <int KS, bool V, bool TG>
+template <int KS, bool V, bool TG, bool L>
 static cudaError_t set_attr() {
-  return cudaFuncSetAttribute(k_plan_search<KS, V, TG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
+  return cudaFuncSetAttribute(k_plan_search<KS, V, TG, L>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
 }
 
-#define FFS_KS_SWITCH(ks, verify, CALL)                  \
-  switch ((ks) * 2 + ((verify) ? 1 : 0)) {               \
-    case 2: CALL(1, false); break;                       \
-    case 3: CALL(1, true); break;                        \
-    case 4: CALL(2, false); break;                       \
-    case 5: CALL(2, true); break;                        \
-    case 6: CALL(3, false); break;                       \
-    case 7: CALL(3, true); break;                        \
-    case 8: CALL(4, false); break;                       \
-    case 9: CALL(4, true); break;                        \
-    case 10: CALL(5, false); break;                      \
-    case 11: CALL(5, true); break;                       \
-    case 12: CALL(6, false); break;                      \
-    case 13: CALL(6, true); break;                       \
-    case 14: CALL(7, false); break;                      \
-    case 15: CALL(7, true); break;                       \
-    case 16: CALL(8, false); break;                      \
-    case 17: CALL(8, true); break;                       \
-    default: return cudaErrorInvalidValue;               \
+// (ks, verify, list) -> instantiation; list kernels exist for KS = 2..4 without verify.
+// KS = 4 runs its list kernel for the task ranges too (A.list == nullptr): the same
+// ks4_pair_h core, and the variant compiled without the list path measured 1 % slower.
+#define FFS_KS_SWITCH(ks, verify, list, CALL)                                        \
+  switch ((ks) * 2 + ((verify) ? 1 : 0) + ((list) && !(verify) && (ks) >= 2 && (ks) <= 4 ? 100 : 0)) { \
+    case 2: CALL(1, false, false); break;                                          \
+    case 3: CALL(1, true, false); break;                                           \
+    case 4: CALL(2, false, false); break;                                          \
+    case 5: CALL(2, true, false); break;                                           \
+    case 6: CALL(3, false, false); break;                                          \
+    case 7: CALL(3, true, false); break;                                           \
+    case 8: CALL(4, false, true); break; /* (the same core: one KS = 4 kernel) */  \
+    case 9: CALL(4, true, false); break;                                           \
+    case 10: CALL(5, false, false); break;                                         \
+    case 11: CALL(5, true, false); break;                                          \
+    case 12: CALL(6, false, false); break;                                         \
+    case 13: CALL(6, true, false); break;                                          \
+    case 14: CALL(7, false, false); break;                                         \
+    case 15: CALL(7, true, false); break;                                          \
+    case 16: CALL(8, false, false); break;                                         \
+    case 17: CALL(8, true, false); break;                                          \
+    case 104: CALL(2, false, true); break;                                         \
+    case 106: CALL(3, false, true); break;                                         \
+    case 108: CALL(4, false, true); break;                                         \
+    default: return cudaErrorInvalidValue;                                         \
   }
 
 template <bool TG>
-static cudaError_t search_config_t(int ks, bool verify, int block, size_t smem, int* blocks_per_sm) {
+static cudaError_t search_config_t(int ks, bool verify, bool list, int block, size_t smem, int* blocks_per_sm) {
   cudaError_t e = cudaSuccess;
-#define CFG(K, V)                                                                                        \
-  do {                                                                                                 \
-    e = set_attr<K, V, TG>();                                                                          \
-    if (e == cudaSuccess)                                                                              \
-      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_plan_search<K, V, TG>, block, smem); \
+#define CFG(K, V, L)                                                                                        \
+  do {                                                                                                    \
+    e = set_attr<K, V, TG, L>();                                                                          \
+    if (e == cudaSuccess)                                                                                 \
+      e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, k_plan_search<K, V, TG, L>, block, smem); \
   } while (0)
-  FFS_KS_SWITCH(ks, verify, CFG)
+  FFS_KS_SWITCH(ks, verify, list, CFG)
 #undef CFG
   return e;
 }
 
 template <bool TG>
-static cudaError_t launch_search_t(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
-                                   cudaStream_t st) {
-#define LAUNCH(K, V) k_plan_search<K, V, TG><<<grid, block, smem, st>>>(a)
-  FFS_KS_SWITCH(ks, verify, LAUNCH)
+static cudaError_t launch_search_t(int ks, bool verify, bool list, const SearchArgs& a, int grid, int block,
+                                   size_t smem, cudaStream_t st) {
+#define LAUNCH(K, V, L) k_plan_search<K, V, TG, L><<<grid, block, smem, st>>>(a)
+  FFS_KS_SWITCH(ks, verify, list, LAUNCH)
 #undef LAUNCH
   return cudaGetLastError();
 }
 
-cudaError_t search_kernel_config(int ks, bool verify, bool tables_global, int block, size_t smem,
+cudaError_t search_kernel_config(int ks, bool verify, bool list, bool tables_global, int block, size_t smem,
                                  int* blocks_per_sm) {
-  return tables_global ? search_config_t<true>(ks, verify, block, smem, blocks_per_sm)
-                       : search_config_t<false>(ks, verify, block, smem, blocks_per_sm);
+  return tables_global ? search_config_t<true>(ks, verify, list, block, smem, blocks_per_sm)
+                       : search_config_t<false>(ks, verify, list, block, smem, blocks_per_sm);
 }
 
-cudaError_t launch_search(int ks, bool verify, const SearchArgs& a, int grid, int block, size_t smem,
+cudaError_t launch_search(int ks, bool verify, bool list, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st) {
-  return a.tables_global ? launch_search_t<true>(ks, verify, a, grid, block, smem, st)
-                         : launch_search_t<false>(ks, verify, a, grid, block, smem, st);
+  return a.tables_global ? launch_search_t<true>(ks, verify, list, a, grid, block, smem, st)
+                         : launch_search_t<false>(ks, verify, list, a, grid, block, smem, st);
 }
 
 // ====================================================================================
