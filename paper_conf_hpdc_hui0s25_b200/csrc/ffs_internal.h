@@ -22,9 +22,8 @@ constexpr uint64_t kKeyNone = 0x7FFFFFFFFFFFFFFFull;
 #define FFS_MINB4 1
 #endif
 constexpr int kBlock = FFS_BLOCK;  // threads per CTA of the search kernel
-// KS = 3 keeps every table in registers; capped at 168 registers it runs 12 warps per SM
-// and is faster (C5: 4.3 -> 3.9 ms).  The f16x2 KS = 4 kernel fits in 113 registers at
-// 16 warps per SM (C5: 66.3 ms at 8 warps, 61.0 at 12, 60.1 at 16).
+// The f16x2 KS = 4 kernel uses 128 registers at 16 warps per SM (round 2, C5: 42.6 ms;
+// 8 / 12 / 14 / 18 / 20 warps measured 52.0 / 45.4 / 43.9 / 44.3 / 44.5 ms).
 #ifndef FFS_BLOCK4
 #define FFS_BLOCK4 512
 #endif
