@@ -97,6 +97,8 @@ struct ffs_ctx {
   uint32_t search_mode = FFS_SEARCH_BOUNDED;
   // bounded mode: group tables (per function x availability pattern) and live-record lists
   DevBuf gofs, grp, live_list, d_vtab;
+  // exhaustive / verify KS = 4: requests grouped by chain length (launch_group_n)
+  DevBuf g_perm, g_cnt, g_tab;
   bool grp_ok = false;
   uint32_t list_cap = 0;
   uint64_t list_cap_max = 1ull << 28;  // FFS_LIST_CAP (tests: force the task-range fallback)
@@ -178,7 +180,7 @@ void ffs_destroy(ffs_ctx* c) {
     for (DevBuf* b : {&c->dag_fu, &c->dag_units, &c->dag_xcut, &c->dag_mt_off, &c->dag_mt_mk, &c->dag_mt_cand, &c->dag_sv,
                       &c->rank_off, &c->rank_mask, &c->image, &c->node_free, &c->free_list, &c->slice_node, &c->slice_prof, &c->prefix,
                       &c->block_sums, &c->keys, &c->req_dev, &c->slo_dev, &c->plans_dev, &c->misses, &c->v_tab, &c->work_ctr,
-                      &c->gofs, &c->grp, &c->live_list, &c->d_vtab})
+                      &c->gofs, &c->grp, &c->live_list, &c->d_vtab, &c->g_perm, &c->g_cnt, &c->g_tab})
       b->release();
   }
   delete c;
@@ -548,6 +550,20 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     CK(cudaEventRecord(c->evs[k], st), "event");
     a.list = nullptr;
     a.list_cap = 0;
+    a.g_perm = nullptr;
+    a.g_tab = nullptr;
+    if (k == 4 && !list && (verify || exhaustive)) {
+      // lanes of a warp = 32 requests of equal chain length walking the same masks
+      const uint64_t glen = 34ull * ((n_req + 2047) / 2048) + 1;
+      CK(c->g_perm.ensure((size_t)n_req * 4), "cudaMalloc(group perm)");
+      CK(c->g_cnt.ensure(glen * 8 + (glen / 2048 + 2) * 8), "cudaMalloc(group offsets)");
+      CK(c->g_tab.ensure(68 * 4), "cudaMalloc(group table)");
+      CK(launch_group_n(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, c->g_cnt.as<uint64_t>(),
+                        c->g_cnt.as<uint64_t>() + glen, c->g_tab.as<uint32_t>(), c->g_perm.as<uint32_t>(), st),
+         "group kernels");
+      a.g_perm = c->g_perm.as<uint32_t>();
+      a.g_tab = c->g_tab.as<uint32_t>();
+    }
     if (list) {
       // compaction right before the segment: the keys of all earlier segments drop the
       // requests already settled with cvq = 0 (a 2- or 3-stage winner with CV^2 < 1/1024

@@ -83,7 +83,13 @@ struct SearchArgs {
   // the task ranges (DESIGN.md §4.3 "live-mask compaction")
   const uint4* list;            // {request, maskA, maskB (0 = none), 0}
   uint32_t list_cap;
+  // exhaustive / verify, KS = 4: the requests grouped by chain length (k_group_*); a warp's
+  // lanes walk the same masks of 32 requests with equal n, so the stage-2/3 tables change
+  // only at row boundaries, warp-uniformly.  Null: plain task ranges.
+  const uint32_t* g_perm;       // [n_req] request ids ordered by n (n >= 4 only)
+  const uint32_t* g_tab;        // [2 x 34]: first index in g_perm of each n, unit prefix per n
 };
+constexpr uint32_t kGrpS = 128;  // masks per work unit of the grouped KS = 4 path
 // work_ctr layout: blocks of kCtrBlock words indexed by KS: [KS] task-chunk grab
 // counters; [kCtrScored + KS] candidates the segment's kernel scored (every candidate whose
 // own score it computed); [kCtrListGrab + KS] record-chunk grab counters, [kCtrListCount +
@@ -155,6 +161,12 @@ cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, co
                                bool skip_full, uint64_t* prefix, uint64_t* block_sums, int64_t* keys,
                                unsigned long long* checks, unsigned long long* work_ctr, uint32_t k_first,
                                uint32_t k_last, cudaStream_t st);
+// requests grouped by chain length (stable) for the exhaustive / verify KS = 4 segment:
+// off [34 * ceil(n_req / 2048) + 1], bsum (scan scratch, like the task prefix's), tab [68],
+// perm [n_req]
+cudaError_t launch_group_n(const ffs_request* req, const uint32_t* image, const ImageLayout& lay, uint32_t n_nodes,
+                           uint32_t n_req, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
+                           cudaStream_t st);
 cudaError_t launch_search(int ks, bool verify, bool list, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st);
 cudaError_t search_kernel_config(int ks, bool verify, bool list, bool tables_global, int block, size_t smem,

@@ -170,6 +170,109 @@ cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, co
   return cudaGetLastError();
 }
 
+// K0b: requests grouped by chain length (exhaustive / verify KS = 4)
+__device__ __forceinline__ uint32_t req_chain_len(const ffs_request* req, const uint32_t* img, const ImageLayout& lay,
+                                                  uint32_t n_nodes, uint32_t r) {
+  const ffs_request q = req[r];
+  return (q.func < lay.F && q.node < n_nodes) ? img[lay.o_fdesc + 4 * q.func + 1] : 0u;
+}
+
+// Stable counting sort of the request ids by chain length n (0..33): the order must be
+// deterministic -- a work unit names (n, group of 32 consecutive requests of the sorted
+// order, mask chunk), and the ranks of a candidate-sharded step (separate calls) must agree
+// on it.  Tiles of kGrpTile requests: per-tile counts, one exclusive scan over (n, tile),
+// then a scatter that keeps the request order within n (the routing sort's pattern).
+constexpr int kGrpT = 256, kGrpItems = 8, kGrpTile = kGrpT * kGrpItems, kGrpD = 34;
+__global__ void __launch_bounds__(kGrpT) k_group_hist(const ffs_request* __restrict__ req, const uint32_t* __restrict__ img,
+                                                      ImageLayout lay, uint32_t n_nodes, uint32_t n_req,
+                                                      uint64_t* __restrict__ off, uint32_t nb) {
+  __shared__ uint32_t h[kGrpD];
+  if (threadIdx.x < kGrpD) h[threadIdx.x] = 0;
+  __syncthreads();
+  const uint32_t base = blockIdx.x * kGrpTile;
+  for (int i = threadIdx.x; i < kGrpTile; i += kGrpT)
+    if (base + i < n_req) atomicAdd(&h[req_chain_len(req, img, lay, n_nodes, base + i)], 1u);
+  __syncthreads();
+  if (threadIdx.x < kGrpD) off[(uint64_t)threadIdx.x * nb + blockIdx.x] = h[threadIdx.x];
+}
+
+// one thread: tab[n] = first index of chain length n in perm (tab[33] = requests with
+// n <= 32), tab[34 + n] = first work unit of n (groups of 32 requests x chunks of kGrpS masks)
+__global__ void k_group_tab(const uint32_t* __restrict__ img, ImageLayout lay, const uint64_t* __restrict__ off,
+                            uint32_t nb, uint32_t* __restrict__ tab) {
+  uint32_t units = 0;
+  for (uint32_t n = 0; n < 34; ++n) {
+    tab[n] = (uint32_t)off[(uint64_t)n * nb];
+    tab[34 + n] = units;
+    if (n >= 4 && n <= 32) {
+      const uint32_t k = (uint32_t)(off[(uint64_t)(n + 1) * nb] - off[(uint64_t)n * nb]);
+      const uint32_t M = binom(img, lay, (int)n - 1, 3);
+      units += ((k + 31) / 32) * ((M + kGrpS - 1) / kGrpS);
+    }
+  }
+}
+
+// stable scatter: warp w owns the contiguous eighth [w * 256, (w + 1) * 256) of the tile
+__global__ void __launch_bounds__(kGrpT) k_group_scatter(const ffs_request* __restrict__ req,
+                                                         const uint32_t* __restrict__ img, ImageLayout lay,
+                                                         uint32_t n_nodes, uint32_t n_req,
+                                                         const uint64_t* __restrict__ off, uint32_t nb,
+                                                         uint32_t* __restrict__ perm) {
+  constexpr int kW = kGrpT / 32;
+  __shared__ uint32_t wh[kW][kGrpD];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int d = threadIdx.x; d < kW * kGrpD; d += kGrpT) (&wh[0][0])[d] = 0;
+  __syncthreads();
+  const uint32_t base = blockIdx.x * kGrpTile + w * (32 * kGrpItems);
+  uint32_t dig[kGrpItems];
+#pragma unroll
+  for (int it = 0; it < kGrpItems; ++it) {  // pass 1: per-warp counts
+    const uint32_t i = base + it * 32 + lane;
+    const bool in = i < n_req;
+    dig[it] = in ? req_chain_len(req, img, lay, n_nodes, i) : 64u + lane;
+    const uint32_t m = __match_any_sync(0xffffffffu, dig[it]);
+    if (in && lane == __ffs(m) - 1) wh[w][dig[it]] += __popc(m);
+    __syncwarp();
+  }
+  __syncthreads();
+  if (threadIdx.x < kGrpD) {  // exclusive prefix over warps per n, plus the (n, tile) offset
+    const uint32_t d = threadIdx.x;
+    uint32_t run = (uint32_t)off[(uint64_t)d * nb + blockIdx.x];
+    for (int ww = 0; ww < kW; ++ww) {
+      const uint32_t c = wh[ww][d];
+      wh[ww][d] = run;
+      run += c;
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int it = 0; it < kGrpItems; ++it) {  // pass 2: scatter in request order
+    const uint32_t i = base + it * 32 + lane;
+    const bool in = i < n_req;
+    const uint32_t m = __match_any_sync(0xffffffffu, dig[it]);
+    if (in) perm[wh[w][dig[it]] + __popc(m & ((1u << lane) - 1))] = i;
+    __syncwarp();
+    if (in && lane == __ffs(m) - 1) wh[w][dig[it]] += __popc(m);
+    __syncwarp();
+  }
+}
+
+cudaError_t launch_group_n(const ffs_request* req, const uint32_t* image, const ImageLayout& lay, uint32_t n_nodes,
+                           uint32_t n_req, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
+                           cudaStream_t st) {
+  const uint32_t nb = (n_req + kGrpTile - 1) / kGrpTile;
+  const uint64_t len = (uint64_t)kGrpD * nb + 1;  // the last entry (0) becomes the total
+  const uint32_t sb = (uint32_t)((len + kScanChunk - 1) / kScanChunk);
+  cudaMemsetAsync(off + len - 1, 0, 8, st);
+  k_group_hist<<<nb, kGrpT, 0, st>>>(req, image, lay, n_nodes, n_req, off, nb);
+  k_scan_reduce<<<dim3(sb, 1), kScanT, 0, st>>>(off, len, bsum, sb);
+  k_scan_top<<<1, kScanT, 0, st>>>(bsum, sb);
+  k_scan_apply<<<dim3(sb, 1), kScanT, 0, st>>>(off, len, bsum, sb);
+  k_group_tab<<<1, 1, 0, st>>>(image, lay, off, nb, tab);
+  k_group_scatter<<<nb, kGrpT, 0, st>>>(req, image, lay, n_nodes, n_req, off, nb, perm);
+  return cudaGetLastError();
+}
+
 // ====================================================================================
 // K1: the search (A2-A5)
 // ====================================================================================
@@ -984,6 +1087,228 @@ __device__ __forceinline__ void ks4_pair_h(SearchState<4>& c, uint32_t maskA, ui
   }
 }
 
+// ---- KS = 4 over requests grouped by chain length (exhaustive / verify) ----------------
+// The warp's lanes hold 32 requests with the same n and walk the same masks in lockstep, so
+// a pair's two highest cuts (its "row": stages 2 and 3) change for all lanes at once, at
+// row boundaries: the stage-2/3 half of ks4_pair_h's setup (prefix rows, memory / floor
+// fold, scaled packing, the s2 / c3 windows, a2, t2) runs once per row pair instead of once
+// per mask pair.  Scale sigma and the last stage's admissibility are taken per row (from
+// B - X(j2, j3) >= B - X(mask)): sigma is no larger and the admissibility test no
+// stricter than per mask, so the filter stays conservative; the group SLO test keeps the
+// mask's own slack.  The core (stage-0 loop) is ks4_pair_h's.
+struct Row4 {
+  uint32_t keyA, keyB;  // rows (mask & (mask - 1)) the state was built for; ~0u = none
+  uint32_t Xr[2];       // transfer cost of the two highest cuts per half
+  float sig[2], v3m[2];
+  bool wide[2];
+  h2 a2[kP], t2[kP];
+};
+
+template <bool VERIFY>
+__device__ __forceinline__ void ks4_pair_rows(SearchState<4>& c, Row4& R, uint32_t maskA, uint32_t maskB, bool haveB,
+                                              bool lane_live, h2* rows, unsigned long long* misses, uint32_t zero,
+                                              uint64_t shiftB, uint32_t* defer) {
+  const float INF = __int_as_float(0x7f800000);
+  constexpr int nb = search_block(4);
+  h2* slot = rows + threadIdx.x;
+  constexpr h2 kInf2 = 0x7c007c00u, kNegInf2 = 0xfc00fc00u, kGuard = 0x80008000u;
+  const float al = c.alpha_h, one_m_a = 1.f - c.alpha_h;
+  const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
+  const uint32_t* PL = c.sm + c.o_pl + c.row0 * kRowW;
+  const uint32_t* PM = c.sm + c.o_pm + c.row0;
+  const uint32_t* XF = c.sm + c.o_xf + c.row0;
+  const uint32_t kA = maskA & (maskA - 1), kB = maskB & (maskB - 1);
+  if (kA != R.keyA || kB != R.keyB) {  // warp-uniform (the lanes walk the same masks)
+    R.keyA = kA;
+    R.keyB = kB;
+    float f[2][2][kP], slr[2];
+    uint32_t ms[2][2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      uint32_t m = h ? kB : kA;
+      const int j2 = __ffs(m) - 1;
+      m &= m - 1;
+      const int j3 = __ffs(m) - 1;
+      const uint32_t b[3] = {(uint32_t)j2 + 1, (uint32_t)j3 + 1, c.n};
+      float pr[3][kP];
+#pragma unroll
+      for (int i = 0; i < 3; ++i) {
+        const float4 l = *reinterpret_cast<const float4*>(PL + b[i] * kRowW);
+        pr[i][0] = l.x;
+        pr[i][1] = l.y;
+        pr[i][2] = l.z;
+        pr[i][3] = l.w;
+        pr[i][4] = __uint_as_float(PL[b[i] * kRowW + 4]);
+      }
+#pragma unroll
+      for (int s = 0; s < 2; ++s) {
+#pragma unroll
+        for (int x = 0; x < kP; ++x) f[h][s][x] = pr[s + 1][x] - pr[s][x];
+        ms[h][s] = PM[b[s + 1]] - PM[b[s]];
+      }
+      R.Xr[h] = XF[j2] + XF[j3];
+      const float bl = (lane_live && R.Xr[h] <= c.B && !c.none_can_win) ? (float)min(c.B - R.Xr[h], 1u << 24) : -1.f;
+      const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+      const uint32_t mb = __float_as_uint(M);
+      const int E = (int)((mb >> 23) & 255u) - 127 + ((mb & 0x7fffffu) != 0u);  // M <= 2^E
+      R.sig[h] = __int_as_float((127 + 5 - E) << 23);
+      R.wide[h] = bl >= 0.f && c.tmin * R.sig[h] < 0.125f;
+      slr[h] = bl >= 0.f ? M * R.sig[h] * (1.f + 1.f / 128.f) : -INF;
+    }
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const uint32_t cap = c.sm[c.o_cap + x];
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 2; ++s)
+          f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+    }
+    R.v3m[0] = INF;
+    R.v3m[1] = INF;
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+      const h2 p2 = h2pack(f[0][0][x], f[1][0][x]);
+      const float u0 = f[0][1][x] <= slr[0] ? f[0][1][x] : INF, u1 = f[1][1][x] <= slr[1] ? f[1][1][x] : INF;
+      const h2 p3 = h2pack(u0, u1);
+      if (fr > 0) {
+        R.v3m[0] = fminf(R.v3m[0], u0);
+        R.v3m[1] = fminf(R.v3m[1], u1);
+      }
+      R.a2[x] = h2mul(h2mul(p2, p2), al2);
+      const uint32_t inf3 = ((p3 & 0xffffu) == 0x7c00u ? 0x0000ffffu : 0u) | ((p3 >> 16) == 0x7c00u ? 0xffff0000u : 0u);
+      R.t2[x] = h2add(p3, p3) & ~inf3;
+      const h2 cc = (h2mul(h2mul(p3, p3), oma2) & ~inf3) | (kNegInf2 & inf3);
+      h2* r = slot + (x * 11) * nb;
+      r[2 * nb] = fr > 0 ? p2 : kInf2;
+      r[3 * nb] = fr > 1 ? p2 : kInf2;
+      r[4 * nb] = fr > 2 ? p2 : kInf2;
+      r[5 * nb] = fr > 0 ? cc : kNegInf2;
+      r[6 * nb] = fr > 1 ? cc : kNegInf2;
+      r[7 * nb] = fr > 2 ? cc : kNegInf2;
+      r[8 * nb] = fr > 3 ? cc : kNegInf2;
+    }
+  }
+  // per mask pair: stages 0 and 1, the mask's own SLO slack
+  float f[2][2][kP], sl[2];
+  uint32_t ms[2][2];
+  bool wide[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    uint32_t m = h ? maskB : maskA;
+    const int j1 = __ffs(m) - 1;
+    m &= m - 1;
+    const int j2 = __ffs(m) - 1;
+    const uint32_t b1 = (uint32_t)j1 + 1, b2 = (uint32_t)j2 + 1;
+    const float4 l1 = *reinterpret_cast<const float4*>(PL + b1 * kRowW);
+    const float4 l2 = *reinterpret_cast<const float4*>(PL + b2 * kRowW);
+    const float p1[kP] = {l1.x, l1.y, l1.z, l1.w, __uint_as_float(PL[b1 * kRowW + 4])};
+    const float p2[kP] = {l2.x, l2.y, l2.z, l2.w, __uint_as_float(PL[b2 * kRowW + 4])};
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      f[h][0][x] = p1[x];  // prefix row 0 is zero
+      f[h][1][x] = p2[x] - p1[x];
+    }
+    ms[h][0] = PM[b1] - PM[0];
+    ms[h][1] = PM[b2] - PM[b1];
+    const uint32_t X = XF[j1] + R.Xr[h];
+    const bool live_h = lane_live && (h == 0 || haveB);  // a single mask's B half is a dummy
+    const float bl = (live_h && X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
+    const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+    sl[h] = bl >= 0.f ? M * R.sig[h] * (1.f + 1.f / 128.f) - R.v3m[h] : -INF;
+    wide[h] = bl >= 0.f && R.wide[h];
+  }
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t cap = c.sm[c.o_cap + x];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int s = 0; s < 2; ++s)
+        f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+  }
+  h2 a1[kP];
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const h2 p0 = h2pack(f[0][0][x], f[1][0][x]), p1 = h2pack(f[0][1][x], f[1][1][x]);
+    a1[x] = h2mul(h2mul(p1, p1), al2);
+    h2* r = slot + (x * 11) * nb;
+    r[0 * nb] = fr > 0 ? p1 : kInf2;
+    r[1 * nb] = fr > 1 ? p1 : kInf2;
+    r[9 * nb] = fr > 0 ? p0 : kInf2;
+    r[10 * nb] = h2mul(h2mul(p0, p0), nal2);
+  }
+  const uint32_t slk = h2guard(h2pack(sl[0], sl[1]));
+  uint32_t pendA = 0, pendB = 0;
+#pragma unroll 1
+  for (int d0 = 0; d0 < kP; ++d0) {  // every stage-0 profile (exhaustive / verify)
+    const h2 S1 = slot[(d0 * 11 + 9) * nb];
+    if (lane_live) c.n_scored += haveB ? 250 : 125;  // 125 candidates per mask of this d0, each y_p computed
+    WinH W[kP];
+    const h2* shifted = slot + nb;  // the d0 profile's windows are read one slot later
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const h2* r = (x == d0 ? shifted : slot) + x * 11 * nb;  // a select + immediate offsets
+      W[x].s1 = r[0];
+      W[x].s2[0] = r[2 * nb];
+      W[x].s2[1] = r[3 * nb];
+      W[x].c3[0] = r[5 * nb];
+      W[x].c3[1] = r[6 * nb];
+      W[x].c3[2] = r[7 * nb];
+    }
+    const h2 NL1 = slot[(d0 * 11 + 10) * nb];  // -alpha t0^2
+    uint32_t mm[kP];
+#pragma unroll
+    for (int d1 = 0; d1 < kP; ++d1) {
+      const h2 S2 = h2add(S1, W[d1].s1), NL2 = h2sub(NL1, a1[d1]);
+      uint32_t acc = ~0u;
+#pragma unroll
+      for (int q = 0; q < kP; ++q) {
+        const h2 S3 = h2add(S2, W[q].s2[q == d1]);
+        const h2 U = h2fma(S3, S3, h2sub(NL2, R.a2[q]));
+        h2 y[kP];
+#pragma unroll
+        for (int p = 0; p < kP; ++p) y[p] = h2fma(S3, R.t2[p], W[p].c3[(p == d1) + (p == q)]);
+        const h2 z = h2add(h2max(h2max(h2max(y[0], y[1]), y[2]), h2max(y[3], y[4])), U);
+        const uint32_t ok = isub(slk, S3, zero);
+        acc &= z | ~ok;
+      }
+      mm[d1] = acc;
+    }
+    if ((mm[0] & mm[1] & mm[2] & mm[3] & mm[4] & kGuard) != kGuard) {
+      uint32_t bA = 0, bB = 0;
+#pragma unroll
+      for (int d1 = 0; d1 < kP; ++d1) {
+        bA |= ((mm[d1] >> 15) & 1u) << d1;
+        bB |= (mm[d1] >> 31) << d1;
+      }
+      pendA |= (bA ^ 31u) << (kP * d0);
+      pendB |= (bB ^ 31u) << (kP * d0);
+    }
+  }
+  constexpr uint32_t kAll = (1u << (kP * kP)) - 1;
+  if (wide[0]) pendA = kAll;  // dynamic range too wide for f16: every block exactly
+  if (wide[1]) pendB = kAll;
+  if (!VERIFY && defer) {  // the caller rescans the flagged blocks warp-cooperatively
+    defer[0] = lane_live ? pendA : 0u;
+    defer[1] = (lane_live && haveB) ? pendB : 0u;
+    return;
+  }
+  if (!lane_live) return;
+  if (VERIFY || pendA) {
+    Geo4 G;
+    geo4(c, maskA, G);
+    pair_rescan<4, VERIFY>(c, G, pendA, VERIFY ? kAll : pendA, 0, misses);
+  }
+  if (haveB && (VERIFY || pendB)) {
+    Geo4 G;
+    geo4(c, maskB, G);
+    pair_rescan<4, VERIFY>(c, G, pendB, VERIFY ? kAll : pendB, shiftB, misses);
+  }
+}
+
 // ---- KS = 3, f16x2 pre-filter ---------------------------------------------------------
 // ks4_pair_h with one stage fewer: masks A / B in the low / high f16 halves, each half
 // scaled by its own power of two sigma, memory / floor / an over-long last stage folded in
@@ -1463,6 +1788,64 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
       }
       if (has) flush(0);
     }
+  } else if (KS == 4 && !LIST && A.g_perm != nullptr) {
+    if constexpr (KS == 4 && !LIST) {
+      // ---- exhaustive / verify KS = 4: 32 requests of equal n per warp, lockstep masks ---
+      // Work unit = (n, group of 32 requests of g_perm, chunk of kGrpS masks in colex
+      // order); rank `rank` owns units j * world + rank; warps grab them dynamically.  Every
+      // lane walks the same masks (Gosper), so ks4_pair_rows rebuilds its stage-2/3 tables
+      // warp-uniformly, only when a half's row changes.  A lane past the group's last
+      // request mirrors the first one's state but scores, flags and flushes nothing.
+      const uint32_t* gt = A.g_tab;
+      const uint32_t U = gt[34 + 33];
+      unsigned long long* ctr = A.work_ctr + KS;
+      for (;;) {
+        unsigned long long jg = 0;
+        if (lane == 0) jg = atomicAdd(ctr, 1ull);
+        jg = __shfl_sync(0xffffffffu, jg, 0);
+        const uint64_t u = (uint64_t)jg * A.world + A.rank;
+        if (u >= U) break;
+        uint32_t n = 4;
+        while (n < 32 && gt[34 + n + 1] <= u) ++n;
+        const uint32_t Mn = binom(tbl, A.lay, (int)n - 1, 3), Cn = (Mn + kGrpS - 1) / kGrpS;
+        const uint32_t loc = (uint32_t)(u - gt[34 + n]), g = loc / Cn, ch = loc - g * Cn;
+        const uint32_t ii = 32 * g + lane;
+        const bool has = ii < gt[n + 1] - gt[n];
+        r = A.g_perm[gt[n] + (has ? ii : 32 * g)];
+        const uint32_t m0 = ch * kGrpS, m1 = min(m0 + kGrpS, Mn);
+        load_request(m0);
+        uint32_t mask = 0;
+        {  // colex unrank of m0 among the 3-subsets of the n - 1 cut positions (uniform)
+          uint32_t mm = m0;
+          int cc = (int)n - 2;
+#pragma unroll
+          for (int i = 3; i >= 1; --i) {
+            while (binom(tbl, A.lay, cc, i) > mm) --cc;
+            mask |= 1u << cc;
+            mm -= binom(tbl, A.lay, cc, i);
+            --cc;
+          }
+        }
+        Row4 R;
+        R.keyA = R.keyB = ~0u;
+        for (uint32_t m = m0; m < m1; m += 2) {
+          const bool haveB = m + 1 < m1;
+          const uint32_t maskB = haveB ? gosper_next(mask) : mask;
+          uint32_t pend[2] = {0u, 0u};
+          const uint64_t i0 = c.idx_base;
+          ks4_pair_rows<VERIFY>(c, R, mask, maskB, haveB, has, reinterpret_cast<h2*>(rows), A.misses, A.zero, PK,
+                                VERIFY ? nullptr : pend);
+          if constexpr (!VERIFY) {
+            __syncwarp();
+            coop_rescan<KS>(c, mask, pend[0], i0);
+            coop_rescan<KS>(c, maskB, pend[1], i0 + PK);
+          }
+          if (haveB) mask = gosper_next(maskB);
+          c.idx_base += 2 * PK;
+        }
+        if (has) flush(m1 - m0);
+      }
+    }
   } else {
     // ---- task ranges (exhaustive and verify modes; bounded mode's fallback) -------------
     const uint64_t T = pre[A.n_req];
@@ -1602,8 +1985,6 @@ static cudaError_t set_attr() {
 }
 
 // (ks, verify, list) -> instantiation; list kernels exist for KS = 2..4 without verify.
-// KS = 4 runs its list kernel for the task ranges too (A.list == nullptr): the same
-// ks4_pair_h core, and the variant compiled without the list path measured 1 % slower.
 #define FFS_KS_SWITCH(ks, verify, list, CALL)                                        \
   switch ((ks) * 2 + ((verify) ? 1 : 0) + ((list) && !(verify) && (ks) >= 2 && (ks) <= 4 ? 100 : 0)) { \
     case 2: CALL(1, false, false); break;                                          \
@@ -1612,7 +1993,7 @@ static cudaError_t set_attr() {
     case 5: CALL(2, true, false); break;                                           \
     case 6: CALL(3, false, false); break;                                          \
     case 7: CALL(3, true, false); break;                                           \
-    case 8: CALL(4, false, true); break; /* (the same core: one KS = 4 kernel) */  \
+    case 8: CALL(4, false, false); break;                                          \
     case 9: CALL(4, true, false); break;                                           \
     case 10: CALL(5, false, false); break;                                         \
     case 11: CALL(5, true, false); break;                                          \

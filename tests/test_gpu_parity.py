@@ -228,6 +228,31 @@ def test_exhaustive_mode_scores_every_candidate(F, planner):
         planner.set_search_mode(7)
 
 
+@pytest.mark.parametrize("world", [2, 3, 8])
+def test_exhaustive_sharding_invariance(F, planner, world):
+    """Exhaustive mode over candidate shards (the KS = 4 segment walks requests grouped by
+    chain length, units interleaved over the ranks): every rank's call must derive the same
+    grouping, so the element-wise MIN of the shards' keys equals one GPU's keys, and the
+    shards' device counters add up to sum_r S(n_r, K)."""
+    prob = W.config3()
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    K = prob.k_max
+    try:
+        planner.set_search_mode(F.SEARCH_EXHAUSTIVE)
+        ref = planner.plan_keys(req, slo, K).clone()
+        total = sum(planner.scored()[:K])
+        keys, scored = [], 0
+        for r in range(world):
+            keys.append(planner.plan_keys(req, slo, K, rank=r, world=world).clone())
+            scored += sum(planner.scored()[:K])
+    finally:
+        planner.set_search_mode(F.SEARCH_BOUNDED)
+    import torch
+    assert torch.equal(torch.stack(keys).min(0).values, ref)
+    assert scored == total
+
+
 @pytest.mark.parametrize("seed", range(16))
 def test_bounded_list_mode_chains(F, planner, seed):
     """Production mode (exact SLO lower bounds: live-mask compaction + list search,
