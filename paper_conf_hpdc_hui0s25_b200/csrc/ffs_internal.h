@@ -89,7 +89,10 @@ struct SearchArgs {
   const uint32_t* g_perm;       // [n_req] request ids ordered by n (n >= 4 only)
   const uint32_t* g_tab;        // [2 x 34]: first index in g_perm of each n, unit prefix per n
 };
-constexpr uint32_t kGrpS = 128;  // masks per work unit of the grouped KS = 4 path
+#ifndef FFS_GRP_S
+#define FFS_GRP_S 128
+#endif
+constexpr uint32_t kGrpS = FFS_GRP_S;  // masks per work unit of the grouped KS = 4 path
 // work_ctr layout: blocks of kCtrBlock words indexed by KS: [KS] task-chunk grab
 // counters; [kCtrScored + KS] candidates the segment's kernel scored (every candidate whose
 // own score it computed); [kCtrListGrab + KS] record-chunk grab counters, [kCtrListCount +
