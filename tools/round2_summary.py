@@ -92,4 +92,28 @@ for f in ("shard_emulation.json", "seg_scaling.log", "issue_bench.log", "smoke.l
     if os.path.exists(p):
         shutil.copy(p, os.path.join(DST, {"shard_emulation.json": "shard_emulation_c5.json"}.get(f, f)))
 json.dump(traffic, open(os.path.join(DST, "dram_per_launch_raw.json"), "w"), indent=1)
+
+
+def _bytes(x):  # "25.004032 Mbyte" -> bytes
+    v, u = x.split()
+    return int(round(float(v) * {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}[u]))
+
+
+# profiles/traffic.json: the bench's roofline.traffic (DRAM read + write per launch)
+tj = os.path.join(ROOT, "profiles", "traffic.json")
+tr = json.load(open(tj)) if os.path.exists(tj) else {}
+for key, d in traffic.items():
+    rep, name = key.split(": ", 1)
+    tot = sum(_bytes(x) for x in d.values())
+    if rep == "prof_ks4_exh" and "k_plan_search<4" in name:
+        tr["k_plan_search<4>"] = tot
+        tr["_source"] = (f"profiles/round2/prof_ks4_exh.ncu-rep (ncu --set full, exhaustive mode, C5): "
+                         f"{d.get('dram__bytes_read.sum')} read + {d.get('dram__bytes_write.sum')} written for one "
+                         f"launch of {name.split('(')[0].replace('void ', '')}")
+    if rep == "prof_c4" and "k_evict_ticks" in name:
+        tr["k_evict_ticks"] = tot
+        tr["_source_k_evict_ticks"] = (f"profiles/round2/prof_c4.ncu-rep (ncu --set full, ffs_evict_step on C4): "
+                                       f"{d.get('dram__bytes_read.sum')} read + {d.get('dram__bytes_write.sum')} "
+                                       f"written per launch")
+json.dump(tr, open(tj, "w"), indent=1)
 print("wrote", sorted(os.listdir(DST)))
