@@ -539,6 +539,7 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     la.work_ctr = a.work_ctr;
   }
   if (init) c->seg_mask = 0;
+  bool grouped = false;
   for (uint32_t k = k_first; k <= kk; ++k) {
     const bool list = use_live && k >= 2 && k <= 4;
     const int var = verify ? 1 : list ? 2 : 0;
@@ -552,15 +553,19 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     a.list_cap = 0;
     a.g_perm = nullptr;
     a.g_tab = nullptr;
-    if (k == 4 && !list && (verify || exhaustive)) {
-      // lanes of a warp = 32 requests of equal chain length walking the same masks
-      const uint64_t glen = 34ull * ((n_req + 2047) / 2048) + 1;
-      CK(c->g_perm.ensure((size_t)n_req * 4), "cudaMalloc(group perm)");
-      CK(c->g_cnt.ensure(glen * 8 + (glen / 2048 + 2) * 8), "cudaMalloc(group offsets)");
-      CK(c->g_tab.ensure(68 * 4), "cudaMalloc(group table)");
-      CK(launch_group_n(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, c->g_cnt.as<uint64_t>(),
-                        c->g_cnt.as<uint64_t>() + glen, c->g_tab.as<uint32_t>(), c->g_perm.as<uint32_t>(), st),
-         "group kernels");
+    if ((k == 3 || k == 4) && !list && (verify || exhaustive)) {
+      // lanes of a warp = 32 requests of equal chain length walking the same masks; the
+      // grouping is built once per call, before the first of the two segments
+      if (!grouped) {
+        const uint64_t glen = 34ull * ((n_req + 2047) / 2048) + 1;
+        CK(c->g_perm.ensure((size_t)n_req * 4), "cudaMalloc(group perm)");
+        CK(c->g_cnt.ensure(glen * 8 + (glen / 2048 + 2) * 8), "cudaMalloc(group offsets)");
+        CK(c->g_tab.ensure(102 * 4), "cudaMalloc(group table)");
+        CK(launch_group_n(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, c->g_cnt.as<uint64_t>(),
+                          c->g_cnt.as<uint64_t>() + glen, c->g_tab.as<uint32_t>(), c->g_perm.as<uint32_t>(), st),
+           "group kernels");
+        grouped = true;
+      }
       a.g_perm = c->g_perm.as<uint32_t>();
       a.g_tab = c->g_tab.as<uint32_t>();
     }

@@ -15,6 +15,7 @@
 // Paper: FluidFaaS, HPDC '25.  P:<line> = line of PAPER.md; R<n> = DESIGN.md §3 reading.
 #include <algorithm>
 #include <cstdio>
+#include <type_traits>
 
 #include "ffs_internal.h"
 
@@ -197,17 +198,19 @@ __global__ void __launch_bounds__(kGrpT) k_group_hist(const ffs_request* __restr
 }
 
 // one thread: tab[n] = first index of chain length n in perm (tab[33] = requests with
-// n <= 32), tab[34 + n] = first work unit of n (groups of 32 requests x chunks of kGrpS masks)
+// n <= 32); tab[34 + n] / tab[68 + n] = first work unit of n for KS = 4 / KS = 3 (groups of
+// 32 requests x chunks of kGrpS masks)
 __global__ void k_group_tab(const uint32_t* __restrict__ img, ImageLayout lay, const uint64_t* __restrict__ off,
                             uint32_t nb, uint32_t* __restrict__ tab) {
-  uint32_t units = 0;
+  uint32_t u4 = 0, u3 = 0;
   for (uint32_t n = 0; n < 34; ++n) {
     tab[n] = (uint32_t)off[(uint64_t)n * nb];
-    tab[34 + n] = units;
-    if (n >= 4 && n <= 32) {
-      const uint32_t k = (uint32_t)(off[(uint64_t)(n + 1) * nb] - off[(uint64_t)n * nb]);
-      const uint32_t M = binom(img, lay, (int)n - 1, 3);
-      units += ((k + 31) / 32) * ((M + kGrpS - 1) / kGrpS);
+    tab[34 + n] = u4;
+    tab[68 + n] = u3;
+    if (n >= 3 && n <= 32) {
+      const uint32_t k = (uint32_t)(off[(uint64_t)(n + 1) * nb] - off[(uint64_t)n * nb]), g = (k + 31) / 32;
+      u3 += g * ((binom(img, lay, (int)n - 1, 2) + kGrpS - 1) / kGrpS);
+      if (n >= 4) u4 += g * ((binom(img, lay, (int)n - 1, 3) + kGrpS - 1) / kGrpS);
     }
   }
 }
@@ -1458,6 +1461,168 @@ __device__ __forceinline__ void ks3_pair_h(SearchState<3>& c, uint32_t maskA, ui
   }
 }
 
+// KS = 3 over requests grouped by chain length (exhaustive / verify): ks3_pair_h with the
+// last stage's tables (its "row" = the highest cut) rebuilt only when a half's row changes,
+// warp-uniformly (the lanes walk the same masks), as ks4_pair_rows does for KS = 4.
+struct Row3 {
+  uint32_t keyA, keyB;  // rows (mask & (mask - 1)) the state was built for; ~0u = none
+  uint32_t Xr[2];
+  float sig[2], v2m[2];
+  bool wide[2];
+  h2 t2[kP], c2w[3][kP];
+};
+
+template <bool VERIFY>
+__device__ __forceinline__ void ks3_pair_rows(SearchState<3>& c, Row3& R, uint32_t maskA, uint32_t maskB, bool haveB,
+                                              bool lane_live, unsigned long long* misses, uint32_t zero,
+                                              uint64_t shiftB, uint32_t* defer) {
+  const float INF = __int_as_float(0x7f800000);
+  constexpr h2 kInf2 = 0x7c007c00u, kNegInf2 = 0xfc00fc00u;
+  const float al = c.alpha_h, one_m_a = 1.f - c.alpha_h;
+  const h2 al2 = h2pack(al, al), nal2 = h2pack(-al, -al), oma2 = h2pack(one_m_a, one_m_a);
+  const uint32_t* PL = c.sm + c.o_pl + c.row0 * kRowW;
+  const uint32_t* PM = c.sm + c.o_pm + c.row0;
+  const uint32_t* XF = c.sm + c.o_xf + c.row0;
+  const uint32_t kA = maskA & (maskA - 1), kB = maskB & (maskB - 1);
+  if (kA != R.keyA || kB != R.keyB) {  // warp-uniform
+    R.keyA = kA;
+    R.keyB = kB;
+    float f2[2][kP], slr[2];
+    uint32_t ms2[2];
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int j2 = __ffs(h ? kB : kA) - 1;
+      const uint32_t b2 = (uint32_t)j2 + 1;
+      const float4 la = *reinterpret_cast<const float4*>(PL + b2 * kRowW);
+      const float4 lb = *reinterpret_cast<const float4*>(PL + c.n * kRowW);
+      f2[h][0] = lb.x - la.x;
+      f2[h][1] = lb.y - la.y;
+      f2[h][2] = lb.z - la.z;
+      f2[h][3] = lb.w - la.w;
+      f2[h][4] = __uint_as_float(PL[c.n * kRowW + 4]) - __uint_as_float(PL[b2 * kRowW + 4]);
+      ms2[h] = PM[c.n] - PM[b2];
+      R.Xr[h] = XF[j2];
+      const float bl = (lane_live && R.Xr[h] <= c.B && !c.none_can_win) ? (float)min(c.B - R.Xr[h], 1u << 24) : -1.f;
+      const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+      const uint32_t mb = __float_as_uint(M);
+      const int E = (int)((mb >> 23) & 255u) - 127 + ((mb & 0x7fffffu) != 0u);
+      R.sig[h] = __int_as_float((127 + 5 - E) << 23);
+      R.wide[h] = bl >= 0.f && c.tmin * R.sig[h] < 0.125f;
+      slr[h] = bl >= 0.f ? M * R.sig[h] * (1.f + 1.f / 128.f) : -INF;
+    }
+    R.v2m[0] = INF;
+    R.v2m[1] = INF;
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+      const uint32_t cap = c.sm[c.o_cap + x];
+      float u[2];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const float v = (ms2[h] <= cap && f2[h][x] <= c.thr) ? f2[h][x] * R.sig[h] : INF;
+        u[h] = v <= slr[h] ? v : INF;  // an over-long last stage is inadmissible
+        if (fr > 0) R.v2m[h] = fminf(R.v2m[h], u[h]);
+      }
+      const h2 p2 = h2pack(u[0], u[1]);
+      const uint32_t inf2 = ((p2 & 0xffffu) == 0x7c00u ? 0x0000ffffu : 0u) | ((p2 >> 16) == 0x7c00u ? 0xffff0000u : 0u);
+      R.t2[x] = h2add(p2, p2) & ~inf2;
+      const h2 cc = (h2mul(h2mul(p2, p2), oma2) & ~inf2) | (kNegInf2 & inf2);
+      R.c2w[0][x] = fr > 0 ? cc : kNegInf2;
+      R.c2w[1][x] = fr > 1 ? cc : kNegInf2;
+      R.c2w[2][x] = fr > 2 ? cc : kNegInf2;
+    }
+  }
+  // per mask pair: stages 0 and 1, the mask's own SLO slack
+  float f[2][2][kP], sl[2];
+  uint32_t ms[2][2];
+  bool wide[2];
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    uint32_t m = h ? maskB : maskA;
+    const int j1 = __ffs(m) - 1;
+    m &= m - 1;
+    const int j2 = __ffs(m) - 1;
+    const uint32_t b1 = (uint32_t)j1 + 1, b2 = (uint32_t)j2 + 1;
+    const float4 l1 = *reinterpret_cast<const float4*>(PL + b1 * kRowW);
+    const float4 l2 = *reinterpret_cast<const float4*>(PL + b2 * kRowW);
+    const float p1[kP] = {l1.x, l1.y, l1.z, l1.w, __uint_as_float(PL[b1 * kRowW + 4])};
+    const float p2[kP] = {l2.x, l2.y, l2.z, l2.w, __uint_as_float(PL[b2 * kRowW + 4])};
+#pragma unroll
+    for (int x = 0; x < kP; ++x) {
+      f[h][0][x] = p1[x];  // prefix row 0 is zero
+      f[h][1][x] = p2[x] - p1[x];
+    }
+    ms[h][0] = PM[b1] - PM[0];
+    ms[h][1] = PM[b2] - PM[b1];
+    const uint32_t X = XF[j1] + R.Xr[h];
+    const bool live_h = lane_live && (h == 0 || haveB);
+    const float bl = (live_h && X <= c.B && !c.none_can_win) ? (float)min(c.B - X, 1u << 24) : -1.f;
+    const float M = fmaxf(fminf(bl, c.tmax), 1.f);
+    sl[h] = bl >= 0.f ? M * R.sig[h] * (1.f + 1.f / 128.f) - R.v2m[h] : -INF;
+    wide[h] = bl >= 0.f && R.wide[h];
+  }
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t cap = c.sm[c.o_cap + x];
+#pragma unroll
+    for (int h = 0; h < 2; ++h)
+#pragma unroll
+      for (int s = 0; s < 2; ++s)
+        f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+  }
+  h2 v0[kP], nl0[kP], s1w[2][kP], a1[kP];
+#pragma unroll
+  for (int x = 0; x < kP; ++x) {
+    const uint32_t fr = (uint32_t)(c.freeb >> (8 * x)) & 255u;
+    const h2 p0 = h2pack(f[0][0][x], f[1][0][x]), p1 = h2pack(f[0][1][x], f[1][1][x]);
+    v0[x] = fr > 0 ? p0 : kInf2;
+    nl0[x] = h2mul(h2mul(p0, p0), nal2);
+    s1w[0][x] = fr > 0 ? p1 : kInf2;
+    s1w[1][x] = fr > 1 ? p1 : kInf2;
+    a1[x] = h2mul(h2mul(p1, p1), al2);
+  }
+  const uint32_t slk = h2guard(h2pack(sl[0], sl[1]));
+  uint32_t pendA = 0, pendB = 0;
+#pragma unroll
+  for (int d0 = 0; d0 < kP; ++d0) {
+    const h2 S1 = v0[d0], NL1 = nl0[d0];
+    if (lane_live) c.n_scored += haveB ? 2 * kP * kP : kP * kP;  // 25 candidates per mask of this d0
+    uint32_t acc = ~0u;
+#pragma unroll
+    for (int q = 0; q < kP; ++q) {
+      const h2 S2 = h2add(S1, s1w[q == d0][q]);
+      const h2 U = h2fma(S2, S2, h2sub(NL1, a1[q]));
+      h2 y[kP];
+#pragma unroll
+      for (int p = 0; p < kP; ++p) y[p] = h2fma(S2, R.t2[p], R.c2w[(p == d0) + (p == q)][p]);
+      const h2 z = h2add(h2max(h2max(h2max(y[0], y[1]), y[2]), h2max(y[3], y[4])), U);
+      const uint32_t ok = isub(slk, S2, zero);
+      acc &= z | ~ok;
+    }
+    pendA |= (((acc >> 15) & 1u) ^ 1u) << d0;
+    pendB |= ((acc >> 31) ^ 1u) << d0;
+  }
+  constexpr uint32_t kAllB = (1u << kP) - 1;
+  if (wide[0]) pendA = kAllB;
+  if (wide[1]) pendB = kAllB;
+  if (!VERIFY && defer) {
+    defer[0] = lane_live ? pendA : 0u;
+    defer[1] = (lane_live && haveB) ? pendB : 0u;
+    return;
+  }
+  if (!lane_live) return;
+  if (VERIFY || pendA) {
+    Geo<3> G;
+    geo<3>(c, maskA, G);
+    pair_rescan<3, VERIFY>(c, G, pendA, VERIFY ? kAllB : pendA, 0, misses);
+  }
+  if (haveB && (VERIFY || pendB)) {
+    Geo<3> G;
+    geo<3>(c, maskB, G);
+    pair_rescan<3, VERIFY>(c, G, pendB, VERIFY ? kAllB : pendB, shiftB, misses);
+  }
+}
+
 template <int KS, bool VERIFY>
 __device__ __forceinline__ void unrolled_mask(SearchState<KS>& c, float* rows, unsigned long long* misses,
                                               uint32_t* defer = nullptr) {
@@ -1788,8 +1953,8 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
       }
       if (has) flush(0);
     }
-  } else if (KS == 4 && !LIST && A.g_perm != nullptr) {
-    if constexpr (KS == 4 && !LIST) {
+  } else if ((KS == 3 || KS == 4) && !LIST && A.g_perm != nullptr) {
+    if constexpr ((KS == 3 || KS == 4) && !LIST) {
       // ---- exhaustive / verify KS = 4: 32 requests of equal n per warp, lockstep masks ---
       // Work unit = (n, group of 32 requests of g_perm, chunk of kGrpS masks in colex
       // order); rank `rank` owns units j * world + rank; warps grab them dynamically.  Every
@@ -1797,7 +1962,8 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
       // warp-uniformly, only when a half's row changes.  A lane past the group's last
       // request mirrors the first one's state but scores, flags and flushes nothing.
       const uint32_t* gt = A.g_tab;
-      const uint32_t U = gt[34 + 33];
+      const uint32_t* gu = gt + (KS == 4 ? 34 : 68);  // unit prefix per n of this segment
+      const uint32_t U = gu[33];
       unsigned long long* ctr = A.work_ctr + KS;
       for (;;) {
         unsigned long long jg = 0;
@@ -1805,36 +1971,39 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
         jg = __shfl_sync(0xffffffffu, jg, 0);
         const uint64_t u = (uint64_t)jg * A.world + A.rank;
         if (u >= U) break;
-        uint32_t n = 4;
-        while (n < 32 && gt[34 + n + 1] <= u) ++n;
-        const uint32_t Mn = binom(tbl, A.lay, (int)n - 1, 3), Cn = (Mn + kGrpS - 1) / kGrpS;
-        const uint32_t loc = (uint32_t)(u - gt[34 + n]), g = loc / Cn, ch = loc - g * Cn;
+        uint32_t n = KS;
+        while (n < 32 && gu[n + 1] <= u) ++n;
+        const uint32_t Mn = binom(tbl, A.lay, (int)n - 1, KS - 1), Cn = (Mn + kGrpS - 1) / kGrpS;
+        const uint32_t loc = (uint32_t)(u - gu[n]), g = loc / Cn, ch = loc - g * Cn;
         const uint32_t ii = 32 * g + lane;
         const bool has = ii < gt[n + 1] - gt[n];
         r = A.g_perm[gt[n] + (has ? ii : 32 * g)];
         const uint32_t m0 = ch * kGrpS, m1 = min(m0 + kGrpS, Mn);
         load_request(m0);
         uint32_t mask = 0;
-        {  // colex unrank of m0 among the 3-subsets of the n - 1 cut positions (uniform)
+        {  // colex unrank of m0 among the (KS-1)-subsets of the n - 1 cut positions (uniform)
           uint32_t mm = m0;
           int cc = (int)n - 2;
 #pragma unroll
-          for (int i = 3; i >= 1; --i) {
+          for (int i = KS - 1; i >= 1; --i) {
             while (binom(tbl, A.lay, cc, i) > mm) --cc;
             mask |= 1u << cc;
             mm -= binom(tbl, A.lay, cc, i);
             --cc;
           }
         }
-        Row4 R;
+        std::conditional_t<KS == 4, Row4, Row3> R;
         R.keyA = R.keyB = ~0u;
         for (uint32_t m = m0; m < m1; m += 2) {
           const bool haveB = m + 1 < m1;
           const uint32_t maskB = haveB ? gosper_next(mask) : mask;
           uint32_t pend[2] = {0u, 0u};
           const uint64_t i0 = c.idx_base;
-          ks4_pair_rows<VERIFY>(c, R, mask, maskB, haveB, has, reinterpret_cast<h2*>(rows), A.misses, A.zero, PK,
-                                VERIFY ? nullptr : pend);
+          if constexpr (KS == 4)
+            ks4_pair_rows<VERIFY>(c, R, mask, maskB, haveB, has, reinterpret_cast<h2*>(rows), A.misses, A.zero, PK,
+                                  VERIFY ? nullptr : pend);
+          else
+            ks3_pair_rows<VERIFY>(c, R, mask, maskB, haveB, has, A.misses, A.zero, PK, VERIFY ? nullptr : pend);
           if constexpr (!VERIFY) {
             __syncwarp();
             coop_rescan<KS>(c, mask, pend[0], i0);
