@@ -561,13 +561,15 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
         CK(c->g_perm.ensure((size_t)n_req * 4), "cudaMalloc(group perm)");
         CK(c->g_cnt.ensure(glen * 8 + (glen / 2048 + 2) * 8), "cudaMalloc(group offsets)");
         CK(c->g_tab.ensure(102 * 4), "cudaMalloc(group table)");
-        CK(launch_group_n(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, c->g_cnt.as<uint64_t>(),
+        CK(launch_group_n(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, grp_unit3(n_req),
+                          c->g_cnt.as<uint64_t>(),
                           c->g_cnt.as<uint64_t>() + glen, c->g_tab.as<uint32_t>(), c->g_perm.as<uint32_t>(), st),
            "group kernels");
         grouped = true;
       }
       a.g_perm = c->g_perm.as<uint32_t>();
       a.g_tab = c->g_tab.as<uint32_t>();
+      a.g_s3 = grp_unit3(n_req);
     }
     if (list) {
       // compaction right before the segment: the keys of all earlier segments drop the

@@ -89,11 +89,19 @@ struct SearchArgs {
   // (DESIGN.md §4.3).  Null: plain task ranges.
   const uint32_t* g_perm;       // [n_req] request ids ordered by n (n >= 4 only)
   const uint32_t* g_tab;        // [3 x 34]: first index in g_perm of each n, unit prefix per n (KS = 4, 3)
+  uint32_t g_s3;                // masks per KS = 3 unit (grp_unit3(n_req)); KS = 4: kGrpS
 };
 #ifndef FFS_GRP_S
 #define FFS_GRP_S 128
 #endif
 constexpr uint32_t kGrpS = FFS_GRP_S;  // masks per work unit of the grouped KS = 4 path
+// masks per work unit of the grouped KS = 3 path: a request shard of C5 has too few KS = 3
+// units of 128 masks for 16 warps per SM (measured per shard size 1, 1/2, 1/4, 1/8, 1/16 of
+// C5 with 128 / 64 / 32: 1.80 / 0.93 / 0.54 / 0.41 / 0.30 ms, 1.82 / 0.94 / 0.52 / 0.33 /
+// 0.24, 1.87 / 0.96 / 0.51 / 0.29 / 0.20), so it shrinks with the batch
+__host__ __device__ constexpr uint32_t grp_unit3(uint32_t n_req) {
+  return n_req >= (1u << 19) ? 128u : n_req >= (1u << 18) ? 64u : 32u;
+}
 // work_ctr layout: blocks of kCtrBlock words indexed by KS: [KS] task-chunk grab
 // counters; [kCtrScored + KS] candidates the segment's kernel scored (every candidate whose
 // own score it computed); [kCtrListGrab + KS] record-chunk grab counters, [kCtrListCount +
@@ -169,7 +177,7 @@ cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, co
 // off [34 * ceil(n_req / 2048) + 1], bsum (scan scratch, like the task prefix's), tab [68],
 // perm [n_req]; tab [102]
 cudaError_t launch_group_n(const ffs_request* req, const uint32_t* image, const ImageLayout& lay, uint32_t n_nodes,
-                           uint32_t n_req, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
+                           uint32_t n_req, uint32_t s3, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
                            cudaStream_t st);
 cudaError_t launch_search(int ks, bool verify, bool list, const SearchArgs& a, int grid, int block, size_t smem,
                           cudaStream_t st);

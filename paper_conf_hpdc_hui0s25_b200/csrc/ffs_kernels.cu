@@ -199,20 +199,24 @@ __global__ void __launch_bounds__(kGrpT) k_group_hist(const ffs_request* __restr
 
 // one thread: tab[n] = first index of chain length n in perm (tab[33] = requests with
 // n <= 32); tab[34 + n] / tab[68 + n] = first work unit of n for KS = 4 / KS = 3 (groups of
-// 32 requests x chunks of kGrpS masks)
+// 32 requests x chunks of kGrpS masks), [34 + 33] / [68 + 33] = the unit counts.  Units are
+// numbered from the longest chains down (n = 32 first): the warps grab the largest units
+// first and the small ones fill the tail.
 __global__ void k_group_tab(const uint32_t* __restrict__ img, ImageLayout lay, const uint64_t* __restrict__ off,
-                            uint32_t nb, uint32_t* __restrict__ tab) {
+                            uint32_t nb, uint32_t s3, uint32_t* __restrict__ tab) {
+  for (uint32_t n = 0; n < 34; ++n) tab[n] = (uint32_t)off[(uint64_t)n * nb];
   uint32_t u4 = 0, u3 = 0;
-  for (uint32_t n = 0; n < 34; ++n) {
-    tab[n] = (uint32_t)off[(uint64_t)n * nb];
+  for (int n = 32; n >= 0; --n) {
     tab[34 + n] = u4;
     tab[68 + n] = u3;
-    if (n >= 3 && n <= 32) {
-      const uint32_t k = (uint32_t)(off[(uint64_t)(n + 1) * nb] - off[(uint64_t)n * nb]), g = (k + 31) / 32;
-      u3 += g * ((binom(img, lay, (int)n - 1, 2) + kGrpS - 1) / kGrpS);
-      if (n >= 4) u4 += g * ((binom(img, lay, (int)n - 1, 3) + kGrpS - 1) / kGrpS);
+    if (n >= 3) {
+      const uint32_t k = tab[n + 1] - tab[n], g = (k + 31) / 32;
+      u3 += g * ((binom(img, lay, n - 1, 2) + s3 - 1) / s3);
+      if (n >= 4) u4 += g * ((binom(img, lay, n - 1, 3) + kGrpS - 1) / kGrpS);
     }
   }
+  tab[34 + 33] = u4;
+  tab[68 + 33] = u3;
 }
 
 // stable scatter: warp w owns the contiguous eighth [w * 256, (w + 1) * 256) of the tile
@@ -261,7 +265,7 @@ __global__ void __launch_bounds__(kGrpT) k_group_scatter(const ffs_request* __re
 }
 
 cudaError_t launch_group_n(const ffs_request* req, const uint32_t* image, const ImageLayout& lay, uint32_t n_nodes,
-                           uint32_t n_req, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
+                           uint32_t n_req, uint32_t s3, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
                            cudaStream_t st) {
   const uint32_t nb = (n_req + kGrpTile - 1) / kGrpTile;
   const uint64_t len = (uint64_t)kGrpD * nb + 1;  // the last entry (0) becomes the total
@@ -271,7 +275,7 @@ cudaError_t launch_group_n(const ffs_request* req, const uint32_t* image, const 
   k_scan_reduce<<<dim3(sb, 1), kScanT, 0, st>>>(off, len, bsum, sb);
   k_scan_top<<<1, kScanT, 0, st>>>(bsum, sb);
   k_scan_apply<<<dim3(sb, 1), kScanT, 0, st>>>(off, len, bsum, sb);
-  k_group_tab<<<1, 1, 0, st>>>(image, lay, off, nb, tab);
+  k_group_tab<<<1, 1, 0, st>>>(image, lay, off, nb, s3, tab);
   k_group_scatter<<<nb, kGrpT, 0, st>>>(req, image, lay, n_nodes, n_req, off, nb, perm);
   return cudaGetLastError();
 }
@@ -1971,14 +1975,15 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
         jg = __shfl_sync(0xffffffffu, jg, 0);
         const uint64_t u = (uint64_t)jg * A.world + A.rank;
         if (u >= U) break;
-        uint32_t n = KS;
-        while (n < 32 && gu[n + 1] <= u) ++n;
-        const uint32_t Mn = binom(tbl, A.lay, (int)n - 1, KS - 1), Cn = (Mn + kGrpS - 1) / kGrpS;
+        uint32_t n = 32;  // units of n: [gu[n], gu[n - 1]) (longest chains first), n = KS: up to gu[33]
+        while (n > KS && gu[n - 1] <= u) --n;
+        const uint32_t S = KS == 3 ? A.g_s3 : kGrpS;
+        const uint32_t Mn = binom(tbl, A.lay, (int)n - 1, KS - 1), Cn = (Mn + S - 1) / S;
         const uint32_t loc = (uint32_t)(u - gu[n]), g = loc / Cn, ch = loc - g * Cn;
         const uint32_t ii = 32 * g + lane;
         const bool has = ii < gt[n + 1] - gt[n];
         r = A.g_perm[gt[n] + (has ? ii : 32 * g)];
-        const uint32_t m0 = ch * kGrpS, m1 = min(m0 + kGrpS, Mn);
+        const uint32_t m0 = ch * S, m1 = min(m0 + S, Mn);
         load_request(m0);
         uint32_t mask = 0;
         {  // colex unrank of m0 among the (KS-1)-subsets of the n - 1 cut positions (uniform)
