@@ -553,14 +553,18 @@ static ffs_status search_keys(ffs_ctx* c, const ffs_request* d_req, const uint32
     a.list_cap = 0;
     a.g_perm = nullptr;
     a.g_tab = nullptr;
-    if ((k == 3 || k == 4) && !list && (verify || exhaustive)) {
+    // KS = 2 walks the groups only on large batches: a request's n - 1 masks form one unit,
+    // and a request shard has too few of them (1/8 of C5: 0.09 ms on the task ranges, 0.18
+    // grouped); at full C5 0.48 -> 0.34 ms
+    const bool grp_k = k == 3 || k == 4 || (k == 2 && n_req >= (1u << 19));
+    if (grp_k && !list && (verify || exhaustive)) {
       // lanes of a warp = 32 requests of equal chain length walking the same masks; the
-      // grouping is built once per call, before the first of the two segments
+      // grouping is built once per call, before the first grouped segment
       if (!grouped) {
         const uint64_t glen = 34ull * ((n_req + 2047) / 2048) + 1;
         CK(c->g_perm.ensure((size_t)n_req * 4), "cudaMalloc(group perm)");
         CK(c->g_cnt.ensure(glen * 8 + (glen / 2048 + 2) * 8), "cudaMalloc(group offsets)");
-        CK(c->g_tab.ensure(102 * 4), "cudaMalloc(group table)");
+        CK(c->g_tab.ensure(136 * 4), "cudaMalloc(group table)");
         CK(launch_group_n(d_req, c->image.as<uint32_t>(), c->lay, c->n_nodes, n_req, grp_unit3(n_req),
                           c->g_cnt.as<uint64_t>(),
                           c->g_cnt.as<uint64_t>() + glen, c->g_tab.as<uint32_t>(), c->g_perm.as<uint32_t>(), st),

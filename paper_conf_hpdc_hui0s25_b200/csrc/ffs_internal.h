@@ -83,12 +83,12 @@ struct SearchArgs {
   // the task ranges (DESIGN.md §4.3 "live-mask compaction")
   const uint4* list;            // {request, maskA, maskB (0 = none), 0}
   uint32_t list_cap;
-  // exhaustive / verify, KS = 3 and 4: the requests grouped by chain length (k_group_*); a
+  // exhaustive / verify, KS = 2..4: the requests grouped by chain length (k_group_*); a
   // warp's lanes walk the same masks of 32 requests with equal n, so the tables of the
   // stages after the second-highest cut change only at row boundaries, warp-uniformly
   // (DESIGN.md §4.3).  Null: plain task ranges.
   const uint32_t* g_perm;       // [n_req] request ids ordered by n (n >= 4 only)
-  const uint32_t* g_tab;        // [3 x 34]: first index in g_perm of each n, unit prefix per n (KS = 4, 3)
+  const uint32_t* g_tab;        // [4 x 34]: first index in g_perm of each n, unit prefix per n (KS = 4, 3, 2)
   uint32_t g_s3;                // masks per KS = 3 unit (grp_unit3(n_req)); KS = 4: kGrpS
 };
 #ifndef FFS_GRP_S
@@ -175,7 +175,7 @@ cudaError_t launch_count_tasks(const ffs_request* req, const uint32_t* image, co
                                uint32_t k_last, cudaStream_t st);
 // requests grouped by chain length (stable) for the exhaustive / verify KS = 4 segment:
 // off [34 * ceil(n_req / 2048) + 1], bsum (scan scratch, like the task prefix's), tab [68],
-// perm [n_req]; tab [102]
+// perm [n_req]; tab [136]
 cudaError_t launch_group_n(const ffs_request* req, const uint32_t* image, const ImageLayout& lay, uint32_t n_nodes,
                            uint32_t n_req, uint32_t s3, uint64_t* off, uint64_t* bsum, uint32_t* tab, uint32_t* perm,
                            cudaStream_t st);

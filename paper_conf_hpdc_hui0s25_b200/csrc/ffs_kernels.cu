@@ -198,8 +198,9 @@ __global__ void __launch_bounds__(kGrpT) k_group_hist(const ffs_request* __restr
 }
 
 // one thread: tab[n] = first index of chain length n in perm (tab[33] = requests with
-// n <= 32); tab[34 + n] / tab[68 + n] = first work unit of n for KS = 4 / KS = 3 (groups of
-// 32 requests x chunks of kGrpS masks), [34 + 33] / [68 + 33] = the unit counts.  Units are
+// n <= 32); tab[34 + n] / tab[68 + n] / tab[102 + n] = first work unit of n for KS = 4 / 3 /
+// 2 (groups of 32 requests x chunks of masks), [34 + 33] / [68 + 33] / [102 + 33] = the unit
+// counts.  Units are
 // numbered from the longest chains down (n = 32 first): the warps grab the largest units
 // first and the small ones fill the tail.
 __global__ void k_group_tab(const uint32_t* __restrict__ img, ImageLayout lay, const uint64_t* __restrict__ off,
@@ -217,6 +218,12 @@ __global__ void k_group_tab(const uint32_t* __restrict__ img, ImageLayout lay, c
   }
   tab[34 + 33] = u4;
   tab[68 + 33] = u3;
+  uint32_t u2 = 0;  // KS = 2: one unit per group (n - 1 <= 31 masks)
+  for (int n = 32; n >= 0; --n) {
+    tab[102 + n] = u2;
+    if (n >= 2) u2 += (tab[n + 1] - tab[n] + 31) / 32;
+  }
+  tab[102 + 33] = u2;
 }
 
 // stable scatter: warp w owns the contiguous eighth [w * 256, (w + 1) * 256) of the tile
@@ -1957,16 +1964,16 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
       }
       if (has) flush(0);
     }
-  } else if ((KS == 3 || KS == 4) && !LIST && A.g_perm != nullptr) {
-    if constexpr ((KS == 3 || KS == 4) && !LIST) {
-      // ---- exhaustive / verify KS = 4: 32 requests of equal n per warp, lockstep masks ---
+  } else if (KS >= 2 && KS <= 4 && !LIST && A.g_perm != nullptr) {
+    if constexpr (KS >= 2 && KS <= 4 && !LIST) {
+      // ---- exhaustive / verify KS = 2..4: 32 requests of equal n per warp, lockstep masks -
       // Work unit = (n, group of 32 requests of g_perm, chunk of kGrpS masks in colex
       // order); rank `rank` owns units j * world + rank; warps grab them dynamically.  Every
       // lane walks the same masks (Gosper), so ks4_pair_rows rebuilds its stage-2/3 tables
       // warp-uniformly, only when a half's row changes.  A lane past the group's last
       // request mirrors the first one's state but scores, flags and flushes nothing.
       const uint32_t* gt = A.g_tab;
-      const uint32_t* gu = gt + (KS == 4 ? 34 : 68);  // unit prefix per n of this segment
+      const uint32_t* gu = gt + (KS == 4 ? 34 : KS == 3 ? 68 : 102);  // unit prefix per n of this segment
       const uint32_t U = gu[33];
       unsigned long long* ctr = A.work_ctr + KS;
       for (;;) {
@@ -1977,7 +1984,7 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
         if (u >= U) break;
         uint32_t n = 32;  // units of n: [gu[n], gu[n - 1]) (longest chains first), n = KS: up to gu[33]
         while (n > KS && gu[n - 1] <= u) --n;
-        const uint32_t S = KS == 3 ? A.g_s3 : kGrpS;
+        const uint32_t S = KS == 4 ? kGrpS : KS == 3 ? A.g_s3 : 32u;  // KS = 2: a request's n - 1 <= 31 masks
         const uint32_t Mn = binom(tbl, A.lay, (int)n - 1, KS - 1), Cn = (Mn + S - 1) / S;
         const uint32_t loc = (uint32_t)(u - gu[n]), g = loc / Cn, ch = loc - g * Cn;
         const uint32_t ii = 32 * g + lane;
@@ -1997,6 +2004,21 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
             --cc;
           }
         }
+        if constexpr (KS == 2) {  // one mask per step (25 candidates, fp32 block_qp)
+          for (uint32_t m = m0; m < m1; ++m) {
+            uint32_t pend[2] = {0u, 0u};
+            const uint64_t i0 = c.idx_base;
+            if (has) process_mask<KS, VERIFY>(c, mask, rows, A.misses, VERIFY ? nullptr : pend);
+            if constexpr (!VERIFY) {
+              __syncwarp();
+              coop_rescan<KS>(c, mask, pend[0], i0);
+            }
+            mask = gosper_next(mask);
+            c.idx_base += PK;
+          }
+          if (has) flush(m1 - m0);
+          continue;
+        }
         std::conditional_t<KS == 4, Row4, Row3> R;
         R.keyA = R.keyB = ~0u;
         for (uint32_t m = m0; m < m1; m += 2) {
@@ -2007,7 +2029,7 @@ __global__ void __launch_bounds__(search_block(KS, LIST), KS <= 4 ? FFS_MINB4 : 
           if constexpr (KS == 4)
             ks4_pair_rows<VERIFY>(c, R, mask, maskB, haveB, has, reinterpret_cast<h2*>(rows), A.misses, A.zero, PK,
                                   VERIFY ? nullptr : pend);
-          else
+          else if constexpr (KS == 3)
             ks3_pair_rows<VERIFY>(c, R, mask, maskB, haveB, has, A.misses, A.zero, PK, VERIFY ? nullptr : pend);
           if constexpr (!VERIFY) {
             __syncwarp();
