@@ -633,7 +633,16 @@ def main():
         if world == 1 and not args.no_cpu_baseline:
             cpu = cpu_baseline(prob, K)
         n_seg = min(K, int(prob.chain_len().max()))
-        launches_per_step = (1 + 3 + n_seg + 1) if shard == "requests" else (K * (1 + 3) + n_seg + 1)
+        # exhaustive step: count + 3 scan kernels per keys call, the chain-length grouping of
+        # the grouped segments (k_group_hist, 3 scan kernels, k_group_tab, k_group_scatter;
+        # once per call: KS = 3, 4, and KS = 2 on >= 2^19 requests), a search kernel per
+        # segment, decode
+        n_rank = (hi - lo) if shard == "requests" else R
+        grouped = [k for k in (2, 3, 4) if k <= n_seg and (k != 2 or n_rank >= 1 << 19)]
+        if shard == "requests":
+            launches_per_step = 1 + 3 + (6 if grouped else 0) + n_seg + 1
+        else:
+            launches_per_step = K * (1 + 3) + 6 * len(grouped) + n_seg + 1
         line = {
             "metric": "candidates_scored_per_s", "value": value, "unit": "candidates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
