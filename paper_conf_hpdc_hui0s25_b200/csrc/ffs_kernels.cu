@@ -2869,6 +2869,20 @@ __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __rest
     for (uint32_t i = threadIdx.x; i < ncell; i += kEvT) cell[i] = ~0ull;
     __syncthreads();
   }
+  // PICK: the first kEvT loads of the tick (one per thread) resolve their request, node and
+  // monolithic profiles before the scoring pass, so those dependent loads overlap it; only
+  // the minimum over the finished cells waits for the barrier
+  uint32_t p_okp = 0, p_node = 0;
+  if constexpr (TAB && PICK) {
+    const uint32_t r = pk.load_off[t] + threadIdx.x;
+    if (r < pk.load_off[t + 1]) {
+      const ffs_request q = pk.req[r];
+      if (q.func < pk.lay.F && q.node < n_nodes) {
+        p_okp = victim_profiles(pk.image, pk.lay, q.func, pk.slo[r]);
+        p_node = q.node;
+      }
+    }
+  }
   for (uint32_t g0 = b + threadIdx.x; g0 < e; g0 += kEvT * kEvU) {
     ffs_instance in[kEvU];
 #pragma unroll
@@ -2895,7 +2909,14 @@ __global__ void __launch_bounds__(kEvT) k_evict_ticks(const ffs_instance* __rest
   if constexpr (TAB && PICK) {  // this tick's loads: the minimum over their monolithic profiles' cells
     __syncthreads();
     const uint32_t lb = pk.load_off[t], le = pk.load_off[t + 1];
-    for (uint32_t r = lb + threadIdx.x; r < le; r += kEvT) {
+    if (lb + threadIdx.x < le) {
+      unsigned long long bs = ~0ull;
+#pragma unroll
+      for (int p = 0; p < kP; ++p)
+        if ((p_okp >> p) & 1u) bs = min(bs, cell[p_node * kP + p]);
+      pk.victim[lb + threadIdx.x] = bs == ~0ull ? -1 : (int32_t)(bs & 0xFFFFFull);
+    }
+    for (uint32_t r = lb + kEvT + threadIdx.x; r < le; r += kEvT) {
       const ffs_request q = pk.req[r];
       unsigned long long bs = ~0ull;
       if (q.func < pk.lay.F && q.node < n_nodes) {
