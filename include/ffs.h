@@ -189,9 +189,10 @@ ffs_status ffs_set_search_mode(ffs_ctx *ctx, uint32_t mode);
  * of 32 equal contiguous pieces; shard `rank` owns the chunks j with j mod world = rank
  * (chunk interleave, DESIGN.md §4.3/§7) and decides every candidate of its chunks
  * (scored, or in bounded mode possibly proved infeasible by the exact SLO bound).  In
- * exhaustive and verify modes the segment k = 4 instead orders the requests by chain
- * length (a stable sort, identical on every rank) and deals work units (32 consecutive
- * requests of that order x 128 consecutive masks) to the shards by unit index mod world.
+ * exhaustive and verify modes the segments k = 3, 4 (and k = 2 on batches of >= 2^19
+ * requests) instead order the requests by chain length (a stable sort, identical on every
+ * rank) and deal work units (32 consecutive requests of that order x a run of consecutive
+ * masks) to the shards by unit index mod world.
  * In bounded mode the segments k = 2..4 are partitioned by a hash of (request, two
  * highest cut positions) -- in every case the shards partition the candidates.  Bounded mode
  * keeps three device lists of live (request, mask pair) records, 16 B each, capacity
