@@ -1172,11 +1172,18 @@ __device__ __forceinline__ void ks4_pair_rows(SearchState<4>& c, Row4& R, uint32
 #pragma unroll
     for (int x = 0; x < kP; ++x) {
       const uint32_t cap = c.sm[c.o_cap + x];
+      if (c.thr_u == 0xffffffffu) {
 #pragma unroll
-      for (int h = 0; h < 2; ++h)
+        for (int h = 0; h < 2; ++h)
 #pragma unroll
-        for (int s = 0; s < 2; ++s)
-          f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+          for (int s = 0; s < 2; ++s) f[h][s][x] = ms[h][s] <= cap ? f[h][s][x] * R.sig[h] : INF;
+      } else {
+#pragma unroll
+        for (int h = 0; h < 2; ++h)
+#pragma unroll
+          for (int s = 0; s < 2; ++s)
+            f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+      }
     }
     R.v3m[0] = INF;
     R.v3m[1] = INF;
@@ -1236,11 +1243,18 @@ __device__ __forceinline__ void ks4_pair_rows(SearchState<4>& c, Row4& R, uint32
 #pragma unroll
   for (int x = 0; x < kP; ++x) {
     const uint32_t cap = c.sm[c.o_cap + x];
+    if (c.thr_u == 0xffffffffu) {  // no throughput floor (the common case; uniform per request)
 #pragma unroll
-    for (int h = 0; h < 2; ++h)
+      for (int h = 0; h < 2; ++h)
 #pragma unroll
-      for (int s = 0; s < 2; ++s)
-        f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+        for (int s = 0; s < 2; ++s) f[h][s][x] = ms[h][s] <= cap ? f[h][s][x] * R.sig[h] : INF;
+    } else {
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 2; ++s)
+          f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+    }
   }
   h2 a1[kP];
 #pragma unroll
@@ -1575,11 +1589,18 @@ __device__ __forceinline__ void ks3_pair_rows(SearchState<3>& c, Row3& R, uint32
 #pragma unroll
   for (int x = 0; x < kP; ++x) {
     const uint32_t cap = c.sm[c.o_cap + x];
+    if (c.thr_u == 0xffffffffu) {  // no throughput floor (the common case; uniform per request)
 #pragma unroll
-    for (int h = 0; h < 2; ++h)
+      for (int h = 0; h < 2; ++h)
 #pragma unroll
-      for (int s = 0; s < 2; ++s)
-        f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+        for (int s = 0; s < 2; ++s) f[h][s][x] = ms[h][s] <= cap ? f[h][s][x] * R.sig[h] : INF;
+    } else {
+#pragma unroll
+      for (int h = 0; h < 2; ++h)
+#pragma unroll
+        for (int s = 0; s < 2; ++s)
+          f[h][s][x] = (ms[h][s] <= cap && f[h][s][x] <= c.thr) ? f[h][s][x] * R.sig[h] : INF;
+    }
   }
   h2 v0[kP], nl0[kP], s1w[2][kP], a1[kP];
 #pragma unroll
