@@ -247,7 +247,12 @@ ffs_status ffs_plan_batch(ffs_ctx *ctx, const ffs_request *d_req, const uint32_t
 
 /* Same with HOST buffers: copies the requests and budgets host->device, plans, copies
  * the plans device->host and synchronises `stream` before returning (the end-to-end
- * call of a user holding host data). */
+ * call of a user holding host data).  A batch of >= 2^20 requests is planned in two
+ * request slices whose copies run on two context-owned non-blocking streams (ordered
+ * after the work already queued on `stream`): the upload of the second and the download
+ * of the first overlap the planning of the other (pinned host buffers are needed for the
+ * overlap; pageable ones work, serialised).  The plans equal ffs_plan_batch's on the whole
+ * batch (requests are planned independently). */
 ffs_status ffs_plan_batch_host(ffs_ctx *ctx, const ffs_request *h_req, const uint32_t *h_slo_us, uint32_t n_req,
                                uint32_t k_max, ffs_plan *h_out, void *stream);
 

@@ -102,6 +102,9 @@ struct ffs_ctx {
   bool grp_ok = false;
   uint32_t list_cap = 0;
   uint64_t list_cap_max = 1ull << 28;  // FFS_LIST_CAP (tests: force the task-range fallback)
+  // ffs_plan_batch_host: copy streams (non-blocking) and the pipeline's events
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  cudaEvent_t h_ev[2 * kHostSlices + 2] = {};
 };
 
 static ffs_status fail(ffs_ctx* c, ffs_status s, const char* fmt, ...) {
@@ -167,6 +170,10 @@ void ffs_destroy(ffs_ctx* c) {
       if (e) cudaEventDestroy(e);
     for (auto& e : c->evs)
       if (e) cudaEventDestroy(e);
+    for (auto& e : c->h_ev)
+      if (e) cudaEventDestroy(e);
+    if (c->s_h2d) cudaStreamDestroy(c->s_h2d);
+    if (c->s_d2h) cudaStreamDestroy(c->s_d2h);
     for (DevBuf* b : {&c->s_res, &c->s_flags, &c->s_busy, &c->s_psl, &c->s_pe2e, &c->s_pk}) b->release();
     for (DevBuf* b : {&c->r_k, &c->r_k2, &c->r_v, &c->r_v2, &c->i_k, &c->i_k2, &c->i_v, &c->i_v2, &c->i_cum, &c->r_f,
                       &c->r_h, &c->r_n, &c->r_ts, &c->r_hist, &c->r_bsum})
@@ -648,19 +655,52 @@ ffs_status ffs_plan_batch_host(ffs_ctx* c, const ffs_request* h_req, const uint3
   if (n_req == 0) return FFS_OK;
   if (!h_req || !h_slo || !h_out) return fail(c, FFS_ERR_ARG, "null host pointer");
   cudaStream_t st = (cudaStream_t)stream;
+  // Large batches are planned in kHostSlices request slices (requests are independent,
+  // R13: a slice plans exactly as within the batch): the upload of slice i+1 and the
+  // download of the plans of slice i-1 run on two copy streams while slice i is planned on
+  // `stream`, so only the first upload and the last download are exposed.  Each slice pays
+  // the per-call fixed costs once more, so the slices stay few and large.
+  const uint32_t nch = n_req >= (1u << 20) ? kHostSlices : 1u;
   {
     DeviceGuard g(c->device);
     CK(c->req_dev.ensure((size_t)n_req * sizeof(ffs_request)), "cudaMalloc(req)");
     CK(c->slo_dev.ensure((size_t)n_req * 4), "cudaMalloc(slo)");
     CK(c->plans_dev.ensure((size_t)n_req * sizeof(ffs_plan)), "cudaMalloc(plans)");
-    CK(cudaMemcpyAsync(c->req_dev.p, h_req, (size_t)n_req * sizeof(ffs_request), cudaMemcpyHostToDevice, st), "H2D req");
-    CK(cudaMemcpyAsync(c->slo_dev.p, h_slo, (size_t)n_req * 4, cudaMemcpyHostToDevice, st), "H2D slo");
+    if (!c->s_h2d) CK(cudaStreamCreateWithFlags(&c->s_h2d, cudaStreamNonBlocking), "copy stream");
+    if (!c->s_d2h) CK(cudaStreamCreateWithFlags(&c->s_d2h, cudaStreamNonBlocking), "copy stream");
+    for (auto& e : c->h_ev)
+      if (!e) CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event");
+    // the copies start after the work already queued on `stream` (its buffers may be in use)
+    CK(cudaEventRecord(c->h_ev[2 * kHostSlices], st), "event");
+    CK(cudaStreamWaitEvent(c->s_h2d, c->h_ev[2 * kHostSlices], 0), "wait");
+    CK(cudaStreamWaitEvent(c->s_d2h, c->h_ev[2 * kHostSlices], 0), "wait");
+    for (uint32_t i = 0; i < nch; ++i) {
+      const size_t lo = (size_t)n_req * i / nch, hi = (size_t)n_req * (i + 1) / nch;
+      CK(cudaMemcpyAsync(c->req_dev.as<ffs_request>() + lo, h_req + lo, (hi - lo) * sizeof(ffs_request),
+                         cudaMemcpyHostToDevice, c->s_h2d), "H2D req");
+      CK(cudaMemcpyAsync(c->slo_dev.as<uint32_t>() + lo, h_slo + lo, (hi - lo) * 4, cudaMemcpyHostToDevice, c->s_h2d),
+         "H2D slo");
+      CK(cudaEventRecord(c->h_ev[i], c->s_h2d), "event");
+    }
   }
-  ffs_status s = ffs_plan_batch(c, c->req_dev.as<ffs_request>(), c->slo_dev.as<uint32_t>(), n_req, k_max,
-                                c->plans_dev.as<ffs_plan>(), stream);
-  if (s != FFS_OK) return s;
+  for (uint32_t i = 0; i < nch; ++i) {
+    const size_t lo = (size_t)n_req * i / nch, hi = (size_t)n_req * (i + 1) / nch;
+    {
+      DeviceGuard g(c->device);
+      CK(cudaStreamWaitEvent(st, c->h_ev[i], 0), "wait");
+    }
+    ffs_status s = ffs_plan_batch(c, c->req_dev.as<ffs_request>() + lo, c->slo_dev.as<uint32_t>() + lo,
+                                  (uint32_t)(hi - lo), k_max, c->plans_dev.as<ffs_plan>() + lo, stream);
+    if (s != FFS_OK) return s;
+    DeviceGuard g(c->device);
+    CK(cudaEventRecord(c->h_ev[kHostSlices + i], st), "event");
+    CK(cudaStreamWaitEvent(c->s_d2h, c->h_ev[kHostSlices + i], 0), "wait");
+    CK(cudaMemcpyAsync(h_out + lo, c->plans_dev.as<ffs_plan>() + lo, (hi - lo) * sizeof(ffs_plan),
+                       cudaMemcpyDeviceToHost, c->s_d2h), "D2H plans");
+  }
   DeviceGuard g(c->device);
-  CK(cudaMemcpyAsync(h_out, c->plans_dev.p, (size_t)n_req * sizeof(ffs_plan), cudaMemcpyDeviceToHost, st), "D2H plans");
+  CK(cudaEventRecord(c->h_ev[2 * kHostSlices + 1], c->s_d2h), "event");
+  CK(cudaStreamWaitEvent(st, c->h_ev[2 * kHostSlices + 1], 0), "wait");
   CK(cudaStreamSynchronize(st), "stream sync");
   return FFS_OK;
 }

@@ -37,6 +37,10 @@ __host__ __device__ constexpr int search_block(int ks, bool list = false) {
   return ks == 3 ? (list ? 384 : FFS_BLOCK3) : ks == 4 ? FFS_BLOCK4 : kBlock;
 }
 constexpr size_t kMaxSmem = 227 * 1024;  // dynamic shared memory per CTA on sm_100
+#ifndef FFS_HOST_SLICES
+#define FFS_HOST_SLICES 2
+#endif
+constexpr uint32_t kHostSlices = FFS_HOST_SLICES;  // request slices of ffs_plan_batch_host (>= 2^20 requests)
 // bytes of per-thread shared memory of the KS = 4 kernel: 5 profiles x 11 packed f16x2
 // windows (ks4_pair_h)
 constexpr size_t kWin4 = 55 * 4;
