@@ -723,6 +723,29 @@ def test_host_entry_point_large(F, planner, cfg):
     np.testing.assert_array_equal(pageable.view(np.uint8), ref.view(np.uint8))
 
 
+def test_host_entry_point_ragged_slices(F, planner):
+    """A batch just above 2^20 requests (two uneven host slices; the exhaustive mode's
+    grouped walks on both): ffs_plan_batch_host = ffs_plan_batch on the device batch."""
+    import torch
+    base = W.config5()
+    idx = np.concatenate([np.arange(base.R), np.arange(0, 37 * 997, 997)])
+    prob = base.subset(idx)
+    planner.stage(prob)
+    req, slo = F.to_device(prob)
+    try:
+        planner.set_search_mode(F.SEARCH_EXHAUSTIVE)
+        ref = F.plans_to_numpy(planner.plan_batch(req, slo, prob.k_max))
+        h_req = torch.from_numpy(np.ascontiguousarray(prob.req).view(np.uint8)).pin_memory()
+        h_slo = torch.from_numpy(np.ascontiguousarray(prob.slo_us).view(np.uint8)).pin_memory()
+        out = torch.zeros(prob.R * 80, dtype=torch.uint8).pin_memory().numpy().view(F.PLAN_DTYPE)
+        planner.plan_batch_host(h_req.numpy().view(W.REQ_DTYPE), h_slo.numpy().view(np.uint32), prob.k_max,
+                                out=out)
+    finally:
+        planner.set_search_mode(F.SEARCH_BOUNDED)
+    np.testing.assert_array_equal(out.view(np.uint8), ref.view(np.uint8))
+    np.testing.assert_array_equal(ref["key"][base.R:], ref["key"][idx[base.R:]])  # duplicated requests
+
+
 def test_c5_full_batch_properties(F, planner):
     prob = W.config5()
     p, _, _ = run_gpu(F, planner, prob, verify=False)
