@@ -91,6 +91,14 @@ def test_tiny_random_bit_exact(F, planner, seed):
     # production (non-verify) path gives the same keys
     p2, keys2, _ = run_gpu(F, planner, prob, verify=False)
     np.testing.assert_array_equal(keys2, o["key"])
+    # and so does the exhaustive mode (KS = 3, 4 walk the chain-length groups: mostly idle
+    # lanes on a tiny batch)
+    try:
+        planner.set_search_mode(F.SEARCH_EXHAUSTIVE)
+        p3, keys3, _ = run_gpu(F, planner, prob, verify=False)
+    finally:
+        planner.set_search_mode(F.SEARCH_BOUNDED)
+    np.testing.assert_array_equal(keys3, o["key"])
 
 
 @pytest.mark.parametrize("K", [1, 2, 3, 4, 5, 6, 7, 8])
