@@ -1028,6 +1028,7 @@ ffs_status ffs_plan_dag(ffs_ctx* c, const ffs_request* d_req, const uint32_t* d_
   a.mt_cand = c->dag_mt_cand.as<unsigned long long>();
   a.out = d_out;
   a.checks = reinterpret_cast<unsigned long long*>(d_checksums);
+  a.tables_global = (size_t)c->lay.words * 4 > kMaxSmem ? 1u : 0u;
   CK(launch_dag(a, (cudaStream_t)stream), "dag kernel");
   return FFS_OK;
 }

@@ -243,6 +243,7 @@ struct DagArgs {
   const unsigned long long* mt_cand;  // first candidate index of the entry
   ffs_dag_plan* out;
   unsigned long long* checks; // [n_req][3] or null
+  uint32_t tables_global;     // 1: the image is too large for shared memory, read it from global
 };
 cudaError_t launch_dag(const DagArgs& a, cudaStream_t st);
 

@@ -4053,8 +4053,9 @@ cudaError_t run_packed_peak(int sms, int mode, double* lane_instr_per_s, double*
 // one-slice sum).  Warp argmin of the packed keys; the winning lane writes and binds.
 constexpr int kDagT = 128;
 
-__device__ __forceinline__ uint32_t dag_lat(const DagArgs& A, uint32_t row0, uint32_t a, uint32_t b, uint32_t p) {
-  return __float2uint_rn(plf(A.image, A.lay.o_pl + (row0 + b) * kRowW + p) - plf(A.image, A.lay.o_pl + (row0 + a) * kRowW + p));
+__device__ __forceinline__ uint32_t dag_lat(const DagArgs& A, const uint32_t* img, uint32_t row0, uint32_t a,
+                                            uint32_t b, uint32_t p) {
+  return __float2uint_rn(plf(img, A.lay.o_pl + (row0 + b) * kRowW + p) - plf(img, A.lay.o_pl + (row0 + a) * kRowW + p));
 }
 
 // options of the stage made of units [u0, u1]: P, plus P^nb splits when it is one
@@ -4072,17 +4073,16 @@ __device__ __forceinline__ uint32_t dag_nopt(const uint32_t* uo, uint32_t u0, ui
 // GPCs and per-profile slice counts, clears ok on a memory / floor miss; returns t.
 // A split's branch profiles are the base-P digits of o - P, branch 0 most significant
 // (sums and max are order-free, so the digits are taken least significant first).
-__device__ __forceinline__ uint32_t dag_stage(const DagArgs& A, uint32_t row0, const uint32_t* uo, uint32_t u0,
-                                              uint32_t u1, uint32_t o, uint32_t thr, uint32_t& gp, uint64_t& use,
-                                              bool& ok, const uint32_t* sv) {
-  const uint32_t* img = A.image;
+__device__ __forceinline__ uint32_t dag_stage(const DagArgs& A, const uint32_t* img, uint32_t row0, const uint32_t* uo,
+                                              uint32_t u0, uint32_t u1, uint32_t o, uint32_t thr, uint32_t& gp,
+                                              uint64_t& use, bool& ok, const uint32_t* sv) {
   const uint32_t* U0 = uo + 6 * u0;
   uint32_t t;
   if (o < (uint32_t)kP) {
     const uint32_t* U1 = uo + 6 * u1;
     const uint32_t c0 = U0[1], c1 = U1[1 + (U1[0] & 0xffu)];  // end of the last branch of unit u1
     // every component in sequence, minus the conditional units' sum - max (R48)
-    t = dag_lat(A, row0, c0, c1, o) - (sv[8 * (u1 + 1) + o] - sv[8 * u0 + o]);
+    t = dag_lat(A, img, row0, c0, c1, o) - (sv[8 * (u1 + 1) + o] - sv[8 * u0 + o]);
     ok &= img[A.lay.o_pm + row0 + c1] - img[A.lay.o_pm + row0 + c0] <= img[A.lay.o_cap + o];
     gp += img[A.lay.o_gpcs + o];
     use += 1ull << (8 * o);
@@ -4094,7 +4094,7 @@ __device__ __forceinline__ uint32_t dag_stage(const DagArgs& A, uint32_t row0, c
       const uint32_t j = jj - 1, p = w % kP;
       w /= kP;
       const uint32_t c = U0[1 + j], e = U0[2 + j];  // branch j = [end of branch j-1 (or c0), e)
-      t = max(t, dag_lat(A, row0, c, e, p));
+      t = max(t, dag_lat(A, img, row0, c, e, p));
       ok &= img[A.lay.o_pm + row0 + e] - img[A.lay.o_pm + row0 + c] <= img[A.lay.o_cap + p];
       gp += img[A.lay.o_gpcs + p];
       use += 1ull << (8 * p);
@@ -4110,18 +4110,16 @@ __device__ __forceinline__ void dag_bounds(uint32_t ends, uint32_t s, uint32_t& 
   u0 = s ? ((ends >> (4 * (s - 1))) & 15u) + 1 : 0;
 }
 
+// one request, the whole warp (img: the table image, staged in shared memory)
 template <bool VERIFY>
-__global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagArgs A) {
+__device__ __forceinline__ void dag_request(const DagArgs& A, const uint32_t* img, uint32_t r) {
   const uint32_t lane = threadIdx.x & 31;
-  const uint64_t r64 = ((uint64_t)blockIdx.x * kDagT + threadIdx.x) >> 5;
-  if (r64 >= A.n_req) return;
-  const uint32_t r = (uint32_t)r64;
   const ffs_request q = A.req[r];
   ffs_dag_plan* out = A.out + r;
   const bool bad = q.func >= A.lay.F || q.node >= A.n_nodes;
   const uint32_t f = bad ? 0 : q.func, v = bad ? 0 : q.node;
-  const uint32_t row0 = A.image[A.lay.o_fdesc + 4 * f];
-  const uint32_t thr = A.image[A.lay.o_thr + f];
+  const uint32_t row0 = img[A.lay.o_fdesc + 4 * f];
+  const uint32_t thr = img[A.lay.o_thr + f];
   const uint32_t B = A.slo[r];
   const uint64_t nf = A.node_free[v];
   const uint32_t* uo = A.units + 6 * A.fu[2 * f];
@@ -4132,7 +4130,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
   uint32_t best_mk = 0, best_c = 0;
   uint32_t gpc[kP];
 #pragma unroll
-  for (int x = 0; x < kP; ++x) gpc[x] = A.image[A.lay.o_gpcs + x];
+  for (int x = 0; x < kP; ++x) gpc[x] = img[A.lay.o_gpcs + x];
   // The warp walks the function's masks together (uniform control flow: k, the stage
   // bounds and option counts are the same on every lane); within a mask the lanes split
   // the outer combinations (stages 0 .. k-2), and each lane scores the last stage's
@@ -4169,7 +4167,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
       uint64_t us = 0;
       lg[o] = 0;
       lok[o] = true;
-      lt[o] = dag_stage(A, row0, uo, lu0, lu1, (uint32_t)o, thr, lg[o], us, lok[o], sv);
+      lt[o] = dag_stage(A, img, row0, uo, lu0, lu1, (uint32_t)o, thr, lg[o], us, lok[o], sv);
     }
     const bool split2 = nl == kP + kP * kP;
     uint32_t bt[2][kP], bok = 0;
@@ -4180,8 +4178,8 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
 #pragma unroll
         for (int x = 0; x < kP; ++x) {
           const uint32_t cb0 = U[1 + j], ce0 = U[2 + j];
-          bt[j][x] = dag_lat(A, row0, cb0, ce0, x);
-          if (A.image[A.lay.o_pm + row0 + ce0] - A.image[A.lay.o_pm + row0 + cb0] <= A.image[A.lay.o_cap + x])
+          bt[j][x] = dag_lat(A, img, row0, cb0, ce0, x);
+          if (img[A.lay.o_pm + row0 + ce0] - img[A.lay.o_pm + row0 + cb0] <= img[A.lay.o_cap + x])
             bok |= 1u << (5 * j + x);
         }
     }
@@ -4194,7 +4192,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         dag_bounds(ends, ss - 1, u0, u1);
         const uint32_t no = dag_nopt(uo, u0, u1), os = rest % no;
         rest /= no;
-        const uint64_t t = dag_stage(A, row0, uo, u0, u1, os, thr, gp0, use0, ok0, sv);
+        const uint64_t t = dag_stage(A, img, row0, uo, u0, u1, os, thr, gp0, use0, ok0, sv);
         T0 += t;
         Q0 += t * t;
       }
@@ -4244,7 +4242,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
           uint64_t use = use0;
           uint32_t gp = gp0;
           bool ok = true;
-          const uint64_t t = dag_stage(A, row0, uo, lu0, lu1, ol, thr, gp, use, ok, sv);
+          const uint64_t t = dag_stage(A, img, row0, uo, lu0, lu1, ol, thr, gp, use, ok, sv);
           score(t, gp, use, ok, ol);
         }
       }
@@ -4311,7 +4309,7 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
         dag_bounds(ends, s + 1, a0, a1);
         div /= dag_nopt(uo, a0, a1);
       }
-      const uint32_t t = dag_stage(A, row0, uo, u0, u1, os, 0xffffffffu, g, use, ok, sv);
+      const uint32_t t = dag_stage(A, img, row0, uo, u0, u1, os, 0xffffffffu, g, use, ok, sv);
       e2e += t;
       bott = max(bott, t);
       // slots: one slice, or the branches in order (branch 0 = most significant digit)
@@ -4339,12 +4337,42 @@ __global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagA
   *out = P;
 }
 
+
+// Persistent CTAs: the table image is staged into shared memory once per CTA (as the search
+// kernel does), then the CTA's warps take requests r = warp, warp + all warps, ...; an image
+// too large for shared memory is read from global memory (A.tables_global).
+template <bool VERIFY>
+__global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagArgs A) {
+  extern __shared__ __align__(16) uint32_t dag_smem[];
+  const uint32_t* img = A.image;
+  if (!A.tables_global) {
+    const uint4* src = reinterpret_cast<const uint4*>(A.image);
+    uint4* dst = reinterpret_cast<uint4*>(dag_smem);
+    for (uint32_t i = threadIdx.x; i < A.lay.words / 4; i += blockDim.x) dst[i] = src[i];
+    __syncthreads();
+    img = dag_smem;
+  }
+  const uint32_t nw = gridDim.x * (kDagT / 32);
+  for (uint32_t r = blockIdx.x * (kDagT / 32) + (threadIdx.x >> 5); r < A.n_req; r += nw) dag_request<VERIFY>(A, img, r);
+}
+
 cudaError_t launch_dag(const DagArgs& a, cudaStream_t st) {
-  const uint64_t threads = (uint64_t)a.n_req * 32;
+  int dev = 0, sms = 0, per = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const size_t smem = a.tables_global ? 0 : (size_t)a.lay.words * 4;
+  cudaError_t e = a.checks ? cudaFuncSetAttribute(k_plan_dag<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem)
+                           : cudaFuncSetAttribute(k_plan_dag<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMaxSmem);
+  if (e != cudaSuccess) return e;
+  e = a.checks ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_plan_dag<true>, kDagT, smem)
+               : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_plan_dag<false>, kDagT, smem);
+  if (e != cudaSuccess) return e;
+  const uint64_t need = ((uint64_t)a.n_req + kDagT / 32 - 1) / (kDagT / 32);
+  const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(need, (uint64_t)sms * std::max(per, 1)));
   if (a.checks)
-    k_plan_dag<true><<<(unsigned)((threads + kDagT - 1) / kDagT), kDagT, 0, st>>>(a);
+    k_plan_dag<true><<<grid, kDagT, smem, st>>>(a);
   else
-    k_plan_dag<false><<<(unsigned)((threads + kDagT - 1) / kDagT), kDagT, 0, st>>>(a);
+    k_plan_dag<false><<<grid, kDagT, smem, st>>>(a);
   return cudaGetLastError();
 }
 
