@@ -4341,8 +4341,14 @@ __device__ __forceinline__ void dag_request(const DagArgs& A, const uint32_t* im
 // Persistent CTAs: the table image is staged into shared memory once per CTA (as the search
 // kernel does), then the CTA's warps take requests r = warp, warp + all warps, ...; an image
 // too large for shared memory is read from global memory (A.tables_global).
+// 6 CTAs of 128 threads per SM (80 registers, a few spills): the kernel is latency-bound
+// (dependent integer chains, wait stalls), more warps win (CD: 18.4 / 17.6 / 14.6 / 15.6 ms
+// at 1 / 4 / 6 / 8)
+#ifndef FFS_DAG_MINB
+#define FFS_DAG_MINB 6
+#endif
 template <bool VERIFY>
-__global__ void __launch_bounds__(kDagT) k_plan_dag(const __grid_constant__ DagArgs A) {
+__global__ void __launch_bounds__(kDagT, FFS_DAG_MINB) k_plan_dag(const __grid_constant__ DagArgs A) {
   extern __shared__ __align__(16) uint32_t dag_smem[];
   const uint32_t* img = A.image;
   if (!A.tables_global) {
