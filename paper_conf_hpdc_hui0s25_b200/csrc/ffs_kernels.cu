@@ -3206,7 +3206,12 @@ __device__ __forceinline__ bool ranked_eval(const RankedArgs& A, uint32_t row0, 
 }
 
 constexpr int kRkT = 128;
-__global__ void __launch_bounds__(kRkT) k_plan_ranked(const __grid_constant__ RankedArgs A) {
+// 12 CTAs of 128 threads per SM (40 registers): one warp per request walking its ranked
+// list is latency-bound, more warps win (C5: 10.4 / 7.9 / 7.6 / 7.5 ms at 1 / 8 / 12 / 16)
+#ifndef FFS_RANKED_MINB
+#define FFS_RANKED_MINB 12
+#endif
+__global__ void __launch_bounds__(kRkT, FFS_RANKED_MINB) k_plan_ranked(const __grid_constant__ RankedArgs A) {
   const uint32_t r = (blockIdx.x * kRkT + threadIdx.x) >> 5, lane = threadIdx.x & 31;
   if (r >= A.n_req) return;
   const uint32_t* img = A.image;
